@@ -1,0 +1,91 @@
+"""Build every native library of the repo in-tree (sm_100a only).
+
+* ``oracle/liblouvain_oracle.so``  -- gcc, plain C (test infrastructure)
+* ``graphgen/libgraphgen.so``      -- nvcc, seeded input generators (host + device)
+* ``paper_conf_ipps_naimmht17_b200/liblouvain.so`` -- nvcc, the product C-ABI
+
+Rebuilds a target only when one of its sources is newer than the .so.
+"""
+from __future__ import annotations
+
+import glob
+import os
+import shutil
+import subprocess
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+NVCC = shutil.which("nvcc") or "/usr/local/cuda/bin/nvcc"
+ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
+
+
+def _site_nccl() -> str:
+    for p in sys.path:
+        cand = os.path.join(p, "nvidia", "nccl")
+        if os.path.isdir(os.path.join(cand, "include")):
+            return cand
+    return ""
+
+
+def _stale(target: str, sources: list[str]) -> bool:
+    if not os.path.exists(target):
+        return True
+    t = os.path.getmtime(target)
+    return any(os.path.getmtime(s) > t for s in sources)
+
+
+def _run(cmd: list[str]) -> None:
+    print("+", " ".join(cmd), flush=True)
+    subprocess.run(cmd, check=True, cwd=ROOT)
+
+
+def build_oracle(force: bool = False) -> str:
+    src = [os.path.join(ROOT, "oracle", "louvain_oracle.c")]
+    hdr = [os.path.join(ROOT, "oracle", "louvain_oracle.h")]
+    out = os.path.join(ROOT, "oracle", "liblouvain_oracle.so")
+    if force or _stale(out, src + hdr + [__file__]):
+        _run(["gcc", "-O2", "-std=c11", "-fPIC", "-shared", "-ffp-contract=off", "-Wall", "-Wextra",
+              "-o", out] + src)
+    return out
+
+
+def build_graphgen(force: bool = False) -> str:
+    d = os.path.join(ROOT, "graphgen", "csrc")
+    srcs = sorted(glob.glob(os.path.join(d, "*.cpp")) + glob.glob(os.path.join(d, "*.cu")))
+    hdrs = glob.glob(os.path.join(d, "*.h"))
+    out = os.path.join(ROOT, "graphgen", "libgraphgen.so")
+    if force or _stale(out, srcs + hdrs + [__file__]):
+        _run([NVCC, "-O3", "-std=c++17", *ARCH, "-lineinfo", "-shared",
+              "-Xcompiler", "-fPIC,-ffp-contract=off", "-o", out] + srcs)
+    return out
+
+
+def build_louvain(force: bool = False) -> str:
+    pkg = os.path.join(ROOT, "paper_conf_ipps_naimmht17_b200")
+    d = os.path.join(pkg, "csrc")
+    srcs = sorted(glob.glob(os.path.join(d, "*.cu")) + glob.glob(os.path.join(d, "*.cpp")))
+    hdrs = glob.glob(os.path.join(d, "*.h")) + glob.glob(os.path.join(d, "*.cuh")) + \
+        glob.glob(os.path.join(ROOT, "include", "*.h"))
+    out = os.path.join(pkg, "liblouvain.so")
+    if not srcs:
+        return out
+    nccl = _site_nccl()
+    nccl_flags = []
+    if nccl:
+        nccl_flags = ["-I", os.path.join(nccl, "include"), "-DLOUVAIN_HAVE_NCCL_HEADERS=1"]
+    if force or _stale(out, srcs + hdrs + [__file__]):
+        _run([NVCC, "-O3", "-std=c++17", *ARCH, "-lineinfo", "-shared", "-Xptxas", "-v",
+              "-Xcompiler", "-fPIC,-ffp-contract=off,-fvisibility=hidden",
+              "-I", os.path.join(ROOT, "include"), *nccl_flags,
+              "-o", out] + srcs + ["-ldl"])
+    return out
+
+
+def build_all(force: bool = False) -> None:
+    build_oracle(force)
+    build_graphgen(force)
+    build_louvain(force)
+
+
+if __name__ == "__main__":
+    build_all(force="--force" in sys.argv)
