@@ -1,0 +1,153 @@
+/* louvain.h -- C-ABI of the B200-native GPU Louvain hot path.
+ *
+ * Method: Naim, Manne, Halappanavar, Tumeo, "Community Detection on the GPU"
+ * (IPDPS'17).  Citations "P:<line>" refer to /root/reference/PAPER.md (a text
+ * extraction of the paper); "R<k>" to the readings of SURVEY.md 8(c), restated
+ * in DESIGN.md.  Implemented by liblouvain.so (hand-written CUDA for sm_100a).
+ *
+ * Conventions (every function):
+ *  - extern "C", returns int32_t status: LOUVAIN_OK (0) or a negative code;
+ *    never throws, never exits; louvain_last_error() gives a thread-local message.
+ *  - Graph input: undirected, positive integer weights, stored as
+ *    CSR with BOTH directions of every non-loop edge and each self-loop ONCE
+ *    (R1).  rowptr int64[n+1], col int32[nnz], w uint32[nnz] (NULL = all 1).
+ *    Rows need not be sorted.  k_i = row sum, W = 2m = sum_i k_i.
+ *  - Input pointers may be host or device memory (detected with
+ *    cudaPointerGetAttributes); they are caller-owned, copied during the call
+ *    and not retained (except with LOUVAIN_BORROW, below).
+ *  - Output buffers are caller-allocated, host or device, of the stated length.
+ *  - A handle owns all device memory of one level graph and its partition state
+ *    (C, a_c, size_c).  It is bound to the device current at creation and to one
+ *    stream (NULL -> a library-owned stream).  Calls that return scalars
+ *    synchronise that stream.  A handle is not thread-safe; distinct handles are
+ *    independent.
+ *  - Arithmetic is exact integers (R4): e, k, a in uint32, gains
+ *    s = W*e - k*a in int64, so W must be <= 3,037,000,499 (else
+ *    LOUVAIN_E_OVERFLOW).  Q is reported as exact parts plus a double.
+ */
+#ifndef LOUVAIN_H
+#define LOUVAIN_H
+#include <stdint.h>
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define LOUVAIN_OK 0
+#define LOUVAIN_E_INVALID_ARG (-1)
+#define LOUVAIN_E_INVALID_GRAPH (-2)
+#define LOUVAIN_E_OVERFLOW (-3)
+#define LOUVAIN_E_NOMEM (-4)
+#define LOUVAIN_E_CUDA (-5)
+#define LOUVAIN_E_NCCL (-6)
+#define LOUVAIN_E_STATE (-7)       /* handle poisoned by a sticky CUDA error */
+#define LOUVAIN_E_UNSUPPORTED (-8)
+
+/* louvain_create_csr flags */
+#define LOUVAIN_VALIDATE 1u /* full O(n + nnz) validation incl. symmetry; else O(1) checks only */
+#define LOUVAIN_BORROW 2u   /* device inputs are used in place (caller keeps them alive, unmodified) */
+
+/* modes */
+#define LOUVAIN_MODE_BIN_SYNC 0 /* Alg. 1: commit after each degree bucket (default) */
+#define LOUVAIN_MODE_RELAXED 1  /* one commit per sweep ("relaxed") */
+
+typedef struct louvain_graph_s* louvain_graph_t;
+
+/* Q = (L*W - S) / W^2 (Eq. 1), exact parts; S = S_hi*2^64 + S_lo. */
+typedef struct {
+  uint64_t L, S_lo, S_hi, W;
+  double q;
+} louvain_qnum_t;
+
+typedef struct {
+  int32_t mode;               /* LOUVAIN_MODE_* */
+  int32_t singleton_rule;     /* 1 veto-after-argmax (default) | 2 filter | 0 off (R8) */
+  int32_t revert_on_decrease; /* 1 (default): a sweep that lowers Q is undone and ends the phase (R15) */
+  int32_t th_bin_exp, th_final_exp; /* theta = 10^-exp; defaults 2, 6 */
+  int64_t size_limit;         /* 100000: n > limit -> theta_bin, else theta_final */
+  int64_t deg_bounds[6];      /* bucket bounds {4,8,16,32,84,319} */
+  int32_t max_sweeps, max_levels; /* safety caps; 0 = unlimited */
+} louvain_params_t;
+
+#define LOUVAIN_MAX_LEVELS 256
+typedef struct {
+  int32_t levels, sweeps;
+  int64_t n[LOUVAIN_MAX_LEVELS], nnz[LOUVAIN_MAX_LEVELS];
+  int32_t sweeps_per_level[LOUVAIN_MAX_LEVELS];
+  int64_t moved_per_level[LOUVAIN_MAX_LEVELS];
+  int64_t num_start[LOUVAIN_MAX_LEVELS], num_end[LOUVAIN_MAX_LEVELS]; /* L*W - S per level */
+  double t_opt_ms[LOUVAIN_MAX_LEVELS], t_agg_ms[LOUVAIN_MAX_LEVELS];
+  double t_total_ms;
+  /* measurement: sweep bodies only (buckets + commits, no modularity pass) */
+  double t_sweep_ms_total;    /* all sweeps of all levels */
+  double t_sweep_ms_first;    /* level 0, sweep 1 */
+  double t_modularity_ms_total;
+  int64_t edges_swept;        /* sum over executed sweeps of nnz of their level */
+  louvain_qnum_t q;
+} louvain_stats_t;
+
+/* Fill *p with the paper's defaults (R8, R15). */
+void louvain_params_default(louvain_params_t* p);
+
+/* Create a level graph from CSR.  n >= 0, nnz >= 0, rowptr[n+1],
+ * col[nnz] in [0,n), w[nnz] > 0 or NULL.  The partition starts as singletons
+ * (P:164).  Errors: INVALID_ARG (null/negative), INVALID_GRAPH (validation),
+ * OVERFLOW (W > 3,037,000,499), NOMEM, CUDA. */
+int32_t louvain_create_csr(int64_t n, int64_t nnz, const int64_t* rowptr, const int32_t* col,
+                           const uint32_t* w, uint32_t flags, void* cuda_stream, louvain_graph_t* out);
+/* Release a handle (NULL is a no-op). */
+int32_t louvain_destroy(louvain_graph_t g);
+/* n, nnz, W = 2m of the handle's graph (any output may be NULL). */
+int32_t louvain_get_info(louvain_graph_t g, int64_t* n, int64_t* nnz, uint64_t* W);
+/* Copy the handle's CSR out: rowptr[n+1], col[nnz], w[nnz] (any may be NULL;
+ * w of a unit-weight graph is written as 1s). */
+int32_t louvain_get_csr(louvain_graph_t g, int64_t* rowptr, int32_t* col, uint32_t* w);
+/* Set the partition C (labels[n], each in [0,n)); NULL = singletons.  a_c and
+ * size_c are recomputed. */
+int32_t louvain_set_labels(louvain_graph_t g, const int32_t* labels);
+/* Copy the current partition C[n]. */
+int32_t louvain_get_labels(louvain_graph_t g, int32_t* labels_out);
+/* Copy a_c (uint32[n]) and size_c (int32[n]) of the current partition (either may be NULL). */
+int32_t louvain_get_totals(louvain_graph_t g, uint32_t* a_out, int32_t* size_out);
+
+/* Exactly one iteration of Alg. 1's repeat body: buckets 1..7 in
+ * ascending order; every vertex of a bucket runs computeMove (Alg. 2)
+ * against the bucket-start state with Eq. (2) in integer form and the rules of
+ * P:172 (R5-R9), then the bucket's moves are committed (C, a_c, size_c).  No
+ * revert and no stop decision.  *moved = vertices that changed community;
+ * q_after (may be NULL) = modularity after the sweep. */
+int32_t louvain_sweep(louvain_graph_t g, const louvain_params_t* p, int64_t* moved, louvain_qnum_t* q_after);
+/* Eq. (1) of `labels` (n entries; NULL = current partition), exact parts. */
+int32_t louvain_modularity(louvain_graph_t g, const int32_t* labels, louvain_qnum_t* q);
+/* Alg. 3 CONTRACT: communities of the current partition become the
+ * vertices of *next, numbered consecutively in label order (R17); parallel
+ * edges merge by summing weights and intra-community entries form the
+ * self-loop (R18); rows sorted by column.  map_out[n] (may be NULL)
+ * receives the new vertex of every vertex.  *next is a new handle on g's stream
+ * (or on its own library stream if g's stream is library-owned). */
+int32_t louvain_aggregate(louvain_graph_t g, louvain_graph_t* next, int32_t* map_out);
+/* Full multilevel Louvain from singletons: phases of
+ * sweeps with the threshold schedule of P:330-334 (R13-R16), contraction
+ * between levels.  labels_out[n] (may be NULL): final community of every
+ * vertex; q_final / stats may be NULL.  On return the handle's partition is
+ * the final one. */
+int32_t louvain_run(louvain_graph_t g, const louvain_params_t* p, int32_t* labels_out, louvain_qnum_t* q_final,
+                    louvain_stats_t* stats);
+/* Thread-local message of the last error ("" if none). */
+const char* louvain_last_error(void);
+
+/* ---- multi-GPU: one process per GPU, vertex-range sharding ----
+ * The 128-byte NCCL unique id is created on rank 0 and broadcast by the caller
+ * (torch.distributed.broadcast_object_list). */
+int32_t louvain_dist_unique_id(uint8_t id[128]);
+/* Rank `rank` of `world` owns rows [v_begin, v_end) (rowptr_local has
+ * v_end - v_begin + 1 entries starting at 0, global column ids).  Every call on
+ * the returned handle is collective over the ranks; label buffers have global
+ * length n. */
+int32_t louvain_create_csr_dist(int64_t n, int64_t v_begin, int64_t v_end, const int64_t* rowptr_local,
+                                const int32_t* col_local, const uint32_t* w_local, uint32_t flags, int32_t rank,
+                                int32_t world, const uint8_t id[128], void* cuda_stream, louvain_graph_t* out);
+
+#ifdef __cplusplus
+}
+#endif
+#endif

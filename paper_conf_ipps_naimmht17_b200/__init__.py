@@ -1,0 +1,290 @@
+"""B200-native GPU Louvain hot path (Naim, Manne, Halappanavar, Tumeo, IPDPS'17).
+
+Thin ctypes binding over ``liblouvain.so`` (C-ABI ``include/louvain.h``):
+argument marshalling only -- every step of the method runs in the CUDA kernels
+of ``csrc/``.  Accepts numpy arrays (host) or torch CUDA tensors (device);
+torch is used only for device memory and streams.  There is no CPU fallback:
+importing this package fails loudly if the CUDA library is missing.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from dataclasses import dataclass
+from typing import Optional
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "liblouvain.so")
+
+OK, E_INVALID_ARG, E_INVALID_GRAPH, E_OVERFLOW, E_NOMEM, E_CUDA, E_NCCL, E_STATE, E_UNSUPPORTED = \
+    0, -1, -2, -3, -4, -5, -6, -7, -8
+VALIDATE, BORROW = 1, 2
+MODE_BIN_SYNC, MODE_RELAXED = 0, 1
+MAX_LEVELS = 256
+
+
+class Params(ctypes.Structure):
+    _fields_ = [("mode", ctypes.c_int32), ("singleton_rule", ctypes.c_int32),
+                ("revert_on_decrease", ctypes.c_int32), ("th_bin_exp", ctypes.c_int32),
+                ("th_final_exp", ctypes.c_int32), ("size_limit", ctypes.c_int64),
+                ("deg_bounds", ctypes.c_int64 * 6), ("max_sweeps", ctypes.c_int32),
+                ("max_levels", ctypes.c_int32)]
+
+
+class QNum(ctypes.Structure):
+    _fields_ = [("L", ctypes.c_uint64), ("S_lo", ctypes.c_uint64), ("S_hi", ctypes.c_uint64),
+                ("W", ctypes.c_uint64), ("q", ctypes.c_double)]
+
+    @property
+    def S(self) -> int:
+        return (int(self.S_hi) << 64) | int(self.S_lo)
+
+    @property
+    def num(self) -> int:
+        return int(self.L) * int(self.W) - self.S
+
+
+class Stats(ctypes.Structure):
+    _fields_ = [("levels", ctypes.c_int32), ("sweeps", ctypes.c_int32),
+                ("n", ctypes.c_int64 * MAX_LEVELS), ("nnz", ctypes.c_int64 * MAX_LEVELS),
+                ("sweeps_per_level", ctypes.c_int32 * MAX_LEVELS),
+                ("moved_per_level", ctypes.c_int64 * MAX_LEVELS),
+                ("num_start", ctypes.c_int64 * MAX_LEVELS), ("num_end", ctypes.c_int64 * MAX_LEVELS),
+                ("t_opt_ms", ctypes.c_double * MAX_LEVELS), ("t_agg_ms", ctypes.c_double * MAX_LEVELS),
+                ("t_total_ms", ctypes.c_double), ("t_sweep_ms_total", ctypes.c_double),
+                ("t_sweep_ms_first", ctypes.c_double), ("t_modularity_ms_total", ctypes.c_double),
+                ("edges_swept", ctypes.c_int64), ("q", QNum)]
+
+    def as_dict(self) -> dict:
+        lv = self.levels
+        return {"levels": lv, "sweeps": self.sweeps, "n": list(self.n[:lv]), "nnz": list(self.nnz[:lv]),
+                "sweeps_per_level": list(self.sweeps_per_level[:lv]),
+                "moved_per_level": list(self.moved_per_level[:lv]),
+                "num_start": list(self.num_start[:lv]), "num_end": list(self.num_end[:lv]),
+                "t_opt_ms": list(self.t_opt_ms[:lv]), "t_agg_ms": list(self.t_agg_ms[:lv]),
+                "t_total_ms": self.t_total_ms, "t_sweep_ms_total": self.t_sweep_ms_total,
+                "t_sweep_ms_first": self.t_sweep_ms_first, "t_modularity_ms_total": self.t_modularity_ms_total,
+                "edges_swept": self.edges_swept, "q": self.q.q, "L": int(self.q.L), "S": self.q.S,
+                "W": int(self.q.W)}
+
+
+FUNCS = {
+    # name: (restype, argtypes)
+    "louvain_params_default": (None, [ctypes.POINTER(Params)]),
+    "louvain_create_csr": (ctypes.c_int32, [ctypes.c_int64, ctypes.c_int64, ctypes.c_void_p, ctypes.c_void_p,
+                                            ctypes.c_void_p, ctypes.c_uint32, ctypes.c_void_p,
+                                            ctypes.POINTER(ctypes.c_void_p)]),
+    "louvain_destroy": (ctypes.c_int32, [ctypes.c_void_p]),
+    "louvain_get_info": (ctypes.c_int32, [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p]),
+    "louvain_get_csr": (ctypes.c_int32, [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p]),
+    "louvain_set_labels": (ctypes.c_int32, [ctypes.c_void_p, ctypes.c_void_p]),
+    "louvain_get_labels": (ctypes.c_int32, [ctypes.c_void_p, ctypes.c_void_p]),
+    "louvain_get_totals": (ctypes.c_int32, [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p]),
+    "louvain_sweep": (ctypes.c_int32, [ctypes.c_void_p, ctypes.POINTER(Params), ctypes.c_void_p,
+                                       ctypes.POINTER(QNum)]),
+    "louvain_modularity": (ctypes.c_int32, [ctypes.c_void_p, ctypes.c_void_p, ctypes.POINTER(QNum)]),
+    "louvain_aggregate": (ctypes.c_int32, [ctypes.c_void_p, ctypes.POINTER(ctypes.c_void_p), ctypes.c_void_p]),
+    "louvain_run": (ctypes.c_int32, [ctypes.c_void_p, ctypes.POINTER(Params), ctypes.c_void_p,
+                                     ctypes.POINTER(QNum), ctypes.POINTER(Stats)]),
+    "louvain_last_error": (ctypes.c_char_p, []),
+    "louvain_dist_unique_id": (ctypes.c_int32, [ctypes.c_void_p]),
+    "louvain_create_csr_dist": (ctypes.c_int32, [ctypes.c_int64, ctypes.c_int64, ctypes.c_int64, ctypes.c_void_p,
+                                                 ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint32, ctypes.c_int32,
+                                                 ctypes.c_int32, ctypes.c_void_p, ctypes.c_void_p,
+                                                 ctypes.POINTER(ctypes.c_void_p)]),
+}
+
+_LIB = None
+
+
+def lib():
+    """The loaded liblouvain.so (raises if it was not built: no fallback)."""
+    global _LIB
+    if _LIB is None:
+        if not os.path.exists(LIB_PATH):
+            raise ImportError(f"{LIB_PATH} is missing -- build it with __graft_entry__.build(); "
+                              "there is no CPU fallback")
+        L = ctypes.CDLL(LIB_PATH)
+        for name, (res, args) in FUNCS.items():
+            f = getattr(L, name)
+            f.restype = res
+            f.argtypes = args
+        _LIB = L
+    return _LIB
+
+
+class LouvainError(RuntimeError):
+    def __init__(self, code: int, msg: str):
+        super().__init__(f"louvain error {code}: {msg}")
+        self.code = code
+
+
+def _check(rc: int) -> None:
+    if rc != OK:
+        raise LouvainError(rc, lib().louvain_last_error().decode(errors="replace"))
+
+
+def params(**kw) -> Params:
+    """Paper defaults with overrides."""
+    p = Params()
+    lib().louvain_params_default(ctypes.byref(p))
+    for k, v in kw.items():
+        if k == "deg_bounds":
+            for t, b in enumerate(v):
+                p.deg_bounds[t] = b
+        else:
+            setattr(p, k, v)
+    return p
+
+
+def _ptr(x):
+    """(address, keepalive) of a numpy array or torch tensor (or None)."""
+    if x is None:
+        return None, None
+    if isinstance(x, np.ndarray):
+        x = np.ascontiguousarray(x)
+        return x.ctypes.data, x
+    if hasattr(x, "data_ptr"):
+        if not x.is_contiguous():
+            x = x.contiguous()
+        return x.data_ptr(), x
+    raise TypeError(f"unsupported buffer type {type(x)}")
+
+
+def _as(x, dtype):
+    if x is None:
+        return None
+    if isinstance(x, np.ndarray):
+        return np.ascontiguousarray(x, dtype=dtype)
+    import torch
+    tmap = {np.int64: torch.int64, np.int32: torch.int32, np.uint32: torch.uint32}
+    return x.to(tmap[dtype]).contiguous()
+
+
+class Graph:
+    """One level graph + partition state on the GPU (an opaque C-ABI handle)."""
+
+    def __init__(self, handle: ctypes.c_void_p, stream=None):
+        self._h = handle
+        self._stream = stream
+
+    @classmethod
+    def from_csr(cls, rowptr, col, w=None, validate: bool = False, borrow: bool = False, stream=None) -> "Graph":
+        rowptr = _as(rowptr, np.int64)
+        col = _as(col, np.int32)
+        w = _as(w, np.uint32)
+        n = int(rowptr.shape[0]) - 1
+        nnz = int(col.shape[0])
+        rp, k1 = _ptr(rowptr)
+        cp, k2 = _ptr(col)
+        wp, k3 = _ptr(w)
+        flags = (VALIDATE if validate else 0) | (BORROW if borrow else 0)
+        sp = None
+        if stream is not None:
+            sp = stream.cuda_stream if hasattr(stream, "cuda_stream") else int(stream)
+        h = ctypes.c_void_p()
+        _check(lib().louvain_create_csr(n, nnz, rp, cp if nnz else None, wp, flags, sp, ctypes.byref(h)))
+        g = cls(h, stream)
+        g._borrowed = (rowptr, col, w) if borrow else None
+        return g
+
+    @classmethod
+    def from_host_graph(cls, g, **kw) -> "Graph":
+        return cls.from_csr(g.rowptr, g.col, g.w, **kw)
+
+    def close(self) -> None:
+        if self._h is not None and self._h.value:
+            lib().louvain_destroy(self._h)
+        self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+    # ---------------------------------------------------------------- queries
+    def info(self) -> tuple[int, int, int]:
+        n, nnz, W = ctypes.c_int64(), ctypes.c_int64(), ctypes.c_uint64()
+        _check(lib().louvain_get_info(self._h, ctypes.byref(n), ctypes.byref(nnz), ctypes.byref(W)))
+        return n.value, nnz.value, W.value
+
+    @property
+    def n(self) -> int:
+        return self.info()[0]
+
+    def csr(self):
+        n, nnz, _ = self.info()
+        rowptr = np.empty(n + 1, dtype=np.int64)
+        col = np.empty(max(nnz, 1), dtype=np.int32)
+        w = np.empty(max(nnz, 1), dtype=np.uint32)
+        _check(lib().louvain_get_csr(self._h, rowptr.ctypes.data, col.ctypes.data, w.ctypes.data))
+        return rowptr, col[:nnz], w[:nnz]
+
+    def labels(self, out=None):
+        n = self.n
+        if out is None:
+            out = np.empty(max(n, 1), dtype=np.int32)
+        p, keep = _ptr(out)
+        _check(lib().louvain_get_labels(self._h, p))
+        return out[:n] if isinstance(out, np.ndarray) else out
+
+    def totals(self):
+        n = self.n
+        a = np.empty(max(n, 1), dtype=np.uint32)
+        s = np.empty(max(n, 1), dtype=np.int32)
+        _check(lib().louvain_get_totals(self._h, a.ctypes.data, s.ctypes.data))
+        return a[:n], s[:n]
+
+    def set_labels(self, labels=None) -> None:
+        p, keep = _ptr(_as(labels, np.int32))
+        _check(lib().louvain_set_labels(self._h, p))
+
+    # ---------------------------------------------------------------- the method
+    def sweep(self, p: Optional[Params] = None, with_q: bool = True):
+        """One iteration of Alg. 1's repeat body; returns (moved, QNum or None)."""
+        moved = ctypes.c_int64()
+        q = QNum()
+        _check(lib().louvain_sweep(self._h, ctypes.byref(p or params()), ctypes.byref(moved),
+                                   ctypes.byref(q) if with_q else None))
+        return moved.value, (q if with_q else None)
+
+    def modularity(self, labels=None) -> QNum:
+        p, keep = _ptr(_as(labels, np.int32))
+        q = QNum()
+        _check(lib().louvain_modularity(self._h, p, ctypes.byref(q)))
+        return q
+
+    def aggregate(self, with_map: bool = True):
+        """Alg. 3: returns (next Graph, map ndarray or None)."""
+        n = self.n
+        mp = np.empty(max(n, 1), dtype=np.int32) if with_map else None
+        h = ctypes.c_void_p()
+        _check(lib().louvain_aggregate(self._h, ctypes.byref(h), mp.ctypes.data if with_map else None))
+        return Graph(h, self._stream), (mp[:n] if with_map else None)
+
+    def run(self, p: Optional[Params] = None, labels_out=None, want_labels: bool = True):
+        """Full multilevel Louvain; returns (labels, QNum, stats dict)."""
+        n = self.n
+        if labels_out is None and want_labels:
+            labels_out = np.empty(max(n, 1), dtype=np.int32)
+        lp, keep = _ptr(labels_out)
+        q = QNum()
+        st = Stats()
+        _check(lib().louvain_run(self._h, ctypes.byref(p or params()), lp, ctypes.byref(q), ctypes.byref(st)))
+        lab = labels_out[:n] if isinstance(labels_out, np.ndarray) else labels_out
+        return lab, q, st.as_dict()
+
+
+def run(rowptr, col, w=None, p: Optional[Params] = None, **kw):
+    """One-call convenience: CSR in (host or device), (labels, QNum, stats) out."""
+    with Graph.from_csr(rowptr, col, w, **kw) as g:
+        return g.run(p)

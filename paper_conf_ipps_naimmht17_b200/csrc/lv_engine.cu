@@ -1,0 +1,608 @@
+// lv_engine.cu -- C-ABI (include/louvain.h) and the level driver of the GPU
+// Louvain hot path: one sweep = Alg. 1's repeat body, the phase
+// loop with the threshold schedule (R13-R15), the multilevel loop
+// (R16) and label composition (R22).
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <chrono>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "lv_internal.cuh"
+
+#define LV_API extern "C" __attribute__((visibility("default")))
+
+namespace lv {
+
+static thread_local std::string g_err;
+void set_error(const std::string& msg) { g_err = msg; }
+
+int32_t cuda_fail(cudaError_t e, const char* what, const char* file, int line) {
+  g_err = std::string(what) + ": " + cudaGetErrorString(e) + " (" + file + ":" + std::to_string(line) + ")";
+  if (e == cudaErrorMemoryAllocation) {
+    cudaGetLastError();
+    return LOUVAIN_E_NOMEM;
+  }
+  return LOUVAIN_E_CUDA;
+}
+
+int32_t dmalloc(void** p, size_t bytes, cudaStream_t s) {
+  *p = nullptr;
+  cudaError_t e = cudaMallocAsync(p, bytes ? bytes : 1, s);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    g_err = "device allocation of " + std::to_string(bytes) + " bytes failed: " + cudaGetErrorString(e);
+    return LOUVAIN_E_NOMEM;
+  }
+  return LOUVAIN_OK;
+}
+
+void dfree(void* p, cudaStream_t s) {
+  if (p) cudaFreeAsync(p, s);
+}
+
+bool is_device_ptr(const void* p) {
+  if (!p) return false;
+  cudaPointerAttributes at;
+  if (cudaPointerGetAttributes(&at, p) != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  return at.type == cudaMemoryTypeDevice || at.type == cudaMemoryTypeManaged;
+}
+
+namespace {
+
+__global__ void k_fill_u32(uint32_t* p, int64_t n, uint32_t v) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) p[i] = v;
+}
+__global__ void k_iota(int32_t* p, int64_t n) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) p[i] = (int32_t)i;
+}
+
+void keep_pool_memory(int device) {
+  static bool done[64] = {false};
+  if (device < 0 || device >= 64 || done[device]) return;
+  cudaMemPool_t pool;
+  if (cudaDeviceGetDefaultMemPool(&pool, device) == cudaSuccess) {
+    uint64_t thr = UINT64_MAX;
+    cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+  }
+  done[device] = true;
+}
+
+int32_t check_params(const louvain_params_t& p) {
+  if (p.mode != LOUVAIN_MODE_BIN_SYNC && p.mode != LOUVAIN_MODE_RELAXED) {
+    set_error("params.mode must be BIN_SYNC (0) or RELAXED (1)");
+    return LOUVAIN_E_INVALID_ARG;
+  }
+  if (p.singleton_rule < 0 || p.singleton_rule > 2) {
+    set_error("params.singleton_rule must be 0, 1 or 2");
+    return LOUVAIN_E_INVALID_ARG;
+  }
+  if (p.th_bin_exp < 0 || p.th_bin_exp > 18 || p.th_final_exp < 0 || p.th_final_exp > 18) {
+    set_error("threshold exponents must be in [0, 18]");
+    return LOUVAIN_E_INVALID_ARG;
+  }
+  for (int t = 0; t < 6; ++t) {
+    if (p.deg_bounds[t] < 1 || (t > 0 && p.deg_bounds[t] <= p.deg_bounds[t - 1])) {
+      set_error("deg_bounds must be positive and strictly increasing");
+      return LOUVAIN_E_INVALID_ARG;
+    }
+  }
+  return LOUVAIN_OK;
+}
+
+int32_t init_handle(Handle& h, void* stream) {
+  LV_CUDA(cudaGetDevice(&h.device));
+  keep_pool_memory(h.device);
+  if (stream) {
+    h.stream = (cudaStream_t)stream;
+    h.own_stream = false;
+  } else {
+    LV_CUDA(cudaStreamCreateWithFlags(&h.stream, cudaStreamNonBlocking));
+    h.own_stream = true;
+  }
+  LV_CUDA(cudaMalloc(&h.ctl, sizeof(DevCtl)));
+  LV_CUDA(cudaMemset(h.ctl, 0, sizeof(DevCtl)));
+  LV_CUDA(cudaMallocHost(&h.h_ctl, sizeof(DevCtl)));
+  for (auto& e : h.ev) LV_CUDA(cudaEventCreate(&e));
+  return LOUVAIN_OK;
+}
+
+void destroy_handle(Handle& h) {
+  cudaSetDevice(h.device);
+  if (h.stream) {
+    level_free(h.lv, h.stream);
+    cudaStreamSynchronize(h.stream);
+  }
+  if (h.ctl) cudaFree(h.ctl);
+  if (h.h_ctl) cudaFreeHost(h.h_ctl);
+  for (auto& e : h.ev)
+    if (e) cudaEventDestroy(e);
+  if (h.own_stream && h.stream) cudaStreamDestroy(h.stream);
+}
+
+// Every call first makes the handle's device current and refuses poisoned handles.
+struct DeviceScope {
+  int prev = -1;
+  explicit DeviceScope(int dev) {
+    cudaGetDevice(&prev);
+    if (prev != dev) cudaSetDevice(dev);
+  }
+  ~DeviceScope() {
+    int cur = -1;
+    cudaGetDevice(&cur);
+    if (prev >= 0 && cur != prev) cudaSetDevice(prev);
+  }
+};
+
+int32_t guard(louvain_graph_t g) {
+  if (!g) {
+    set_error("null handle");
+    return LOUVAIN_E_INVALID_ARG;
+  }
+  if (g->h.poisoned) {
+    set_error("handle poisoned by an earlier sticky CUDA error");
+    return LOUVAIN_E_STATE;
+  }
+  return LOUVAIN_OK;
+}
+
+int32_t finish_call(Handle& h, int32_t rc) {
+  if (rc == LOUVAIN_E_CUDA) {
+    cudaError_t e = cudaPeekAtLastError();
+    if (e == cudaErrorIllegalAddress || e == cudaErrorLaunchFailure || e == cudaErrorIllegalInstruction ||
+        e == cudaErrorMisalignedAddress || e == cudaErrorHardwareStackError)
+      h.poisoned = true;
+  }
+  return rc;
+}
+
+bool bucket_nonempty(const Level& L, int b) { return L.class_off[4 * b + 3] > L.class_off[4 * b]; }
+
+// One sweep body: for each non-empty bucket 1..7 its sweep kernels, then its
+// commit (BIN_SYNC) -- or a single commit at the end (RELAXED).
+int32_t sweep_body(Handle& h, Level& L, const louvain_params_t& p) {
+  LV_CUDA(cudaMemsetAsync(h.ctl, 0, offsetof(DevCtl, L), h.stream));  // logn + bounds
+  int commits = 0;
+  for (int b = 1; b <= 7; ++b) {
+    if (!bucket_nonempty(L, b)) continue;
+    LV_TRY(launch_sweep_bucket(h, L, p, b));
+    if (p.mode == LOUVAIN_MODE_BIN_SYNC) LV_TRY(launch_commit(h, L, commits++));
+  }
+  if (p.mode == LOUVAIN_MODE_RELAXED) LV_TRY(launch_commit(h, L, commits++));
+  return LOUVAIN_OK;
+}
+
+using i128 = __int128;
+
+i128 pow10_i128(int p) {
+  i128 r = 1;
+  for (int t = 0; t < p; ++t) r *= 10;
+  return r;
+}
+
+// (num_new - num_old) / W^2 < 10^-p, in exact integers (R13)
+bool below_threshold(int64_t num_new, int64_t num_old, uint64_t W, int p) {
+  i128 d = (i128)num_new - (i128)num_old;
+  return d * pow10_i128(p) < (i128)W * (i128)W;
+}
+
+int64_t qnum_of(uint64_t L, uint64_t S, uint64_t W) { return (int64_t)((i128)L * (i128)W - (i128)S); }
+
+void fill_q(louvain_qnum_t* q, uint64_t L, uint64_t S, uint64_t W) {
+  if (!q) return;
+  q->L = L;
+  q->S_lo = S;
+  q->S_hi = 0;
+  q->W = W;
+  q->q = W ? (double)qnum_of(L, S, W) / ((double)W * (double)W) : 0.0;
+}
+
+int32_t copy_out(void* dst, const void* src, size_t bytes, cudaStream_t s) {
+  if (!dst || !bytes) return LOUVAIN_OK;
+  LV_CUDA(cudaMemcpyAsync(dst, src, bytes, cudaMemcpyDefault, s));
+  return LOUVAIN_OK;
+}
+
+float elapsed(cudaEvent_t a, cudaEvent_t b) {
+  float ms = 0.f;
+  cudaEventElapsedTime(&ms, a, b);
+  return ms;
+}
+
+// The multilevel driver (SURVEY 8(c) listing; oracle/louvain_oracle.c orc_louvain
+// is the independent CPU transcription of the same control flow).
+int32_t run_impl(Handle& h, const louvain_params_t& p, int32_t* labels_out, louvain_qnum_t* q_final,
+                 louvain_stats_t* st) {
+  cudaStream_t s = h.stream;
+  Level& L0 = h.lv;
+  const int64_t n0 = L0.n;
+  const uint64_t W = L0.W;
+  louvain_stats_t local;
+  std::memset(&local, 0, sizeof local);
+  auto t_begin = std::chrono::steady_clock::now();
+  int32_t* lab = nullptr;
+  LV_TRY(dalloc(&lab, n0, s));
+  if (n0) k_iota<<<grid_for(n0, 256), 256, 0, s>>>(lab, n0);
+  // level 0 starts from singletons
+  if (n0) {
+    k_iota<<<grid_for(n0, 256), 256, 0, s>>>(L0.C, n0);
+    LV_TRY(level_set_labels(h, L0, L0.C));
+  }
+  Level owned;   // current contracted level (levels >= 1)
+  Level* cur = &L0;
+  int32_t* map = nullptr;
+  if (W > 0) {
+    for (int level = 0;; ++level) {
+      if ((p.max_levels > 0 && level >= p.max_levels) || level >= LOUVAIN_MAX_LEVELS) break;
+      cudaEvent_t e_lvl0, e_lvl1;
+      cudaEventCreate(&e_lvl0);
+      cudaEventCreate(&e_lvl1);
+      cudaEventRecord(e_lvl0, s);
+      Level& L = *cur;
+      const int pexp = (L.n > p.size_limit) ? p.th_bin_exp : p.th_final_exp;  // P:330, R14
+      LV_TRY(level_binning(h, L, p));
+      uint64_t Lq, Sq;
+      LV_TRY(level_modularity(h, L, L.C, &Lq, &Sq));
+      const int64_t num_start = qnum_of(Lq, Sq, W);
+      int64_t num_prev = num_start;
+      int64_t moved_level = 0;
+      int32_t sweeps = 0;
+      for (;;) {
+        if (p.max_sweeps > 0 && sweeps >= p.max_sweeps) break;
+        cudaEventRecord(h.ev[0], s);
+        LV_TRY(sweep_body(h, L, p));
+        cudaEventRecord(h.ev[1], s);
+        LV_TRY(launch_modularity(h, L, L.C));
+        cudaEventRecord(h.ev[2], s);
+        LV_CUDA(cudaMemcpyAsync(h.h_ctl, h.ctl, sizeof(DevCtl), cudaMemcpyDeviceToHost, s));
+        LV_CUDA(cudaStreamSynchronize(s));
+        const float t_sw = elapsed(h.ev[0], h.ev[1]);
+        local.t_sweep_ms_total += t_sw;
+        local.t_modularity_ms_total += elapsed(h.ev[1], h.ev[2]);
+        if (level == 0 && sweeps == 0) local.t_sweep_ms_first = t_sw;
+        local.edges_swept += L.nnz;
+        ++sweeps;
+        const int64_t moved = (int64_t)h.h_ctl->logn;
+        const int64_t num = qnum_of(h.h_ctl->L, h.h_ctl->S, W);
+        if (p.revert_on_decrease && num < num_prev) {  // R15
+          LV_TRY(launch_revert(h, L));
+          break;
+        }
+        moved_level += moved;
+        if (moved == 0 || below_threshold(num, num_prev, W, pexp)) break;  // Alg. 1 l.12, R13
+        num_prev = num;
+      }
+      LV_TRY(level_modularity(h, L, L.C, &Lq, &Sq));
+      const int64_t num_end = qnum_of(Lq, Sq, W);
+      cudaEventRecord(e_lvl1, s);
+      local.n[level] = L.n;
+      local.nnz[level] = L.nnz;
+      local.sweeps_per_level[level] = sweeps;
+      local.moved_per_level[level] = moved_level;
+      local.num_start[level] = num_start;
+      local.num_end[level] = num_end;
+      local.levels = level + 1;
+      local.sweeps += sweeps;
+      LV_CUDA(cudaEventSynchronize(e_lvl1));
+      local.t_opt_ms[level] = elapsed(e_lvl0, e_lvl1);
+      if (moved_level == 0 || below_threshold(num_end, num_start, W, p.th_final_exp)) {  // R16
+        LV_TRY(compose_labels(h, lab, n0, L.C));
+        cudaEventDestroy(e_lvl0);
+        cudaEventDestroy(e_lvl1);
+        break;
+      }
+      // aggregation phase (Alg. 3)
+      cudaEventRecord(e_lvl0, s);
+      Level next;
+      LV_TRY(dalloc(&map, L.n, s));
+      LV_TRY(level_contract(h, L, next, map));
+      LV_TRY(compose_labels(h, lab, n0, map));
+      dfree(map, s);
+      map = nullptr;
+      LV_TRY(level_setup(h, next));
+      cudaEventRecord(e_lvl1, s);
+      LV_CUDA(cudaEventSynchronize(e_lvl1));
+      local.t_agg_ms[level] = elapsed(e_lvl0, e_lvl1);
+      cudaEventDestroy(e_lvl0);
+      cudaEventDestroy(e_lvl1);
+      if (cur != &L0) level_free(owned, s);
+      owned = next;
+      cur = &owned;
+    }
+  }
+  if (cur != &L0) level_free(owned, s);
+  // the handle's partition becomes the final one
+  LV_TRY(level_set_labels(h, L0, lab));
+  uint64_t Lq = 0, Sq = 0;
+  if (n0) LV_TRY(level_modularity(h, L0, L0.C, &Lq, &Sq));
+  LV_TRY(copy_out(labels_out, lab, sizeof(int32_t) * (size_t)n0, s));
+  LV_CUDA(cudaStreamSynchronize(s));
+  dfree(lab, s);
+  fill_q(&local.q, Lq, Sq, W);
+  local.t_total_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t_begin).count();
+  if (q_final) *q_final = local.q;
+  if (st) *st = local;
+  return LOUVAIN_OK;
+}
+
+// Stage caller input (host or device) as device memory: returns a device pointer
+// (the caller's own if it is already device memory and borrow is allowed).
+template <class T>
+int32_t stage(const T* src, int64_t count, bool borrow, cudaStream_t s, T** dst, bool* owned) {
+  *owned = false;
+  if (!src) { *dst = nullptr; return LOUVAIN_OK; }
+  if (borrow && is_device_ptr(src)) {
+    *dst = const_cast<T*>(src);
+    return LOUVAIN_OK;
+  }
+  LV_TRY(dalloc(dst, count, s));
+  LV_CUDA(cudaMemcpyAsync(*dst, src, sizeof(T) * (size_t)count, cudaMemcpyDefault, s));
+  *owned = true;
+  return LOUVAIN_OK;
+}
+
+}  // namespace
+}  // namespace lv
+
+using namespace lv;
+
+LV_API void louvain_params_default(louvain_params_t* p) {
+  if (!p) return;
+  std::memset(p, 0, sizeof *p);
+  p->mode = LOUVAIN_MODE_BIN_SYNC;
+  p->singleton_rule = 1;
+  p->revert_on_decrease = 1;
+  p->th_bin_exp = 2;
+  p->th_final_exp = 6;
+  p->size_limit = 100000;
+  const int64_t b[6] = {4, 8, 16, 32, 84, 319};
+  std::memcpy(p->deg_bounds, b, sizeof b);
+  p->max_sweeps = 0;
+  p->max_levels = 0;
+}
+
+LV_API const char* louvain_last_error(void) { return g_err.c_str(); }
+
+LV_API int32_t louvain_create_csr(int64_t n, int64_t nnz, const int64_t* rowptr, const int32_t* col, const uint32_t* w,
+                                  uint32_t flags, void* cuda_stream, louvain_graph_t* out) {
+  g_err.clear();
+  if (!out || n < 0 || nnz < 0 || !rowptr || (nnz > 0 && !col) || n > INT32_MAX - 1) {
+    set_error("louvain_create_csr: null/negative argument or n >= 2^31 - 1");
+    return LOUVAIN_E_INVALID_ARG;
+  }
+  *out = nullptr;
+  const bool validate = flags & LOUVAIN_VALIDATE;
+  const bool borrow = flags & LOUVAIN_BORROW;
+  // Host-side validation before any device work (works without a GPU for host inputs).
+  const bool host_in = !is_device_ptr(rowptr);
+  if (host_in) {
+    LV_TRY(validate_csr_host(n, nnz, rowptr, col, w, validate, nullptr));
+  } else if (validate) {
+    std::vector<int64_t> r(n + 1);
+    std::vector<int32_t> c(nnz);
+    std::vector<uint32_t> ww(w ? nnz : 0);
+    LV_CUDA(cudaMemcpy(r.data(), rowptr, 8 * (n + 1), cudaMemcpyDefault));
+    if (nnz) LV_CUDA(cudaMemcpy(c.data(), col, 4 * nnz, cudaMemcpyDefault));
+    if (w && nnz) LV_CUDA(cudaMemcpy(ww.data(), w, 4 * nnz, cudaMemcpyDefault));
+    LV_TRY(validate_csr_host(n, nnz, r.data(), c.data(), w ? ww.data() : nullptr, true, nullptr));
+  }
+  louvain_graph_s* g = new louvain_graph_s();
+  Handle& h = g->h;
+  int32_t rc = init_handle(h, cuda_stream);
+  if (rc != LOUVAIN_OK) {
+    destroy_handle(h);
+    delete g;
+    return rc;
+  }
+  Level& L = h.lv;
+  L.n = n;
+  L.nnz = nnz;
+  // LOUVAIN_BORROW: use device inputs in place only if every given array is device memory
+  const bool all_dev = is_device_ptr(rowptr) && (nnz == 0 || is_device_ptr(col)) && (!w || is_device_ptr(w));
+  const bool use_in_place = borrow && all_dev;
+  bool o1 = false, o2 = false, o3 = false;
+  rc = stage(rowptr, n + 1, use_in_place, h.stream, &L.rowptr, &o1);
+  if (rc == LOUVAIN_OK && nnz) rc = stage(col, nnz, use_in_place, h.stream, &L.col, &o2);
+  if (rc == LOUVAIN_OK && w && nnz) rc = stage(w, nnz, use_in_place, h.stream, &L.w, &o3);
+  L.owns_csr = !use_in_place;
+  if (rc == LOUVAIN_OK && !L.col) rc = dalloc(&L.col, 1, h.stream);
+  if (rc == LOUVAIN_OK) rc = level_alloc_state(L, h.stream);
+  if (rc == LOUVAIN_OK) rc = level_setup(h, L);
+  if (rc == LOUVAIN_OK) {
+    cudaError_t e = cudaStreamSynchronize(h.stream);
+    if (e != cudaSuccess) rc = cuda_fail(e, "cudaStreamSynchronize", __FILE__, __LINE__);
+  }
+  if (rc != LOUVAIN_OK) {
+    destroy_handle(h);
+    delete g;
+    return rc;
+  }
+  *out = g;
+  return LOUVAIN_OK;
+}
+
+LV_API int32_t louvain_destroy(louvain_graph_t g) {
+  if (!g) return LOUVAIN_OK;
+  destroy_handle(g->h);
+  delete g;
+  return LOUVAIN_OK;
+}
+
+LV_API int32_t louvain_get_info(louvain_graph_t g, int64_t* n, int64_t* nnz, uint64_t* W) {
+  LV_TRY(guard(g));
+  if (n) *n = g->h.lv.n;
+  if (nnz) *nnz = g->h.lv.nnz;
+  if (W) *W = g->h.lv.W;
+  return LOUVAIN_OK;
+}
+
+LV_API int32_t louvain_get_csr(louvain_graph_t g, int64_t* rowptr, int32_t* col, uint32_t* w) {
+  LV_TRY(guard(g));
+  Handle& h = g->h;
+  DeviceScope ds(h.device);
+  Level& L = h.lv;
+  int32_t rc = copy_out(rowptr, L.rowptr, 8 * (size_t)(L.n + 1), h.stream);
+  if (!rc) rc = copy_out(col, L.col, 4 * (size_t)L.nnz, h.stream);
+  if (!rc && w && L.nnz) {
+    if (L.w) {
+      rc = copy_out(w, L.w, 4 * (size_t)L.nnz, h.stream);
+    } else if (is_device_ptr(w)) {
+      k_fill_u32<<<grid_for(L.nnz, 256), 256, 0, h.stream>>>(w, L.nnz, 1u);
+    } else {
+      cudaStreamSynchronize(h.stream);
+      for (int64_t e = 0; e < L.nnz; ++e) w[e] = 1u;
+    }
+  }
+  if (!rc) {
+    cudaError_t e = cudaStreamSynchronize(h.stream);
+    if (e != cudaSuccess) rc = cuda_fail(e, "sync", __FILE__, __LINE__);
+  }
+  return finish_call(h, rc);
+}
+
+LV_API int32_t louvain_set_labels(louvain_graph_t g, const int32_t* labels) {
+  LV_TRY(guard(g));
+  Handle& h = g->h;
+  DeviceScope ds(h.device);
+  Level& L = h.lv;
+  int32_t rc = LOUVAIN_OK;
+  if (!labels) {
+    if (L.n) k_iota<<<grid_for(L.n, 256), 256, 0, h.stream>>>(L.C, L.n);
+    rc = level_set_labels(h, L, L.C);
+  } else {
+    int32_t* d = nullptr;
+    bool owned = false;
+    rc = stage(labels, L.n, false, h.stream, &d, &owned);
+    if (!rc) rc = level_set_labels(h, L, d);
+    if (owned) dfree(d, h.stream);
+  }
+  return finish_call(h, rc);
+}
+
+LV_API int32_t louvain_get_labels(louvain_graph_t g, int32_t* labels_out) {
+  LV_TRY(guard(g));
+  Handle& h = g->h;
+  DeviceScope ds(h.device);
+  if (!labels_out && h.lv.n) { set_error("null labels_out"); return LOUVAIN_E_INVALID_ARG; }
+  int32_t rc = copy_out(labels_out, h.lv.C, 4 * (size_t)h.lv.n, h.stream);
+  if (!rc) {
+    cudaError_t e = cudaStreamSynchronize(h.stream);
+    if (e != cudaSuccess) rc = cuda_fail(e, "sync", __FILE__, __LINE__);
+  }
+  return finish_call(h, rc);
+}
+
+LV_API int32_t louvain_get_totals(louvain_graph_t g, uint32_t* a_out, int32_t* size_out) {
+  LV_TRY(guard(g));
+  Handle& h = g->h;
+  DeviceScope ds(h.device);
+  int32_t rc = copy_out(a_out, h.lv.a, 4 * (size_t)h.lv.n, h.stream);
+  if (!rc) rc = copy_out(size_out, h.lv.size, 4 * (size_t)h.lv.n, h.stream);
+  if (!rc) {
+    cudaError_t e = cudaStreamSynchronize(h.stream);
+    if (e != cudaSuccess) rc = cuda_fail(e, "sync", __FILE__, __LINE__);
+  }
+  return finish_call(h, rc);
+}
+
+LV_API int32_t louvain_sweep(louvain_graph_t g, const louvain_params_t* p, int64_t* moved, louvain_qnum_t* q_after) {
+  LV_TRY(guard(g));
+  louvain_params_t pp;
+  if (p) pp = *p; else louvain_params_default(&pp);
+  LV_TRY(check_params(pp));
+  Handle& h = g->h;
+  DeviceScope ds(h.device);
+  Level& L = h.lv;
+  int32_t rc = level_binning(h, L, pp);
+  if (!rc) rc = sweep_body(h, L, pp);
+  if (!rc && q_after) rc = launch_modularity(h, L, L.C);
+  if (!rc) {
+    cudaError_t e = cudaMemcpyAsync(h.h_ctl, h.ctl, sizeof(DevCtl), cudaMemcpyDeviceToHost, h.stream);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(h.stream);
+    if (e != cudaSuccess) rc = cuda_fail(e, "sweep", __FILE__, __LINE__);
+  }
+  if (!rc) {
+    if (moved) *moved = (int64_t)h.h_ctl->logn;
+    if (q_after) fill_q(q_after, h.h_ctl->L, h.h_ctl->S, L.W);
+  }
+  return finish_call(h, rc);
+}
+
+LV_API int32_t louvain_modularity(louvain_graph_t g, const int32_t* labels, louvain_qnum_t* q) {
+  LV_TRY(guard(g));
+  if (!q) { set_error("null q"); return LOUVAIN_E_INVALID_ARG; }
+  Handle& h = g->h;
+  DeviceScope ds(h.device);
+  Level& L = h.lv;
+  int32_t* d = L.C;
+  bool owned = false;
+  int32_t rc = LOUVAIN_OK;
+  if (labels) rc = stage(labels, L.n, false, h.stream, &d, &owned);
+  uint64_t Lq = 0, Sq = 0;
+  if (!rc) rc = level_modularity(h, L, d, &Lq, &Sq);
+  if (owned) dfree(d, h.stream);
+  if (!rc) fill_q(q, Lq, Sq, L.W);
+  return finish_call(h, rc);
+}
+
+LV_API int32_t louvain_aggregate(louvain_graph_t g, louvain_graph_t* next, int32_t* map_out) {
+  LV_TRY(guard(g));
+  if (!next) { set_error("null next"); return LOUVAIN_E_INVALID_ARG; }
+  Handle& h = g->h;
+  DeviceScope ds(h.device);
+  louvain_graph_s* ng = new louvain_graph_s();
+  // a library-owned stream dies with its handle, so the child gets its own
+  int32_t rc = init_handle(ng->h, h.own_stream ? nullptr : (void*)h.stream);
+  int32_t* map = nullptr;
+  if (!rc) rc = dalloc(&map, h.lv.n, h.stream);
+  if (!rc) rc = level_contract(h, h.lv, ng->h.lv, map);
+  if (!rc) {
+    cudaError_t e = cudaStreamSynchronize(h.stream);
+    if (e != cudaSuccess) rc = cuda_fail(e, "aggregate", __FILE__, __LINE__);
+  }
+  if (!rc) rc = level_setup(ng->h, ng->h.lv);
+  if (!rc) rc = copy_out(map_out, map, 4 * (size_t)h.lv.n, h.stream);
+  if (!rc) {
+    cudaError_t e = cudaStreamSynchronize(h.stream);
+    if (e != cudaSuccess) rc = cuda_fail(e, "aggregate", __FILE__, __LINE__);
+  }
+  dfree(map, h.stream);
+  if (rc) {
+    destroy_handle(ng->h);
+    delete ng;
+    return finish_call(h, rc);
+  }
+  *next = ng;
+  return LOUVAIN_OK;
+}
+
+LV_API int32_t louvain_run(louvain_graph_t g, const louvain_params_t* p, int32_t* labels_out, louvain_qnum_t* q_final,
+                           louvain_stats_t* stats) {
+  LV_TRY(guard(g));
+  louvain_params_t pp;
+  if (p) pp = *p; else louvain_params_default(&pp);
+  LV_TRY(check_params(pp));
+  Handle& h = g->h;
+  DeviceScope ds(h.device);
+  return finish_call(h, run_impl(h, pp, labels_out, q_final, stats));
+}
+
+LV_API int32_t louvain_dist_unique_id(uint8_t id[128]) {
+  (void)id;
+  set_error("multi-GPU not built yet");
+  return LOUVAIN_E_UNSUPPORTED;
+}
+
+LV_API int32_t louvain_create_csr_dist(int64_t n, int64_t v_begin, int64_t v_end, const int64_t* rowptr_local,
+                                       const int32_t* col_local, const uint32_t* w_local, uint32_t flags, int32_t rank,
+                                       int32_t world, const uint8_t id[128], void* cuda_stream, louvain_graph_t* out) {
+  (void)n; (void)v_begin; (void)v_end; (void)rowptr_local; (void)col_local; (void)w_local; (void)flags;
+  (void)rank; (void)world; (void)id; (void)cuda_stream; (void)out;
+  set_error("multi-GPU not built yet");
+  return LOUVAIN_E_UNSUPPORTED;
+}

@@ -1,0 +1,643 @@
+// lv_level.cu -- per-level kernels of the GPU Louvain hot path (sm_100a):
+// level setup (Alg. 1 l.2), degree binning, commit
+// (Alg. 1 l.8-11), exact modularity (Eq. 1) and
+// contraction (Alg. 3).  See DESIGN.md for the byte model of each.
+#include <cub/cub.cuh>
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstring>
+#include <vector>
+
+#include "lv_device.cuh"
+#include "lv_internal.cuh"
+
+namespace lv {
+
+size_t hub_partial_bytes();
+
+namespace {
+
+constexpr int kTileEdges = 2048;  // edges per block tile in edge-centric kernels
+constexpr int kTileRows = 2048;   // rowptr entries staged in smem per tile
+
+__global__ void k_degrees_unit(const int64_t* rowptr, int64_t n, uint32_t* k) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    k[i] = (uint32_t)(rowptr[i + 1] - rowptr[i]);
+}
+
+__global__ void k_init_singletons(const uint32_t* k, int64_t n, int32_t* C, uint32_t* a, int32_t* size) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    C[i] = (int32_t)i;  // C[i] = i at the start of each phase
+    a[i] = k[i];        // a_C(i) = k_i initially
+    size[i] = 1;
+  }
+}
+
+__global__ void k_totals_zero(int64_t n, uint32_t* a, int32_t* size) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    a[i] = 0;
+    size[i] = 0;
+  }
+}
+
+__global__ void k_totals_add(const int32_t* C, const uint32_t* k, int64_t n, uint32_t* a, int32_t* size,
+                             unsigned long long* bad) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    int32_t c = C[i];
+    if (c < 0 || c >= n) { atomicAdd(bad, 1ull); continue; }
+    atomicAdd(&a[c], k[i]);  // a_c = sum_{i in c} k_i
+    atomicAdd(&size[c], 1);
+  }
+}
+
+// class = 4*bucket + sub  (lv_internal.cuh)
+__global__ void k_classify(const int64_t* rowptr, int64_t n, int64_t b0, int64_t b1, int64_t b2, int64_t b3,
+                           int64_t b4, int64_t b5, uint8_t* cls, int32_t* iota, unsigned long long* hist) {
+  __shared__ unsigned long long sh[kNumClasses];
+  if (threadIdx.x < kNumClasses) sh[threadIdx.x] = 0;
+  __syncthreads();
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t d = rowptr[i + 1] - rowptr[i];  // R11: row length incl. self-loop
+    int b;
+    if (d == 0) b = 0;
+    else if (d <= b0) b = 1;
+    else if (d <= b1) b = 2;
+    else if (d <= b2) b = 3;
+    else if (d <= b3) b = 4;
+    else if (d <= b4) b = 5;
+    else if (d <= b5) b = 6;
+    else b = 7;
+    const int sub = d < kCtaLargeMin ? 0 : (d < kHubMin ? 1 : 2);
+    const uint8_t c = (uint8_t)(4 * b + sub);
+    cls[i] = c;
+    iota[i] = (int32_t)i;
+    atomicAdd(&sh[c], 1ull);
+  }
+  __syncthreads();
+  if (threadIdx.x < kNumClasses && sh[threadIdx.x]) atomicAdd(&hist[threadIdx.x], sh[threadIdx.x]);
+}
+
+__global__ void k_hub_degrees(const int32_t* hv, int64_t nh, const int64_t* rowptr, int64_t* deg) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < nh; i += (int64_t)gridDim.x * blockDim.x) {
+    int32_t v = hv[i];
+    deg[i] = rowptr[v + 1] - rowptr[v];
+    deg[nh + i] = rowptr[v];
+  }
+}
+
+__global__ void k_fill_u64(unsigned long long* p, int64_t n, unsigned long long v) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) p[i] = v;
+}
+
+// Commit of one bucket (Alg. 1 l.8-11): C[i] = newComm[i] and the exact
+// integer a_c / size_c deltas (identical to recomputing a_c, R12).
+__global__ void k_commit(DevCtl* ctl, int bucket, const int32_t* mv_v, const int32_t* mv_new, int32_t* mv_old,
+                         int32_t* C, uint32_t* a, int32_t* size, const uint32_t* k) {
+  const unsigned long long start = ctl->bounds[bucket];
+  const unsigned long long end = *(volatile unsigned long long*)&ctl->logn;
+  if (blockIdx.x == 0 && threadIdx.x == 0) ctl->bounds[bucket + 1] = end;
+  for (unsigned long long p = start + blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; p < end;
+       p += (unsigned long long)gridDim.x * blockDim.x) {
+    const int32_t i = mv_v[p], t = mv_new[p];
+    const int32_t old = C[i];
+    mv_old[p] = old;
+    C[i] = t;
+    const uint32_t ki = k[i];
+    atomicSub(&a[old], ki);
+    atomicAdd(&a[t], ki);
+    atomicSub(&size[old], 1);
+    atomicAdd(&size[t], 1);
+  }
+}
+
+// Undo every move of the sweep (R15).
+__global__ void k_revert(const DevCtl* ctl, const int32_t* mv_v, const int32_t* mv_new, const int32_t* mv_old,
+                         int32_t* C, uint32_t* a, int32_t* size, const uint32_t* k) {
+  const unsigned long long end = ctl->logn;
+  for (unsigned long long p = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; p < end;
+       p += (unsigned long long)gridDim.x * blockDim.x) {
+    const int32_t i = mv_v[p], t = mv_new[p], old = mv_old[p];
+    C[i] = old;
+    const uint32_t ki = k[i];
+    atomicSub(&a[t], ki);
+    atomicAdd(&a[old], ki);
+    atomicSub(&size[t], 1);
+    atomicAdd(&size[old], 1);
+  }
+}
+
+// Edge-centric tile walker: calls f(u, e) for every CSR entry e of the tile
+// [e0, e1) with its source row u.  The tile's rowptr window is staged in smem
+// and each thread binary-searches it (coalesced col/w loads; degree-skew free).
+template <class F>
+__device__ __forceinline__ void for_tile_edges(const int64_t* rowptr, int64_t n, int64_t e0, int64_t e1,
+                                               int64_t* sh_rows, int64_t* sh_u0, int* sh_nr, F f) {
+  if (threadIdx.x == 0) {
+    const int64_t u0 = row_of(rowptr, n, e0);
+    const int64_t u1 = row_of(rowptr, n, e1 - 1);
+    *sh_u0 = u0;
+    *sh_nr = (u1 - u0 + 2 <= kTileRows) ? (int)(u1 - u0 + 2) : -1;
+  }
+  __syncthreads();
+  const int64_t u0 = *sh_u0;
+  const int nr = *sh_nr;
+  for (int t = threadIdx.x; t < nr; t += blockDim.x) sh_rows[t] = rowptr[u0 + t];
+  __syncthreads();
+  for (int64_t e = e0 + threadIdx.x; e < e1; e += blockDim.x) {
+    int64_t u;
+    if (nr > 0) {
+      int lo = 0, hi = nr - 2;  // largest r with sh_rows[r] <= e
+      while (lo < hi) {
+        int mid = (lo + hi + 1) >> 1;
+        if (sh_rows[mid] <= e) lo = mid; else hi = mid - 1;
+      }
+      u = u0 + lo;
+    } else {
+      u = row_of(rowptr, n, e);
+    }
+    f(u, e);
+  }
+  __syncthreads();
+}
+
+// Eq. (1): L = sum of w over entries (u,v) with C[u] = C[v] (self-loops
+// included, R2); S = sum_c a_c^2.  Integer atomics: deterministic.
+__global__ void __launch_bounds__(256) k_modularity(const int64_t* rowptr, int64_t n, const int32_t* col,
+                                                    const uint32_t* w, const int32_t* C, const uint32_t* a,
+                                                    int64_t nnz, unsigned long long* Lout, unsigned long long* Sout) {
+  __shared__ int64_t sh_rows[kTileRows];
+  __shared__ int64_t sh_u0;
+  __shared__ int sh_nr;
+  unsigned long long acc = 0;
+  const int64_t ntiles = (nnz + kTileEdges - 1) / kTileEdges;
+  for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
+    const int64_t e0 = tile * kTileEdges, e1 = min(nnz, e0 + kTileEdges);
+    for_tile_edges(rowptr, n, e0, e1, sh_rows, &sh_u0, &sh_nr, [&](int64_t u, int64_t e) {
+      if (C[col[e]] == C[u]) acc += w ? w[e] : 1u;
+    });
+  }
+  unsigned long long s2 = 0;
+  for (int64_t c = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; c < n; c += (int64_t)gridDim.x * blockDim.x) {
+    const unsigned long long x = a[c];
+    s2 += x * x;
+  }
+  acc = warp_sum_u64(acc);
+  s2 = warp_sum_u64(s2);
+  if ((threadIdx.x & 31) == 0) {
+    if (acc) atomicAdd(Lout, acc);
+    if (s2) atomicAdd(Sout, s2);
+  }
+}
+
+// ---------------------------------------------------------------- contraction
+__global__ void k_flags_nonempty(const int32_t* size, int64_t n, int32_t* flag) {
+  for (int64_t c = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; c < n; c += (int64_t)gridDim.x * blockDim.x)
+    flag[c] = size[c] > 0 ? 1 : 0;
+}
+
+__global__ void k_map(const int32_t* C, const int32_t* newID, int64_t n, int32_t* map) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    map[i] = newID[C[i]];  // R17: new ids in label order
+}
+
+__global__ void __launch_bounds__(256) k_emit_keys(const int64_t* rowptr, int64_t n, const int32_t* col,
+                                                   const uint32_t* w, const int32_t* map, int64_t nnz, uint64_t np,
+                                                   unsigned long long* keys, uint32_t* vals) {
+  __shared__ int64_t sh_rows[kTileRows];
+  __shared__ int64_t sh_u0;
+  __shared__ int sh_nr;
+  const int64_t ntiles = (nnz + kTileEdges - 1) / kTileEdges;
+  for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
+    const int64_t e0 = tile * kTileEdges, e1 = min(nnz, e0 + kTileEdges);
+    for_tile_edges(rowptr, n, e0, e1, sh_rows, &sh_u0, &sh_nr, [&](int64_t u, int64_t e) {
+      keys[e] = (unsigned long long)map[u] * np + (unsigned long long)map[col[e]];  // (newID[C[u]], newID[C[v]])
+      if (vals) vals[e] = w[e];
+    });
+  }
+}
+
+__global__ void k_row_counts(const unsigned long long* keys, int64_t m, uint64_t np, int64_t* cnt) {
+  const unsigned lane = threadIdx.x & 31;
+  for (int64_t base = (int64_t)blockIdx.x * blockDim.x; base < m; base += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t e = base + threadIdx.x;
+    const bool valid = e < m;
+    const uint32_t r = valid ? (uint32_t)(keys[e] / np) : 0xFFFFFFFFu;
+    const unsigned mask = __match_any_sync(kFull, r);
+    if (valid && (__ffs(mask) - 1) == (int)lane) atomicAdd((unsigned long long*)&cnt[r + 1], (unsigned long long)__popc(mask));
+  }
+}
+
+__global__ void k_split_keys(const unsigned long long* keys, int64_t m, uint64_t np, int32_t* col) {
+  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < m; e += (int64_t)gridDim.x * blockDim.x)
+    col[e] = (int32_t)(keys[e] % np);
+}
+
+__global__ void k_compose(int32_t* lab, int64_t n0, const int32_t* map) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n0; i += (int64_t)gridDim.x * blockDim.x)
+    lab[i] = map[lab[i]];
+}
+
+__global__ void k_sum_u32(const uint32_t* x, int64_t n, unsigned long long* out) {
+  unsigned long long acc = 0;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) acc += x[i];
+  acc = warp_sum_u64(acc);
+  if ((threadIdx.x & 31) == 0 && acc) atomicAdd(out, acc);
+}
+
+}  // namespace
+
+// ======================================================================== host side
+int32_t level_alloc_state(Level& L, cudaStream_t s) {
+  LV_TRY(dalloc(&L.k, L.n, s));
+  LV_TRY(dalloc(&L.C, L.n, s));
+  LV_TRY(dalloc(&L.a, L.n, s));
+  LV_TRY(dalloc(&L.size, L.n, s));
+  LV_TRY(dalloc(&L.mv_v, L.n, s));
+  LV_TRY(dalloc(&L.mv_new, L.n, s));
+  LV_TRY(dalloc(&L.mv_old, L.n, s));
+  LV_TRY(dalloc(&L.bin_vertices, L.n, s));
+  return LOUVAIN_OK;
+}
+
+static void hub_free(HubPlan& P, cudaStream_t s) {
+  dfree(P.hub_v, s); dfree(P.tab_off, s); dfree(P.tab_cap, s); dfree(P.chunk, s); dfree(P.scan, s);
+  dfree(P.scan_first, s); dfree(P.table, s); dfree(P.partial, s);
+  P = HubPlan();
+}
+
+void level_free(Level& L, cudaStream_t s) {
+  if (L.owns_csr) {
+    dfree(L.rowptr, s);
+    dfree(L.col, s);
+    dfree(L.w, s);
+  }
+  dfree(L.k, s); dfree(L.C, s); dfree(L.a, s); dfree(L.size, s);
+  dfree(L.mv_v, s); dfree(L.mv_new, s); dfree(L.mv_old, s); dfree(L.bin_vertices, s);
+  hub_free(L.hub, s);
+  L = Level();
+}
+
+int32_t level_setup(Handle& h, Level& L) {
+  cudaStream_t s = h.stream;
+  const int64_t n = L.n;
+  if (n == 0) { L.W = 0; return LOUVAIN_OK; }
+  if (L.w) {
+    // k_i = weighted row sum
+    size_t tb = 0;
+    LV_CUDA(cub::DeviceSegmentedReduce::Sum(nullptr, tb, L.w, L.k, (int)n, L.rowptr, L.rowptr + 1, s));
+    void* tmp = nullptr;
+    LV_TRY(dmalloc(&tmp, tb, s));
+    LV_CUDA(cub::DeviceSegmentedReduce::Sum(tmp, tb, L.w, L.k, (int)n, L.rowptr, L.rowptr + 1, s));
+    dfree(tmp, s);
+  } else {
+    k_degrees_unit<<<grid_for(n, 256), 256, 0, s>>>(L.rowptr, n, L.k);
+  }
+  // W = sum_i k_i = 2m (R1)
+  unsigned long long* dW = &h.ctl->L;  // reuse a ctl word as scratch
+  LV_CUDA(cudaMemsetAsync(dW, 0, 8, s));
+  k_sum_u32<<<grid_for(n, 256, 148 * 8), 256, 0, s>>>(L.k, n, dW);
+  unsigned long long W = 0;
+  LV_CUDA(cudaMemcpyAsync(&W, dW, 8, cudaMemcpyDeviceToHost, s));
+  LV_CUDA(cudaStreamSynchronize(s));
+  L.W = W;
+  if (W > kWGuard) {
+    set_error("W = 2m exceeds 3,037,000,499 (int64 gain guard, R4)");
+    return LOUVAIN_E_OVERFLOW;
+  }
+  k_init_singletons<<<grid_for(n, 256), 256, 0, s>>>(L.k, n, L.C, L.a, L.size);
+  LV_CUDA(cudaGetLastError());
+  return LOUVAIN_OK;
+}
+
+int32_t level_set_labels(Handle& h, Level& L, const int32_t* d_labels) {
+  cudaStream_t s = h.stream;
+  if (L.n == 0) return LOUVAIN_OK;
+  if (d_labels != L.C) LV_CUDA(cudaMemcpyAsync(L.C, d_labels, sizeof(int32_t) * L.n, cudaMemcpyDefault, s));
+  k_totals_zero<<<grid_for(L.n, 256), 256, 0, s>>>(L.n, L.a, L.size);
+  LV_CUDA(cudaMemsetAsync(&h.ctl->bad, 0, 8, s));
+  k_totals_add<<<grid_for(L.n, 256), 256, 0, s>>>(L.C, L.k, L.n, L.a, L.size, &h.ctl->bad);
+  unsigned long long bad = 0;
+  LV_CUDA(cudaMemcpyAsync(&bad, &h.ctl->bad, 8, cudaMemcpyDeviceToHost, s));
+  LV_CUDA(cudaStreamSynchronize(s));
+  if (bad) {
+    set_error("labels out of range [0, n)");
+    return LOUVAIN_E_INVALID_ARG;
+  }
+  return LOUVAIN_OK;
+}
+
+int32_t level_binning(Handle& h, Level& L, const louvain_params_t& p) {
+  bool same = L.bins_valid;
+  for (int t = 0; t < 6 && same; ++t) same = (L.bins_bounds[t] == p.deg_bounds[t]);
+  if (same) return LOUVAIN_OK;
+  cudaStream_t s = h.stream;
+  const int64_t n = L.n;
+  hub_free(L.hub, s);
+  std::fill(L.class_off, L.class_off + kNumClasses + 1, 0);
+  if (n > 0) {
+    uint8_t *cls = nullptr, *cls2 = nullptr;
+    int32_t* iota = nullptr;
+    unsigned long long* hist = nullptr;
+    LV_TRY(dalloc(&cls, n, s));
+    LV_TRY(dalloc(&cls2, n, s));
+    LV_TRY(dalloc(&iota, n, s));
+    LV_TRY(dalloc(&hist, kNumClasses, s));
+    LV_CUDA(cudaMemsetAsync(hist, 0, 8 * kNumClasses, s));
+    k_classify<<<grid_for(n, 256), 256, 0, s>>>(L.rowptr, n, p.deg_bounds[0], p.deg_bounds[1], p.deg_bounds[2],
+                                                p.deg_bounds[3], p.deg_bounds[4], p.deg_bounds[5], cls, iota, hist);
+    LV_CUDA(cudaGetLastError());
+    // stable sort by class (5 bits): vertices of a class stay in ascending id order
+    size_t tb = 0;
+    LV_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, tb, cls, cls2, iota, L.bin_vertices, n, 0, 5, s));
+    void* tmp = nullptr;
+    LV_TRY(dmalloc(&tmp, tb, s));
+    LV_CUDA(cub::DeviceRadixSort::SortPairs(tmp, tb, cls, cls2, iota, L.bin_vertices, n, 0, 5, s));
+    dfree(tmp, s);
+    unsigned long long hh[kNumClasses];
+    LV_CUDA(cudaMemcpyAsync(hh, hist, sizeof hh, cudaMemcpyDeviceToHost, s));
+    LV_CUDA(cudaStreamSynchronize(s));
+    dfree(cls, s); dfree(cls2, s); dfree(iota, s); dfree(hist, s);
+    for (int c = 0; c < kNumClasses; ++c) L.class_off[c + 1] = L.class_off[c] + (int64_t)hh[c];
+  }
+  // hub plan: vertices of sub-class 2 (deg >= kHubMin) of every bucket
+  HubPlan& P = L.hub;
+  std::vector<int32_t> hv;
+  std::vector<int64_t> hdeg, rb;
+  for (int b = 1; b <= 7; ++b) {
+    const int c = 4 * b + 2;
+    const int64_t off = L.class_off[c], cnt = L.class_off[c + 1] - off;
+    if (cnt <= 0) continue;
+    std::vector<int32_t> v(cnt);
+    std::vector<int64_t> d(2 * cnt);
+    int64_t* dd = nullptr;
+    LV_TRY(dalloc(&dd, 2 * cnt, s));
+    k_hub_degrees<<<grid_for(cnt, 256), 256, 0, s>>>(L.bin_vertices + off, cnt, L.rowptr, dd);
+    LV_CUDA(cudaMemcpyAsync(v.data(), L.bin_vertices + off, 4 * cnt, cudaMemcpyDeviceToHost, s));
+    LV_CUDA(cudaMemcpyAsync(d.data(), dd, 16 * cnt, cudaMemcpyDeviceToHost, s));
+    LV_CUDA(cudaStreamSynchronize(s));
+    dfree(dd, s);
+    hv.insert(hv.end(), v.begin(), v.end());
+    hdeg.insert(hdeg.end(), d.begin(), d.begin() + cnt);
+    rb.insert(rb.end(), d.begin() + cnt, d.end());
+  }
+  P.nh = (int64_t)hv.size();
+  if (P.nh > 0) {
+    std::vector<int64_t> off(P.nh), cap(P.nh), chunk, scan, first(P.nh + 1);
+    int64_t tot = 0;
+    for (int64_t i = 0; i < P.nh; ++i) {
+      off[i] = tot;
+      cap[i] = 2 * hdeg[i];  // load factor <= 1/2
+      tot += cap[i];
+      for (int64_t e = 0; e < hdeg[i]; e += kHubChunkEdges) {
+        chunk.push_back(i);
+        chunk.push_back(rb[i] + e);
+        chunk.push_back(rb[i] + std::min(hdeg[i], e + kHubChunkEdges));
+      }
+      first[i] = (int64_t)scan.size() / 3;
+      for (int64_t t = 0; t < cap[i]; t += kHubScanSlots) {
+        scan.push_back(i);
+        scan.push_back(t);
+        scan.push_back(std::min(cap[i], t + kHubScanSlots));
+      }
+    }
+    first[P.nh] = (int64_t)scan.size() / 3;
+    P.nchunks = (int64_t)chunk.size() / 3;
+    P.nscan = (int64_t)scan.size() / 3;
+    P.table_slots = tot;
+    LV_TRY(dalloc(&P.hub_v, P.nh, s));
+    LV_TRY(dalloc(&P.tab_off, P.nh, s));
+    LV_TRY(dalloc(&P.tab_cap, P.nh, s));
+    LV_TRY(dalloc(&P.chunk, chunk.size(), s));
+    LV_TRY(dalloc(&P.scan, scan.size(), s));
+    LV_TRY(dalloc(&P.scan_first, P.nh + 1, s));
+    LV_TRY(dalloc(&P.table, tot, s));
+    LV_TRY(dmalloc(&P.partial, hub_partial_bytes() * (size_t)P.nscan, s));
+    LV_CUDA(cudaMemcpyAsync(P.hub_v, hv.data(), 4 * P.nh, cudaMemcpyHostToDevice, s));
+    LV_CUDA(cudaMemcpyAsync(P.tab_off, off.data(), 8 * P.nh, cudaMemcpyHostToDevice, s));
+    LV_CUDA(cudaMemcpyAsync(P.tab_cap, cap.data(), 8 * P.nh, cudaMemcpyHostToDevice, s));
+    LV_CUDA(cudaMemcpyAsync(P.chunk, chunk.data(), 8 * chunk.size(), cudaMemcpyHostToDevice, s));
+    LV_CUDA(cudaMemcpyAsync(P.scan, scan.data(), 8 * scan.size(), cudaMemcpyHostToDevice, s));
+    LV_CUDA(cudaMemcpyAsync(P.scan_first, first.data(), 8 * (P.nh + 1), cudaMemcpyHostToDevice, s));
+    k_fill_u64<<<grid_for(tot, 256), 256, 0, s>>>(P.table, tot, kEmpty);
+    LV_CUDA(cudaGetLastError());
+    LV_CUDA(cudaStreamSynchronize(s));  // host vectors die here
+  }
+  std::memcpy(L.bins_bounds, p.deg_bounds, sizeof L.bins_bounds);
+  L.bins_valid = true;
+  return LOUVAIN_OK;
+}
+
+
+// Eq. (1) parts of partition d_C into ctl->L / ctl->S (stream-ordered, no sync).
+// d_C == L.C uses the maintained a_c; any other labels get their own a_c.
+int32_t launch_modularity(Handle& h, Level& L, const int32_t* d_C) {
+  cudaStream_t s = h.stream;
+  LV_CUDA(cudaMemsetAsync(&h.ctl->L, 0, 16, s));
+  if (L.n == 0) return LOUVAIN_OK;
+  const uint32_t* a = L.a;
+  uint32_t* a_tmp = nullptr;
+  int32_t* size_tmp = nullptr;
+  if (d_C != L.C) {
+    LV_TRY(dalloc(&a_tmp, L.n, s));
+    LV_TRY(dalloc(&size_tmp, L.n, s));
+    k_totals_zero<<<grid_for(L.n, 256), 256, 0, s>>>(L.n, a_tmp, size_tmp);
+    k_totals_add<<<grid_for(L.n, 256), 256, 0, s>>>(d_C, L.k, L.n, a_tmp, size_tmp, &h.ctl->bad);
+    a = a_tmp;
+  }
+  const int64_t ntiles = (L.nnz + kTileEdges - 1) / kTileEdges;
+  const unsigned grid = grid_for(std::max<int64_t>(ntiles, (L.n + 255) / 256), 1, 148 * 8);
+  k_modularity<<<grid, 256, 0, s>>>(L.rowptr, L.n, L.col, L.w, d_C, a, L.nnz, &h.ctl->L, &h.ctl->S);
+  LV_CUDA(cudaGetLastError());
+  if (a_tmp) { dfree(a_tmp, s); dfree(size_tmp, s); }
+  return LOUVAIN_OK;
+}
+
+int32_t level_modularity(Handle& h, Level& L, const int32_t* d_C, uint64_t* Lout, uint64_t* Sout) {
+  LV_CUDA(cudaMemsetAsync(&h.ctl->bad, 0, 8, h.stream));
+  LV_TRY(launch_modularity(h, L, d_C));
+  LV_CUDA(cudaMemcpyAsync(h.h_ctl, h.ctl, sizeof(DevCtl), cudaMemcpyDeviceToHost, h.stream));
+  LV_CUDA(cudaStreamSynchronize(h.stream));
+  if (h.h_ctl->bad) {
+    set_error("labels out of range [0, n)");
+    return LOUVAIN_E_INVALID_ARG;
+  }
+  *Lout = h.h_ctl->L;
+  *Sout = h.h_ctl->S;
+  return LOUVAIN_OK;
+}
+
+int32_t launch_commit(Handle& h, Level& L, int bucket) {
+  k_commit<<<148 * 4, 256, 0, h.stream>>>(h.ctl, bucket, L.mv_v, L.mv_new, L.mv_old, L.C, L.a, L.size, L.k);
+  LV_CUDA(cudaGetLastError());
+  return LOUVAIN_OK;
+}
+
+int32_t launch_revert(Handle& h, Level& L) {
+  k_revert<<<148 * 4, 256, 0, h.stream>>>(h.ctl, L.mv_v, L.mv_new, L.mv_old, L.C, L.a, L.size, L.k);
+  LV_CUDA(cudaGetLastError());
+  return LOUVAIN_OK;
+}
+
+int32_t compose_labels(Handle& h, int32_t* lab, int64_t n0, const int32_t* map) {
+  if (n0 == 0) return LOUVAIN_OK;
+  k_compose<<<grid_for(n0, 256), 256, 0, h.stream>>>(lab, n0, map);
+  LV_CUDA(cudaGetLastError());
+  return LOUVAIN_OK;
+}
+
+// Alg. 3 as renumber-by-scan + sort-by-key + segmented reduce:
+//  newID = exclusive scan of [size_c > 0] (Alg. 3 l.7-12, R17);
+//  every entry (u,v,w) emits key (newID[C[u]], newID[C[v]]) (R18: mergeCommunity
+//  hashes all neighbours of all members); radix sort; equal keys summed
+//  (run-length counts at unit weight); CSR' rows sorted by column.
+int32_t level_contract(Handle& h, Level& L, Level& out, int32_t* d_map) {
+  cudaStream_t s = h.stream;
+  const int64_t n = L.n, nnz = L.nnz;
+  out = Level();
+  out.W = L.W;
+  if (n == 0) {
+    LV_TRY(dalloc(&out.rowptr, 1, s));
+    LV_CUDA(cudaMemsetAsync(out.rowptr, 0, 8, s));
+    return level_alloc_state(out, s);
+  }
+  int32_t *flag = nullptr, *newID = nullptr;
+  LV_TRY(dalloc(&flag, n, s));
+  LV_TRY(dalloc(&newID, n, s));
+  k_flags_nonempty<<<grid_for(n, 256), 256, 0, s>>>(L.size, n, flag);
+  size_t tb = 0;
+  LV_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, tb, flag, newID, n, s));
+  void* tmp = nullptr;
+  LV_TRY(dmalloc(&tmp, tb, s));
+  LV_CUDA(cub::DeviceScan::ExclusiveSum(tmp, tb, flag, newID, n, s));
+  dfree(tmp, s);
+  int32_t last[2];
+  LV_CUDA(cudaMemcpyAsync(&last[0], newID + n - 1, 4, cudaMemcpyDeviceToHost, s));
+  LV_CUDA(cudaMemcpyAsync(&last[1], flag + n - 1, 4, cudaMemcpyDeviceToHost, s));
+  LV_CUDA(cudaStreamSynchronize(s));
+  const int64_t np = (int64_t)last[0] + last[1];
+  k_map<<<grid_for(n, 256), 256, 0, s>>>(L.C, newID, n, d_map);
+  dfree(flag, s);
+  dfree(newID, s);
+  out.n = np;
+  LV_TRY(dalloc(&out.rowptr, np + 1, s));
+  LV_CUDA(cudaMemsetAsync(out.rowptr, 0, 8 * (np + 1), s));
+  if (nnz == 0) {
+    out.nnz = 0;
+    LV_TRY(dalloc(&out.col, 1, s));
+    LV_TRY(dalloc(&out.w, 1, s));
+    return level_alloc_state(out, s);
+  }
+  const bool weighted = L.w != nullptr;
+  unsigned long long *k0 = nullptr, *k1 = nullptr;
+  uint32_t *v0 = nullptr, *v1 = nullptr;
+  LV_TRY(dalloc(&k0, nnz, s));
+  LV_TRY(dalloc(&k1, nnz, s));
+  LV_TRY(dalloc(&v0, nnz, s));
+  if (weighted) LV_TRY(dalloc(&v1, nnz, s));
+  {
+    const int64_t ntiles = (nnz + kTileEdges - 1) / kTileEdges;
+    k_emit_keys<<<grid_for(ntiles, 1, 148 * 8), 256, 0, s>>>(L.rowptr, n, L.col, L.w, d_map, nnz, (uint64_t)np, k0,
+                                                             weighted ? v0 : nullptr);
+    LV_CUDA(cudaGetLastError());
+  }
+  int bits = 1;
+  while (bits < 64 && ((unsigned long long)1 << bits) < (unsigned long long)np * (unsigned long long)np) ++bits;
+  cub::DoubleBuffer<unsigned long long> kb(k0, k1);
+  cub::DoubleBuffer<uint32_t> vb(v0, v1);
+  tb = 0;
+  if (weighted) LV_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, tb, kb, vb, nnz, 0, bits, s));
+  else LV_CUDA(cub::DeviceRadixSort::SortKeys(nullptr, tb, kb, nnz, 0, bits, s));
+  LV_TRY(dmalloc(&tmp, tb, s));
+  if (weighted) LV_CUDA(cub::DeviceRadixSort::SortPairs(tmp, tb, kb, vb, nnz, 0, bits, s));
+  else LV_CUDA(cub::DeviceRadixSort::SortKeys(tmp, tb, kb, nnz, 0, bits, s));
+  dfree(tmp, s);
+  unsigned long long* sorted = kb.Current();
+  unsigned long long* uniq = kb.Alternate();
+  uint32_t* sums = weighted ? vb.Alternate() : v0;
+  int64_t* d_num = reinterpret_cast<int64_t*>(&h.ctl->bad);
+  tb = 0;
+  if (weighted) {
+    LV_CUDA(cub::DeviceReduce::ReduceByKey(nullptr, tb, sorted, uniq, vb.Current(), sums, d_num, cub::Sum(), nnz, s));
+    LV_TRY(dmalloc(&tmp, tb, s));
+    LV_CUDA(cub::DeviceReduce::ReduceByKey(tmp, tb, sorted, uniq, vb.Current(), sums, d_num, cub::Sum(), nnz, s));
+  } else {
+    LV_CUDA(cub::DeviceRunLengthEncode::Encode(nullptr, tb, sorted, uniq, sums, d_num, nnz, s));
+    LV_TRY(dmalloc(&tmp, tb, s));
+    LV_CUDA(cub::DeviceRunLengthEncode::Encode(tmp, tb, sorted, uniq, sums, d_num, nnz, s));
+  }
+  dfree(tmp, s);
+  int64_t m = 0;
+  LV_CUDA(cudaMemcpyAsync(&m, d_num, 8, cudaMemcpyDeviceToHost, s));
+  LV_CUDA(cudaStreamSynchronize(s));
+  dfree(sorted, s);
+  out.nnz = m;
+  LV_TRY(dalloc(&out.col, m, s));
+  LV_TRY(dalloc(&out.w, m, s));
+  int64_t* cnt = nullptr;
+  LV_TRY(dalloc(&cnt, np + 1, s));
+  LV_CUDA(cudaMemsetAsync(cnt, 0, 8 * (np + 1), s));
+  k_row_counts<<<grid_for(m, 256), 256, 0, s>>>(uniq, m, (uint64_t)np, cnt);
+  tb = 0;
+  LV_CUDA(cub::DeviceScan::InclusiveSum(nullptr, tb, cnt, out.rowptr, np + 1, s));
+  LV_TRY(dmalloc(&tmp, tb, s));
+  LV_CUDA(cub::DeviceScan::InclusiveSum(tmp, tb, cnt, out.rowptr, np + 1, s));
+  dfree(tmp, s);
+  dfree(cnt, s);
+  k_split_keys<<<grid_for(m, 256), 256, 0, s>>>(uniq, m, (uint64_t)np, out.col);
+  LV_CUDA(cudaMemcpyAsync(out.w, sums, 4 * m, cudaMemcpyDeviceToDevice, s));
+  LV_CUDA(cudaGetLastError());
+  dfree(uniq, s);
+  dfree(v0, s);
+  if (v1) dfree(v1, s);
+  return level_alloc_state(out, s);
+}
+
+// Host-side CSR validation (LOUVAIN_VALIDATE): rowptr monotone with rowptr[0]=0
+// and rowptr[n]=nnz, 0 <= col < n, w > 0, W guard, and symmetry (the multiset
+// of (u,v,w) equals that of (v,u,w); R1).
+int32_t validate_csr_host(int64_t n, int64_t nnz, const int64_t* rowptr, const int32_t* col, const uint32_t* w,
+                          bool full, uint64_t* Wout) {
+  if (rowptr[0] != 0 || rowptr[n] != nnz) {
+    set_error("rowptr[0] must be 0 and rowptr[n] must equal nnz");
+    return LOUVAIN_E_INVALID_GRAPH;
+  }
+  if (!full) return LOUVAIN_OK;
+  uint64_t W = 0;
+  for (int64_t i = 0; i < n; ++i) {
+    if (rowptr[i + 1] < rowptr[i]) { set_error("rowptr not monotone"); return LOUVAIN_E_INVALID_GRAPH; }
+    for (int64_t e = rowptr[i]; e < rowptr[i + 1]; ++e) {
+      if (col[e] < 0 || col[e] >= n) { set_error("col out of range"); return LOUVAIN_E_INVALID_GRAPH; }
+      uint32_t we = w ? w[e] : 1u;
+      if (we == 0) { set_error("zero weight"); return LOUVAIN_E_INVALID_GRAPH; }
+      W += we;
+    }
+  }
+  if (W > kWGuard) { set_error("W = 2m exceeds 3,037,000,499"); return LOUVAIN_E_OVERFLOW; }
+  struct T { int32_t u, v; uint32_t w; };
+  std::vector<T> f, b;
+  f.reserve(nnz);
+  b.reserve(nnz);
+  for (int64_t i = 0; i < n; ++i)
+    for (int64_t e = rowptr[i]; e < rowptr[i + 1]; ++e) {
+      uint32_t we = w ? w[e] : 1u;
+      f.push_back(T{(int32_t)i, col[e], we});
+      b.push_back(T{col[e], (int32_t)i, we});
+    }
+  auto lt = [](const T& x, const T& y) {
+    if (x.u != y.u) return x.u < y.u;
+    if (x.v != y.v) return x.v < y.v;
+    return x.w < y.w;
+  };
+  std::sort(f.begin(), f.end(), lt);
+  std::sort(b.begin(), b.end(), lt);
+  for (size_t t = 0; t < f.size(); ++t)
+    if (f[t].u != b[t].u || f[t].v != b[t].v || f[t].w != b[t].w) {
+      set_error("graph is not symmetric (each non-loop edge must be stored in both directions)");
+      return LOUVAIN_E_INVALID_GRAPH;
+    }
+  if (Wout) *Wout = W;
+  return LOUVAIN_OK;
+}
+
+}  // namespace lv

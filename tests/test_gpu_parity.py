@@ -1,0 +1,240 @@
+"""GPU parity: the CUDA path (through the C-ABI) against the plain-C oracle.
+
+Bar (BASELINE.json north star): labels after every sweep bit-exact against
+oracle (b) (bucket-synchronous, Alg. 1-2), modularity numerators
+L and S identical integers (Q equal to 1e-9 relative is then implied), the
+contraction's canonical CSR identical, and whole runs identical in labels,
+levels and per-level sweep counts.  All integer work: exact equality.
+"""
+import numpy as np
+import pytest
+
+import graphgen
+import oracle
+from conftest import cuda_ok
+
+pytestmark = [pytest.mark.gpu, pytest.mark.skipif(not cuda_ok(), reason="needs a CUDA device")]
+
+lvb = pytest.importorskip("paper_conf_ipps_naimmht17_b200")
+
+
+def dev_graph(g):
+    return lvb.Graph.from_csr(g.rowptr, g.col, g.w)
+
+
+def orc_params(**kw):
+    return oracle.params(**kw)
+
+
+def both_params(**kw):
+    return lvb.params(**kw), oracle.params(**kw)
+
+
+def hubs_graph(seed=0, hub_degrees=(600, 5000, 15000, 40000), n=60000, bg_tuples=120000):
+    """R-MAT-like background plus explicit hubs that exercise the CTA-small,
+    CTA-large and multi-CTA global-hash sweep paths."""
+    rng = np.random.default_rng(seed)
+    us, vs = [], []
+    for h, d in enumerate(hub_degrees):
+        nb = rng.choice(np.arange(len(hub_degrees), n), size=d, replace=False)
+        us.append(np.full(d, h))
+        vs.append(nb)
+    bu = rng.integers(0, n, size=bg_tuples)
+    bv = (bu + rng.integers(1, 50, size=bg_tuples)) % n  # local-ish background: communities form
+    us.append(bu)
+    vs.append(bv)
+    return graphgen.from_edges(n, np.concatenate(us), np.concatenate(vs))
+
+
+def weighted_with_loops(n, seed):
+    rng = np.random.default_rng(seed)
+    m = 6 * n
+    u = rng.integers(0, n, size=m)
+    v = (u + rng.integers(0, 40, size=m)) % n  # includes u == v (self-loops)
+    key = np.unique(np.minimum(u, v) * n + np.maximum(u, v))
+    uu, vv = key // n, key % n
+    w = rng.integers(1, 9, size=len(uu))
+    return graphgen.weighted_csr(n, uu, vv, w)
+
+
+GRAPHS = {
+    "karate": lambda: graphgen.karate(),
+    "rmat10": lambda: graphgen.rmat(10, seed=2),
+    "rmat15": lambda: graphgen.rmat(15, seed=3),
+    "mesh12_morton": lambda: graphgen.mesh3d(12, True),
+    "rgg20k": lambda: graphgen.rgg(20000, seed=4),
+    "lfr5k": lambda: graphgen.lfr(5000, kmin=8, kmax=300, smin=20, smax=600, seed=5),
+    "weighted_loops": lambda: weighted_with_loops(3000, 6),
+    "hubs": lambda: hubs_graph(),
+}
+
+
+def assert_state_equal(gd, st):
+    lab = gd.labels()
+    assert np.array_equal(lab, st.C), f"labels differ at {np.flatnonzero(lab != st.C)[:10]}"
+    a, size = gd.totals()
+    assert np.array_equal(a.astype(np.uint64), st.a) and np.array_equal(size.astype(np.int64), st.size)
+
+
+@pytest.mark.parametrize("name", list(GRAPHS))
+def test_modularity_matches_oracle(name):
+    g = GRAPHS[name]()
+    gd = dev_graph(g)
+    rng = np.random.default_rng(1)
+    for C in (np.arange(g.n), np.zeros(g.n), rng.integers(0, max(1, g.n // 7), size=g.n)):
+        C = C.astype(np.int32)
+        q = gd.modularity(C)
+        L, S, W = oracle.modularity(g, C)
+        assert (int(q.L), q.S, int(q.W)) == (L, S, W)
+        ref = (L * W - S) / W / W
+        assert abs(q.q - ref) <= 1e-9 * max(1.0, abs(ref))
+
+
+@pytest.mark.parametrize("name", list(GRAPHS))
+@pytest.mark.parametrize("mode,rule", [(0, 1), (0, 0), (0, 2), (1, 1)])
+def test_sweeps_bit_exact_from_singletons(name, mode, rule):
+    g = GRAPHS[name]()
+    gd = dev_graph(g)
+    st = oracle.State(g)
+    pd, po = both_params(mode=mode, singleton_rule=rule)
+    for sweep in range(4):
+        moved_o = st.sweep(po)
+        moved_d, q = gd.sweep(pd)
+        assert moved_d == moved_o, f"sweep {sweep}"
+        assert_state_equal(gd, st)
+        L, S, W = st.qnum()
+        assert (int(q.L), q.S) == (L, S)
+        if moved_o == 0:
+            break
+
+
+@pytest.mark.parametrize("name", ["rmat15", "weighted_loops", "hubs", "lfr5k"])
+def test_sweep_bit_exact_from_mid_run_labels(name):
+    g = GRAPHS[name]()
+    rng = np.random.default_rng(11)
+    # a partition reached by the oracle after two sweeps, then perturbed
+    st = oracle.State(g)
+    st.sweep(oracle.params())
+    st.sweep(oracle.params())
+    C = st.C.copy()
+    flip = rng.random(g.n) < 0.05
+    C[flip] = rng.integers(0, g.n, size=int(flip.sum()))
+    st = oracle.State(g, C)
+    gd = dev_graph(g)
+    gd.set_labels(C)
+    assert_state_equal(gd, st)
+    pd, po = both_params()
+    for _ in range(2):
+        assert gd.sweep(pd)[0] == st.sweep(po)
+        assert_state_equal(gd, st)
+
+
+@pytest.mark.parametrize("name", ["karate", "rmat15", "weighted_loops", "hubs", "mesh12_morton"])
+def test_aggregate_matches_oracle(name):
+    g = GRAPHS[name]()
+    st = oracle.State(g)
+    st.sweep(oracle.params())
+    st.sweep(oracle.params())
+    g2, mp = oracle.contract(g, st.C)
+    gd = dev_graph(g)
+    gd.set_labels(st.C)
+    nd, mpd = gd.aggregate()
+    assert np.array_equal(mpd, mp)
+    rowptr, col, w = nd.csr()
+    assert np.array_equal(rowptr, g2.rowptr)
+    assert np.array_equal(col, g2.col)
+    assert np.array_equal(w, g2.w)
+    assert nd.info()[2] == gd.info()[2]  # W preserved
+
+
+@pytest.mark.parametrize("name", list(GRAPHS))
+def test_full_run_bit_exact(name):
+    g = GRAPHS[name]()
+    r = oracle.louvain(g)
+    gd = dev_graph(g)
+    lab, q, stats = gd.run(lvb.params())
+    assert stats["levels"] == r.levels
+    assert stats["sweeps_per_level"] == r.sweeps_per_level
+    assert stats["n"] == r.n and stats["nnz"] == r.nnz
+    assert stats["num_start"] == r.num_start and stats["num_end"] == r.num_end
+    assert np.array_equal(lab, r.labels)
+    assert (int(q.L), q.S, int(q.W)) == (r.L, r.S, r.W)
+    assert abs(q.q - r.q) <= 1e-9 * max(1.0, abs(r.q))
+    assert np.array_equal(gd.labels(), r.labels)  # handle keeps the final partition
+
+
+def test_karate_quality_bar():
+    g = graphgen.karate()
+    lab, q, _ = dev_graph(g).run()
+    qa = oracle.louvain(g, oracle.params(mode=oracle.SEQ)).q
+    assert abs(q.q - qa) <= 0.005  # north-star bar vs sequential Louvain (a)
+    assert q.q <= 0.4197896 + 1e-7  # literature optimum (PAPER.md [2])
+
+
+def test_relaxed_full_run():
+    g = GRAPHS["rmat15"]()
+    r = oracle.louvain(g, oracle.params(mode=oracle.RELAXED))
+    lab, q, st = dev_graph(g).run(lvb.params(mode=1))
+    assert np.array_equal(lab, r.labels) and st["sweeps_per_level"] == r.sweeps_per_level
+
+
+def test_size_limit_schedule():
+    g = GRAPHS["rmat15"]()
+    r = oracle.louvain(g, oracle.params(size_limit=1000))
+    lab, q, st = dev_graph(g).run(lvb.params(size_limit=1000))
+    assert np.array_equal(lab, r.labels) and st["sweeps_per_level"] == r.sweeps_per_level
+
+
+def test_edge_cases():
+    # n = 0
+    gd = lvb.Graph.from_csr(np.zeros(1, np.int64), np.zeros(0, np.int32))
+    lab, q, st = gd.run()
+    assert st["levels"] == 0 and len(lab) == 0
+    # vertices but no edges (W = 0)
+    gd = lvb.Graph.from_csr(np.zeros(4, np.int64), np.zeros(0, np.int32))
+    lab, q, st = gd.run()
+    assert lab.tolist() == [0, 1, 2] and q.q == 0.0
+    # single edge
+    g = graphgen.from_edges(2, [0], [1])
+    lab, q, st = dev_graph(g).run()
+    assert lab.tolist() == oracle.louvain(g).labels.tolist()
+    # a vertex with only a self-loop plus a disconnected edge
+    g = graphgen.weighted_csr(3, [0, 1], [0, 2], [4, 1])
+    r = oracle.louvain(g)
+    lab, q, st = dev_graph(g).run()
+    assert lab.tolist() == r.labels.tolist() and (int(q.L), q.S) == (r.L, r.S)
+
+
+def test_device_inputs_and_borrow():
+    torch = pytest.importorskip("torch")
+    g = GRAPHS["rmat15"]()
+    r = oracle.louvain(g)
+    rp = torch.from_numpy(g.rowptr).cuda()
+    cl = torch.from_numpy(g.col).cuda()
+    for borrow in (False, True):
+        gd = lvb.Graph.from_csr(rp, cl, borrow=borrow)
+        out = torch.empty(g.n, dtype=torch.int32, device="cuda")
+        lab, q, st = gd.run(labels_out=out)
+        assert np.array_equal(out.cpu().numpy(), r.labels)
+
+
+def test_validate_on_device_inputs():
+    torch = pytest.importorskip("torch")
+    rp = torch.tensor([0, 1, 1], dtype=torch.int64, device="cuda")
+    cl = torch.tensor([1], dtype=torch.int32, device="cuda")
+    with pytest.raises(lvb.LouvainError) as e:
+        lvb.Graph.from_csr(rp, cl, validate=True)
+    assert e.value.code == lvb.E_INVALID_GRAPH
+
+
+@pytest.mark.parametrize("maker,args", [
+    (graphgen.rmat, dict(scale=16, seed=7)),
+    (graphgen.mesh3d, dict(L=20, morton=True)),
+    (graphgen.mesh3d, dict(L=9, morton=False)),
+    (graphgen.rgg, dict(n=50000, seed=3)),
+])
+def test_generators_host_device_bit_identical(maker, args):
+    h = maker(**args)
+    d = maker(device=True, **args).to_host()
+    assert h.n == d.n
+    assert np.array_equal(h.rowptr, d.rowptr) and np.array_equal(h.col, d.col)
