@@ -1,0 +1,340 @@
+#!/usr/bin/env python
+"""Benchmark of the B200 GPU Louvain hot path (BASELINE.json metric:
+"sweep edges/s + Louvain wall time at 1/2/4/8 B200; % HBM roofline; final Q").
+
+One step = one full multilevel ``louvain_run`` (every SURVEY 8(a) row: level
+setup, binning, sweeps, commits, modularity, contraction, level driver) over the
+C5 workload -- R-MAT scale 27, 8*2^27 undirected tuples (~2.0e9 directed CSR
+entries, the north star's ">= 1B edge power-law graph") -- with the graph
+already resident in HBM.  value = directed edges swept per second over the
+whole run (sum over executed sweeps of the level's nnz / run time).
+
+Also reported: the roofline of the dominant kernel sequence (the level-0
+sweep body), the oracle timed on the host (cpu_baseline), an end-to-end number
+through the C-ABI with host buffers (e2e), SM clocks during the timed region.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "sweep edges/s (multilevel Louvain run)"
+UNIT = "edges/s"
+
+
+def parse_args():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=3)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    ap.add_argument("--scale", type=int, default=27, help="R-MAT scale (27 = C5)")
+    ap.add_argument("--seed", type=int, default=1)
+    ap.add_argument("--e2e-steps", type=int, default=1)
+    ap.add_argument("--cpu-seconds", type=float, default=15.0, help="oracle sample budget")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    return ap.parse_args()
+
+
+# ----------------------------------------------------------------------------- clocks
+class ClockSampler:
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, device: int):
+        self.device = device
+        self.proc = None
+        self.path = None
+
+    def __enter__(self):
+        fd, self.path = tempfile.mkstemp(suffix=".csv")
+        os.close(fd)
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.device), f"--query-gpu={self.FIELDS}", "--format=csv,noheader",
+                 "-lms", "200"], stdout=open(self.path, "w"), stderr=subprocess.DEVNULL)
+        except FileNotFoundError:
+            self.proc = None
+        return self
+
+    def __exit__(self, *a):
+        if self.proc is not None:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except subprocess.TimeoutExpired:
+                self.proc.kill()
+
+    def summary(self) -> dict:
+        sm, mx, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        try:
+            for line in open(self.path):
+                parts = [p.strip() for p in line.split(",")]
+                if len(parts) < 9:
+                    continue
+                try:
+                    sm.append(float(parts[1].split()[0]))
+                    mx.append(float(parts[2].split()[0]))
+                except ValueError:
+                    continue
+                for nm, v in zip(names, parts[5:9]):
+                    if v.lower() == "active":
+                        reasons.add(nm)
+        finally:
+            os.unlink(self.path)
+        if not sm:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": [], "samples": 0}
+        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": max(mx), "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+# ----------------------------------------------------------------------------- helpers
+def measured_peak_hbm():
+    path = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        with open(path) as f:
+            return float(json.load(f)["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    except Exception:
+        return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+def recorded_traffic():
+    """DRAM bytes of the level-0 sweep body from the committed ncu capture (profiles/)."""
+    path = os.path.join(ROOT, "profiles", "sweep_traffic.json")
+    try:
+        with open(path) as f:
+            d = json.load(f)
+        return d.get("dram_bytes_per_sweep"), d.get("source")
+    except Exception:
+        return None, None
+
+
+def sweep_bytes(n_act: int, nnz: int, D: int, moved: int, weighted: bool = False) -> int:
+    """SURVEY 8(d) algorithmic bytes of one sweep."""
+    return 36 * n_act + nnz * (4 + (4 if weighted else 0) + 4) + 4 * D + 44 * moved
+
+
+def oracle_rate(hg, seconds: float, seed: int = 0):
+    """The C oracle's computeMove (Alg. 2) over a bounded vertex sample of the
+    level-0 singleton state: returns (edges/s, edges, seconds, vertices)."""
+    import numpy as np
+    import oracle
+    n = hg.n
+    deg = np.diff(hg.rowptr)
+    C = np.arange(n, dtype=np.int32)
+    a = deg.astype(np.uint64)
+    size = np.ones(n, dtype=np.int64)
+    W = int(deg.sum())
+    rng = np.random.default_rng(seed)
+
+    def sample(edges):
+        frac = min(1.0, edges / max(1, hg.nnz))
+        verts = np.flatnonzero(rng.random(n) < frac).astype(np.int64)
+        return verts
+
+    # calibrate on ~2M edges, then size the sample to the budget
+    v0 = sample(2_000_000)
+    t = time.perf_counter()
+    oracle.decide_batch(hg, C, a, size, W, v0)
+    dt = max(time.perf_counter() - t, 1e-3)
+    rate0 = float(deg[v0].sum()) / dt
+    verts = sample(rate0 * seconds)
+    t = time.perf_counter()
+    oracle.decide_batch(hg, C, a, size, W, verts)
+    dt = time.perf_counter() - t
+    e = int(deg[verts].sum())
+    return e / dt, e, dt, len(verts)
+
+
+def emit(d: dict):
+    print(json.dumps(d), flush=True)
+
+
+# ----------------------------------------------------------------------------- arms
+def run_reference(args, rank, world):
+    """--impl reference: the oracle (plain single-threaded C) on the host cores,
+    each step a bounded sample of the same workload, same metric/unit."""
+    if rank != 0:
+        return
+    import graphgen
+    t0 = time.perf_counter()
+    hg = graphgen.rmat(args.scale, seed=args.seed, device=True).to_host()
+    gen_s = time.perf_counter() - t0
+    per_step = max(2.0, min(args.cpu_seconds, 150.0 / max(1, args.steps + args.warmup)))
+    for _ in range(args.warmup):
+        oracle_rate(hg, per_step / 4)
+    rates, edges, secs = [], 0, 0.0
+    for k in range(args.steps):
+        r, e, dt, nv = oracle_rate(hg, per_step, seed=k + 1)
+        rates.append(r)
+        edges += e
+        secs += dt
+    value = edges / secs
+    sample = (f"oracle computeMove (Alg. 2) on {args.steps} random vertex samples of the level-0 singleton "
+              f"state of R-MAT s{args.scale}, {edges} directed edges total")
+    emit({"metric": METRIC, "value": value, "unit": UNIT, "impl": "reference", "n_gpus": world,
+          "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * secs / args.steps,
+          "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int64",
+          "data": "synthetic",
+          "config": {"workload": f"C5 R-MAT scale {args.scale}, {8 << args.scale} tuples, seed {args.seed}",
+                     "n": hg.n, "nnz": hg.nnz, "parallelism": "1 host core"},
+          "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
+          "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+          "gen_s": gen_s})
+
+
+def run_ours(args, rank, world):
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+
+    import graphgen
+    import paper_conf_ipps_naimmht17_b200 as lvb
+
+    dev = torch.device("cuda", torch.cuda.current_device())
+    t0 = time.perf_counter()
+    dg = graphgen.rmat(args.scale, seed=args.seed, device=True)
+    torch.cuda.synchronize()
+    gen_s = time.perf_counter() - t0
+    n, nnz = dg.n, dg.nnz
+    deg = dg.rowptr[1:] - dg.rowptr[:-1]
+    n_act = int((deg > 0).sum().item())
+    stream = torch.cuda.Stream()
+    g = lvb.Graph.from_csr(dg.rowptr, dg.col, borrow=True, stream=stream)
+    p = lvb.params()
+    labels_dev = torch.empty(n, dtype=torch.int32, device=dev)
+
+    def one_run():
+        return g.run(p, labels_out=labels_dev)
+
+    for _ in range(args.warmup):
+        one_run()
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    stats = []
+    with ClockSampler(dev.index) as clk:
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        ev0.record(stream)
+        for _ in range(args.steps):
+            _, q, st = one_run()
+            stats.append(st)
+        ev1.record(stream)
+        torch.cuda.synchronize()
+    clocks = clk.summary()
+    ms = ev0.elapsed_time(ev1)
+    if world > 1:
+        t = torch.tensor([ms], device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t.item())
+    ms_per_step = ms / args.steps
+    st0 = stats[0]
+    edges_per_run = st0["edges_swept"]
+    value = world * edges_per_run / (ms_per_step / 1e3)  # replicas: every rank sweeps its own copy
+
+    # roofline of the dominant kernel sequence: the level-0 sweep body (sweep 1)
+    t_sw1 = statistics.mean(s["t_sweep_ms_first"] for s in stats)
+    moved1 = st0["moved_first"]
+    B = sweep_bytes(n_act, nnz, D=nnz, moved=moved1)
+    achieved = B / (t_sw1 / 1e3) / 1e9
+    peak, peak_src = measured_peak_hbm()
+    traffic, traffic_src = recorded_traffic()
+    roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
+                "traffic": traffic, "kernel": "level-0 sweep 1 body (7 bucket kernels + commits)",
+                "algorithmic_bytes": B, "t_ms": t_sw1, "peak_source": peak_src,
+                "traffic_source": traffic_src}
+
+    out = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+           "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
+           "scaling": "weak", "vs_baseline": None, "dtype": "int64", "data": "synthetic",
+           "config": {"workload": f"C5 R-MAT scale {args.scale}, {8 << args.scale} tuples, seed {args.seed}, "
+                                  "unit weights, isolated vertices removed",
+                      "n": n, "nnz": nnz, "n_active": n_act,
+                      "l2": "inputs larger than L2 (col array alone is 4*nnz bytes >> 126 MB)",
+                      "parallelism": "1 GPU" if world == 1 else f"{world} independent replicas"},
+           "roofline": roofline, "clocks": clocks,
+           "gpu_launches": int(sum(s["kernel_launches"] for s in stats)),
+           "cub_calls": int(sum(s["cub_calls"] for s in stats)),
+           "louvain_wall_ms": ms_per_step, "q_final": st0["q"], "levels": st0["levels"],
+           "sweeps_per_level": st0["sweeps_per_level"], "n_per_level": st0["n"], "nnz_per_level": st0["nnz"],
+           "sweep1_ms": t_sw1, "sweep1_edges_per_s": nnz / (t_sw1 / 1e3),
+           "sweep_edges_per_s_all": edges_per_run / (st0["t_sweep_ms_total"] / 1e3),
+           "t_sweep_ms_total": st0["t_sweep_ms_total"], "t_modularity_ms_total": st0["t_modularity_ms_total"],
+           "t_opt_ms": sum(st0["t_opt_ms"]), "t_agg_ms": sum(st0["t_agg_ms"]), "gen_s": gen_s}
+
+    # end to end through the C-ABI with host buffers (H2D of the CSR and D2H of labels every step)
+    h_rowptr = torch.empty(n + 1, dtype=torch.int64, pin_memory=True)
+    h_col = torch.empty(nnz, dtype=torch.int32, pin_memory=True)
+    h_lab = torch.empty(n, dtype=torch.int32, pin_memory=True)
+    h_rowptr.copy_(dg.rowptr)
+    h_col.copy_(dg.col)
+    del g
+    torch.cuda.synchronize()
+    e2e_s = []
+    for _ in range(max(1, args.e2e_steps)):
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        t = time.perf_counter()
+        with lvb.Graph.from_csr(h_rowptr, h_col) as ge:
+            ge.run(p, labels_out=h_lab)
+        torch.cuda.synchronize()
+        e2e_s.append(time.perf_counter() - t)
+    t_e2e = statistics.median(e2e_s)
+    if world > 1:
+        t = torch.tensor([t_e2e], device=dev, dtype=torch.float64)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        t_e2e = float(t.item())
+    out["e2e"] = {"value": world * edges_per_run / t_e2e, "unit": UNIT,
+                  "h2d_bytes_per_step": 8 * (n + 1) + 4 * nnz, "d2h_bytes_per_step": 4 * n,
+                  "ms_per_step": 1e3 * t_e2e}
+
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        hg = graphgen.Graph(n, h_rowptr.numpy(), h_col.numpy())
+        r, e, dt, nv = oracle_rate(hg, args.cpu_seconds)
+        out["cpu_baseline"] = {"value": r, "unit": UNIT, "cores": 1, "kind": "oracle",
+                               "sample": f"oracle computeMove (Alg. 2) for {nv} random vertices ({e} directed "
+                                         f"edges, {dt:.1f} s) of the level-0 singleton state of the same graph"}
+    if rank == 0:
+        emit(out)
+
+
+def main():
+    args = parse_args()
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference":
+        run_reference(args, rank, world)
+        return
+    import torch
+    torch.cuda.set_device(local)
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    try:
+        run_ours(args, rank, world)
+    finally:
+        if world > 1:
+            import torch.distributed as dist
+            dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -55,7 +55,8 @@ class Stats(ctypes.Structure):
                 ("t_opt_ms", ctypes.c_double * MAX_LEVELS), ("t_agg_ms", ctypes.c_double * MAX_LEVELS),
                 ("t_total_ms", ctypes.c_double), ("t_sweep_ms_total", ctypes.c_double),
                 ("t_sweep_ms_first", ctypes.c_double), ("t_modularity_ms_total", ctypes.c_double),
-                ("edges_swept", ctypes.c_int64), ("q", QNum)]
+                ("edges_swept", ctypes.c_int64), ("moved_first", ctypes.c_int64),
+                ("kernel_launches", ctypes.c_int64), ("cub_calls", ctypes.c_int64), ("q", QNum)]
 
     def as_dict(self) -> dict:
         lv = self.levels
@@ -66,7 +67,8 @@ class Stats(ctypes.Structure):
                 "t_opt_ms": list(self.t_opt_ms[:lv]), "t_agg_ms": list(self.t_agg_ms[:lv]),
                 "t_total_ms": self.t_total_ms, "t_sweep_ms_total": self.t_sweep_ms_total,
                 "t_sweep_ms_first": self.t_sweep_ms_first, "t_modularity_ms_total": self.t_modularity_ms_total,
-                "edges_swept": self.edges_swept, "q": self.q.q, "L": int(self.q.L), "S": self.q.S,
+                "edges_swept": self.edges_swept, "moved_first": self.moved_first,
+                "kernel_launches": self.kernel_launches, "cub_calls": self.cub_calls, "q": self.q.q, "L": int(self.q.L), "S": self.q.S,
                 "W": int(self.q.W)}
 
 

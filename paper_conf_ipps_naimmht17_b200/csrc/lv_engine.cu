@@ -17,6 +17,7 @@
 namespace lv {
 
 static thread_local std::string g_err;
+long long g_launches = 0, g_cub_calls = 0;
 void set_error(const std::string& msg) { g_err = msg; }
 
 int32_t cuda_fail(cudaError_t e, const char* what, const char* file, int line) {
@@ -225,12 +226,14 @@ int32_t run_impl(Handle& h, const louvain_params_t& p, int32_t* labels_out, louv
   louvain_stats_t local;
   std::memset(&local, 0, sizeof local);
   auto t_begin = std::chrono::steady_clock::now();
+  const long long launches0 = g_launches, cub0 = g_cub_calls;
   int32_t* lab = nullptr;
   LV_TRY(dalloc(&lab, n0, s));
-  if (n0) k_iota<<<grid_for(n0, 256), 256, 0, s>>>(lab, n0);
+  if (n0) { k_iota<<<grid_for(n0, 256), 256, 0, s>>>(lab, n0); LV_LAUNCHED(); }
   // level 0 starts from singletons
   if (n0) {
     k_iota<<<grid_for(n0, 256), 256, 0, s>>>(L0.C, n0);
+    LV_LAUNCHED();
     LV_TRY(level_set_labels(h, L0, L0.C));
   }
   Level owned;   // current contracted level (levels >= 1)
@@ -264,7 +267,10 @@ int32_t run_impl(Handle& h, const louvain_params_t& p, int32_t* labels_out, louv
         const float t_sw = elapsed(h.ev[0], h.ev[1]);
         local.t_sweep_ms_total += t_sw;
         local.t_modularity_ms_total += elapsed(h.ev[1], h.ev[2]);
-        if (level == 0 && sweeps == 0) local.t_sweep_ms_first = t_sw;
+        if (level == 0 && sweeps == 0) {
+          local.t_sweep_ms_first = t_sw;
+          local.moved_first = (int64_t)h.h_ctl->logn;
+        }
         local.edges_swept += L.nnz;
         ++sweeps;
         const int64_t moved = (int64_t)h.h_ctl->logn;
@@ -325,6 +331,8 @@ int32_t run_impl(Handle& h, const louvain_params_t& p, int32_t* labels_out, louv
   dfree(lab, s);
   fill_q(&local.q, Lq, Sq, W);
   local.t_total_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t_begin).count();
+  local.kernel_launches = g_launches - launches0;
+  local.cub_calls = g_cub_calls - cub0;
   if (q_final) *q_final = local.q;
   if (st) *st = local;
   return LOUVAIN_OK;
@@ -453,6 +461,7 @@ LV_API int32_t louvain_get_csr(louvain_graph_t g, int64_t* rowptr, int32_t* col,
       rc = copy_out(w, L.w, 4 * (size_t)L.nnz, h.stream);
     } else if (is_device_ptr(w)) {
       k_fill_u32<<<grid_for(L.nnz, 256), 256, 0, h.stream>>>(w, L.nnz, 1u);
+      LV_LAUNCHED();
     } else {
       cudaStreamSynchronize(h.stream);
       for (int64_t e = 0; e < L.nnz; ++e) w[e] = 1u;
@@ -472,7 +481,7 @@ LV_API int32_t louvain_set_labels(louvain_graph_t g, const int32_t* labels) {
   Level& L = h.lv;
   int32_t rc = LOUVAIN_OK;
   if (!labels) {
-    if (L.n) k_iota<<<grid_for(L.n, 256), 256, 0, h.stream>>>(L.C, L.n);
+    if (L.n) { k_iota<<<grid_for(L.n, 256), 256, 0, h.stream>>>(L.C, L.n); LV_LAUNCHED(); }
     rc = level_set_labels(h, L, L.C);
   } else {
     int32_t* d = nullptr;

@@ -102,6 +102,13 @@ struct Handle {
   void* dist = nullptr;
 };
 
+// ------------------------------------------------------------------ launch accounting
+// Every explicit <<<>>> launch is followed by LV_LAUNCHED(); every device-wide
+// CUB call (scan / radix sort / reduce) by LV_CUB().  Reported in louvain_stats_t.
+extern long long g_launches, g_cub_calls;
+#define LV_LAUNCHED() (++lv::g_launches)
+#define LV_CUB() (++lv::g_cub_calls)
+
 // ------------------------------------------------------------------ memory helpers
 int32_t dmalloc(void** p, size_t bytes, cudaStream_t s);
 void dfree(void* p, cudaStream_t s);

@@ -288,15 +288,17 @@ int32_t level_setup(Handle& h, Level& L) {
     LV_CUDA(cub::DeviceSegmentedReduce::Sum(nullptr, tb, L.w, L.k, (int)n, L.rowptr, L.rowptr + 1, s));
     void* tmp = nullptr;
     LV_TRY(dmalloc(&tmp, tb, s));
-    LV_CUDA(cub::DeviceSegmentedReduce::Sum(tmp, tb, L.w, L.k, (int)n, L.rowptr, L.rowptr + 1, s));
+    LV_CUDA(cub::DeviceSegmentedReduce::Sum(tmp, tb, L.w, L.k, (int)n, L.rowptr, L.rowptr + 1, s)); LV_CUB();
     dfree(tmp, s);
   } else {
     k_degrees_unit<<<grid_for(n, 256), 256, 0, s>>>(L.rowptr, n, L.k);
+    LV_LAUNCHED();
   }
   // W = sum_i k_i = 2m (R1)
   unsigned long long* dW = &h.ctl->L;  // reuse a ctl word as scratch
   LV_CUDA(cudaMemsetAsync(dW, 0, 8, s));
   k_sum_u32<<<grid_for(n, 256, 148 * 8), 256, 0, s>>>(L.k, n, dW);
+  LV_LAUNCHED();
   unsigned long long W = 0;
   LV_CUDA(cudaMemcpyAsync(&W, dW, 8, cudaMemcpyDeviceToHost, s));
   LV_CUDA(cudaStreamSynchronize(s));
@@ -306,6 +308,7 @@ int32_t level_setup(Handle& h, Level& L) {
     return LOUVAIN_E_OVERFLOW;
   }
   k_init_singletons<<<grid_for(n, 256), 256, 0, s>>>(L.k, n, L.C, L.a, L.size);
+  LV_LAUNCHED();
   LV_CUDA(cudaGetLastError());
   return LOUVAIN_OK;
 }
@@ -315,8 +318,10 @@ int32_t level_set_labels(Handle& h, Level& L, const int32_t* d_labels) {
   if (L.n == 0) return LOUVAIN_OK;
   if (d_labels != L.C) LV_CUDA(cudaMemcpyAsync(L.C, d_labels, sizeof(int32_t) * L.n, cudaMemcpyDefault, s));
   k_totals_zero<<<grid_for(L.n, 256), 256, 0, s>>>(L.n, L.a, L.size);
+  LV_LAUNCHED();
   LV_CUDA(cudaMemsetAsync(&h.ctl->bad, 0, 8, s));
   k_totals_add<<<grid_for(L.n, 256), 256, 0, s>>>(L.C, L.k, L.n, L.a, L.size, &h.ctl->bad);
+  LV_LAUNCHED();
   unsigned long long bad = 0;
   LV_CUDA(cudaMemcpyAsync(&bad, &h.ctl->bad, 8, cudaMemcpyDeviceToHost, s));
   LV_CUDA(cudaStreamSynchronize(s));
@@ -346,13 +351,14 @@ int32_t level_binning(Handle& h, Level& L, const louvain_params_t& p) {
     LV_CUDA(cudaMemsetAsync(hist, 0, 8 * kNumClasses, s));
     k_classify<<<grid_for(n, 256), 256, 0, s>>>(L.rowptr, n, p.deg_bounds[0], p.deg_bounds[1], p.deg_bounds[2],
                                                 p.deg_bounds[3], p.deg_bounds[4], p.deg_bounds[5], cls, iota, hist);
+    LV_LAUNCHED();
     LV_CUDA(cudaGetLastError());
     // stable sort by class (5 bits): vertices of a class stay in ascending id order
     size_t tb = 0;
     LV_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, tb, cls, cls2, iota, L.bin_vertices, n, 0, 5, s));
     void* tmp = nullptr;
     LV_TRY(dmalloc(&tmp, tb, s));
-    LV_CUDA(cub::DeviceRadixSort::SortPairs(tmp, tb, cls, cls2, iota, L.bin_vertices, n, 0, 5, s));
+    LV_CUDA(cub::DeviceRadixSort::SortPairs(tmp, tb, cls, cls2, iota, L.bin_vertices, n, 0, 5, s)); LV_CUB();
     dfree(tmp, s);
     unsigned long long hh[kNumClasses];
     LV_CUDA(cudaMemcpyAsync(hh, hist, sizeof hh, cudaMemcpyDeviceToHost, s));
@@ -373,6 +379,7 @@ int32_t level_binning(Handle& h, Level& L, const louvain_params_t& p) {
     int64_t* dd = nullptr;
     LV_TRY(dalloc(&dd, 2 * cnt, s));
     k_hub_degrees<<<grid_for(cnt, 256), 256, 0, s>>>(L.bin_vertices + off, cnt, L.rowptr, dd);
+    LV_LAUNCHED();
     LV_CUDA(cudaMemcpyAsync(v.data(), L.bin_vertices + off, 4 * cnt, cudaMemcpyDeviceToHost, s));
     LV_CUDA(cudaMemcpyAsync(d.data(), dd, 16 * cnt, cudaMemcpyDeviceToHost, s));
     LV_CUDA(cudaStreamSynchronize(s));
@@ -420,6 +427,7 @@ int32_t level_binning(Handle& h, Level& L, const louvain_params_t& p) {
     LV_CUDA(cudaMemcpyAsync(P.scan, scan.data(), 8 * scan.size(), cudaMemcpyHostToDevice, s));
     LV_CUDA(cudaMemcpyAsync(P.scan_first, first.data(), 8 * (P.nh + 1), cudaMemcpyHostToDevice, s));
     k_fill_u64<<<grid_for(tot, 256), 256, 0, s>>>(P.table, tot, kEmpty);
+    LV_LAUNCHED();
     LV_CUDA(cudaGetLastError());
     LV_CUDA(cudaStreamSynchronize(s));  // host vectors die here
   }
@@ -442,12 +450,15 @@ int32_t launch_modularity(Handle& h, Level& L, const int32_t* d_C) {
     LV_TRY(dalloc(&a_tmp, L.n, s));
     LV_TRY(dalloc(&size_tmp, L.n, s));
     k_totals_zero<<<grid_for(L.n, 256), 256, 0, s>>>(L.n, a_tmp, size_tmp);
+    LV_LAUNCHED();
     k_totals_add<<<grid_for(L.n, 256), 256, 0, s>>>(d_C, L.k, L.n, a_tmp, size_tmp, &h.ctl->bad);
+    LV_LAUNCHED();
     a = a_tmp;
   }
   const int64_t ntiles = (L.nnz + kTileEdges - 1) / kTileEdges;
   const unsigned grid = grid_for(std::max<int64_t>(ntiles, (L.n + 255) / 256), 1, 148 * 8);
   k_modularity<<<grid, 256, 0, s>>>(L.rowptr, L.n, L.col, L.w, d_C, a, L.nnz, &h.ctl->L, &h.ctl->S);
+  LV_LAUNCHED();
   LV_CUDA(cudaGetLastError());
   if (a_tmp) { dfree(a_tmp, s); dfree(size_tmp, s); }
   return LOUVAIN_OK;
@@ -469,12 +480,14 @@ int32_t level_modularity(Handle& h, Level& L, const int32_t* d_C, uint64_t* Lout
 
 int32_t launch_commit(Handle& h, Level& L, int bucket) {
   k_commit<<<148 * 4, 256, 0, h.stream>>>(h.ctl, bucket, L.mv_v, L.mv_new, L.mv_old, L.C, L.a, L.size, L.k);
+  LV_LAUNCHED();
   LV_CUDA(cudaGetLastError());
   return LOUVAIN_OK;
 }
 
 int32_t launch_revert(Handle& h, Level& L) {
   k_revert<<<148 * 4, 256, 0, h.stream>>>(h.ctl, L.mv_v, L.mv_new, L.mv_old, L.C, L.a, L.size, L.k);
+  LV_LAUNCHED();
   LV_CUDA(cudaGetLastError());
   return LOUVAIN_OK;
 }
@@ -482,6 +495,7 @@ int32_t launch_revert(Handle& h, Level& L) {
 int32_t compose_labels(Handle& h, int32_t* lab, int64_t n0, const int32_t* map) {
   if (n0 == 0) return LOUVAIN_OK;
   k_compose<<<grid_for(n0, 256), 256, 0, h.stream>>>(lab, n0, map);
+  LV_LAUNCHED();
   LV_CUDA(cudaGetLastError());
   return LOUVAIN_OK;
 }
@@ -505,11 +519,12 @@ int32_t level_contract(Handle& h, Level& L, Level& out, int32_t* d_map) {
   LV_TRY(dalloc(&flag, n, s));
   LV_TRY(dalloc(&newID, n, s));
   k_flags_nonempty<<<grid_for(n, 256), 256, 0, s>>>(L.size, n, flag);
+  LV_LAUNCHED();
   size_t tb = 0;
   LV_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, tb, flag, newID, n, s));
   void* tmp = nullptr;
   LV_TRY(dmalloc(&tmp, tb, s));
-  LV_CUDA(cub::DeviceScan::ExclusiveSum(tmp, tb, flag, newID, n, s));
+  LV_CUDA(cub::DeviceScan::ExclusiveSum(tmp, tb, flag, newID, n, s)); LV_CUB();
   dfree(tmp, s);
   int32_t last[2];
   LV_CUDA(cudaMemcpyAsync(&last[0], newID + n - 1, 4, cudaMemcpyDeviceToHost, s));
@@ -517,6 +532,7 @@ int32_t level_contract(Handle& h, Level& L, Level& out, int32_t* d_map) {
   LV_CUDA(cudaStreamSynchronize(s));
   const int64_t np = (int64_t)last[0] + last[1];
   k_map<<<grid_for(n, 256), 256, 0, s>>>(L.C, newID, n, d_map);
+  LV_LAUNCHED();
   dfree(flag, s);
   dfree(newID, s);
   out.n = np;
@@ -539,6 +555,7 @@ int32_t level_contract(Handle& h, Level& L, Level& out, int32_t* d_map) {
     const int64_t ntiles = (nnz + kTileEdges - 1) / kTileEdges;
     k_emit_keys<<<grid_for(ntiles, 1, 148 * 8), 256, 0, s>>>(L.rowptr, n, L.col, L.w, d_map, nnz, (uint64_t)np, k0,
                                                              weighted ? v0 : nullptr);
+    LV_LAUNCHED();
     LV_CUDA(cudaGetLastError());
   }
   int bits = 1;
@@ -551,6 +568,7 @@ int32_t level_contract(Handle& h, Level& L, Level& out, int32_t* d_map) {
   LV_TRY(dmalloc(&tmp, tb, s));
   if (weighted) LV_CUDA(cub::DeviceRadixSort::SortPairs(tmp, tb, kb, vb, nnz, 0, bits, s));
   else LV_CUDA(cub::DeviceRadixSort::SortKeys(tmp, tb, kb, nnz, 0, bits, s));
+  LV_CUB();
   dfree(tmp, s);
   unsigned long long* sorted = kb.Current();
   unsigned long long* uniq = kb.Alternate();
@@ -560,11 +578,11 @@ int32_t level_contract(Handle& h, Level& L, Level& out, int32_t* d_map) {
   if (weighted) {
     LV_CUDA(cub::DeviceReduce::ReduceByKey(nullptr, tb, sorted, uniq, vb.Current(), sums, d_num, cub::Sum(), nnz, s));
     LV_TRY(dmalloc(&tmp, tb, s));
-    LV_CUDA(cub::DeviceReduce::ReduceByKey(tmp, tb, sorted, uniq, vb.Current(), sums, d_num, cub::Sum(), nnz, s));
+    LV_CUDA(cub::DeviceReduce::ReduceByKey(tmp, tb, sorted, uniq, vb.Current(), sums, d_num, cub::Sum(), nnz, s)); LV_CUB();
   } else {
     LV_CUDA(cub::DeviceRunLengthEncode::Encode(nullptr, tb, sorted, uniq, sums, d_num, nnz, s));
     LV_TRY(dmalloc(&tmp, tb, s));
-    LV_CUDA(cub::DeviceRunLengthEncode::Encode(tmp, tb, sorted, uniq, sums, d_num, nnz, s));
+    LV_CUDA(cub::DeviceRunLengthEncode::Encode(tmp, tb, sorted, uniq, sums, d_num, nnz, s)); LV_CUB();
   }
   dfree(tmp, s);
   int64_t m = 0;
@@ -578,13 +596,15 @@ int32_t level_contract(Handle& h, Level& L, Level& out, int32_t* d_map) {
   LV_TRY(dalloc(&cnt, np + 1, s));
   LV_CUDA(cudaMemsetAsync(cnt, 0, 8 * (np + 1), s));
   k_row_counts<<<grid_for(m, 256), 256, 0, s>>>(uniq, m, (uint64_t)np, cnt);
+  LV_LAUNCHED();
   tb = 0;
   LV_CUDA(cub::DeviceScan::InclusiveSum(nullptr, tb, cnt, out.rowptr, np + 1, s));
   LV_TRY(dmalloc(&tmp, tb, s));
-  LV_CUDA(cub::DeviceScan::InclusiveSum(tmp, tb, cnt, out.rowptr, np + 1, s));
+  LV_CUDA(cub::DeviceScan::InclusiveSum(tmp, tb, cnt, out.rowptr, np + 1, s)); LV_CUB();
   dfree(tmp, s);
   dfree(cnt, s);
   k_split_keys<<<grid_for(m, 256), 256, 0, s>>>(uniq, m, (uint64_t)np, out.col);
+  LV_LAUNCHED();
   LV_CUDA(cudaMemcpyAsync(out.w, sums, 4 * m, cudaMemcpyDeviceToDevice, s));
   LV_CUDA(cudaGetLastError());
   dfree(uniq, s);

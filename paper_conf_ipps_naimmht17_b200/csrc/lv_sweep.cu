@@ -311,10 +311,13 @@ int32_t dispatch_class(Handle& h, Level& L, const SweepArgs& A, int bucket, int 
       case 16: sweep_small<16, UNIT><<<grid, 256, 0, s>>>(verts, nv, A); break;
       default: sweep_small<32, UNIT><<<grid, 256, 0, s>>>(verts, nv, A); break;
     }
+    LV_LAUNCHED();
   } else if (sub == 0 && max_deg <= 84) {
     sweep_warp<128, UNIT><<<grid_for(nv, 8, 148 * 8), 256, 0, s>>>(verts, nv, A);
+    LV_LAUNCHED();
   } else if (sub == 0 && max_deg <= 340) {
     sweep_warp<512, UNIT><<<grid_for(nv, 8, 148 * 6), 256, 0, s>>>(verts, nv, A);
+    LV_LAUNCHED();
   } else if (sub <= 1) {
     const int cap = (sub == 0) ? kCtaSmallCap : kCtaLargeCap;
     const int threads = (sub == 0) ? 256 : 1024;
@@ -326,14 +329,18 @@ int32_t dispatch_class(Handle& h, Level& L, const SweepArgs& A, int bucket, int 
     }
     const unsigned grid = grid_for(nv, 1, 148 * (sub == 0 ? 3 : 1));
     sweep_cta<UNIT><<<grid, threads, smem, s>>>(verts, nv, A, cap);
+    LV_LAUNCHED();
   } else {
     HubPlan& P = L.hub;
     if (P.nh > 0) {
       hub_insert<UNIT><<<grid_for(P.nchunks, 1, 148 * 4), 512, 0, s>>>(P.chunk, P.nchunks, P.hub_v, P.tab_off,
                                                                        P.tab_cap, P.table, A);
+      LV_LAUNCHED();
       hub_scan<<<grid_for(P.nscan, 1, 148 * 4), 512, 0, s>>>(P.scan, P.nscan, P.hub_v, P.tab_off, P.table,
                                                              (Partial*)P.partial, A);
+      LV_LAUNCHED();
       hub_final<<<grid_for(P.nh, 8), 256, 0, s>>>(P.nh, P.scan_first, (const Partial*)P.partial, P.hub_v, A);
+      LV_LAUNCHED();
     }
   }
   LV_CUDA(cudaGetLastError());
