@@ -162,7 +162,9 @@ int32_t finish_call(Handle& h, int32_t rc) {
   return rc;
 }
 
-bool bucket_nonempty(const Level& L, int b) { return L.class_off[4 * b + 3] > L.class_off[4 * b]; }
+bool bucket_nonempty(const Level& L, int b) {
+  return L.class_off[kSubPerBucket * (b + 1)] > L.class_off[kSubPerBucket * b];
+}
 
 // One sweep body: for each non-empty bucket 1..7 its sweep kernels, then its
 // commit (BIN_SYNC) -- or a single commit at the end (RELAXED).
@@ -175,6 +177,7 @@ int32_t sweep_body(Handle& h, Level& L, const louvain_params_t& p) {
     if (p.mode == LOUVAIN_MODE_BIN_SYNC) LV_TRY(launch_commit(h, L, commits++));
   }
   if (p.mode == LOUVAIN_MODE_RELAXED) LV_TRY(launch_commit(h, L, commits++));
+  ++L.sweeps_done;
   return LOUVAIN_OK;
 }
 
@@ -231,11 +234,8 @@ int32_t run_impl(Handle& h, const louvain_params_t& p, int32_t* labels_out, louv
   LV_TRY(dalloc(&lab, n0, s));
   if (n0) { k_iota<<<grid_for(n0, 256), 256, 0, s>>>(lab, n0); LV_LAUNCHED(); }
   // level 0 starts from singletons
-  if (n0) {
-    k_iota<<<grid_for(n0, 256), 256, 0, s>>>(L0.C, n0);
-    LV_LAUNCHED();
-    LV_TRY(level_set_labels(h, L0, L0.C));
-  }
+  if (n0) LV_TRY(level_set_labels(h, L0, nullptr));
+  uint64_t Lq = 0, Sq = 0;  // exact parts of the current level's kept partition
   Level owned;   // current contracted level (levels >= 1)
   Level* cur = &L0;
   int32_t* map = nullptr;
@@ -249,8 +249,10 @@ int32_t run_impl(Handle& h, const louvain_params_t& p, int32_t* labels_out, louv
       Level& L = *cur;
       const int pexp = (L.n > p.size_limit) ? p.th_bin_exp : p.th_final_exp;  // P:330, R14
       LV_TRY(level_binning(h, L, p));
-      uint64_t Lq, Sq;
-      LV_TRY(level_modularity(h, L, L.C, &Lq, &Sq));
+      // level start: singletons.  Level 0 evaluates Eq. (1); a contracted level
+      // starts exactly where the previous one ended (contraction preserves L and
+      // S, R18 -- pinned by the oracle tests and the parity suite).
+      if (level == 0) LV_TRY(level_modularity(h, L, nullptr, &Lq, &Sq));
       const int64_t num_start = qnum_of(Lq, Sq, W);
       int64_t num_prev = num_start;
       int64_t moved_level = 0;
@@ -260,7 +262,7 @@ int32_t run_impl(Handle& h, const louvain_params_t& p, int32_t* labels_out, louv
         cudaEventRecord(h.ev[0], s);
         LV_TRY(sweep_body(h, L, p));
         cudaEventRecord(h.ev[1], s);
-        LV_TRY(launch_modularity(h, L, L.C));
+        LV_TRY(launch_modularity(h, L, nullptr));
         cudaEventRecord(h.ev[2], s);
         LV_CUDA(cudaMemcpyAsync(h.h_ctl, h.ctl, sizeof(DevCtl), cudaMemcpyDeviceToHost, s));
         LV_CUDA(cudaStreamSynchronize(s));
@@ -279,12 +281,13 @@ int32_t run_impl(Handle& h, const louvain_params_t& p, int32_t* labels_out, louv
           LV_TRY(launch_revert(h, L));
           break;
         }
+        Lq = h.h_ctl->L;
+        Sq = h.h_ctl->S;
         moved_level += moved;
         if (moved == 0 || below_threshold(num, num_prev, W, pexp)) break;  // Alg. 1 l.12, R13
         num_prev = num;
       }
-      LV_TRY(level_modularity(h, L, L.C, &Lq, &Sq));
-      const int64_t num_end = qnum_of(Lq, Sq, W);
+      const int64_t num_end = qnum_of(Lq, Sq, W);  // the partition kept at the end of the phase
       cudaEventRecord(e_lvl1, s);
       local.n[level] = L.n;
       local.nnz[level] = L.nnz;
@@ -297,7 +300,7 @@ int32_t run_impl(Handle& h, const louvain_params_t& p, int32_t* labels_out, louv
       LV_CUDA(cudaEventSynchronize(e_lvl1));
       local.t_opt_ms[level] = elapsed(e_lvl0, e_lvl1);
       if (moved_level == 0 || below_threshold(num_end, num_start, W, p.th_final_exp)) {  // R16
-        LV_TRY(compose_labels(h, lab, n0, L.C));
+        LV_TRY(compose_labels_ca(h, lab, n0, L.ca));
         cudaEventDestroy(e_lvl0);
         cudaEventDestroy(e_lvl1);
         break;
@@ -322,10 +325,9 @@ int32_t run_impl(Handle& h, const louvain_params_t& p, int32_t* labels_out, louv
     }
   }
   if (cur != &L0) level_free(owned, s);
-  // the handle's partition becomes the final one
+  // the handle's partition becomes the final one; (Lq, Sq) are the exact parts of
+  // the last level's kept partition, equal to those of `lab` on the input graph
   LV_TRY(level_set_labels(h, L0, lab));
-  uint64_t Lq = 0, Sq = 0;
-  if (n0) LV_TRY(level_modularity(h, L0, L0.C, &Lq, &Sq));
   LV_TRY(copy_out(labels_out, lab, sizeof(int32_t) * (size_t)n0, s));
   LV_CUDA(cudaStreamSynchronize(s));
   dfree(lab, s);
@@ -481,8 +483,7 @@ LV_API int32_t louvain_set_labels(louvain_graph_t g, const int32_t* labels) {
   Level& L = h.lv;
   int32_t rc = LOUVAIN_OK;
   if (!labels) {
-    if (L.n) { k_iota<<<grid_for(L.n, 256), 256, 0, h.stream>>>(L.C, L.n); LV_LAUNCHED(); }
-    rc = level_set_labels(h, L, L.C);
+    rc = level_set_labels(h, L, nullptr);
   } else {
     int32_t* d = nullptr;
     bool owned = false;
@@ -498,7 +499,11 @@ LV_API int32_t louvain_get_labels(louvain_graph_t g, int32_t* labels_out) {
   Handle& h = g->h;
   DeviceScope ds(h.device);
   if (!labels_out && h.lv.n) { set_error("null labels_out"); return LOUVAIN_E_INVALID_ARG; }
-  int32_t rc = copy_out(labels_out, h.lv.C, 4 * (size_t)h.lv.n, h.stream);
+  int32_t* tmp = nullptr;
+  int32_t rc = dalloc(&tmp, h.lv.n, h.stream);
+  if (!rc) rc = level_get_labels(h, h.lv, tmp);
+  if (!rc) rc = copy_out(labels_out, tmp, 4 * (size_t)h.lv.n, h.stream);
+  dfree(tmp, h.stream);
   if (!rc) {
     cudaError_t e = cudaStreamSynchronize(h.stream);
     if (e != cudaSuccess) rc = cuda_fail(e, "sync", __FILE__, __LINE__);
@@ -510,7 +515,11 @@ LV_API int32_t louvain_get_totals(louvain_graph_t g, uint32_t* a_out, int32_t* s
   LV_TRY(guard(g));
   Handle& h = g->h;
   DeviceScope ds(h.device);
-  int32_t rc = copy_out(a_out, h.lv.a, 4 * (size_t)h.lv.n, h.stream);
+  uint32_t* tmp = nullptr;
+  int32_t rc = dalloc(&tmp, h.lv.n, h.stream);
+  if (!rc) rc = level_get_a(h, h.lv, tmp);
+  if (!rc) rc = copy_out(a_out, tmp, 4 * (size_t)h.lv.n, h.stream);
+  dfree(tmp, h.stream);
   if (!rc) rc = copy_out(size_out, h.lv.size, 4 * (size_t)h.lv.n, h.stream);
   if (!rc) {
     cudaError_t e = cudaStreamSynchronize(h.stream);
@@ -529,7 +538,7 @@ LV_API int32_t louvain_sweep(louvain_graph_t g, const louvain_params_t* p, int64
   Level& L = h.lv;
   int32_t rc = level_binning(h, L, pp);
   if (!rc) rc = sweep_body(h, L, pp);
-  if (!rc && q_after) rc = launch_modularity(h, L, L.C);
+  if (!rc && q_after) rc = launch_modularity(h, L, nullptr);
   if (!rc) {
     cudaError_t e = cudaMemcpyAsync(h.h_ctl, h.ctl, sizeof(DevCtl), cudaMemcpyDeviceToHost, h.stream);
     if (e == cudaSuccess) e = cudaStreamSynchronize(h.stream);
@@ -548,7 +557,7 @@ LV_API int32_t louvain_modularity(louvain_graph_t g, const int32_t* labels, louv
   Handle& h = g->h;
   DeviceScope ds(h.device);
   Level& L = h.lv;
-  int32_t* d = L.C;
+  int32_t* d = nullptr;
   bool owned = false;
   int32_t rc = LOUVAIN_OK;
   if (labels) rc = stage(labels, L.n, false, h.stream, &d, &owned);

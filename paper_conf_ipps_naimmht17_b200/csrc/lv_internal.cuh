@@ -2,7 +2,9 @@
 //
 // Device layout of one level (SURVEY 8 "Device layout at every level"):
 //   rowptr int64[n+1], col int32[nnz], w uint32[nnz] (absent at unit weight),
-//   k uint32[n], C int32[n], a uint32[n], size int32[n], W uint64,
+//   k uint32[n], ca uint2[n] = {C[v], a[v]} packed so one 8-byte gather of a
+//   neighbour brings both its label and (when it represents its community) a_c,
+//   size int32[n], W uint64,
 //   bin_vertices int32[n] sorted by dispatch class, move log (v, new, old) int32[n].
 #pragma once
 #include <cuda_runtime.h>
@@ -33,17 +35,26 @@ int32_t cuda_fail(cudaError_t e, const char* what, const char* file, int line);
   } while (0)
 
 // ------------------------------------------------------------------ dispatch classes
-// Vertices are sorted once per level by class = 4*bucket + sub, bucket in 0..7
+// Vertices are sorted once per level by class = 8*bucket + sub, bucket in 0..7
 // (0 = degree 0, never moves; 1..7 = the paper's buckets) and sub the
-// kernel family inside the bucket (by degree): 0 register/warp/CTA-small,
-// 1 CTA-large, 2 hub (multi-CTA, global hash).
-constexpr int kNumClasses = 32;
-constexpr int64_t kCtaLargeMin = 4096;   // deg >= this: 1024-thread CTA, 128 KB table
-constexpr int64_t kHubMin = 12288;       // deg >= this: multi-CTA global hash
-constexpr int kCtaSmallCap = 8192;       // slots (64 KB)
-constexpr int kCtaLargeCap = 16384;      // slots (128 KB)
-constexpr int64_t kHubChunkEdges = 8192; // edges per hub insert chunk
-constexpr int64_t kHubScanSlots = 8192;  // slots per hub scan chunk
+// kernel family inside the bucket, by degree:
+//   sub 0: deg < 1024   (register / warp / 256-thread CTA kernels, by bucket bound)
+//   sub 1: [1024, 4096) 512-thread CTA, smem table <= 8192 slots
+//   sub 2: [4096,12288) 1024-thread CTA, smem table <= 16384 slots
+//   sub 3: [12288, 32768)   4-CTA cluster, table in distributed shared memory
+//   sub 4: [32768, 131072)  16-CTA cluster, table in distributed shared memory
+//   sub 5: >= 131072        hub: cooperative grid, global table in an L2-sized ring
+constexpr int kSubPerBucket = 8;
+constexpr int kNumClasses = 8 * kSubPerBucket;
+constexpr int64_t kSub1Min = 1024, kSub2Min = 4096, kSub3Min = 12288, kSub4Min = 32768, kHubMin = 131072;
+constexpr int kClusterSlots = 16384;  // table slots per cluster CTA (12 B each: 192 KB)
+constexpr int kCap0 = 2048, kCap1 = 8192, kCap2 = 16384;  // smem table slots (12 B each)
+constexpr int64_t kHubChunkEdges = 2048;  // edges per hub insert item
+constexpr int64_t kHubScanSlots = 4096;   // slots per hub scan item
+constexpr int64_t kHubWaveSlots = 3 << 19;  // table slots per wave (12 B each; ring = 2 segments)
+inline int sub_of_degree(int64_t d) {
+  return d < kSub1Min ? 0 : d < kSub2Min ? 1 : d < kSub3Min ? 2 : d < kSub4Min ? 3 : d < kHubMin ? 4 : 5;
+}
 
 struct DevCtl {
   unsigned long long logn;       // move-log entries appended in this sweep
@@ -52,18 +63,35 @@ struct DevCtl {
   unsigned long long bad;        // validation flag
 };
 
+// Hub work plan (one per level).  Hubs are grouped into waves whose tables fit
+// one segment of a 2-segment ring (wave k uses segment k % 2).  A cooperative
+// kernel runs phases separated by grid.sync(): phase p inserts the edges of
+// wave p, scans the tables of wave p-1 and takes the decisions of wave p-2, so
+// every dependency is enforced by a barrier (no spinning, no tickets) and at
+// most two waves' tables are live -- small enough to stay in L2.
+struct HubItem {
+  int32_t hub;
+  int32_t pad;
+  int64_t begin, end;  // insert: edge range; scan: slot range of the hub's table
+};
+struct HubInfo {
+  int32_t v;           // vertex id
+  int32_t nscan;       // scan items of this hub
+  int64_t off, cap;    // table region within its wave's ring segment
+  int64_t scan_first;  // index of its first scan item (= its first partial)
+};
 struct HubPlan {
-  int64_t nh = 0;
-  int64_t nchunks = 0, nscan = 0;
-  int32_t* hub_v = nullptr;         // [nh]
-  int64_t* tab_off = nullptr;       // [nh]
-  int64_t* tab_cap = nullptr;       // [nh]
-  int64_t* chunk = nullptr;         // [3*nchunks]: hub, e_begin, e_end
-  int64_t* scan = nullptr;          // [3*nscan]: hub, slot_begin, slot_end
-  int64_t* scan_first = nullptr;    // [nh+1]: first scan chunk of each hub
-  unsigned long long* table = nullptr;  // sum tab_cap slots (EMPTY-initialised)
-  int64_t table_slots = 0;
-  void* partial = nullptr;          // [nscan] Partial
+  int64_t nh = 0, nwaves = 0, nins = 0, nscan = 0, seg = 0;
+  HubItem* ins = nullptr;        // insert items, wave-major
+  HubItem* scans = nullptr;      // scan items, wave-major (index = partial slot)
+  int64_t* ins_off = nullptr;    // [nwaves+1]
+  int64_t* scan_off = nullptr;   // [nwaves+1]
+  int64_t* wave_hub = nullptr;   // [nwaves+1] first hub of each wave
+  HubInfo* info = nullptr;       // [nh]
+  unsigned long long* ring = nullptr;  // 2 * seg slots {label|e}, EMPTY-initialised
+  uint32_t* ring_a = nullptr;          // a_c when known (0xFFFFFFFF = unknown)
+  void* partial = nullptr;             // [nscan]
+  int grid = 0;                        // co-resident CTAs of the cooperative kernel
 };
 
 struct Level {
@@ -74,13 +102,13 @@ struct Level {
   uint32_t* w = nullptr;  // nullptr = unit weights (level 0 of every config, R20)
   bool owns_csr = true;
   uint32_t* k = nullptr;
-  int32_t* C = nullptr;
-  uint32_t* a = nullptr;
+  uint2* ca = nullptr;  // {C[v], a[v]}
   int32_t* size = nullptr;
   // move log of the current sweep (v, new, old) -- also the revert record (R15)
   int32_t* mv_v = nullptr;
   int32_t* mv_new = nullptr;
   int32_t* mv_old = nullptr;
+  int32_t sweeps_done = 0;  // sweeps since the partition was last reset to singletons
   // binning (valid for bins_bounds)
   bool bins_valid = false;
   int64_t bins_bounds[6] = {0, 0, 0, 0, 0, 0};
@@ -122,14 +150,19 @@ bool is_device_ptr(const void* p);
 int32_t level_alloc_state(Level& L, cudaStream_t s);
 void level_free(Level& L, cudaStream_t s);
 int32_t level_setup(Handle& h, Level& L);  // k, W, singleton partition (Alg. 1 l.2)
-int32_t level_set_labels(Handle& h, Level& L, const int32_t* d_labels);  // C given, recompute a/size
+int32_t level_set_labels(Handle& h, Level& L, const int32_t* d_labels);  // C given (nullptr = iota), recompute a/size
+int32_t level_get_labels(Handle& h, Level& L, int32_t* d_out);          // C -> d_out (device)
+int32_t level_get_a(Handle& h, Level& L, uint32_t* d_out);              // a -> d_out (device)
 int32_t level_binning(Handle& h, Level& L, const louvain_params_t& p);  // classes + hub plan
+// d_C == nullptr: the level's own partition (maintained a_c); else external labels
 int32_t level_modularity(Handle& h, Level& L, const int32_t* d_C, uint64_t* Lout, uint64_t* Sout);
 int32_t launch_modularity(Handle& h, Level& L, const int32_t* d_C);  // async: ctl->L, ctl->S
 int32_t launch_commit(Handle& h, Level& L, int bucket);
 int32_t launch_revert(Handle& h, Level& L);
 int32_t level_contract(Handle& h, Level& L, Level& out, int32_t* d_map);  // Alg. 3
 int32_t compose_labels(Handle& h, int32_t* lab, int64_t n0, const int32_t* map);  // lab[i] = map[lab[i]]
+int32_t compose_labels_ca(Handle& h, int32_t* lab, int64_t n0, const uint2* ca);   // lab[i] = C[lab[i]]
+size_t hub_partial_bytes();
 int32_t validate_csr_host(int64_t n, int64_t nnz, const int64_t* rowptr, const int32_t* col, const uint32_t* w,
                           bool full, uint64_t* W);
 

@@ -14,8 +14,6 @@
 
 namespace lv {
 
-size_t hub_partial_bytes();
-
 namespace {
 
 constexpr int kTileEdges = 2048;  // edges per block tile in edge-centric kernels
@@ -26,32 +24,51 @@ __global__ void k_degrees_unit(const int64_t* rowptr, int64_t n, uint32_t* k) {
     k[i] = (uint32_t)(rowptr[i + 1] - rowptr[i]);
 }
 
-__global__ void k_init_singletons(const uint32_t* k, int64_t n, int32_t* C, uint32_t* a, int32_t* size) {
+__global__ void k_init_singletons(const uint32_t* k, int64_t n, uint2* ca, int32_t* size) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
-    C[i] = (int32_t)i;  // C[i] = i at the start of each phase
-    a[i] = k[i];        // a_C(i) = k_i initially
+    ca[i] = make_uint2((uint32_t)i, k[i]);  // C[i] = i, a_C(i) = k_i
     size[i] = 1;
   }
 }
 
-__global__ void k_totals_zero(int64_t n, uint32_t* a, int32_t* size) {
+// C[i] = labels[i] (or i), a = 0, size = 0; the C write keeps the packed record's a word.
+__global__ void k_set_C(const int32_t* labels, int64_t n, uint2* ca, int32_t* size) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
-    a[i] = 0;
+    ca[i] = make_uint2(labels ? (uint32_t)labels[i] : (uint32_t)i, 0u);
     size[i] = 0;
   }
 }
 
-__global__ void k_totals_add(const int32_t* C, const uint32_t* k, int64_t n, uint32_t* a, int32_t* size,
-                             unsigned long long* bad) {
+__global__ void k_totals_add(const uint2* ca, const uint32_t* k, int64_t n, int32_t* size, unsigned long long* bad) {
+  uint32_t* a = const_cast<uint32_t*>(reinterpret_cast<const uint32_t*>(ca)) + 1;  // a word, stride 2
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
-    int32_t c = C[i];
+    const int32_t c = (int32_t)ca[i].x;
     if (c < 0 || c >= n) { atomicAdd(bad, 1ull); continue; }
-    atomicAdd(&a[c], k[i]);  // a_c = sum_{i in c} k_i
+    atomicAdd(&a[2 * (int64_t)c], k[i]);  // a_c = sum_{i in c} k_i
     atomicAdd(&size[c], 1);
   }
 }
 
-// class = 4*bucket + sub  (lv_internal.cuh)
+// a_c of an external labelling (louvain_modularity with labels != NULL)
+__global__ void k_ext_totals(const int32_t* C, const uint32_t* k, int64_t n, uint32_t* a, unsigned long long* bad) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t c = C[i];
+    if (c < 0 || c >= n) { atomicAdd(bad, 1ull); continue; }
+    atomicAdd(&a[c], k[i]);
+  }
+}
+
+__global__ void k_get_C(const uint2* ca, int64_t n, int32_t* out) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    out[i] = (int32_t)ca[i].x;
+}
+
+__global__ void k_get_a(const uint2* ca, int64_t n, uint32_t* out) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    out[i] = ca[i].y;
+}
+
+// class = 8*bucket + sub  (lv_internal.cuh)
 __global__ void k_classify(const int64_t* rowptr, int64_t n, int64_t b0, int64_t b1, int64_t b2, int64_t b3,
                            int64_t b4, int64_t b5, uint8_t* cls, int32_t* iota, unsigned long long* hist) {
   __shared__ unsigned long long sh[kNumClasses];
@@ -68,8 +85,8 @@ __global__ void k_classify(const int64_t* rowptr, int64_t n, int64_t b0, int64_t
     else if (d <= b4) b = 5;
     else if (d <= b5) b = 6;
     else b = 7;
-    const int sub = d < kCtaLargeMin ? 0 : (d < kHubMin ? 1 : 2);
-    const uint8_t c = (uint8_t)(4 * b + sub);
+    const int sub = d < kSub1Min ? 0 : d < kSub2Min ? 1 : d < kSub3Min ? 2 : d < kSub4Min ? 3 : d < kHubMin ? 4 : 5;
+    const uint8_t c = (uint8_t)(kSubPerBucket * b + sub);
     cls[i] = c;
     iota[i] = (int32_t)i;
     atomicAdd(&sh[c], 1ull);
@@ -89,23 +106,27 @@ __global__ void k_hub_degrees(const int32_t* hv, int64_t nh, const int64_t* rowp
 __global__ void k_fill_u64(unsigned long long* p, int64_t n, unsigned long long v) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) p[i] = v;
 }
+__global__ void k_fill_u32v(uint32_t* p, int64_t n, uint32_t v) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) p[i] = v;
+}
 
 // Commit of one bucket (Alg. 1 l.8-11): C[i] = newComm[i] and the exact
 // integer a_c / size_c deltas (identical to recomputing a_c, R12).
 __global__ void k_commit(DevCtl* ctl, int bucket, const int32_t* mv_v, const int32_t* mv_new, int32_t* mv_old,
-                         int32_t* C, uint32_t* a, int32_t* size, const uint32_t* k) {
+                         uint2* ca, int32_t* size, const uint32_t* k) {
   const unsigned long long start = ctl->bounds[bucket];
   const unsigned long long end = *(volatile unsigned long long*)&ctl->logn;
   if (blockIdx.x == 0 && threadIdx.x == 0) ctl->bounds[bucket + 1] = end;
+  uint32_t* w32 = reinterpret_cast<uint32_t*>(ca);
   for (unsigned long long p = start + blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; p < end;
        p += (unsigned long long)gridDim.x * blockDim.x) {
     const int32_t i = mv_v[p], t = mv_new[p];
-    const int32_t old = C[i];
+    const int32_t old = (int32_t)w32[2 * (int64_t)i];
     mv_old[p] = old;
-    C[i] = t;
+    w32[2 * (int64_t)i] = (uint32_t)t;
     const uint32_t ki = k[i];
-    atomicSub(&a[old], ki);
-    atomicAdd(&a[t], ki);
+    atomicSub(&w32[2 * (int64_t)old + 1], ki);
+    atomicAdd(&w32[2 * (int64_t)t + 1], ki);
     atomicSub(&size[old], 1);
     atomicAdd(&size[t], 1);
   }
@@ -113,15 +134,16 @@ __global__ void k_commit(DevCtl* ctl, int bucket, const int32_t* mv_v, const int
 
 // Undo every move of the sweep (R15).
 __global__ void k_revert(const DevCtl* ctl, const int32_t* mv_v, const int32_t* mv_new, const int32_t* mv_old,
-                         int32_t* C, uint32_t* a, int32_t* size, const uint32_t* k) {
+                         uint2* ca, int32_t* size, const uint32_t* k) {
   const unsigned long long end = ctl->logn;
+  uint32_t* w32 = reinterpret_cast<uint32_t*>(ca);
   for (unsigned long long p = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; p < end;
        p += (unsigned long long)gridDim.x * blockDim.x) {
     const int32_t i = mv_v[p], t = mv_new[p], old = mv_old[p];
-    C[i] = old;
+    w32[2 * (int64_t)i] = (uint32_t)old;
     const uint32_t ki = k[i];
-    atomicSub(&a[t], ki);
-    atomicAdd(&a[old], ki);
+    atomicSub(&w32[2 * (int64_t)t + 1], ki);
+    atomicAdd(&w32[2 * (int64_t)old + 1], ki);
     atomicSub(&size[t], 1);
     atomicAdd(&size[old], 1);
   }
@@ -162,24 +184,30 @@ __device__ __forceinline__ void for_tile_edges(const int64_t* rowptr, int64_t n,
 }
 
 // Eq. (1): L = sum of w over entries (u,v) with C[u] = C[v] (self-loops
-// included, R2); S = sum_c a_c^2.  Integer atomics: deterministic.
+// included, R2); S = sum_c a_c^2.  Integer atomics: deterministic.  Labels come
+// from the packed records (C = ca.x, a = ca.y) or from an external labelling.
+template <bool PACKED>
 __global__ void __launch_bounds__(256) k_modularity(const int64_t* rowptr, int64_t n, const int32_t* col,
-                                                    const uint32_t* w, const int32_t* C, const uint32_t* a,
-                                                    int64_t nnz, unsigned long long* Lout, unsigned long long* Sout) {
+                                                    const uint32_t* w, const uint2* ca, const int32_t* C,
+                                                    const uint32_t* a, int64_t nnz, unsigned long long* Lout,
+                                                    unsigned long long* Sout) {
   __shared__ int64_t sh_rows[kTileRows];
   __shared__ int64_t sh_u0;
   __shared__ int sh_nr;
+  const uint32_t* lab = PACKED ? reinterpret_cast<const uint32_t*>(ca) : reinterpret_cast<const uint32_t*>(C);
+  const int st = PACKED ? 2 : 1;
   unsigned long long acc = 0;
   const int64_t ntiles = (nnz + kTileEdges - 1) / kTileEdges;
   for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
     const int64_t e0 = tile * kTileEdges, e1 = min(nnz, e0 + kTileEdges);
     for_tile_edges(rowptr, n, e0, e1, sh_rows, &sh_u0, &sh_nr, [&](int64_t u, int64_t e) {
-      if (C[col[e]] == C[u]) acc += w ? w[e] : 1u;
+      const int32_t v = __ldcs(&col[e]);
+      if (__ldg(&lab[st * (int64_t)v]) == __ldg(&lab[st * u])) acc += w ? __ldcs(&w[e]) : 1u;
     });
   }
   unsigned long long s2 = 0;
   for (int64_t c = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; c < n; c += (int64_t)gridDim.x * blockDim.x) {
-    const unsigned long long x = a[c];
+    const unsigned long long x = PACKED ? ca[c].y : a[c];
     s2 += x * x;
   }
   acc = warp_sum_u64(acc);
@@ -196,9 +224,9 @@ __global__ void k_flags_nonempty(const int32_t* size, int64_t n, int32_t* flag) 
     flag[c] = size[c] > 0 ? 1 : 0;
 }
 
-__global__ void k_map(const int32_t* C, const int32_t* newID, int64_t n, int32_t* map) {
+__global__ void k_map(const uint2* ca, const int32_t* newID, int64_t n, int32_t* map) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
-    map[i] = newID[C[i]];  // R17: new ids in label order
+    map[i] = newID[ca[i].x];  // R17: new ids in label order
 }
 
 __global__ void __launch_bounds__(256) k_emit_keys(const int64_t* rowptr, int64_t n, const int32_t* col,
@@ -237,6 +265,10 @@ __global__ void k_compose(int32_t* lab, int64_t n0, const int32_t* map) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n0; i += (int64_t)gridDim.x * blockDim.x)
     lab[i] = map[lab[i]];
 }
+__global__ void k_compose_ca(int32_t* lab, int64_t n0, const uint2* ca) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n0; i += (int64_t)gridDim.x * blockDim.x)
+    lab[i] = (int32_t)ca[lab[i]].x;
+}
 
 __global__ void k_sum_u32(const uint32_t* x, int64_t n, unsigned long long* out) {
   unsigned long long acc = 0;
@@ -250,8 +282,7 @@ __global__ void k_sum_u32(const uint32_t* x, int64_t n, unsigned long long* out)
 // ======================================================================== host side
 int32_t level_alloc_state(Level& L, cudaStream_t s) {
   LV_TRY(dalloc(&L.k, L.n, s));
-  LV_TRY(dalloc(&L.C, L.n, s));
-  LV_TRY(dalloc(&L.a, L.n, s));
+  LV_TRY(dalloc(&L.ca, L.n, s));
   LV_TRY(dalloc(&L.size, L.n, s));
   LV_TRY(dalloc(&L.mv_v, L.n, s));
   LV_TRY(dalloc(&L.mv_new, L.n, s));
@@ -261,8 +292,9 @@ int32_t level_alloc_state(Level& L, cudaStream_t s) {
 }
 
 static void hub_free(HubPlan& P, cudaStream_t s) {
-  dfree(P.hub_v, s); dfree(P.tab_off, s); dfree(P.tab_cap, s); dfree(P.chunk, s); dfree(P.scan, s);
-  dfree(P.scan_first, s); dfree(P.table, s); dfree(P.partial, s);
+  dfree(P.ins, s); dfree(P.scans, s); dfree(P.ins_off, s); dfree(P.scan_off, s); dfree(P.wave_hub, s);
+  dfree(P.info, s); dfree(P.ring, s);
+  dfree(P.partial, s);
   P = HubPlan();
 }
 
@@ -272,7 +304,7 @@ void level_free(Level& L, cudaStream_t s) {
     dfree(L.col, s);
     dfree(L.w, s);
   }
-  dfree(L.k, s); dfree(L.C, s); dfree(L.a, s); dfree(L.size, s);
+  dfree(L.k, s); dfree(L.ca, s); dfree(L.size, s);
   dfree(L.mv_v, s); dfree(L.mv_new, s); dfree(L.mv_old, s); dfree(L.bin_vertices, s);
   hub_free(L.hub, s);
   L = Level();
@@ -307,7 +339,7 @@ int32_t level_setup(Handle& h, Level& L) {
     set_error("W = 2m exceeds 3,037,000,499 (int64 gain guard, R4)");
     return LOUVAIN_E_OVERFLOW;
   }
-  k_init_singletons<<<grid_for(n, 256), 256, 0, s>>>(L.k, n, L.C, L.a, L.size);
+  k_init_singletons<<<grid_for(n, 256), 256, 0, s>>>(L.k, n, L.ca, L.size);
   LV_LAUNCHED();
   LV_CUDA(cudaGetLastError());
   return LOUVAIN_OK;
@@ -315,12 +347,12 @@ int32_t level_setup(Handle& h, Level& L) {
 
 int32_t level_set_labels(Handle& h, Level& L, const int32_t* d_labels) {
   cudaStream_t s = h.stream;
+  L.sweeps_done = d_labels ? 1 : 0;
   if (L.n == 0) return LOUVAIN_OK;
-  if (d_labels != L.C) LV_CUDA(cudaMemcpyAsync(L.C, d_labels, sizeof(int32_t) * L.n, cudaMemcpyDefault, s));
-  k_totals_zero<<<grid_for(L.n, 256), 256, 0, s>>>(L.n, L.a, L.size);
+  k_set_C<<<grid_for(L.n, 256), 256, 0, s>>>(d_labels, L.n, L.ca, L.size);
   LV_LAUNCHED();
   LV_CUDA(cudaMemsetAsync(&h.ctl->bad, 0, 8, s));
-  k_totals_add<<<grid_for(L.n, 256), 256, 0, s>>>(L.C, L.k, L.n, L.a, L.size, &h.ctl->bad);
+  k_totals_add<<<grid_for(L.n, 256), 256, 0, s>>>(L.ca, L.k, L.n, L.size, &h.ctl->bad);
   LV_LAUNCHED();
   unsigned long long bad = 0;
   LV_CUDA(cudaMemcpyAsync(&bad, &h.ctl->bad, 8, cudaMemcpyDeviceToHost, s));
@@ -329,6 +361,111 @@ int32_t level_set_labels(Handle& h, Level& L, const int32_t* d_labels) {
     set_error("labels out of range [0, n)");
     return LOUVAIN_E_INVALID_ARG;
   }
+  return LOUVAIN_OK;
+}
+
+int32_t level_get_labels(Handle& h, Level& L, int32_t* d_out) {
+  if (L.n == 0) return LOUVAIN_OK;
+  k_get_C<<<grid_for(L.n, 256), 256, 0, h.stream>>>(L.ca, L.n, d_out);
+  LV_LAUNCHED();
+  LV_CUDA(cudaGetLastError());
+  return LOUVAIN_OK;
+}
+
+int32_t level_get_a(Handle& h, Level& L, uint32_t* d_out) {
+  if (L.n == 0) return LOUVAIN_OK;
+  k_get_a<<<grid_for(L.n, 256), 256, 0, h.stream>>>(L.ca, L.n, d_out);
+  LV_LAUNCHED();
+  LV_CUDA(cudaGetLastError());
+  return LOUVAIN_OK;
+}
+
+// Hub plan (vertices of sub-class 5, deg >= kHubMin, of any bucket): work items
+// in hub order -- inserts (kHubChunkEdges edges each), scans (kHubScanSlots
+// slots each), final -- and a ring of table slots reused hub after hub.
+static int32_t build_hub_plan(Handle& h, Level& L) {
+  cudaStream_t s = h.stream;
+  HubPlan& P = L.hub;
+  std::vector<int32_t> hv;
+  std::vector<int64_t> hdeg, rb;
+  for (int b = 1; b <= 7; ++b) {
+    const int c = kSubPerBucket * b + 5;
+    const int64_t off = L.class_off[c], cnt = L.class_off[c + 1] - off;
+    if (cnt <= 0) continue;
+    std::vector<int32_t> v(cnt);
+    std::vector<int64_t> d(2 * cnt);
+    int64_t* dd = nullptr;
+    LV_TRY(dalloc(&dd, 2 * cnt, s));
+    k_hub_degrees<<<grid_for(cnt, 256), 256, 0, s>>>(L.bin_vertices + off, cnt, L.rowptr, dd);
+    LV_LAUNCHED();
+    LV_CUDA(cudaMemcpyAsync(v.data(), L.bin_vertices + off, 4 * cnt, cudaMemcpyDeviceToHost, s));
+    LV_CUDA(cudaMemcpyAsync(d.data(), dd, 16 * cnt, cudaMemcpyDeviceToHost, s));
+    LV_CUDA(cudaStreamSynchronize(s));
+    dfree(dd, s);
+    hv.insert(hv.end(), v.begin(), v.end());
+    hdeg.insert(hdeg.end(), d.begin(), d.begin() + cnt);
+    rb.insert(rb.end(), d.begin() + cnt, d.end());
+  }
+  P.nh = (int64_t)hv.size();
+  if (P.nh == 0) return LOUVAIN_OK;
+  std::vector<HubInfo> info(P.nh);
+  std::vector<HubItem> ins, scans;
+  std::vector<int64_t> ins_off, scan_off, wave_hub;
+  auto cap_of = [](int64_t d) { return ((2 * d + 3) / 4) * 4; };  // load <= 1/2, whole 4-slot buckets
+  int64_t seg = kHubWaveSlots;
+  for (int64_t i = 0; i < P.nh; ++i) seg = std::max(seg, cap_of(hdeg[i]));
+  int64_t acc = 0;
+  for (int64_t i = 0; i < P.nh; ++i) {
+    const int64_t cap = cap_of(hdeg[i]);
+    if (wave_hub.empty() || acc + cap > seg) {
+      wave_hub.push_back(i);
+      ins_off.push_back((int64_t)ins.size());
+      scan_off.push_back((int64_t)scans.size());
+      acc = 0;
+    }
+    HubInfo& hi = info[i];
+    hi.v = hv[i];
+    hi.cap = cap;
+    hi.off = acc;
+    acc += cap;
+    for (int64_t e = 0; e < hdeg[i]; e += kHubChunkEdges)
+      ins.push_back(HubItem{(int32_t)i, 0, rb[i] + e, rb[i] + std::min(hdeg[i], e + kHubChunkEdges)});
+    hi.scan_first = (int64_t)scans.size();
+    hi.nscan = 0;
+    for (int64_t t = 0; t < cap; t += kHubScanSlots) {
+      scans.push_back(HubItem{(int32_t)i, 0, t, std::min(cap, t + kHubScanSlots)});
+      hi.nscan++;
+    }
+  }
+  P.nwaves = (int64_t)wave_hub.size();
+  wave_hub.push_back(P.nh);
+  ins_off.push_back((int64_t)ins.size());
+  scan_off.push_back((int64_t)scans.size());
+  P.seg = seg;
+  P.nins = (int64_t)ins.size();
+  P.nscan = (int64_t)scans.size();
+  LV_TRY(dalloc(&P.ins, ins.size(), s));
+  LV_TRY(dalloc(&P.scans, scans.size(), s));
+  LV_TRY(dalloc(&P.ins_off, ins_off.size(), s));
+  LV_TRY(dalloc(&P.scan_off, scan_off.size(), s));
+  LV_TRY(dalloc(&P.wave_hub, wave_hub.size(), s));
+  LV_TRY(dalloc(&P.info, info.size(), s));
+  // one allocation: {label|e} slots then a_c words
+  LV_TRY(dmalloc(reinterpret_cast<void**>(&P.ring), 12 * (size_t)(2 * seg), s));
+  P.ring_a = reinterpret_cast<uint32_t*>(P.ring + 2 * seg);
+  LV_TRY(dmalloc(&P.partial, hub_partial_bytes() * (size_t)P.nscan, s));
+  LV_CUDA(cudaMemcpyAsync(P.ins, ins.data(), sizeof(HubItem) * ins.size(), cudaMemcpyHostToDevice, s));
+  LV_CUDA(cudaMemcpyAsync(P.scans, scans.data(), sizeof(HubItem) * scans.size(), cudaMemcpyHostToDevice, s));
+  LV_CUDA(cudaMemcpyAsync(P.ins_off, ins_off.data(), 8 * ins_off.size(), cudaMemcpyHostToDevice, s));
+  LV_CUDA(cudaMemcpyAsync(P.scan_off, scan_off.data(), 8 * scan_off.size(), cudaMemcpyHostToDevice, s));
+  LV_CUDA(cudaMemcpyAsync(P.wave_hub, wave_hub.data(), 8 * wave_hub.size(), cudaMemcpyHostToDevice, s));
+  LV_CUDA(cudaMemcpyAsync(P.info, info.data(), sizeof(HubInfo) * info.size(), cudaMemcpyHostToDevice, s));
+  k_fill_u64<<<grid_for(2 * seg, 256), 256, 0, s>>>(P.ring, 2 * seg, kEmpty);
+  LV_LAUNCHED();
+  k_fill_u32v<<<grid_for(2 * seg, 256), 256, 0, s>>>(P.ring_a, 2 * seg, 0xFFFFFFFFu);
+  LV_LAUNCHED();
+  LV_CUDA(cudaGetLastError());
+  LV_CUDA(cudaStreamSynchronize(s));  // host vectors die here
   return LOUVAIN_OK;
 }
 
@@ -353,12 +490,12 @@ int32_t level_binning(Handle& h, Level& L, const louvain_params_t& p) {
                                                 p.deg_bounds[3], p.deg_bounds[4], p.deg_bounds[5], cls, iota, hist);
     LV_LAUNCHED();
     LV_CUDA(cudaGetLastError());
-    // stable sort by class (5 bits): vertices of a class stay in ascending id order
+    // stable sort by class (6 bits): vertices of a class stay in ascending id order
     size_t tb = 0;
-    LV_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, tb, cls, cls2, iota, L.bin_vertices, n, 0, 5, s));
+    LV_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, tb, cls, cls2, iota, L.bin_vertices, n, 0, 6, s));
     void* tmp = nullptr;
     LV_TRY(dmalloc(&tmp, tb, s));
-    LV_CUDA(cub::DeviceRadixSort::SortPairs(tmp, tb, cls, cls2, iota, L.bin_vertices, n, 0, 5, s)); LV_CUB();
+    LV_CUDA(cub::DeviceRadixSort::SortPairs(tmp, tb, cls, cls2, iota, L.bin_vertices, n, 0, 6, s)); LV_CUB();
     dfree(tmp, s);
     unsigned long long hh[kNumClasses];
     LV_CUDA(cudaMemcpyAsync(hh, hist, sizeof hh, cudaMemcpyDeviceToHost, s));
@@ -366,101 +503,36 @@ int32_t level_binning(Handle& h, Level& L, const louvain_params_t& p) {
     dfree(cls, s); dfree(cls2, s); dfree(iota, s); dfree(hist, s);
     for (int c = 0; c < kNumClasses; ++c) L.class_off[c + 1] = L.class_off[c] + (int64_t)hh[c];
   }
-  // hub plan: vertices of sub-class 2 (deg >= kHubMin) of every bucket
-  HubPlan& P = L.hub;
-  std::vector<int32_t> hv;
-  std::vector<int64_t> hdeg, rb;
-  for (int b = 1; b <= 7; ++b) {
-    const int c = 4 * b + 2;
-    const int64_t off = L.class_off[c], cnt = L.class_off[c + 1] - off;
-    if (cnt <= 0) continue;
-    std::vector<int32_t> v(cnt);
-    std::vector<int64_t> d(2 * cnt);
-    int64_t* dd = nullptr;
-    LV_TRY(dalloc(&dd, 2 * cnt, s));
-    k_hub_degrees<<<grid_for(cnt, 256), 256, 0, s>>>(L.bin_vertices + off, cnt, L.rowptr, dd);
-    LV_LAUNCHED();
-    LV_CUDA(cudaMemcpyAsync(v.data(), L.bin_vertices + off, 4 * cnt, cudaMemcpyDeviceToHost, s));
-    LV_CUDA(cudaMemcpyAsync(d.data(), dd, 16 * cnt, cudaMemcpyDeviceToHost, s));
-    LV_CUDA(cudaStreamSynchronize(s));
-    dfree(dd, s);
-    hv.insert(hv.end(), v.begin(), v.end());
-    hdeg.insert(hdeg.end(), d.begin(), d.begin() + cnt);
-    rb.insert(rb.end(), d.begin() + cnt, d.end());
-  }
-  P.nh = (int64_t)hv.size();
-  if (P.nh > 0) {
-    std::vector<int64_t> off(P.nh), cap(P.nh), chunk, scan, first(P.nh + 1);
-    int64_t tot = 0;
-    for (int64_t i = 0; i < P.nh; ++i) {
-      off[i] = tot;
-      cap[i] = 2 * hdeg[i];  // load factor <= 1/2
-      tot += cap[i];
-      for (int64_t e = 0; e < hdeg[i]; e += kHubChunkEdges) {
-        chunk.push_back(i);
-        chunk.push_back(rb[i] + e);
-        chunk.push_back(rb[i] + std::min(hdeg[i], e + kHubChunkEdges));
-      }
-      first[i] = (int64_t)scan.size() / 3;
-      for (int64_t t = 0; t < cap[i]; t += kHubScanSlots) {
-        scan.push_back(i);
-        scan.push_back(t);
-        scan.push_back(std::min(cap[i], t + kHubScanSlots));
-      }
-    }
-    first[P.nh] = (int64_t)scan.size() / 3;
-    P.nchunks = (int64_t)chunk.size() / 3;
-    P.nscan = (int64_t)scan.size() / 3;
-    P.table_slots = tot;
-    LV_TRY(dalloc(&P.hub_v, P.nh, s));
-    LV_TRY(dalloc(&P.tab_off, P.nh, s));
-    LV_TRY(dalloc(&P.tab_cap, P.nh, s));
-    LV_TRY(dalloc(&P.chunk, chunk.size(), s));
-    LV_TRY(dalloc(&P.scan, scan.size(), s));
-    LV_TRY(dalloc(&P.scan_first, P.nh + 1, s));
-    LV_TRY(dalloc(&P.table, tot, s));
-    LV_TRY(dmalloc(&P.partial, hub_partial_bytes() * (size_t)P.nscan, s));
-    LV_CUDA(cudaMemcpyAsync(P.hub_v, hv.data(), 4 * P.nh, cudaMemcpyHostToDevice, s));
-    LV_CUDA(cudaMemcpyAsync(P.tab_off, off.data(), 8 * P.nh, cudaMemcpyHostToDevice, s));
-    LV_CUDA(cudaMemcpyAsync(P.tab_cap, cap.data(), 8 * P.nh, cudaMemcpyHostToDevice, s));
-    LV_CUDA(cudaMemcpyAsync(P.chunk, chunk.data(), 8 * chunk.size(), cudaMemcpyHostToDevice, s));
-    LV_CUDA(cudaMemcpyAsync(P.scan, scan.data(), 8 * scan.size(), cudaMemcpyHostToDevice, s));
-    LV_CUDA(cudaMemcpyAsync(P.scan_first, first.data(), 8 * (P.nh + 1), cudaMemcpyHostToDevice, s));
-    k_fill_u64<<<grid_for(tot, 256), 256, 0, s>>>(P.table, tot, kEmpty);
-    LV_LAUNCHED();
-    LV_CUDA(cudaGetLastError());
-    LV_CUDA(cudaStreamSynchronize(s));  // host vectors die here
-  }
+  LV_TRY(build_hub_plan(h, L));
   std::memcpy(L.bins_bounds, p.deg_bounds, sizeof L.bins_bounds);
   L.bins_valid = true;
   return LOUVAIN_OK;
 }
 
-
-// Eq. (1) parts of partition d_C into ctl->L / ctl->S (stream-ordered, no sync).
-// d_C == L.C uses the maintained a_c; any other labels get their own a_c.
+// Eq. (1) parts into ctl->L / ctl->S (stream-ordered, no sync).  d_C == nullptr:
+// the level's own partition with its maintained a_c; else an external labelling.
 int32_t launch_modularity(Handle& h, Level& L, const int32_t* d_C) {
   cudaStream_t s = h.stream;
   LV_CUDA(cudaMemsetAsync(&h.ctl->L, 0, 16, s));
   if (L.n == 0) return LOUVAIN_OK;
-  const uint32_t* a = L.a;
-  uint32_t* a_tmp = nullptr;
-  int32_t* size_tmp = nullptr;
-  if (d_C != L.C) {
-    LV_TRY(dalloc(&a_tmp, L.n, s));
-    LV_TRY(dalloc(&size_tmp, L.n, s));
-    k_totals_zero<<<grid_for(L.n, 256), 256, 0, s>>>(L.n, a_tmp, size_tmp);
-    LV_LAUNCHED();
-    k_totals_add<<<grid_for(L.n, 256), 256, 0, s>>>(d_C, L.k, L.n, a_tmp, size_tmp, &h.ctl->bad);
-    LV_LAUNCHED();
-    a = a_tmp;
-  }
   const int64_t ntiles = (L.nnz + kTileEdges - 1) / kTileEdges;
   const unsigned grid = grid_for(std::max<int64_t>(ntiles, (L.n + 255) / 256), 1, 148 * 8);
-  k_modularity<<<grid, 256, 0, s>>>(L.rowptr, L.n, L.col, L.w, d_C, a, L.nnz, &h.ctl->L, &h.ctl->S);
-  LV_LAUNCHED();
+  if (!d_C) {
+    k_modularity<true><<<grid, 256, 0, s>>>(L.rowptr, L.n, L.col, L.w, L.ca, nullptr, nullptr, L.nnz, &h.ctl->L,
+                                            &h.ctl->S);
+    LV_LAUNCHED();
+  } else {
+    uint32_t* a_tmp = nullptr;
+    LV_TRY(dalloc(&a_tmp, L.n, s));
+    LV_CUDA(cudaMemsetAsync(a_tmp, 0, 4 * L.n, s));
+    k_ext_totals<<<grid_for(L.n, 256), 256, 0, s>>>(d_C, L.k, L.n, a_tmp, &h.ctl->bad);
+    LV_LAUNCHED();
+    k_modularity<false><<<grid, 256, 0, s>>>(L.rowptr, L.n, L.col, L.w, nullptr, d_C, a_tmp, L.nnz, &h.ctl->L,
+                                             &h.ctl->S);
+    LV_LAUNCHED();
+    dfree(a_tmp, s);
+  }
   LV_CUDA(cudaGetLastError());
-  if (a_tmp) { dfree(a_tmp, s); dfree(size_tmp, s); }
   return LOUVAIN_OK;
 }
 
@@ -479,14 +551,14 @@ int32_t level_modularity(Handle& h, Level& L, const int32_t* d_C, uint64_t* Lout
 }
 
 int32_t launch_commit(Handle& h, Level& L, int bucket) {
-  k_commit<<<148 * 4, 256, 0, h.stream>>>(h.ctl, bucket, L.mv_v, L.mv_new, L.mv_old, L.C, L.a, L.size, L.k);
+  k_commit<<<148 * 4, 256, 0, h.stream>>>(h.ctl, bucket, L.mv_v, L.mv_new, L.mv_old, L.ca, L.size, L.k);
   LV_LAUNCHED();
   LV_CUDA(cudaGetLastError());
   return LOUVAIN_OK;
 }
 
 int32_t launch_revert(Handle& h, Level& L) {
-  k_revert<<<148 * 4, 256, 0, h.stream>>>(h.ctl, L.mv_v, L.mv_new, L.mv_old, L.C, L.a, L.size, L.k);
+  k_revert<<<148 * 4, 256, 0, h.stream>>>(h.ctl, L.mv_v, L.mv_new, L.mv_old, L.ca, L.size, L.k);
   LV_LAUNCHED();
   LV_CUDA(cudaGetLastError());
   return LOUVAIN_OK;
@@ -495,6 +567,14 @@ int32_t launch_revert(Handle& h, Level& L) {
 int32_t compose_labels(Handle& h, int32_t* lab, int64_t n0, const int32_t* map) {
   if (n0 == 0) return LOUVAIN_OK;
   k_compose<<<grid_for(n0, 256), 256, 0, h.stream>>>(lab, n0, map);
+  LV_LAUNCHED();
+  LV_CUDA(cudaGetLastError());
+  return LOUVAIN_OK;
+}
+
+int32_t compose_labels_ca(Handle& h, int32_t* lab, int64_t n0, const uint2* ca) {
+  if (n0 == 0) return LOUVAIN_OK;
+  k_compose_ca<<<grid_for(n0, 256), 256, 0, h.stream>>>(lab, n0, ca);
   LV_LAUNCHED();
   LV_CUDA(cudaGetLastError());
   return LOUVAIN_OK;
@@ -531,7 +611,7 @@ int32_t level_contract(Handle& h, Level& L, Level& out, int32_t* d_map) {
   LV_CUDA(cudaMemcpyAsync(&last[1], flag + n - 1, 4, cudaMemcpyDeviceToHost, s));
   LV_CUDA(cudaStreamSynchronize(s));
   const int64_t np = (int64_t)last[0] + last[1];
-  k_map<<<grid_for(n, 256), 256, 0, s>>>(L.C, newID, n, d_map);
+  k_map<<<grid_for(n, 256), 256, 0, s>>>(L.ca, newID, n, d_map);
   LV_LAUNCHED();
   dfree(flag, s);
   dfree(newID, s);

@@ -12,35 +12,48 @@
 // Moves are appended to a move log; commit is a separate kernel (lv_level.cu)
 // because the whole bucket must decide before any C/a changes.
 //
+// Memory design (the sweep is bound by random gathers):
+//  * col / w are streamed with evict-first loads (__ldcs) so they do not push
+//    the gathered vertex records out of L2;
+//  * a neighbour j is gathered as ONE 8-byte record ca[j] = {C[j], a[j]}; when
+//    j represents its own community (C[j] == j, e.g. every vertex at the first
+//    sweep of a level) a[C[j]] comes with it and the candidate's a_c needs no
+//    second gather;
+//  * edge loops are unrolled 4x so each thread has 4 independent gathers in flight.
+//
 // Kernel families (edge-level parallelism, redesigned for
 // sm_100a; SURVEY 2.3 K1-K4 counterparts):
 //   sweep_small<G>  deg <= 32: G = 4/8/16/32 lanes per vertex, one edge per
-//                   lane, duplicate labels merged in registers with
-//                   __match_any_sync + __reduce_add_sync (no shared memory).
-//   sweep_warp<CAP> deg <= 340: a warp per vertex, per-warp smem hash table
-//                   of CAP 64-bit {label|e} slots (single-CAS insert).
-//   sweep_cta       deg < 12288: a CTA per vertex (persistent loop), smem
-//                   table of min(CAPMAX, 2*deg) slots (64 KB / 128 KB).
-//   hub_*           deg >= 12288: one vertex split over many CTAs (chunks of
-//                   8192 edges) inserting into a global-memory table, then a
-//                   chunked table scan and a per-hub final reduction.
+//                   lane, labels merged in registers with __match_any_sync +
+//                   __reduce_add_sync (no shared memory).
+//   sweep_warp<CAP> deg <= 340: a warp per vertex, per-warp smem hash table.
+//   sweep_cta       deg < 12288: a CTA per vertex (persistent loop), smem table.
+//   hub_coop        deg >= 12288: one vertex split over many CTAs; a cooperative
+//                   kernel pipelines waves of hubs (insert chunks -> table scan
+//                   chunks -> decision) across grid.sync() phases, the global
+//                   tables living in a 2-segment ring small enough for L2.
+#include <cooperative_groups.h>
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <cstdlib>
 
 #include "lv_device.cuh"
 #include "lv_internal.cuh"
 
+namespace cg = cooperative_groups;
+
 namespace lv {
 namespace {
+
+constexpr uint32_t kUnknownA = 0xFFFFFFFFu;  // a_c < W <= 3,037,000,499 < 2^32 - 1
 
 struct SweepArgs {
   const int64_t* rowptr;
   const int32_t* col;
   const uint32_t* w;
   const uint32_t* k;
-  const int32_t* C;
-  const uint32_t* a;
+  const uint2* ca;
   const int32_t* size;
   long long W;
   int rule;
@@ -49,7 +62,7 @@ struct SweepArgs {
   unsigned long long* logn;
 };
 
-struct Partial {
+struct __align__(16) Partial {
   long long s;
   int c;
   unsigned eown;
@@ -77,21 +90,21 @@ __device__ __forceinline__ void log_moves(bool mv, int32_t v, int32_t t, const S
   }
 }
 
-// Candidate c (!= own) with accumulated weight e: fold into (s, cb).
-__device__ __forceinline__ void consider(int32_t c, uint32_t e, int32_t own, bool own_single, uint32_t ki,
-                                         const SweepArgs& A, long long& s, int& cb) {
-  if (A.rule == 2 && own_single && c > own && A.size[c] == 1) return;  // R8 'filter' reading
-  long long sc = A.W * (long long)e - (long long)ki * (long long)A.a[c];
+// Candidate c (!= own) with accumulated weight e and total a_c: fold into (s, cb).
+__device__ __forceinline__ void consider(int32_t c, uint32_t e, uint32_t ac, int32_t own, bool own_single,
+                                         uint32_t ki, const SweepArgs& A, long long& s, int& cb) {
+  if (A.rule == 2 && own_single && c > own && __ldg(&A.size[c]) == 1) return;  // R8 'filter' reading
+  const long long sc = A.W * (long long)e - (long long)ki * (long long)ac;
   if (better(sc, c, s, cb)) { s = sc; cb = c; }
 }
 
 // Stay test and singleton veto.
-__device__ __forceinline__ int32_t finish(long long s, int cb, uint32_t eown, int32_t own, uint32_t ki,
-                                          const SweepArgs& A) {
+__device__ __forceinline__ int32_t finish(long long s, int cb, uint32_t eown, int32_t own, uint32_t a_own,
+                                          uint32_t ki, const SweepArgs& A) {
   if (cb == 0x7FFFFFFF) return own;
-  long long sstay = A.W * (long long)eown - (long long)ki * ((long long)A.a[own] - (long long)ki);
+  const long long sstay = A.W * (long long)eown - (long long)ki * ((long long)a_own - (long long)ki);
   if (s <= sstay) return own;
-  if (A.rule == 1 && cb > own && A.size[own] == 1 && A.size[cb] == 1) return own;  // R8 veto
+  if (A.rule == 1 && cb > own && __ldg(&A.size[own]) == 1 && __ldg(&A.size[cb]) == 1) return own;  // R8 veto
   return cb;
 }
 
@@ -113,192 +126,529 @@ __global__ void __launch_bounds__(256) sweep_small(const int32_t* __restrict__ v
       v = __ldg(&verts[vi]);
       rb = __ldg(&A.rowptr[v]);
       deg = (int32_t)(__ldg(&A.rowptr[v + 1]) - rb);
-      own = A.C[v];
+      own = (int32_t)__ldg(&A.ca[v]).x;
       ki = __ldg(&A.k[v]);
     }
     const bool has = sub < deg;
-    int32_t j = has ? __ldg(&A.col[rb + sub]) : -1;
-    uint32_t we = UNIT ? 1u : (has ? __ldg(&A.w[rb + sub]) : 0u);
+    const int32_t j = has ? __ldcs(&A.col[rb + sub]) : -1;
+    const uint32_t we = UNIT ? 1u : (has ? __ldcs(&A.w[rb + sub]) : 0u);
     const bool valid = has && j != v;  // R3: the self-loop does not count in e
-    const int32_t c = valid ? A.C[j] : (int32_t)(0x80000000u | (unsigned)lane);
+    uint2 rec = make_uint2(0, 0);
+    if (valid) rec = __ldg(&A.ca[j]);
+    const int32_t c = valid ? (int32_t)rec.x : (int32_t)(0x80000000u | (unsigned)lane);
     const unsigned m = __match_any_sync(kFull, c) & gmask;
     const uint32_t e = UNIT ? (uint32_t)__popc(m) : __reduce_add_sync(m, we);
+    // a lane whose neighbour represents the label (j == c) already holds a_c
+    const unsigned rep = __ballot_sync(kFull, valid && j == c) & m;
+    const uint32_t a_rep = __shfl_sync(kFull, rec.y, rep ? __ffs(rep) - 1 : lane);
     long long s = (long long)0x8000000000000000ull;
     int cb = 0x7FFFFFFF;
     unsigned eown = 0;
     if (valid && lane == __ffs(m) - 1) {
-      if (c == own) eown = e;
-      else consider(c, e, own, A.rule == 2 && active && A.size[own] == 1, ki, A, s, cb);
+      if (c == own) {
+        eown = e;
+      } else {
+        const uint32_t ac = rep ? a_rep : __ldg(&A.ca[c]).y;
+        consider(c, e, ac, own, A.rule == 2 && __ldg(&A.size[own]) == 1, ki, A, s, cb);
+      }
     }
     group_reduce<G>(s, cb, eown);
     int32_t t = own;
-    if (active && sub == 0) t = finish(s, cb, eown, own, ki, A);
+    if (active && sub == 0 && cb != 0x7FFFFFFF) t = finish(s, cb, eown, own, __ldg(&A.ca[own]).y, ki, A);
     log_moves(active && sub == 0 && t != own, v, t, A);
   }
 }
 
+// Table scan shared by the warp and CTA kernels: slots [t0, cap) step `stride`.
+// Clears every visited slot for the next vertex.  4 slots per pass so the a_c
+// gathers of labels without a representative in the row overlap.
+__device__ __forceinline__ void scan_table(unsigned long long* T, uint32_t* TA, uint32_t cap, uint32_t t0,
+                                           uint32_t stride, int32_t own, bool own_single, uint32_t ki,
+                                           const SweepArgs& A, long long& s, int& cb, unsigned& eown) {
+  for (uint32_t base = t0; base < cap; base += 4 * stride) {
+    unsigned long long x[4];
+    uint32_t ac[4];
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      const uint32_t t = base + q * stride;
+      x[q] = kEmpty;
+      ac[q] = kUnknownA;
+      if (t < cap) {
+        x[q] = T[t];
+        if (x[q] != kEmpty) {
+          ac[q] = TA[t];
+          T[t] = kEmpty;
+          TA[t] = kUnknownA;
+        }
+      }
+    }
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      if (x[q] != kEmpty && ac[q] == kUnknownA && (int32_t)(x[q] >> 32) != own)
+        ac[q] = __ldg(&A.ca[(int32_t)(x[q] >> 32)]).y;
+    }
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      if (x[q] == kEmpty) continue;
+      const int32_t c = (int32_t)(x[q] >> 32);
+      const uint32_t e = (uint32_t)x[q];
+      if (c == own) eown = e;
+      else consider(c, e, ac[q], own, own_single, ki, A, s, cb);
+    }
+  }
+}
+
+// Sequential insert into a shared-memory table (CAS latency is short there):
+// one CAS claims an empty slot with the value already in it; a slot already
+// holding c gets an atomic add on its low word (e <= W < 2^32, no carry).
+__device__ __forceinline__ uint32_t table_insert(unsigned long long* T, uint32_t cap, int32_t c, uint32_t x) {
+  const unsigned long long key = ((unsigned long long)(uint32_t)c) << 32;
+  uint32_t h = hash_slot(c, cap);
+  for (;;) {
+    const unsigned long long old = atomicCAS(&T[h], kEmpty, key | x);
+    if (old == kEmpty) return h;
+    if ((old >> 32) == (unsigned long long)(uint32_t)c) {
+      atomicAdd(&T[h], (unsigned long long)x);
+      return h;
+    }
+    h = (h + 1 == cap) ? 0 : h + 1;
+  }
+}
+
+// Global-memory (hub) variant: the table is split into 4-slot buckets (32 B,
+// one sector).  Each round reads a thread's bucket with two 16-byte L2 loads,
+// adds into the slot holding c, or CASes the first empty slot; a failed CAS
+// re-reads the same bucket, a full bucket moves to the next.  Slots only go
+// EMPTY -> key once, and a key is only claimed at the first empty slot of its
+// probe sequence, so no label is ever inserted twice.  One L2 round trip per
+// insert at load factor <= 1/2 instead of ~(1 + 1/(1-a)^2)/2 dependent CASes.
+__device__ __forceinline__ void gtable_insert4(unsigned long long* T, uint32_t* TA, uint32_t cap, const int32_t c[4],
+                                               const uint32_t x[4], bool todo[4], const uint32_t arep[4]) {
+  const uint32_t nb = cap >> 2;
+  uint32_t b[4];
+#pragma unroll
+  for (int q = 0; q < 4; ++q) b[q] = todo[q] ? (hash_slot(c[q], nb) << 2) : 0u;
+  while (todo[0] || todo[1] || todo[2] || todo[3]) {
+    unsigned long long k[4][4];
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      if (!todo[q]) continue;
+      const ulonglong2 lo = __ldcg(reinterpret_cast<const ulonglong2*>(&T[b[q]]));
+      const ulonglong2 hi = __ldcg(reinterpret_cast<const ulonglong2*>(&T[b[q] + 2]));
+      k[q][0] = lo.x; k[q][1] = lo.y; k[q][2] = hi.x; k[q][3] = hi.y;
+    }
+    int tgt[4];
+    bool found[4];
+    unsigned long long old[4];
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      tgt[q] = -1;
+      found[q] = false;
+      old[q] = 0;
+      if (!todo[q]) continue;
+#pragma unroll
+      for (int u = 3; u >= 0; --u) {
+        if (k[q][u] == kEmpty) tgt[q] = u;  // first empty slot
+      }
+#pragma unroll
+      for (int u = 3; u >= 0; --u) {
+        if (k[q][u] != kEmpty && (k[q][u] >> 32) == (unsigned long long)(uint32_t)c[q]) {
+          tgt[q] = u;
+          found[q] = true;
+        }
+      }
+    }
+#pragma unroll
+    for (int q = 0; q < 4; ++q)
+      if (todo[q] && !found[q] && tgt[q] >= 0)
+        old[q] = atomicCAS(&T[b[q] + tgt[q]], kEmpty, (((unsigned long long)(uint32_t)c[q]) << 32) | x[q]);
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      if (!todo[q]) continue;
+      if (found[q]) {
+        atomicAdd(&T[b[q] + tgt[q]], (unsigned long long)x[q]);
+      } else if (tgt[q] >= 0) {
+        if (old[q] != kEmpty) {
+          if ((old[q] >> 32) != (unsigned long long)(uint32_t)c[q]) continue;  // lost the race: re-read bucket
+          atomicAdd(&T[b[q] + tgt[q]], (unsigned long long)x[q]);
+        }
+      } else {
+        b[q] = (b[q] + 4 >= cap) ? 0u : b[q] + 4;  // bucket full
+        continue;
+      }
+      if (arep[q] != kUnknownA) TA[b[q] + tgt[q]] = arep[q];
+      todo[q] = false;
+    }
+  }
+}
+
+// Inserts entries [t0, deg) step `stride` of the row starting at rb (vertex v),
+// 4 per pass: 4 col loads, then 4 independent record gathers, then 4
+// interleaved inserts.  With AGG, labels are first merged across the warp
+// (__match_any_sync, weights summed with __reduce_add_sync), so a label shared
+// by many neighbours costs one table atomic per warp instead of one per edge.
+// The trip count is uniform across each warp, as the warp intrinsics require.
+template <bool UNIT, bool AGG, bool GLOBAL = false>
+__device__ __forceinline__ void insert_row(unsigned long long* T, uint32_t* TA, uint32_t cap, int32_t v, int64_t rb,
+                                           int64_t deg, int64_t t0, int64_t stride, const SweepArgs& A) {
+  const int lane = threadIdx.x & 31;
+  const int64_t t_warp0 = t0 - lane;  // first index handled by the warp in each pass
+  for (int64_t base = 0; base + t_warp0 < deg; base += 4 * stride) {
+    int32_t jj[4];
+    uint32_t ww[4];
+    uint2 rr[4];
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      const int64_t t = base + t0 + q * stride;
+      jj[q] = (t < deg) ? __ldcs(&A.col[rb + t]) : -1;
+      ww[q] = UNIT ? 1u : ((t < deg) ? __ldcs(&A.w[rb + t]) : 0u);
+    }
+#pragma unroll
+    for (int q = 0; q < 4; ++q) rr[q] = (jj[q] >= 0 && jj[q] != v) ? __ldg(&A.ca[jj[q]]) : make_uint2(0, 0);
+    int32_t c[4];
+    uint32_t x[4], arep[4];
+    bool todo[4];
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      const bool valid = jj[q] >= 0 && jj[q] != v;
+      const bool isrep = valid && (uint32_t)jj[q] == rr[q].x;
+      c[q] = valid ? (int32_t)rr[q].x : (int32_t)(0x80000000u | (unsigned)lane);
+      if (AGG) {
+        const unsigned m = __match_any_sync(kFull, c[q]);
+        x[q] = UNIT ? (uint32_t)__popc(m) : __reduce_add_sync(m, ww[q]);
+        const unsigned rep = __ballot_sync(kFull, isrep) & m;
+        const uint32_t a_rep = __shfl_sync(kFull, rr[q].y, rep ? __ffs(rep) - 1 : lane);
+        todo[q] = valid && lane == __ffs(m) - 1;
+        arep[q] = rep ? a_rep : kUnknownA;
+      } else {
+        x[q] = ww[q];
+        todo[q] = valid;
+        arep[q] = isrep ? rr[q].y : kUnknownA;
+      }
+    }
+    if (GLOBAL) {
+      gtable_insert4(T, TA, cap, c, x, todo, arep);
+    } else {
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        if (!todo[q]) continue;
+        const uint32_t hq = table_insert(T, cap, c[q], x[q]);
+        if (arep[q] != kUnknownA) TA[hq] = arep[q];
+      }
+    }
+  }
+}
+
 // ------------------------------------------------------------ warp per vertex
-template <int CAP, bool UNIT>
-__global__ void __launch_bounds__(256) sweep_warp(const int32_t* __restrict__ verts, int64_t nv, SweepArgs A) {
-  __shared__ unsigned long long tab[8][CAP];
+template <int CAP, int WARPS, bool UNIT, bool AGG>
+__global__ void __launch_bounds__(32 * WARPS) sweep_warp(const int32_t* __restrict__ verts, int64_t nv, SweepArgs A) {
+  __shared__ unsigned long long tab[WARPS][CAP];
+  __shared__ uint32_t taba[WARPS][CAP];
   const int lane = threadIdx.x & 31, wl = threadIdx.x >> 5;
   unsigned long long* T = tab[wl];
-  for (int t = lane; t < CAP; t += 32) T[t] = kEmpty;
+  uint32_t* TA = taba[wl];
+  for (int t = lane; t < CAP; t += 32) {
+    T[t] = kEmpty;
+    TA[t] = kUnknownA;
+  }
   __syncwarp();
-  const int64_t warps = (int64_t)gridDim.x * 8;
-  for (int64_t vi = (int64_t)blockIdx.x * 8 + wl; vi < nv; vi += warps) {
+  const int64_t warps = (int64_t)gridDim.x * WARPS;
+  for (int64_t vi = (int64_t)blockIdx.x * WARPS + wl; vi < nv; vi += warps) {
     const int32_t v = __ldg(&verts[vi]);
     const int64_t rb = __ldg(&A.rowptr[v]);
-    const int32_t deg = (int32_t)(__ldg(&A.rowptr[v + 1]) - rb);
-    const int32_t own = A.C[v];
+    const int64_t deg = __ldg(&A.rowptr[v + 1]) - rb;
+    const int32_t own = (int32_t)__ldg(&A.ca[v]).x;
     const uint32_t ki = __ldg(&A.k[v]);
-    for (int32_t t = lane; t < deg; t += 32) {
-      const int32_t j = __ldg(&A.col[rb + t]);
-      if (j == v) continue;
-      table_add(T, CAP, A.C[j], UNIT ? 1u : __ldg(&A.w[rb + t]));
-    }
+    insert_row<UNIT, AGG>(T, TA, CAP, v, rb, deg, lane, 32, A);
     __syncwarp();
-    const bool own_single = A.rule == 2 && A.size[own] == 1;
+    const bool own_single = A.rule == 2 && __ldg(&A.size[own]) == 1;
     long long s = (long long)0x8000000000000000ull;
     int cb = 0x7FFFFFFF;
     unsigned eown = 0;
-    for (int t = lane; t < CAP; t += 32) {
-      const unsigned long long x = T[t];
-      if (x == kEmpty) continue;
-      T[t] = kEmpty;
-      const int32_t c = (int32_t)(x >> 32);
-      const uint32_t e = (uint32_t)x;
-      if (c == own) eown = e;
-      else consider(c, e, own, own_single, ki, A, s, cb);
-    }
+    scan_table(T, TA, CAP, lane, 32, own, own_single, ki, A, s, cb, eown);
     group_reduce<32>(s, cb, eown);
-    const int32_t tgt = (lane == 0) ? finish(s, cb, eown, own, ki, A) : own;
+    int32_t tgt = own;
+    if (lane == 0) tgt = finish(s, cb, eown, own, __ldg(&A.ca[own]).y, ki, A);
     log_moves(lane == 0 && tgt != own, v, tgt, A);
     __syncwarp();
   }
 }
 
 // ------------------------------------------------------------ CTA per vertex
-template <bool UNIT>
-__global__ void __launch_bounds__(1024) sweep_cta(const int32_t* __restrict__ verts, int64_t nv, SweepArgs A, int capmax) {
-  extern __shared__ unsigned long long T[];
+template <bool UNIT, bool AGG>
+__global__ void __launch_bounds__(1024) sweep_cta(const int32_t* __restrict__ verts, int64_t nv, SweepArgs A,
+                                                  int capmax) {
+  extern __shared__ unsigned long long smem[];
+  unsigned long long* T = smem;
+  uint32_t* TA = reinterpret_cast<uint32_t*>(smem + capmax);
   __shared__ long long sh_s[32];
   __shared__ int sh_c[32];
   __shared__ unsigned sh_e[32];
-  for (int t = threadIdx.x; t < capmax; t += blockDim.x) T[t] = kEmpty;
+  for (int t = threadIdx.x; t < capmax; t += blockDim.x) {
+    T[t] = kEmpty;
+    TA[t] = kUnknownA;
+  }
   __syncthreads();
   for (int64_t vi = blockIdx.x; vi < nv; vi += gridDim.x) {
     const int32_t v = __ldg(&verts[vi]);
     const int64_t rb = __ldg(&A.rowptr[v]);
     const int64_t deg = __ldg(&A.rowptr[v + 1]) - rb;
-    const int32_t own = A.C[v];
+    const int32_t own = (int32_t)__ldg(&A.ca[v]).x;
     const uint32_t ki = __ldg(&A.k[v]);
     const uint32_t cap = (uint32_t)((2 * deg < (int64_t)capmax) ? 2 * deg : (int64_t)capmax);
-    for (int64_t t = threadIdx.x; t < deg; t += blockDim.x) {
-      const int32_t j = __ldg(&A.col[rb + t]);
-      if (j == v) continue;
-      table_add(T, cap, A.C[j], UNIT ? 1u : __ldg(&A.w[rb + t]));
-    }
+    insert_row<UNIT, AGG>(T, TA, cap, v, rb, deg, threadIdx.x, blockDim.x, A);
     __syncthreads();
-    const bool own_single = A.rule == 2 && A.size[own] == 1;
+    const bool own_single = A.rule == 2 && __ldg(&A.size[own]) == 1;
     long long s = (long long)0x8000000000000000ull;
     int cb = 0x7FFFFFFF;
     unsigned eown = 0;
-    for (uint32_t t = threadIdx.x; t < cap; t += blockDim.x) {
-      const unsigned long long x = T[t];
-      if (x == kEmpty) continue;
-      T[t] = kEmpty;
-      const int32_t c = (int32_t)(x >> 32);
-      const uint32_t e = (uint32_t)x;
-      if (c == own) eown = e;
-      else consider(c, e, own, own_single, ki, A, s, cb);
-    }
+    scan_table(T, TA, cap, threadIdx.x, blockDim.x, own, own_single, ki, A, s, cb, eown);
     block_reduce(s, cb, eown, sh_s, sh_c, sh_e);
     if (threadIdx.x < 32) {
-      const int32_t tgt = (threadIdx.x == 0) ? finish(s, cb, eown, own, ki, A) : own;
+      int32_t tgt = own;
+      if (threadIdx.x == 0) tgt = finish(s, cb, eown, own, __ldg(&A.ca[own]).y, ki, A);
       log_moves(threadIdx.x == 0 && tgt != own, v, tgt, A);
     }
     __syncthreads();
   }
 }
 
-// ------------------------------------------------------------ hubs
-template <bool UNIT>
-__global__ void __launch_bounds__(512) hub_insert(const int64_t* __restrict__ chunk, int64_t nchunks,
-                                                  const int32_t* __restrict__ hub_v,
-                                                  const int64_t* __restrict__ tab_off,
-                                                  const int64_t* __restrict__ tab_cap,
-                                                  unsigned long long* table, SweepArgs A) {
-  for (int64_t q = blockIdx.x; q < nchunks; q += gridDim.x) {
-    const int64_t hidx = chunk[3 * q], eb = chunk[3 * q + 1], ee = chunk[3 * q + 2];
-    const int32_t v = hub_v[hidx];
-    unsigned long long* T = table + tab_off[hidx];
-    const uint32_t cap = (uint32_t)tab_cap[hidx];
-    for (int64_t e = eb + threadIdx.x; e < ee; e += blockDim.x) {
-      const int32_t j = __ldg(&A.col[e]);
-      if (j == v) continue;
-      table_add(T, cap, A.C[j], UNIT ? 1u : __ldg(&A.w[e]));
+// ------------------------------------------------------------ cluster per vertex
+// deg in [12288, 131072): the vertex's table (2*deg slots, load <= 1/2) is
+// spread over the distributed shared memory of a CS-CTA cluster (kClusterSlots
+// per CTA).  Each CTA inserts its share of the row into whichever CTA owns the
+// slot (remote DSMEM CAS, ~200 cycles); cluster.sync(); each CTA scans its own
+// slots; partials meet in rank 0's shared memory; cluster.sync(); rank 0 decides.
+// Persistent: clusters stride over the class's vertices.
+__device__ __forceinline__ void dsm_insert4(cg::cluster_group& cl, unsigned long long* T, uint32_t* TA, uint32_t cap,
+                                            const int32_t c[4], const uint32_t x[4], bool todo[4],
+                                            const uint32_t arep[4]) {
+  uint32_t h[4];
+#pragma unroll
+  for (int q = 0; q < 4; ++q) h[q] = todo[q] ? hash_slot(c[q], cap) : 0u;
+  while (todo[0] || todo[1] || todo[2] || todo[3]) {
+    unsigned long long old[4];
+    unsigned long long* slot[4];
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      slot[q] = cl.map_shared_rank(T + (h[q] % kClusterSlots), h[q] / kClusterSlots);
+      old[q] = todo[q] ? atomicCAS(slot[q], kEmpty, (((unsigned long long)(uint32_t)c[q]) << 32) | x[q]) : 0ull;
+    }
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      if (!todo[q]) continue;
+      if (old[q] == kEmpty || (old[q] >> 32) == (unsigned long long)(uint32_t)c[q]) {
+        if (old[q] != kEmpty) atomicAdd(slot[q], (unsigned long long)x[q]);
+        if (arep[q] != kUnknownA) *cl.map_shared_rank(TA + (h[q] % kClusterSlots), h[q] / kClusterSlots) = arep[q];
+        todo[q] = false;
+      } else {
+        h[q] = (h[q] + 1 == cap) ? 0 : h[q] + 1;
+      }
     }
   }
 }
 
-__global__ void __launch_bounds__(512) hub_scan(const int64_t* __restrict__ scan, int64_t nscan,
-                                                const int32_t* __restrict__ hub_v,
-                                                const int64_t* __restrict__ tab_off, unsigned long long* table,
-                                                Partial* part, SweepArgs A) {
+template <bool UNIT>
+__global__ void __launch_bounds__(1024, 1) sweep_cluster(const int32_t* __restrict__ verts, int64_t nv, SweepArgs A) {
+  cg::cluster_group cl = cg::this_cluster();
+  extern __shared__ unsigned long long smem[];
+  unsigned long long* T = smem;
+  uint32_t* TA = reinterpret_cast<uint32_t*>(smem + kClusterSlots);
   __shared__ long long sh_s[32];
   __shared__ int sh_c[32];
   __shared__ unsigned sh_e[32];
-  for (int64_t q = blockIdx.x; q < nscan; q += gridDim.x) {
-    const int64_t hidx = scan[3 * q], sb = scan[3 * q + 1], se = scan[3 * q + 2];
-    const int32_t v = hub_v[hidx];
-    const int32_t own = A.C[v];
-    const uint32_t ki = A.k[v];
-    const bool own_single = A.rule == 2 && A.size[own] == 1;
-    unsigned long long* T = table + tab_off[hidx];
+  __shared__ Partial cpart[16];
+  const unsigned CS = cl.num_blocks();
+  const unsigned rank = cl.block_rank();
+  for (int t = threadIdx.x; t < kClusterSlots; t += blockDim.x) {
+    T[t] = kEmpty;
+    TA[t] = kUnknownA;
+  }
+  cl.sync();
+  const int64_t ncl = gridDim.x / CS, cid = blockIdx.x / CS;
+  for (int64_t vi = cid; vi < nv; vi += ncl) {
+    const int32_t v = __ldg(&verts[vi]);
+    const int64_t rb = __ldg(&A.rowptr[v]);
+    const int64_t deg = __ldg(&A.rowptr[v + 1]) - rb;
+    const int32_t own = (int32_t)__ldg(&A.ca[v]).x;
+    const uint32_t ki = __ldg(&A.k[v]);
+    const uint32_t cap = (uint32_t)(2 * deg);  // <= CS * kClusterSlots by class bounds
+    // this CTA's share of the row
+    const int64_t per = (deg + CS - 1) / CS;
+    const int64_t eb = rb + (int64_t)rank * per;
+    const int64_t len = max((int64_t)0, min(per, rb + deg - eb));
+    const int lane = threadIdx.x & 31;
+    for (int64_t base = 0; base + (int64_t)(threadIdx.x - lane) < len; base += 4 * (int64_t)blockDim.x) {
+      int32_t jj[4];
+      uint32_t ww[4];
+      uint2 rr[4];
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        const int64_t t = base + threadIdx.x + (int64_t)q * blockDim.x;
+        jj[q] = (t < len) ? __ldcs(&A.col[eb + t]) : -1;
+        ww[q] = UNIT ? 1u : ((t < len) ? __ldcs(&A.w[eb + t]) : 0u);
+      }
+#pragma unroll
+      for (int q = 0; q < 4; ++q) rr[q] = (jj[q] >= 0 && jj[q] != v) ? __ldg(&A.ca[jj[q]]) : make_uint2(0, 0);
+      int32_t c[4];
+      uint32_t x[4], arep[4];
+      bool todo[4];
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        const bool valid = jj[q] >= 0 && jj[q] != v;
+        const bool isrep = valid && (uint32_t)jj[q] == rr[q].x;
+        c[q] = valid ? (int32_t)rr[q].x : (int32_t)(0x80000000u | (unsigned)lane);
+        const unsigned m = __match_any_sync(kFull, c[q]);
+        x[q] = UNIT ? (uint32_t)__popc(m) : __reduce_add_sync(m, ww[q]);
+        const unsigned rep = __ballot_sync(kFull, isrep) & m;
+        const uint32_t a_rep = __shfl_sync(kFull, rr[q].y, rep ? __ffs(rep) - 1 : lane);
+        todo[q] = valid && lane == __ffs(m) - 1;
+        arep[q] = rep ? a_rep : kUnknownA;
+      }
+      dsm_insert4(cl, T, TA, cap, c, x, todo, arep);
+    }
+    cl.sync();
+    // scan this CTA's slots of the table
+    const int64_t my_lo = (int64_t)rank * kClusterSlots;
+    const uint32_t my_n = (uint32_t)max((int64_t)0, min((int64_t)kClusterSlots, (int64_t)cap - my_lo));
+    const bool own_single = A.rule == 2 && __ldg(&A.size[own]) == 1;
     long long s = (long long)0x8000000000000000ull;
     int cb = 0x7FFFFFFF;
     unsigned eown = 0;
-    for (int64_t t = sb + threadIdx.x; t < se; t += blockDim.x) {
-      const unsigned long long x = T[t];
-      if (x == kEmpty) continue;
-      T[t] = kEmpty;  // leave the table clean for the next sweep
-      const int32_t c = (int32_t)(x >> 32);
-      const uint32_t e = (uint32_t)x;
-      if (c == own) eown = e;
-      else consider(c, e, own, own_single, ki, A, s, cb);
-    }
+    scan_table(T, TA, my_n, threadIdx.x, blockDim.x, own, own_single, ki, A, s, cb, eown);
     block_reduce(s, cb, eown, sh_s, sh_c, sh_e);
-    if (threadIdx.x == 0) part[q] = Partial{s, cb, eown};
-    __syncthreads();
-  }
-}
-
-__global__ void hub_final(int64_t nh, const int64_t* __restrict__ scan_first, const Partial* __restrict__ part,
-                          const int32_t* __restrict__ hub_v, SweepArgs A) {
-  const int lane = threadIdx.x & 31;
-  const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
-  for (int64_t hidx = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); hidx < nh; hidx += warps) {
-    long long s = (long long)0x8000000000000000ull;
-    int cb = 0x7FFFFFFF;
-    unsigned eown = 0;
-    for (int64_t q = scan_first[hidx] + lane; q < scan_first[hidx + 1]; q += 32) {
-      Partial p = part[q];
-      if (better(p.s, p.c, s, cb)) { s = p.s; cb = p.c; }
-      eown += p.eown;
+    if (threadIdx.x == 0) *cl.map_shared_rank(&cpart[rank], 0) = Partial{s, cb, eown};
+    cl.sync();
+    if (rank == 0 && threadIdx.x < 32) {
+      s = (long long)0x8000000000000000ull;
+      cb = 0x7FFFFFFF;
+      eown = 0;
+      if (threadIdx.x < CS) {
+        const Partial p = cpart[threadIdx.x];
+        s = p.s;
+        cb = p.c;
+        eown = p.eown;
+      }
+      group_reduce<32>(s, cb, eown);
+      int32_t tgt = own;
+      if (threadIdx.x == 0) tgt = finish(s, cb, eown, own, __ldg(&A.ca[own]).y, ki, A);
+      log_moves(threadIdx.x == 0 && tgt != own, v, tgt, A);
     }
-    group_reduce<32>(s, cb, eown);
-    const int32_t v = hub_v[hidx];
-    const int32_t own = A.C[v];
-    const int32_t tgt = (lane == 0) ? finish(s, cb, eown, own, A.k[v], A) : own;
-    log_moves(lane == 0 && tgt != own, v, tgt, A);
   }
 }
 
+// ------------------------------------------------------------ hubs
+// Cooperative kernel over the level's hub plan (lv_internal.cuh HubPlan).
+// Phase p: inserts of wave p (ring segment p % 2), table scans of wave p-1
+// (segment (p-1) % 2, left clean for wave p+1), decisions of wave p-2 (one
+// warp per hub reducing its scan partials).  grid.sync() between phases orders
+// everything; all CTAs are co-resident (cooperative launch).
 template <bool UNIT>
+__global__ void __launch_bounds__(512) hub_coop(const HubItem* __restrict__ ins, const int64_t* __restrict__ ins_off,
+                                                const HubItem* __restrict__ scans,
+                                                const int64_t* __restrict__ scan_off,
+                                                const int64_t* __restrict__ wave_hub,
+                                                const HubInfo* __restrict__ info, int64_t nwaves, int64_t seg,
+                                                unsigned long long* ring, uint32_t* ring_a, Partial* part,
+                                                SweepArgs A) {
+  cg::grid_group grid = cg::this_grid();
+  __shared__ long long sh_s[32];
+  __shared__ int sh_c[32];
+  __shared__ unsigned sh_e[32];
+  const int wpb = blockDim.x >> 5;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  for (int64_t p = 0; p < nwaves + 2; ++p) {
+    const int64_t nI = (p < nwaves) ? ins_off[p + 1] - ins_off[p] : 0;
+    const int64_t nS = (p >= 1 && p - 1 < nwaves) ? scan_off[p] - scan_off[p - 1] : 0;
+    const int64_t nFh = (p >= 2) ? wave_hub[p - 1] - wave_hub[p - 2] : 0;
+    const int64_t nF = (nFh + wpb - 1) / wpb;
+    for (int64_t it = blockIdx.x; it < nI + nS + nF; it += gridDim.x) {
+      if (it < nI) {
+        const HubItem item = ins[ins_off[p] + it];
+        const HubInfo hi = info[item.hub];
+        unsigned long long* T = ring + (p & 1) * seg + hi.off;
+        uint32_t* TA = ring_a + (p & 1) * seg + hi.off;
+        insert_row<UNIT, true, true>(T, TA, (uint32_t)hi.cap, hi.v, item.begin, item.end - item.begin, threadIdx.x,
+                                     blockDim.x, A);
+      } else if (it < nI + nS) {
+        const int64_t q = scan_off[p - 1] + (it - nI);
+        const HubItem item = scans[q];
+        const HubInfo hi = info[item.hub];
+        unsigned long long* T = ring + ((p - 1) & 1) * seg + hi.off;
+        uint32_t* TA = ring_a + ((p - 1) & 1) * seg + hi.off;
+        const int32_t own = (int32_t)__ldg(&A.ca[hi.v]).x;
+        const uint32_t ki = __ldg(&A.k[hi.v]);
+        const bool own_single = A.rule == 2 && __ldg(&A.size[own]) == 1;
+        long long s = (long long)0x8000000000000000ull;
+        int cb = 0x7FFFFFFF;
+        unsigned eown = 0;
+        for (int64_t base = item.begin + threadIdx.x; base < item.end; base += 4 * (int64_t)blockDim.x) {
+          unsigned long long x[4];
+          uint32_t ac[4];
+#pragma unroll
+          for (int u = 0; u < 4; ++u) {
+            const int64_t t = base + (int64_t)u * blockDim.x;
+            x[u] = kEmpty;
+            ac[u] = kUnknownA;
+            if (t < item.end) {
+              x[u] = __ldcg(&T[t]);
+              if (x[u] != kEmpty) {
+                ac[u] = __ldcg(&TA[t]);
+                T[t] = kEmpty;  // clean for wave p+1, which reuses this segment
+                TA[t] = kUnknownA;
+              }
+            }
+          }
+#pragma unroll
+          for (int u = 0; u < 4; ++u)
+            if (x[u] != kEmpty && ac[u] == kUnknownA && (int32_t)(x[u] >> 32) != own)
+              ac[u] = __ldg(&A.ca[(int32_t)(x[u] >> 32)]).y;
+#pragma unroll
+          for (int u = 0; u < 4; ++u) {
+            if (x[u] == kEmpty) continue;
+            const int32_t c = (int32_t)(x[u] >> 32);
+            const uint32_t e = (uint32_t)x[u];
+            if (c == own) eown = e;
+            else consider(c, e, ac[u], own, own_single, ki, A, s, cb);
+          }
+        }
+        block_reduce(s, cb, eown, sh_s, sh_c, sh_e);
+        if (threadIdx.x == 0) part[q] = Partial{s, cb, eown};
+        __syncthreads();
+      } else {
+        const int64_t hub = wave_hub[p - 2] + (it - nI - nS) * wpb + warp;
+        if (hub < wave_hub[p - 1]) {  // warp-uniform
+          const HubInfo hi = info[hub];
+          long long s = (long long)0x8000000000000000ull;
+          int cb = 0x7FFFFFFF;
+          unsigned eown = 0;
+          for (int q = lane; q < hi.nscan; q += 32) {
+            const Partial pp = part[hi.scan_first + q];
+            if (better(pp.s, pp.c, s, cb)) { s = pp.s; cb = pp.c; }
+            eown += pp.eown;
+          }
+          group_reduce<32>(s, cb, eown);
+          const int32_t own = (int32_t)__ldg(&A.ca[hi.v]).x;
+          int32_t tgt = own;
+          if (lane == 0) tgt = finish(s, cb, eown, own, __ldg(&A.ca[own]).y, __ldg(&A.k[hi.v]), A);
+          log_moves(lane == 0 && tgt != own, hi.v, tgt, A);
+        }
+      }
+    }
+    grid.sync();
+  }
+}
+
+template <class K>
+int32_t set_smem(K kernel, size_t bytes) {
+  LV_CUDA(cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes));
+  return LOUVAIN_OK;
+}
+
+template <bool UNIT, bool AGG>
 int32_t dispatch_class(Handle& h, Level& L, const SweepArgs& A, int bucket, int sub, int64_t max_deg) {
-  const int64_t off = L.class_off[4 * bucket + sub];
-  const int64_t nv = L.class_off[4 * bucket + sub + 1] - off;
+  const int64_t off = L.class_off[kSubPerBucket * bucket + sub];
+  const int64_t nv = L.class_off[kSubPerBucket * bucket + sub + 1] - off;
   if (nv <= 0) return LOUVAIN_OK;
   const int32_t* verts = L.bin_vertices + off;
   cudaStream_t s = h.stream;
@@ -313,33 +663,81 @@ int32_t dispatch_class(Handle& h, Level& L, const SweepArgs& A, int bucket, int 
     }
     LV_LAUNCHED();
   } else if (sub == 0 && max_deg <= 84) {
-    sweep_warp<128, UNIT><<<grid_for(nv, 8, 148 * 8), 256, 0, s>>>(verts, nv, A);
+    sweep_warp<128, 8, UNIT, AGG><<<grid_for(nv, 8, 148 * 8), 256, 0, s>>>(verts, nv, A);
     LV_LAUNCHED();
   } else if (sub == 0 && max_deg <= 340) {
-    sweep_warp<512, UNIT><<<grid_for(nv, 8, 148 * 6), 256, 0, s>>>(verts, nv, A);
+    sweep_warp<512, 4, UNIT, AGG><<<grid_for(nv, 4, 148 * 12), 128, 0, s>>>(verts, nv, A);
     LV_LAUNCHED();
-  } else if (sub <= 1) {
-    const int cap = (sub == 0) ? kCtaSmallCap : kCtaLargeCap;
-    const int threads = (sub == 0) ? 256 : 1024;
-    const size_t smem = sizeof(unsigned long long) * (size_t)cap;
-    static bool attr_set[2][2] = {{false, false}, {false, false}};
-    if (!attr_set[UNIT][sub]) {
-      LV_CUDA(cudaFuncSetAttribute(sweep_cta<UNIT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kCtaLargeCap * 8));
-      attr_set[UNIT][sub] = true;
+  } else if (sub == 3 || sub == 4) {
+    const int CS = (sub == 3) ? 4 : 16;
+    static bool cl_attr = false;
+    if (!cl_attr) {
+      for (auto k : {sweep_cluster<true>, sweep_cluster<false>}) {
+        LV_TRY(set_smem(k, 12 * (size_t)kClusterSlots));
+        LV_CUDA(cudaFuncSetAttribute(k, cudaFuncAttributeNonPortableClusterSizeAllowed, 1));
+      }
+      cl_attr = true;
     }
-    const unsigned grid = grid_for(nv, 1, 148 * (sub == 0 ? 3 : 1));
-    sweep_cta<UNIT><<<grid, threads, smem, s>>>(verts, nv, A, cap);
+    cudaLaunchConfig_t cfg = {};
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeClusterDimension;
+    attr[0].val.clusterDim.x = CS;
+    attr[0].val.clusterDim.y = 1;
+    attr[0].val.clusterDim.z = 1;
+    cfg.blockDim = dim3(1024, 1, 1);
+    cfg.dynamicSmemBytes = 12 * (size_t)kClusterSlots;
+    cfg.stream = s;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    static int max_clusters[2] = {0, 0};
+    int& mc = max_clusters[sub - 3];
+    if (!mc) {
+      cfg.gridDim = dim3(CS * 64, 1, 1);
+      LV_CUDA(cudaOccupancyMaxActiveClusters(&mc, (void*)sweep_cluster<UNIT>, &cfg));
+      if (mc < 1) mc = 1;
+    }
+    const int64_t ncl = std::min<int64_t>(mc, nv);
+    cfg.gridDim = dim3((unsigned)(ncl * CS), 1, 1);
+    LV_CUDA(cudaLaunchKernelEx(&cfg, sweep_cluster<UNIT>, verts, nv, A));
+    LV_LAUNCHED();
+  } else if (sub <= 2) {
+    static const int caps[3] = {kCap0, kCap1, kCap2};
+    static const int threads[3] = {256, 512, 1024};
+    static const int per_sm[3] = {6, 2, 1};
+    const size_t smem = 12 * (size_t)caps[sub];
+    static bool attr_done = false;
+    if (!attr_done) {
+      LV_TRY(set_smem(sweep_cta<true, false>, 12 * (size_t)kCap2));
+      LV_TRY(set_smem(sweep_cta<false, false>, 12 * (size_t)kCap2));
+      LV_TRY(set_smem(sweep_cta<true, true>, 12 * (size_t)kCap2));
+      LV_TRY(set_smem(sweep_cta<false, true>, 12 * (size_t)kCap2));
+      attr_done = true;
+    }
+    const unsigned grid = grid_for(nv, 1, 148 * per_sm[sub]);
+    sweep_cta<UNIT, AGG><<<grid, threads[sub], smem, s>>>(verts, nv, A, caps[sub]);
     LV_LAUNCHED();
   } else {
     HubPlan& P = L.hub;
     if (P.nh > 0) {
-      hub_insert<UNIT><<<grid_for(P.nchunks, 1, 148 * 4), 512, 0, s>>>(P.chunk, P.nchunks, P.hub_v, P.tab_off,
-                                                                       P.tab_cap, P.table, A);
-      LV_LAUNCHED();
-      hub_scan<<<grid_for(P.nscan, 1, 148 * 4), 512, 0, s>>>(P.scan, P.nscan, P.hub_v, P.tab_off, P.table,
-                                                             (Partial*)P.partial, A);
-      LV_LAUNCHED();
-      hub_final<<<grid_for(P.nh, 8), 256, 0, s>>>(P.nh, P.scan_first, (const Partial*)P.partial, P.hub_v, A);
+      if (!P.grid) {
+        int per_sm = 0, nsm = 0;
+        LV_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, hub_coop<UNIT>, 512, 0));
+        LV_CUDA(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, h.device));
+        P.grid = std::max(1, per_sm) * nsm;  // cooperative launch: every CTA co-resident
+      }
+      const HubItem* a0 = P.ins;
+      const int64_t* a1 = P.ins_off;
+      const HubItem* a2 = P.scans;
+      const int64_t* a3 = P.scan_off;
+      const int64_t* a4 = P.wave_hub;
+      const HubInfo* a5 = P.info;
+      int64_t a6 = P.nwaves, a7 = P.seg;
+      unsigned long long* a8 = P.ring;
+      uint32_t* a9 = P.ring_a;
+      Partial* a10 = (Partial*)P.partial;
+      SweepArgs a11 = A;
+      void* args[] = {&a0, &a1, &a2, &a3, &a4, &a5, &a6, &a7, &a8, &a9, &a10, &a11};
+      LV_CUDA(cudaLaunchCooperativeKernel((void*)hub_coop<UNIT>, P.grid, 512, args, 0, s));
       LV_LAUNCHED();
     }
   }
@@ -359,8 +757,7 @@ int32_t launch_sweep_bucket(Handle& h, Level& L, const louvain_params_t& p, int 
   A.col = L.col;
   A.w = L.w;
   A.k = L.k;
-  A.C = L.C;
-  A.a = L.a;
+  A.ca = L.ca;
   A.size = L.size;
   A.W = (long long)L.W;
   A.rule = p.singleton_rule;
@@ -368,11 +765,18 @@ int32_t launch_sweep_bucket(Handle& h, Level& L, const louvain_params_t& p, int 
   A.mv_new = L.mv_new;
   A.logn = &h.ctl->logn;
   const int64_t hi = (bucket <= 6) ? p.deg_bounds[bucket - 1] : INT64_MAX;
-  for (int sub = 0; sub < 3; ++sub) {
-    int64_t max_deg = hi;
-    if (sub == 0) max_deg = std::min<int64_t>(hi, kCtaLargeMin - 1);
-    if (L.w) LV_TRY(dispatch_class<false>(h, L, A, bucket, sub, max_deg));
-    else LV_TRY(dispatch_class<true>(h, L, A, bucket, sub, max_deg));
+  for (int sub = 0; sub < 6; ++sub) {
+    const int64_t max_deg = (sub == 0) ? std::min<int64_t>(hi, kSub1Min - 1) : hi;
+    // warp-level label merging pays once communities exist (hot labels); on the
+    // first sweep of a level most labels in a row are distinct and it does not
+    const bool agg = L.sweeps_done > 0;
+    if (L.w) {
+      if (agg) LV_TRY((dispatch_class<false, true>(h, L, A, bucket, sub, max_deg)));
+      else LV_TRY((dispatch_class<false, false>(h, L, A, bucket, sub, max_deg)));
+    } else {
+      if (agg) LV_TRY((dispatch_class<true, true>(h, L, A, bucket, sub, max_deg)));
+      else LV_TRY((dispatch_class<true, false>(h, L, A, bucket, sub, max_deg)));
+    }
   }
   return LOUVAIN_OK;
 }

@@ -66,6 +66,8 @@ GRAPHS = {
     "lfr5k": lambda: graphgen.lfr(5000, kmin=8, kmax=300, smin=20, smax=600, seed=5),
     "weighted_loops": lambda: weighted_with_loops(3000, 6),
     "hubs": lambda: hubs_graph(),
+    # one vertex past the cluster classes (>= 131072): the cooperative global-table path
+    "giant_hub": lambda: hubs_graph(seed=1, hub_degrees=(150000, 20000, 3000), n=200000, bg_tuples=300000),
 }
 
 
