@@ -138,17 +138,36 @@ int32_t louvain_run(louvain_graph_t g, const louvain_params_t* p, int32_t* label
 /* Thread-local message of the last error ("" if none). */
 const char* louvain_last_error(void);
 
-/* ---- multi-GPU: one process per GPU, vertex-range sharding ----
- * The 128-byte NCCL unique id is created on rank 0 and broadcast by the caller
- * (torch.distributed.broadcast_object_list). */
-int32_t louvain_dist_unique_id(uint8_t id[128]);
-/* Rank `rank` of `world` owns rows [v_begin, v_end) (rowptr_local has
- * v_end - v_begin + 1 entries starting at 0, global column ids).  Every call on
- * the returned handle is collective over the ranks; label buffers have global
- * length n. */
-int32_t louvain_create_csr_dist(int64_t n, int64_t v_begin, int64_t v_end, const int64_t* rowptr_local,
-                                const int32_t* col_local, const uint32_t* w_local, uint32_t flags, int32_t rank,
-                                int32_t world, const uint8_t id[128], void* cuda_stream, louvain_graph_t* out);
+/* ---- sharded sweep primitives (multi-GPU, one process per GPU) ----
+ * Every rank holds the same level graph and a replica of the partition state.
+ * Rank r owns the vertex range [v_begin, v_end): it decides only its own
+ * vertices, exchanges the moves of each bucket with the other ranks (the
+ * caller's collective, e.g. an NCCL all-gather through torch.distributed), and
+ * every rank commits ALL moves of the bucket, so the replicas stay bit-identical
+ * (integer updates, order-independent).  A single rank owning [0, n) reproduces
+ * louvain_sweep exactly. */
+/* Restrict decisions (and louvain_modularity_owned's L) to [v_begin, v_end). */
+int32_t louvain_set_owned_range(louvain_graph_t g, int64_t v_begin, int64_t v_end);
+/* Start a sweep: clears the sweep's move log (the revert record, R15). */
+int32_t louvain_begin_sweep(louvain_graph_t g);
+/* computeMove (Alg. 2) for the owned vertices of bucket `bucket` (1..7) against
+ * the current state, without committing.  moves_out: int32 pairs (v, new),
+ * capacity `cap` pairs (host or device); *count = moves written.  Bucket
+ * bounds come from p->deg_bounds. */
+int32_t louvain_decide_bucket(louvain_graph_t g, const louvain_params_t* p, int32_t bucket, int32_t* moves_out,
+                              int64_t cap, int64_t* count);
+/* Commit `count` moves (v, new) (any owner; each v at most once per sweep):
+ * C, a_c, size_c updated with exact integer deltas (Alg. 1 l.8-11) and the
+ * moves appended to the sweep's log. */
+int32_t louvain_commit_moves(louvain_graph_t g, const int32_t* moves, int64_t count);
+/* Undo every move committed since louvain_begin_sweep (R15). */
+int32_t louvain_revert_sweep(louvain_graph_t g);
+/* Label composition across levels (R22): lab[i] = map[lab[i]] for i < n0
+ * (device pointers; runs on `cuda_stream`, NULL = default stream). */
+int32_t louvain_compose_labels(int32_t* lab, int64_t n0, const int32_t* map, void* cuda_stream);
+/* Eq. (1) parts of the current partition with L summed over the owned rows
+ * only (the ranks' L add up to the graph's L); S and W are global. */
+int32_t louvain_modularity_owned(louvain_graph_t g, uint64_t* L_owned, uint64_t* S, uint64_t* W);
 
 #ifdef __cplusplus
 }

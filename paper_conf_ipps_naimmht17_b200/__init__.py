@@ -91,11 +91,15 @@ FUNCS = {
     "louvain_run": (ctypes.c_int32, [ctypes.c_void_p, ctypes.POINTER(Params), ctypes.c_void_p,
                                      ctypes.POINTER(QNum), ctypes.POINTER(Stats)]),
     "louvain_last_error": (ctypes.c_char_p, []),
-    "louvain_dist_unique_id": (ctypes.c_int32, [ctypes.c_void_p]),
-    "louvain_create_csr_dist": (ctypes.c_int32, [ctypes.c_int64, ctypes.c_int64, ctypes.c_int64, ctypes.c_void_p,
-                                                 ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint32, ctypes.c_int32,
-                                                 ctypes.c_int32, ctypes.c_void_p, ctypes.c_void_p,
-                                                 ctypes.POINTER(ctypes.c_void_p)]),
+    "louvain_set_owned_range": (ctypes.c_int32, [ctypes.c_void_p, ctypes.c_int64, ctypes.c_int64]),
+    "louvain_begin_sweep": (ctypes.c_int32, [ctypes.c_void_p]),
+    "louvain_decide_bucket": (ctypes.c_int32, [ctypes.c_void_p, ctypes.POINTER(Params), ctypes.c_int32,
+                                               ctypes.c_void_p, ctypes.c_int64, ctypes.POINTER(ctypes.c_int64)]),
+    "louvain_commit_moves": (ctypes.c_int32, [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int64]),
+    "louvain_revert_sweep": (ctypes.c_int32, [ctypes.c_void_p]),
+    "louvain_compose_labels": (ctypes.c_int32, [ctypes.c_void_p, ctypes.c_int64, ctypes.c_void_p, ctypes.c_void_p]),
+    "louvain_modularity_owned": (ctypes.c_int32, [ctypes.c_void_p, ctypes.POINTER(ctypes.c_uint64),
+                                                  ctypes.POINTER(ctypes.c_uint64), ctypes.POINTER(ctypes.c_uint64)]),
 }
 
 _LIB = None
@@ -265,13 +269,45 @@ class Graph:
         _check(lib().louvain_modularity(self._h, p, ctypes.byref(q)))
         return q
 
-    def aggregate(self, with_map: bool = True):
-        """Alg. 3: returns (next Graph, map ndarray or None)."""
+    def aggregate(self, with_map: bool = True, map_out=None):
+        """Alg. 3: returns (next Graph, map) -- map in `map_out` (host or device) if given."""
         n = self.n
-        mp = np.empty(max(n, 1), dtype=np.int32) if with_map else None
+        if map_out is None and with_map:
+            map_out = np.empty(max(n, 1), dtype=np.int32)
+        mp, keep = _ptr(map_out)
         h = ctypes.c_void_p()
-        _check(lib().louvain_aggregate(self._h, ctypes.byref(h), mp.ctypes.data if with_map else None))
-        return Graph(h, self._stream), (mp[:n] if with_map else None)
+        _check(lib().louvain_aggregate(self._h, ctypes.byref(h), mp))
+        if isinstance(map_out, np.ndarray):
+            map_out = map_out[:n]
+        return Graph(h, self._stream), map_out
+
+    # ---------------------------------------------------------------- sharded-sweep primitives
+    def set_owned_range(self, lo: int, hi: int) -> None:
+        _check(lib().louvain_set_owned_range(self._h, lo, hi))
+
+    def begin_sweep(self) -> None:
+        _check(lib().louvain_begin_sweep(self._h))
+
+    def decide_bucket(self, p: Params, bucket: int, out) -> int:
+        """Moves (v, new) of the owned vertices of `bucket` into out (int32 [cap, 2]); returns count."""
+        ptr, keep = _ptr(out)
+        cnt = ctypes.c_int64()
+        _check(lib().louvain_decide_bucket(self._h, ctypes.byref(p), bucket, ptr, int(out.shape[0]),
+                                           ctypes.byref(cnt)))
+        return cnt.value
+
+    def commit_moves(self, moves, count: int) -> None:
+        ptr, keep = _ptr(moves)
+        _check(lib().louvain_commit_moves(self._h, ptr if count else None, count))
+
+    def revert_sweep(self) -> None:
+        _check(lib().louvain_revert_sweep(self._h))
+
+    def modularity_owned(self) -> tuple[int, int, int]:
+        L, S, W = ctypes.c_uint64(), ctypes.c_uint64(), ctypes.c_uint64()
+        _check(lib().louvain_modularity_owned(self._h, ctypes.byref(L), ctypes.byref(S), ctypes.byref(W)))
+        return L.value, S.value, W.value
+
 
     def run(self, p: Optional[Params] = None, labels_out=None, want_labels: bool = True):
         """Full multilevel Louvain; returns (labels, QNum, stats dict)."""
@@ -284,6 +320,14 @@ class Graph:
         _check(lib().louvain_run(self._h, ctypes.byref(p or params()), lp, ctypes.byref(q), ctypes.byref(st)))
         lab = labels_out[:n] if isinstance(labels_out, np.ndarray) else labels_out
         return lab, q, st.as_dict()
+
+
+def compose_labels(lab, mp, stream=None) -> None:
+    """lab[i] = mp[lab[i]] on the device (torch int32 CUDA tensors)."""
+    sp = None
+    if stream is not None:
+        sp = stream.cuda_stream if hasattr(stream, "cuda_stream") else int(stream)
+    _check(lib().louvain_compose_labels(lab.data_ptr(), int(lab.numel()), mp.data_ptr(), sp))
 
 
 def run(rowptr, col, w=None, p: Optional[Params] = None, **kw):

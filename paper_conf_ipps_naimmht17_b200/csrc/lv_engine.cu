@@ -233,7 +233,11 @@ int32_t run_impl(Handle& h, const louvain_params_t& p, int32_t* labels_out, louv
   int32_t* lab = nullptr;
   LV_TRY(dalloc(&lab, n0, s));
   if (n0) { k_iota<<<grid_for(n0, 256), 256, 0, s>>>(lab, n0); LV_LAUNCHED(); }
-  // level 0 starts from singletons
+  // level 0 starts from singletons; a full run owns every vertex
+  if (L0.own_hi >= 0) {
+    L0.own_hi = -1;
+    L0.bins_valid = false;
+  }
   if (n0) LV_TRY(level_set_labels(h, L0, nullptr));
   uint64_t Lq = 0, Sq = 0;  // exact parts of the current level's kept partition
   Level owned;   // current contracted level (levels >= 1)
@@ -610,17 +614,162 @@ LV_API int32_t louvain_run(louvain_graph_t g, const louvain_params_t* p, int32_t
   return finish_call(h, run_impl(h, pp, labels_out, q_final, stats));
 }
 
-LV_API int32_t louvain_dist_unique_id(uint8_t id[128]) {
-  (void)id;
-  set_error("multi-GPU not built yet");
-  return LOUVAIN_E_UNSUPPORTED;
+LV_API int32_t louvain_set_owned_range(louvain_graph_t g, int64_t v_begin, int64_t v_end) {
+  LV_TRY(guard(g));
+  Handle& h = g->h;
+  DeviceScope ds(h.device);
+  Level& L = h.lv;
+  if (v_begin < 0 || v_end < v_begin || v_end > L.n) {
+    set_error("owned range must satisfy 0 <= v_begin <= v_end <= n");
+    return LOUVAIN_E_INVALID_ARG;
+  }
+  int64_t e[2] = {0, 0};
+  LV_CUDA(cudaMemcpy(&e[0], L.rowptr + v_begin, 8, cudaMemcpyDeviceToHost));
+  LV_CUDA(cudaMemcpy(&e[1], L.rowptr + v_end, 8, cudaMemcpyDeviceToHost));
+  L.own_lo = v_begin;
+  L.own_hi = v_end;
+  L.own_e0 = e[0];
+  L.own_e1 = e[1];
+  L.bins_valid = false;  // bucket lists hold the owned vertices only
+  return LOUVAIN_OK;
 }
 
-LV_API int32_t louvain_create_csr_dist(int64_t n, int64_t v_begin, int64_t v_end, const int64_t* rowptr_local,
-                                       const int32_t* col_local, const uint32_t* w_local, uint32_t flags, int32_t rank,
-                                       int32_t world, const uint8_t id[128], void* cuda_stream, louvain_graph_t* out) {
-  (void)n; (void)v_begin; (void)v_end; (void)rowptr_local; (void)col_local; (void)w_local; (void)flags;
-  (void)rank; (void)world; (void)id; (void)cuda_stream; (void)out;
-  set_error("multi-GPU not built yet");
-  return LOUVAIN_E_UNSUPPORTED;
+LV_API int32_t louvain_begin_sweep(louvain_graph_t g) {
+  LV_TRY(guard(g));
+  Handle& h = g->h;
+  DeviceScope ds(h.device);
+  Level& L = h.lv;
+  if (L.log_committed > 0) ++L.sweeps_done;
+  L.log_committed = 0;
+  return finish_call(h, set_ctl_u64(h, &h.ctl->logn, 0));
+}
+
+LV_API int32_t louvain_decide_bucket(louvain_graph_t g, const louvain_params_t* p, int32_t bucket, int32_t* moves_out,
+                                     int64_t cap, int64_t* count) {
+  LV_TRY(guard(g));
+  if (bucket < 1 || bucket > 7 || !count || cap < 0 || (cap > 0 && !moves_out)) {
+    set_error("louvain_decide_bucket: bucket in 1..7, count and moves_out required");
+    return LOUVAIN_E_INVALID_ARG;
+  }
+  louvain_params_t pp;
+  if (p) pp = *p; else louvain_params_default(&pp);
+  LV_TRY(check_params(pp));
+  Handle& h = g->h;
+  DeviceScope ds(h.device);
+  Level& L = h.lv;
+  const int64_t c0 = L.log_committed;
+  int32_t rc = level_binning(h, L, pp);
+  if (!rc) rc = set_ctl_u64(h, &h.ctl->logn, (unsigned long long)c0);
+  if (!rc && bucket_nonempty(L, bucket)) rc = launch_sweep_bucket(h, L, pp, bucket);
+  unsigned long long c1 = c0;
+  if (!rc) {
+    cudaError_t e = cudaMemcpyAsync(&c1, &h.ctl->logn, 8, cudaMemcpyDeviceToHost, h.stream);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(h.stream);
+    if (e != cudaSuccess) rc = cuda_fail(e, "decide_bucket", __FILE__, __LINE__);
+  }
+  const int64_t cnt = (int64_t)c1 - c0;
+  if (!rc && cnt > cap) {
+    set_error("louvain_decide_bucket: moves_out capacity too small");
+    rc = LOUVAIN_E_INVALID_ARG;
+  }
+  if (!rc && cnt > 0) {
+    int32_t* tmp = nullptr;
+    rc = dalloc(&tmp, 2 * cnt, h.stream);
+    if (!rc) rc = pack_moves(h, L, c0, cnt, tmp);
+    if (!rc) rc = copy_out(moves_out, tmp, 8 * (size_t)cnt, h.stream);
+    dfree(tmp, h.stream);
+  }
+  if (!rc) rc = set_ctl_u64(h, &h.ctl->logn, (unsigned long long)c0);  // nothing committed yet
+  if (!rc) {
+    cudaError_t e = cudaStreamSynchronize(h.stream);
+    if (e != cudaSuccess) rc = cuda_fail(e, "decide_bucket", __FILE__, __LINE__);
+  }
+  if (!rc) *count = cnt;
+  return finish_call(h, rc);
+}
+
+LV_API int32_t louvain_commit_moves(louvain_graph_t g, const int32_t* moves, int64_t count) {
+  LV_TRY(guard(g));
+  Handle& h = g->h;
+  Level& L = h.lv;
+  if (count < 0 || (count > 0 && !moves) || L.log_committed + count > L.n) {
+    set_error("louvain_commit_moves: bad count (each vertex moves at most once per sweep)");
+    return LOUVAIN_E_INVALID_ARG;
+  }
+  DeviceScope ds(h.device);
+  const int64_t c0 = L.log_committed;
+  int32_t rc = LOUVAIN_OK;
+  if (count > 0) {
+    int32_t* d = nullptr;
+    bool owned = false;
+    rc = stage(moves, 2 * count, false, h.stream, &d, &owned);
+    if (!rc) rc = unpack_moves(h, L, c0, count, d);
+    if (owned) dfree(d, h.stream);
+    if (!rc) rc = set_ctl_u64(h, &h.ctl->bounds[0], (unsigned long long)c0);
+    if (!rc) rc = set_ctl_u64(h, &h.ctl->logn, (unsigned long long)(c0 + count));
+    if (!rc) rc = launch_commit(h, L, 0);
+    if (!rc) {
+      cudaError_t e = cudaStreamSynchronize(h.stream);
+      if (e != cudaSuccess) rc = cuda_fail(e, "commit_moves", __FILE__, __LINE__);
+    }
+  }
+  if (!rc) L.log_committed = c0 + count;
+  return finish_call(h, rc);
+}
+
+LV_API int32_t louvain_revert_sweep(louvain_graph_t g) {
+  LV_TRY(guard(g));
+  Handle& h = g->h;
+  DeviceScope ds(h.device);
+  Level& L = h.lv;
+  int32_t rc = set_ctl_u64(h, &h.ctl->logn, (unsigned long long)L.log_committed);
+  if (!rc) rc = launch_revert(h, L);
+  if (!rc) rc = set_ctl_u64(h, &h.ctl->logn, 0);
+  if (!rc) {
+    cudaError_t e = cudaStreamSynchronize(h.stream);
+    if (e != cudaSuccess) rc = cuda_fail(e, "revert", __FILE__, __LINE__);
+  }
+  if (!rc) L.log_committed = 0;
+  return finish_call(h, rc);
+}
+
+namespace lv {
+namespace abi_kernels {
+__global__ void k_compose_ext(int32_t* lab, int64_t n0, const int32_t* map) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n0; i += (int64_t)gridDim.x * blockDim.x)
+    lab[i] = map[lab[i]];
+}
+}  // namespace abi_kernels
+}  // namespace lv
+
+LV_API int32_t louvain_compose_labels(int32_t* lab, int64_t n0, const int32_t* map, void* cuda_stream) {
+  if (n0 < 0 || (n0 > 0 && (!lab || !map))) {
+    set_error("louvain_compose_labels: null pointer");
+    return LOUVAIN_E_INVALID_ARG;
+  }
+  if (n0 == 0) return LOUVAIN_OK;
+  if (!is_device_ptr(lab) || !is_device_ptr(map)) {
+    set_error("louvain_compose_labels: lab and map must be device pointers");
+    return LOUVAIN_E_INVALID_ARG;
+  }
+  lv::abi_kernels::k_compose_ext<<<grid_for(n0, 256), 256, 0, (cudaStream_t)cuda_stream>>>(lab, n0, map);
+  LV_LAUNCHED();
+  LV_CUDA(cudaGetLastError());
+  LV_CUDA(cudaStreamSynchronize((cudaStream_t)cuda_stream));
+  return LOUVAIN_OK;
+}
+
+LV_API int32_t louvain_modularity_owned(louvain_graph_t g, uint64_t* L_owned, uint64_t* S, uint64_t* W) {
+  LV_TRY(guard(g));
+  Handle& h = g->h;
+  DeviceScope ds(h.device);
+  Level& L = h.lv;
+  uint64_t Lq = 0, Sq = 0;
+  int32_t rc = level_modularity(h, L, nullptr, &Lq, &Sq);
+  if (!rc) {
+    if (L_owned) *L_owned = Lq;
+    if (S) *S = Sq;
+    if (W) *W = L.W;
+  }
+  return finish_call(h, rc);
 }

@@ -109,6 +109,10 @@ struct Level {
   int32_t* mv_new = nullptr;
   int32_t* mv_old = nullptr;
   int32_t sweeps_done = 0;  // sweeps since the partition was last reset to singletons
+  // sharded sweeps: owned vertex range (decisions, L) and its edge range
+  int64_t own_lo = 0, own_hi = -1;  // own_hi < 0: all vertices
+  int64_t own_e0 = 0, own_e1 = -1;
+  int64_t log_committed = 0;        // entries of the sweep's move log already committed
   // binning (valid for bins_bounds)
   bool bins_valid = false;
   int64_t bins_bounds[6] = {0, 0, 0, 0, 0, 0};
@@ -158,6 +162,9 @@ int32_t level_binning(Handle& h, Level& L, const louvain_params_t& p);  // class
 int32_t level_modularity(Handle& h, Level& L, const int32_t* d_C, uint64_t* Lout, uint64_t* Sout);
 int32_t launch_modularity(Handle& h, Level& L, const int32_t* d_C);  // async: ctl->L, ctl->S
 int32_t launch_commit(Handle& h, Level& L, int bucket);
+int32_t set_ctl_u64(Handle& h, unsigned long long* dst, unsigned long long v);
+int32_t pack_moves(Handle& h, Level& L, int64_t c0, int64_t cnt, int32_t* out);          // log -> (v,new) pairs
+int32_t unpack_moves(Handle& h, Level& L, int64_t c0, int64_t cnt, const int32_t* in);   // (v,new) pairs -> log
 int32_t launch_revert(Handle& h, Level& L);
 int32_t level_contract(Handle& h, Level& L, Level& out, int32_t* d_map);  // Alg. 3
 int32_t compose_labels(Handle& h, int32_t* lab, int64_t n0, const int32_t* map);  // lab[i] = map[lab[i]]

@@ -70,14 +70,15 @@ __global__ void k_get_a(const uint2* ca, int64_t n, uint32_t* out) {
 
 // class = 8*bucket + sub  (lv_internal.cuh)
 __global__ void k_classify(const int64_t* rowptr, int64_t n, int64_t b0, int64_t b1, int64_t b2, int64_t b3,
-                           int64_t b4, int64_t b5, uint8_t* cls, int32_t* iota, unsigned long long* hist) {
+                           int64_t b4, int64_t b5, int64_t lo, int64_t hi, uint8_t* cls, int32_t* iota,
+                           unsigned long long* hist) {
   __shared__ unsigned long long sh[kNumClasses];
   if (threadIdx.x < kNumClasses) sh[threadIdx.x] = 0;
   __syncthreads();
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
     const int64_t d = rowptr[i + 1] - rowptr[i];  // R11: row length incl. self-loop
     int b;
-    if (d == 0) b = 0;
+    if (d == 0 || i < lo || i >= hi) b = 0;  // not decided here (no edges, or owned by another rank)
     else if (d <= b0) b = 1;
     else if (d <= b1) b = 2;
     else if (d <= b2) b = 3;
@@ -189,17 +190,17 @@ __device__ __forceinline__ void for_tile_edges(const int64_t* rowptr, int64_t n,
 template <bool PACKED>
 __global__ void __launch_bounds__(256) k_modularity(const int64_t* rowptr, int64_t n, const int32_t* col,
                                                     const uint32_t* w, const uint2* ca, const int32_t* C,
-                                                    const uint32_t* a, int64_t nnz, unsigned long long* Lout,
-                                                    unsigned long long* Sout) {
+                                                    const uint32_t* a, int64_t e_begin, int64_t nnz,
+                                                    unsigned long long* Lout, unsigned long long* Sout) {
   __shared__ int64_t sh_rows[kTileRows];
   __shared__ int64_t sh_u0;
   __shared__ int sh_nr;
   const uint32_t* lab = PACKED ? reinterpret_cast<const uint32_t*>(ca) : reinterpret_cast<const uint32_t*>(C);
   const int st = PACKED ? 2 : 1;
   unsigned long long acc = 0;
-  const int64_t ntiles = (nnz + kTileEdges - 1) / kTileEdges;
+  const int64_t ntiles = (nnz - e_begin + kTileEdges - 1) / kTileEdges;
   for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
-    const int64_t e0 = tile * kTileEdges, e1 = min(nnz, e0 + kTileEdges);
+    const int64_t e0 = e_begin + tile * kTileEdges, e1 = min(nnz, e0 + kTileEdges);
     for_tile_edges(rowptr, n, e0, e1, sh_rows, &sh_u0, &sh_nr, [&](int64_t u, int64_t e) {
       const int32_t v = __ldcs(&col[e]);
       if (__ldg(&lab[st * (int64_t)v]) == __ldg(&lab[st * u])) acc += w ? __ldcs(&w[e]) : 1u;
@@ -486,8 +487,10 @@ int32_t level_binning(Handle& h, Level& L, const louvain_params_t& p) {
     LV_TRY(dalloc(&iota, n, s));
     LV_TRY(dalloc(&hist, kNumClasses, s));
     LV_CUDA(cudaMemsetAsync(hist, 0, 8 * kNumClasses, s));
+    const int64_t lo = L.own_hi < 0 ? 0 : L.own_lo, hi = L.own_hi < 0 ? n : L.own_hi;
     k_classify<<<grid_for(n, 256), 256, 0, s>>>(L.rowptr, n, p.deg_bounds[0], p.deg_bounds[1], p.deg_bounds[2],
-                                                p.deg_bounds[3], p.deg_bounds[4], p.deg_bounds[5], cls, iota, hist);
+                                                p.deg_bounds[3], p.deg_bounds[4], p.deg_bounds[5], lo, hi, cls,
+                                                iota, hist);
     LV_LAUNCHED();
     LV_CUDA(cudaGetLastError());
     // stable sort by class (6 bits): vertices of a class stay in ascending id order
@@ -515,10 +518,11 @@ int32_t launch_modularity(Handle& h, Level& L, const int32_t* d_C) {
   cudaStream_t s = h.stream;
   LV_CUDA(cudaMemsetAsync(&h.ctl->L, 0, 16, s));
   if (L.n == 0) return LOUVAIN_OK;
-  const int64_t ntiles = (L.nnz + kTileEdges - 1) / kTileEdges;
+  const int64_t e0 = (d_C || L.own_hi < 0) ? 0 : L.own_e0, e1 = (d_C || L.own_hi < 0) ? L.nnz : L.own_e1;
+  const int64_t ntiles = (e1 - e0 + kTileEdges - 1) / kTileEdges;
   const unsigned grid = grid_for(std::max<int64_t>(ntiles, (L.n + 255) / 256), 1, 148 * 8);
   if (!d_C) {
-    k_modularity<true><<<grid, 256, 0, s>>>(L.rowptr, L.n, L.col, L.w, L.ca, nullptr, nullptr, L.nnz, &h.ctl->L,
+    k_modularity<true><<<grid, 256, 0, s>>>(L.rowptr, L.n, L.col, L.w, L.ca, nullptr, nullptr, e0, e1, &h.ctl->L,
                                             &h.ctl->S);
     LV_LAUNCHED();
   } else {
@@ -527,7 +531,7 @@ int32_t launch_modularity(Handle& h, Level& L, const int32_t* d_C) {
     LV_CUDA(cudaMemsetAsync(a_tmp, 0, 4 * L.n, s));
     k_ext_totals<<<grid_for(L.n, 256), 256, 0, s>>>(d_C, L.k, L.n, a_tmp, &h.ctl->bad);
     LV_LAUNCHED();
-    k_modularity<false><<<grid, 256, 0, s>>>(L.rowptr, L.n, L.col, L.w, nullptr, d_C, a_tmp, L.nnz, &h.ctl->L,
+    k_modularity<false><<<grid, 256, 0, s>>>(L.rowptr, L.n, L.col, L.w, nullptr, d_C, a_tmp, 0, L.nnz, &h.ctl->L,
                                              &h.ctl->S);
     LV_LAUNCHED();
     dfree(a_tmp, s);
@@ -552,6 +556,45 @@ int32_t level_modularity(Handle& h, Level& L, const int32_t* d_C, uint64_t* Lout
 
 int32_t launch_commit(Handle& h, Level& L, int bucket) {
   k_commit<<<148 * 4, 256, 0, h.stream>>>(h.ctl, bucket, L.mv_v, L.mv_new, L.mv_old, L.ca, L.size, L.k);
+  LV_LAUNCHED();
+  LV_CUDA(cudaGetLastError());
+  return LOUVAIN_OK;
+}
+
+namespace {
+__global__ void k_set_u64(unsigned long long* p, unsigned long long v) { *p = v; }
+__global__ void k_pack_moves(const int32_t* mv_v, const int32_t* mv_new, int64_t c0, int64_t cnt, int32_t* out) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < cnt; i += (int64_t)gridDim.x * blockDim.x) {
+    out[2 * i] = mv_v[c0 + i];
+    out[2 * i + 1] = mv_new[c0 + i];
+  }
+}
+__global__ void k_unpack_moves(const int32_t* in, int64_t c0, int64_t cnt, int32_t* mv_v, int32_t* mv_new) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < cnt; i += (int64_t)gridDim.x * blockDim.x) {
+    mv_v[c0 + i] = in[2 * i];
+    mv_new[c0 + i] = in[2 * i + 1];
+  }
+}
+}  // namespace
+
+int32_t set_ctl_u64(Handle& h, unsigned long long* dst, unsigned long long v) {
+  k_set_u64<<<1, 1, 0, h.stream>>>(dst, v);
+  LV_LAUNCHED();
+  LV_CUDA(cudaGetLastError());
+  return LOUVAIN_OK;
+}
+
+int32_t pack_moves(Handle& h, Level& L, int64_t c0, int64_t cnt, int32_t* out) {
+  if (cnt <= 0) return LOUVAIN_OK;
+  k_pack_moves<<<grid_for(cnt, 256), 256, 0, h.stream>>>(L.mv_v, L.mv_new, c0, cnt, out);
+  LV_LAUNCHED();
+  LV_CUDA(cudaGetLastError());
+  return LOUVAIN_OK;
+}
+
+int32_t unpack_moves(Handle& h, Level& L, int64_t c0, int64_t cnt, const int32_t* in) {
+  if (cnt <= 0) return LOUVAIN_OK;
+  k_unpack_moves<<<grid_for(cnt, 256), 256, 0, h.stream>>>(in, c0, cnt, L.mv_v, L.mv_new);
   LV_LAUNCHED();
   LV_CUDA(cudaGetLastError());
   return LOUVAIN_OK;

