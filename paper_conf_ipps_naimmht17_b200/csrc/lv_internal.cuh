@@ -79,6 +79,7 @@ struct HubInfo {
   int32_t nscan;       // scan items of this hub
   int64_t off, cap;    // table region within its wave's ring segment
   int64_t scan_first;  // index of its first scan item (= its first partial)
+  int64_t sbase;       // stage index of edge e of the hub = sbase + e
 };
 struct HubPlan {
   int64_t nh = 0, nwaves = 0, nins = 0, nscan = 0, seg = 0;
@@ -118,6 +119,10 @@ struct Level {
   int64_t bins_bounds[6] = {0, 0, 0, 0, 0, 0};
   int32_t* bin_vertices = nullptr;
   int64_t class_off[kNumClasses + 1] = {0};
+  // gather staging (two-phase sweep): soff[i] = sum of degrees of bin_vertices[0..i),
+  // stage[soff[i] + t] = {label, a_c or 0xFFFFFFFF} of the t-th neighbour of bin_vertices[i]
+  int64_t* soff = nullptr;
+  uint2* stage = nullptr;
   HubPlan hub;
 };
 
@@ -175,6 +180,7 @@ int32_t validate_csr_host(int64_t n, int64_t nnz, const int64_t* rowptr, const i
 
 // ------------------------------------------------------------------ sweep (lv_sweep.cu)
 int32_t launch_sweep_bucket(Handle& h, Level& L, const louvain_params_t& p, int bucket);
+int32_t launch_stage(Handle& h, Level& L, int64_t pos0, int64_t pos1);  // phase 1 gather for positions [pos0,pos1)
 
 // ------------------------------------------------------------------ launch geometry
 inline unsigned grid_for(int64_t items, int per_block, int max_blocks = 148 * 16) {

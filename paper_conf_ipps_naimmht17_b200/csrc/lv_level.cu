@@ -104,6 +104,11 @@ __global__ void k_hub_degrees(const int32_t* hv, int64_t nh, const int64_t* rowp
   }
 }
 
+__global__ void k_bin_degrees(const int32_t* bv, int64_t n, const int64_t* rowptr, int64_t* dg) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i <= n; i += (int64_t)gridDim.x * blockDim.x)
+    dg[i] = (i < n) ? rowptr[bv[i] + 1] - rowptr[bv[i]] : 0;
+}
+
 __global__ void k_fill_u64(unsigned long long* p, int64_t n, unsigned long long v) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) p[i] = v;
 }
@@ -307,6 +312,7 @@ void level_free(Level& L, cudaStream_t s) {
   }
   dfree(L.k, s); dfree(L.ca, s); dfree(L.size, s);
   dfree(L.mv_v, s); dfree(L.mv_new, s); dfree(L.mv_old, s); dfree(L.bin_vertices, s);
+  dfree(L.soff, s); dfree(L.stage, s);
   hub_free(L.hub, s);
   L = Level();
 }
@@ -388,7 +394,7 @@ static int32_t build_hub_plan(Handle& h, Level& L) {
   cudaStream_t s = h.stream;
   HubPlan& P = L.hub;
   std::vector<int32_t> hv;
-  std::vector<int64_t> hdeg, rb;
+  std::vector<int64_t> hdeg, rb, hsoff;
   for (int b = 1; b <= 7; ++b) {
     const int c = kSubPerBucket * b + 5;
     const int64_t off = L.class_off[c], cnt = L.class_off[c + 1] - off;
@@ -399,10 +405,13 @@ static int32_t build_hub_plan(Handle& h, Level& L) {
     LV_TRY(dalloc(&dd, 2 * cnt, s));
     k_hub_degrees<<<grid_for(cnt, 256), 256, 0, s>>>(L.bin_vertices + off, cnt, L.rowptr, dd);
     LV_LAUNCHED();
+    std::vector<int64_t> so(cnt);
     LV_CUDA(cudaMemcpyAsync(v.data(), L.bin_vertices + off, 4 * cnt, cudaMemcpyDeviceToHost, s));
     LV_CUDA(cudaMemcpyAsync(d.data(), dd, 16 * cnt, cudaMemcpyDeviceToHost, s));
+    LV_CUDA(cudaMemcpyAsync(so.data(), L.soff + off, 8 * cnt, cudaMemcpyDeviceToHost, s));
     LV_CUDA(cudaStreamSynchronize(s));
     dfree(dd, s);
+    hsoff.insert(hsoff.end(), so.begin(), so.end());
     hv.insert(hv.end(), v.begin(), v.end());
     hdeg.insert(hdeg.end(), d.begin(), d.begin() + cnt);
     rb.insert(rb.end(), d.begin() + cnt, d.end());
@@ -428,6 +437,7 @@ static int32_t build_hub_plan(Handle& h, Level& L) {
     hi.v = hv[i];
     hi.cap = cap;
     hi.off = acc;
+    hi.sbase = hsoff[i] - rb[i];
     acc += cap;
     for (int64_t e = 0; e < hdeg[i]; e += kHubChunkEdges)
       ins.push_back(HubItem{(int32_t)i, 0, rb[i] + e, rb[i] + std::min(hdeg[i], e + kHubChunkEdges)});
@@ -505,6 +515,20 @@ int32_t level_binning(Handle& h, Level& L, const louvain_params_t& p) {
     LV_CUDA(cudaStreamSynchronize(s));
     dfree(cls, s); dfree(cls2, s); dfree(iota, s); dfree(hist, s);
     for (int c = 0; c < kNumClasses; ++c) L.class_off[c + 1] = L.class_off[c] + (int64_t)hh[c];
+    // staging offsets: exclusive scan of the degrees in bin order
+    if (!L.soff) LV_TRY(dalloc(&L.soff, n + 1, s));
+    if (!L.stage) LV_TRY(dalloc(&L.stage, L.nnz, s));
+    int64_t* dg = nullptr;
+    LV_TRY(dalloc(&dg, n + 1, s));
+    k_bin_degrees<<<grid_for(n, 256), 256, 0, s>>>(L.bin_vertices, n, L.rowptr, dg);
+    LV_LAUNCHED();
+    size_t tb2 = 0;
+    LV_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, tb2, dg, L.soff, n + 1, s));
+    void* tmp2 = nullptr;
+    LV_TRY(dmalloc(&tmp2, tb2, s));
+    LV_CUDA(cub::DeviceScan::ExclusiveSum(tmp2, tb2, dg, L.soff, n + 1, s)); LV_CUB();
+    dfree(tmp2, s);
+    dfree(dg, s);
   }
   LV_TRY(build_hub_plan(h, L));
   std::memcpy(L.bins_bounds, p.deg_bounds, sizeof L.bins_bounds);

@@ -282,48 +282,136 @@ __device__ __forceinline__ void gtable_insert4(unsigned long long* T, uint32_t* 
   }
 }
 
-// Inserts entries [t0, deg) step `stride` of the row starting at rb (vertex v),
-// 4 per pass: 4 col loads, then 4 independent record gathers, then 4
-// interleaved inserts.  With AGG, labels are first merged across the warp
-// (__match_any_sync, weights summed with __reduce_add_sync), so a label shared
-// by many neighbours costs one table atomic per warp instead of one per edge.
-// The trip count is uniform across each warp, as the warp intrinsics require.
+// Phase 1 of the two-phase sweep (edge-parallel gather): for every neighbour
+// slot of the bucket's table-based vertices, stage[soff[i] + t] = the packed
+// record of the t-th neighbour of bin_vertices[i] as {label, a_c if that
+// neighbour represents its label else kUnknownA}, or {kSelf, 0} for the
+// self-loop (R3).  Flat over the bucket's edges in 4096-entry tiles (the tile's
+// vertices are staged in smem and found by binary search), 4 gathers in flight
+// per thread -- the random gathers run at the memory system's throughput
+// instead of inside per-vertex latency chains.
+constexpr uint32_t kSelf = 0xFFFFFFFFu;
+constexpr int kStageTile = 4096;
+constexpr int kStageRows = 256;
+
+__global__ void __launch_bounds__(256) k_stage(const int32_t* __restrict__ bv, const int64_t* __restrict__ soff,
+                                               int64_t pos0, int64_t pos1, const int64_t* __restrict__ rowptr,
+                                               const int32_t* __restrict__ col, const uint2* __restrict__ ca,
+                                               uint2* __restrict__ stage) {
+  __shared__ int64_t sh_so[kStageRows + 1];
+  __shared__ int64_t sh_rb[kStageRows];
+  __shared__ int32_t sh_v[kStageRows];
+  __shared__ int64_t sh_i0;
+  __shared__ int sh_nr;
+  const int64_t s0 = soff[pos0], s1 = soff[pos1];
+  const int64_t ntiles = (s1 - s0 + kStageTile - 1) / kStageTile;
+  for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
+    const int64_t t0 = s0 + tile * kStageTile, t1 = min(s1, t0 + kStageTile);
+    if (threadIdx.x == 0) {
+      // largest i in [pos0, pos1) with soff[i] <= x
+      auto find = [&](int64_t x) {
+        int64_t lo = pos0, hi = pos1 - 1;
+        while (lo < hi) {
+          const int64_t mid = (lo + hi + 1) >> 1;
+          if (soff[mid] <= x) lo = mid; else hi = mid - 1;
+        }
+        return lo;
+      };
+      const int64_t i0 = find(t0), i1 = find(t1 - 1);
+      sh_i0 = i0;
+      sh_nr = (i1 - i0 + 1 <= kStageRows) ? (int)(i1 - i0 + 1) : -1;
+    }
+    __syncthreads();
+    const int64_t i0 = sh_i0;
+    const int nr = sh_nr;
+    for (int r = threadIdx.x; r < nr; r += blockDim.x) {
+      const int32_t v = bv[i0 + r];
+      sh_v[r] = v;
+      sh_so[r] = soff[i0 + r];
+      sh_rb[r] = rowptr[v];
+    }
+    __syncthreads();
+    for (int64_t base = t0 + threadIdx.x; base < t1; base += 4 * (int64_t)blockDim.x) {
+      int32_t jj[4], vv[4];
+      uint2 rr[4];
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        const int64_t t = base + (int64_t)q * blockDim.x;
+        jj[q] = -1;
+        vv[q] = -1;
+        if (t < t1) {
+          int64_t e;
+          if (nr > 0) {
+            int lo = 0, hi = nr - 1;
+            while (lo < hi) {
+              const int mid = (lo + hi + 1) >> 1;
+              if (sh_so[mid] <= t) lo = mid; else hi = mid - 1;
+            }
+            vv[q] = sh_v[lo];
+            e = sh_rb[lo] + (t - sh_so[lo]);
+          } else {
+            int64_t lo = pos0, hi = pos1 - 1;
+            while (lo < hi) {
+              const int64_t mid = (lo + hi + 1) >> 1;
+              if (soff[mid] <= t) lo = mid; else hi = mid - 1;
+            }
+            vv[q] = bv[lo];
+            e = rowptr[vv[q]] + (t - soff[lo]);
+          }
+          jj[q] = __ldcs(&col[e]);
+        }
+      }
+#pragma unroll
+      for (int q = 0; q < 4; ++q) rr[q] = (jj[q] >= 0 && jj[q] != vv[q]) ? __ldg(&ca[jj[q]]) : make_uint2(kSelf, 0);
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        const int64_t t = base + (int64_t)q * blockDim.x;
+        if (t < t1) stage[t] = (jj[q] == vv[q]) ? make_uint2(kSelf, 0u)
+                                                : make_uint2(rr[q].x, rr[q].x == (uint32_t)jj[q] ? rr[q].y : kUnknownA);
+      }
+    }
+    __syncthreads();
+  }
+}
+
+// Phase 2 insert: entries [t0, deg) step `stride` of one vertex's staged
+// neighbours S (and weights Wt), 4 per pass, no random loads.  With AGG,
+// labels are first merged across the warp (__match_any_sync, weights summed
+// with __reduce_add_sync): a label shared by many neighbours costs one table
+// atomic per warp.  The trip count is uniform across each warp.
 template <bool UNIT, bool AGG, bool GLOBAL = false>
-__device__ __forceinline__ void insert_row(unsigned long long* T, uint32_t* TA, uint32_t cap, int32_t v, int64_t rb,
-                                           int64_t deg, int64_t t0, int64_t stride, const SweepArgs& A) {
+__device__ __forceinline__ void insert_staged(unsigned long long* T, uint32_t* TA, uint32_t cap,
+                                              const uint2* __restrict__ S, const uint32_t* __restrict__ Wt,
+                                              int64_t deg, int64_t t0, int64_t stride) {
   const int lane = threadIdx.x & 31;
-  const int64_t t_warp0 = t0 - lane;  // first index handled by the warp in each pass
+  const int64_t t_warp0 = t0 - lane;
   for (int64_t base = 0; base + t_warp0 < deg; base += 4 * stride) {
-    int32_t jj[4];
-    uint32_t ww[4];
     uint2 rr[4];
+    uint32_t ww[4];
 #pragma unroll
     for (int q = 0; q < 4; ++q) {
       const int64_t t = base + t0 + q * stride;
-      jj[q] = (t < deg) ? __ldcs(&A.col[rb + t]) : -1;
-      ww[q] = UNIT ? 1u : ((t < deg) ? __ldcs(&A.w[rb + t]) : 0u);
+      rr[q] = (t < deg) ? __ldcs(&S[t]) : make_uint2(kSelf, 0u);
+      ww[q] = UNIT ? 1u : ((t < deg) ? __ldcs(&Wt[t]) : 0u);
     }
-#pragma unroll
-    for (int q = 0; q < 4; ++q) rr[q] = (jj[q] >= 0 && jj[q] != v) ? __ldg(&A.ca[jj[q]]) : make_uint2(0, 0);
     int32_t c[4];
     uint32_t x[4], arep[4];
     bool todo[4];
 #pragma unroll
     for (int q = 0; q < 4; ++q) {
-      const bool valid = jj[q] >= 0 && jj[q] != v;
-      const bool isrep = valid && (uint32_t)jj[q] == rr[q].x;
+      const bool valid = rr[q].x != kSelf;
       c[q] = valid ? (int32_t)rr[q].x : (int32_t)(0x80000000u | (unsigned)lane);
       if (AGG) {
         const unsigned m = __match_any_sync(kFull, c[q]);
         x[q] = UNIT ? (uint32_t)__popc(m) : __reduce_add_sync(m, ww[q]);
-        const unsigned rep = __ballot_sync(kFull, isrep) & m;
+        const unsigned rep = __ballot_sync(kFull, valid && rr[q].y != kUnknownA) & m;
         const uint32_t a_rep = __shfl_sync(kFull, rr[q].y, rep ? __ffs(rep) - 1 : lane);
         todo[q] = valid && lane == __ffs(m) - 1;
         arep[q] = rep ? a_rep : kUnknownA;
       } else {
         x[q] = ww[q];
         todo[q] = valid;
-        arep[q] = isrep ? rr[q].y : kUnknownA;
+        arep[q] = rr[q].y;
       }
     }
     if (GLOBAL) {
@@ -341,7 +429,9 @@ __device__ __forceinline__ void insert_row(unsigned long long* T, uint32_t* TA, 
 
 // ------------------------------------------------------------ warp per vertex
 template <int CAP, int WARPS, bool UNIT, bool AGG>
-__global__ void __launch_bounds__(32 * WARPS) sweep_warp(const int32_t* __restrict__ verts, int64_t nv, SweepArgs A) {
+__global__ void __launch_bounds__(32 * WARPS) sweep_warp(const int32_t* __restrict__ verts,
+                                                         const int64_t* __restrict__ soff, int64_t nv,
+                                                         const uint2* __restrict__ stage, SweepArgs A) {
   __shared__ unsigned long long tab[WARPS][CAP];
   __shared__ uint32_t taba[WARPS][CAP];
   const int lane = threadIdx.x & 31, wl = threadIdx.x >> 5;
@@ -359,7 +449,7 @@ __global__ void __launch_bounds__(32 * WARPS) sweep_warp(const int32_t* __restri
     const int64_t deg = __ldg(&A.rowptr[v + 1]) - rb;
     const int32_t own = (int32_t)__ldg(&A.ca[v]).x;
     const uint32_t ki = __ldg(&A.k[v]);
-    insert_row<UNIT, AGG>(T, TA, CAP, v, rb, deg, lane, 32, A);
+    insert_staged<UNIT, AGG>(T, TA, CAP, stage + __ldg(&soff[vi]), UNIT ? nullptr : A.w + rb, deg, lane, 32);
     __syncwarp();
     const bool own_single = A.rule == 2 && __ldg(&A.size[own]) == 1;
     long long s = (long long)0x8000000000000000ull;
@@ -376,7 +466,8 @@ __global__ void __launch_bounds__(32 * WARPS) sweep_warp(const int32_t* __restri
 
 // ------------------------------------------------------------ CTA per vertex
 template <bool UNIT, bool AGG>
-__global__ void __launch_bounds__(1024) sweep_cta(const int32_t* __restrict__ verts, int64_t nv, SweepArgs A,
+__global__ void __launch_bounds__(1024) sweep_cta(const int32_t* __restrict__ verts, const int64_t* __restrict__ soff,
+                                                  int64_t nv, const uint2* __restrict__ stage, SweepArgs A,
                                                   int capmax) {
   extern __shared__ unsigned long long smem[];
   unsigned long long* T = smem;
@@ -396,7 +487,8 @@ __global__ void __launch_bounds__(1024) sweep_cta(const int32_t* __restrict__ ve
     const int32_t own = (int32_t)__ldg(&A.ca[v]).x;
     const uint32_t ki = __ldg(&A.k[v]);
     const uint32_t cap = (uint32_t)((2 * deg < (int64_t)capmax) ? 2 * deg : (int64_t)capmax);
-    insert_row<UNIT, AGG>(T, TA, cap, v, rb, deg, threadIdx.x, blockDim.x, A);
+    insert_staged<UNIT, AGG>(T, TA, cap, stage + __ldg(&soff[vi]), UNIT ? nullptr : A.w + rb, deg, threadIdx.x,
+                             blockDim.x);
     __syncthreads();
     const bool own_single = A.rule == 2 && __ldg(&A.size[own]) == 1;
     long long s = (long long)0x8000000000000000ull;
@@ -415,13 +507,13 @@ __global__ void __launch_bounds__(1024) sweep_cta(const int32_t* __restrict__ ve
 
 // ------------------------------------------------------------ cluster per vertex
 // deg in [12288, 131072): the vertex's table (2*deg slots, load <= 1/2) is
-// spread over the distributed shared memory of a CS-CTA cluster (kClusterSlots
-// per CTA).  Each CTA inserts its share of the row into whichever CTA owns the
+// spread over the distributed shared memory of a CS-CTA cluster (slot g lives
+// in CTA g % CS at index g / CS, so every CTA holds an equal share).  Each CTA inserts its share of the row into whichever CTA owns the
 // slot (remote DSMEM CAS, ~200 cycles); cluster.sync(); each CTA scans its own
 // slots; partials meet in rank 0's shared memory; cluster.sync(); rank 0 decides.
 // Persistent: clusters stride over the class's vertices.
-__device__ __forceinline__ void dsm_insert4(cg::cluster_group& cl, unsigned long long* T, uint32_t* TA, uint32_t cap,
-                                            const int32_t c[4], const uint32_t x[4], bool todo[4],
+__device__ __forceinline__ void dsm_insert4(cg::cluster_group& cl, unsigned CS, unsigned long long* T, uint32_t* TA,
+                                            uint32_t cap, const int32_t c[4], const uint32_t x[4], bool todo[4],
                                             const uint32_t arep[4]) {
   uint32_t h[4];
 #pragma unroll
@@ -431,7 +523,7 @@ __device__ __forceinline__ void dsm_insert4(cg::cluster_group& cl, unsigned long
     unsigned long long* slot[4];
 #pragma unroll
     for (int q = 0; q < 4; ++q) {
-      slot[q] = cl.map_shared_rank(T + (h[q] % kClusterSlots), h[q] / kClusterSlots);
+      slot[q] = cl.map_shared_rank(T + (h[q] / CS), h[q] % CS);  // slots interleaved over the CTAs
       old[q] = todo[q] ? atomicCAS(slot[q], kEmpty, (((unsigned long long)(uint32_t)c[q]) << 32) | x[q]) : 0ull;
     }
 #pragma unroll
@@ -439,7 +531,7 @@ __device__ __forceinline__ void dsm_insert4(cg::cluster_group& cl, unsigned long
       if (!todo[q]) continue;
       if (old[q] == kEmpty || (old[q] >> 32) == (unsigned long long)(uint32_t)c[q]) {
         if (old[q] != kEmpty) atomicAdd(slot[q], (unsigned long long)x[q]);
-        if (arep[q] != kUnknownA) *cl.map_shared_rank(TA + (h[q] % kClusterSlots), h[q] / kClusterSlots) = arep[q];
+        if (arep[q] != kUnknownA) *cl.map_shared_rank(TA + (h[q] / CS), h[q] % CS) = arep[q];
         todo[q] = false;
       } else {
         h[q] = (h[q] + 1 == cap) ? 0 : h[q] + 1;
@@ -449,7 +541,9 @@ __device__ __forceinline__ void dsm_insert4(cg::cluster_group& cl, unsigned long
 }
 
 template <bool UNIT>
-__global__ void __launch_bounds__(1024, 1) sweep_cluster(const int32_t* __restrict__ verts, int64_t nv, SweepArgs A) {
+__global__ void __launch_bounds__(1024, 1) sweep_cluster(const int32_t* __restrict__ verts,
+                                                         const int64_t* __restrict__ soff, int64_t nv,
+                                                         const uint2* __restrict__ stage, SweepArgs A) {
   cg::cluster_group cl = cg::this_cluster();
   extern __shared__ unsigned long long smem[];
   unsigned long long* T = smem;
@@ -478,39 +572,35 @@ __global__ void __launch_bounds__(1024, 1) sweep_cluster(const int32_t* __restri
     const int64_t eb = rb + (int64_t)rank * per;
     const int64_t len = max((int64_t)0, min(per, rb + deg - eb));
     const int lane = threadIdx.x & 31;
+    const uint2* S = stage + __ldg(&soff[vi]) + (eb - rb);
     for (int64_t base = 0; base + (int64_t)(threadIdx.x - lane) < len; base += 4 * (int64_t)blockDim.x) {
-      int32_t jj[4];
-      uint32_t ww[4];
       uint2 rr[4];
+      uint32_t ww[4];
 #pragma unroll
       for (int q = 0; q < 4; ++q) {
         const int64_t t = base + threadIdx.x + (int64_t)q * blockDim.x;
-        jj[q] = (t < len) ? __ldcs(&A.col[eb + t]) : -1;
+        rr[q] = (t < len) ? __ldcs(&S[t]) : make_uint2(kSelf, 0u);
         ww[q] = UNIT ? 1u : ((t < len) ? __ldcs(&A.w[eb + t]) : 0u);
       }
-#pragma unroll
-      for (int q = 0; q < 4; ++q) rr[q] = (jj[q] >= 0 && jj[q] != v) ? __ldg(&A.ca[jj[q]]) : make_uint2(0, 0);
       int32_t c[4];
       uint32_t x[4], arep[4];
       bool todo[4];
 #pragma unroll
       for (int q = 0; q < 4; ++q) {
-        const bool valid = jj[q] >= 0 && jj[q] != v;
-        const bool isrep = valid && (uint32_t)jj[q] == rr[q].x;
+        const bool valid = rr[q].x != kSelf;
         c[q] = valid ? (int32_t)rr[q].x : (int32_t)(0x80000000u | (unsigned)lane);
         const unsigned m = __match_any_sync(kFull, c[q]);
         x[q] = UNIT ? (uint32_t)__popc(m) : __reduce_add_sync(m, ww[q]);
-        const unsigned rep = __ballot_sync(kFull, isrep) & m;
+        const unsigned rep = __ballot_sync(kFull, valid && rr[q].y != kUnknownA) & m;
         const uint32_t a_rep = __shfl_sync(kFull, rr[q].y, rep ? __ffs(rep) - 1 : lane);
         todo[q] = valid && lane == __ffs(m) - 1;
         arep[q] = rep ? a_rep : kUnknownA;
       }
-      dsm_insert4(cl, T, TA, cap, c, x, todo, arep);
+      dsm_insert4(cl, CS, T, TA, cap, c, x, todo, arep);
     }
     cl.sync();
-    // scan this CTA's slots of the table
-    const int64_t my_lo = (int64_t)rank * kClusterSlots;
-    const uint32_t my_n = (uint32_t)max((int64_t)0, min((int64_t)kClusterSlots, (int64_t)cap - my_lo));
+    // scan this CTA's slots of the table (global slots g with g % CS == rank)
+    const uint32_t my_n = (cap > rank) ? (cap - rank + CS - 1) / CS : 0u;
     const bool own_single = A.rule == 2 && __ldg(&A.size[own]) == 1;
     long long s = (long long)0x8000000000000000ull;
     int cb = 0x7FFFFFFF;
@@ -550,7 +640,7 @@ __global__ void __launch_bounds__(512) hub_coop(const HubItem* __restrict__ ins,
                                                 const int64_t* __restrict__ wave_hub,
                                                 const HubInfo* __restrict__ info, int64_t nwaves, int64_t seg,
                                                 unsigned long long* ring, uint32_t* ring_a, Partial* part,
-                                                SweepArgs A) {
+                                                const uint2* __restrict__ stage, SweepArgs A) {
   cg::grid_group grid = cg::this_grid();
   __shared__ long long sh_s[32];
   __shared__ int sh_c[32];
@@ -568,8 +658,9 @@ __global__ void __launch_bounds__(512) hub_coop(const HubItem* __restrict__ ins,
         const HubInfo hi = info[item.hub];
         unsigned long long* T = ring + (p & 1) * seg + hi.off;
         uint32_t* TA = ring_a + (p & 1) * seg + hi.off;
-        insert_row<UNIT, true, true>(T, TA, (uint32_t)hi.cap, hi.v, item.begin, item.end - item.begin, threadIdx.x,
-                                     blockDim.x, A);
+        insert_staged<UNIT, true, true>(T, TA, (uint32_t)hi.cap, stage + hi.sbase + item.begin,
+                                        UNIT ? nullptr : A.w + item.begin, item.end - item.begin, threadIdx.x,
+                                        blockDim.x);
       } else if (it < nI + nS) {
         const int64_t q = scan_off[p - 1] + (it - nI);
         const HubItem item = scans[q];
@@ -651,6 +742,8 @@ int32_t dispatch_class(Handle& h, Level& L, const SweepArgs& A, int bucket, int 
   const int64_t nv = L.class_off[kSubPerBucket * bucket + sub + 1] - off;
   if (nv <= 0) return LOUVAIN_OK;
   const int32_t* verts = L.bin_vertices + off;
+  const int64_t* soff = L.soff + off;
+  const uint2* stage = L.stage;
   cudaStream_t s = h.stream;
   if (sub == 0 && max_deg <= 32) {
     const int G = max_deg <= 4 ? 4 : max_deg <= 8 ? 8 : max_deg <= 16 ? 16 : 32;
@@ -663,10 +756,10 @@ int32_t dispatch_class(Handle& h, Level& L, const SweepArgs& A, int bucket, int 
     }
     LV_LAUNCHED();
   } else if (sub == 0 && max_deg <= 84) {
-    sweep_warp<128, 8, UNIT, AGG><<<grid_for(nv, 8, 148 * 8), 256, 0, s>>>(verts, nv, A);
+    sweep_warp<128, 8, UNIT, AGG><<<grid_for(nv, 8, 148 * 8), 256, 0, s>>>(verts, soff, nv, stage, A);
     LV_LAUNCHED();
   } else if (sub == 0 && max_deg <= 340) {
-    sweep_warp<512, 4, UNIT, AGG><<<grid_for(nv, 4, 148 * 12), 128, 0, s>>>(verts, nv, A);
+    sweep_warp<512, 4, UNIT, AGG><<<grid_for(nv, 4, 148 * 12), 128, 0, s>>>(verts, soff, nv, stage, A);
     LV_LAUNCHED();
   } else if (sub == 3 || sub == 4) {
     const int CS = (sub == 3) ? 4 : 16;
@@ -698,7 +791,7 @@ int32_t dispatch_class(Handle& h, Level& L, const SweepArgs& A, int bucket, int 
     }
     const int64_t ncl = std::min<int64_t>(mc, nv);
     cfg.gridDim = dim3((unsigned)(ncl * CS), 1, 1);
-    LV_CUDA(cudaLaunchKernelEx(&cfg, sweep_cluster<UNIT>, verts, nv, A));
+    LV_CUDA(cudaLaunchKernelEx(&cfg, sweep_cluster<UNIT>, verts, soff, nv, stage, A));
     LV_LAUNCHED();
   } else if (sub <= 2) {
     static const int caps[3] = {kCap0, kCap1, kCap2};
@@ -714,7 +807,7 @@ int32_t dispatch_class(Handle& h, Level& L, const SweepArgs& A, int bucket, int 
       attr_done = true;
     }
     const unsigned grid = grid_for(nv, 1, 148 * per_sm[sub]);
-    sweep_cta<UNIT, AGG><<<grid, threads[sub], smem, s>>>(verts, nv, A, caps[sub]);
+    sweep_cta<UNIT, AGG><<<grid, threads[sub], smem, s>>>(verts, soff, nv, stage, A, caps[sub]);
     LV_LAUNCHED();
   } else {
     HubPlan& P = L.hub;
@@ -735,8 +828,9 @@ int32_t dispatch_class(Handle& h, Level& L, const SweepArgs& A, int bucket, int 
       unsigned long long* a8 = P.ring;
       uint32_t* a9 = P.ring_a;
       Partial* a10 = (Partial*)P.partial;
-      SweepArgs a11 = A;
-      void* args[] = {&a0, &a1, &a2, &a3, &a4, &a5, &a6, &a7, &a8, &a9, &a10, &a11};
+      const uint2* a11 = stage;
+      SweepArgs a12 = A;
+      void* args[] = {&a0, &a1, &a2, &a3, &a4, &a5, &a6, &a7, &a8, &a9, &a10, &a11, &a12};
       LV_CUDA(cudaLaunchCooperativeKernel((void*)hub_coop<UNIT>, P.grid, 512, args, 0, s));
       LV_LAUNCHED();
     }
@@ -748,6 +842,13 @@ int32_t dispatch_class(Handle& h, Level& L, const SweepArgs& A, int bucket, int 
 }  // namespace
 
 size_t hub_partial_bytes() { return sizeof(Partial); }
+
+int32_t launch_stage(Handle& h, Level& L, int64_t pos0, int64_t pos1) {
+  k_stage<<<148 * 8, 256, 0, h.stream>>>(L.bin_vertices, L.soff, pos0, pos1, L.rowptr, L.col, L.ca, L.stage);
+  LV_LAUNCHED();
+  LV_CUDA(cudaGetLastError());
+  return LOUVAIN_OK;
+}
 
 // All kernels of bucket `bucket` (1..7).  Bucket b's degree range is
 // (bounds[b-2], bounds[b-1]] with bounds[-1] = 0 and bounds[6] = inf.
@@ -765,6 +866,13 @@ int32_t launch_sweep_bucket(Handle& h, Level& L, const louvain_params_t& p, int 
   A.mv_new = L.mv_new;
   A.logn = &h.ctl->logn;
   const int64_t hi = (bucket <= 6) ? p.deg_bounds[bucket - 1] : INT64_MAX;
+  // phase 1: gather the records of every neighbour of the bucket's table-based vertices
+  {
+    const bool sub0_small = std::min<int64_t>(hi, kSub1Min - 1) <= 32;
+    const int64_t pos0 = L.class_off[kSubPerBucket * bucket + (sub0_small ? 1 : 0)];
+    const int64_t pos1 = L.class_off[kSubPerBucket * (bucket + 1)];
+    if (pos1 > pos0) LV_TRY(launch_stage(h, L, pos0, pos1));
+  }
   for (int sub = 0; sub < 6; ++sub) {
     const int64_t max_deg = (sub == 0) ? std::min<int64_t>(hi, kSub1Min - 1) : hi;
     // warp-level label merging pays once communities exist (hot labels); on the
