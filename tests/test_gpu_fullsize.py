@@ -1,0 +1,118 @@
+"""Full-size parity (BASELINE.json configs, the launch configuration bench.py times).
+
+* C5 (R-MAT scale 27, 2.1e9 entries) and C3 (scale 24): one BIN_SYNC sweep from
+  singletons on the GPU; the oracle then recomputes computeMove (Alg. 2) for
+  sampled vertices of EVERY bucket against that bucket's snapshot, reconstructed
+  exactly: at sweep 1 a vertex of a bucket < b carries its committed label, every
+  other vertex still its own (each vertex moves at most once per sweep).  The
+  modularity numerators after the sweep are checked against the oracle's Eq. (1)
+  on the whole graph (exact integers).
+* Whole runs on the configs of tests/golden/oracle_runs.json (written by
+  tools/make_golden.py from oracle/ only): exact numerators, levels, sweeps per
+  level and the sha256 of the labels; and the north-star quality bar
+  |Q_gpu - Q_oracle(a)| <= 0.005 reported per config.
+"""
+import hashlib
+import json
+import os
+
+import numpy as np
+import pytest
+
+import graphgen
+import oracle
+from conftest import cuda_ok
+
+pytestmark = [pytest.mark.gpu, pytest.mark.skipif(not cuda_ok(), reason="needs a CUDA device")]
+lvb = pytest.importorskip("paper_conf_ipps_naimmht17_b200")
+GOLD = os.path.join(os.path.dirname(__file__), "golden", "oracle_runs.json")
+
+
+def _bucket_ids(deg, bounds):
+    b = np.zeros(len(deg), dtype=np.int8)
+    b[deg > 0] = 7
+    for t in range(5, -1, -1):
+        b[(deg > 0) & (deg <= bounds[t])] = t + 1
+    return b
+
+
+@pytest.mark.parametrize("scale", [24, 27])
+def test_sweep1_sampled_decisions_full_size(scale):
+    import torch
+    dg = graphgen.rmat(scale, seed=1, device=True)
+    g = lvb.Graph.from_csr(dg.rowptr, dg.col, borrow=True)
+    p = lvb.params()
+    moved, q = g.sweep(p)
+    C1 = g.labels()
+    hg = dg.to_host()
+    del dg
+    torch.cuda.empty_cache()
+    n = hg.n
+    deg = np.diff(hg.rowptr)
+    W = int(deg.sum())
+    bucket = _bucket_ids(deg, list(p.deg_bounds))
+    rng = np.random.default_rng(scale)
+    iota = np.arange(n, dtype=np.int32)
+    changed = int(np.count_nonzero(C1 != iota))
+    assert changed == moved
+    checked = 0
+    for b in range(1, 8):
+        members = np.flatnonzero(bucket == b)
+        if len(members) == 0:
+            continue
+        # sample: 1500 random vertices of the bucket plus its largest-degree ones (hub paths)
+        top = members[np.argsort(deg[members])[-200:]]
+        sample = np.unique(np.concatenate([rng.choice(members, size=min(1500, len(members)), replace=False), top]))
+        snap = np.where(bucket < b, C1, iota).astype(np.int32)
+        a, size = oracle.totals(hg, snap)
+        got = C1[sample]
+        want = oracle.decide_batch(hg, snap, a, size, W, sample.astype(np.int64), p.singleton_rule)
+        bad = np.flatnonzero(got != want)
+        assert len(bad) == 0, f"bucket {b}: {len(bad)} of {len(sample)} differ, e.g. v={sample[bad[:5]]}"
+        checked += len(sample)
+    assert checked > 5000
+    L, S, W2 = oracle.modularity(hg, C1)
+    assert (int(q.L), q.S, int(q.W)) == (L, S, W2)
+
+
+def _golden():
+    if not os.path.exists(GOLD):
+        return {}
+    with open(GOLD) as f:
+        return json.load(f)
+
+
+BUILD = {
+    "C1": lambda: graphgen.karate(),
+    "C2-small": lambda: graphgen.lfr(20_000, seed=1),
+    "C3-small": lambda: graphgen.rmat(16, seed=1),
+    "C4a-small": lambda: graphgen.mesh3d(40, True),
+    "C4b-small": lambda: graphgen.rgg(200_000, seed=1),
+    "C3-s20": lambda: graphgen.rmat(20, seed=1),
+    "C2": lambda: graphgen.lfr(1_000_000, seed=1),
+    "C3": lambda: graphgen.rmat(24, seed=1, device=True),
+}
+
+
+@pytest.mark.parametrize("name", list(BUILD))
+def test_full_run_matches_stored_oracle(name):
+    gold = _golden().get(name)
+    if gold is None:
+        pytest.skip(f"{name} not in tests/golden/oracle_runs.json")
+    g = BUILD[name]()
+    gd = lvb.Graph.from_csr(g.rowptr, g.col, getattr(g, "w", None), borrow=hasattr(g, "to_host"))
+    lab, q, st = gd.run(lvb.params(), labels_out=None)
+    ref = gold["b"]
+    assert st["levels"] == ref["levels"] and st["sweeps_per_level"] == ref["sweeps_per_level"]
+    assert st["num_start"] == ref["num_start"] and st["num_end"] == ref["num_end"]
+    assert (int(q.L), q.S, int(q.W)) == (ref["L"], ref["S"], ref["W"])
+    assert hashlib.sha256(np.ascontiguousarray(lab, dtype=np.int32).tobytes()).hexdigest() == ref["labels_sha256"]
+
+
+def test_quality_bar_report():
+    """North-star bar |Q(b) - Q(a)| <= 0.005 (the GPU equals oracle (b) exactly, checked above).
+    Configs that miss it are reported in DESIGN.md; this test pins the small configs."""
+    gold = _golden()
+    for name in ("C1", "C2-small", "C3-small", "C4a-small", "C4b-small", "C2"):
+        if name in gold:
+            assert abs(gold[name]["gap_a_minus_b"]) <= 0.005, name
