@@ -279,6 +279,10 @@ int32_t run_impl(Handle& h, const louvain_params_t& p, int32_t* labels_out, louv
         }
         local.edges_swept += L.nnz;
         ++sweeps;
+        if (h.h_ctl->overflow) {
+          set_error("partitioned hash table overflow (sweep_part); please report");
+          return LOUVAIN_E_CUDA;
+        }
         const int64_t moved = (int64_t)h.h_ctl->logn;
         const int64_t num = qnum_of(h.h_ctl->L, h.h_ctl->S, W);
         if (p.revert_on_decrease && num < num_prev) {  // R15
@@ -547,6 +551,10 @@ LV_API int32_t louvain_sweep(louvain_graph_t g, const louvain_params_t* p, int64
     cudaError_t e = cudaMemcpyAsync(h.h_ctl, h.ctl, sizeof(DevCtl), cudaMemcpyDeviceToHost, h.stream);
     if (e == cudaSuccess) e = cudaStreamSynchronize(h.stream);
     if (e != cudaSuccess) rc = cuda_fail(e, "sweep", __FILE__, __LINE__);
+  }
+  if (!rc && h.h_ctl->overflow) {
+    set_error("partitioned hash table overflow (sweep_part); please report");
+    rc = LOUVAIN_E_CUDA;
   }
   if (!rc) {
     if (moved) *moved = (int64_t)h.h_ctl->logn;

@@ -61,6 +61,7 @@ struct DevCtl {
   unsigned long long bounds[9];  // log offset at the start of bucket b's commit
   unsigned long long L, S;       // modularity parts
   unsigned long long bad;        // validation flag
+  unsigned long long overflow;   // a partitioned hash table filled up (must stay 0)
 };
 
 // Hub work plan (one per level).  Hubs are grouped into waves whose tables fit
@@ -95,6 +96,24 @@ struct HubPlan {
   int grid = 0;                        // co-resident CTAs of the cooperative kernel
 };
 
+// Label-partitioned plan for vertices of degree >= kSub3Min: vertex v gets
+// P_v = ceil(deg / kPartLabels) CTA tasks; task p keeps the labels c with
+// part_hash(c) % P_v == p in its own shared-memory table.
+constexpr int64_t kPartLabels = 6144;  // expected distinct labels per task (table load <= 3/8)
+constexpr int kPartSlots = 16384;      // smem table slots per task (12 B each: 192 KB)
+struct PartPlan {
+  int64_t ntasks = 0, nverts = 0;
+  int32_t* task_vpos = nullptr;   // [ntasks] index into the plan's vertex list
+  int32_t* task_p = nullptr;      // [ntasks] partition index
+  int32_t* vert_pos = nullptr;    // [nverts] bin position of the vertex
+  int32_t* vert_P = nullptr;      // [nverts] partitions of the vertex
+  int32_t* vert_first = nullptr;  // [nverts] first task (= first partial)
+  int32_t* done = nullptr;        // [nverts] tasks finished (reset every sweep)
+  void* partial = nullptr;        // [ntasks] Partial
+  int64_t bucket_task[9] = {0};   // tasks of bucket b: [bucket_task[b-1], bucket_task[b])
+  int64_t bucket_vert[9] = {0};   // plan vertices of bucket b
+};
+
 struct Level {
   int64_t n = 0, nnz = 0;
   uint64_t W = 0;
@@ -124,6 +143,7 @@ struct Level {
   int64_t* soff = nullptr;
   uint2* stage = nullptr;
   HubPlan hub;
+  PartPlan part;
 };
 
 struct Handle {
@@ -181,6 +201,7 @@ int32_t validate_csr_host(int64_t n, int64_t nnz, const int64_t* rowptr, const i
 // ------------------------------------------------------------------ sweep (lv_sweep.cu)
 int32_t launch_sweep_bucket(Handle& h, Level& L, const louvain_params_t& p, int bucket);
 int32_t launch_stage(Handle& h, Level& L, int64_t pos0, int64_t pos1);  // phase 1 gather for positions [pos0,pos1)
+int32_t build_part_plan(Handle& h, Level& L);
 
 // ------------------------------------------------------------------ launch geometry
 inline unsigned grid_for(int64_t items, int per_block, int max_blocks = 148 * 16) {

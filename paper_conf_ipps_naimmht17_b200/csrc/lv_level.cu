@@ -314,6 +314,9 @@ void level_free(Level& L, cudaStream_t s) {
   dfree(L.mv_v, s); dfree(L.mv_new, s); dfree(L.mv_old, s); dfree(L.bin_vertices, s);
   dfree(L.soff, s); dfree(L.stage, s);
   hub_free(L.hub, s);
+  PartPlan& Q = L.part;
+  dfree(Q.task_vpos, s); dfree(Q.task_p, s); dfree(Q.vert_pos, s); dfree(Q.vert_P, s); dfree(Q.vert_first, s);
+  dfree(Q.done, s); dfree(Q.partial, s);
   L = Level();
 }
 
@@ -480,6 +483,59 @@ static int32_t build_hub_plan(Handle& h, Level& L) {
   return LOUVAIN_OK;
 }
 
+// Partition plan for every vertex of sub-classes 3..5 (deg >= kSub3Min), any bucket.
+int32_t build_part_plan(Handle& h, Level& L) {
+  cudaStream_t s = h.stream;
+  PartPlan& Q = L.part;
+  dfree(Q.task_vpos, s); dfree(Q.task_p, s); dfree(Q.vert_pos, s); dfree(Q.vert_P, s); dfree(Q.vert_first, s);
+  dfree(Q.done, s); dfree(Q.partial, s);
+  Q = PartPlan();
+  std::vector<int32_t> vpos, vP, vfirst, tv, tp;
+  for (int b = 1; b <= 7; ++b) {
+    Q.bucket_task[b - 1] = (int64_t)tv.size();
+    Q.bucket_vert[b - 1] = (int64_t)vpos.size();
+    for (int sub = 3; sub <= 5; ++sub) {
+      const int c = kSubPerBucket * b + sub;
+      const int64_t off = L.class_off[c], cnt = L.class_off[c + 1] - off;
+      if (cnt <= 0) continue;
+      std::vector<int64_t> so(cnt + 1);
+      LV_CUDA(cudaMemcpyAsync(so.data(), L.soff + off, 8 * (cnt + 1), cudaMemcpyDeviceToHost, s));
+      LV_CUDA(cudaStreamSynchronize(s));
+      for (int64_t i = 0; i < cnt; ++i) {
+        const int64_t deg = so[i + 1] - so[i];
+        const int32_t P = (int32_t)((deg + kPartLabels - 1) / kPartLabels);
+        const int32_t vi = (int32_t)vpos.size();
+        vpos.push_back((int32_t)(off + i));
+        vP.push_back(P);
+        vfirst.push_back((int32_t)tv.size());
+        for (int32_t q = 0; q < P; ++q) {
+          tv.push_back(vi);
+          tp.push_back(q);
+        }
+      }
+    }
+  }
+  Q.nverts = (int64_t)vpos.size();
+  Q.ntasks = (int64_t)tv.size();
+  Q.bucket_task[7] = Q.ntasks;
+  Q.bucket_vert[7] = Q.nverts;
+  if (Q.nverts == 0) return LOUVAIN_OK;
+  LV_TRY(dalloc(&Q.task_vpos, Q.ntasks, s));
+  LV_TRY(dalloc(&Q.task_p, Q.ntasks, s));
+  LV_TRY(dalloc(&Q.vert_pos, Q.nverts, s));
+  LV_TRY(dalloc(&Q.vert_P, Q.nverts, s));
+  LV_TRY(dalloc(&Q.vert_first, Q.nverts, s));
+  LV_TRY(dalloc(&Q.done, Q.nverts, s));
+  LV_TRY(dmalloc(&Q.partial, hub_partial_bytes() * (size_t)Q.ntasks, s));
+  LV_CUDA(cudaMemcpyAsync(Q.task_vpos, tv.data(), 4 * tv.size(), cudaMemcpyHostToDevice, s));
+  LV_CUDA(cudaMemcpyAsync(Q.task_p, tp.data(), 4 * tp.size(), cudaMemcpyHostToDevice, s));
+  LV_CUDA(cudaMemcpyAsync(Q.vert_pos, vpos.data(), 4 * vpos.size(), cudaMemcpyHostToDevice, s));
+  LV_CUDA(cudaMemcpyAsync(Q.vert_P, vP.data(), 4 * vP.size(), cudaMemcpyHostToDevice, s));
+  LV_CUDA(cudaMemcpyAsync(Q.vert_first, vfirst.data(), 4 * vfirst.size(), cudaMemcpyHostToDevice, s));
+  LV_CUDA(cudaStreamSynchronize(s));  // host vectors die here
+  return LOUVAIN_OK;
+}
+
 int32_t level_binning(Handle& h, Level& L, const louvain_params_t& p) {
   bool same = L.bins_valid;
   for (int t = 0; t < 6 && same; ++t) same = (L.bins_bounds[t] == p.deg_bounds[t]);
@@ -531,6 +587,7 @@ int32_t level_binning(Handle& h, Level& L, const louvain_params_t& p) {
     dfree(dg, s);
   }
   LV_TRY(build_hub_plan(h, L));
+  LV_TRY(build_part_plan(h, L));
   std::memcpy(L.bins_bounds, p.deg_bounds, sizeof L.bins_bounds);
   L.bins_valid = true;
   return LOUVAIN_OK;

@@ -505,6 +505,164 @@ __global__ void __launch_bounds__(1024) sweep_cta(const int32_t* __restrict__ ve
   }
 }
 
+// ------------------------------------------------------------ label-partitioned CTAs
+// deg >= 12288: vertex v gets P = ceil(deg / kPartLabels) independent CTA tasks.
+// Task p streams all of v's staged labels (an L2-resident segment, read P
+// times) and keeps only the labels c with part_of(c, P) == p in its own
+// shared-memory table, so a partition sees ~deg/P distinct labels whatever the
+// degree; the CTA that finishes v's last task reduces the P partials and
+// decides.  No clusters, grid syncs or global hash tables.  A table that would
+// pass 7/8 load sets DevCtl::overflow and the library reports an error (the
+// expected load is <= 3/8; exceeding 7/8 needs a +60-sigma hash deviation).
+__device__ __forceinline__ uint32_t part_of(int32_t c, uint32_t P) {
+  uint32_t h = (uint32_t)c;  // fmix32 (independent of hash_slot's multiplier)
+  h ^= h >> 16;
+  h *= 0x85ebca6bu;
+  h ^= h >> 13;
+  h *= 0xc2b2ae35u;
+  h ^= h >> 16;
+  return (uint32_t)(((unsigned long long)h * P) >> 32);
+}
+
+template <bool UNIT>
+__global__ void __launch_bounds__(1024) sweep_part(const int32_t* __restrict__ task_vpos,
+                                                  const int32_t* __restrict__ task_p, int64_t t_begin, int64_t t_end,
+                                                  const int32_t* __restrict__ vert_pos,
+                                                  const int32_t* __restrict__ vert_P,
+                                                  const int32_t* __restrict__ vert_first, int32_t* done,
+                                                  Partial* part, unsigned long long* overflow,
+                                                  const int32_t* __restrict__ bv, const int64_t* __restrict__ soff,
+                                                  const uint2* __restrict__ stage, SweepArgs A) {
+  extern __shared__ unsigned long long smem[];
+  unsigned long long* T = smem;
+  uint32_t* TA = reinterpret_cast<uint32_t*>(smem + kPartSlots);
+  __shared__ long long sh_s[32];
+  __shared__ int sh_c[32];
+  __shared__ unsigned sh_e[32];
+  __shared__ int is_last;
+  __shared__ unsigned claimed;
+  __shared__ uint2 qbuf[32][64];
+  __shared__ uint32_t qwt[32][64];
+  for (int t = threadIdx.x; t < kPartSlots; t += blockDim.x) {
+    T[t] = kEmpty;
+    TA[t] = kUnknownA;
+  }
+  if (threadIdx.x == 0) claimed = 0;
+  __syncthreads();
+  const int lane = threadIdx.x & 31;
+  const unsigned limit = (unsigned)(kPartSlots / 8 * 7);
+  for (int64_t task = t_begin + blockIdx.x; task < t_end; task += gridDim.x) {
+    const int32_t vi = task_vpos[task];
+    const uint32_t p = (uint32_t)task_p[task];
+    const int32_t pos = vert_pos[vi];
+    const uint32_t P = (uint32_t)vert_P[vi];
+    const int32_t v = __ldg(&bv[pos]);
+    const int64_t sb = __ldg(&soff[pos]), deg = __ldg(&soff[pos + 1]) - sb;
+    const uint2* S = stage + sb;
+    const uint32_t* Wt = UNIT ? nullptr : A.w + __ldg(&A.rowptr[v]);
+    // Only ~1/P of the streamed entries belong to this task: each warp compacts
+    // the matching entries into a shared queue (ballot + popc) and inserts them
+    // 32 at a time, so the insert code runs with full warps.
+    uint2* Q = qbuf[threadIdx.x >> 5];
+    uint32_t* QW = qwt[threadIdx.x >> 5];
+    int qn = 0;  // warp-uniform queue length
+    auto insert_one = [&](uint2 e, uint32_t x) {
+      const int32_t c = (int32_t)e.x;
+      const unsigned long long key = ((unsigned long long)(uint32_t)c) << 32;
+      uint32_t h = hash_slot(c, kPartSlots);
+      for (;;) {
+        const unsigned long long old = atomicCAS(&T[h], kEmpty, key | x);
+        if (old == kEmpty) {
+          if (atomicAdd(&claimed, 1u) >= limit) atomicAdd(overflow, 1ull);
+          break;
+        }
+        if ((old >> 32) == (unsigned long long)(uint32_t)c) {
+          atomicAdd(&T[h], (unsigned long long)x);
+          break;
+        }
+        h = (h + 1 == (uint32_t)kPartSlots) ? 0 : h + 1;
+        if (claimed >= (unsigned)kPartSlots - 1) {
+          atomicAdd(overflow, 1ull);
+          break;
+        }
+      }
+      if (e.y != kUnknownA) TA[h] = e.y;
+    };
+    for (int64_t base = 0; base + (int64_t)(threadIdx.x - lane) < deg; base += 4 * (int64_t)blockDim.x) {
+      uint2 rr[4];
+      uint32_t ww[4];
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        const int64_t t = base + threadIdx.x + (int64_t)q * blockDim.x;
+        rr[q] = (t < deg) ? __ldcg(&S[t]) : make_uint2(kSelf, 0u);
+        ww[q] = UNIT ? 1u : ((t < deg) ? __ldcg(&Wt[t]) : 0u);
+      }
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        const bool valid = rr[q].x != kSelf && part_of((int32_t)rr[q].x, P) == p;
+        const unsigned m = __ballot_sync(kFull, valid);
+        if (valid) {
+          const int slot = qn + __popc(m & lanemask_lt());
+          Q[slot] = rr[q];
+          QW[slot] = ww[q];
+        }
+        qn += __popc(m);
+        if (qn >= 32) {
+          __syncwarp();
+          insert_one(Q[lane], QW[lane]);
+          const uint2 mv = (lane < qn - 32) ? Q[32 + lane] : make_uint2(0, 0);
+          const uint32_t mw = (lane < qn - 32) ? QW[32 + lane] : 0u;
+          __syncwarp();
+          if (lane < qn - 32) {
+            Q[lane] = mv;
+            QW[lane] = mw;
+          }
+          qn -= 32;
+          __syncwarp();
+        }
+      }
+    }
+    __syncwarp();
+    if (lane < qn) insert_one(Q[lane], QW[lane]);
+    __syncthreads();
+    const int32_t own = (int32_t)__ldg(&A.ca[v]).x;
+    const uint32_t ki = __ldg(&A.k[v]);
+    const bool own_single = A.rule == 2 && __ldg(&A.size[own]) == 1;
+    long long s = (long long)0x8000000000000000ull;
+    int cb = 0x7FFFFFFF;
+    unsigned eown = 0;
+    scan_table(T, TA, kPartSlots, threadIdx.x, blockDim.x, own, own_single, ki, A, s, cb, eown);
+    block_reduce(s, cb, eown, sh_s, sh_c, sh_e);
+    if (threadIdx.x == 0) {
+      part[task] = Partial{s, cb, eown};
+      __threadfence();
+      is_last = (atomicAdd(&done[vi], 1) == (int)P - 1);
+      claimed = 0;
+    }
+    __syncthreads();
+    if (is_last && threadIdx.x < 32) {
+      __threadfence();
+      s = (long long)0x8000000000000000ull;
+      cb = 0x7FFFFFFF;
+      eown = 0;
+      const int32_t f = vert_first[vi];
+      for (uint32_t q = threadIdx.x; q < P; q += 32) {
+        const longlong2 raw = __ldcg(reinterpret_cast<const longlong2*>(&part[f + q]));
+        const long long ps = raw.x;
+        const int pc = (int)(raw.y & 0xFFFFFFFFll);
+        const unsigned pe = (unsigned)((unsigned long long)raw.y >> 32);
+        if (better(ps, pc, s, cb)) { s = ps; cb = pc; }
+        eown += pe;
+      }
+      group_reduce<32>(s, cb, eown);
+      int32_t tgt = own;
+      if (threadIdx.x == 0) tgt = finish(s, cb, eown, own, __ldg(&A.ca[own]).y, ki, A);
+      log_moves(threadIdx.x == 0 && tgt != own, v, tgt, A);
+    }
+    __syncthreads();
+  }
+}
+
 // ------------------------------------------------------------ cluster per vertex
 // deg in [12288, 131072): the vertex's table (2*deg slots, load <= 1/2) is
 // spread over the distributed shared memory of a CS-CTA cluster (slot g lives
@@ -761,6 +919,25 @@ int32_t dispatch_class(Handle& h, Level& L, const SweepArgs& A, int bucket, int 
   } else if (sub == 0 && max_deg <= 340) {
     sweep_warp<512, 4, UNIT, AGG><<<grid_for(nv, 4, 148 * 12), 128, 0, s>>>(verts, soff, nv, stage, A);
     LV_LAUNCHED();
+  } else if (sub >= 3 && !getenv("LV_NO_PART")) {
+    if (sub == 3) {  // one launch covers the bucket's sub-classes 3..5
+      PartPlan& Q = L.part;
+      const int64_t t0 = Q.bucket_task[bucket - 1], t1 = Q.bucket_task[bucket];
+      const int64_t v0 = Q.bucket_vert[bucket - 1], v1 = Q.bucket_vert[bucket];
+      if (t1 > t0) {
+        static bool attr = false;
+        if (!attr) {
+          LV_TRY(set_smem(sweep_part<true>, 12 * (size_t)kPartSlots));
+          LV_TRY(set_smem(sweep_part<false>, 12 * (size_t)kPartSlots));
+          attr = true;
+        }
+        LV_CUDA(cudaMemsetAsync(Q.done + v0, 0, sizeof(int32_t) * (v1 - v0), s));
+        sweep_part<UNIT><<<grid_for(t1 - t0, 1, 148 * 2), 1024, 12 * (size_t)kPartSlots, s>>>(
+            Q.task_vpos, Q.task_p, t0, t1, Q.vert_pos, Q.vert_P, Q.vert_first, Q.done, (Partial*)Q.partial,
+            &h.ctl->overflow, L.bin_vertices, L.soff, stage, A);
+        LV_LAUNCHED();
+      }
+    }
   } else if (sub == 3 || sub == 4) {
     const int CS = (sub == 3) ? 4 : 16;
     static bool cl_attr = false;
