@@ -6,6 +6,8 @@
 
 #include <algorithm>
 #include <chrono>
+#include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <string>
 #include <vector>
@@ -183,6 +185,20 @@ int32_t sweep_body(Handle& h, Level& L, const louvain_params_t& p) {
 
 using i128 = __int128;
 
+// LV_TRACE=1: per-level phase timeline on stderr (host wall clock after a stream sync)
+struct Trace {
+  bool on = getenv("LV_TRACE") != nullptr;
+  std::chrono::steady_clock::time_point t0 = std::chrono::steady_clock::now();
+  void mark(cudaStream_t s, const char* what, int level) {
+    if (!on) return;
+    cudaStreamSynchronize(s);
+    const auto t1 = std::chrono::steady_clock::now();
+    fprintf(stderr, "[lv] level %d %-12s %9.3f ms\n", level, what,
+            std::chrono::duration<double, std::milli>(t1 - t0).count());
+    t0 = t1;
+  }
+};
+
 i128 pow10_i128(int p) {
   i128 r = 1;
   for (int t = 0; t < p; ++t) r *= 10;
@@ -243,6 +259,7 @@ int32_t run_impl(Handle& h, const louvain_params_t& p, int32_t* labels_out, louv
   Level owned;   // current contracted level (levels >= 1)
   Level* cur = &L0;
   int32_t* map = nullptr;
+  Trace tr;
   if (W > 0) {
     for (int level = 0;; ++level) {
       if ((p.max_levels > 0 && level >= p.max_levels) || level >= LOUVAIN_MAX_LEVELS) break;
@@ -252,7 +269,9 @@ int32_t run_impl(Handle& h, const louvain_params_t& p, int32_t* labels_out, louv
       cudaEventRecord(e_lvl0, s);
       Level& L = *cur;
       const int pexp = (L.n > p.size_limit) ? p.th_bin_exp : p.th_final_exp;  // P:330, R14
+      tr.mark(s, "start", level);
       LV_TRY(level_binning(h, L, p));
+      tr.mark(s, "binning", level);
       // level start: singletons.  Level 0 evaluates Eq. (1); a contracted level
       // starts exactly where the previous one ended (contraction preserves L and
       // S, R18 -- pinned by the oracle tests and the parity suite).
@@ -266,8 +285,10 @@ int32_t run_impl(Handle& h, const louvain_params_t& p, int32_t* labels_out, louv
         cudaEventRecord(h.ev[0], s);
         LV_TRY(sweep_body(h, L, p));
         cudaEventRecord(h.ev[1], s);
+        tr.mark(s, "sweep", level);
         LV_TRY(launch_modularity(h, L, nullptr));
         cudaEventRecord(h.ev[2], s);
+        tr.mark(s, "modularity", level);
         LV_CUDA(cudaMemcpyAsync(h.h_ctl, h.ctl, sizeof(DevCtl), cudaMemcpyDeviceToHost, s));
         LV_CUDA(cudaStreamSynchronize(s));
         const float t_sw = elapsed(h.ev[0], h.ev[1]);
@@ -317,11 +338,14 @@ int32_t run_impl(Handle& h, const louvain_params_t& p, int32_t* labels_out, louv
       cudaEventRecord(e_lvl0, s);
       Level next;
       LV_TRY(dalloc(&map, L.n, s));
+      tr.mark(s, "pre-contract", level);
       LV_TRY(level_contract(h, L, next, map));
+      tr.mark(s, "contract", level);
       LV_TRY(compose_labels(h, lab, n0, map));
       dfree(map, s);
       map = nullptr;
       LV_TRY(level_setup(h, next));
+      tr.mark(s, "setup", level);
       cudaEventRecord(e_lvl1, s);
       LV_CUDA(cudaEventSynchronize(e_lvl1));
       local.t_agg_ms[level] = elapsed(e_lvl0, e_lvl1);

@@ -41,12 +41,13 @@ int32_t cuda_fail(cudaError_t e, const char* what, const char* file, int line);
 //   sub 0: deg < 1024   (register / warp / 256-thread CTA kernels, by bucket bound)
 //   sub 1: [1024, 4096) 512-thread CTA, smem table <= 8192 slots
 //   sub 2: [4096,12288) 1024-thread CTA, smem table <= 16384 slots
-//   sub 3: [12288, 32768)   4-CTA cluster, table in distributed shared memory
-//   sub 4: [32768, 131072)  16-CTA cluster, table in distributed shared memory
-//   sub 5: >= 131072        hub: cooperative grid, global table in an L2-sized ring
+//   sub 3: [12288, 32768)   label-partitioned CTA tasks (P = ceil(deg/6144) smem tables)
+//   sub 4: [32768, 393216)  label-partitioned CTA tasks (P <= 64)
+//   sub 5: >= 393216        hub: cooperative grid, global table in an L2-sized ring
+//   (P * deg streamed entries would grow quadratically beyond sub 4)
 constexpr int kSubPerBucket = 8;
 constexpr int kNumClasses = 8 * kSubPerBucket;
-constexpr int64_t kSub1Min = 1024, kSub2Min = 4096, kSub3Min = 12288, kSub4Min = 32768, kHubMin = 131072;
+constexpr int64_t kSub1Min = 1024, kSub2Min = 4096, kSub3Min = 12288, kSub4Min = 32768, kHubMin = 393216;
 constexpr int kClusterSlots = 16384;  // table slots per cluster CTA (12 B each: 192 KB)
 constexpr int kCap0 = 2048, kCap1 = 8192, kCap2 = 16384;  // smem table slots (12 B each)
 constexpr int64_t kHubChunkEdges = 2048;  // edges per hub insert item

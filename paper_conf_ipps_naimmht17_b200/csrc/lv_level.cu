@@ -483,7 +483,7 @@ static int32_t build_hub_plan(Handle& h, Level& L) {
   return LOUVAIN_OK;
 }
 
-// Partition plan for every vertex of sub-classes 3..5 (deg >= kSub3Min), any bucket.
+// Partition plan for every vertex of sub-classes 3..4 (kSub3Min <= deg < kHubMin), any bucket.
 int32_t build_part_plan(Handle& h, Level& L) {
   cudaStream_t s = h.stream;
   PartPlan& Q = L.part;
@@ -494,7 +494,7 @@ int32_t build_part_plan(Handle& h, Level& L) {
   for (int b = 1; b <= 7; ++b) {
     Q.bucket_task[b - 1] = (int64_t)tv.size();
     Q.bucket_vert[b - 1] = (int64_t)vpos.size();
-    for (int sub = 3; sub <= 5; ++sub) {
+    for (int sub = 3; sub <= 4; ++sub) {
       const int c = kSubPerBucket * b + sub;
       const int64_t off = L.class_off[c], cnt = L.class_off[c + 1] - off;
       if (cnt <= 0) continue;

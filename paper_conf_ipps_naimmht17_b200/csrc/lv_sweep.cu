@@ -919,8 +919,8 @@ int32_t dispatch_class(Handle& h, Level& L, const SweepArgs& A, int bucket, int 
   } else if (sub == 0 && max_deg <= 340) {
     sweep_warp<512, 4, UNIT, AGG><<<grid_for(nv, 4, 148 * 12), 128, 0, s>>>(verts, soff, nv, stage, A);
     LV_LAUNCHED();
-  } else if (sub >= 3 && !getenv("LV_NO_PART")) {
-    if (sub == 3) {  // one launch covers the bucket's sub-classes 3..5
+  } else if ((sub == 3 || sub == 4) && !getenv("LV_NO_PART")) {
+    if (sub == 3) {  // one launch covers the bucket's sub-classes 3..4
       PartPlan& Q = L.part;
       const int64_t t0 = Q.bucket_task[bucket - 1], t1 = Q.bucket_task[bucket];
       const int64_t v0 = Q.bucket_vert[bucket - 1], v1 = Q.bucket_vert[bucket];
