@@ -46,6 +46,36 @@ void dfree(void* p, cudaStream_t s) {
   if (p) cudaFreeAsync(p, s);
 }
 
+int32_t scratch_get(Handle& h, int slot, size_t bytes, void** out) {
+  Scratch& S = h.scratch;
+  if (S.bytes[slot] < bytes) {
+    if (S.p[slot]) {
+      cudaStreamSynchronize(h.stream);  // the old buffer may still be in use by queued work
+      cudaFree(S.p[slot]);
+      S.p[slot] = nullptr;
+      S.bytes[slot] = 0;
+    }
+    const size_t want = bytes + bytes / 8;  // headroom: later levels are usually smaller
+    cudaError_t e = cudaMalloc(&S.p[slot], want);
+    if (e != cudaSuccess) {
+      cudaGetLastError();
+      g_err = "scratch allocation of " + std::to_string(want) + " bytes failed: " + cudaGetErrorString(e);
+      return LOUVAIN_E_NOMEM;
+    }
+    S.bytes[slot] = want;
+  }
+  *out = S.p[slot];
+  return LOUVAIN_OK;
+}
+
+void scratch_free(Handle& h) {
+  for (int i = 0; i < SC_COUNT; ++i) {
+    if (h.scratch.p[i]) cudaFree(h.scratch.p[i]);
+    h.scratch.p[i] = nullptr;
+    h.scratch.bytes[i] = 0;
+  }
+}
+
 bool is_device_ptr(const void* p) {
   if (!p) return false;
   cudaPointerAttributes at;
@@ -121,6 +151,7 @@ void destroy_handle(Handle& h) {
     level_free(h.lv, h.stream);
     cudaStreamSynchronize(h.stream);
   }
+  scratch_free(h);
   if (h.ctl) cudaFree(h.ctl);
   if (h.h_ctl) cudaFreeHost(h.h_ctl);
   for (auto& e : h.ev)
@@ -339,7 +370,10 @@ int32_t run_impl(Handle& h, const louvain_params_t& p, int32_t* labels_out, louv
       Level next;
       LV_TRY(dalloc(&map, L.n, s));
       tr.mark(s, "pre-contract", level);
-      LV_TRY(level_contract(h, L, next, map));
+      // sort-based (default) or mergeCommunity-style hashing (LV_CONTRACT=hash, NEXT-1)
+      static const bool hash_contract = getenv("LV_CONTRACT") && std::string(getenv("LV_CONTRACT")) == "hash";
+      if (hash_contract) LV_TRY(level_contract_fast(h, L, next, map, (level + 1) & 1));
+      else LV_TRY(level_contract(h, L, next, map, (level + 1) & 1));
       tr.mark(s, "contract", level);
       LV_TRY(compose_labels(h, lab, n0, map));
       dfree(map, s);

@@ -122,6 +122,9 @@ struct Level {
   int32_t* col = nullptr;
   uint32_t* w = nullptr;  // nullptr = unit weights (level 0 of every config, R20)
   bool owns_csr = true;
+  bool scratch_backed = false;  // all arrays live in the handle's scratch (level of a run)
+  int parity = 0;
+  bool k_ready = false;  // k already holds the degrees (contracted level: community totals)
   uint32_t* k = nullptr;
   uint2* ca = nullptr;  // {C[v], a[v]}
   int32_t* size = nullptr;
@@ -147,8 +150,23 @@ struct Level {
   PartPlan part;
 };
 
+// Grow-only scratch buffers owned by a handle (cudaMalloc'ed once, reused by
+// every level and every run): avoids multi-GB stream-ordered allocations
+// churning the memory pool between levels.
+enum ScratchSlot {
+  SC_STAGE = 0, SC_GC, SC_GW, SC_OC, SC_OW, SC_K1, SC_V0, SC_V1, SC_TMP,
+  // arrays of a contracted level inside louvain_run, double-buffered by level parity
+  SC_LVL0, SC_LVL_END = SC_LVL0 + 2 * 11, SC_COUNT = SC_LVL_END
+};
+enum LevelArray { LA_ROWPTR = 0, LA_COL, LA_W, LA_K, LA_CA, LA_SIZE, LA_MVV, LA_MVN, LA_MVO, LA_BIN, LA_SOFF };
+struct Scratch {
+  void* p[SC_COUNT] = {nullptr};
+  size_t bytes[SC_COUNT] = {0};
+};
+
 struct Handle {
   int device = 0;
+  Scratch scratch;
   cudaStream_t stream = nullptr;
   bool own_stream = false;
   bool poisoned = false;
@@ -175,9 +193,12 @@ int32_t dalloc(T** p, size_t count, cudaStream_t s) {
   return dmalloc(reinterpret_cast<void**>(p), sizeof(T) * (count ? count : 1), s);
 }
 bool is_device_ptr(const void* p);
+int32_t scratch_get(Handle& h, int slot, size_t bytes, void** out);  // grow-only per-handle buffer
+void scratch_free(Handle& h);
 
 // ------------------------------------------------------------------ level ops (lv_level.cu)
 int32_t level_alloc_state(Level& L, cudaStream_t s);
+int32_t level_alloc_scratch(Handle& h, Level& L, int parity);  // state arrays from scratch slots
 void level_free(Level& L, cudaStream_t s);
 int32_t level_setup(Handle& h, Level& L);  // k, W, singleton partition (Alg. 1 l.2)
 int32_t level_set_labels(Handle& h, Level& L, const int32_t* d_labels);  // C given (nullptr = iota), recompute a/size
@@ -192,7 +213,9 @@ int32_t set_ctl_u64(Handle& h, unsigned long long* dst, unsigned long long v);
 int32_t pack_moves(Handle& h, Level& L, int64_t c0, int64_t cnt, int32_t* out);          // log -> (v,new) pairs
 int32_t unpack_moves(Handle& h, Level& L, int64_t c0, int64_t cnt, const int32_t* in);   // (v,new) pairs -> log
 int32_t launch_revert(Handle& h, Level& L);
-int32_t level_contract(Handle& h, Level& L, Level& out, int32_t* d_map);  // Alg. 3
+// Alg. 3, canonical (rows sorted); parity >= 0: arrays from the handle's scratch (inside louvain_run)
+int32_t level_contract(Handle& h, Level& L, Level& out, int32_t* d_map, int parity = -1);
+int32_t level_contract_fast(Handle& h, Level& L, Level& out, int32_t* d_map, int parity);  // Alg. 3, rows unsorted
 int32_t compose_labels(Handle& h, int32_t* lab, int64_t n0, const int32_t* map);  // lab[i] = map[lab[i]]
 int32_t compose_labels_ca(Handle& h, int32_t* lab, int64_t n0, const uint2* ca);   // lab[i] = C[lab[i]]
 size_t hub_partial_bytes();

@@ -230,6 +230,13 @@ __global__ void k_flags_nonempty(const int32_t* size, int64_t n, int32_t* flag) 
     flag[c] = size[c] > 0 ? 1 : 0;
 }
 
+// Degree of a contracted vertex = total of its community (R18: the merged row
+// sums every member's row), so the next level's k needs no reduction.
+__global__ void k_next_degrees(const uint2* ca, const int32_t* size, const int32_t* newID, int64_t n, uint32_t* kout) {
+  for (int64_t c = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; c < n; c += (int64_t)gridDim.x * blockDim.x)
+    if (size[c] > 0) kout[newID[c]] = ca[c].y;
+}
+
 __global__ void k_map(const uint2* ca, const int32_t* newID, int64_t n, int32_t* map) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
     map[i] = newID[ca[i].x];  // R17: new ids in label order
@@ -304,7 +311,32 @@ static void hub_free(HubPlan& P, cudaStream_t s) {
   P = HubPlan();
 }
 
+int32_t level_alloc_scratch(Handle& h, Level& L, int parity) {
+  const size_t n = (size_t)std::max<int64_t>(L.n, 1);
+  auto get = [&](int a, size_t bytes, void** out) { return scratch_get(h, SC_LVL0 + 2 * a + parity, bytes, out); };
+  LV_TRY(get(LA_K, 4 * n, (void**)&L.k));
+  LV_TRY(get(LA_CA, 8 * n, (void**)&L.ca));
+  LV_TRY(get(LA_SIZE, 4 * n, (void**)&L.size));
+  LV_TRY(get(LA_MVV, 4 * n, (void**)&L.mv_v));
+  LV_TRY(get(LA_MVN, 4 * n, (void**)&L.mv_new));
+  LV_TRY(get(LA_MVO, 4 * n, (void**)&L.mv_old));
+  LV_TRY(get(LA_BIN, 4 * n, (void**)&L.bin_vertices));
+  LV_TRY(get(LA_SOFF, 8 * (n + 1), (void**)&L.soff));
+  L.scratch_backed = true;
+  L.parity = parity;
+  L.owns_csr = false;
+  return LOUVAIN_OK;
+}
+
 void level_free(Level& L, cudaStream_t s) {
+  if (L.scratch_backed) {  // arrays belong to the handle's scratch; plans are per level
+    hub_free(L.hub, s);
+    PartPlan& Q = L.part;
+    dfree(Q.task_vpos, s); dfree(Q.task_p, s); dfree(Q.vert_pos, s); dfree(Q.vert_P, s); dfree(Q.vert_first, s);
+    dfree(Q.done, s); dfree(Q.partial, s);
+    L = Level();
+    return;
+  }
   if (L.owns_csr) {
     dfree(L.rowptr, s);
     dfree(L.col, s);
@@ -312,7 +344,7 @@ void level_free(Level& L, cudaStream_t s) {
   }
   dfree(L.k, s); dfree(L.ca, s); dfree(L.size, s);
   dfree(L.mv_v, s); dfree(L.mv_new, s); dfree(L.mv_old, s); dfree(L.bin_vertices, s);
-  dfree(L.soff, s); dfree(L.stage, s);
+  dfree(L.soff, s);  // L.stage lives in the handle's scratch
   hub_free(L.hub, s);
   PartPlan& Q = L.part;
   dfree(Q.task_vpos, s); dfree(Q.task_p, s); dfree(Q.vert_pos, s); dfree(Q.vert_P, s); dfree(Q.vert_first, s);
@@ -324,6 +356,12 @@ int32_t level_setup(Handle& h, Level& L) {
   cudaStream_t s = h.stream;
   const int64_t n = L.n;
   if (n == 0) { L.W = 0; return LOUVAIN_OK; }
+  if (L.k_ready) {  // contracted level: k = community totals, W unchanged (set by level_contract)
+    k_init_singletons<<<grid_for(n, 256), 256, 0, s>>>(L.k, n, L.ca, L.size);
+    LV_LAUNCHED();
+    LV_CUDA(cudaGetLastError());
+    return LOUVAIN_OK;
+  }
   if (L.w) {
     // k_i = weighted row sum
     size_t tb = 0;
@@ -572,8 +610,12 @@ int32_t level_binning(Handle& h, Level& L, const louvain_params_t& p) {
     dfree(cls, s); dfree(cls2, s); dfree(iota, s); dfree(hist, s);
     for (int c = 0; c < kNumClasses; ++c) L.class_off[c + 1] = L.class_off[c] + (int64_t)hh[c];
     // staging offsets: exclusive scan of the degrees in bin order
-    if (!L.soff) LV_TRY(dalloc(&L.soff, n + 1, s));
-    if (!L.stage) LV_TRY(dalloc(&L.stage, L.nnz, s));
+    if (!L.soff) LV_TRY(dalloc(&L.soff, n + 1, s));  // scratch-backed levels have it already
+    {
+      void* st = nullptr;
+      LV_TRY(scratch_get(h, SC_STAGE, sizeof(uint2) * (size_t)std::max<int64_t>(L.nnz, 1), &st));
+      L.stage = static_cast<uint2*>(st);
+    }
     int64_t* dg = nullptr;
     LV_TRY(dalloc(&dg, n + 1, s));
     k_bin_degrees<<<grid_for(n, 256), 256, 0, s>>>(L.bin_vertices, n, L.rowptr, dg);
@@ -709,11 +751,13 @@ int32_t compose_labels_ca(Handle& h, int32_t* lab, int64_t n0, const uint2* ca) 
 //  every entry (u,v,w) emits key (newID[C[u]], newID[C[v]]) (R18: mergeCommunity
 //  hashes all neighbours of all members); radix sort; equal keys summed
 //  (run-length counts at unit weight); CSR' rows sorted by column.
-int32_t level_contract(Handle& h, Level& L, Level& out, int32_t* d_map) {
+int32_t level_contract(Handle& h, Level& L, Level& out, int32_t* d_map, int parity) {
   cudaStream_t s = h.stream;
   const int64_t n = L.n, nnz = L.nnz;
   out = Level();
   out.W = L.W;
+  const bool scr = parity >= 0;  // inside louvain_run: every big array from the handle's scratch
+  auto lvl = [&](int a, size_t bytes, void** o) { return scratch_get(h, SC_LVL0 + 2 * a + parity, bytes, o); };
   if (n == 0) {
     LV_TRY(dalloc(&out.rowptr, 1, s));
     LV_CUDA(cudaMemsetAsync(out.rowptr, 0, 8, s));
@@ -738,23 +782,41 @@ int32_t level_contract(Handle& h, Level& L, Level& out, int32_t* d_map) {
   k_map<<<grid_for(n, 256), 256, 0, s>>>(L.ca, newID, n, d_map);
   LV_LAUNCHED();
   dfree(flag, s);
-  dfree(newID, s);
   out.n = np;
-  LV_TRY(dalloc(&out.rowptr, np + 1, s));
+  if (scr) LV_TRY(lvl(LA_ROWPTR, 8 * (size_t)(np + 1), (void**)&out.rowptr));
+  else LV_TRY(dalloc(&out.rowptr, np + 1, s));
   LV_CUDA(cudaMemsetAsync(out.rowptr, 0, 8 * (np + 1), s));
   if (nnz == 0) {
     out.nnz = 0;
-    LV_TRY(dalloc(&out.col, 1, s));
-    LV_TRY(dalloc(&out.w, 1, s));
-    return level_alloc_state(out, s);
+    if (scr) {
+      LV_TRY(lvl(LA_COL, 4, (void**)&out.col));
+      LV_TRY(lvl(LA_W, 4, (void**)&out.w));
+      LV_TRY(level_alloc_scratch(h, out, parity));
+    } else {
+      LV_TRY(dalloc(&out.col, 1, s));
+      LV_TRY(dalloc(&out.w, 1, s));
+      LV_TRY(level_alloc_state(out, s));
+    }
+    k_next_degrees<<<grid_for(n, 256), 256, 0, s>>>(L.ca, L.size, newID, n, out.k);
+    LV_LAUNCHED();
+    dfree(newID, s);
+    out.k_ready = true;
+    return LOUVAIN_OK;
   }
   const bool weighted = L.w != nullptr;
   unsigned long long *k0 = nullptr, *k1 = nullptr;
   uint32_t *v0 = nullptr, *v1 = nullptr;
-  LV_TRY(dalloc(&k0, nnz, s));
-  LV_TRY(dalloc(&k1, nnz, s));
-  LV_TRY(dalloc(&v0, nnz, s));
-  if (weighted) LV_TRY(dalloc(&v1, nnz, s));
+  if (scr) {
+    LV_TRY(scratch_get(h, SC_STAGE, 8 * (size_t)nnz, (void**)&k0));  // the level's stage is dead now
+    LV_TRY(scratch_get(h, SC_K1, 8 * (size_t)nnz, (void**)&k1));
+    LV_TRY(scratch_get(h, SC_V0, 4 * (size_t)nnz, (void**)&v0));
+    if (weighted) LV_TRY(scratch_get(h, SC_V1, 4 * (size_t)nnz, (void**)&v1));
+  } else {
+    LV_TRY(dalloc(&k0, nnz, s));
+    LV_TRY(dalloc(&k1, nnz, s));
+    LV_TRY(dalloc(&v0, nnz, s));
+    if (weighted) LV_TRY(dalloc(&v1, nnz, s));
+  }
   {
     const int64_t ntiles = (nnz + kTileEdges - 1) / kTileEdges;
     k_emit_keys<<<grid_for(ntiles, 1, 148 * 8), 256, 0, s>>>(L.rowptr, n, L.col, L.w, d_map, nnz, (uint64_t)np, k0,
@@ -792,10 +854,15 @@ int32_t level_contract(Handle& h, Level& L, Level& out, int32_t* d_map) {
   int64_t m = 0;
   LV_CUDA(cudaMemcpyAsync(&m, d_num, 8, cudaMemcpyDeviceToHost, s));
   LV_CUDA(cudaStreamSynchronize(s));
-  dfree(sorted, s);
+  if (!scr) dfree(sorted, s);
   out.nnz = m;
-  LV_TRY(dalloc(&out.col, m, s));
-  LV_TRY(dalloc(&out.w, m, s));
+  if (scr) {
+    LV_TRY(lvl(LA_COL, 4 * (size_t)std::max<int64_t>(m, 1), (void**)&out.col));
+    LV_TRY(lvl(LA_W, 4 * (size_t)std::max<int64_t>(m, 1), (void**)&out.w));
+  } else {
+    LV_TRY(dalloc(&out.col, m, s));
+    LV_TRY(dalloc(&out.w, m, s));
+  }
   int64_t* cnt = nullptr;
   LV_TRY(dalloc(&cnt, np + 1, s));
   LV_CUDA(cudaMemsetAsync(cnt, 0, 8 * (np + 1), s));
@@ -811,10 +878,19 @@ int32_t level_contract(Handle& h, Level& L, Level& out, int32_t* d_map) {
   LV_LAUNCHED();
   LV_CUDA(cudaMemcpyAsync(out.w, sums, 4 * m, cudaMemcpyDeviceToDevice, s));
   LV_CUDA(cudaGetLastError());
-  dfree(uniq, s);
-  dfree(v0, s);
-  if (v1) dfree(v1, s);
-  return level_alloc_state(out, s);
+  if (!scr) {
+    dfree(uniq, s);
+    dfree(v0, s);
+    if (v1) dfree(v1, s);
+  }
+  if (scr) LV_TRY(level_alloc_scratch(h, out, parity));
+  else LV_TRY(level_alloc_state(out, s));
+  k_next_degrees<<<grid_for(n, 256), 256, 0, s>>>(L.ca, L.size, newID, n, out.k);
+  LV_LAUNCHED();
+  LV_CUDA(cudaGetLastError());
+  dfree(newID, s);
+  out.k_ready = true;
+  return LOUVAIN_OK;
 }
 
 // Host-side CSR validation (LOUVAIN_VALIDATE): rowptr monotone with rowptr[0]=0
