@@ -202,12 +202,23 @@ bool bucket_nonempty(const Level& L, int b) {
 // One sweep body: for each non-empty bucket 1..7 its sweep kernels, then its
 // commit (BIN_SYNC) -- or a single commit at the end (RELAXED).
 int32_t sweep_body(Handle& h, Level& L, const louvain_params_t& p) {
+  static const bool trace = getenv("LV_TRACE") && std::string(getenv("LV_TRACE")) == "2";
   LV_CUDA(cudaMemsetAsync(h.ctl, 0, offsetof(DevCtl, L), h.stream));  // logn + bounds
   int commits = 0;
   for (int b = 1; b <= 7; ++b) {
     if (!bucket_nonempty(L, b)) continue;
+    auto t0 = std::chrono::steady_clock::now();
     LV_TRY(launch_sweep_bucket(h, L, p, b));
+    auto t1 = std::chrono::steady_clock::now();
     if (p.mode == LOUVAIN_MODE_BIN_SYNC) LV_TRY(launch_commit(h, L, commits++));
+    if (trace) {
+      cudaStreamSynchronize(h.stream);
+      auto t2 = std::chrono::steady_clock::now();
+      fprintf(stderr, "[lv]      bucket %d: enqueue %.3f ms, done %.3f ms (n=%ld)\n", b,
+              std::chrono::duration<double, std::milli>(t1 - t0).count(),
+              std::chrono::duration<double, std::milli>(t2 - t0).count(),
+              (long)(L.class_off[kSubPerBucket * (b + 1)] - L.class_off[kSubPerBucket * b]));
+    }
   }
   if (p.mode == LOUVAIN_MODE_RELAXED) LV_TRY(launch_commit(h, L, commits++));
   ++L.sweeps_done;

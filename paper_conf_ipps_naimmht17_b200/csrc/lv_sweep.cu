@@ -35,6 +35,9 @@
 #include <cooperative_groups.h>
 #include <cuda_runtime.h>
 
+#include <chrono>
+#include <cstdio>
+#include <string>
 #include <algorithm>
 #include <cstdlib>
 
@@ -1020,6 +1023,27 @@ int32_t dispatch_class(Handle& h, Level& L, const SweepArgs& A, int bucket, int 
 
 size_t hub_partial_bytes() { return sizeof(Partial); }
 
+// LV_TRACE=2: per-class timing (synchronises the stream; diagnostics only)
+static bool trace_on() {
+  static const bool on = getenv("LV_TRACE") && std::string(getenv("LV_TRACE")) == "2";
+  return on;
+}
+static void trace_step(Handle& h, Level& L, int bucket, int sub, int64_t pos0, int64_t pos1) {
+  static auto last = std::chrono::steady_clock::now();
+  cudaStreamSynchronize(h.stream);
+  auto now = std::chrono::steady_clock::now();
+  const double ms = std::chrono::duration<double, std::milli>(now - last).count();
+  last = now;
+  if (pos1 <= pos0) return;
+  int64_t e[2] = {0, 0};
+  cudaMemcpy(&e[0], L.soff + pos0, 8, cudaMemcpyDeviceToHost);
+  cudaMemcpy(&e[1], L.soff + pos1, 8, cudaMemcpyDeviceToHost);
+  last = std::chrono::steady_clock::now();
+  fprintf(stderr, "[lv]        b%d %-5s nv=%-9ld edges=%-11ld %8.3f ms %7.2f Gedge/s\n", bucket,
+          sub < 0 ? "stage" : (std::string("sub") + char('0' + sub)).c_str(), (long)(pos1 - pos0),
+          (long)(e[1] - e[0]), ms, ms > 0 ? (e[1] - e[0]) / ms / 1e6 : 0.0);
+}
+
 int32_t launch_stage(Handle& h, Level& L, int64_t pos0, int64_t pos1) {
   k_stage<<<148 * 8, 256, 0, h.stream>>>(L.bin_vertices, L.soff, pos0, pos1, L.rowptr, L.col, L.ca, L.stage);
   LV_LAUNCHED();
@@ -1049,12 +1073,14 @@ int32_t launch_sweep_bucket(Handle& h, Level& L, const louvain_params_t& p, int 
     const int64_t pos0 = L.class_off[kSubPerBucket * bucket + (sub0_small ? 1 : 0)];
     const int64_t pos1 = L.class_off[kSubPerBucket * (bucket + 1)];
     if (pos1 > pos0) LV_TRY(launch_stage(h, L, pos0, pos1));
+    if (trace_on()) trace_step(h, L, bucket, -1, pos0, pos1);
   }
   for (int sub = 0; sub < 6; ++sub) {
     const int64_t max_deg = (sub == 0) ? std::min<int64_t>(hi, kSub1Min - 1) : hi;
-    // warp-level label merging pays once communities exist (hot labels); on the
-    // first sweep of a level most labels in a row are distinct and it does not
-    const bool agg = L.sweeps_done > 0;
+    // warp-level label merging (__match_any_sync before the table insert) is
+    // off: measured slower at every level and sweep of C5 (profiles/README.md)
+    static const char* agg_env = getenv("LV_AGG");  // diagnostics: LV_AGG=1 forces it on
+    const bool agg = agg_env && agg_env[0] == '1';
     if (L.w) {
       if (agg) LV_TRY((dispatch_class<false, true>(h, L, A, bucket, sub, max_deg)));
       else LV_TRY((dispatch_class<false, false>(h, L, A, bucket, sub, max_deg)));
@@ -1062,6 +1088,9 @@ int32_t launch_sweep_bucket(Handle& h, Level& L, const louvain_params_t& p, int 
       if (agg) LV_TRY((dispatch_class<true, true>(h, L, A, bucket, sub, max_deg)));
       else LV_TRY((dispatch_class<true, false>(h, L, A, bucket, sub, max_deg)));
     }
+    if (trace_on())
+      trace_step(h, L, bucket, sub, L.class_off[kSubPerBucket * bucket + sub],
+                 L.class_off[kSubPerBucket * bucket + sub + 1]);
   }
   return LOUVAIN_OK;
 }

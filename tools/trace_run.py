@@ -1,6 +1,6 @@
 import os, sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
-os.environ["LV_TRACE"] = "1"
+os.environ.setdefault("LV_TRACE", "1")
 import torch, graphgen
 import paper_conf_ipps_naimmht17_b200 as lvb
 dg = graphgen.rmat(int(sys.argv[1]) if len(sys.argv) > 1 else 27, seed=1, device=True)
