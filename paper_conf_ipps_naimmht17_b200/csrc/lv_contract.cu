@@ -92,7 +92,8 @@ __global__ void __launch_bounds__(256) k_group_copy(const int32_t* __restrict__ 
                                                     const int64_t* __restrict__ gpos, int64_t n,
                                                     const int64_t* __restrict__ rowptr,
                                                     const int32_t* __restrict__ col, const uint32_t* __restrict__ w,
-                                                    const int32_t* __restrict__ map, int32_t* gc, uint32_t* gw) {
+                                                    const int32_t* __restrict__ map, const int64_t* __restrict__ tr,
+                                                    int32_t* gc, uint32_t* gw) {
   __shared__ int64_t sh_g[kCRows + 1];
   __shared__ int64_t sh_rb[kCRows];
   __shared__ int64_t sh_i0;
@@ -101,16 +102,8 @@ __global__ void __launch_bounds__(256) k_group_copy(const int32_t* __restrict__ 
   const int64_t ntiles = (total + kCTile - 1) / kCTile;
   for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
     const int64_t t0 = tile * kCTile, t1 = min(total, t0 + kCTile);
-    if (threadIdx.x == 0) {
-      auto find = [&](int64_t x) {  // largest i in [0, n) with gpos[i] <= x
-        int64_t lo = 0, hi = n - 1;
-        while (lo < hi) {
-          const int64_t mid = (lo + hi + 1) >> 1;
-          if (gpos[mid] <= x) lo = mid; else hi = mid - 1;
-        }
-        return lo;
-      };
-      const int64_t i0 = find(t0), i1 = find(t1 - 1);
+    if (threadIdx.x == 0) {  // tile plan (tile_starts)
+      const int64_t i0 = tr[tile], i1 = tr[tile + 1];
       sh_i0 = i0;
       sh_nr = (i1 - i0 + 1 <= kCRows) ? (int)(i1 - i0 + 1) : -1;
     }
@@ -155,9 +148,9 @@ __global__ void __launch_bounds__(256) k_group_copy(const int32_t* __restrict__ 
 #pragma unroll
       for (int q = 0; q < 4; ++q) {
         const int64_t t = base + (int64_t)q * blockDim.x;
-        if (t < t1) {
-          gc[t] = mm[q];
-          if (gw) gw[t] = w ? __ldcs(&w[ee[q]]) : 1u;
+        if (t < t1) {  // evict-first: streamed once, must not displace map[] in L2
+          __stcs(&gc[t], mm[q]);
+          if (gw) __stcs(&gw[t], w ? __ldcs(&w[ee[q]]) : 1u);
         }
       }
     }
@@ -332,12 +325,134 @@ __global__ void k_big_place(const unsigned long long* __restrict__ ukeys, const 
   }
 }
 
+
+// Step 4d (default): big segments merged in global-memory hash tables kept
+// L2-resident by processing the segments in waves (each wave's tables <= kBigWaveSlots
+// slots).  Table of a segment: cap = 2 * min(len, n') slots (load <= 1/2), split into
+// 4-slot buckets read with two 16-byte loads; a label is claimed at the first
+// empty slot of its probe sequence (one CAS) and summed with atomicAdd afterwards.
+struct BigSeg {
+  int64_t src;   // segment start in gc/gw and in oc/ow
+  int64_t toff;  // table offset in the wave table
+  int64_t cap;   // slots, multiple of 4
+  int32_t row;
+  int32_t pad;
+};
+struct BigItem {
+  int32_t seg;
+  int32_t pad;
+  int64_t begin, end;  // insert: entries [begin, end) of the segment; extract: slots
+};
+constexpr int64_t kBigWaveSlots = 6 << 20;  // 48 MB of 8-byte slots per wave
+constexpr int64_t kBigChunk = 4096;
+
+__device__ __forceinline__ void big_insert4(unsigned long long* T, uint32_t cap, const int32_t c[4],
+                                            const uint32_t x[4], bool todo[4]) {
+  const uint32_t nb = cap >> 2;
+  uint32_t b[4];
+#pragma unroll
+  for (int q = 0; q < 4; ++q) b[q] = todo[q] ? (hash_slot(c[q], nb) << 2) : 0u;
+  while (todo[0] || todo[1] || todo[2] || todo[3]) {
+    unsigned long long k[4][4];
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      if (!todo[q]) continue;
+      const ulonglong2 lo = __ldcg(reinterpret_cast<const ulonglong2*>(&T[b[q]]));
+      const ulonglong2 hi = __ldcg(reinterpret_cast<const ulonglong2*>(&T[b[q] + 2]));
+      k[q][0] = lo.x; k[q][1] = lo.y; k[q][2] = hi.x; k[q][3] = hi.y;
+    }
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      if (!todo[q]) continue;
+      int tgt = -1;
+      bool found = false;
+#pragma unroll
+      for (int u = 3; u >= 0; --u)
+        if (k[q][u] == kEmpty) tgt = u;
+#pragma unroll
+      for (int u = 3; u >= 0; --u)
+        if (k[q][u] != kEmpty && (k[q][u] >> 32) == (unsigned long long)(uint32_t)c[q]) { tgt = u; found = true; }
+      if (tgt < 0) {  // bucket full: next bucket
+        b[q] = (b[q] + 4 >= cap) ? 0u : b[q] + 4;
+        continue;
+      }
+      if (!found) {
+        const unsigned long long old =
+            atomicCAS(&T[b[q] + tgt], kEmpty, (((unsigned long long)(uint32_t)c[q]) << 32) | x[q]);
+        if (old == kEmpty) { todo[q] = false; continue; }
+        if ((old >> 32) != (unsigned long long)(uint32_t)c[q]) continue;  // lost the slot: re-read the bucket
+      }
+      atomicAdd(&T[b[q] + tgt], (unsigned long long)x[q]);
+      todo[q] = false;
+    }
+  }
+}
+
+__global__ void __launch_bounds__(256) k_big_insert(const BigItem* __restrict__ items, int64_t nitems,
+                                                    const BigSeg* __restrict__ segs, const int32_t* __restrict__ gc,
+                                                    const uint32_t* __restrict__ gw, unsigned long long* T) {
+  for (int64_t it = blockIdx.x; it < nitems; it += gridDim.x) {
+    const BigItem item = items[it];
+    const BigSeg sg = segs[item.seg];
+    unsigned long long* Ts = T + sg.toff;
+    for (int64_t base = item.begin + threadIdx.x; base < item.end; base += 4 * (int64_t)blockDim.x) {
+      int32_t c[4];
+      uint32_t x[4];
+      bool todo[4];
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        const int64_t t = base + (int64_t)q * blockDim.x;
+        todo[q] = t < item.end;
+        c[q] = todo[q] ? __ldcs(&gc[sg.src + t]) : 0;
+        x[q] = todo[q] ? (gw ? __ldcs(&gw[sg.src + t]) : 1u) : 0u;
+      }
+      big_insert4(Ts, (uint32_t)sg.cap, c, x, todo);
+    }
+  }
+}
+
+__global__ void __launch_bounds__(256) k_big_extract(const BigItem* __restrict__ items, int64_t nitems,
+                                                     const BigSeg* __restrict__ segs, unsigned long long* T,
+                                                     int32_t* oc, uint32_t* ow, int64_t* cnt) {
+  const int lane = threadIdx.x & 31;
+  for (int64_t it = blockIdx.x; it < nitems; it += gridDim.x) {
+    const BigItem item = items[it];
+    const BigSeg sg = segs[item.seg];
+    unsigned long long* Ts = T + sg.toff;
+    for (int64_t t0 = item.begin + (threadIdx.x - lane); t0 < item.end; t0 += blockDim.x) {  // warp-uniform trips
+      const int64_t t = t0 + lane;
+      unsigned long long x = kEmpty;
+      if (t < item.end) {
+        x = __ldcg(&Ts[t]);
+        if (x != kEmpty) Ts[t] = kEmpty;  // clean for the next wave
+      }
+      const bool has = x != kEmpty;
+      const unsigned m = __ballot_sync(kFull, has);
+      if (!m) continue;
+      unsigned long long base = 0;
+      const int leader = __ffs(m) - 1;
+      if (lane == leader) base = atomicAdd(reinterpret_cast<unsigned long long*>(&cnt[sg.row]), (unsigned long long)__popc(m));
+      base = __shfl_sync(kFull, base, leader);
+      if (has) {
+        const int64_t pos = sg.src + (int64_t)base + __popc(m & ((1u << lane) - 1u));
+        oc[pos] = (int32_t)(x >> 32);
+        ow[pos] = (uint32_t)x;
+      }
+    }
+  }
+}
+
+__global__ void k_fill_empty(unsigned long long* p, int64_t n) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    p[i] = kEmpty;
+}
+
 // Step 5: compaction into the final CSR, edge-parallel over the output entries
 // (tile of 4096 outputs: its rows' bounds staged in smem, binary search).
 __global__ void __launch_bounds__(256) k_compact(const int64_t* __restrict__ sstart,
                                                  const int64_t* __restrict__ rowptr_out, int64_t np,
                                                  const int32_t* __restrict__ oc, const uint32_t* __restrict__ ow,
-                                                 int32_t* col, uint32_t* w) {
+                                                 const int64_t* __restrict__ tr, int32_t* col, uint32_t* w) {
   __shared__ int64_t sh_r[kCRows + 1];
   __shared__ int64_t sh_s[kCRows];
   __shared__ int64_t sh_r0;
@@ -346,16 +461,8 @@ __global__ void __launch_bounds__(256) k_compact(const int64_t* __restrict__ sst
   const int64_t ntiles = (total + kCTile - 1) / kCTile;
   for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
     const int64_t q0 = tile * kCTile, q1 = min(total, q0 + kCTile);
-    if (threadIdx.x == 0) {
-      auto find = [&](int64_t x) {  // largest r with rowptr_out[r] <= x
-        int64_t lo = 0, hi = np - 1;
-        while (lo < hi) {
-          const int64_t mid = (lo + hi + 1) >> 1;
-          if (rowptr_out[mid] <= x) lo = mid; else hi = mid - 1;
-        }
-        return lo;
-      };
-      const int64_t r0 = find(q0), r1 = find(q1 - 1);
+    if (threadIdx.x == 0) {  // tile plan (tile_starts)
+      const int64_t r0 = tr[tile], r1 = tr[tile + 1];
       sh_r0 = r0;
       sh_nr = (r1 - r0 + 1 <= kCRows) ? (int)(r1 - r0 + 1) : -1;
     }
@@ -384,8 +491,8 @@ __global__ void __launch_bounds__(256) k_compact(const int64_t* __restrict__ sst
         }
         src = sstart[lo] + (q - rowptr_out[lo]);
       }
-      col[q] = oc[src];
-      w[q] = ow[src];
+      col[q] = __ldcs(&oc[src]);
+      w[q] = __ldcs(&ow[src]);
     }
     __syncthreads();
   }
@@ -488,8 +595,12 @@ int32_t level_contract_fast(Handle& h, Level& L, Level& out, int32_t* d_map, int
       gw = static_cast<uint32_t*>(p0);
     }
   }
-  k_group_copy<<<grid_for((nnz + kCTile - 1) / kCTile, 1, 148 * 8), 256, 0, s>>>(vorder, gpos, n, L.rowptr, L.col,
-                                                                                    L.w, d_map, gc, gw);
+  {
+    const int64_t* tr = nullptr;
+    LV_TRY(tile_starts(h, gpos, 0, n, 0, nnz, kCTile, &tr));
+    k_group_copy<<<grid_for((nnz + kCTile - 1) / kCTile, 1, 148 * 8), 256, 0, s>>>(vorder, gpos, n, L.rowptr, L.col,
+                                                                                      L.w, d_map, tr, gc, gw);
+  }
   LV_LAUNCHED();
   dfree(vorder, s);
   tr.mark(s, "copy");
@@ -561,7 +672,71 @@ int32_t level_contract_fast(Handle& h, Level& L, Level& out, int32_t* d_map, int
     LV_LAUNCHED();
   }
   tr.mark(s, "merge-sm");
-  if (nbig > 0) {
+  static const bool big_sort = getenv("LV_BIG_SORT") && getenv("LV_BIG_SORT")[0] == '1';
+  if (nbig > 0 && !big_sort) {
+    const int32_t* brows = rows + nsmall + nwarp + nmid;
+    std::vector<int32_t> hb(nbig);
+    LV_CUDA(cudaMemcpyAsync(hb.data(), brows, 4 * nbig, cudaMemcpyDeviceToHost, s));
+    std::vector<int64_t> hs(np + 1);
+    LV_CUDA(cudaMemcpyAsync(hs.data(), sstart, 8 * (np + 1), cudaMemcpyDeviceToHost, s));
+    LV_CUDA(cudaStreamSynchronize(s));
+    // waves of segments whose tables fit kBigWaveSlots (a larger segment gets a wave of its own)
+    std::vector<BigSeg> segs(nbig);
+    std::vector<BigItem> ins, ext;
+    std::vector<int64_t> ins_off{0}, ext_off{0};
+    int64_t acc = 0, maxslots = 0, big_entries = 0;
+    for (int64_t k = 0; k < nbig; ++k) {
+      const int32_t r = hb[k];
+      const int64_t len = hs[r + 1] - hs[r];
+      big_entries += len;
+      const int64_t cap = ((2 * std::min<int64_t>(len, np) + 3) / 4) * 4;
+      if (acc > 0 && acc + cap > kBigWaveSlots) {
+        ins_off.push_back((int64_t)ins.size());
+        ext_off.push_back((int64_t)ext.size());
+        acc = 0;
+      }
+      segs[k] = BigSeg{hs[r], acc, cap, r, 0};
+      for (int64_t e = 0; e < len; e += kBigChunk) ins.push_back(BigItem{(int32_t)k, 0, e, std::min(len, e + kBigChunk)});
+      for (int64_t e = 0; e < cap; e += kBigChunk) ext.push_back(BigItem{(int32_t)k, 0, e, std::min(cap, e + kBigChunk)});
+      acc += cap;
+      maxslots = std::max(maxslots, acc);
+    }
+    ins_off.push_back((int64_t)ins.size());
+    ext_off.push_back((int64_t)ext.size());
+    const int64_t nwaves = (int64_t)ins_off.size() - 1;
+    if (tr.on)
+      fprintf(stderr, "[lv]    contract segments: small %lld warp %lld mid %lld big %lld (big entries %lld of %lld, "
+              "%lld waves)\n", (long long)nsmall, (long long)nwarp, (long long)nmid, (long long)nbig,
+              (long long)big_entries, (long long)nnz, (long long)nwaves);
+    BigSeg* dsegs = nullptr;
+    BigItem *dins = nullptr, *dext = nullptr;
+    LV_TRY(dalloc(&dsegs, nbig, s));
+    LV_TRY(dalloc(&dins, ins.size(), s));
+    LV_TRY(dalloc(&dext, ext.size(), s));
+    LV_CUDA(cudaMemcpyAsync(dsegs, segs.data(), sizeof(BigSeg) * nbig, cudaMemcpyHostToDevice, s));
+    LV_CUDA(cudaMemcpyAsync(dins, ins.data(), sizeof(BigItem) * ins.size(), cudaMemcpyHostToDevice, s));
+    LV_CUDA(cudaMemcpyAsync(dext, ext.data(), sizeof(BigItem) * ext.size(), cudaMemcpyHostToDevice, s));
+    unsigned long long* T = nullptr;
+    {
+      void* p0 = nullptr;
+      LV_TRY(scratch_get(h, SC_K1, 8 * (size_t)maxslots, &p0));
+      T = static_cast<unsigned long long*>(p0);
+    }
+    k_fill_empty<<<grid_for(maxslots, 256, 148 * 8), 256, 0, s>>>(T, maxslots);
+    LV_LAUNCHED();
+    for (int64_t wv = 0; wv < nwaves; ++wv) {
+      const int64_t i0 = ins_off[wv], i1 = ins_off[wv + 1], x0 = ext_off[wv], x1 = ext_off[wv + 1];
+      k_big_insert<<<grid_for(i1 - i0, 1, 148 * 8), 256, 0, s>>>(dins + i0, i1 - i0, dsegs, gc, gw, T);
+      LV_LAUNCHED();
+      k_big_extract<<<grid_for(x1 - x0, 1, 148 * 8), 256, 0, s>>>(dext + x0, x1 - x0, dsegs, T, oc, ow, cnt);
+      LV_LAUNCHED();
+    }
+    LV_CUDA(cudaGetLastError());
+    dfree(dsegs, s);
+    dfree(dins, s);
+    dfree(dext, s);
+    LV_CUDA(cudaStreamSynchronize(s));  // host vectors die here
+  } else if (nbig > 0) {  // LV_BIG_SORT=1: radix sort of (segment rank, neighbour) keys + reduce-by-key
     const int32_t* brows = rows + nsmall + nwarp + nmid;
     // offsets of big segments in the key array (their lengths, host-side: nbig is small)
     std::vector<int32_t> hb(nbig);
@@ -572,6 +747,9 @@ int32_t level_contract_fast(Handle& h, Level& L, Level& out, int32_t* d_map, int
     std::vector<int64_t> boff(nbig + 1, 0);
     for (int64_t k = 0; k < nbig; ++k) boff[k + 1] = boff[k] + (hs[hb[k] + 1] - hs[hb[k]]);
     const int64_t m = boff[nbig];
+    if (tr.on)
+      fprintf(stderr, "[lv]    contract segments: small %lld warp %lld mid %lld big %lld (big entries %lld of %lld)\n",
+              (long long)nsmall, (long long)nwarp, (long long)nmid, (long long)nbig, (long long)m, (long long)nnz);
     int64_t* dboff = nullptr;
     LV_TRY(dalloc(&dboff, nbig + 1, s));
     LV_CUDA(cudaMemcpyAsync(dboff, boff.data(), 8 * (nbig + 1), cudaMemcpyHostToDevice, s));
@@ -635,8 +813,12 @@ int32_t level_contract_fast(Handle& h, Level& L, Level& out, int32_t* d_map, int
   out.nnz = m2;
   LV_TRY(lvl(LA_COL, 4 * (size_t)std::max<int64_t>(m2, 1), (void**)&out.col));
   LV_TRY(lvl(LA_W, 4 * (size_t)std::max<int64_t>(m2, 1), (void**)&out.w));
-  k_compact<<<grid_for((m2 + kCTile - 1) / kCTile, 1, 148 * 8), 256, 0, s>>>(sstart, out.rowptr, np, oc, ow, out.col,
-                                                                              out.w);
+  if (m2 > 0) {
+    const int64_t* tr = nullptr;
+    LV_TRY(tile_starts(h, out.rowptr, 0, np, 0, m2, kCTile, &tr));
+    k_compact<<<grid_for((m2 + kCTile - 1) / kCTile, 1, 148 * 8), 256, 0, s>>>(sstart, out.rowptr, np, oc, ow, tr,
+                                                                                out.col, out.w);
+  }
   LV_LAUNCHED();
   LV_CUDA(cudaGetLastError());
   dfree(cnt, s);

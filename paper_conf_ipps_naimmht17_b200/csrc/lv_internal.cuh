@@ -115,6 +115,21 @@ struct PartPlan {
   int64_t bucket_vert[9] = {0};   // plan vertices of bucket b
 };
 
+// Batched plan for the table-based vertices of degree <= kBatchMaxDeg (sub-class 0
+// of buckets whose bound exceeds 32): consecutive bin positions are cut into
+// batches of bounded total weight (deg + kBatchVertexWeight each), so a CTA
+// inserts a whole batch edge-parallel into per-vertex regions of one
+// shared-memory table (sweep_batch, lv_sweep.cu).
+constexpr int kBatchSlots = 8448;        // table slots per CTA (12 B each)
+constexpr int kBatchMaxVerts = 136;      // vertices per batch (<= kBatchSlots / 2 / kBatchVertexWeight + 1)
+constexpr int kBatchVertexWeight = 32;   // per-vertex weight added to its degree when cutting batches
+constexpr int64_t kBatchMaxDeg = 1023;
+struct BatchPlan {
+  int32_t* bstart = nullptr;      // batch start positions of every bucket, concatenated (+ end sentinels)
+  int64_t off[9] = {0};           // batches of bucket b: bstart[off[b-1] .. off[b]) (each list + 1 sentinel)
+  int64_t cap = 0;
+};
+
 struct Level {
   int64_t n = 0, nnz = 0;
   uint64_t W = 0;
@@ -142,19 +157,21 @@ struct Level {
   int64_t bins_bounds[6] = {0, 0, 0, 0, 0, 0};
   int32_t* bin_vertices = nullptr;
   int64_t class_off[kNumClasses + 1] = {0};
+  int64_t class_soff[kNumClasses + 1] = {0};  // soff[class_off[c]] (host copy)
   // gather staging (two-phase sweep): soff[i] = sum of degrees of bin_vertices[0..i),
   // stage[soff[i] + t] = {label, a_c or 0xFFFFFFFF} of the t-th neighbour of bin_vertices[i]
   int64_t* soff = nullptr;
   uint2* stage = nullptr;
   HubPlan hub;
   PartPlan part;
+  BatchPlan batch;
 };
 
 // Grow-only scratch buffers owned by a handle (cudaMalloc'ed once, reused by
 // every level and every run): avoids multi-GB stream-ordered allocations
 // churning the memory pool between levels.
 enum ScratchSlot {
-  SC_STAGE = 0, SC_GC, SC_GW, SC_OC, SC_OW, SC_K1, SC_V0, SC_V1, SC_TMP,
+  SC_STAGE = 0, SC_GC, SC_GW, SC_OC, SC_OW, SC_K1, SC_V0, SC_V1, SC_TMP, SC_TILES,
   // arrays of a contracted level inside louvain_run, double-buffered by level parity
   SC_LVL0, SC_LVL_END = SC_LVL0 + 2 * 11, SC_COUNT = SC_LVL_END
 };
@@ -217,6 +234,12 @@ int32_t launch_revert(Handle& h, Level& L);
 int32_t level_contract(Handle& h, Level& L, Level& out, int32_t* d_map, int parity = -1);
 int32_t level_contract_fast(Handle& h, Level& L, Level& out, int32_t* d_map, int parity);  // Alg. 3, rows unsorted
 int32_t compose_labels(Handle& h, int32_t* lab, int64_t n0, const int32_t* map);  // lab[i] = map[lab[i]]
+// Tile plan of an edge-centric kernel over the entries [base, end) of rows [lo, hi) with
+// prefix offsets offs (offs[hi] >= end): out[t] = the row holding entry min(base + t*T, end - 1),
+// t = 0..ntiles (ntiles = ceil((end - base) / T)).  One binary search per tile, all in
+// parallel, instead of a serial search by one thread at the start of every tile.
+int32_t tile_starts(Handle& h, const int64_t* offs, int64_t lo, int64_t hi, int64_t base, int64_t end, int64_t T,
+                    const int64_t** out);
 int32_t compose_labels_ca(Handle& h, int32_t* lab, int64_t n0, const uint2* ca);   // lab[i] = C[lab[i]]
 size_t hub_partial_bytes();
 int32_t validate_csr_host(int64_t n, int64_t nnz, const int64_t* rowptr, const int32_t* col, const uint32_t* w,
@@ -224,8 +247,11 @@ int32_t validate_csr_host(int64_t n, int64_t nnz, const int64_t* rowptr, const i
 
 // ------------------------------------------------------------------ sweep (lv_sweep.cu)
 int32_t launch_sweep_bucket(Handle& h, Level& L, const louvain_params_t& p, int bucket);
-int32_t launch_stage(Handle& h, Level& L, int64_t pos0, int64_t pos1);  // phase 1 gather for positions [pos0,pos1)
+// phase 1 gather for bin positions [pos0,pos1), staged entries [s0,s1)
+int32_t launch_stage(Handle& h, Level& L, int64_t pos0, int64_t pos1, int64_t s0, int64_t s1);
 int32_t build_part_plan(Handle& h, Level& L);
+int32_t build_batch_plan(Handle& h, Level& L, const louvain_params_t& p);
+void batch_free(BatchPlan& B, cudaStream_t s);
 
 // ------------------------------------------------------------------ launch geometry
 inline unsigned grid_for(int64_t items, int per_block, int max_blocks = 148 * 16) {

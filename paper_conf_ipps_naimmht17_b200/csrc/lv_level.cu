@@ -158,12 +158,14 @@ __global__ void k_revert(const DevCtl* ctl, const int32_t* mv_v, const int32_t* 
 // Edge-centric tile walker: calls f(u, e) for every CSR entry e of the tile
 // [e0, e1) with its source row u.  The tile's rowptr window is staged in smem
 // and each thread binary-searches it (coalesced col/w loads; degree-skew free).
+// tr = tile plan (tile_starts): rows tr[tile] .. tr[tile + 1] cover the tile.
 template <class F>
 __device__ __forceinline__ void for_tile_edges(const int64_t* rowptr, int64_t n, int64_t e0, int64_t e1,
-                                               int64_t* sh_rows, int64_t* sh_u0, int* sh_nr, F f) {
+                                               const int64_t* tr, int64_t tile, int64_t* sh_rows, int64_t* sh_u0,
+                                               int* sh_nr, F f) {
   if (threadIdx.x == 0) {
-    const int64_t u0 = row_of(rowptr, n, e0);
-    const int64_t u1 = row_of(rowptr, n, e1 - 1);
+    const int64_t u0 = tr[tile];
+    const int64_t u1 = tr[tile + 1];
     *sh_u0 = u0;
     *sh_nr = (u1 - u0 + 2 <= kTileRows) ? (int)(u1 - u0 + 2) : -1;
   }
@@ -196,7 +198,8 @@ template <bool PACKED>
 __global__ void __launch_bounds__(256) k_modularity(const int64_t* rowptr, int64_t n, const int32_t* col,
                                                     const uint32_t* w, const uint2* ca, const int32_t* C,
                                                     const uint32_t* a, int64_t e_begin, int64_t nnz,
-                                                    unsigned long long* Lout, unsigned long long* Sout) {
+                                                    const int64_t* __restrict__ tr, unsigned long long* Lout,
+                                                    unsigned long long* Sout) {
   __shared__ int64_t sh_rows[kTileRows];
   __shared__ int64_t sh_u0;
   __shared__ int sh_nr;
@@ -206,7 +209,7 @@ __global__ void __launch_bounds__(256) k_modularity(const int64_t* rowptr, int64
   const int64_t ntiles = (nnz - e_begin + kTileEdges - 1) / kTileEdges;
   for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
     const int64_t e0 = e_begin + tile * kTileEdges, e1 = min(nnz, e0 + kTileEdges);
-    for_tile_edges(rowptr, n, e0, e1, sh_rows, &sh_u0, &sh_nr, [&](int64_t u, int64_t e) {
+    for_tile_edges(rowptr, n, e0, e1, tr, tile, sh_rows, &sh_u0, &sh_nr, [&](int64_t u, int64_t e) {
       const int32_t v = __ldcs(&col[e]);
       if (__ldg(&lab[st * (int64_t)v]) == __ldg(&lab[st * u])) acc += w ? __ldcs(&w[e]) : 1u;
     });
@@ -244,14 +247,15 @@ __global__ void k_map(const uint2* ca, const int32_t* newID, int64_t n, int32_t*
 
 __global__ void __launch_bounds__(256) k_emit_keys(const int64_t* rowptr, int64_t n, const int32_t* col,
                                                    const uint32_t* w, const int32_t* map, int64_t nnz, uint64_t np,
-                                                   unsigned long long* keys, uint32_t* vals) {
+                                                   const int64_t* __restrict__ tr, unsigned long long* keys,
+                                                   uint32_t* vals) {
   __shared__ int64_t sh_rows[kTileRows];
   __shared__ int64_t sh_u0;
   __shared__ int sh_nr;
   const int64_t ntiles = (nnz + kTileEdges - 1) / kTileEdges;
   for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
     const int64_t e0 = tile * kTileEdges, e1 = min(nnz, e0 + kTileEdges);
-    for_tile_edges(rowptr, n, e0, e1, sh_rows, &sh_u0, &sh_nr, [&](int64_t u, int64_t e) {
+    for_tile_edges(rowptr, n, e0, e1, tr, tile, sh_rows, &sh_u0, &sh_nr, [&](int64_t u, int64_t e) {
       keys[e] = (unsigned long long)map[u] * np + (unsigned long long)map[col[e]];  // (newID[C[u]], newID[C[v]])
       if (vals) vals[e] = w[e];
     });
@@ -290,7 +294,33 @@ __global__ void k_sum_u32(const uint32_t* x, int64_t n, unsigned long long* out)
   if ((threadIdx.x & 31) == 0 && acc) atomicAdd(out, acc);
 }
 
+__global__ void k_tile_starts(const int64_t* __restrict__ offs, int64_t lo, int64_t hi, int64_t base, int64_t end,
+                              int64_t T, int64_t ntiles, int64_t* out) {
+  for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t <= ntiles; t += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t x = min(base + t * T, end - 1);
+    int64_t a = lo, b = hi - 1;  // largest i in [lo, hi) with offs[i] <= x
+    while (a < b) {
+      const int64_t mid = (a + b + 1) >> 1;
+      if (offs[mid] <= x) a = mid; else b = mid - 1;
+    }
+    out[t] = a;
+  }
+}
+
 }  // namespace
+
+int32_t tile_starts(Handle& h, const int64_t* offs, int64_t lo, int64_t hi, int64_t base, int64_t end, int64_t T,
+                    const int64_t** out) {
+  const int64_t ntiles = (end - base + T - 1) / T;
+  void* p = nullptr;
+  LV_TRY(scratch_get(h, SC_TILES, 8 * (size_t)(ntiles + 1), &p));
+  k_tile_starts<<<grid_for(ntiles + 1, 256), 256, 0, h.stream>>>(offs, lo, hi, base, end, T, ntiles,
+                                                                 static_cast<int64_t*>(p));
+  LV_LAUNCHED();
+  LV_CUDA(cudaGetLastError());
+  *out = static_cast<const int64_t*>(p);
+  return LOUVAIN_OK;
+}
 
 // ======================================================================== host side
 int32_t level_alloc_state(Level& L, cudaStream_t s) {
@@ -334,6 +364,7 @@ void level_free(Level& L, cudaStream_t s) {
     PartPlan& Q = L.part;
     dfree(Q.task_vpos, s); dfree(Q.task_p, s); dfree(Q.vert_pos, s); dfree(Q.vert_P, s); dfree(Q.vert_first, s);
     dfree(Q.done, s); dfree(Q.partial, s);
+    batch_free(L.batch, s);
     L = Level();
     return;
   }
@@ -349,6 +380,7 @@ void level_free(Level& L, cudaStream_t s) {
   PartPlan& Q = L.part;
   dfree(Q.task_vpos, s); dfree(Q.task_p, s); dfree(Q.vert_pos, s); dfree(Q.vert_P, s); dfree(Q.vert_first, s);
   dfree(Q.done, s); dfree(Q.partial, s);
+  batch_free(L.batch, s);
   L = Level();
 }
 
@@ -627,9 +659,16 @@ int32_t level_binning(Handle& h, Level& L, const louvain_params_t& p) {
     LV_CUDA(cub::DeviceScan::ExclusiveSum(tmp2, tb2, dg, L.soff, n + 1, s)); LV_CUB();
     dfree(tmp2, s);
     dfree(dg, s);
+    // staged-entry offsets of every class boundary, for host-side tile plans
+    for (int c = 0; c <= kNumClasses; ++c)
+      LV_CUDA(cudaMemcpyAsync(&L.class_soff[c], L.soff + L.class_off[c], 8, cudaMemcpyDeviceToHost, s));
+    LV_CUDA(cudaStreamSynchronize(s));
+  } else {
+    std::fill(L.class_soff, L.class_soff + kNumClasses + 1, 0);
   }
   LV_TRY(build_hub_plan(h, L));
   LV_TRY(build_part_plan(h, L));
+  LV_TRY(build_batch_plan(h, L, p));
   std::memcpy(L.bins_bounds, p.deg_bounds, sizeof L.bins_bounds);
   L.bins_valid = true;
   return LOUVAIN_OK;
@@ -644,8 +683,14 @@ int32_t launch_modularity(Handle& h, Level& L, const int32_t* d_C) {
   const int64_t e0 = (d_C || L.own_hi < 0) ? 0 : L.own_e0, e1 = (d_C || L.own_hi < 0) ? L.nnz : L.own_e1;
   const int64_t ntiles = (e1 - e0 + kTileEdges - 1) / kTileEdges;
   const unsigned grid = grid_for(std::max<int64_t>(ntiles, (L.n + 255) / 256), 1, 148 * 8);
+  const int64_t* tr = nullptr;
+  if (e1 > e0) {
+    LV_TRY(tile_starts(h, L.rowptr, 0, L.n, e0, e1, kTileEdges, &tr));
+  } else {
+    LV_TRY(tile_starts(h, L.rowptr, 0, L.n, 0, 1, kTileEdges, &tr));  // unused (no tiles)
+  }
   if (!d_C) {
-    k_modularity<true><<<grid, 256, 0, s>>>(L.rowptr, L.n, L.col, L.w, L.ca, nullptr, nullptr, e0, e1, &h.ctl->L,
+    k_modularity<true><<<grid, 256, 0, s>>>(L.rowptr, L.n, L.col, L.w, L.ca, nullptr, nullptr, e0, e1, tr, &h.ctl->L,
                                             &h.ctl->S);
     LV_LAUNCHED();
   } else {
@@ -654,8 +699,8 @@ int32_t launch_modularity(Handle& h, Level& L, const int32_t* d_C) {
     LV_CUDA(cudaMemsetAsync(a_tmp, 0, 4 * L.n, s));
     k_ext_totals<<<grid_for(L.n, 256), 256, 0, s>>>(d_C, L.k, L.n, a_tmp, &h.ctl->bad);
     LV_LAUNCHED();
-    k_modularity<false><<<grid, 256, 0, s>>>(L.rowptr, L.n, L.col, L.w, nullptr, d_C, a_tmp, 0, L.nnz, &h.ctl->L,
-                                             &h.ctl->S);
+    k_modularity<false><<<grid, 256, 0, s>>>(L.rowptr, L.n, L.col, L.w, nullptr, d_C, a_tmp, 0, L.nnz, tr,
+                                             &h.ctl->L, &h.ctl->S);
     LV_LAUNCHED();
     dfree(a_tmp, s);
   }
@@ -819,8 +864,10 @@ int32_t level_contract(Handle& h, Level& L, Level& out, int32_t* d_map, int pari
   }
   {
     const int64_t ntiles = (nnz + kTileEdges - 1) / kTileEdges;
-    k_emit_keys<<<grid_for(ntiles, 1, 148 * 8), 256, 0, s>>>(L.rowptr, n, L.col, L.w, d_map, nnz, (uint64_t)np, k0,
-                                                             weighted ? v0 : nullptr);
+    const int64_t* tr = nullptr;
+    LV_TRY(tile_starts(h, L.rowptr, 0, n, 0, nnz, kTileEdges, &tr));
+    k_emit_keys<<<grid_for(ntiles, 1, 148 * 8), 256, 0, s>>>(L.rowptr, n, L.col, L.w, d_map, nnz, (uint64_t)np, tr,
+                                                             k0, weighted ? v0 : nullptr);
     LV_LAUNCHED();
     LV_CUDA(cudaGetLastError());
   }

@@ -41,6 +41,9 @@
 #include <algorithm>
 #include <cstdlib>
 
+#include <cub/cub.cuh>
+#include <thrust/iterator/counting_iterator.h>
+
 #include "lv_device.cuh"
 #include "lv_internal.cuh"
 
@@ -298,9 +301,10 @@ constexpr int kStageTile = 4096;
 constexpr int kStageRows = 256;
 
 __global__ void __launch_bounds__(256) k_stage(const int32_t* __restrict__ bv, const int64_t* __restrict__ soff,
-                                               int64_t pos0, int64_t pos1, const int64_t* __restrict__ rowptr,
+                                               int64_t pos0, int64_t pos1, const int64_t* __restrict__ tr,
+                                               const int64_t* __restrict__ rowptr,
                                                const int32_t* __restrict__ col, const uint2* __restrict__ ca,
-                                               uint2* __restrict__ stage) {
+                                               uint2* __restrict__ stage, bool cs_store) {
   __shared__ int64_t sh_so[kStageRows + 1];
   __shared__ int64_t sh_rb[kStageRows];
   __shared__ int32_t sh_v[kStageRows];
@@ -310,17 +314,8 @@ __global__ void __launch_bounds__(256) k_stage(const int32_t* __restrict__ bv, c
   const int64_t ntiles = (s1 - s0 + kStageTile - 1) / kStageTile;
   for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
     const int64_t t0 = s0 + tile * kStageTile, t1 = min(s1, t0 + kStageTile);
-    if (threadIdx.x == 0) {
-      // largest i in [pos0, pos1) with soff[i] <= x
-      auto find = [&](int64_t x) {
-        int64_t lo = pos0, hi = pos1 - 1;
-        while (lo < hi) {
-          const int64_t mid = (lo + hi + 1) >> 1;
-          if (soff[mid] <= x) lo = mid; else hi = mid - 1;
-        }
-        return lo;
-      };
-      const int64_t i0 = find(t0), i1 = find(t1 - 1);
+    if (threadIdx.x == 0) {  // tile plan: positions tr[tile] .. tr[tile + 1] cover the tile
+      const int64_t i0 = tr[tile], i1 = tr[tile + 1];
       sh_i0 = i0;
       sh_nr = (i1 - i0 + 1 <= kStageRows) ? (int)(i1 - i0 + 1) : -1;
     }
@@ -369,8 +364,14 @@ __global__ void __launch_bounds__(256) k_stage(const int32_t* __restrict__ bv, c
 #pragma unroll
       for (int q = 0; q < 4; ++q) {
         const int64_t t = base + (int64_t)q * blockDim.x;
-        if (t < t1) stage[t] = (jj[q] == vv[q]) ? make_uint2(kSelf, 0u)
-                                                : make_uint2(rr[q].x, rr[q].x == (uint32_t)jj[q] ? rr[q].y : kUnknownA);
+        // evict-first store: the stage streams through L2 once and must not
+        // displace the gathered records (LV_STAGE_WB=1: plain write-back store)
+        const uint2 val = (jj[q] == vv[q]) ? make_uint2(kSelf, 0u)
+                                           : make_uint2(rr[q].x, rr[q].x == (uint32_t)jj[q] ? rr[q].y : kUnknownA);
+        if (t < t1) {
+          if (cs_store) __stcs(&stage[t], val);
+          else stage[t] = val;
+        }
       }
     }
     __syncthreads();
@@ -505,6 +506,149 @@ __global__ void __launch_bounds__(1024) sweep_cta(const int32_t* __restrict__ ve
       log_moves(threadIdx.x == 0 && tgt != own, v, tgt, A);
     }
     __syncthreads();
+  }
+}
+
+
+// ------------------------------------------------------------ batched vertices
+// Table-based vertices of degree <= kBatchMaxDeg (33..1023 with the paper's
+// bounds): a CTA takes a batch of consecutive bin positions (total weight
+// bounded by the batch plan) and works on all of them at once, so the per-vertex
+// latency chains (row bounds, records, finish) overlap instead of serialising:
+//   1. batch metadata into smem (vertex, row start, entry offset);
+//   2. edge-parallel over the batch's staged entries: insert into the vertex's
+//      own region of the table (2*deg slots at offset 2*x0);
+//   3. each vertex's region is scanned by a group of G warps (G = 16 / nv
+//      rounded down to a power of two), partials to smem;
+//   4. a warp per vertex reduces its partials and decides (stay test, veto).
+// The records come from the staging array (k_stage gathered them edge-parallel
+// at full occupancy; gathering here, inside the batch's latency chain, measured
+// 3x slower on C5).
+template <bool UNIT>
+__global__ void __launch_bounds__(512, 2) sweep_batch(const int32_t* __restrict__ bv,
+                                                    const int64_t* __restrict__ soff,
+                                                    const int32_t* __restrict__ bstart, int64_t nbatch,
+                                                    const uint2* __restrict__ stage, SweepArgs A) {
+  extern __shared__ unsigned long long smem[];
+  unsigned long long* T = smem;
+  uint32_t* TA = reinterpret_cast<uint32_t*>(smem + kBatchSlots);
+  __shared__ int32_t s_v[kBatchMaxVerts];
+  __shared__ int64_t s_rb[kBatchMaxVerts];
+  __shared__ int32_t s_x[kBatchMaxVerts + 1];
+  __shared__ Partial s_part[16];
+  __shared__ int s_nv;
+  constexpr int NW = 16;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  for (int t = threadIdx.x; t < kBatchSlots; t += blockDim.x) {
+    T[t] = kEmpty;
+    TA[t] = kUnknownA;
+  }
+  for (int64_t b = blockIdx.x; b < nbatch; b += gridDim.x) {
+    // 1. metadata
+    const int32_t p0 = __ldg(&bstart[b]), p1 = __ldg(&bstart[b + 1]);
+    const int nv = p1 - p0;
+    const int64_t base = __ldg(&soff[p0]);
+    for (int r = threadIdx.x; r <= nv; r += blockDim.x) {
+      s_x[r] = (int32_t)(__ldg(&soff[p0 + r]) - base);
+      if (r < nv) {
+        const int32_t v = __ldg(&bv[p0 + r]);
+        s_v[r] = v;
+        s_rb[r] = __ldg(&A.rowptr[v]);
+      }
+    }
+    if (threadIdx.x == 0) s_nv = nv;
+    __syncthreads();
+    const int E = s_x[nv];
+    // 2. inserts from the staged records (coalesced), 4 entries per thread per pass
+    const uint2* S = stage + base;
+    for (int x0 = threadIdx.x; x0 < E; x0 += 4 * blockDim.x) {
+      uint2 rec[4];
+      uint32_t ww[4];
+      int rr[4];
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        const int x = x0 + q * blockDim.x;
+        rec[q] = (x < E) ? __ldcs(&S[x]) : make_uint2(kSelf, 0u);
+        rr[q] = 0;
+        ww[q] = 1u;
+        if (x < E) {
+          int lo = 0, hi = nv - 1;  // largest r with s_x[r] <= x
+          while (lo < hi) {
+            const int mid = (lo + hi + 1) >> 1;
+            if (s_x[mid] <= x) lo = mid; else hi = mid - 1;
+          }
+          rr[q] = lo;
+          if (!UNIT) ww[q] = __ldcs(&A.w[s_rb[lo] + (x - s_x[lo])]);
+        }
+      }
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        if (rec[q].x == kSelf) continue;  // padding or the self-loop (R3)
+        const int r = rr[q];
+        const uint32_t off = 2u * (uint32_t)s_x[r];
+        const uint32_t cap = 2u * (uint32_t)(s_x[r + 1] - s_x[r]);
+        const uint32_t hq = table_insert(T + off, cap, (int32_t)rec[q].x, ww[q]);
+        if (rec[q].y != kUnknownA) TA[off + hq] = rec[q].y;  // the neighbour represents its label: a_c known
+      }
+    }
+    __syncthreads();
+    // 3. scan: vertex r by warps [r*G, r*G + G) (nv <= 16), else warp-strided vertices
+    int G = 1;
+    while (G * 2 * nv <= NW) G *= 2;
+    const int gw = warp % G;  // warp index inside its group
+    for (int r = warp / G; r < nv; r += NW / G) {
+      const int32_t v = s_v[r];
+      const int32_t own = (int32_t)__ldg(&A.ca[v]).x;
+      const uint32_t ki = __ldg(&A.k[v]);
+      const bool own_single = A.rule == 2 && __ldg(&A.size[own]) == 1;
+      const uint32_t off = 2u * (uint32_t)s_x[r];
+      const uint32_t cap = 2u * (uint32_t)(s_x[r + 1] - s_x[r]);
+      long long sc = (long long)0x8000000000000000ull;
+      int cb = 0x7FFFFFFF;
+      unsigned eown = 0;
+      scan_table(T + off, TA + off, cap, (uint32_t)(gw * 32 + lane), (uint32_t)(32 * G), own, own_single, ki, A, sc,
+                 cb, eown);
+      group_reduce<32>(sc, cb, eown);
+      if (G == 1) {
+        int32_t tgt = own;
+        if (lane == 0 && cb != 0x7FFFFFFF) tgt = finish(sc, cb, eown, own, __ldg(&A.ca[own]).y, ki, A);
+        log_moves(lane == 0 && tgt != own, v, tgt, A);
+      } else if (lane == 0) {
+        s_part[warp] = Partial{sc, cb, eown};
+      }
+    }
+    if (G > 1) {
+      __syncthreads();
+      // 4. a warp per vertex reduces its G partials
+      if (warp < nv) {
+        const int r = warp;
+        long long sc = (long long)0x8000000000000000ull;
+        int cb = 0x7FFFFFFF;
+        unsigned eown = 0;
+        if (lane < G) {
+          const Partial pp = s_part[r * G + lane];
+          sc = pp.s;
+          cb = pp.c;
+          eown = pp.eown;
+        }
+        group_reduce<32>(sc, cb, eown);
+        const int32_t v = s_v[r];
+        const int32_t own = (int32_t)__ldg(&A.ca[v]).x;
+        int32_t tgt = own;
+        if (lane == 0 && cb != 0x7FFFFFFF) tgt = finish(sc, cb, eown, own, __ldg(&A.ca[own]).y, __ldg(&A.k[v]), A);
+        log_moves(lane == 0 && tgt != own, v, tgt, A);
+      }
+    }
+    __syncthreads();
+  }
+}
+
+__global__ void k_batch_flags(const int64_t* __restrict__ soff, int64_t p0, int64_t p1, int64_t s0, int64_t bw,
+                              uint8_t* flag) {
+  for (int64_t i = p0 + blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < p1; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t wi = (soff[i] - s0 + kBatchVertexWeight * (i - p0)) / bw;
+    const int64_t wp = (i == p0) ? -1 : (soff[i - 1] - s0 + kBatchVertexWeight * (i - 1 - p0)) / bw;
+    flag[i - p0] = (wi != wp) ? 1 : 0;
   }
 }
 
@@ -897,6 +1041,10 @@ int32_t set_smem(K kernel, size_t bytes) {
   return LOUVAIN_OK;
 }
 
+bool batch_on(const Level& L, int bucket) {
+  return L.batch.bstart && L.batch.off[bucket] - L.batch.off[bucket - 1] > 1;
+}
+
 template <bool UNIT, bool AGG>
 int32_t dispatch_class(Handle& h, Level& L, const SweepArgs& A, int bucket, int sub, int64_t max_deg) {
   const int64_t off = L.class_off[kSubPerBucket * bucket + sub];
@@ -915,6 +1063,17 @@ int32_t dispatch_class(Handle& h, Level& L, const SweepArgs& A, int bucket, int 
       case 16: sweep_small<16, UNIT><<<grid, 256, 0, s>>>(verts, nv, A); break;
       default: sweep_small<32, UNIT><<<grid, 256, 0, s>>>(verts, nv, A); break;
     }
+    LV_LAUNCHED();
+  } else if (sub == 0 && batch_on(L, bucket)) {
+    static bool battr = false;
+    if (!battr) {
+      LV_TRY(set_smem(sweep_batch<true>, 12 * (size_t)kBatchSlots));
+      LV_TRY(set_smem(sweep_batch<false>, 12 * (size_t)kBatchSlots));
+      battr = true;
+    }
+    const int64_t b0 = L.batch.off[bucket - 1], nb = L.batch.off[bucket] - b0 - 1;  // minus the sentinel
+    sweep_batch<UNIT><<<grid_for(nb, 1, 148 * 2), 512, 12 * (size_t)kBatchSlots, s>>>(L.bin_vertices, L.soff,
+                                                                                    L.batch.bstart + b0, nb, stage, A);
     LV_LAUNCHED();
   } else if (sub == 0 && max_deg <= 84) {
     sweep_warp<128, 8, UNIT, AGG><<<grid_for(nv, 8, 148 * 8), 256, 0, s>>>(verts, soff, nv, stage, A);
@@ -1023,6 +1182,65 @@ int32_t dispatch_class(Handle& h, Level& L, const SweepArgs& A, int bucket, int 
 
 size_t hub_partial_bytes() { return sizeof(Partial); }
 
+void batch_free(BatchPlan& B, cudaStream_t s) {
+  dfree(B.bstart, s);
+  B = BatchPlan();
+}
+
+// Batch plan (see kBatchSlots): for every bucket whose sub-class 0 is table-based
+// (bound > 32), positions where floor((soff[i] - soff[p0] + 32 (i - p0)) / bw)
+// changes start a batch; bw keeps every batch's entries <= kBatchSlots / 2.
+// Experimental, off by default (LV_BATCH=1): on C5 it measured 2x slower than the
+// warp / CTA kernels it replaces (per-batch phases serialise the per-vertex loads).
+int32_t build_batch_plan(Handle& h, Level& L, const louvain_params_t& p) {
+  cudaStream_t s = h.stream;
+  batch_free(L.batch, s);
+  static const bool on = getenv("LV_BATCH") && getenv("LV_BATCH")[0] == '1';
+  if (!on || L.n == 0) return LOUVAIN_OK;
+  BatchPlan& B = L.batch;
+  int64_t total = 0;
+  for (int b = 1; b <= 7; ++b) {
+    const int c = kSubPerBucket * b;
+    total += L.class_off[c + 1] - L.class_off[c] + 1;
+  }
+  LV_TRY(dalloc(&B.bstart, total + 1, s));
+  uint8_t* flag = nullptr;
+  LV_TRY(dalloc(&flag, std::max<int64_t>(L.n, 1), s));
+  int64_t* d_num = reinterpret_cast<int64_t*>(&h.ctl->bad);
+  int64_t pos = 0;
+  B.off[0] = 0;
+  for (int b = 1; b <= 7; ++b) {
+    const int c = kSubPerBucket * b;
+    const int64_t p0 = L.class_off[c], p1 = L.class_off[c + 1];
+    const int64_t hi = (b <= 6) ? p.deg_bounds[b - 1] : INT64_MAX;
+    const int64_t max_deg = std::min<int64_t>(hi, kSub1Min - 1);
+    if (p1 > p0 && max_deg > 32 && max_deg <= kBatchMaxDeg) {
+      const int64_t bw = kBatchSlots / 2 - (max_deg + kBatchVertexWeight);
+      k_batch_flags<<<grid_for(p1 - p0, 256), 256, 0, s>>>(L.soff, p0, p1, L.class_soff[c], bw, flag);
+      LV_LAUNCHED();
+      thrust::counting_iterator<int32_t> it((int32_t)p0);
+      size_t tb = 0;
+      LV_CUDA(cub::DeviceSelect::Flagged(nullptr, tb, it, flag, B.bstart + pos, d_num, p1 - p0, s));
+      void* tmp = nullptr;
+      LV_TRY(dmalloc(&tmp, tb, s));
+      LV_CUDA(cub::DeviceSelect::Flagged(tmp, tb, it, flag, B.bstart + pos, d_num, p1 - p0, s));
+      LV_CUB();
+      dfree(tmp, s);
+      int64_t cnt = 0;
+      LV_CUDA(cudaMemcpyAsync(&cnt, d_num, 8, cudaMemcpyDeviceToHost, s));
+      LV_CUDA(cudaStreamSynchronize(s));
+      const int32_t end = (int32_t)p1;
+      LV_CUDA(cudaMemcpyAsync(B.bstart + pos + cnt, &end, 4, cudaMemcpyHostToDevice, s));
+      LV_CUDA(cudaStreamSynchronize(s));  // `end` is a host stack value
+      pos += cnt + 1;
+    }
+    B.off[b] = pos;
+  }
+  dfree(flag, s);
+  LV_CUDA(cudaMemsetAsync(&h.ctl->bad, 0, 8, s));
+  return LOUVAIN_OK;
+}
+
 // LV_TRACE=2: per-class timing (synchronises the stream; diagnostics only)
 static bool trace_on() {
   static const bool on = getenv("LV_TRACE") && std::string(getenv("LV_TRACE")) == "2";
@@ -1044,8 +1262,13 @@ static void trace_step(Handle& h, Level& L, int bucket, int sub, int64_t pos0, i
           (long)(e[1] - e[0]), ms, ms > 0 ? (e[1] - e[0]) / ms / 1e6 : 0.0);
 }
 
-int32_t launch_stage(Handle& h, Level& L, int64_t pos0, int64_t pos1) {
-  k_stage<<<148 * 8, 256, 0, h.stream>>>(L.bin_vertices, L.soff, pos0, pos1, L.rowptr, L.col, L.ca, L.stage);
+int32_t launch_stage(Handle& h, Level& L, int64_t pos0, int64_t pos1, int64_t s0, int64_t s1) {
+  if (s1 <= s0) return LOUVAIN_OK;
+  static const bool wb = getenv("LV_STAGE_WB") && getenv("LV_STAGE_WB")[0] == '1';
+  const int64_t* tr = nullptr;
+  LV_TRY(tile_starts(h, L.soff, pos0, pos1, s0, s1, kStageTile, &tr));
+  k_stage<<<grid_for((s1 - s0 + kStageTile - 1) / kStageTile, 1, 148 * 8), 256, 0, h.stream>>>(
+      L.bin_vertices, L.soff, pos0, pos1, tr, L.rowptr, L.col, L.ca, L.stage, !wb);
   LV_LAUNCHED();
   LV_CUDA(cudaGetLastError());
   return LOUVAIN_OK;
@@ -1072,7 +1295,8 @@ int32_t launch_sweep_bucket(Handle& h, Level& L, const louvain_params_t& p, int 
     const bool sub0_small = std::min<int64_t>(hi, kSub1Min - 1) <= 32;
     const int64_t pos0 = L.class_off[kSubPerBucket * bucket + (sub0_small ? 1 : 0)];
     const int64_t pos1 = L.class_off[kSubPerBucket * (bucket + 1)];
-    if (pos1 > pos0) LV_TRY(launch_stage(h, L, pos0, pos1));
+    const int c0 = kSubPerBucket * bucket + (sub0_small ? 1 : 0), c1 = kSubPerBucket * (bucket + 1);
+    if (pos1 > pos0) LV_TRY(launch_stage(h, L, pos0, pos1, L.class_soff[c0], L.class_soff[c1]));
     if (trace_on()) trace_step(h, L, bucket, -1, pos0, pos1);
   }
   for (int sub = 0; sub < 6; ++sub) {
