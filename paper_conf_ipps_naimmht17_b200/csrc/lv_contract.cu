@@ -158,6 +158,87 @@ __global__ void __launch_bounds__(256) k_group_copy(const int32_t* __restrict__ 
   }
 }
 
+
+// Step 3 (default): the same copy in source order -- rows read sequentially, each
+// row's entries written to its member's slot of the grouped layout (dbase[u] =
+// gpos[rank of u]); the only random access per entry is the map[col] gather.
+__global__ void k_dest_base(const int32_t* __restrict__ vorder, const int64_t* __restrict__ gpos, int64_t n,
+                            int64_t* dbase) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    dbase[vorder[i]] = gpos[i];
+}
+
+constexpr int kSTile = 4096;  // CSR entries per scatter-copy tile
+constexpr int kSRows = 1024;  // rows staged per tile (else per-entry search in global memory)
+__global__ void __launch_bounds__(256) k_scatter_copy(const int64_t* __restrict__ rowptr, int64_t n,
+                                                      const int32_t* __restrict__ col,
+                                                      const uint32_t* __restrict__ w,
+                                                      const int32_t* __restrict__ map,
+                                                      const int64_t* __restrict__ dbase, int64_t nnz,
+                                                      const int64_t* __restrict__ tr, int32_t* gc, uint32_t* gw) {
+  __shared__ int64_t sh_rp[kSRows + 1];
+  __shared__ int64_t sh_db[kSRows];
+  __shared__ int64_t sh_u0;
+  __shared__ int sh_nr;
+  const int64_t ntiles = (nnz + kSTile - 1) / kSTile;
+  for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
+    const int64_t e0 = tile * kSTile, e1 = min(nnz, e0 + kSTile);
+    if (threadIdx.x == 0) {
+      const int64_t u0 = tr[tile], u1 = tr[tile + 1];
+      sh_u0 = u0;
+      sh_nr = (u1 - u0 + 1 <= kSRows) ? (int)(u1 - u0 + 1) : -1;
+    }
+    __syncthreads();
+    const int64_t u0 = sh_u0;
+    const int nr = sh_nr;
+    for (int r = threadIdx.x; r < nr; r += blockDim.x) {
+      sh_rp[r] = rowptr[u0 + r];
+      sh_db[r] = dbase[u0 + r];
+    }
+    __syncthreads();
+    for (int64_t base = e0 + threadIdx.x; base < e1; base += 4 * (int64_t)blockDim.x) {
+      int32_t jj[4];
+      int64_t dd[4];
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        const int64_t e = base + (int64_t)q * blockDim.x;
+        jj[q] = -1;
+        dd[q] = 0;
+        if (e < e1) {
+          if (nr > 0) {
+            int lo = 0, hi = nr - 1;  // largest r with sh_rp[r] <= e
+            while (lo < hi) {
+              const int mid = (lo + hi + 1) >> 1;
+              if (sh_rp[mid] <= e) lo = mid; else hi = mid - 1;
+            }
+            dd[q] = sh_db[lo] + (e - sh_rp[lo]);
+          } else {
+            int64_t lo = 0, hi = n - 1;
+            while (lo < hi) {
+              const int64_t mid = (lo + hi + 1) >> 1;
+              if (rowptr[mid] <= e) lo = mid; else hi = mid - 1;
+            }
+            dd[q] = dbase[lo] + (e - rowptr[lo]);
+          }
+          jj[q] = __ldcs(&col[e]);
+        }
+      }
+      int32_t mm[4];
+#pragma unroll
+      for (int q = 0; q < 4; ++q) mm[q] = jj[q] >= 0 ? __ldg(&map[jj[q]]) : 0;
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        const int64_t e = base + (int64_t)q * blockDim.x;
+        if (e < e1) {
+          gc[dd[q]] = mm[q];
+          if (gw) gw[dd[q]] = w ? __ldcs(&w[e]) : 1u;
+        }
+      }
+    }
+    __syncthreads();
+  }
+}
+
 // Step 4a: segments of <= 32 entries, one warp each; distinct neighbours written
 // compactly from the segment start; cnt[r] = distinct count.
 __global__ void __launch_bounds__(256) k_merge_small(const int32_t* __restrict__ rows, int64_t nr,
@@ -326,7 +407,217 @@ __global__ void k_big_place(const unsigned long long* __restrict__ ukeys, const 
 }
 
 
-// Step 4d (default): big segments merged in global-memory hash tables kept
+
+// Step 4d (LV_BIG_PART=1): big segments merged by label partitioning.  Segment k gets
+// P_k = ceil(min(len, n') / kCPartLabels) partitions (part_of(label, P_k)); its
+// entries are scattered into partition order (histogram -> per-segment scan ->
+// scatter, in chunks), then one CTA per (segment, partition) sums its share in a
+// shared-memory table and appends the distinct (neighbour, weight) pairs to the
+// segment's output (warp-aggregated cursor cnt[row]).  A table passing 7/8 load
+// sets a flag and the host redoes the big segments with the radix sort.
+constexpr int64_t kCPartLabels = 4096;  // expected distinct labels per partition (load <= 1/4)
+constexpr int kCPartSlots = 16384;      // 8-byte slots per partition table (128 KB)
+constexpr int kCPartMaxP = 4096;
+constexpr int64_t kCPartChunk = 32768;
+struct CSeg {
+  int64_t src;    // segment start in gc/gw (== its output start in oc/ow)
+  int64_t pbase;  // first poff index (sum of P + 1 of earlier segments)
+  int32_t row;
+  int32_t P;
+  int32_t first;  // first task / cursor index
+  int32_t pad;
+};
+struct CChunk {
+  int32_t seg;
+  int32_t pad;
+  int64_t begin, end;
+};
+struct CTask {
+  int32_t seg;
+  int32_t p;
+};
+
+__global__ void __launch_bounds__(1024) k_cpart_hist(const CChunk* __restrict__ chunks, int64_t nch,
+                                                     const CSeg* __restrict__ segs, const int32_t* __restrict__ gc,
+                                                     int64_t* poff) {
+  __shared__ uint32_t hist[kCPartMaxP];
+  const int lane = threadIdx.x & 31;
+  for (int64_t ci = blockIdx.x; ci < nch; ci += gridDim.x) {
+    const CChunk ch = chunks[ci];
+    const CSeg sg = segs[ch.seg];
+    const uint32_t P = (uint32_t)sg.P;
+    for (uint32_t q = threadIdx.x; q < P; q += blockDim.x) hist[q] = 0;
+    __syncthreads();
+    for (int64_t t0 = ch.begin + (threadIdx.x - lane); t0 < ch.end; t0 += blockDim.x) {
+      const int64_t t = t0 + lane;
+      const uint32_t q = (t < ch.end) ? part_of(__ldcs(&gc[sg.src + t]), P) : 0xFFFFFFFFu;
+      const unsigned m = __match_any_sync(kFull, q);
+      if (q != 0xFFFFFFFFu && lane == __ffs(m) - 1) atomicAdd(&hist[q], (uint32_t)__popc(m));
+    }
+    __syncthreads();
+    for (uint32_t q = threadIdx.x; q < P; q += blockDim.x)
+      if (hist[q]) atomicAdd(reinterpret_cast<unsigned long long*>(&poff[sg.pbase + 1 + q]), (unsigned long long)hist[q]);
+    __syncthreads();
+  }
+}
+
+// warp per segment: counts -> partition starts (relative to the segment) + scatter cursors
+__global__ void k_cpart_scan(const CSeg* __restrict__ segs, int64_t nseg, int64_t* poff, unsigned long long* cur) {
+  const int lane = threadIdx.x & 31;
+  const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
+  for (int64_t k = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); k < nseg; k += warps) {
+    const CSeg sg = segs[k];
+    long long run = 0;
+    for (int32_t q0 = 0; q0 < sg.P; q0 += 32) {
+      const int32_t q = q0 + lane;
+      const long long c = (q < sg.P) ? poff[sg.pbase + 1 + q] : 0;
+      long long x = c;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const long long y = __shfl_up_sync(kFull, x, o);
+        if (lane >= o) x += y;
+      }
+      if (q < sg.P) {
+        poff[sg.pbase + q] = run + x - c;
+        cur[sg.first + q] = (unsigned long long)(run + x - c);
+      }
+      run += __shfl_sync(kFull, x, 31);
+    }
+    if (lane == 0) poff[sg.pbase + sg.P] = run;
+  }
+}
+
+__global__ void __launch_bounds__(1024) k_cpart_scatter(const CChunk* __restrict__ chunks, int64_t nch,
+                                                        const CSeg* __restrict__ segs, const int32_t* __restrict__ gc,
+                                                        const uint32_t* __restrict__ gw, unsigned long long* cur,
+                                                        uint2* P2) {
+  __shared__ uint32_t hist[kCPartMaxP];
+  constexpr uint32_t kSeg = 1024;
+  __shared__ unsigned long long base[kSeg];
+  const int lane = threadIdx.x & 31;
+  for (int64_t ci = blockIdx.x; ci < nch; ci += gridDim.x) {
+    const CChunk ch = chunks[ci];
+    const CSeg sg = segs[ch.seg];
+    const uint32_t P = (uint32_t)sg.P;
+    for (uint32_t q = threadIdx.x; q < P; q += blockDim.x) hist[q] = 0;
+    __syncthreads();
+    for (int64_t t0 = ch.begin + (threadIdx.x - lane); t0 < ch.end; t0 += blockDim.x) {
+      const int64_t t = t0 + lane;
+      const uint32_t q = (t < ch.end) ? part_of(__ldcs(&gc[sg.src + t]), P) : 0xFFFFFFFFu;
+      const unsigned m = __match_any_sync(kFull, q);
+      if (q != 0xFFFFFFFFu && lane == __ffs(m) - 1) atomicAdd(&hist[q], (uint32_t)__popc(m));
+    }
+    __syncthreads();
+    for (uint32_t h0 = 0; h0 < P; h0 += kSeg) {
+      const uint32_t h1 = min(P, h0 + kSeg);
+      for (uint32_t q = h0 + threadIdx.x; q < h1; q += blockDim.x)
+        base[q - h0] = hist[q] ? atomicAdd(&cur[sg.first + q], (unsigned long long)hist[q]) : 0ull;
+      __syncthreads();
+      for (int64_t t0 = ch.begin + (threadIdx.x - lane); t0 < ch.end; t0 += blockDim.x) {
+        const int64_t t = t0 + lane;
+        int32_t c = 0;
+        uint32_t q = 0xFFFFFFFFu;
+        if (t < ch.end) {
+          c = __ldcs(&gc[sg.src + t]);
+          q = part_of(c, P);
+          if (q < h0 || q >= h1) q = 0xFFFFFFFFu;
+        }
+        const unsigned m = __match_any_sync(kFull, q);
+        unsigned long long b = 0;
+        const int leader = __ffs(m) - 1;
+        if (q != 0xFFFFFFFFu && lane == leader) b = atomicAdd(&base[q - h0], (unsigned long long)__popc(m));
+        b = __shfl_sync(m, b, leader);
+        if (q != 0xFFFFFFFFu) {
+          const unsigned long long dst = sg.src + b + __popc(m & ((1u << lane) - 1u));
+          __stcs(&P2[dst], make_uint2((uint32_t)c, gw ? __ldcs(&gw[sg.src + t]) : 1u));
+        }
+      }
+      __syncthreads();
+    }
+  }
+}
+
+// Task (segment, partition): insert the partition's entries into the smem table
+// (2 * n_p slots: no overflow possible; kCPartSlots with a distinct-label count
+// when n_p is larger), append the distinct (neighbour, weight) pairs to the
+// segment's output (warp-aggregated cursor cnt[row]), clearing the table.
+__global__ void __launch_bounds__(1024) k_cpart_merge(const CTask* __restrict__ tasks, int64_t ntasks,
+                                                      const CSeg* __restrict__ segs, const int64_t* __restrict__ poff,
+                                                      const uint2* __restrict__ P2, int32_t* oc, uint32_t* ow,
+                                                      int64_t* cnt, unsigned long long* overflow) {
+  extern __shared__ unsigned long long T[];  // kCPartSlots
+  __shared__ unsigned claimed;
+  for (int t = threadIdx.x; t < kCPartSlots; t += blockDim.x) T[t] = kEmpty;
+  if (threadIdx.x == 0) claimed = 0;
+  __syncthreads();
+  const int lane = threadIdx.x & 31;
+  const unsigned limit = (unsigned)(kCPartSlots / 8 * 7);
+  for (int64_t k = blockIdx.x; k < ntasks; k += gridDim.x) {
+    const CTask tk = tasks[k];
+    const CSeg sg = segs[tk.seg];
+    const int64_t q0 = sg.src + poff[sg.pbase + tk.p], q1 = sg.src + poff[sg.pbase + tk.p + 1];
+    const int64_t n_p = q1 - q0;
+    const bool big = 2 * n_p > kCPartSlots;
+    const uint32_t cap = big ? (uint32_t)kCPartSlots : (uint32_t)(n_p > 0 ? 2 * n_p : 1);
+    unsigned claims = 0;
+    // warp-uniform trips; equal labels of a warp summed first (hot labels: one atomic per warp)
+    for (int64_t base = q0 + (threadIdx.x - lane); base < q1; base += 4 * (int64_t)blockDim.x) {
+      uint2 rr[4];
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        const int64_t t = base + lane + (int64_t)u * blockDim.x;
+        rr[u] = (t < q1) ? __ldcs(&P2[t]) : make_uint2(0xFFFFFFFFu, 0u);
+      }
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        const unsigned m = __match_any_sync(kFull, rr[u].x);
+        const uint32_t sum = __reduce_add_sync(m, rr[u].y);
+        bool cl = false;
+        if (rr[u].x != 0xFFFFFFFFu && lane == __ffs(m) - 1) {
+          const int32_t c = (int32_t)rr[u].x;
+          const unsigned long long key = ((unsigned long long)(uint32_t)c) << 32;
+          uint32_t h = hash_slot(c, cap);
+          for (uint32_t probes = 0; probes < cap; ++probes) {
+            const unsigned long long old = atomicCAS(&T[h], kEmpty, key | sum);
+            if (old == kEmpty) { cl = true; break; }
+            if ((old >> 32) == (unsigned long long)(uint32_t)c) {
+              atomicAdd(&T[h], (unsigned long long)sum);
+              break;
+            }
+            h = (h + 1 == cap) ? 0 : h + 1;
+          }
+        }
+        if (big) claims += __popc(__ballot_sync(kFull, cl));
+      }
+    }
+    if (big && lane == 0 && claims) atomicAdd(&claimed, claims);
+    __syncthreads();
+    if (big && threadIdx.x == 0) {
+      if (claimed > limit) atomicAdd(overflow, 1ull);
+      claimed = 0;
+    }
+    for (uint32_t t0 = 0; t0 < cap; t0 += blockDim.x) {
+      const uint32_t t = t0 + threadIdx.x;
+      const unsigned long long x = (t < cap) ? T[t] : kEmpty;
+      const bool has = x != kEmpty;
+      if (has) T[t] = kEmpty;
+      const unsigned m = __ballot_sync(kFull, has);
+      if (!m) continue;
+      unsigned long long b = 0;
+      const int leader = __ffs(m) - 1;
+      if (lane == leader) b = atomicAdd(reinterpret_cast<unsigned long long*>(&cnt[sg.row]), (unsigned long long)__popc(m));
+      b = __shfl_sync(kFull, b, leader);
+      if (has) {
+        const int64_t pos = sg.src + (int64_t)b + __popc(m & ((1u << lane) - 1u));
+        oc[pos] = (int32_t)(x >> 32);
+        ow[pos] = (uint32_t)x;
+      }
+    }
+    __syncthreads();
+  }
+}
+
+// Step 4d (LV_BIG_HASH=1, experimental): big segments merged in global-memory hash tables kept
 // L2-resident by processing the segments in waves (each wave's tables <= kBigWaveSlots
 // slots).  Table of a segment: cap = 2 * min(len, n') slots (load <= 1/2), split into
 // 4-slot buckets read with two 16-byte loads; a label is claimed at the first
@@ -595,13 +886,25 @@ int32_t level_contract_fast(Handle& h, Level& L, Level& out, int32_t* d_map, int
       gw = static_cast<uint32_t*>(p0);
     }
   }
-  {
+  static const bool grouped_copy = getenv("LV_GROUPED_COPY") && getenv("LV_GROUPED_COPY")[0] == '1';
+  if (grouped_copy) {  // grouped order (reads member rows where they lie)
     const int64_t* tr = nullptr;
     LV_TRY(tile_starts(h, gpos, 0, n, 0, nnz, kCTile, &tr));
     k_group_copy<<<grid_for((nnz + kCTile - 1) / kCTile, 1, 148 * 8), 256, 0, s>>>(vorder, gpos, n, L.rowptr, L.col,
                                                                                       L.w, d_map, tr, gc, gw);
+    LV_LAUNCHED();
+  } else {  // source order (default)
+    int64_t* dbase = nullptr;
+    LV_TRY(dalloc(&dbase, n, s));
+    k_dest_base<<<grid_for(n, 256), 256, 0, s>>>(vorder, gpos, n, dbase);
+    LV_LAUNCHED();
+    const int64_t* tr = nullptr;
+    LV_TRY(tile_starts(h, L.rowptr, 0, n, 0, nnz, kSTile, &tr));
+    k_scatter_copy<<<grid_for((nnz + kSTile - 1) / kSTile, 1, 148 * 8), 256, 0, s>>>(L.rowptr, n, L.col, L.w, d_map,
+                                                                                       dbase, nnz, tr, gc, gw);
+    LV_LAUNCHED();
+    dfree(dbase, s);
   }
-  LV_LAUNCHED();
   dfree(vorder, s);
   tr.mark(s, "copy");
   // segment bounds and classes
@@ -653,27 +956,123 @@ int32_t level_contract_fast(Handle& h, Level& L, Level& out, int32_t* d_map, int
   }
   LV_TRY(dalloc(&cnt, np + 1, s));
   LV_CUDA(cudaMemsetAsync(cnt, 0, 8 * (np + 1), s));
+  // small / warp / mid merges on the side stream, concurrent with the big-segment
+  // waves on the main stream (independent segments, disjoint outputs)
+  static const bool serial = getenv("LV_SERIAL") && getenv("LV_SERIAL")[0] == '1';
+  cudaStream_t ms = (serial || tr.on) ? s : h.side;
+  if (ms != s) {
+    LV_CUDA(cudaEventRecord(h.ev_fork, s));
+    LV_CUDA(cudaStreamWaitEvent(ms, h.ev_fork, 0));
+  }
   if (nsmall > 0) {
-    k_merge_small<<<grid_for(nsmall, 8, 148 * 16), 256, 0, s>>>(rows, nsmall, sstart, send_, gc, gw, oc, ow, cnt);
+    k_merge_small<<<grid_for(nsmall, 8, 148 * 16), 256, 0, ms>>>(rows, nsmall, sstart, send_, gc, gw, oc, ow, cnt);
     LV_LAUNCHED();
   }
+  tr.mark(s, "merge-small");
   if (nwarp > 0) {
-    k_merge_warp<<<grid_for(nwarp, 4, 148 * 12), 128, 0, s>>>(rows + nsmall, nwarp, sstart, send_, gc, gw, oc, ow, cnt);
+    k_merge_warp<<<grid_for(nwarp, 4, 148 * 12), 128, 0, ms>>>(rows + nsmall, nwarp, sstart, send_, gc, gw, oc, ow, cnt);
     LV_LAUNCHED();
   }
+  tr.mark(s, "merge-warp");
   if (nmid > 0) {
     static bool attr = false;
     if (!attr) {
       LV_CUDA(cudaFuncSetAttribute(k_merge_mid, cudaFuncAttributeMaxDynamicSharedMemorySize, 8 * kMidSlots));
       attr = true;
     }
-    k_merge_mid<<<grid_for(nmid, 1, 148), 512, 8 * kMidSlots, s>>>(rows + nsmall + nwarp, nmid, sstart, send_, gc, gw,
+    k_merge_mid<<<grid_for(nmid, 1, 148 * 3), 512, 8 * kMidSlots, ms>>>(rows + nsmall + nwarp, nmid, sstart, send_, gc, gw,
                                                                     oc, ow, cnt);
     LV_LAUNCHED();
   }
-  tr.mark(s, "merge-sm");
-  static const bool big_sort = getenv("LV_BIG_SORT") && getenv("LV_BIG_SORT")[0] == '1';
-  if (nbig > 0 && !big_sort) {
+  tr.mark(s, "merge-mid");
+  // LV_BIG_HASH=1: L2-wave global hash tables for the big segments (measured slower
+  // than the radix sort on C5: 70/99/240 ms vs 63/69/72 ms at levels 0/1/2 -- atomic
+  // round trips and hot-label contention), kept as an experiment
+  static const bool big_hash = getenv("LV_BIG_HASH") && getenv("LV_BIG_HASH")[0] == '1';
+  // LV_BIG_PART=1: label-partitioned smem merge of the big segments (measured 66/75/114 ms
+  // vs the radix sort's 63/69/72 ms at C5 levels 0/1/2; kept as an option)
+  static const bool big_part = getenv("LV_BIG_PART") && getenv("LV_BIG_PART")[0] == '1';
+  bool big_done = false;
+  if (nbig > 0 && !big_hash && big_part) {
+    const int32_t* brows = rows + nsmall + nwarp + nmid;
+    std::vector<int32_t> hb(nbig);
+    LV_CUDA(cudaMemcpyAsync(hb.data(), brows, 4 * nbig, cudaMemcpyDeviceToHost, s));
+    std::vector<int64_t> hs(np + 1);
+    LV_CUDA(cudaMemcpyAsync(hs.data(), sstart, 8 * (np + 1), cudaMemcpyDeviceToHost, s));
+    LV_CUDA(cudaStreamSynchronize(s));
+    std::vector<CSeg> segs;
+    std::vector<CChunk> chunks;
+    std::vector<CTask> tasks;
+    int64_t pb = 0, big_entries = 0;
+    bool fits = true;
+    std::stable_sort(hb.begin(), hb.end(),  // longest first: one CTA walks a whole segment
+                     [&](int32_t a, int32_t b) { return hs[a + 1] - hs[a] > hs[b + 1] - hs[b]; });
+    for (int64_t k = 0; k < nbig; ++k) {
+      const int32_t r = hb[k];
+      const int64_t len = hs[r + 1] - hs[r];
+      big_entries += len;
+      const int64_t P = (std::min<int64_t>(len, np) + kCPartLabels - 1) / kCPartLabels;
+      if (P > kCPartMaxP) { fits = false; break; }
+      segs.push_back(CSeg{hs[r], pb, r, (int32_t)P, (int32_t)tasks.size(), 0});
+      pb += P + 1;
+      for (int32_t q = 0; q < (int32_t)P; ++q) tasks.push_back(CTask{(int32_t)k, q});
+      for (int64_t e = 0; e < len; e += kCPartChunk) chunks.push_back(CChunk{(int32_t)k, 0, e, std::min(len, e + kCPartChunk)});
+    }
+    if (tr.on)
+      fprintf(stderr, "[lv]    contract segments: small %lld warp %lld mid %lld big %lld (big entries %lld of %lld, "
+              "%zu partition tasks)\n", (long long)nsmall, (long long)nwarp, (long long)nmid, (long long)nbig,
+              (long long)big_entries, (long long)nnz, tasks.size());
+    if (fits) {
+      const int64_t ns = (int64_t)segs.size(), nt = (int64_t)tasks.size(), nc = (int64_t)chunks.size();
+      CSeg* dsegs = nullptr;
+      CChunk* dch = nullptr;
+      CTask* dt = nullptr;
+      int64_t* poff = nullptr;
+      unsigned long long* cur = nullptr;
+      LV_TRY(dalloc(&dsegs, ns, s));
+      LV_TRY(dalloc(&dch, nc, s));
+      LV_TRY(dalloc(&dt, nt, s));
+      LV_TRY(dalloc(&poff, pb, s));
+      LV_TRY(dalloc(&cur, nt, s));
+      LV_CUDA(cudaMemcpyAsync(dsegs, segs.data(), sizeof(CSeg) * ns, cudaMemcpyHostToDevice, s));
+      LV_CUDA(cudaMemcpyAsync(dch, chunks.data(), sizeof(CChunk) * nc, cudaMemcpyHostToDevice, s));
+      LV_CUDA(cudaMemcpyAsync(dt, tasks.data(), sizeof(CTask) * nt, cudaMemcpyHostToDevice, s));
+      LV_CUDA(cudaMemsetAsync(poff, 0, 8 * (size_t)pb, s));
+      LV_CUDA(cudaMemsetAsync(&h.ctl->overflow, 0, 8, s));
+      uint2* P2 = nullptr;
+      {
+        void* p0 = nullptr;
+        LV_TRY(scratch_get(h, SC_STAGE, 8 * (size_t)nnz, &p0));  // the level's stage is dead during contraction
+        P2 = static_cast<uint2*>(p0);
+      }
+      static bool attr = false;
+      if (!attr) {
+        LV_CUDA(cudaFuncSetAttribute(k_cpart_merge, cudaFuncAttributeMaxDynamicSharedMemorySize, 8 * kCPartSlots));
+        attr = true;
+      }
+      k_cpart_hist<<<grid_for(nc, 1, 148 * 2), 1024, 0, s>>>(dch, nc, dsegs, gc, poff);
+      LV_LAUNCHED();
+      k_cpart_scan<<<grid_for(ns, 8, 148 * 4), 256, 0, s>>>(dsegs, ns, poff, cur);
+      LV_LAUNCHED();
+      k_cpart_scatter<<<grid_for(nc, 1, 148 * 2), 1024, 0, s>>>(dch, nc, dsegs, gc, gw, cur, P2);
+      LV_LAUNCHED();
+      k_cpart_merge<<<grid_for(nt, 1, 148), 1024, 8 * kCPartSlots, s>>>(dt, nt, dsegs, poff, P2, oc, ow, cnt,
+                                                                        &h.ctl->overflow);
+      LV_LAUNCHED();
+      LV_CUDA(cudaGetLastError());
+      unsigned long long ovf = 0;
+      LV_CUDA(cudaMemcpyAsync(&ovf, &h.ctl->overflow, 8, cudaMemcpyDeviceToHost, s));
+      LV_CUDA(cudaStreamSynchronize(s));  // host vectors die here
+      dfree(dsegs, s);
+      dfree(dch, s);
+      dfree(dt, s);
+      dfree(poff, s);
+      dfree(cur, s);
+      big_done = ovf == 0;  // else: a partition table overflowed -> radix-sort fallback below
+      if (ovf) LV_CUDA(cudaMemsetAsync(&h.ctl->overflow, 0, 8, s));
+    }
+  }
+  if (nbig > 0 && big_hash && !big_done) {
     const int32_t* brows = rows + nsmall + nwarp + nmid;
     std::vector<int32_t> hb(nbig);
     LV_CUDA(cudaMemcpyAsync(hb.data(), brows, 4 * nbig, cudaMemcpyDeviceToHost, s));
@@ -736,7 +1135,9 @@ int32_t level_contract_fast(Handle& h, Level& L, Level& out, int32_t* d_map, int
     dfree(dins, s);
     dfree(dext, s);
     LV_CUDA(cudaStreamSynchronize(s));  // host vectors die here
-  } else if (nbig > 0) {  // LV_BIG_SORT=1: radix sort of (segment rank, neighbour) keys + reduce-by-key
+    big_done = true;
+  }
+  if (nbig > 0 && !big_done) {  // radix sort of (segment rank, neighbour) keys + reduce-by-key
     const int32_t* brows = rows + nsmall + nwarp + nmid;
     // offsets of big segments in the key array (their lengths, host-side: nbig is small)
     std::vector<int32_t> hb(nbig);
@@ -800,6 +1201,10 @@ int32_t level_contract_fast(Handle& h, Level& L, Level& out, int32_t* d_map, int
     LV_LAUNCHED();
     dfree(first_run, s);
     dfree(dboff, s);
+  }
+  if (ms != s) {
+    LV_CUDA(cudaEventRecord(h.ev_join, ms));
+    LV_CUDA(cudaStreamWaitEvent(s, h.ev_join, 0));
   }
   tr.mark(s, "merge-big");
   dfree(rows, s);

@@ -41,6 +41,18 @@ __device__ __forceinline__ void table_add(unsigned long long* T, uint32_t cap, i
   }
 }
 
+// Partition of label c among P label-partitioned tasks: fmix32 (independent of
+// hash_slot's multiplier) scaled to [0, P).
+__device__ __forceinline__ uint32_t part_of(int32_t c, uint32_t P) {
+  uint32_t h = (uint32_t)c;  // fmix32 (independent of hash_slot's multiplier)
+  h ^= h >> 16;
+  h *= 0x85ebca6bu;
+  h ^= h >> 13;
+  h *= 0xc2b2ae35u;
+  h ^= h >> 16;
+  return (uint32_t)(((unsigned long long)h * P) >> 32);
+}
+
 // xor-butterfly reduction over aligned groups of G lanes: best candidate + sum.
 template <int G>
 __device__ __forceinline__ void group_reduce(long long& s, int& c, unsigned& eown) {

@@ -142,6 +142,9 @@ int32_t init_handle(Handle& h, void* stream) {
   LV_CUDA(cudaMemset(h.ctl, 0, sizeof(DevCtl)));
   LV_CUDA(cudaMallocHost(&h.h_ctl, sizeof(DevCtl)));
   for (auto& e : h.ev) LV_CUDA(cudaEventCreate(&e));
+  LV_CUDA(cudaStreamCreateWithFlags(&h.side, cudaStreamNonBlocking));
+  LV_CUDA(cudaEventCreateWithFlags(&h.ev_fork, cudaEventDisableTiming));
+  LV_CUDA(cudaEventCreateWithFlags(&h.ev_join, cudaEventDisableTiming));
   return LOUVAIN_OK;
 }
 
@@ -156,6 +159,12 @@ void destroy_handle(Handle& h) {
   if (h.h_ctl) cudaFreeHost(h.h_ctl);
   for (auto& e : h.ev)
     if (e) cudaEventDestroy(e);
+  if (h.side) {
+    cudaStreamSynchronize(h.side);
+    cudaStreamDestroy(h.side);
+  }
+  if (h.ev_fork) cudaEventDestroy(h.ev_fork);
+  if (h.ev_join) cudaEventDestroy(h.ev_join);
   if (h.own_stream && h.stream) cudaStreamDestroy(h.stream);
 }
 
@@ -403,8 +412,8 @@ int32_t run_impl(Handle& h, const louvain_params_t& p, int32_t* labels_out, louv
       Level next;
       LV_TRY(dalloc(&map, L.n, s));
       tr.mark(s, "pre-contract", level);
-      // sort-based (default) or mergeCommunity-style hashing (LV_CONTRACT=hash, NEXT-1)
-      static const bool hash_contract = getenv("LV_CONTRACT") && std::string(getenv("LV_CONTRACT")) == "hash";
+      // mergeCommunity-style grouping + hashing (default, NEXT-1) or the canonical sort-based one (LV_CONTRACT=sort)
+      static const bool hash_contract = !(getenv("LV_CONTRACT") && std::string(getenv("LV_CONTRACT")) == "sort");
       if (hash_contract) LV_TRY(level_contract_fast(h, L, next, map, (level + 1) & 1));
       else LV_TRY(level_contract(h, L, next, map, (level + 1) & 1));
       tr.mark(s, "contract", level);

@@ -41,14 +41,12 @@ int32_t cuda_fail(cudaError_t e, const char* what, const char* file, int line);
 //   sub 0: deg < 1024   (register / warp / 256-thread CTA kernels, by bucket bound)
 //   sub 1: [1024, 4096) 512-thread CTA, smem table <= 8192 slots
 //   sub 2: [4096,12288) 1024-thread CTA, smem table <= 16384 slots
-//   sub 3: [12288, 32768)   label-partitioned CTA tasks (P = ceil(deg/6144) smem tables)
-//   sub 4: [32768, 393216)  label-partitioned CTA tasks (P <= 64)
-//   sub 5: >= 393216        hub: cooperative grid, global table in an L2-sized ring
-//   (P * deg streamed entries would grow quadratically beyond sub 4)
+//   sub 3..5: >= 12288      label-partitioned CTA tasks (P = ceil(deg/6144) smem tables,
+//                           the staged entries pre-partitioned); sub 5 (>= 393216) with
+//                           P > kPartMaxP only: hub, cooperative grid, global table ring
 constexpr int kSubPerBucket = 8;
 constexpr int kNumClasses = 8 * kSubPerBucket;
 constexpr int64_t kSub1Min = 1024, kSub2Min = 4096, kSub3Min = 12288, kSub4Min = 32768, kHubMin = 393216;
-constexpr int kClusterSlots = 16384;  // table slots per cluster CTA (12 B each: 192 KB)
 constexpr int kCap0 = 2048, kCap1 = 8192, kCap2 = 16384;  // smem table slots (12 B each)
 constexpr int64_t kHubChunkEdges = 2048;  // edges per hub insert item
 constexpr int64_t kHubScanSlots = 4096;   // slots per hub scan item
@@ -95,25 +93,45 @@ struct HubPlan {
   uint32_t* ring_a = nullptr;          // a_c when known (0xFFFFFFFF = unknown)
   void* partial = nullptr;             // [nscan]
   int grid = 0;                        // co-resident CTAs of the cooperative kernel
+  int64_t bucket_wave[9] = {0};        // waves of bucket b: [bucket_wave[b-1], bucket_wave[b])
 };
 
 // Label-partitioned plan for vertices of degree >= kSub3Min: vertex v gets
-// P_v = ceil(deg / kPartLabels) CTA tasks; task p keeps the labels c with
-// part_hash(c) % P_v == p in its own shared-memory table.
+// P_v = ceil(deg / kPartLabels) CTA tasks; task p owns the labels c with
+// part_of(c, P_v) == p.  Each sweep the vertex's staged entries are first
+// scattered into partition order (histogram -> per-vertex scan -> scatter, in
+// chunks of kPartChunk entries), so task p reads only its own share and keeps
+// it in one shared-memory table.  Vertices with P_v > kPartMaxP (deg > 50 M)
+// go to the cooperative hub kernel instead.
 constexpr int64_t kPartLabels = 6144;  // expected distinct labels per task (table load <= 3/8)
 constexpr int kPartSlots = 16384;      // smem table slots per task (12 B each: 192 KB)
+constexpr int kPartMaxP = 8192;        // partitions per vertex (smem histogram of a chunk)
+constexpr int64_t kPartChunk = 32768;  // staged entries per histogram / scatter item
+struct PartChunk {
+  int32_t vi;  // plan vertex
+  int32_t pad;
+  int64_t begin, end;  // entries of the vertex's staged segment
+};
 struct PartPlan {
-  int64_t ntasks = 0, nverts = 0;
+  int64_t ntasks = 0, nverts = 0, nchunks = 0, npoff = 0;
   int32_t* task_vpos = nullptr;   // [ntasks] index into the plan's vertex list
   int32_t* task_p = nullptr;      // [ntasks] partition index
   int32_t* vert_pos = nullptr;    // [nverts] bin position of the vertex
   int32_t* vert_P = nullptr;      // [nverts] partitions of the vertex
   int32_t* vert_first = nullptr;  // [nverts] first task (= first partial)
+  int64_t* vert_pbase = nullptr;  // [nverts] first poff index (sum of (P+1) of earlier vertices)
   int32_t* done = nullptr;        // [nverts] tasks finished (reset every sweep)
   void* partial = nullptr;        // [ntasks] Partial
+  int64_t* poff = nullptr;        // [npoff] partition starts in the partitioned stage (+ end)
+  unsigned long long* pcur = nullptr;  // [ntasks] scatter cursors
+  PartChunk* chunks = nullptr;    // [nchunks]
   int64_t bucket_task[9] = {0};   // tasks of bucket b: [bucket_task[b-1], bucket_task[b])
   int64_t bucket_vert[9] = {0};   // plan vertices of bucket b
+  int64_t bucket_chunk[9] = {0};  // chunks of bucket b (pre-partitioned vertices only)
+  int64_t bucket_vsplit[8] = {0};  // bucket b's vertices [bucket_vert[b-1], vsplit) are pre-partitioned,
+  int64_t bucket_tsplit[8] = {0};  // tasks [bucket_task[b-1], tsplit); the rest stream (P <= kStreamMaxP)
 };
+constexpr int64_t kStreamMaxP = 64;
 
 // Batched plan for the table-based vertices of degree <= kBatchMaxDeg (sub-class 0
 // of buckets whose bound exceeds 32): consecutive bin positions are cut into
@@ -142,6 +160,7 @@ struct Level {
   bool k_ready = false;  // k already holds the degrees (contracted level: community totals)
   uint32_t* k = nullptr;
   uint2* ca = nullptr;  // {C[v], a[v]}
+  int32_t* C = nullptr;  // copy of C[v] (4-byte label gathers of the modularity pass)
   int32_t* size = nullptr;
   // move log of the current sweep (v, new, old) -- also the revert record (R15)
   int32_t* mv_v = nullptr;
@@ -173,9 +192,9 @@ struct Level {
 enum ScratchSlot {
   SC_STAGE = 0, SC_GC, SC_GW, SC_OC, SC_OW, SC_K1, SC_V0, SC_V1, SC_TMP, SC_TILES,
   // arrays of a contracted level inside louvain_run, double-buffered by level parity
-  SC_LVL0, SC_LVL_END = SC_LVL0 + 2 * 11, SC_COUNT = SC_LVL_END
+  SC_LVL0, SC_LVL_END = SC_LVL0 + 2 * 12, SC_COUNT = SC_LVL_END
 };
-enum LevelArray { LA_ROWPTR = 0, LA_COL, LA_W, LA_K, LA_CA, LA_SIZE, LA_MVV, LA_MVN, LA_MVO, LA_BIN, LA_SOFF };
+enum LevelArray { LA_ROWPTR = 0, LA_COL, LA_W, LA_K, LA_CA, LA_SIZE, LA_MVV, LA_MVN, LA_MVO, LA_BIN, LA_SOFF, LA_C };
 struct Scratch {
   void* p[SC_COUNT] = {nullptr};
   size_t bytes[SC_COUNT] = {0};
@@ -191,6 +210,9 @@ struct Handle {
   DevCtl* ctl = nullptr;     // device
   DevCtl* h_ctl = nullptr;   // pinned host mirror
   cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
+  // side stream for independent kernels inside one phase (fork/join through events)
+  cudaStream_t side = nullptr;
+  cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
   // distributed (nullptr when single GPU)
   void* dist = nullptr;
 };

@@ -6,6 +6,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <cstdlib>
 #include <cstring>
 #include <vector>
 
@@ -24,17 +25,19 @@ __global__ void k_degrees_unit(const int64_t* rowptr, int64_t n, uint32_t* k) {
     k[i] = (uint32_t)(rowptr[i + 1] - rowptr[i]);
 }
 
-__global__ void k_init_singletons(const uint32_t* k, int64_t n, uint2* ca, int32_t* size) {
+__global__ void k_init_singletons(const uint32_t* k, int64_t n, uint2* ca, int32_t* size, int32_t* C) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
     ca[i] = make_uint2((uint32_t)i, k[i]);  // C[i] = i, a_C(i) = k_i
+    C[i] = (int32_t)i;
     size[i] = 1;
   }
 }
 
 // C[i] = labels[i] (or i), a = 0, size = 0; the C write keeps the packed record's a word.
-__global__ void k_set_C(const int32_t* labels, int64_t n, uint2* ca, int32_t* size) {
+__global__ void k_set_C(const int32_t* labels, int64_t n, uint2* ca, int32_t* size, int32_t* C) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
     ca[i] = make_uint2(labels ? (uint32_t)labels[i] : (uint32_t)i, 0u);
+    C[i] = labels ? labels[i] : (int32_t)i;
     size[i] = 0;
   }
 }
@@ -119,7 +122,7 @@ __global__ void k_fill_u32v(uint32_t* p, int64_t n, uint32_t v) {
 // Commit of one bucket (Alg. 1 l.8-11): C[i] = newComm[i] and the exact
 // integer a_c / size_c deltas (identical to recomputing a_c, R12).
 __global__ void k_commit(DevCtl* ctl, int bucket, const int32_t* mv_v, const int32_t* mv_new, int32_t* mv_old,
-                         uint2* ca, int32_t* size, const uint32_t* k) {
+                         uint2* ca, int32_t* size, const uint32_t* k, int32_t* C) {
   const unsigned long long start = ctl->bounds[bucket];
   const unsigned long long end = *(volatile unsigned long long*)&ctl->logn;
   if (blockIdx.x == 0 && threadIdx.x == 0) ctl->bounds[bucket + 1] = end;
@@ -130,6 +133,7 @@ __global__ void k_commit(DevCtl* ctl, int bucket, const int32_t* mv_v, const int
     const int32_t old = (int32_t)w32[2 * (int64_t)i];
     mv_old[p] = old;
     w32[2 * (int64_t)i] = (uint32_t)t;
+    C[i] = t;
     const uint32_t ki = k[i];
     atomicSub(&w32[2 * (int64_t)old + 1], ki);
     atomicAdd(&w32[2 * (int64_t)t + 1], ki);
@@ -140,13 +144,14 @@ __global__ void k_commit(DevCtl* ctl, int bucket, const int32_t* mv_v, const int
 
 // Undo every move of the sweep (R15).
 __global__ void k_revert(const DevCtl* ctl, const int32_t* mv_v, const int32_t* mv_new, const int32_t* mv_old,
-                         uint2* ca, int32_t* size, const uint32_t* k) {
+                         uint2* ca, int32_t* size, const uint32_t* k, int32_t* C) {
   const unsigned long long end = ctl->logn;
   uint32_t* w32 = reinterpret_cast<uint32_t*>(ca);
   for (unsigned long long p = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; p < end;
        p += (unsigned long long)gridDim.x * blockDim.x) {
     const int32_t i = mv_v[p], t = mv_new[p], old = mv_old[p];
     w32[2 * (int64_t)i] = (uint32_t)old;
+    C[i] = old;
     const uint32_t ki = k[i];
     atomicSub(&w32[2 * (int64_t)t + 1], ki);
     atomicAdd(&w32[2 * (int64_t)old + 1], ki);
@@ -203,15 +208,14 @@ __global__ void __launch_bounds__(256) k_modularity(const int64_t* rowptr, int64
   __shared__ int64_t sh_rows[kTileRows];
   __shared__ int64_t sh_u0;
   __shared__ int sh_nr;
-  const uint32_t* lab = PACKED ? reinterpret_cast<const uint32_t*>(ca) : reinterpret_cast<const uint32_t*>(C);
-  const int st = PACKED ? 2 : 1;
+  const uint32_t* lab = reinterpret_cast<const uint32_t*>(C);  // 4-byte labels (the level's copy, or external)
   unsigned long long acc = 0;
   const int64_t ntiles = (nnz - e_begin + kTileEdges - 1) / kTileEdges;
   for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
     const int64_t e0 = e_begin + tile * kTileEdges, e1 = min(nnz, e0 + kTileEdges);
     for_tile_edges(rowptr, n, e0, e1, tr, tile, sh_rows, &sh_u0, &sh_nr, [&](int64_t u, int64_t e) {
       const int32_t v = __ldcs(&col[e]);
-      if (__ldg(&lab[st * (int64_t)v]) == __ldg(&lab[st * u])) acc += w ? __ldcs(&w[e]) : 1u;
+      if (__ldg(&lab[v]) == __ldg(&lab[u])) acc += w ? __ldcs(&w[e]) : 1u;
     });
   }
   unsigned long long s2 = 0;
@@ -326,6 +330,7 @@ int32_t tile_starts(Handle& h, const int64_t* offs, int64_t lo, int64_t hi, int6
 int32_t level_alloc_state(Level& L, cudaStream_t s) {
   LV_TRY(dalloc(&L.k, L.n, s));
   LV_TRY(dalloc(&L.ca, L.n, s));
+  LV_TRY(dalloc(&L.C, L.n, s));
   LV_TRY(dalloc(&L.size, L.n, s));
   LV_TRY(dalloc(&L.mv_v, L.n, s));
   LV_TRY(dalloc(&L.mv_new, L.n, s));
@@ -334,6 +339,27 @@ int32_t level_alloc_state(Level& L, cudaStream_t s) {
   return LOUVAIN_OK;
 }
 
+static void part_free(PartPlan& Q, cudaStream_t s);
+// Most partitions a vertex may get on the label-partitioned path (more: hub kernel).
+// LV_PART_MAXP lowers it (tests use it to exercise the cooperative hub kernel).
+static int64_t part_maxp() {
+  static const int64_t v = [] {
+    const char* e = getenv("LV_PART_MAXP");
+    const long long x = e ? atoll(e) : 0;
+    return (x >= 1 && x < kPartMaxP) ? (int64_t)x : (int64_t)kPartMaxP;
+  }();
+  return v;
+}
+// Vertices with more partitions than this take the pre-partitioned tasks, the
+// others stream.  Measured on C5: streaming wins at levels 0/1 (31 vs 34 ms,
+// 16 vs 25 ms), pre-partitioning at level 2 (34 vs 47 ms), where the rows are
+// long (mean degree ~300) and labels concentrate; so a level with mean degree
+// >= 256 pre-partitions every hub vertex.  LV_STREAM_MAXP overrides.
+static int64_t stream_maxp(const Level& L) {
+  static const char* e = getenv("LV_STREAM_MAXP");
+  if (e) return (int64_t)atoll(e);
+  return (L.n > 0 && L.nnz / L.n >= 256) ? 0 : kStreamMaxP;
+}
 static void hub_free(HubPlan& P, cudaStream_t s) {
   dfree(P.ins, s); dfree(P.scans, s); dfree(P.ins_off, s); dfree(P.scan_off, s); dfree(P.wave_hub, s);
   dfree(P.info, s); dfree(P.ring, s);
@@ -346,6 +372,7 @@ int32_t level_alloc_scratch(Handle& h, Level& L, int parity) {
   auto get = [&](int a, size_t bytes, void** out) { return scratch_get(h, SC_LVL0 + 2 * a + parity, bytes, out); };
   LV_TRY(get(LA_K, 4 * n, (void**)&L.k));
   LV_TRY(get(LA_CA, 8 * n, (void**)&L.ca));
+  LV_TRY(get(LA_C, 4 * n, (void**)&L.C));
   LV_TRY(get(LA_SIZE, 4 * n, (void**)&L.size));
   LV_TRY(get(LA_MVV, 4 * n, (void**)&L.mv_v));
   LV_TRY(get(LA_MVN, 4 * n, (void**)&L.mv_new));
@@ -361,9 +388,7 @@ int32_t level_alloc_scratch(Handle& h, Level& L, int parity) {
 void level_free(Level& L, cudaStream_t s) {
   if (L.scratch_backed) {  // arrays belong to the handle's scratch; plans are per level
     hub_free(L.hub, s);
-    PartPlan& Q = L.part;
-    dfree(Q.task_vpos, s); dfree(Q.task_p, s); dfree(Q.vert_pos, s); dfree(Q.vert_P, s); dfree(Q.vert_first, s);
-    dfree(Q.done, s); dfree(Q.partial, s);
+    part_free(L.part, s);
     batch_free(L.batch, s);
     L = Level();
     return;
@@ -373,13 +398,11 @@ void level_free(Level& L, cudaStream_t s) {
     dfree(L.col, s);
     dfree(L.w, s);
   }
-  dfree(L.k, s); dfree(L.ca, s); dfree(L.size, s);
+  dfree(L.k, s); dfree(L.ca, s); dfree(L.C, s); dfree(L.size, s);
   dfree(L.mv_v, s); dfree(L.mv_new, s); dfree(L.mv_old, s); dfree(L.bin_vertices, s);
   dfree(L.soff, s);  // L.stage lives in the handle's scratch
   hub_free(L.hub, s);
-  PartPlan& Q = L.part;
-  dfree(Q.task_vpos, s); dfree(Q.task_p, s); dfree(Q.vert_pos, s); dfree(Q.vert_P, s); dfree(Q.vert_first, s);
-  dfree(Q.done, s); dfree(Q.partial, s);
+  part_free(L.part, s);
   batch_free(L.batch, s);
   L = Level();
 }
@@ -389,7 +412,7 @@ int32_t level_setup(Handle& h, Level& L) {
   const int64_t n = L.n;
   if (n == 0) { L.W = 0; return LOUVAIN_OK; }
   if (L.k_ready) {  // contracted level: k = community totals, W unchanged (set by level_contract)
-    k_init_singletons<<<grid_for(n, 256), 256, 0, s>>>(L.k, n, L.ca, L.size);
+    k_init_singletons<<<grid_for(n, 256), 256, 0, s>>>(L.k, n, L.ca, L.size, L.C);
     LV_LAUNCHED();
     LV_CUDA(cudaGetLastError());
     return LOUVAIN_OK;
@@ -419,7 +442,7 @@ int32_t level_setup(Handle& h, Level& L) {
     set_error("W = 2m exceeds 3,037,000,499 (int64 gain guard, R4)");
     return LOUVAIN_E_OVERFLOW;
   }
-  k_init_singletons<<<grid_for(n, 256), 256, 0, s>>>(L.k, n, L.ca, L.size);
+  k_init_singletons<<<grid_for(n, 256), 256, 0, s>>>(L.k, n, L.ca, L.size, L.C);
   LV_LAUNCHED();
   LV_CUDA(cudaGetLastError());
   return LOUVAIN_OK;
@@ -429,7 +452,7 @@ int32_t level_set_labels(Handle& h, Level& L, const int32_t* d_labels) {
   cudaStream_t s = h.stream;
   L.sweeps_done = d_labels ? 1 : 0;
   if (L.n == 0) return LOUVAIN_OK;
-  k_set_C<<<grid_for(L.n, 256), 256, 0, s>>>(d_labels, L.n, L.ca, L.size);
+  k_set_C<<<grid_for(L.n, 256), 256, 0, s>>>(d_labels, L.n, L.ca, L.size, L.C);
   LV_LAUNCHED();
   LV_CUDA(cudaMemsetAsync(&h.ctl->bad, 0, 8, s));
   k_totals_add<<<grid_for(L.n, 256), 256, 0, s>>>(L.ca, L.k, L.n, L.size, &h.ctl->bad);
@@ -460,7 +483,7 @@ int32_t level_get_a(Handle& h, Level& L, uint32_t* d_out) {
   return LOUVAIN_OK;
 }
 
-// Hub plan (vertices of sub-class 5, deg >= kHubMin, of any bucket): work items
+// Hub plan (vertices of sub-class 5 with more than kPartMaxP partitions, of any bucket): work items
 // in hub order -- inserts (kHubChunkEdges edges each), scans (kHubScanSlots
 // slots each), final -- and a ring of table slots reused hub after hub.
 static int32_t build_hub_plan(Handle& h, Level& L) {
@@ -468,9 +491,10 @@ static int32_t build_hub_plan(Handle& h, Level& L) {
   HubPlan& P = L.hub;
   std::vector<int32_t> hv;
   std::vector<int64_t> hdeg, rb, hsoff;
+  std::vector<int32_t> hbucket;
   for (int b = 1; b <= 7; ++b) {
-    const int c = kSubPerBucket * b + 5;
-    const int64_t off = L.class_off[c], cnt = L.class_off[c + 1] - off;
+    const int c = kSubPerBucket * b + 3;  // sub-classes 3..5 (P > part_maxp() only)
+    const int64_t off = L.class_off[c], cnt = L.class_off[c + 3] - off;
     if (cnt <= 0) continue;
     std::vector<int32_t> v(cnt);
     std::vector<int64_t> d(2 * cnt);
@@ -484,12 +508,17 @@ static int32_t build_hub_plan(Handle& h, Level& L) {
     LV_CUDA(cudaMemcpyAsync(so.data(), L.soff + off, 8 * cnt, cudaMemcpyDeviceToHost, s));
     LV_CUDA(cudaStreamSynchronize(s));
     dfree(dd, s);
-    hsoff.insert(hsoff.end(), so.begin(), so.end());
-    hv.insert(hv.end(), v.begin(), v.end());
-    hdeg.insert(hdeg.end(), d.begin(), d.begin() + cnt);
-    rb.insert(rb.end(), d.begin() + cnt, d.end());
+    for (int64_t i = 0; i < cnt; ++i) {
+      if ((d[i] + kPartLabels - 1) / kPartLabels <= part_maxp()) continue;  // label-partitioned path
+      hsoff.push_back(so[i]);
+      hv.push_back(v[i]);
+      hdeg.push_back(d[i]);
+      rb.push_back(d[cnt + i]);
+      hbucket.push_back(b);
+    }
   }
   P.nh = (int64_t)hv.size();
+  std::fill(P.bucket_wave, P.bucket_wave + 9, 0);
   if (P.nh == 0) return LOUVAIN_OK;
   std::vector<HubInfo> info(P.nh);
   std::vector<HubItem> ins, scans;
@@ -500,7 +529,8 @@ static int32_t build_hub_plan(Handle& h, Level& L) {
   int64_t acc = 0;
   for (int64_t i = 0; i < P.nh; ++i) {
     const int64_t cap = cap_of(hdeg[i]);
-    if (wave_hub.empty() || acc + cap > seg) {
+    if (wave_hub.empty() || acc + cap > seg || hbucket[i] != hbucket[i - 1]) {  // a wave never spans buckets
+      for (int b = (i == 0) ? 1 : hbucket[i - 1] + 1; b <= hbucket[i]; ++b) P.bucket_wave[b - 1] = (int64_t)wave_hub.size();
       wave_hub.push_back(i);
       ins_off.push_back((int64_t)ins.size());
       scan_off.push_back((int64_t)scans.size());
@@ -522,6 +552,7 @@ static int32_t build_hub_plan(Handle& h, Level& L) {
     }
   }
   P.nwaves = (int64_t)wave_hub.size();
+  for (int b = hbucket[P.nh - 1] + 1; b <= 8; ++b) P.bucket_wave[b - 1] = P.nwaves;
   wave_hub.push_back(P.nh);
   ins_off.push_back((int64_t)ins.size());
   scan_off.push_back((int64_t)scans.size());
@@ -553,55 +584,87 @@ static int32_t build_hub_plan(Handle& h, Level& L) {
   return LOUVAIN_OK;
 }
 
-// Partition plan for every vertex of sub-classes 3..4 (kSub3Min <= deg < kHubMin), any bucket.
+static void part_free(PartPlan& Q, cudaStream_t s) {
+  dfree(Q.task_vpos, s); dfree(Q.task_p, s); dfree(Q.vert_pos, s); dfree(Q.vert_P, s); dfree(Q.vert_first, s);
+  dfree(Q.vert_pbase, s); dfree(Q.done, s); dfree(Q.partial, s); dfree(Q.poff, s); dfree(Q.pcur, s);
+  dfree(Q.chunks, s);
+  Q = PartPlan();
+}
+
+// Partition plan for every vertex of sub-classes 3..5 (deg >= kSub3Min) with
+// P <= kPartMaxP, any bucket.
 int32_t build_part_plan(Handle& h, Level& L) {
   cudaStream_t s = h.stream;
   PartPlan& Q = L.part;
-  dfree(Q.task_vpos, s); dfree(Q.task_p, s); dfree(Q.vert_pos, s); dfree(Q.vert_P, s); dfree(Q.vert_first, s);
-  dfree(Q.done, s); dfree(Q.partial, s);
-  Q = PartPlan();
+  part_free(Q, s);
   std::vector<int32_t> vpos, vP, vfirst, tv, tp;
+  std::vector<int64_t> vpb;
+  std::vector<PartChunk> ch;
+  int64_t pb = 0;
   for (int b = 1; b <= 7; ++b) {
     Q.bucket_task[b - 1] = (int64_t)tv.size();
     Q.bucket_vert[b - 1] = (int64_t)vpos.size();
-    for (int sub = 3; sub <= 4; ++sub) {
-      const int c = kSubPerBucket * b + sub;
-      const int64_t off = L.class_off[c], cnt = L.class_off[c + 1] - off;
-      if (cnt <= 0) continue;
-      std::vector<int64_t> so(cnt + 1);
-      LV_CUDA(cudaMemcpyAsync(so.data(), L.soff + off, 8 * (cnt + 1), cudaMemcpyDeviceToHost, s));
-      LV_CUDA(cudaStreamSynchronize(s));
-      for (int64_t i = 0; i < cnt; ++i) {
-        const int64_t deg = so[i + 1] - so[i];
-        const int32_t P = (int32_t)((deg + kPartLabels - 1) / kPartLabels);
-        const int32_t vi = (int32_t)vpos.size();
-        vpos.push_back((int32_t)(off + i));
-        vP.push_back(P);
-        vfirst.push_back((int32_t)tv.size());
-        for (int32_t q = 0; q < P; ++q) {
-          tv.push_back(vi);
-          tp.push_back(q);
-        }
+    Q.bucket_chunk[b - 1] = (int64_t)ch.size();
+    Q.bucket_vsplit[b - 1] = (int64_t)vpos.size();
+    Q.bucket_tsplit[b - 1] = (int64_t)tv.size();
+    const int c0 = kSubPerBucket * b + 3, c1 = kSubPerBucket * b + 6;
+    const int64_t off = L.class_off[c0], cnt = L.class_off[c1] - off;
+    if (cnt <= 0) continue;
+    std::vector<int64_t> so(cnt + 1);
+    LV_CUDA(cudaMemcpyAsync(so.data(), L.soff + off, 8 * (cnt + 1), cudaMemcpyDeviceToHost, s));
+    LV_CUDA(cudaStreamSynchronize(s));
+    // longest first: a CTA walks all partitions of one vertex (sweep_part)
+    std::vector<int64_t> ord(cnt);
+    for (int64_t i = 0; i < cnt; ++i) ord[i] = i;
+    std::stable_sort(ord.begin(), ord.end(),
+                     [&](int64_t a, int64_t b) { return so[a + 1] - so[a] > so[b + 1] - so[b]; });
+    for (int64_t i : ord) {
+      const int64_t deg = so[i + 1] - so[i];
+      const int64_t P = (deg + kPartLabels - 1) / kPartLabels;
+      if (P > part_maxp()) continue;  // giant: cooperative hub kernel
+      const int32_t vi = (int32_t)vpos.size();
+      vpos.push_back((int32_t)(off + i));
+      vP.push_back((int32_t)P);
+      vfirst.push_back((int32_t)tv.size());
+      vpb.push_back(pb);
+      pb += P + 1;
+      for (int32_t q = 0; q < (int32_t)P; ++q) {
+        tv.push_back(vi);
+        tp.push_back(q);
+      }
+      if (P > stream_maxp(L)) {  // pre-partitioned (a prefix: degrees descending)
+        for (int64_t e = 0; e < deg; e += kPartChunk) ch.push_back(PartChunk{vi, 0, e, std::min(deg, e + kPartChunk)});
+        Q.bucket_vsplit[b - 1] = (int64_t)vpos.size();
+        Q.bucket_tsplit[b - 1] = (int64_t)tv.size();
       }
     }
   }
   Q.nverts = (int64_t)vpos.size();
   Q.ntasks = (int64_t)tv.size();
+  Q.nchunks = (int64_t)ch.size();
+  Q.npoff = pb;
   Q.bucket_task[7] = Q.ntasks;
   Q.bucket_vert[7] = Q.nverts;
+  Q.bucket_chunk[7] = Q.nchunks;
   if (Q.nverts == 0) return LOUVAIN_OK;
   LV_TRY(dalloc(&Q.task_vpos, Q.ntasks, s));
   LV_TRY(dalloc(&Q.task_p, Q.ntasks, s));
   LV_TRY(dalloc(&Q.vert_pos, Q.nverts, s));
   LV_TRY(dalloc(&Q.vert_P, Q.nverts, s));
   LV_TRY(dalloc(&Q.vert_first, Q.nverts, s));
+  LV_TRY(dalloc(&Q.vert_pbase, Q.nverts, s));
   LV_TRY(dalloc(&Q.done, Q.nverts, s));
   LV_TRY(dmalloc(&Q.partial, hub_partial_bytes() * (size_t)Q.ntasks, s));
+  LV_TRY(dalloc(&Q.poff, Q.npoff, s));
+  LV_TRY(dalloc(&Q.pcur, Q.ntasks, s));
+  LV_TRY(dalloc(&Q.chunks, Q.nchunks, s));
   LV_CUDA(cudaMemcpyAsync(Q.task_vpos, tv.data(), 4 * tv.size(), cudaMemcpyHostToDevice, s));
   LV_CUDA(cudaMemcpyAsync(Q.task_p, tp.data(), 4 * tp.size(), cudaMemcpyHostToDevice, s));
   LV_CUDA(cudaMemcpyAsync(Q.vert_pos, vpos.data(), 4 * vpos.size(), cudaMemcpyHostToDevice, s));
   LV_CUDA(cudaMemcpyAsync(Q.vert_P, vP.data(), 4 * vP.size(), cudaMemcpyHostToDevice, s));
   LV_CUDA(cudaMemcpyAsync(Q.vert_first, vfirst.data(), 4 * vfirst.size(), cudaMemcpyHostToDevice, s));
+  LV_CUDA(cudaMemcpyAsync(Q.vert_pbase, vpb.data(), 8 * vpb.size(), cudaMemcpyHostToDevice, s));
+  LV_CUDA(cudaMemcpyAsync(Q.chunks, ch.data(), sizeof(PartChunk) * ch.size(), cudaMemcpyHostToDevice, s));
   LV_CUDA(cudaStreamSynchronize(s));  // host vectors die here
   return LOUVAIN_OK;
 }
@@ -690,7 +753,7 @@ int32_t launch_modularity(Handle& h, Level& L, const int32_t* d_C) {
     LV_TRY(tile_starts(h, L.rowptr, 0, L.n, 0, 1, kTileEdges, &tr));  // unused (no tiles)
   }
   if (!d_C) {
-    k_modularity<true><<<grid, 256, 0, s>>>(L.rowptr, L.n, L.col, L.w, L.ca, nullptr, nullptr, e0, e1, tr, &h.ctl->L,
+    k_modularity<true><<<grid, 256, 0, s>>>(L.rowptr, L.n, L.col, L.w, L.ca, L.C, nullptr, e0, e1, tr, &h.ctl->L,
                                             &h.ctl->S);
     LV_LAUNCHED();
   } else {
@@ -723,7 +786,7 @@ int32_t level_modularity(Handle& h, Level& L, const int32_t* d_C, uint64_t* Lout
 }
 
 int32_t launch_commit(Handle& h, Level& L, int bucket) {
-  k_commit<<<148 * 4, 256, 0, h.stream>>>(h.ctl, bucket, L.mv_v, L.mv_new, L.mv_old, L.ca, L.size, L.k);
+  k_commit<<<148 * 4, 256, 0, h.stream>>>(h.ctl, bucket, L.mv_v, L.mv_new, L.mv_old, L.ca, L.size, L.k, L.C);
   LV_LAUNCHED();
   LV_CUDA(cudaGetLastError());
   return LOUVAIN_OK;
@@ -769,7 +832,7 @@ int32_t unpack_moves(Handle& h, Level& L, int64_t c0, int64_t cnt, const int32_t
 }
 
 int32_t launch_revert(Handle& h, Level& L) {
-  k_revert<<<148 * 4, 256, 0, h.stream>>>(h.ctl, L.mv_v, L.mv_new, L.mv_old, L.ca, L.size, L.k);
+  k_revert<<<148 * 4, 256, 0, h.stream>>>(h.ctl, L.mv_v, L.mv_new, L.mv_old, L.ca, L.size, L.k, L.C);
   LV_LAUNCHED();
   LV_CUDA(cudaGetLastError());
   return LOUVAIN_OK;

@@ -28,7 +28,9 @@
 //                   __reduce_add_sync (no shared memory).
 //   sweep_warp<CAP> deg <= 340: a warp per vertex, per-warp smem hash table.
 //   sweep_cta       deg < 12288: a CTA per vertex (persistent loop), smem table.
-//   hub_coop        deg >= 12288: one vertex split over many CTAs; a cooperative
+//   sweep_part      deg >= 12288: label-partitioned CTA tasks over the staged
+//                   entries, pre-scattered into partition order.
+//   hub_coop        deg > 50 M (more than kPartMaxP partitions): a cooperative
 //                   kernel pipelines waves of hubs (insert chunks -> table scan
 //                   chunks -> decision) across grid.sync() phases, the global
 //                   tables living in a 2-segment ring small enough for L2.
@@ -50,6 +52,7 @@
 namespace cg = cooperative_groups;
 
 namespace lv {
+static bool trace_on();  // LV_TRACE=2 (per-class / per-step timing, diagnostics only)
 namespace {
 
 constexpr uint32_t kUnknownA = 0xFFFFFFFFu;  // a_c < W <= 3,037,000,499 < 2^32 - 1
@@ -378,6 +381,83 @@ __global__ void __launch_bounds__(256) k_stage(const int32_t* __restrict__ bv, c
   }
 }
 
+// Warp-chunked variant of phase 1 (LV_STAGE_W=1): every warp takes chunks of
+// kStageChunk staged entries on its own -- no CTA barriers.  Lane r holds the
+// descriptor (entry offset, row start, vertex) of the r-th row touching the
+// chunk (tile plan at chunk granularity); a lane finds the row of each of its
+// entries by a 5-step shuffle search, and keeps 8 gathers in flight.  A chunk
+// touching more than 32 rows (rows shorter than 32 entries on average) falls
+// back to a binary search over soff.
+constexpr int kStageChunk = 1024;
+__global__ void __launch_bounds__(256) k_stage_w(const int32_t* __restrict__ bv, const int64_t* __restrict__ soff,
+                                                 int64_t pos0, int64_t pos1, int64_t s0, int64_t s1,
+                                                 const int64_t* __restrict__ tr, const int64_t* __restrict__ rowptr,
+                                                 const int32_t* __restrict__ col, const uint2* __restrict__ ca,
+                                                 uint2* __restrict__ stage) {
+  const int lane = threadIdx.x & 31;
+  const int64_t nchunks = (s1 - s0 + kStageChunk - 1) / kStageChunk;
+  const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
+  for (int64_t ch = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); ch < nchunks; ch += warps) {
+    const int64_t t0 = s0 + ch * kStageChunk, t1 = min(s1, t0 + kStageChunk);
+    const int64_t i0 = tr[ch], i1 = tr[ch + 1];
+    const int nr = (int)((i1 - i0 + 1 < 33) ? i1 - i0 + 1 : 33);
+    const bool fits = i1 - i0 + 1 <= 32;
+    // lane r: row i0 + r
+    int64_t my_so = INT64_MAX, my_rb = 0;
+    int32_t my_v = -1;
+    if (fits && lane < nr && i0 + lane < pos1) {
+      my_v = bv[i0 + lane];
+      my_so = soff[i0 + lane];
+      my_rb = rowptr[my_v];
+    }
+    for (int64_t b0 = t0; b0 < t1; b0 += 8 * 32) {  // warp-uniform trips (shuffles below)
+      const int64_t base = b0 + lane;
+      int32_t jj[8], vv[8];
+#pragma unroll
+      for (int q = 0; q < 8; ++q) {
+        const int64_t t = base + 32 * q;
+        int64_t e = 0;
+        vv[q] = -1;
+        jj[q] = -1;
+        if (fits) {
+          int lo = 0;  // largest r with so_r <= t (all lanes take part in the shuffles)
+#pragma unroll
+          for (int step = 16; step >= 1; step >>= 1) {
+            const int64_t so_mid = __shfl_sync(kFull, my_so, lo + step);
+            if (lo + step < nr && so_mid <= t) lo += step;
+          }
+          const int64_t so_r = __shfl_sync(kFull, my_so, lo);
+          const int64_t rb_r = __shfl_sync(kFull, my_rb, lo);
+          const int32_t v_r = __shfl_sync(kFull, my_v, lo);
+          if (t < t1) {
+            vv[q] = v_r;
+            e = rb_r + (t - so_r);
+          }
+        } else if (t < t1) {
+          int64_t lo = pos0, hi = pos1 - 1;
+          while (lo < hi) {
+            const int64_t mid = (lo + hi + 1) >> 1;
+            if (soff[mid] <= t) lo = mid; else hi = mid - 1;
+          }
+          vv[q] = bv[lo];
+          e = rowptr[vv[q]] + (t - soff[lo]);
+        }
+        if (t < t1) jj[q] = __ldcs(&col[e]);
+      }
+      uint2 rr[8];
+#pragma unroll
+      for (int q = 0; q < 8; ++q) rr[q] = (jj[q] >= 0 && jj[q] != vv[q]) ? __ldg(&ca[jj[q]]) : make_uint2(kSelf, 0);
+#pragma unroll
+      for (int q = 0; q < 8; ++q) {
+        const int64_t t = base + 32 * q;
+        if (t < t1)
+          __stcs(&stage[t], (jj[q] == vv[q]) ? make_uint2(kSelf, 0u)
+                                             : make_uint2(rr[q].x, rr[q].x == (uint32_t)jj[q] ? rr[q].y : kUnknownA));
+      }
+    }
+  }
+}
+
 // Phase 2 insert: entries [t0, deg) step `stride` of one vertex's staged
 // neighbours S (and weights Wt), 4 per pass, no random loads.  With AGG,
 // labels are first merged across the warp (__match_any_sync, weights summed
@@ -405,6 +485,9 @@ __device__ __forceinline__ void insert_staged(unsigned long long* T, uint32_t* T
     for (int q = 0; q < 4; ++q) {
       const bool valid = rr[q].x != kSelf;
       c[q] = valid ? (int32_t)rr[q].x : (int32_t)(0x80000000u | (unsigned)lane);
+      // (adaptive merging here measured 2-3x slower on the warp kernels of C5: the
+      // smem tables of these small rows tolerate same-slot atomics better than
+      // __match_any_sync costs; only the hub paths merge adaptively)
       if (AGG) {
         const unsigned m = __match_any_sync(kFull, c[q]);
         x[q] = UNIT ? (uint32_t)__popc(m) : __reduce_add_sync(m, ww[q]);
@@ -468,7 +551,7 @@ __global__ void __launch_bounds__(32 * WARPS) sweep_warp(const int32_t* __restri
   }
 }
 
-// ------------------------------------------------------------ CTA per vertex
+// ------------------------------------------------------------ CTA per vertex (default)
 template <bool UNIT, bool AGG>
 __global__ void __launch_bounds__(1024) sweep_cta(const int32_t* __restrict__ verts, const int64_t* __restrict__ soff,
                                                   int64_t nv, const uint2* __restrict__ stage, SweepArgs A,
@@ -509,6 +592,136 @@ __global__ void __launch_bounds__(1024) sweep_cta(const int32_t* __restrict__ ve
   }
 }
 
+
+// ------------------------------------------------------------ CTA per vertex, pipelined (LV_CTA_PIPE=1)
+// Persistent CTAs, one vertex at a time, software-pipelined so the per-vertex
+// chain of dependent global loads is off the critical path: while the CTA
+// hashes vertex j, lanes of warp 0 already load the bin entry of vertex j+2 and
+// the row bounds / record / degree of vertex j+1 (results parked in registers and
+// stored to shared memory at the end of the iteration), and a_own / size_own of
+// vertex j for its decision.  Moves go to a shared buffer flushed with one
+// atomic per kLogBuf moves.
+constexpr int kLogBuf = 128;
+
+__device__ __forceinline__ void flush_moves(int32_t* buf_v, int32_t* buf_t, int n, const SweepArgs& A) {
+  // warp 0, all lanes
+  const int lane = threadIdx.x & 31;
+  unsigned long long base = 0;
+  if (lane == 0 && n) base = atomicAdd(A.logn, (unsigned long long)n);
+  base = __shfl_sync(kFull, base, 0);
+  for (int i = lane; i < n; i += 32) {
+    A.mv_v[base + i] = buf_v[i];
+    A.mv_new[base + i] = buf_t[i];
+  }
+}
+
+template <bool UNIT, bool AGG>
+__global__ void __launch_bounds__(1024) sweep_cta_pipe(const int32_t* __restrict__ verts, const int64_t* __restrict__ soff,
+                                                  int64_t nv, const uint2* __restrict__ stage, SweepArgs A,
+                                                  int capmax) {
+  extern __shared__ unsigned long long smem[];
+  unsigned long long* T = smem;
+  uint32_t* TA = reinterpret_cast<uint32_t*>(smem + capmax);
+  __shared__ long long sh_s[32];
+  __shared__ int sh_c[32];
+  __shared__ unsigned sh_e[32];
+  // header of the current vertex (j) and the bin entry of the next one (j+1)
+  __shared__ int64_t h_rb, h_deg, h_so;
+  __shared__ int32_t h_v, h_own, h_vnext;
+  __shared__ uint32_t h_ki;
+  __shared__ int32_t buf_v[kLogBuf], buf_t[kLogBuf];
+  __shared__ int nbuf;
+  const int lane = threadIdx.x & 31;
+  const int64_t G = gridDim.x;
+  for (int t = threadIdx.x; t < capmax; t += blockDim.x) {
+    T[t] = kEmpty;
+    TA[t] = kUnknownA;
+  }
+  if (threadIdx.x == 0) {  // prologue: header of vertex 0, bin entry of vertex 1
+    nbuf = 0;
+    const int64_t vi = blockIdx.x;
+    if (vi < nv) {
+      const int32_t v = verts[vi];
+      h_v = v;
+      h_rb = A.rowptr[v];
+      h_deg = A.rowptr[v + 1] - h_rb;
+      h_so = soff[vi];
+      h_own = (int32_t)A.ca[v].x;
+      h_ki = A.k[v];
+    }
+    h_vnext = (vi + G < nv) ? verts[vi + G] : -1;
+  }
+  __syncthreads();
+  for (int64_t vi = blockIdx.x; vi < nv; vi += G) {
+    const int32_t v = h_v, own = h_own, vn = h_vnext;
+    const int64_t rb = h_rb, deg = h_deg, so = h_so;
+    const uint32_t ki = h_ki;
+    // warp 0 issues the loads of the next vertices now and consumes them at the end
+    int64_t pf = 0;
+    if (threadIdx.x < 32) {
+      if (lane == 0 && vi + 2 * G < nv) pf = verts[vi + 2 * G];
+      if (vn >= 0) {
+        if (lane == 1) pf = A.rowptr[vn];
+        if (lane == 2) pf = A.rowptr[vn + 1];
+        if (lane == 3) pf = soff[vi + G];
+        if (lane == 4) pf = (int64_t)A.ca[vn].x;
+        if (lane == 5) pf = (int64_t)A.k[vn];
+      }
+      if (lane == 6) pf = (int64_t)A.ca[own].y;
+      if (lane == 7) pf = (int64_t)A.size[own];
+    }
+    const uint32_t cap = (uint32_t)((2 * deg < (int64_t)capmax) ? 2 * deg : (int64_t)capmax);
+    insert_staged<UNIT, AGG>(T, TA, cap, stage + so, UNIT ? nullptr : A.w + rb, deg, threadIdx.x, blockDim.x);
+    __syncthreads();
+    const bool own_single = A.rule == 2 && __ldg(&A.size[own]) == 1;
+    long long s = (long long)0x8000000000000000ull;
+    int cb = 0x7FFFFFFF;
+    unsigned eown = 0;
+    scan_table(T, TA, cap, threadIdx.x, blockDim.x, own, own_single, ki, A, s, cb, eown);
+    block_reduce(s, cb, eown, sh_s, sh_c, sh_e);
+    if (threadIdx.x < 32) {
+      const uint32_t a_own = (uint32_t)__shfl_sync(kFull, pf, 6);
+      const int32_t size_own = (int32_t)__shfl_sync(kFull, pf, 7);
+      if (threadIdx.x == 0 && cb != 0x7FFFFFFF) {
+        int32_t tgt = own;
+        const long long sstay = A.W * (long long)eown - (long long)ki * ((long long)a_own - (long long)ki);
+        if (s > sstay) {
+          tgt = cb;
+          if (A.rule == 1 && cb > own && size_own == 1 && __ldg(&A.size[cb]) == 1) tgt = own;  // R8 veto
+        }
+        if (tgt != own) {
+          buf_v[nbuf] = v;
+          buf_t[nbuf] = tgt;
+          ++nbuf;
+        }
+      }
+      __syncwarp();
+      if (nbuf == kLogBuf) {
+        flush_moves(buf_v, buf_t, kLogBuf, A);
+        __syncwarp();
+        if (lane == 0) nbuf = 0;
+      }
+      // park the prefetched header of vertex j+1 and the bin entry of vertex j+2
+      if (lane == 0) h_vnext = (vi + 2 * G < nv) ? (int32_t)pf : -1;
+      if (vn >= 0) {
+        if (lane == 0) h_v = vn;
+        if (lane == 1) h_rb = pf;
+        if (lane == 2) h_deg = pf;  // rowptr[v+1]; minus rb below
+        if (lane == 3) h_so = pf;
+        if (lane == 4) h_own = (int32_t)pf;
+        if (lane == 5) h_ki = (uint32_t)pf;
+      }
+      __syncwarp();
+      if (lane == 0 && vn >= 0) h_deg -= h_rb;
+    }
+    __syncthreads();
+  }
+  if (threadIdx.x < 32) {
+    __syncwarp();
+    const int n = nbuf;
+    flush_moves(buf_v, buf_t, n, A);
+  }
+}
 
 // ------------------------------------------------------------ batched vertices
 // Table-based vertices of degree <= kBatchMaxDeg (33..1023 with the paper's
@@ -653,26 +866,201 @@ __global__ void k_batch_flags(const int64_t* __restrict__ soff, int64_t p0, int6
 }
 
 // ------------------------------------------------------------ label-partitioned CTAs
-// deg >= 12288: vertex v gets P = ceil(deg / kPartLabels) independent CTA tasks.
-// Task p streams all of v's staged labels (an L2-resident segment, read P
-// times) and keeps only the labels c with part_of(c, P) == p in its own
-// shared-memory table, so a partition sees ~deg/P distinct labels whatever the
-// degree; the CTA that finishes v's last task reduces the P partials and
-// decides.  No clusters, grid syncs or global hash tables.  A table that would
-// pass 7/8 load sets DevCtl::overflow and the library reports an error (the
-// expected load is <= 3/8; exceeding 7/8 needs a +60-sigma hash deviation).
-__device__ __forceinline__ uint32_t part_of(int32_t c, uint32_t P) {
-  uint32_t h = (uint32_t)c;  // fmix32 (independent of hash_slot's multiplier)
-  h ^= h >> 16;
-  h *= 0x85ebca6bu;
-  h ^= h >> 13;
-  h *= 0xc2b2ae35u;
-  h ^= h >> 16;
-  return (uint32_t)(((unsigned long long)h * P) >> 32);
+// deg >= 12288: vertex v gets P = ceil(deg / kPartLabels) independent CTA tasks;
+// task p owns the labels c with part_of(c, P) == p, so a partition sees
+// ~deg/P distinct labels whatever the degree.  The staged entries are first
+// scattered into partition order (k_part_hist / k_part_scan / k_part_scatter),
+// so each task reads only its own share; the CTA that finishes v's last task
+// reduces the P partials and decides.  No clusters, grid syncs or global hash
+// tables.  A table that would pass 7/8 load sets DevCtl::overflow and the
+// library reports an error (the expected load is <= 3/8).
+
+// Pre-partitioning of the staged entries of the plan's vertices (every sweep,
+// after k_stage): histogram of partition sizes per chunk -> per-vertex scan into
+// poff / cursors -> scatter into S2 (and the weights into W2) in partition order.
+// Labels of a warp are merged per partition with __match_any_sync so a hot
+// partition costs one shared atomic per warp.
+__global__ void __launch_bounds__(1024) k_part_hist(const PartChunk* __restrict__ chunks, int64_t c0, int64_t c1,
+                                                    const int32_t* __restrict__ vert_pos,
+                                                    const int32_t* __restrict__ vert_P,
+                                                    const int64_t* __restrict__ vert_pbase,
+                                                    const int64_t* __restrict__ soff, const uint2* __restrict__ stage,
+                                                    int64_t* poff) {
+  __shared__ uint32_t hist[kPartMaxP];
+  for (int64_t ci = c0 + blockIdx.x; ci < c1; ci += gridDim.x) {
+    const PartChunk ch = chunks[ci];
+    const uint32_t P = (uint32_t)vert_P[ch.vi];
+    const uint2* S = stage + soff[vert_pos[ch.vi]];
+    for (uint32_t q = threadIdx.x; q < P; q += blockDim.x) hist[q] = 0;
+    __syncthreads();
+    const int lane = threadIdx.x & 31;
+    for (int64_t t0 = ch.begin + (threadIdx.x - lane); t0 < ch.end; t0 += blockDim.x) {  // warp-uniform trips
+      const int64_t t = t0 + lane;
+      const uint32_t lab = (t < ch.end) ? __ldcs(&S[t]).x : kSelf;
+      const uint32_t q = (lab != kSelf) ? part_of((int32_t)lab, P) : 0xFFFFFFFFu;
+      const unsigned m = __match_any_sync(kFull, q);
+      if (q != 0xFFFFFFFFu && lane == __ffs(m) - 1) atomicAdd(&hist[q], (uint32_t)__popc(m));
+    }
+    __syncthreads();
+    int64_t* cnt = poff + vert_pbase[ch.vi] + 1;
+    for (uint32_t q = threadIdx.x; q < P; q += blockDim.x)
+      if (hist[q]) atomicAdd(reinterpret_cast<unsigned long long*>(&cnt[q]), (unsigned long long)hist[q]);
+    __syncthreads();
+  }
+}
+
+// One warp per plan vertex: poff[pb + q] = segment start + sum of earlier counts,
+// cursors of the scatter initialised to the partition starts.
+__global__ void k_part_scan(int64_t v0, int64_t v1, const int32_t* __restrict__ vert_pos,
+                            const int32_t* __restrict__ vert_P, const int64_t* __restrict__ vert_pbase,
+                            const int32_t* __restrict__ vert_first, const int64_t* __restrict__ soff, int64_t* poff,
+                            unsigned long long* pcur) {
+  const int lane = threadIdx.x & 31;
+  const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
+  for (int64_t vi = v0 + (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); vi < v1; vi += warps) {
+    const int32_t P = vert_P[vi];
+    const int64_t pb = vert_pbase[vi];
+    const int64_t f = vert_first[vi];
+    long long run = soff[vert_pos[vi]];
+    for (int32_t q0 = 0; q0 < P; q0 += 32) {
+      const int32_t q = q0 + lane;
+      const long long c = (q < P) ? poff[pb + 1 + q] : 0;
+      long long x = c;  // inclusive warp scan
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const long long y = __shfl_up_sync(kFull, x, o);
+        if (lane >= o) x += y;
+      }
+      if (q < P) {
+        const long long start = run + x - c;
+        poff[pb + q] = start;
+        pcur[f + q] = (unsigned long long)start;
+      }
+      run += __shfl_sync(kFull, x, 31);
+    }
+    if (lane == 0) poff[pb + P] = run;
+  }
 }
 
 template <bool UNIT>
-__global__ void __launch_bounds__(1024) sweep_part(const int32_t* __restrict__ task_vpos,
+__global__ void __launch_bounds__(1024) k_part_scatter(const PartChunk* __restrict__ chunks, int64_t c0, int64_t c1,
+                                                       const int32_t* __restrict__ vert_pos,
+                                                       const int32_t* __restrict__ vert_P,
+                                                       const int32_t* __restrict__ vert_first,
+                                                       const int32_t* __restrict__ bv,
+                                                       const int64_t* __restrict__ soff,
+                                                       const uint2* __restrict__ stage, unsigned long long* pcur,
+                                                       uint2* S2, uint32_t* W2, SweepArgs A) {
+  __shared__ uint32_t hist[kPartMaxP];
+  constexpr uint32_t kSeg = 1024;  // partitions reserved per round (the chunk is re-read when P > kSeg)
+  __shared__ unsigned long long base[kSeg];
+  for (int64_t ci = c0 + blockIdx.x; ci < c1; ci += gridDim.x) {
+    const PartChunk ch = chunks[ci];
+    const uint32_t P = (uint32_t)vert_P[ch.vi];
+    const int32_t pos = vert_pos[ch.vi];
+    const uint2* S = stage + soff[pos];
+    const uint32_t* Wt = UNIT ? nullptr : A.w + A.rowptr[bv[pos]];
+    unsigned long long* cur = pcur + vert_first[ch.vi];
+    const int lane = threadIdx.x & 31;
+    // the chunk's partition sizes
+    for (uint32_t q = threadIdx.x; q < P; q += blockDim.x) hist[q] = 0;
+    __syncthreads();
+    for (int64_t t0 = ch.begin + (threadIdx.x - lane); t0 < ch.end; t0 += blockDim.x) {
+      const int64_t t = t0 + lane;
+      const uint32_t lab = (t < ch.end) ? __ldcs(&S[t]).x : kSelf;
+      const uint32_t q = (lab != kSelf) ? part_of((int32_t)lab, P) : 0xFFFFFFFFu;
+      const unsigned m = __match_any_sync(kFull, q);
+      if (q != 0xFFFFFFFFu && lane == __ffs(m) - 1) atomicAdd(&hist[q], (uint32_t)__popc(m));
+    }
+    __syncthreads();
+    // reserve the chunk's ranges, then scatter with local cursors (P in rounds of kSeg)
+    for (uint32_t h0 = 0; h0 < P; h0 += kSeg) {
+      const uint32_t h1 = min(P, h0 + kSeg);
+      for (uint32_t q = h0 + threadIdx.x; q < h1; q += blockDim.x)
+        base[q - h0] = hist[q] ? atomicAdd(&cur[q], (unsigned long long)hist[q]) : 0ull;
+      __syncthreads();
+      for (int64_t t0 = ch.begin + (threadIdx.x - lane); t0 < ch.end; t0 += blockDim.x) {
+        const int64_t t = t0 + lane;
+        const uint2 rec = (t < ch.end) ? __ldcs(&S[t]) : make_uint2(kSelf, 0u);
+        uint32_t q = (rec.x != kSelf) ? part_of((int32_t)rec.x, P) : 0xFFFFFFFFu;
+        if (q < h0 || q >= h1) q = 0xFFFFFFFFu;
+        const unsigned m = __match_any_sync(kFull, q);
+        unsigned long long b = 0;
+        const int leader = __ffs(m) - 1;
+        if (q != 0xFFFFFFFFu && lane == leader) b = atomicAdd(&base[q - h0], (unsigned long long)__popc(m));
+        b = __shfl_sync(m, b, leader);
+        if (q != 0xFFFFFFFFu) {
+          const unsigned long long dst = b + __popc(m & lanemask_lt());
+          __stcs(&S2[dst], rec);
+          if (!UNIT) __stcs(&W2[dst], __ldcs(&Wt[t]));
+        }
+      }
+      __syncthreads();
+    }
+  }
+}
+
+// Shared-memory insert of one partition's entries (warp-uniform trips; equal
+// labels of a warp merged first with __match_any_sync, so the hot labels of later
+// sweeps cost one shared atomic per warp).  Returns, in every lane, how many new
+// slots this thread's warp claimed (only counted when `count`).
+template <bool UNIT, bool AGG>
+__device__ __forceinline__ unsigned part_insert(unsigned long long* T, uint32_t* TA, uint32_t cap,
+                                                const uint2* __restrict__ S, const uint32_t* __restrict__ Wt,
+                                                int64_t q0, int64_t q1, bool count) {
+  const int lane = threadIdx.x & 31;
+  unsigned claims = 0;
+  for (int64_t base = q0 + (threadIdx.x - lane); base < q1; base += 4 * (int64_t)blockDim.x) {
+    uint2 rr[4];
+    uint32_t ww[4];
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      const int64_t t = base + lane + (int64_t)u * blockDim.x;
+      rr[u] = (t < q1) ? __ldcs(&S[t]) : make_uint2(kSelf, 0u);
+      ww[u] = (t < q1) ? (UNIT ? 1u : __ldcs(&Wt[t])) : 0u;
+    }
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      unsigned m = 1u << lane, rep = (rr[u].y != kUnknownA) ? m : 0u;
+      uint32_t x = ww[u], a_rep = rr[u].y;
+      const uint32_t key_u = (rr[u].x != kSelf) ? rr[u].x : (0x80000000u | (unsigned)lane);
+      if (AGG || __any_sync(kFull, key_u == __shfl_xor_sync(kFull, key_u, 1))) {  // adaptive merge
+        m = __match_any_sync(kFull, rr[u].x);
+        x = __reduce_add_sync(m, ww[u]);
+        rep = __ballot_sync(kFull, rr[u].y != kUnknownA) & m;
+        a_rep = __shfl_sync(kFull, rr[u].y, rep ? __ffs(rep) - 1 : lane);
+      }
+      bool claimed = false;
+      if (rr[u].x != kSelf && lane == __ffs(m) - 1) {
+        const int32_t c = (int32_t)rr[u].x;
+        const unsigned long long key = ((unsigned long long)(uint32_t)c) << 32;
+        uint32_t hq = hash_slot(c, cap);
+        for (uint32_t probes = 0;; ++probes) {
+          const unsigned long long old = atomicCAS(&T[hq], kEmpty, key | x);
+          if (old == kEmpty) { claimed = true; break; }
+          if ((old >> 32) == (unsigned long long)(uint32_t)c) {
+            atomicAdd(&T[hq], (unsigned long long)x);
+            break;
+          }
+          hq = (hq + 1 == cap) ? 0 : hq + 1;
+          if (probes >= cap) { hq = 0xFFFFFFFFu; break; }  // full table (only possible when counting)
+        }
+        if (rep && hq != 0xFFFFFFFFu) TA[hq] = a_rep;
+      }
+      if (count) claims += __popc(__ballot_sync(kFull, claimed));
+    }
+  }
+  return claims;
+}
+
+// Streaming variant for vertices with P <= kStreamMaxP (the default for them):
+// task p streams all of v's staged labels (an L2-resident segment, read P times)
+// and keeps only the labels with part_of(c, P) == p; each warp compacts its
+// matching entries into a shared queue (ballot + popc) and inserts 32 at a time.
+// Measured faster than pre-partitioning at C5 level 0 (15 vs 24 ms), slower for
+// the giant hubs of the contracted levels, which take the pre-partitioned tasks.
+template <bool UNIT>
+__global__ void __launch_bounds__(1024) sweep_part_stream(const int32_t* __restrict__ task_vpos,
                                                   const int32_t* __restrict__ task_p, int64_t t_begin, int64_t t_end,
                                                   const int32_t* __restrict__ vert_pos,
                                                   const int32_t* __restrict__ vert_P,
@@ -735,6 +1123,20 @@ __global__ void __launch_bounds__(1024) sweep_part(const int32_t* __restrict__ t
       }
       if (e.y != kUnknownA) TA[h] = e.y;
     };
+    // a full warp inserts its 32 queued entries (lanes >= n idle); equal labels are
+    // merged first when adjacent lanes share one (hot labels of later sweeps)
+    auto insert_warp = [&](uint2 e, uint32_t x, bool valid) {
+      const uint32_t key = valid ? e.x : (0x80000000u | (unsigned)lane);
+      if (__any_sync(kFull, key == __shfl_xor_sync(kFull, key, 1))) {
+        const unsigned m = __match_any_sync(kFull, key);
+        const uint32_t sx = __reduce_add_sync(m, x);
+        const unsigned rep = __ballot_sync(kFull, valid && e.y != kUnknownA) & m;
+        const uint32_t a_rep = __shfl_sync(kFull, e.y, rep ? __ffs(rep) - 1 : lane);
+        if (valid && lane == __ffs(m) - 1) insert_one(make_uint2(e.x, rep ? a_rep : kUnknownA), sx);
+      } else if (valid) {
+        insert_one(e, x);
+      }
+    };
     for (int64_t base = 0; base + (int64_t)(threadIdx.x - lane) < deg; base += 4 * (int64_t)blockDim.x) {
       uint2 rr[4];
       uint32_t ww[4];
@@ -756,7 +1158,7 @@ __global__ void __launch_bounds__(1024) sweep_part(const int32_t* __restrict__ t
         qn += __popc(m);
         if (qn >= 32) {
           __syncwarp();
-          insert_one(Q[lane], QW[lane]);
+          insert_warp(Q[lane], QW[lane], true);
           const uint2 mv = (lane < qn - 32) ? Q[32 + lane] : make_uint2(0, 0);
           const uint32_t mw = (lane < qn - 32) ? QW[32 + lane] : 0u;
           __syncwarp();
@@ -770,7 +1172,7 @@ __global__ void __launch_bounds__(1024) sweep_part(const int32_t* __restrict__ t
       }
     }
     __syncwarp();
-    if (lane < qn) insert_one(Q[lane], QW[lane]);
+    insert_warp(lane < qn ? Q[lane] : make_uint2(0u, kUnknownA), lane < qn ? QW[lane] : 0u, lane < qn);
     __syncthreads();
     const int32_t own = (int32_t)__ldg(&A.ca[v]).x;
     const uint32_t ki = __ldg(&A.k[v]);
@@ -810,125 +1212,92 @@ __global__ void __launch_bounds__(1024) sweep_part(const int32_t* __restrict__ t
   }
 }
 
-// ------------------------------------------------------------ cluster per vertex
-// deg in [12288, 131072): the vertex's table (2*deg slots, load <= 1/2) is
-// spread over the distributed shared memory of a CS-CTA cluster (slot g lives
-// in CTA g % CS at index g / CS, so every CTA holds an equal share).  Each CTA inserts its share of the row into whichever CTA owns the
-// slot (remote DSMEM CAS, ~200 cycles); cluster.sync(); each CTA scans its own
-// slots; partials meet in rank 0's shared memory; cluster.sync(); rank 0 decides.
-// Persistent: clusters stride over the class's vertices.
-__device__ __forceinline__ void dsm_insert4(cg::cluster_group& cl, unsigned CS, unsigned long long* T, uint32_t* TA,
-                                            uint32_t cap, const int32_t c[4], const uint32_t x[4], bool todo[4],
-                                            const uint32_t arep[4]) {
-  uint32_t h[4];
-#pragma unroll
-  for (int q = 0; q < 4; ++q) h[q] = todo[q] ? hash_slot(c[q], cap) : 0u;
-  while (todo[0] || todo[1] || todo[2] || todo[3]) {
-    unsigned long long old[4];
-    unsigned long long* slot[4];
-#pragma unroll
-    for (int q = 0; q < 4; ++q) {
-      slot[q] = cl.map_shared_rank(T + (h[q] / CS), h[q] % CS);  // slots interleaved over the CTAs
-      old[q] = todo[q] ? atomicCAS(slot[q], kEmpty, (((unsigned long long)(uint32_t)c[q]) << 32) | x[q]) : 0ull;
-    }
-#pragma unroll
-    for (int q = 0; q < 4; ++q) {
-      if (!todo[q]) continue;
-      if (old[q] == kEmpty || (old[q] >> 32) == (unsigned long long)(uint32_t)c[q]) {
-        if (old[q] != kEmpty) atomicAdd(slot[q], (unsigned long long)x[q]);
-        if (arep[q] != kUnknownA) *cl.map_shared_rank(TA + (h[q] / CS), h[q] % CS) = arep[q];
-        todo[q] = false;
-      } else {
-        h[q] = (h[q] + 1 == cap) ? 0 : h[q] + 1;
-      }
-    }
-  }
-}
 
-template <bool UNIT>
-__global__ void __launch_bounds__(1024, 1) sweep_cluster(const int32_t* __restrict__ verts,
-                                                         const int64_t* __restrict__ soff, int64_t nv,
-                                                         const uint2* __restrict__ stage, SweepArgs A) {
-  cg::cluster_group cl = cg::this_cluster();
+// Task (v, p) of the plan: inserts the partition's pre-scattered entries
+// (S2[poff[p] .. poff[p+1])) into a smem table of 2 * n_p slots (n_p = entries >=
+// distinct labels: load <= 1/2, no overflow possible) -- or kPartSlots with a
+// distinct-label count when the partition is larger (passing 7/8 load sets
+// DevCtl::overflow; expected load <= 3/8) -- scans it, and the CTA finishing v's
+// last task reduces the P partials and decides.  (Measured on C5: one CTA walking
+// all partitions of a vertex was 20% slower than independent tasks.)
+template <bool UNIT, bool AGG>
+__global__ void __launch_bounds__(1024) sweep_part(const int32_t* __restrict__ task_vpos,
+                                                  const int32_t* __restrict__ task_p, int64_t t_begin, int64_t t_end,
+                                                  const int32_t* __restrict__ vert_pos,
+                                                  const int32_t* __restrict__ vert_P,
+                                                  const int32_t* __restrict__ vert_first,
+                                                  const int64_t* __restrict__ vert_pbase,
+                                                  const int64_t* __restrict__ poff, int32_t* done, Partial* part,
+                                                  unsigned long long* overflow, const int32_t* __restrict__ bv,
+                                                  const uint2* __restrict__ S2, const uint32_t* __restrict__ W2,
+                                                  SweepArgs A) {
   extern __shared__ unsigned long long smem[];
   unsigned long long* T = smem;
-  uint32_t* TA = reinterpret_cast<uint32_t*>(smem + kClusterSlots);
+  uint32_t* TA = reinterpret_cast<uint32_t*>(smem + kPartSlots);
   __shared__ long long sh_s[32];
   __shared__ int sh_c[32];
   __shared__ unsigned sh_e[32];
-  __shared__ Partial cpart[16];
-  const unsigned CS = cl.num_blocks();
-  const unsigned rank = cl.block_rank();
-  for (int t = threadIdx.x; t < kClusterSlots; t += blockDim.x) {
+  __shared__ int is_last;
+  __shared__ unsigned claimed;
+  for (int t = threadIdx.x; t < kPartSlots; t += blockDim.x) {
     T[t] = kEmpty;
     TA[t] = kUnknownA;
   }
-  cl.sync();
-  const int64_t ncl = gridDim.x / CS, cid = blockIdx.x / CS;
-  for (int64_t vi = cid; vi < nv; vi += ncl) {
-    const int32_t v = __ldg(&verts[vi]);
-    const int64_t rb = __ldg(&A.rowptr[v]);
-    const int64_t deg = __ldg(&A.rowptr[v + 1]) - rb;
+  if (threadIdx.x == 0) claimed = 0;
+  __syncthreads();
+  const unsigned limit = (unsigned)(kPartSlots / 8 * 7);
+  for (int64_t task = t_begin + blockIdx.x; task < t_end; task += gridDim.x) {
+    const int32_t vi = task_vpos[task];
+    const int32_t p = task_p[task];
+    const int32_t pos = vert_pos[vi];
+    const uint32_t P = (uint32_t)vert_P[vi];
+    const int32_t v = __ldg(&bv[pos]);
+    const int64_t pb = vert_pbase[vi];
+    const int64_t q0 = poff[pb + p], q1 = poff[pb + p + 1];
+    const int64_t n_p = q1 - q0;
+    const bool big = 2 * n_p > kPartSlots;
+    const uint32_t cap = big ? (uint32_t)kPartSlots : (uint32_t)(n_p > 0 ? 2 * n_p : 1);
+    const unsigned cl = part_insert<UNIT, AGG>(T, TA, cap, S2, UNIT ? nullptr : W2, q0, q1, big);
+    if (big && (threadIdx.x & 31) == 0 && cl) atomicAdd(&claimed, cl);
+    __syncthreads();
+    if (big && threadIdx.x == 0) {
+      if (claimed > limit) atomicAdd(overflow, 1ull);
+      claimed = 0;
+    }
     const int32_t own = (int32_t)__ldg(&A.ca[v]).x;
     const uint32_t ki = __ldg(&A.k[v]);
-    const uint32_t cap = (uint32_t)(2 * deg);  // <= CS * kClusterSlots by class bounds
-    // this CTA's share of the row
-    const int64_t per = (deg + CS - 1) / CS;
-    const int64_t eb = rb + (int64_t)rank * per;
-    const int64_t len = max((int64_t)0, min(per, rb + deg - eb));
-    const int lane = threadIdx.x & 31;
-    const uint2* S = stage + __ldg(&soff[vi]) + (eb - rb);
-    for (int64_t base = 0; base + (int64_t)(threadIdx.x - lane) < len; base += 4 * (int64_t)blockDim.x) {
-      uint2 rr[4];
-      uint32_t ww[4];
-#pragma unroll
-      for (int q = 0; q < 4; ++q) {
-        const int64_t t = base + threadIdx.x + (int64_t)q * blockDim.x;
-        rr[q] = (t < len) ? __ldcs(&S[t]) : make_uint2(kSelf, 0u);
-        ww[q] = UNIT ? 1u : ((t < len) ? __ldcs(&A.w[eb + t]) : 0u);
-      }
-      int32_t c[4];
-      uint32_t x[4], arep[4];
-      bool todo[4];
-#pragma unroll
-      for (int q = 0; q < 4; ++q) {
-        const bool valid = rr[q].x != kSelf;
-        c[q] = valid ? (int32_t)rr[q].x : (int32_t)(0x80000000u | (unsigned)lane);
-        const unsigned m = __match_any_sync(kFull, c[q]);
-        x[q] = UNIT ? (uint32_t)__popc(m) : __reduce_add_sync(m, ww[q]);
-        const unsigned rep = __ballot_sync(kFull, valid && rr[q].y != kUnknownA) & m;
-        const uint32_t a_rep = __shfl_sync(kFull, rr[q].y, rep ? __ffs(rep) - 1 : lane);
-        todo[q] = valid && lane == __ffs(m) - 1;
-        arep[q] = rep ? a_rep : kUnknownA;
-      }
-      dsm_insert4(cl, CS, T, TA, cap, c, x, todo, arep);
-    }
-    cl.sync();
-    // scan this CTA's slots of the table (global slots g with g % CS == rank)
-    const uint32_t my_n = (cap > rank) ? (cap - rank + CS - 1) / CS : 0u;
     const bool own_single = A.rule == 2 && __ldg(&A.size[own]) == 1;
     long long s = (long long)0x8000000000000000ull;
     int cb = 0x7FFFFFFF;
     unsigned eown = 0;
-    scan_table(T, TA, my_n, threadIdx.x, blockDim.x, own, own_single, ki, A, s, cb, eown);
+    scan_table(T, TA, cap, threadIdx.x, blockDim.x, own, own_single, ki, A, s, cb, eown);  // clears the slots
     block_reduce(s, cb, eown, sh_s, sh_c, sh_e);
-    if (threadIdx.x == 0) *cl.map_shared_rank(&cpart[rank], 0) = Partial{s, cb, eown};
-    cl.sync();
-    if (rank == 0 && threadIdx.x < 32) {
+    if (threadIdx.x == 0) {
+      part[task] = Partial{s, cb, eown};
+      __threadfence();
+      is_last = (atomicAdd(&done[vi], 1) == (int)P - 1);
+    }
+    __syncthreads();
+    if (is_last && threadIdx.x < 32) {
+      __threadfence();
       s = (long long)0x8000000000000000ull;
       cb = 0x7FFFFFFF;
       eown = 0;
-      if (threadIdx.x < CS) {
-        const Partial p = cpart[threadIdx.x];
-        s = p.s;
-        cb = p.c;
-        eown = p.eown;
+      const int32_t f = vert_first[vi];
+      for (uint32_t q = threadIdx.x; q < P; q += 32) {
+        const longlong2 raw = __ldcg(reinterpret_cast<const longlong2*>(&part[f + q]));
+        const long long ps = raw.x;
+        const int pc = (int)(raw.y & 0xFFFFFFFFll);
+        const unsigned pe = (unsigned)((unsigned long long)raw.y >> 32);
+        if (better(ps, pc, s, cb)) { s = ps; cb = pc; }
+        eown += pe;
       }
       group_reduce<32>(s, cb, eown);
       int32_t tgt = own;
       if (threadIdx.x == 0) tgt = finish(s, cb, eown, own, __ldg(&A.ca[own]).y, ki, A);
       log_moves(threadIdx.x == 0 && tgt != own, v, tgt, A);
     }
+    __syncthreads();
   }
 }
 
@@ -1041,6 +1410,133 @@ int32_t set_smem(K kernel, size_t bytes) {
   return LOUVAIN_OK;
 }
 
+template <bool UNIT>
+int32_t launch_hub(Handle& h, Level& L, const SweepArgs& A, const uint2* stage, int bucket) {
+  HubPlan& P = L.hub;
+  const int64_t w0 = P.bucket_wave[bucket - 1], w1 = P.bucket_wave[bucket];
+  if (w1 <= w0) return LOUVAIN_OK;
+  if (!P.grid) {
+    int per_sm = 0, nsm = 0;
+    LV_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, hub_coop<UNIT>, 512, 0));
+    LV_CUDA(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, h.device));
+    P.grid = std::max(1, per_sm) * nsm;  // cooperative launch: every CTA co-resident
+  }
+  const HubItem* a0 = P.ins;
+  const int64_t* a1 = P.ins_off + w0;  // the bucket's waves only (wave parity is relative: the ring is clean)
+  const HubItem* a2 = P.scans;
+  const int64_t* a3 = P.scan_off + w0;
+  const int64_t* a4 = P.wave_hub + w0;
+  const HubInfo* a5 = P.info;
+  int64_t a6 = w1 - w0, a7 = P.seg;
+  unsigned long long* a8 = P.ring;
+  uint32_t* a9 = P.ring_a;
+  Partial* a10 = (Partial*)P.partial;
+  const uint2* a11 = stage;
+  SweepArgs a12 = A;
+  void* args[] = {&a0, &a1, &a2, &a3, &a4, &a5, &a6, &a7, &a8, &a9, &a10, &a11, &a12};
+  LV_CUDA(cudaLaunchCooperativeKernel((void*)hub_coop<UNIT>, P.grid, 512, args, 0, h.stream));
+  LV_LAUNCHED();
+  return LOUVAIN_OK;
+}
+
+// The label-partitioned path of one bucket.  Plan vertices are ordered by degree
+// (descending); those with P > kStreamMaxP form a prefix and take the
+// pre-partitioned pipeline (histogram -> scan -> scatter -> tasks), the rest
+// the streaming tasks.  The partitioned stage lives in contraction-only scratch.
+template <bool UNIT, bool AGG>
+void launch_part_tasks(Handle& h, Level& L, const SweepArgs& A, int64_t t0, int64_t t1, uint2* S2, uint32_t* W2) {
+  PartPlan& Q = L.part;
+  sweep_part<UNIT, AGG><<<grid_for(t1 - t0, 1, 148), 1024, 12 * (size_t)kPartSlots, h.stream>>>(
+      Q.task_vpos, Q.task_p, t0, t1, Q.vert_pos, Q.vert_P, Q.vert_first, Q.vert_pbase, Q.poff, Q.done,
+      (Partial*)Q.partial, &h.ctl->overflow, L.bin_vertices, S2, W2, A);
+  LV_LAUNCHED();
+}
+
+int32_t launch_part(Handle& h, Level& L, const SweepArgs& A, int bucket, bool unit) {
+  PartPlan& Q = L.part;
+  const int64_t t0 = Q.bucket_task[bucket - 1], t1 = Q.bucket_task[bucket];
+  const int64_t v0 = Q.bucket_vert[bucket - 1], v1 = Q.bucket_vert[bucket];
+  const int64_t c0 = Q.bucket_chunk[bucket - 1], c1 = Q.bucket_chunk[bucket];
+  const int64_t vs = Q.bucket_vsplit[bucket - 1], ts = Q.bucket_tsplit[bucket - 1];
+  if (t1 <= t0) return LOUVAIN_OK;
+  cudaStream_t s = h.stream;
+  static bool attr = false;
+  if (!attr) {
+    LV_TRY(set_smem(sweep_part<true, false>, 12 * (size_t)kPartSlots));
+    LV_TRY(set_smem(sweep_part<false, false>, 12 * (size_t)kPartSlots));
+    LV_TRY(set_smem(sweep_part<true, true>, 12 * (size_t)kPartSlots));
+    LV_TRY(set_smem(sweep_part<false, true>, 12 * (size_t)kPartSlots));
+    LV_TRY(set_smem(sweep_part_stream<true>, 12 * (size_t)kPartSlots));
+    LV_TRY(set_smem(sweep_part_stream<false>, 12 * (size_t)kPartSlots));
+    attr = true;
+  }
+  auto mark = [&](const char* what) {
+    if (!trace_on()) return;
+    static auto last = std::chrono::steady_clock::now();
+    cudaStreamSynchronize(s);
+    const auto now = std::chrono::steady_clock::now();
+    fprintf(stderr, "[lv]          part %-8s %8.3f ms\n", what, std::chrono::duration<double, std::milli>(now - last).count());
+    last = now;
+  };
+  mark("setup");
+  LV_CUDA(cudaMemsetAsync(Q.done + v0, 0, sizeof(int32_t) * (v1 - v0), s));
+  const uint2* stage = L.stage;
+  if (ts > t0) {  // pre-partitioned prefix: vertices [v0, vs), tasks [t0, ts), chunks [c0, c1)
+    void *p2 = nullptr, *pw = nullptr;
+    LV_TRY(scratch_get(h, SC_K1, 8 * (size_t)std::max<int64_t>(L.nnz, 1), &p2));
+    if (!unit) LV_TRY(scratch_get(h, SC_V0, 4 * (size_t)std::max<int64_t>(L.nnz, 1), &pw));
+    uint2* S2 = static_cast<uint2*>(p2);
+    uint32_t* W2 = static_cast<uint32_t*>(pw);
+    int64_t pb0 = 0, pb1 = Q.npoff;
+    if (v0 > 0) LV_CUDA(cudaMemcpyAsync(&pb0, Q.vert_pbase + v0, 8, cudaMemcpyDeviceToHost, s));
+    if (vs < Q.nverts) LV_CUDA(cudaMemcpyAsync(&pb1, Q.vert_pbase + vs, 8, cudaMemcpyDeviceToHost, s));
+    LV_CUDA(cudaStreamSynchronize(s));
+    LV_CUDA(cudaMemsetAsync(Q.poff + pb0, 0, 8 * (size_t)(pb1 - pb0), s));
+    k_part_hist<<<grid_for(c1 - c0, 1, 148 * 2), 1024, 0, s>>>(Q.chunks, c0, c1, Q.vert_pos, Q.vert_P, Q.vert_pbase,
+                                                                L.soff, stage, Q.poff);
+    LV_LAUNCHED();
+    mark("hist");
+    k_part_scan<<<grid_for(vs - v0, 8, 148 * 4), 256, 0, s>>>(v0, vs, Q.vert_pos, Q.vert_P, Q.vert_pbase, Q.vert_first,
+                                                               L.soff, Q.poff, Q.pcur);
+    LV_LAUNCHED();
+    mark("scan");
+    static const char* agg_env = getenv("LV_PART_AGG");
+    const bool agg = agg_env ? agg_env[0] == '1' : !unit;  // merging pays off once labels concentrate
+    if (unit) {
+      k_part_scatter<true><<<grid_for(c1 - c0, 1, 148 * 2), 1024, 0, s>>>(Q.chunks, c0, c1, Q.vert_pos, Q.vert_P,
+                                                                          Q.vert_first, L.bin_vertices, L.soff, stage,
+                                                                          Q.pcur, S2, W2, A);
+      LV_LAUNCHED();
+      mark("scatter");
+      if (agg) launch_part_tasks<true, true>(h, L, A, t0, ts, S2, W2);
+      else launch_part_tasks<true, false>(h, L, A, t0, ts, S2, W2);
+    } else {
+      k_part_scatter<false><<<grid_for(c1 - c0, 1, 148 * 2), 1024, 0, s>>>(Q.chunks, c0, c1, Q.vert_pos, Q.vert_P,
+                                                                           Q.vert_first, L.bin_vertices, L.soff, stage,
+                                                                           Q.pcur, S2, W2, A);
+      LV_LAUNCHED();
+      mark("scatter");
+      if (agg) launch_part_tasks<false, true>(h, L, A, t0, ts, S2, W2);
+      else launch_part_tasks<false, false>(h, L, A, t0, ts, S2, W2);
+    }
+    mark("pre-tasks");
+  }
+  if (t1 > ts) {  // streaming tasks
+    if (unit)
+      sweep_part_stream<true><<<grid_for(t1 - ts, 1, 148 * 2), 1024, 12 * (size_t)kPartSlots, s>>>(
+          Q.task_vpos, Q.task_p, ts, t1, Q.vert_pos, Q.vert_P, Q.vert_first, Q.done, (Partial*)Q.partial,
+          &h.ctl->overflow, L.bin_vertices, L.soff, stage, A);
+    else
+      sweep_part_stream<false><<<grid_for(t1 - ts, 1, 148 * 2), 1024, 12 * (size_t)kPartSlots, s>>>(
+          Q.task_vpos, Q.task_p, ts, t1, Q.vert_pos, Q.vert_P, Q.vert_first, Q.done, (Partial*)Q.partial,
+          &h.ctl->overflow, L.bin_vertices, L.soff, stage, A);
+    LV_LAUNCHED();
+    mark("stream");
+  }
+  LV_CUDA(cudaGetLastError());
+  return LOUVAIN_OK;
+}
+
 bool batch_on(const Level& L, int bucket) {
   return L.batch.bstart && L.batch.off[bucket] - L.batch.off[bucket - 1] > 1;
 }
@@ -1081,57 +1577,9 @@ int32_t dispatch_class(Handle& h, Level& L, const SweepArgs& A, int bucket, int 
   } else if (sub == 0 && max_deg <= 340) {
     sweep_warp<512, 4, UNIT, AGG><<<grid_for(nv, 4, 148 * 12), 128, 0, s>>>(verts, soff, nv, stage, A);
     LV_LAUNCHED();
-  } else if ((sub == 3 || sub == 4) && !getenv("LV_NO_PART")) {
-    if (sub == 3) {  // one launch covers the bucket's sub-classes 3..4
-      PartPlan& Q = L.part;
-      const int64_t t0 = Q.bucket_task[bucket - 1], t1 = Q.bucket_task[bucket];
-      const int64_t v0 = Q.bucket_vert[bucket - 1], v1 = Q.bucket_vert[bucket];
-      if (t1 > t0) {
-        static bool attr = false;
-        if (!attr) {
-          LV_TRY(set_smem(sweep_part<true>, 12 * (size_t)kPartSlots));
-          LV_TRY(set_smem(sweep_part<false>, 12 * (size_t)kPartSlots));
-          attr = true;
-        }
-        LV_CUDA(cudaMemsetAsync(Q.done + v0, 0, sizeof(int32_t) * (v1 - v0), s));
-        sweep_part<UNIT><<<grid_for(t1 - t0, 1, 148 * 2), 1024, 12 * (size_t)kPartSlots, s>>>(
-            Q.task_vpos, Q.task_p, t0, t1, Q.vert_pos, Q.vert_P, Q.vert_first, Q.done, (Partial*)Q.partial,
-            &h.ctl->overflow, L.bin_vertices, L.soff, stage, A);
-        LV_LAUNCHED();
-      }
-    }
-  } else if (sub == 3 || sub == 4) {
-    const int CS = (sub == 3) ? 4 : 16;
-    static bool cl_attr = false;
-    if (!cl_attr) {
-      for (auto k : {sweep_cluster<true>, sweep_cluster<false>}) {
-        LV_TRY(set_smem(k, 12 * (size_t)kClusterSlots));
-        LV_CUDA(cudaFuncSetAttribute(k, cudaFuncAttributeNonPortableClusterSizeAllowed, 1));
-      }
-      cl_attr = true;
-    }
-    cudaLaunchConfig_t cfg = {};
-    cudaLaunchAttribute attr[1];
-    attr[0].id = cudaLaunchAttributeClusterDimension;
-    attr[0].val.clusterDim.x = CS;
-    attr[0].val.clusterDim.y = 1;
-    attr[0].val.clusterDim.z = 1;
-    cfg.blockDim = dim3(1024, 1, 1);
-    cfg.dynamicSmemBytes = 12 * (size_t)kClusterSlots;
-    cfg.stream = s;
-    cfg.attrs = attr;
-    cfg.numAttrs = 1;
-    static int max_clusters[2] = {0, 0};
-    int& mc = max_clusters[sub - 3];
-    if (!mc) {
-      cfg.gridDim = dim3(CS * 64, 1, 1);
-      LV_CUDA(cudaOccupancyMaxActiveClusters(&mc, (void*)sweep_cluster<UNIT>, &cfg));
-      if (mc < 1) mc = 1;
-    }
-    const int64_t ncl = std::min<int64_t>(mc, nv);
-    cfg.gridDim = dim3((unsigned)(ncl * CS), 1, 1);
-    LV_CUDA(cudaLaunchKernelEx(&cfg, sweep_cluster<UNIT>, verts, soff, nv, stage, A));
-    LV_LAUNCHED();
+  } else if (sub >= 3) {
+    if (sub == 3) LV_TRY(launch_part(h, L, A, bucket, UNIT));  // one pipeline covers sub-classes 3..5
+    if (sub == 5 && L.hub.nh > 0) LV_TRY(launch_hub<UNIT>(h, L, A, stage, bucket));  // giants (P > kPartMaxP)
   } else if (sub <= 2) {
     static const int caps[3] = {kCap0, kCap1, kCap2};
     static const int threads[3] = {256, 512, 1024};
@@ -1146,33 +1594,21 @@ int32_t dispatch_class(Handle& h, Level& L, const SweepArgs& A, int bucket, int 
       attr_done = true;
     }
     const unsigned grid = grid_for(nv, 1, 148 * per_sm[sub]);
-    sweep_cta<UNIT, AGG><<<grid, threads[sub], smem, s>>>(verts, soff, nv, stage, A, caps[sub]);
-    LV_LAUNCHED();
-  } else {
-    HubPlan& P = L.hub;
-    if (P.nh > 0) {
-      if (!P.grid) {
-        int per_sm = 0, nsm = 0;
-        LV_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, hub_coop<UNIT>, 512, 0));
-        LV_CUDA(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, h.device));
-        P.grid = std::max(1, per_sm) * nsm;  // cooperative launch: every CTA co-resident
+    static const bool pipe = getenv("LV_CTA_PIPE") && getenv("LV_CTA_PIPE")[0] == '1';
+    if (pipe) {
+      static bool pattr = false;
+      if (!pattr) {
+        LV_TRY(set_smem(sweep_cta_pipe<true, false>, 12 * (size_t)kCap2));
+        LV_TRY(set_smem(sweep_cta_pipe<false, false>, 12 * (size_t)kCap2));
+        LV_TRY(set_smem(sweep_cta_pipe<true, true>, 12 * (size_t)kCap2));
+        LV_TRY(set_smem(sweep_cta_pipe<false, true>, 12 * (size_t)kCap2));
+        pattr = true;
       }
-      const HubItem* a0 = P.ins;
-      const int64_t* a1 = P.ins_off;
-      const HubItem* a2 = P.scans;
-      const int64_t* a3 = P.scan_off;
-      const int64_t* a4 = P.wave_hub;
-      const HubInfo* a5 = P.info;
-      int64_t a6 = P.nwaves, a7 = P.seg;
-      unsigned long long* a8 = P.ring;
-      uint32_t* a9 = P.ring_a;
-      Partial* a10 = (Partial*)P.partial;
-      const uint2* a11 = stage;
-      SweepArgs a12 = A;
-      void* args[] = {&a0, &a1, &a2, &a3, &a4, &a5, &a6, &a7, &a8, &a9, &a10, &a11, &a12};
-      LV_CUDA(cudaLaunchCooperativeKernel((void*)hub_coop<UNIT>, P.grid, 512, args, 0, s));
-      LV_LAUNCHED();
+      sweep_cta_pipe<UNIT, AGG><<<grid, threads[sub], smem, s>>>(verts, soff, nv, stage, A, caps[sub]);
+    } else {
+      sweep_cta<UNIT, AGG><<<grid, threads[sub], smem, s>>>(verts, soff, nv, stage, A, caps[sub]);
     }
+    LV_LAUNCHED();
   }
   LV_CUDA(cudaGetLastError());
   return LOUVAIN_OK;
@@ -1265,10 +1701,17 @@ static void trace_step(Handle& h, Level& L, int bucket, int sub, int64_t pos0, i
 int32_t launch_stage(Handle& h, Level& L, int64_t pos0, int64_t pos1, int64_t s0, int64_t s1) {
   if (s1 <= s0) return LOUVAIN_OK;
   static const bool wb = getenv("LV_STAGE_WB") && getenv("LV_STAGE_WB")[0] == '1';
+  static const bool tiled = !(getenv("LV_STAGE_W") && getenv("LV_STAGE_W")[0] == '1');
   const int64_t* tr = nullptr;
-  LV_TRY(tile_starts(h, L.soff, pos0, pos1, s0, s1, kStageTile, &tr));
-  k_stage<<<grid_for((s1 - s0 + kStageTile - 1) / kStageTile, 1, 148 * 8), 256, 0, h.stream>>>(
-      L.bin_vertices, L.soff, pos0, pos1, tr, L.rowptr, L.col, L.ca, L.stage, !wb);
+  if (tiled || wb) {  // CTA-tiled variant (default)
+    LV_TRY(tile_starts(h, L.soff, pos0, pos1, s0, s1, kStageTile, &tr));
+    k_stage<<<grid_for((s1 - s0 + kStageTile - 1) / kStageTile, 1, 148 * 8), 256, 0, h.stream>>>(
+        L.bin_vertices, L.soff, pos0, pos1, tr, L.rowptr, L.col, L.ca, L.stage, !wb);
+  } else {
+    LV_TRY(tile_starts(h, L.soff, pos0, pos1, s0, s1, kStageChunk, &tr));
+    k_stage_w<<<grid_for((s1 - s0 + kStageChunk - 1) / kStageChunk, 8, 148 * 8), 256, 0, h.stream>>>(
+        L.bin_vertices, L.soff, pos0, pos1, s0, s1, tr, L.rowptr, L.col, L.ca, L.stage);
+  }
   LV_LAUNCHED();
   LV_CUDA(cudaGetLastError());
   return LOUVAIN_OK;

@@ -66,7 +66,7 @@ GRAPHS = {
     "lfr5k": lambda: graphgen.lfr(5000, kmin=8, kmax=300, smin=20, smax=600, seed=5),
     "weighted_loops": lambda: weighted_with_loops(3000, 6),
     "hubs": lambda: hubs_graph(),
-    # one vertex past the cluster classes (>= 131072): the cooperative global-table path
+    # a 150000-degree hub: 25 label partitions (the hub kernel with LV_PART_MAXP < 25)
     "giant_hub": lambda: hubs_graph(seed=1, hub_degrees=(150000, 20000, 3000), n=200000, bg_tuples=300000),
 }
 
@@ -297,3 +297,53 @@ def test_sharded_two_ranks_one_gpu_matches_oracle():
         assert res[1][name][0] == lab0
         assert lab0 == r.labels.tolist(), name
         assert st0["sweeps_per_level"] == r.sweeps_per_level and (st0["L"], st0["S"]) == (r.L, r.S)
+
+
+def _alt_path_worker(env_items, names, q):
+    """Runs in a fresh process so the library reads the path-selection env vars anew."""
+    import os
+    for k, v in env_items:
+        os.environ[k] = v
+    import numpy as np  # noqa: F811
+    import oracle as orc
+    import paper_conf_ipps_naimmht17_b200 as lv
+    out = {}
+    for name in names:
+        g = GRAPHS[name]()
+        r = orc.louvain(g)
+        gd = lv.Graph.from_csr(g.rowptr, g.col, g.w)
+        lab, qq, st = gd.run(lv.params())
+        out[name] = (bool(np.array_equal(lab, r.labels)), st["sweeps_per_level"] == r.sweeps_per_level,
+                     (int(qq.L), qq.S) == (r.L, r.S))
+        # one sweep from singletons, state after it
+        gd2 = lv.Graph.from_csr(g.rowptr, g.col, g.w)
+        st2 = orc.State(g)
+        moved = gd2.sweep(lv.params())[0]
+        out[name + "/sweep"] = (moved == st2.sweep(orc.params()), bool(np.array_equal(gd2.labels(), st2.C)), True)
+    q.put(out)
+
+
+@pytest.mark.parametrize("env", [
+    # every vertex with > 2 partitions (deg > 12288) on the cooperative hub kernel
+    (("LV_PART_MAXP", "2"),),
+    # contraction: canonical sort-based variant inside louvain_run
+    (("LV_CONTRACT", "sort"),),
+    # contraction: big segments through label-partitioned smem tables instead of the radix sort
+    (("LV_BIG_PART", "1"),),
+    # contraction: big segments through L2-wave global hash tables
+    (("LV_BIG_HASH", "1"),),
+    # sweep: batched table kernel for sub-class 0
+    (("LV_BATCH", "1"),),
+])
+def test_alternative_paths_match_oracle(env):
+    import torch.multiprocessing as tmp
+    ctx = tmp.get_context("spawn")
+    q = ctx.Queue()
+    names = ["hubs", "giant_hub", "weighted_loops"]
+    pr = ctx.Process(target=_alt_path_worker, args=(env, names, q))
+    pr.start()
+    out = q.get(timeout=900)
+    pr.join(timeout=60)
+    assert pr.exitcode == 0
+    for k, v in out.items():
+        assert all(v), (env, k, v)
