@@ -366,6 +366,52 @@ __global__ void __launch_bounds__(512) k_merge_mid(const int32_t* __restrict__ r
   }
 }
 
+
+// Batched 32-bit variant (default when n' < 2^31): the big segments are cut into
+// batches of at most 2^(32 - nb) segments and kBigBatchEntries entries (a larger
+// segment is a batch of its own); each batch is sorted with 32-bit keys
+// (local segment << nb | neighbour) -- 8 instead of 12 bytes per element and
+// pass, and small batches stay L2-resident -- then reduced and placed.  The run
+// count stays on the device (no host round trip per batch).
+constexpr int64_t kBigBatchEntries = 4 << 20;
+__global__ void k_big_keys32(const int32_t* __restrict__ rows, int64_t nseg, const int64_t* __restrict__ boff,
+                             int64_t base, int64_t m, const int64_t* __restrict__ sstart,
+                             const int32_t* __restrict__ gc, const uint32_t* __restrict__ gw, int nb, uint32_t* keys,
+                             uint32_t* vals) {
+  for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < m; t += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t g = base + t;
+    int64_t lo = 0, hi = nseg - 1;  // largest k with boff[k] <= g
+    while (lo < hi) {
+      const int64_t mid = (lo + hi + 1) >> 1;
+      if (boff[mid] <= g) lo = mid; else hi = mid - 1;
+    }
+    const int64_t src = sstart[rows[lo]] + (g - boff[lo]);
+    keys[t] = ((uint32_t)lo << nb) | (uint32_t)gc[src];
+    vals[t] = gw ? __ldcs(&gw[src]) : 1u;
+  }
+}
+
+__global__ void k_big_place32(const uint32_t* __restrict__ ukeys, const uint32_t* __restrict__ sums,
+                              const int64_t* __restrict__ dnum, int nb, const int32_t* __restrict__ rows,
+                              const int64_t* __restrict__ sstart, int32_t* oc, uint32_t* ow, int64_t* cnt) {
+  const int64_t nruns = *dnum;
+  const uint32_t mask = (nb >= 32) ? 0xFFFFFFFFu : ((1u << nb) - 1u);
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < nruns; i += (int64_t)gridDim.x * blockDim.x) {
+    const uint32_t k = ukeys[i] >> nb;
+    // first run of segment k: binary search back over the sorted run keys
+    int64_t lo = 0, hi = i;
+    while (lo < hi) {
+      const int64_t mid = (lo + hi) >> 1;
+      if ((ukeys[mid] >> nb) < k) lo = mid + 1; else hi = mid;
+    }
+    const int32_t r = rows[k];
+    const int64_t local = i - lo;
+    oc[sstart[r] + local] = (int32_t)(ukeys[i] & mask);
+    ow[sstart[r] + local] = sums[i];
+    if (i == nruns - 1 || (ukeys[i + 1] >> nb) != k) cnt[r] = local + 1;
+  }
+}
+
 // Step 4d: big segments.  keys = (rank of segment among big ones) << nb | neighbour,
 // edge-parallel over the concatenated big segments (boff = their prefix offsets).
 __global__ void k_big_keys(const int32_t* __restrict__ rows, int64_t nbig, const int64_t* __restrict__ sstart,
@@ -1137,7 +1183,82 @@ int32_t level_contract_fast(Handle& h, Level& L, Level& out, int32_t* d_map, int
     LV_CUDA(cudaStreamSynchronize(s));  // host vectors die here
     big_done = true;
   }
-  if (nbig > 0 && !big_done) {  // radix sort of (segment rank, neighbour) keys + reduce-by-key
+  static const bool big_sort64 = getenv("LV_BIG_SORT64") && getenv("LV_BIG_SORT64")[0] == '1';
+  if (nbig > 0 && !big_done && !big_sort64 && nb < 32) {  // batched 32-bit sorts
+    const int32_t* brows = rows + nsmall + nwarp + nmid;
+    std::vector<int32_t> hb(nbig);
+    LV_CUDA(cudaMemcpyAsync(hb.data(), brows, 4 * nbig, cudaMemcpyDeviceToHost, s));
+    std::vector<int64_t> hs(np + 1);
+    LV_CUDA(cudaMemcpyAsync(hs.data(), sstart, 8 * (np + 1), cudaMemcpyDeviceToHost, s));
+    LV_CUDA(cudaStreamSynchronize(s));
+    std::vector<int64_t> boff(nbig + 1, 0);
+    for (int64_t k = 0; k < nbig; ++k) boff[k + 1] = boff[k] + (hs[hb[k] + 1] - hs[hb[k]]);
+    const int64_t maxseg = (int64_t)1 << (32 - nb);
+    std::vector<int64_t> cuts{0};  // batch boundaries in segment index
+    int64_t mmax = 0;
+    for (int64_t k = 0; k < nbig; ++k) {
+      const int64_t k0 = cuts.back();
+      if (k > k0 && (k - k0 >= maxseg || boff[k + 1] - boff[k0] > kBigBatchEntries)) {
+        mmax = std::max(mmax, boff[k] - boff[k0]);
+        cuts.push_back(k);
+      }
+    }
+    mmax = std::max(mmax, boff[nbig] - boff[cuts.back()]);
+    cuts.push_back(nbig);
+    if (tr.on)
+      fprintf(stderr, "[lv]    contract segments: small %lld warp %lld mid %lld big %lld (big entries %lld of %lld, "
+              "%zu sort batches)\n", (long long)nsmall, (long long)nwarp, (long long)nmid, (long long)nbig,
+              (long long)boff[nbig], (long long)nnz, cuts.size() - 1);
+    int64_t* dboff = nullptr;
+    LV_TRY(dalloc(&dboff, nbig + 1, s));
+    LV_CUDA(cudaMemcpyAsync(dboff, boff.data(), 8 * (nbig + 1), cudaMemcpyHostToDevice, s));
+    uint32_t *k0b = nullptr, *k1b = nullptr, *v0b = nullptr, *v1b = nullptr;
+    {
+      void* p0 = nullptr;
+      LV_TRY(scratch_get(h, SC_STAGE, 8 * (size_t)mmax, &p0));  // the level's stage is dead during contraction
+      k0b = static_cast<uint32_t*>(p0);
+      k1b = k0b + mmax;
+      LV_TRY(scratch_get(h, SC_K1, 8 * (size_t)mmax, &p0));
+      v0b = static_cast<uint32_t*>(p0);
+      v1b = v0b + mmax;
+    }
+    int64_t* dnum = reinterpret_cast<int64_t*>(&h.ctl->bad);
+    size_t tb_sort = 0, tb_red = 0;
+    {
+      cub::DoubleBuffer<uint32_t> kq(k0b, k1b), vq(v0b, v1b);
+      LV_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, tb_sort, kq, vq, mmax, 0, 32, s));
+      LV_CUDA(cub::DeviceReduce::ReduceByKey(nullptr, tb_red, k0b, k1b, v0b, v1b, dnum, cub::Sum(), mmax, s));
+    }
+    void* tmp = nullptr;
+    LV_TRY(dmalloc(&tmp, std::max(tb_sort, tb_red), s));
+    for (size_t bi = 0; bi + 1 < cuts.size(); ++bi) {
+      const int64_t ka = cuts[bi], kz = cuts[bi + 1], nseg = kz - ka;
+      const int64_t base = boff[ka], mb = boff[kz] - base;
+      if (mb <= 0) continue;
+      int kbits = 0;
+      while (kbits < 32 && ((int64_t)1 << kbits) < nseg) ++kbits;
+      k_big_keys32<<<grid_for(mb, 256, 148 * 16), 256, 0, s>>>(brows + ka, nseg, dboff + ka, base, mb, sstart, gc, gw,
+                                                               nb, k0b, v0b);
+      LV_LAUNCHED();
+      cub::DoubleBuffer<uint32_t> kq(k0b, k1b), vq(v0b, v1b);
+      size_t tbs = tb_sort;
+      LV_CUDA(cub::DeviceRadixSort::SortPairs(tmp, tbs, kq, vq, mb, 0, nb + kbits, s));
+      LV_CUB();
+      size_t tbr = tb_red;
+      LV_CUDA(cub::DeviceReduce::ReduceByKey(tmp, tbr, kq.Current(), kq.Alternate(), vq.Current(), vq.Alternate(), dnum,
+                                             cub::Sum(), mb, s));
+      LV_CUB();
+      k_big_place32<<<grid_for(mb, 256, 148 * 16), 256, 0, s>>>(kq.Alternate(), vq.Alternate(), dnum, nb, brows + ka,
+                                                                sstart, oc, ow, cnt);
+      LV_LAUNCHED();
+    }
+    LV_CUDA(cudaGetLastError());
+    dfree(tmp, s);
+    dfree(dboff, s);
+    LV_CUDA(cudaStreamSynchronize(s));  // host vectors die here
+    big_done = true;
+  }
+  if (nbig > 0 && !big_done) {  // one radix sort of 64-bit (segment rank, neighbour) keys + reduce-by-key
     const int32_t* brows = rows + nsmall + nwarp + nmid;
     // offsets of big segments in the key array (their lengths, host-side: nbig is small)
     std::vector<int32_t> hb(nbig);
