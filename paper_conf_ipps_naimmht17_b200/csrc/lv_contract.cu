@@ -412,24 +412,8 @@ __global__ void k_big_place32(const uint32_t* __restrict__ ukeys, const uint32_t
   }
 }
 
-// Step 4d: big segments.  keys = (rank of segment among big ones) << nb | neighbour,
-// edge-parallel over the concatenated big segments (boff = their prefix offsets).
-__global__ void k_big_keys(const int32_t* __restrict__ rows, int64_t nbig, const int64_t* __restrict__ sstart,
-                           const int64_t* __restrict__ boff, const int32_t* __restrict__ gc,
-                           const uint32_t* __restrict__ gw, int nb, unsigned long long* keys, uint32_t* vals) {
-  const int64_t m = boff[nbig];
-  for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < m; t += (int64_t)gridDim.x * blockDim.x) {
-    int64_t lo = 0, hi = nbig - 1;  // largest k with boff[k] <= t
-    while (lo < hi) {
-      const int64_t mid = (lo + hi + 1) >> 1;
-      if (boff[mid] <= t) lo = mid; else hi = mid - 1;
-    }
-    const int64_t src = sstart[rows[lo]] + (t - boff[lo]);
-    keys[t] = ((unsigned long long)lo << nb) | (unsigned long long)(uint32_t)gc[src];
-    vals[t] = gw ? gw[src] : 1u;
-  }
-}
-
+// Step 4d: big segments.  keys = (rank of segment among big ones) << nb | neighbour
+// (k_big_keys_t below), one 64-bit radix sort, reduce-by-key, then placement.
 __global__ void k_big_first(const unsigned long long* __restrict__ ukeys, int64_t nruns, int nb, int64_t* first_run) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < nruns; i += (int64_t)gridDim.x * blockDim.x) {
     const int64_t k = (int64_t)(ukeys[i] >> nb);
@@ -453,6 +437,62 @@ __global__ void k_big_place(const unsigned long long* __restrict__ ukeys, const 
 }
 
 
+
+// Lengths of the big segments (the scan turns them into key-array offsets).
+__global__ void k_big_len(const int32_t* __restrict__ rows, int64_t nbig, const int64_t* __restrict__ sstart,
+                          int64_t* len) {
+  for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k <= nbig; k += (int64_t)gridDim.x * blockDim.x)
+    len[k] = (k < nbig) ? sstart[rows[k] + 1] - sstart[rows[k]] : 0;
+}
+
+// Tiled key build: tile plan btr gives the first big segment of every
+// kBigTile-entry tile; the tile's segment offsets are staged in smem.
+constexpr int kBigTile = 8192;
+constexpr int kBigTileSegs = 256;
+template <typename K>
+__global__ void __launch_bounds__(256) k_big_keys_t(const int32_t* __restrict__ rows, int64_t nbig,
+                                                    const int64_t* __restrict__ sstart,
+                                                    const int64_t* __restrict__ boff, const int64_t* __restrict__ btr,
+                                                    int64_t m, const int32_t* __restrict__ gc,
+                                                    const uint32_t* __restrict__ gw, int nb,
+                                                    K* __restrict__ keys, uint32_t* __restrict__ vals) {
+  __shared__ int64_t sh_b[kBigTileSegs + 1];
+  __shared__ int64_t sh_src[kBigTileSegs];
+  const int64_t ntiles = (m + kBigTile - 1) / kBigTile;
+  for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
+    const int64_t t0 = tile * kBigTile, t1 = min(m, t0 + kBigTile);
+    const int64_t k0 = btr[tile], k1 = btr[tile + 1];
+    const int ns = (k1 - k0 + 1 <= kBigTileSegs) ? (int)(k1 - k0 + 1) : -1;
+    __syncthreads();
+    for (int r = threadIdx.x; r < ns; r += blockDim.x) {
+      sh_b[r] = boff[k0 + r];
+      sh_src[r] = sstart[rows[k0 + r]];
+    }
+    __syncthreads();
+    for (int64_t t = t0 + threadIdx.x; t < t1; t += blockDim.x) {
+      int64_t k, src;
+      if (ns > 0) {
+        int lo = 0, hi = ns - 1;
+        while (lo < hi) {
+          const int mid = (lo + hi + 1) >> 1;
+          if (sh_b[mid] <= t) lo = mid; else hi = mid - 1;
+        }
+        k = k0 + lo;
+        src = sh_src[lo] + (t - sh_b[lo]);
+      } else {
+        int64_t lo = k0, hi = min(k1, nbig - 1);
+        while (lo < hi) {
+          const int64_t mid = (lo + hi + 1) >> 1;
+          if (boff[mid] <= t) lo = mid; else hi = mid - 1;
+        }
+        k = lo;
+        src = sstart[rows[lo]] + (t - boff[lo]);
+      }
+      keys[t] = ((K)k << nb) | (K)(uint32_t)__ldcs(&gc[src]);
+      vals[t] = gw ? __ldcs(&gw[src]) : 1u;
+    }
+  }
+}
 
 // Step 4d (LV_BIG_PART=1): big segments merged by label partitioning.  Segment k gets
 // P_k = ceil(min(len, n') / kCPartLabels) partitions (part_of(label, P_k)); its
@@ -1183,8 +1223,8 @@ int32_t level_contract_fast(Handle& h, Level& L, Level& out, int32_t* d_map, int
     LV_CUDA(cudaStreamSynchronize(s));  // host vectors die here
     big_done = true;
   }
-  static const bool big_sort64 = getenv("LV_BIG_SORT64") && getenv("LV_BIG_SORT64")[0] == '1';
-  if (nbig > 0 && !big_done && !big_sort64 && nb < 32) {  // batched 32-bit sorts
+  static const bool big_sort32 = getenv("LV_BIG_SORT32") && getenv("LV_BIG_SORT32")[0] == '1';
+  if (nbig > 0 && !big_done && big_sort32 && nb < 32) {  // batched 32-bit sorts
     const int32_t* brows = rows + nsmall + nwarp + nmid;
     std::vector<int32_t> hb(nbig);
     LV_CUDA(cudaMemcpyAsync(hb.data(), brows, 4 * nbig, cudaMemcpyDeviceToHost, s));
@@ -1260,68 +1300,120 @@ int32_t level_contract_fast(Handle& h, Level& L, Level& out, int32_t* d_map, int
   }
   if (nbig > 0 && !big_done) {  // one radix sort of 64-bit (segment rank, neighbour) keys + reduce-by-key
     const int32_t* brows = rows + nsmall + nwarp + nmid;
-    // offsets of big segments in the key array (their lengths, host-side: nbig is small)
-    std::vector<int32_t> hb(nbig);
-    LV_CUDA(cudaMemcpyAsync(hb.data(), brows, 4 * nbig, cudaMemcpyDeviceToHost, s));
-    std::vector<int64_t> hs(np + 1);
-    LV_CUDA(cudaMemcpyAsync(hs.data(), sstart, 8 * (np + 1), cudaMemcpyDeviceToHost, s));
+    // offsets of the big segments in the key array: lengths + scan on the device
+    int64_t* dboff = nullptr;
+    LV_TRY(dalloc(&dboff, nbig + 1, s));
+    k_big_len<<<grid_for(nbig + 1, 256), 256, 0, s>>>(brows, nbig, sstart, dboff);
+    LV_LAUNCHED();
+    LV_TRY(cub_scan_excl(s, dboff, dboff, nbig + 1));
+    int64_t m = 0;
+    LV_CUDA(cudaMemcpyAsync(&m, dboff + nbig, 8, cudaMemcpyDeviceToHost, s));
     LV_CUDA(cudaStreamSynchronize(s));
-    std::vector<int64_t> boff(nbig + 1, 0);
-    for (int64_t k = 0; k < nbig; ++k) boff[k + 1] = boff[k] + (hs[hb[k] + 1] - hs[hb[k]]);
-    const int64_t m = boff[nbig];
     if (tr.on)
       fprintf(stderr, "[lv]    contract segments: small %lld warp %lld mid %lld big %lld (big entries %lld of %lld)\n",
               (long long)nsmall, (long long)nwarp, (long long)nmid, (long long)nbig, (long long)m, (long long)nnz);
-    int64_t* dboff = nullptr;
-    LV_TRY(dalloc(&dboff, nbig + 1, s));
-    LV_CUDA(cudaMemcpyAsync(dboff, boff.data(), 8 * (nbig + 1), cudaMemcpyHostToDevice, s));
     int kb = 1;
     while (kb < 40 && (1ll << kb) < nbig) ++kb;
-    unsigned long long *k0 = nullptr, *k1 = nullptr;
-    uint32_t *v0 = nullptr, *v1 = nullptr;
-    {
-      void* p0 = nullptr;
-      LV_TRY(scratch_get(h, SC_STAGE, 8 * (size_t)m, &p0));  // the level's stage is dead during contraction
-      k0 = static_cast<unsigned long long*>(p0);
-      LV_TRY(scratch_get(h, SC_K1, 8 * (size_t)m, &p0));
-      k1 = static_cast<unsigned long long*>(p0);
-      LV_TRY(scratch_get(h, SC_V0, 4 * (size_t)m, &p0));
-      v0 = static_cast<uint32_t*>(p0);
-      LV_TRY(scratch_get(h, SC_V1, 4 * (size_t)m, &p0));
-      v1 = static_cast<uint32_t*>(p0);
+    if (nb + kb <= 32) {  // 32-bit keys: 8 instead of 12 bytes per element and pass
+      uint32_t *k0 = nullptr, *k1 = nullptr, *v0 = nullptr, *v1 = nullptr;
+      {
+        void* p0 = nullptr;
+        LV_TRY(scratch_get(h, SC_STAGE, 8 * (size_t)m, &p0));  // the level's stage is dead during contraction
+        k0 = static_cast<uint32_t*>(p0);
+        k1 = k0 + m;
+        LV_TRY(scratch_get(h, SC_K1, 8 * (size_t)m, &p0));
+        v0 = static_cast<uint32_t*>(p0);
+        v1 = v0 + m;
+      }
+      {
+        const int64_t* btr = nullptr;
+        LV_TRY(tile_starts(h, dboff, 0, nbig, 0, m, kBigTile, &btr));
+        k_big_keys_t<uint32_t><<<grid_for((m + kBigTile - 1) / kBigTile, 1, 148 * 8), 256, 0, s>>>(
+            brows, nbig, sstart, dboff, btr, m, gc, gw, nb, k0, v0);
+        LV_LAUNCHED();
+      }
+      tr.mark(s, "big-keys");
+      cub::DoubleBuffer<uint32_t> kq(k0, k1), vq(v0, v1);
+      size_t tb = 0;
+      LV_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, tb, kq, vq, m, 0, nb + kb, s));
+      void* tmp = nullptr;
+      LV_TRY(dmalloc(&tmp, tb, s));
+      LV_CUDA(cub::DeviceRadixSort::SortPairs(tmp, tb, kq, vq, m, 0, nb + kb, s));
+      LV_CUB();
+      dfree(tmp, s);
+      tr.mark(s, "big-sort");
+      int64_t* dnum = reinterpret_cast<int64_t*>(&h.ctl->bad);
+      tb = 0;
+      LV_CUDA(cub::DeviceReduce::ReduceByKey(nullptr, tb, kq.Current(), kq.Alternate(), vq.Current(), vq.Alternate(),
+                                             dnum, cub::Sum(), m, s));
+      LV_TRY(dmalloc(&tmp, tb, s));
+      LV_CUDA(cub::DeviceReduce::ReduceByKey(tmp, tb, kq.Current(), kq.Alternate(), vq.Current(), vq.Alternate(),
+                                             dnum, cub::Sum(), m, s));
+      LV_CUB();
+      dfree(tmp, s);
+      tr.mark(s, "big-reduce");
+      k_big_place32<<<grid_for(m, 256, 148 * 16), 256, 0, s>>>(kq.Alternate(), vq.Alternate(), dnum, nb, brows, sstart,
+                                                               oc, ow, cnt);
+      LV_LAUNCHED();
+      dfree(dboff, s);
+      LV_CUDA(cudaMemsetAsync(&h.ctl->bad, 0, 8, s));
+    } else {
+      unsigned long long *k0 = nullptr, *k1 = nullptr;
+      uint32_t *v0 = nullptr, *v1 = nullptr;
+      {
+        void* p0 = nullptr;
+        LV_TRY(scratch_get(h, SC_STAGE, 8 * (size_t)m, &p0));  // the level's stage is dead during contraction
+        k0 = static_cast<unsigned long long*>(p0);
+        LV_TRY(scratch_get(h, SC_K1, 8 * (size_t)m, &p0));
+        k1 = static_cast<unsigned long long*>(p0);
+        LV_TRY(scratch_get(h, SC_V0, 4 * (size_t)m, &p0));
+        v0 = static_cast<uint32_t*>(p0);
+        LV_TRY(scratch_get(h, SC_V1, 4 * (size_t)m, &p0));
+        v1 = static_cast<uint32_t*>(p0);
+      }
+      {
+        const int64_t* btr = nullptr;
+        LV_TRY(tile_starts(h, dboff, 0, nbig, 0, m, kBigTile, &btr));
+        k_big_keys_t<<<grid_for((m + kBigTile - 1) / kBigTile, 1, 148 * 8), 256, 0, s>>>(brows, nbig, sstart, dboff, btr,
+                                                                                        m, gc, gw, nb, k0, v0);
+        LV_LAUNCHED();
+      }
+      tr.mark(s, "big-keys");
+      cub::DoubleBuffer<unsigned long long> kbuf(k0, k1);
+      cub::DoubleBuffer<uint32_t> vbuf(v0, v1);
+      size_t tb = 0;
+      LV_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, tb, kbuf, vbuf, m, 0, nb + kb, s));
+      void* tmp = nullptr;
+      LV_TRY(dmalloc(&tmp, tb, s));
+      LV_CUDA(cub::DeviceRadixSort::SortPairs(tmp, tb, kbuf, vbuf, m, 0, nb + kb, s));
+      LV_CUB();
+      dfree(tmp, s);
+      tr.mark(s, "big-sort");
+      int64_t* dnum = reinterpret_cast<int64_t*>(&h.ctl->bad);
+      tb = 0;
+      LV_CUDA(cub::DeviceReduce::ReduceByKey(nullptr, tb, kbuf.Current(), kbuf.Alternate(), vbuf.Current(),
+                                             vbuf.Alternate(), dnum, cub::Sum(), m, s));
+      LV_TRY(dmalloc(&tmp, tb, s));
+      LV_CUDA(cub::DeviceReduce::ReduceByKey(tmp, tb, kbuf.Current(), kbuf.Alternate(), vbuf.Current(),
+                                             vbuf.Alternate(), dnum, cub::Sum(), m, s));
+      LV_CUB();
+      dfree(tmp, s);
+      int64_t nruns = 0;
+      LV_CUDA(cudaMemcpyAsync(&nruns, dnum, 8, cudaMemcpyDeviceToHost, s));
+      LV_CUDA(cudaStreamSynchronize(s));
+      tr.mark(s, "big-reduce");
+      int64_t* first_run = nullptr;
+      LV_TRY(dalloc(&first_run, nbig, s));
+      k_big_first<<<grid_for(nruns, 256), 256, 0, s>>>(kbuf.Alternate(), nruns, nb, first_run);
+      LV_LAUNCHED();
+      k_big_place<<<grid_for(nruns, 256), 256, 0, s>>>(kbuf.Alternate(), vbuf.Alternate(), nruns, nb, brows, sstart,
+                                                        first_run, oc, ow, cnt);
+      LV_LAUNCHED();
+      dfree(first_run, s);
+      dfree(dboff, s);
+      LV_CUDA(cudaMemsetAsync(&h.ctl->bad, 0, 8, s));
     }
-    k_big_keys<<<grid_for(m, 256, 148 * 16), 256, 0, s>>>(brows, nbig, sstart, dboff, gc, gw, nb, k0, v0);
-    LV_LAUNCHED();
-    cub::DoubleBuffer<unsigned long long> kbuf(k0, k1);
-    cub::DoubleBuffer<uint32_t> vbuf(v0, v1);
-    size_t tb = 0;
-    LV_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, tb, kbuf, vbuf, m, 0, nb + kb, s));
-    void* tmp = nullptr;
-    LV_TRY(dmalloc(&tmp, tb, s));
-    LV_CUDA(cub::DeviceRadixSort::SortPairs(tmp, tb, kbuf, vbuf, m, 0, nb + kb, s));
-    LV_CUB();
-    dfree(tmp, s);
-    int64_t* dnum = reinterpret_cast<int64_t*>(&h.ctl->bad);
-    tb = 0;
-    LV_CUDA(cub::DeviceReduce::ReduceByKey(nullptr, tb, kbuf.Current(), kbuf.Alternate(), vbuf.Current(),
-                                           vbuf.Alternate(), dnum, cub::Sum(), m, s));
-    LV_TRY(dmalloc(&tmp, tb, s));
-    LV_CUDA(cub::DeviceReduce::ReduceByKey(tmp, tb, kbuf.Current(), kbuf.Alternate(), vbuf.Current(),
-                                           vbuf.Alternate(), dnum, cub::Sum(), m, s));
-    LV_CUB();
-    dfree(tmp, s);
-    int64_t nruns = 0;
-    LV_CUDA(cudaMemcpyAsync(&nruns, dnum, 8, cudaMemcpyDeviceToHost, s));
-    LV_CUDA(cudaStreamSynchronize(s));
-    int64_t* first_run = nullptr;
-    LV_TRY(dalloc(&first_run, nbig, s));
-    k_big_first<<<grid_for(nruns, 256), 256, 0, s>>>(kbuf.Alternate(), nruns, nb, first_run);
-    LV_LAUNCHED();
-    k_big_place<<<grid_for(nruns, 256), 256, 0, s>>>(kbuf.Alternate(), vbuf.Alternate(), nruns, nb, brows, sstart,
-                                                      first_run, oc, ow, cnt);
-    LV_LAUNCHED();
-    dfree(first_run, s);
-    dfree(dboff, s);
+    tr.mark(s, "big-place");
   }
   if (ms != s) {
     LV_CUDA(cudaEventRecord(h.ev_join, ms));

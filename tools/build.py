@@ -73,11 +73,25 @@ def build_louvain(force: bool = False) -> str:
     nccl_flags = []
     if nccl:
         nccl_flags = ["-I", os.path.join(nccl, "include"), "-DLOUVAIN_HAVE_NCCL_HEADERS=1"]
-    if force or _stale(out, srcs + hdrs + [__file__]):
-        _run([NVCC, "-O3", "-std=c++17", *ARCH, "-lineinfo", "-shared", "-Xptxas", "-v",
-              "-Xcompiler", "-fPIC,-ffp-contract=off,-fvisibility=hidden",
-              "-I", os.path.join(ROOT, "include"), *nccl_flags,
-              "-o", out] + srcs + ["-ldl"])
+    # one object per translation unit (compiled in parallel, only when stale), then one link
+    objdir = os.path.join(ROOT, "build", "louvain")
+    os.makedirs(objdir, exist_ok=True)
+    flags = [NVCC, "-O3", "-std=c++17", *ARCH, "-lineinfo", "-Xptxas", "-v",
+             "-Xcompiler", "-fPIC,-ffp-contract=off,-fvisibility=hidden",
+             "-I", os.path.join(ROOT, "include"), *nccl_flags]
+    objs, procs = [], []
+    for src in srcs:
+        obj = os.path.join(objdir, os.path.basename(src) + ".o")
+        objs.append(obj)
+        if force or _stale(obj, [src] + hdrs + [__file__]):
+            cmd = flags + ["-c", "-o", obj, src]
+            print("+", " ".join(cmd), flush=True)
+            procs.append((src, subprocess.Popen(cmd, cwd=ROOT)))
+    for src, pr in procs:
+        if pr.wait() != 0:
+            raise subprocess.CalledProcessError(pr.returncode, f"nvcc {src}")
+    if force or procs or _stale(out, objs):
+        _run([NVCC, *ARCH, "-shared", "-o", out] + objs + ["-ldl"])
     return out
 
 
