@@ -38,22 +38,30 @@ int32_t cuda_fail(cudaError_t e, const char* what, const char* file, int line);
 // Vertices are sorted once per level by class = 8*bucket + sub, bucket in 0..7
 // (0 = degree 0, never moves; 1..7 = the paper's buckets) and sub the
 // kernel family inside the bucket, by degree:
-//   sub 0: deg < 1024   (register / warp / 256-thread CTA kernels, by bucket bound)
-//   sub 1: [1024, 4096) 512-thread CTA, smem table <= 8192 slots
-//   sub 2: [4096,12288) 1024-thread CTA, smem table <= 16384 slots
-//   sub 3..5: >= 12288      label-partitioned CTA tasks (P = ceil(deg/6144) smem tables,
-//                           the staged entries pre-partitioned); sub 5 (>= 393216) with
+//   sub 0: deg < 512    (register / warp / 128-thread CTA kernels, by bucket bound)
+//   sub 1..4: CTA per vertex, table of <= kCap[sub] slots sized to the tier's
+//             degree range so that small tiers keep more vertices in flight per SM:
+//             [512,1024) 256 thr, [1024,2048) 512, [2048,4096) 512, [4096,12288) 1024
+//   sub 5..7: >= 12288      label-partitioned CTA tasks (P = ceil(deg/6144) smem tables,
+//                           the staged entries pre-partitioned); sub 7 (>= 393216) with
 //                           P > kPartMaxP only: hub, cooperative grid, global table ring
 constexpr int kSubPerBucket = 8;
 constexpr int kNumClasses = 8 * kSubPerBucket;
-constexpr int64_t kSub1Min = 1024, kSub2Min = 4096, kSub3Min = 12288, kSub4Min = 32768, kHubMin = 393216;
-constexpr int kCap0 = 2048, kCap1 = 8192, kCap2 = 16384;  // smem table slots (12 B each)
+constexpr int kSubPart = 5, kSubHub = 7;  // first partitioned sub-class, hub sub-class
+constexpr int64_t kSub1Min = 512, kSub2Min = 1024, kSub3Min = 2048, kSub4Min = 4096, kSub5Min = 12288,
+                  kSub6Min = 32768, kHubMin = 393216;
+constexpr int kCapT[5] = {1024, 2048, 4096, 8192, 16384};  // smem table slots (12 B each) of sub 0..4
+constexpr int kThrT[5] = {128, 256, 512, 512, 1024};
+constexpr int kPerSmT[5] = {16, 8, 4, 2, 1};
+constexpr int kCapMax = 16384;
+__host__ __device__ inline int sub_of_degree(int64_t d) {
+  return d < kSub1Min ? 0 : d < kSub2Min ? 1 : d < kSub3Min ? 2 : d < kSub4Min ? 3 : d < kSub5Min ? 4
+       : d < kSub6Min ? 5 : d < kHubMin ? 6 : 7;
+}
+
 constexpr int64_t kHubChunkEdges = 2048;  // edges per hub insert item
 constexpr int64_t kHubScanSlots = 4096;   // slots per hub scan item
 constexpr int64_t kHubWaveSlots = 3 << 19;  // table slots per wave (12 B each; ring = 2 segments)
-inline int sub_of_degree(int64_t d) {
-  return d < kSub1Min ? 0 : d < kSub2Min ? 1 : d < kSub3Min ? 2 : d < kSub4Min ? 3 : d < kHubMin ? 4 : 5;
-}
 
 struct DevCtl {
   unsigned long long logn;       // move-log entries appended in this sweep
@@ -96,7 +104,7 @@ struct HubPlan {
   int64_t bucket_wave[9] = {0};        // waves of bucket b: [bucket_wave[b-1], bucket_wave[b])
 };
 
-// Label-partitioned plan for vertices of degree >= kSub3Min: vertex v gets
+// Label-partitioned plan for vertices of degree >= kSub5Min: vertex v gets
 // P_v = ceil(deg / kPartLabels) CTA tasks; task p owns the labels c with
 // part_of(c, P_v) == p.  Each sweep the vertex's staged entries are first
 // scattered into partition order (histogram -> per-vertex scan -> scatter, in

@@ -89,7 +89,7 @@ __global__ void k_classify(const int64_t* rowptr, int64_t n, int64_t b0, int64_t
     else if (d <= b4) b = 5;
     else if (d <= b5) b = 6;
     else b = 7;
-    const int sub = d < kSub1Min ? 0 : d < kSub2Min ? 1 : d < kSub3Min ? 2 : d < kSub4Min ? 3 : d < kHubMin ? 4 : 5;
+    const int sub = sub_of_degree(d);
     const uint8_t c = (uint8_t)(kSubPerBucket * b + sub);
     cls[i] = c;
     iota[i] = (int32_t)i;
@@ -483,7 +483,7 @@ int32_t level_get_a(Handle& h, Level& L, uint32_t* d_out) {
   return LOUVAIN_OK;
 }
 
-// Hub plan (vertices of sub-class 5 with more than kPartMaxP partitions, of any bucket): work items
+// Hub plan (vertices of sub-class kSubHub with more than kPartMaxP partitions, of any bucket): work items
 // in hub order -- inserts (kHubChunkEdges edges each), scans (kHubScanSlots
 // slots each), final -- and a ring of table slots reused hub after hub.
 static int32_t build_hub_plan(Handle& h, Level& L) {
@@ -493,8 +493,8 @@ static int32_t build_hub_plan(Handle& h, Level& L) {
   std::vector<int64_t> hdeg, rb, hsoff;
   std::vector<int32_t> hbucket;
   for (int b = 1; b <= 7; ++b) {
-    const int c = kSubPerBucket * b + 3;  // sub-classes 3..5 (P > part_maxp() only)
-    const int64_t off = L.class_off[c], cnt = L.class_off[c + 3] - off;
+    const int c = kSubPerBucket * b + kSubPart;  // partitioned sub-classes (P > part_maxp() only)
+    const int64_t off = L.class_off[c], cnt = L.class_off[kSubPerBucket * (b + 1)] - off;
     if (cnt <= 0) continue;
     std::vector<int32_t> v(cnt);
     std::vector<int64_t> d(2 * cnt);
@@ -591,7 +591,7 @@ static void part_free(PartPlan& Q, cudaStream_t s) {
   Q = PartPlan();
 }
 
-// Partition plan for every vertex of sub-classes 3..5 (deg >= kSub3Min) with
+// Partition plan for every vertex of sub-classes kSubPart.. (deg >= kSub5Min) with
 // P <= kPartMaxP, any bucket.
 int32_t build_part_plan(Handle& h, Level& L) {
   cudaStream_t s = h.stream;
@@ -607,7 +607,7 @@ int32_t build_part_plan(Handle& h, Level& L) {
     Q.bucket_chunk[b - 1] = (int64_t)ch.size();
     Q.bucket_vsplit[b - 1] = (int64_t)vpos.size();
     Q.bucket_tsplit[b - 1] = (int64_t)tv.size();
-    const int c0 = kSubPerBucket * b + 3, c1 = kSubPerBucket * b + 6;
+    const int c0 = kSubPerBucket * b + kSubPart, c1 = kSubPerBucket * (b + 1);
     const int64_t off = L.class_off[c0], cnt = L.class_off[c1] - off;
     if (cnt <= 0) continue;
     std::vector<int64_t> so(cnt + 1);

@@ -593,6 +593,209 @@ __global__ void __launch_bounds__(1024) sweep_cta(const int32_t* __restrict__ ve
 }
 
 
+// ------------------------------------------------------------ claimed-slot lists (default)
+// The thread whose CAS claims an empty slot appends the slot index to the
+// table's list (warp-aggregated, one shared atomic per warp and pass), so the
+// scan visits exactly the distinct labels with full warps instead of every
+// slot of the table (ncu, C5 sweep 1: the slot scan of the warp / CTA kernels
+// ran at 10-20 active lanes per instruction and was ~45% of their instructions).
+// The four inserts of a pass share one retry loop (independent CASes in flight
+// instead of four divergent probe loops).
+template <bool UNIT>
+__device__ __forceinline__ void insert_list(unsigned long long* T, uint32_t* TA, uint32_t cap,
+                                            const uint2* __restrict__ S, const uint32_t* __restrict__ Wt,
+                                            int64_t deg, int64_t t0, int64_t stride, uint16_t* Lst, int* nL) {
+  const int lane = threadIdx.x & 31;
+  const int64_t t_warp0 = t0 - lane;
+  for (int64_t base = 0; base + t_warp0 < deg; base += 4 * stride) {  // trip count uniform across the warp
+    uint2 rr[4];
+    uint32_t ww[4];
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      const int64_t t = base + t0 + q * stride;
+      rr[q] = (t < deg) ? __ldcs(&S[t]) : make_uint2(kSelf, 0u);
+      ww[q] = UNIT ? 1u : ((t < deg) ? __ldcs(&Wt[t]) : 0u);
+    }
+    uint32_t h[4];
+    bool todo[4], claimed[4];
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      todo[q] = rr[q].x != kSelf;
+      claimed[q] = false;
+      h[q] = todo[q] ? hash_slot((int32_t)rr[q].x, cap) : 0u;
+    }
+    while (todo[0] || todo[1] || todo[2] || todo[3]) {
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        if (!todo[q]) continue;
+        const unsigned long long kx = ((unsigned long long)rr[q].x << 32) | ww[q];
+        const unsigned long long old = atomicCAS(&T[h[q]], kEmpty, kx);
+        if (old == kEmpty) {
+          claimed[q] = true;
+          todo[q] = false;
+        } else if ((uint32_t)(old >> 32) == rr[q].x) {
+          atomicAdd(&T[h[q]], (unsigned long long)ww[q]);
+          todo[q] = false;
+        } else {
+          h[q] = (h[q] + 1 == cap) ? 0u : h[q] + 1;
+        }
+      }
+    }
+#pragma unroll
+    for (int q = 0; q < 4; ++q)
+      if (rr[q].x != kSelf && rr[q].y != kUnknownA) TA[h[q]] = rr[q].y;
+    unsigned m[4];
+    int tot = 0;
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      m[q] = __ballot_sync(kFull, claimed[q]);
+      tot += __popc(m[q]);
+    }
+    if (tot) {
+      int b0 = 0;
+      if (lane == 0) b0 = atomicAdd(nL, tot);
+      b0 = __shfl_sync(kFull, b0, 0);
+      const unsigned lt = lanemask_lt();
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        if (claimed[q]) Lst[b0 + __popc(m[q] & lt)] = (uint16_t)h[q];
+        b0 += __popc(m[q]);
+      }
+    }
+  }
+}
+
+// Scan of the claimed slots (entries [t0, nl) step `stride` of the list); clears
+// each visited slot for the next vertex.
+__device__ __forceinline__ void scan_list(unsigned long long* T, uint32_t* TA, const uint16_t* Lst, int nl, int t0,
+                                          int stride, int32_t own, bool own_single, uint32_t ki, const SweepArgs& A,
+                                          long long& s, int& cb, unsigned& eown) {
+  for (int base = t0; base < nl; base += 4 * stride) {
+    unsigned long long x[4];
+    uint32_t ac[4];
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      const int t = base + q * stride;
+      x[q] = kEmpty;
+      ac[q] = kUnknownA;
+      if (t < nl) {
+        const uint32_t sl = Lst[t];
+        x[q] = T[sl];
+        ac[q] = TA[sl];
+        T[sl] = kEmpty;
+        TA[sl] = kUnknownA;
+      }
+    }
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      if (x[q] != kEmpty && ac[q] == kUnknownA && (int32_t)(x[q] >> 32) != own)
+        ac[q] = __ldg(&A.ca[(int32_t)(x[q] >> 32)]).y;
+    }
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      if (x[q] == kEmpty) continue;
+      const int32_t c = (int32_t)(x[q] >> 32);
+      const uint32_t e = (uint32_t)x[q];
+      if (c == own) eown = e;
+      else consider(c, e, ac[q], own, own_single, ki, A, s, cb);
+    }
+  }
+}
+
+template <int CAP, int LCAP, int WARPS, bool UNIT>
+__global__ void __launch_bounds__(32 * WARPS) sweep_warp_l(const int32_t* __restrict__ verts,
+                                                           const int64_t* __restrict__ soff, int64_t nv,
+                                                           const uint2* __restrict__ stage, SweepArgs A) {
+  __shared__ unsigned long long tab[WARPS][CAP];
+  __shared__ uint32_t taba[WARPS][CAP];
+  __shared__ uint16_t lst[WARPS][LCAP];
+  __shared__ int nls[WARPS];
+  const int lane = threadIdx.x & 31, wl = threadIdx.x >> 5;
+  unsigned long long* T = tab[wl];
+  uint32_t* TA = taba[wl];
+  for (int t = lane; t < CAP; t += 32) {
+    T[t] = kEmpty;
+    TA[t] = kUnknownA;
+  }
+  if (lane == 0) nls[wl] = 0;
+  __syncwarp();
+  const int64_t warps = (int64_t)gridDim.x * WARPS;
+  for (int64_t vi = (int64_t)blockIdx.x * WARPS + wl; vi < nv; vi += warps) {
+    const int32_t v = __ldg(&verts[vi]);
+    const int64_t rb = __ldg(&A.rowptr[v]);
+    const int64_t deg = __ldg(&A.rowptr[v + 1]) - rb;
+    const int32_t own = (int32_t)__ldg(&A.ca[v]).x;
+    const uint32_t ki = __ldg(&A.k[v]);
+    insert_list<UNIT>(T, TA, CAP, stage + __ldg(&soff[vi]), UNIT ? nullptr : A.w + rb, deg, lane, 32, lst[wl],
+                      &nls[wl]);
+    __syncwarp();
+    const int nl = nls[wl];
+    const bool own_single = A.rule == 2 && __ldg(&A.size[own]) == 1;
+    long long s = (long long)0x8000000000000000ull;
+    int cb = 0x7FFFFFFF;
+    unsigned eown = 0;
+    scan_list(T, TA, lst[wl], nl, lane, 32, own, own_single, ki, A, s, cb, eown);
+    group_reduce<32>(s, cb, eown);
+    int32_t tgt = own;
+    if (lane == 0) {
+      tgt = finish(s, cb, eown, own, __ldg(&A.ca[own]).y, ki, A);
+      nls[wl] = 0;
+    }
+    log_moves(lane == 0 && tgt != own, v, tgt, A);
+    __syncwarp();
+  }
+}
+
+// CTA per vertex with a claimed-slot list; dynamic smem = capmax slots (12 B)
+// + lcap list entries (2 B).
+template <bool UNIT>
+__global__ void __launch_bounds__(1024) sweep_cta_l(const int32_t* __restrict__ verts,
+                                                    const int64_t* __restrict__ soff, int64_t nv,
+                                                    const uint2* __restrict__ stage, SweepArgs A, int capmax) {
+  extern __shared__ unsigned long long smem[];
+  unsigned long long* T = smem;
+  uint32_t* TA = reinterpret_cast<uint32_t*>(smem + capmax);
+  uint16_t* Lst = reinterpret_cast<uint16_t*>(TA + capmax);
+  __shared__ long long sh_s[32];
+  __shared__ int sh_c[32];
+  __shared__ unsigned sh_e[32];
+  __shared__ int sh_n;
+  for (int t = threadIdx.x; t < capmax; t += blockDim.x) {
+    T[t] = kEmpty;
+    TA[t] = kUnknownA;
+  }
+  if (threadIdx.x == 0) sh_n = 0;
+  __syncthreads();
+  for (int64_t vi = blockIdx.x; vi < nv; vi += gridDim.x) {
+    const int32_t v = __ldg(&verts[vi]);
+    const int64_t rb = __ldg(&A.rowptr[v]);
+    const int64_t deg = __ldg(&A.rowptr[v + 1]) - rb;
+    const int32_t own = (int32_t)__ldg(&A.ca[v]).x;
+    const uint32_t ki = __ldg(&A.k[v]);
+    const uint32_t cap = (uint32_t)((2 * deg < (int64_t)capmax) ? 2 * deg : (int64_t)capmax);
+    insert_list<UNIT>(T, TA, cap, stage + __ldg(&soff[vi]), UNIT ? nullptr : A.w + rb, deg, threadIdx.x, blockDim.x,
+                      Lst, &sh_n);
+    __syncthreads();
+    const int nl = sh_n;
+    const bool own_single = A.rule == 2 && __ldg(&A.size[own]) == 1;
+    long long s = (long long)0x8000000000000000ull;
+    int cb = 0x7FFFFFFF;
+    unsigned eown = 0;
+    scan_list(T, TA, Lst, nl, threadIdx.x, blockDim.x, own, own_single, ki, A, s, cb, eown);
+    block_reduce(s, cb, eown, sh_s, sh_c, sh_e);  // its barrier orders every read of sh_n before the reset
+    if (threadIdx.x < 32) {
+      int32_t tgt = own;
+      if (threadIdx.x == 0) {
+        tgt = finish(s, cb, eown, own, __ldg(&A.ca[own]).y, ki, A);
+        sh_n = 0;
+      }
+      log_moves(threadIdx.x == 0 && tgt != own, v, tgt, A);
+    }
+    __syncthreads();
+  }
+}
+
+
 // ------------------------------------------------------------ CTA per vertex, pipelined (LV_CTA_PIPE=1)
 // Persistent CTAs, one vertex at a time, software-pipelined so the per-vertex
 // chain of dependent global loads is off the critical path: while the CTA
@@ -1541,6 +1744,25 @@ bool batch_on(const Level& L, int bucket) {
   return L.batch.bstart && L.batch.off[bucket] - L.batch.off[bucket - 1] > 1;
 }
 
+// Claimed-slot lists pay where the table is much larger than the distinct count:
+// the fixed 512-slot warp tables of bucket 6 (C5 level 0: 10.2 -> 6.3 ms per 2
+// sweeps).  The CTA tables are sized 2*deg, where the list measured slower
+// (b7 [1024,2048): 12.5 -> 19.4 ms), and so was the 128-slot warp table of bucket 5.
+// LV_LIST=0 turns it off; LV_LIST_CTA=1 turns it on for the CTA tiers (A/B only).
+static bool use_list() {
+  static const bool on = !(getenv("LV_LIST") && getenv("LV_LIST")[0] == '0');
+  return on;
+}
+static bool list_cta() {
+  static const bool on = getenv("LV_LIST_CTA") && getenv("LV_LIST_CTA")[0] == '1';
+  return on;
+}
+// largest degree of CTA tier `sub` (lv_internal.cuh)
+static int64_t max_deg_of_tier(int sub) {
+  static const int64_t ub[5] = {kSub1Min - 1, kSub2Min - 1, kSub3Min - 1, kSub4Min - 1, kSub5Min - 1};
+  return ub[sub];
+}
+
 template <bool UNIT, bool AGG>
 int32_t dispatch_class(Handle& h, Level& L, const SweepArgs& A, int bucket, int sub, int64_t max_deg) {
   const int64_t off = L.class_off[kSubPerBucket * bucket + sub];
@@ -1571,37 +1793,61 @@ int32_t dispatch_class(Handle& h, Level& L, const SweepArgs& A, int bucket, int 
     sweep_batch<UNIT><<<grid_for(nb, 1, 148 * 2), 512, 12 * (size_t)kBatchSlots, s>>>(L.bin_vertices, L.soff,
                                                                                     L.batch.bstart + b0, nb, stage, A);
     LV_LAUNCHED();
+  } else if (sub == 0 && max_deg > 84 && max_deg <= 340 && use_list()) {
+    sweep_warp_l<512, 352, 4, UNIT><<<grid_for(nv, 4, 148 * 8), 128, 0, s>>>(verts, soff, nv, stage, A);
+    LV_LAUNCHED();
   } else if (sub == 0 && max_deg <= 84) {
     sweep_warp<128, 8, UNIT, AGG><<<grid_for(nv, 8, 148 * 8), 256, 0, s>>>(verts, soff, nv, stage, A);
     LV_LAUNCHED();
   } else if (sub == 0 && max_deg <= 340) {
     sweep_warp<512, 4, UNIT, AGG><<<grid_for(nv, 4, 148 * 12), 128, 0, s>>>(verts, soff, nv, stage, A);
     LV_LAUNCHED();
-  } else if (sub >= 3) {
-    if (sub == 3) LV_TRY(launch_part(h, L, A, bucket, UNIT));  // one pipeline covers sub-classes 3..5
-    if (sub == 5 && L.hub.nh > 0) LV_TRY(launch_hub<UNIT>(h, L, A, stage, bucket));  // giants (P > kPartMaxP)
-  } else if (sub <= 2) {
-    static const int caps[3] = {kCap0, kCap1, kCap2};
-    static const int threads[3] = {256, 512, 1024};
-    static const int per_sm[3] = {6, 2, 1};
+  } else if (sub >= kSubPart) {
+    if (sub == kSubPart) LV_TRY(launch_part(h, L, A, bucket, UNIT));  // one pipeline covers sub-classes kSubPart..
+    if (sub == kSubHub && L.hub.nh > 0) LV_TRY(launch_hub<UNIT>(h, L, A, stage, bucket));  // giants (P > kPartMaxP)
+  } else {
+    static const int* caps = kCapT;
+    static const int* threads = kThrT;
+    static const int* per_sm = kPerSmT;
     const size_t smem = 12 * (size_t)caps[sub];
     static bool attr_done = false;
     if (!attr_done) {
-      LV_TRY(set_smem(sweep_cta<true, false>, 12 * (size_t)kCap2));
-      LV_TRY(set_smem(sweep_cta<false, false>, 12 * (size_t)kCap2));
-      LV_TRY(set_smem(sweep_cta<true, true>, 12 * (size_t)kCap2));
-      LV_TRY(set_smem(sweep_cta<false, true>, 12 * (size_t)kCap2));
+      LV_TRY(set_smem(sweep_cta<true, false>, 12 * (size_t)kCapMax));
+      LV_TRY(set_smem(sweep_cta<false, false>, 12 * (size_t)kCapMax));
+      LV_TRY(set_smem(sweep_cta<true, true>, 12 * (size_t)kCapMax));
+      LV_TRY(set_smem(sweep_cta<false, true>, 12 * (size_t)kCapMax));
       attr_done = true;
+    }
+    if (list_cta()) {  // claimed-slot list variant (LV_LIST_CTA=1; measured slower on C5, tables are 2*deg here)
+      static int resident[5] = {0, 0, 0, 0, 0};
+      const int lcap = (int)std::min<int64_t>(caps[sub], max_deg_of_tier(sub));
+      const size_t lsmem = 12 * (size_t)caps[sub] + 2 * (size_t)((lcap + 7) & ~7);
+      static bool lattr = false;
+      if (!lattr) {
+        LV_TRY(set_smem(sweep_cta_l<true>, 12 * (size_t)kCapMax + 2 * 12288));
+        LV_TRY(set_smem(sweep_cta_l<false>, 12 * (size_t)kCapMax + 2 * 12288));
+        lattr = true;
+      }
+      if (resident[sub] == 0) {
+        int nb = 0;
+        LV_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, sweep_cta_l<UNIT>, threads[sub], lsmem));
+        resident[sub] = std::max(nb, 1);
+      }
+      const unsigned lgrid = grid_for(nv, 1, 148 * resident[sub]);
+      sweep_cta_l<UNIT><<<lgrid, threads[sub], lsmem, s>>>(verts, soff, nv, stage, A, caps[sub]);
+      LV_LAUNCHED();
+      LV_CUDA(cudaGetLastError());
+      return LOUVAIN_OK;
     }
     const unsigned grid = grid_for(nv, 1, 148 * per_sm[sub]);
     static const bool pipe = getenv("LV_CTA_PIPE") && getenv("LV_CTA_PIPE")[0] == '1';
     if (pipe) {
       static bool pattr = false;
       if (!pattr) {
-        LV_TRY(set_smem(sweep_cta_pipe<true, false>, 12 * (size_t)kCap2));
-        LV_TRY(set_smem(sweep_cta_pipe<false, false>, 12 * (size_t)kCap2));
-        LV_TRY(set_smem(sweep_cta_pipe<true, true>, 12 * (size_t)kCap2));
-        LV_TRY(set_smem(sweep_cta_pipe<false, true>, 12 * (size_t)kCap2));
+        LV_TRY(set_smem(sweep_cta_pipe<true, false>, 12 * (size_t)kCapMax));
+        LV_TRY(set_smem(sweep_cta_pipe<false, false>, 12 * (size_t)kCapMax));
+        LV_TRY(set_smem(sweep_cta_pipe<true, true>, 12 * (size_t)kCapMax));
+        LV_TRY(set_smem(sweep_cta_pipe<false, true>, 12 * (size_t)kCapMax));
         pattr = true;
       }
       sweep_cta_pipe<UNIT, AGG><<<grid, threads[sub], smem, s>>>(verts, soff, nv, stage, A, caps[sub]);
@@ -1742,7 +1988,7 @@ int32_t launch_sweep_bucket(Handle& h, Level& L, const louvain_params_t& p, int 
     if (pos1 > pos0) LV_TRY(launch_stage(h, L, pos0, pos1, L.class_soff[c0], L.class_soff[c1]));
     if (trace_on()) trace_step(h, L, bucket, -1, pos0, pos1);
   }
-  for (int sub = 0; sub < 6; ++sub) {
+  for (int sub = 0; sub < kSubPerBucket; ++sub) {
     const int64_t max_deg = (sub == 0) ? std::min<int64_t>(hi, kSub1Min - 1) : hi;
     // warp-level label merging (__match_any_sync before the table insert) is
     // off: measured slower at every level and sweep of C5 (profiles/README.md)
