@@ -136,10 +136,15 @@ struct PartPlan {
   int64_t bucket_task[9] = {0};   // tasks of bucket b: [bucket_task[b-1], bucket_task[b])
   int64_t bucket_vert[9] = {0};   // plan vertices of bucket b
   int64_t bucket_chunk[9] = {0};  // chunks of bucket b (pre-partitioned vertices only)
+  int64_t ngroups = 0;            // cluster groups of the streaming vertices (sweep_part_clu)
+  int32_t* grp_vi = nullptr;      // [ngroups] plan vertex of the group
+  int32_t* grp_p0 = nullptr;      // [ngroups] first partition of the group (multiple of kCluCS)
+  int64_t bucket_grp[9] = {0};    // groups of bucket b: [bucket_grp[b-1], bucket_grp[b])
   int64_t bucket_vsplit[8] = {0};  // bucket b's vertices [bucket_vert[b-1], vsplit) are pre-partitioned,
   int64_t bucket_tsplit[8] = {0};  // tasks [bucket_task[b-1], tsplit); the rest stream (P <= kStreamMaxP)
 };
 constexpr int64_t kStreamMaxP = 64;
+constexpr int kCluGroup = 8;  // partitions per cluster group (= sweep_part_clu's cluster size)
 
 // Batched plan for the table-based vertices of degree <= kBatchMaxDeg (sub-class 0
 // of buckets whose bound exceeds 32): consecutive bin positions are cut into

@@ -587,7 +587,7 @@ static int32_t build_hub_plan(Handle& h, Level& L) {
 static void part_free(PartPlan& Q, cudaStream_t s) {
   dfree(Q.task_vpos, s); dfree(Q.task_p, s); dfree(Q.vert_pos, s); dfree(Q.vert_P, s); dfree(Q.vert_first, s);
   dfree(Q.vert_pbase, s); dfree(Q.done, s); dfree(Q.partial, s); dfree(Q.poff, s); dfree(Q.pcur, s);
-  dfree(Q.chunks, s);
+  dfree(Q.chunks, s); dfree(Q.grp_vi, s); dfree(Q.grp_p0, s);
   Q = PartPlan();
 }
 
@@ -597,11 +597,12 @@ int32_t build_part_plan(Handle& h, Level& L) {
   cudaStream_t s = h.stream;
   PartPlan& Q = L.part;
   part_free(Q, s);
-  std::vector<int32_t> vpos, vP, vfirst, tv, tp;
+  std::vector<int32_t> vpos, vP, vfirst, tv, tp, gvi, gp0;
   std::vector<int64_t> vpb;
   std::vector<PartChunk> ch;
   int64_t pb = 0;
   for (int b = 1; b <= 7; ++b) {
+    Q.bucket_grp[b - 1] = (int64_t)gvi.size();
     Q.bucket_task[b - 1] = (int64_t)tv.size();
     Q.bucket_vert[b - 1] = (int64_t)vpos.size();
     Q.bucket_chunk[b - 1] = (int64_t)ch.size();
@@ -636,9 +637,16 @@ int32_t build_part_plan(Handle& h, Level& L) {
         for (int64_t e = 0; e < deg; e += kPartChunk) ch.push_back(PartChunk{vi, 0, e, std::min(deg, e + kPartChunk)});
         Q.bucket_vsplit[b - 1] = (int64_t)vpos.size();
         Q.bucket_tsplit[b - 1] = (int64_t)tv.size();
+      } else {  // streaming: cluster groups of kCluGroup partitions
+        for (int32_t q = 0; q < (int32_t)P; q += kCluGroup) {
+          gvi.push_back(vi);
+          gp0.push_back(q);
+        }
       }
     }
   }
+  Q.bucket_grp[7] = (int64_t)gvi.size();
+  Q.ngroups = (int64_t)gvi.size();
   Q.nverts = (int64_t)vpos.size();
   Q.ntasks = (int64_t)tv.size();
   Q.nchunks = (int64_t)ch.size();
@@ -665,6 +673,12 @@ int32_t build_part_plan(Handle& h, Level& L) {
   LV_CUDA(cudaMemcpyAsync(Q.vert_first, vfirst.data(), 4 * vfirst.size(), cudaMemcpyHostToDevice, s));
   LV_CUDA(cudaMemcpyAsync(Q.vert_pbase, vpb.data(), 8 * vpb.size(), cudaMemcpyHostToDevice, s));
   LV_CUDA(cudaMemcpyAsync(Q.chunks, ch.data(), sizeof(PartChunk) * ch.size(), cudaMemcpyHostToDevice, s));
+  if (Q.ngroups > 0) {
+    LV_TRY(dalloc(&Q.grp_vi, Q.ngroups, s));
+    LV_TRY(dalloc(&Q.grp_p0, Q.ngroups, s));
+    LV_CUDA(cudaMemcpyAsync(Q.grp_vi, gvi.data(), 4 * gvi.size(), cudaMemcpyHostToDevice, s));
+    LV_CUDA(cudaMemcpyAsync(Q.grp_p0, gp0.data(), 4 * gp0.size(), cudaMemcpyHostToDevice, s));
+  }
   LV_CUDA(cudaStreamSynchronize(s));  // host vectors die here
   return LOUVAIN_OK;
 }

@@ -1416,6 +1416,140 @@ __global__ void __launch_bounds__(1024) sweep_part_stream(const int32_t* __restr
 }
 
 
+// Cluster variant of the streaming tasks (LV_CLU=1, experiment): a cluster of kCluCS CTAs
+// takes kCluCS consecutive partitions p0 .. p0+kCluCS-1 of one vertex.  Every
+// CTA streams 1/kCluCS of the vertex's staged labels and inserts each label of
+// those partitions into the table of the CTA that owns it, through distributed
+// shared memory (one remote CAS per distinct label), so the vertex's list is read
+// ceil(P / kCluCS) times instead of P times.  After a cluster barrier each CTA
+// scans its own table exactly like sweep_part_stream and the CTA finishing v's
+// last partition reduces the partials.
+constexpr int kCluCS = 8;
+template <bool UNIT>
+__global__ void __launch_bounds__(1024, 1) sweep_part_clu(const int32_t* __restrict__ grp_vi,
+                                                          const int32_t* __restrict__ grp_p0, int64_t g_begin,
+                                                          int64_t g_end, const int32_t* __restrict__ vert_pos,
+                                                          const int32_t* __restrict__ vert_P,
+                                                          const int32_t* __restrict__ vert_first, int32_t* done,
+                                                          Partial* part, unsigned long long* overflow,
+                                                          const int32_t* __restrict__ bv,
+                                                          const int64_t* __restrict__ soff,
+                                                          const uint2* __restrict__ stage, SweepArgs A) {
+  namespace cg = cooperative_groups;
+  cg::cluster_group cl = cg::this_cluster();
+  const unsigned rank = cl.block_rank();
+  extern __shared__ unsigned long long smem[];
+  unsigned long long* T = smem;
+  uint32_t* TA = reinterpret_cast<uint32_t*>(smem + kPartSlots);
+  __shared__ long long sh_s[32];
+  __shared__ int sh_c[32];
+  __shared__ unsigned sh_e[32];
+  __shared__ int is_last;
+  for (int t = threadIdx.x; t < kPartSlots; t += blockDim.x) {
+    T[t] = kEmpty;
+    TA[t] = kUnknownA;
+  }
+  cl.sync();  // every table of the cluster is initialised before remote inserts
+  const int lane = threadIdx.x & 31;
+  const int64_t ncl = gridDim.x / kCluCS, cid = blockIdx.x / kCluCS;
+  for (int64_t g = g_begin + cid; g < g_end; g += ncl) {
+    const int32_t vi = grp_vi[g];
+    const uint32_t p0 = (uint32_t)grp_p0[g];
+    const int32_t pos = vert_pos[vi];
+    const uint32_t P = (uint32_t)vert_P[vi];
+    const int32_t v = __ldg(&bv[pos]);
+    const int64_t sb = __ldg(&soff[pos]), deg = __ldg(&soff[pos + 1]) - sb;
+    // table size of this group: 2x the expected labels per partition + slack
+    const uint32_t cap = (uint32_t)min((int64_t)kPartSlots, 2 * ((deg + P - 1) / P) + 512);
+    const uint2* S = stage + sb;
+    const uint32_t* Wt = UNIT ? nullptr : A.w + __ldg(&A.rowptr[v]);
+    const int64_t lo = deg * rank / kCluCS, hi = deg * (rank + 1) / kCluCS;
+    for (int64_t base = lo; base + (int64_t)(threadIdx.x - lane) < hi; base += 4 * (int64_t)blockDim.x) {
+      uint2 rr[4];
+      uint32_t ww[4];
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        const int64_t t = base + threadIdx.x + (int64_t)q * blockDim.x;
+        rr[q] = (t < hi) ? __ldcg(&S[t]) : make_uint2(kSelf, 0u);
+        ww[q] = UNIT ? 1u : ((t < hi) ? __ldcg(&Wt[t]) : 0u);
+      }
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        const uint32_t d = (rr[q].x != kSelf) ? part_of((int32_t)rr[q].x, P) - p0 : 0xFFFFFFFFu;
+        bool keep = d < (uint32_t)kCluCS;
+        uint32_t x = ww[q], arep = rr[q].y;
+        // equal labels of a warp are merged first when adjacent lanes share one
+        const uint32_t key = keep ? rr[q].x : (0x80000000u | (unsigned)lane);
+        if (__any_sync(kFull, key == __shfl_xor_sync(kFull, key, 1))) {
+          const unsigned m = __match_any_sync(kFull, key);
+          x = __reduce_add_sync(m, x);
+          const unsigned rep = __ballot_sync(kFull, keep && rr[q].y != kUnknownA) & m;
+          arep = __shfl_sync(kFull, rr[q].y, rep ? __ffs(rep) - 1 : lane);
+          if (!rep) arep = kUnknownA;
+          keep = keep && lane == __ffs(m) - 1;
+        }
+        if (!keep) continue;
+        unsigned long long* Tr = cl.map_shared_rank(T, d);
+        const unsigned long long kx = ((unsigned long long)rr[q].x << 32) | x;
+        uint32_t h = hash_slot((int32_t)rr[q].x, cap);
+        uint32_t probes = 0;
+        for (;;) {
+          const unsigned long long old = atomicCAS(&Tr[h], kEmpty, kx);
+          if (old == kEmpty) break;
+          if ((uint32_t)(old >> 32) == rr[q].x) {
+            atomicAdd(&Tr[h], (unsigned long long)x);
+            break;
+          }
+          h = (h + 1 == cap) ? 0u : h + 1;
+          if (++probes >= cap) {  // table full: cannot happen at the planned load; reported as an error
+            atomicAdd(overflow, 1ull);
+            break;
+          }
+        }
+        if (arep != kUnknownA) cl.map_shared_rank(TA, d)[h] = arep;
+      }
+    }
+    cl.sync();  // all inserts into every table of the cluster are done
+    const uint32_t p = p0 + rank;
+    if (p < P) {
+      const int32_t own = (int32_t)__ldg(&A.ca[v]).x;
+      const uint32_t ki = __ldg(&A.k[v]);
+      const bool own_single = A.rule == 2 && __ldg(&A.size[own]) == 1;
+      long long s = (long long)0x8000000000000000ull;
+      int cb = 0x7FFFFFFF;
+      unsigned eown = 0;
+      scan_table(T, TA, cap, threadIdx.x, blockDim.x, own, own_single, ki, A, s, cb, eown);
+      block_reduce(s, cb, eown, sh_s, sh_c, sh_e);
+      const int32_t f = vert_first[vi];
+      if (threadIdx.x == 0) {
+        part[f + p] = Partial{s, cb, eown};
+        __threadfence();
+        is_last = (atomicAdd(&done[vi], 1) == (int)P - 1);
+      }
+      __syncthreads();
+      if (is_last && threadIdx.x < 32) {
+        __threadfence();
+        s = (long long)0x8000000000000000ull;
+        cb = 0x7FFFFFFF;
+        eown = 0;
+        for (uint32_t q = threadIdx.x; q < P; q += 32) {
+          const longlong2 raw = __ldcg(reinterpret_cast<const longlong2*>(&part[f + q]));
+          const long long ps = raw.x;
+          const int pc = (int)(raw.y & 0xFFFFFFFFll);
+          const unsigned pe = (unsigned)((unsigned long long)raw.y >> 32);
+          if (better(ps, pc, s, cb)) { s = ps; cb = pc; }
+          eown += pe;
+        }
+        group_reduce<32>(s, cb, eown);
+        int32_t tgt = own;
+        if (threadIdx.x == 0) tgt = finish(s, cb, eown, own, __ldg(&A.ca[own]).y, ki, A);
+        log_moves(threadIdx.x == 0 && tgt != own, v, tgt, A);
+      }
+    }
+    cl.sync();  // every table is scanned (and cleared) before the next group's inserts
+  }
+}
+
 // Task (v, p) of the plan: inserts the partition's pre-scattered entries
 // (S2[poff[p] .. poff[p+1])) into a smem table of 2 * n_p slots (n_p = entries >=
 // distinct labels: load <= 1/2, no overflow possible) -- or kPartSlots with a
@@ -1642,6 +1776,15 @@ int32_t launch_hub(Handle& h, Level& L, const SweepArgs& A, const uint2* stage, 
   return LOUVAIN_OK;
 }
 
+// LV_CLU=1: cluster (DSMEM) streaming groups instead of single-CTA streaming tasks.
+// Measured 2.4x slower on C5 (level 0: 30.7 -> 72.5 ms per 2 sweeps; level 1:
+// 14.9 -> 36.9 ms): one remote CAS round trip per label costs more than the
+// redundant L2 streaming it saves.  Kept as an experiment (parity-tested).
+static bool clu_on() {
+  static const bool on = getenv("LV_CLU") && getenv("LV_CLU")[0] == '1';
+  return on;
+}
+
 // The label-partitioned path of one bucket.  Plan vertices are ordered by degree
 // (descending); those with P > kStreamMaxP form a prefix and take the
 // pre-partitioned pipeline (histogram -> scan -> scatter -> tasks), the rest
@@ -1724,7 +1867,48 @@ int32_t launch_part(Handle& h, Level& L, const SweepArgs& A, int bucket, bool un
     }
     mark("pre-tasks");
   }
-  if (t1 > ts) {  // streaming tasks
+  const int64_t g0 = Q.bucket_grp[bucket - 1], g1 = Q.bucket_grp[bucket];
+  if (t1 > ts && clu_on() && g1 > g0) {  // streaming tasks, cluster variant (LV_CLU=1)
+    static bool cattr = false;
+    if (!cattr) {
+      LV_TRY(set_smem(sweep_part_clu<true>, 12 * (size_t)kPartSlots));
+      LV_TRY(set_smem(sweep_part_clu<false>, 12 * (size_t)kPartSlots));
+      cattr = true;
+    }
+    static_assert(kCluCS == kCluGroup, "cluster size must match the plan's group size");
+    cudaLaunchConfig_t cfg = {};
+    cfg.blockDim = dim3(1024, 1, 1);
+    cfg.dynamicSmemBytes = 12 * (size_t)kPartSlots;
+    cfg.stream = s;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeClusterDimension;
+    at[0].val.clusterDim.x = kCluCS;
+    at[0].val.clusterDim.y = 1;
+    at[0].val.clusterDim.z = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    static int max_clu = 0;  // co-resident clusters (GPC packing decides, not 148 / kCluCS)
+    if (max_clu == 0) {
+      cfg.gridDim = dim3(148 / kCluCS * kCluCS, 1, 1);
+      int nc = 0;
+      LV_CUDA(cudaOccupancyMaxActiveClusters(&nc, sweep_part_clu<true>, &cfg));
+      max_clu = std::max(nc, 1);
+    }
+    const int64_t nclu = std::min<int64_t>(g1 - g0, max_clu);
+    cfg.gridDim = dim3((unsigned)(nclu * kCluCS), 1, 1);
+    if (unit)
+      LV_CUDA(cudaLaunchKernelEx(&cfg, sweep_part_clu<true>, (const int32_t*)Q.grp_vi, (const int32_t*)Q.grp_p0, g0, g1,
+                                 (const int32_t*)Q.vert_pos, (const int32_t*)Q.vert_P, (const int32_t*)Q.vert_first,
+                                 Q.done, (Partial*)Q.partial, &h.ctl->overflow, (const int32_t*)L.bin_vertices,
+                                 (const int64_t*)L.soff, stage, A));
+    else
+      LV_CUDA(cudaLaunchKernelEx(&cfg, sweep_part_clu<false>, (const int32_t*)Q.grp_vi, (const int32_t*)Q.grp_p0, g0,
+                                 g1, (const int32_t*)Q.vert_pos, (const int32_t*)Q.vert_P,
+                                 (const int32_t*)Q.vert_first, Q.done, (Partial*)Q.partial, &h.ctl->overflow,
+                                 (const int32_t*)L.bin_vertices, (const int64_t*)L.soff, stage, A));
+    LV_LAUNCHED();
+    mark("stream");
+  } else if (t1 > ts) {  // streaming tasks
     if (unit)
       sweep_part_stream<true><<<grid_for(t1 - ts, 1, 148 * 2), 1024, 12 * (size_t)kPartSlots, s>>>(
           Q.task_vpos, Q.task_p, ts, t1, Q.vert_pos, Q.vert_P, Q.vert_first, Q.done, (Partial*)Q.partial,

@@ -334,6 +334,16 @@ def _alt_path_worker(env_items, names, q):
     (("LV_BIG_HASH", "1"),),
     # sweep: batched table kernel for sub-class 0
     (("LV_BATCH", "1"),),
+    # sweep: cluster (DSMEM) streaming groups instead of single-CTA streaming tasks
+    (("LV_CLU", "1"),),
+    (("LV_CLU", "1"), ("LV_STREAM_MAXP", "100000")),
+    # sweep: every hub vertex on the streaming path (no pre-partitioned prefix)
+    (("LV_STREAM_MAXP", "100000"),),
+    # sweep: full-table scans instead of claimed-slot lists; lists on the CTA tiers
+    (("LV_LIST", "0"),),
+    (("LV_LIST_CTA", "1"),),
+    # contraction: batched 32-bit sorts of the big segments
+    (("LV_BIG_SORT32", "1"),),
 ])
 def test_alternative_paths_match_oracle(env):
     import torch.multiprocessing as tmp

@@ -1,0 +1,6 @@
+#!/bin/bash
+cd "$GRAFT_REPO_ROOT"; mkdir -p gpurun_out
+timeout 1500 python -m pytest tests -m gpu -x -q > gpurun_out/pytest_ab9.log 2>&1; echo "rc=$?" >> gpurun_out/pytest_ab9.log
+LV_TRACE=2 timeout 300 python tools/trace_run.py 27 > /dev/null 2> gpurun_out/ab9_clu.err
+LV_TRACE=2 LV_STREAM_MAXP=100000 timeout 300 python tools/trace_run.py 27 > /dev/null 2> gpurun_out/ab9_cluall.err
+timeout 600 python bench.py > gpurun_out/bench9.jsonl 2> gpurun_out/bench9.err
