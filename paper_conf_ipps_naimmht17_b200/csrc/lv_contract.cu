@@ -851,25 +851,39 @@ __global__ void __launch_bounds__(256) k_compact(const int64_t* __restrict__ sst
       sh_s[r] = sstart[r0 + r];
     }
     __syncthreads();
-    for (int64_t q = q0 + threadIdx.x; q < q1; q += blockDim.x) {
-      int64_t src;
-      if (nr > 0) {
-        int lo = 0, hi = nr - 1;
-        while (lo < hi) {
-          const int mid = (lo + hi + 1) >> 1;
-          if (sh_r[mid] <= q) lo = mid; else hi = mid - 1;
+    for (int64_t qb = q0 + threadIdx.x; qb < q1; qb += 4 * (int64_t)blockDim.x) {  // 4 entries in flight
+      int32_t cc[4];
+      uint32_t ww[4];
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        const int64_t q = qb + (int64_t)u * blockDim.x;
+        if (q >= q1) continue;
+        int64_t src;
+        if (nr > 0) {
+          int lo = 0, hi = nr - 1;
+          while (lo < hi) {
+            const int mid = (lo + hi + 1) >> 1;
+            if (sh_r[mid] <= q) lo = mid; else hi = mid - 1;
+          }
+          src = sh_s[lo] + (q - sh_r[lo]);
+        } else {
+          int64_t lo = 0, hi = np - 1;
+          while (lo < hi) {
+            const int64_t mid = (lo + hi + 1) >> 1;
+            if (rowptr_out[mid] <= q) lo = mid; else hi = mid - 1;
+          }
+          src = sstart[lo] + (q - rowptr_out[lo]);
         }
-        src = sh_s[lo] + (q - sh_r[lo]);
-      } else {
-        int64_t lo = 0, hi = np - 1;
-        while (lo < hi) {
-          const int64_t mid = (lo + hi + 1) >> 1;
-          if (rowptr_out[mid] <= q) lo = mid; else hi = mid - 1;
-        }
-        src = sstart[lo] + (q - rowptr_out[lo]);
+        cc[u] = __ldcs(&oc[src]);
+        ww[u] = __ldcs(&ow[src]);
       }
-      col[q] = __ldcs(&oc[src]);
-      w[q] = __ldcs(&ow[src]);
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        const int64_t q = qb + (int64_t)u * blockDim.x;
+        if (q >= q1) continue;
+        col[q] = cc[u];
+        w[q] = ww[u];
+      }
     }
     __syncthreads();
   }
