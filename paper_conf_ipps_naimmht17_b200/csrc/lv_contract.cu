@@ -37,6 +37,12 @@ constexpr int kWarpMax = 512;      // segments merged by one warp (1024-slot tab
 constexpr int kWarpSlots = 1024;
 constexpr int kMidMax = 8192;      // segments merged by one CTA (16384-slot table)
 constexpr int kMidSlots = 16384;
+// segment classes: 0 small (<= 32), 1..2 warp ([33,128] with 256-slot tables,
+// [129,kWarpMax] with 1024), 3..6 CTA tiers with tables sized to the tier
+// ([513,1024), [1024,2048), [2048,4096), [4096,kMidMax]), 7 big
+constexpr int kSegClasses = 8;
+constexpr int kMidTierCap[4] = {2048, 4096, 8192, kMidSlots};
+constexpr int kMidTierThr[4] = {128, 256, 512, 512};
 
 __global__ void k_flags(const int32_t* size, int64_t n, int32_t* flag) {
   for (int64_t c = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; c < n; c += (int64_t)gridDim.x * blockDim.x)
@@ -71,20 +77,21 @@ __global__ void k_group_meta(const int32_t* skey, const int32_t* vorder, int64_t
 
 __global__ void k_seg_bounds(const int64_t* rfirst, const int64_t* gpos, int64_t np, int64_t n, int64_t* sstart,
                              uint8_t* scls, int32_t* rid, unsigned long long* hist) {
-  __shared__ unsigned long long sh[4];
-  if (threadIdx.x < 4) sh[threadIdx.x] = 0;
+  __shared__ unsigned long long sh[kSegClasses];
+  if (threadIdx.x < kSegClasses) sh[threadIdx.x] = 0;
   __syncthreads();
   for (int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; r < np; r += (int64_t)gridDim.x * blockDim.x) {
     const int64_t b = gpos[rfirst[r]], e = gpos[(r + 1 < np) ? rfirst[r + 1] : n];
     sstart[r] = b;
     const int64_t len = e - b;
-    const int c = len <= 32 ? 0 : (len <= kWarpMax ? 1 : (len <= kMidMax ? 2 : 3));
+    const int c = len <= 32 ? 0 : len <= 128 ? 1 : len <= kWarpMax ? 2 : len < 1024 ? 3 : len < 2048 ? 4
+                : len < 4096 ? 5 : len <= kMidMax ? 6 : 7;
     scls[r] = (uint8_t)c;
     rid[r] = (int32_t)r;
     atomicAdd(&sh[c], 1ull);
   }
   __syncthreads();
-  if (threadIdx.x < 4 && sh[threadIdx.x]) atomicAdd(&hist[threadIdx.x], sh[threadIdx.x]);
+  if (threadIdx.x < kSegClasses && sh[threadIdx.x]) atomicAdd(&hist[threadIdx.x], sh[threadIdx.x]);
 }
 
 // Step 3: grouped[t] = (map[col[e]], w[e]) for the t-th grouped entry.
@@ -268,15 +275,16 @@ __global__ void __launch_bounds__(256) k_merge_small(const int32_t* __restrict__
 }
 
 // Step 4b: segments of 33..512 entries, one warp each with a 1024-slot smem table.
+template <int SLOTS>
 __global__ void __launch_bounds__(128) k_merge_warp(const int32_t* __restrict__ rows, int64_t nr,
                                                     const int64_t* __restrict__ sstart,
                                                     const int64_t* __restrict__ send_, const int32_t* __restrict__ gc,
                                                     const uint32_t* __restrict__ gw, int32_t* oc, uint32_t* ow,
                                                     int64_t* cnt) {
-  __shared__ unsigned long long tab[4][kWarpSlots];  // 4 warps x 8 KB
+  __shared__ unsigned long long tab[4][SLOTS];  // 4 warps x SLOTS x 8 B
   const int lane = threadIdx.x & 31, wl = threadIdx.x >> 5;
   unsigned long long* T = tab[wl];
-  for (int t = lane; t < kWarpSlots; t += 32) T[t] = kEmpty;
+  for (int t = lane; t < SLOTS; t += 32) T[t] = kEmpty;
   __syncwarp();
   const int64_t warps = (int64_t)gridDim.x * 4;
   for (int64_t k = (int64_t)blockIdx.x * 4 + wl; k < nr; k += warps) {
@@ -323,16 +331,16 @@ __global__ void __launch_bounds__(512) k_merge_mid(const int32_t* __restrict__ r
                                                    const int64_t* __restrict__ sstart,
                                                    const int64_t* __restrict__ send_, const int32_t* __restrict__ gc,
                                                    const uint32_t* __restrict__ gw, int32_t* oc, uint32_t* ow,
-                                                   int64_t* cnt) {
-  extern __shared__ unsigned long long T[];  // kMidSlots slots (dynamic: 64 KB)
+                                                   int64_t* cnt, int capmax) {
+  extern __shared__ unsigned long long T[];  // capmax slots (dynamic)
   __shared__ unsigned ncnt;
-  for (int t = threadIdx.x; t < kMidSlots; t += blockDim.x) T[t] = kEmpty;
+  for (int t = threadIdx.x; t < capmax; t += blockDim.x) T[t] = kEmpty;
   if (threadIdx.x == 0) ncnt = 0;
   __syncthreads();
   for (int64_t k = blockIdx.x; k < nr; k += gridDim.x) {
     const int32_t r = rows[k];
     const int64_t b = sstart[r], len = send_[r] - b;
-    const uint32_t cap = (uint32_t)((2 * len < (int64_t)kMidSlots) ? 2 * len : (int64_t)kMidSlots);
+    const uint32_t cap = (uint32_t)((2 * len < (int64_t)capmax) ? 2 * len : (int64_t)capmax);
     for (int64_t t = threadIdx.x; t < len; t += blockDim.x) {
       const int32_t c = gc[b + t];
       const uint32_t x = gw ? gw[b + t] : 1u;
@@ -1017,28 +1025,29 @@ int32_t level_contract_fast(Handle& h, Level& L, Level& out, int32_t* d_map, int
   LV_TRY(dalloc(&rid, np, s));
   LV_TRY(dalloc(&rows, np, s));
   unsigned long long* hist = nullptr;
-  LV_TRY(dalloc(&hist, 4, s));
-  LV_CUDA(cudaMemsetAsync(hist, 0, 32, s));
+  LV_TRY(dalloc(&hist, kSegClasses, s));
+  LV_CUDA(cudaMemsetAsync(hist, 0, 8 * kSegClasses, s));
   k_seg_bounds<<<grid_for(np, 256), 256, 0, s>>>(rfirst, gpos, np, n, sstart, scls, rid, hist);
   LV_LAUNCHED();
-  unsigned long long hh[4];
-  LV_CUDA(cudaMemcpyAsync(hh, hist, 32, cudaMemcpyDeviceToHost, s));
+  unsigned long long hh[kSegClasses];
+  LV_CUDA(cudaMemcpyAsync(hh, hist, 8 * kSegClasses, cudaMemcpyDeviceToHost, s));
   LV_CUDA(cudaMemcpyAsync(sstart + np, gpos + n, 8, cudaMemcpyDeviceToDevice, s));
   send_ = sstart + 1;
   dfree(rfirst, s);
   dfree(gpos, s);
   {
     size_t tb = 0;
-    LV_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, tb, scls, scls2, rid, rows, np, 0, 2, s));
+    LV_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, tb, scls, scls2, rid, rows, np, 0, 3, s));
     void* tmp = nullptr;
     LV_TRY(dmalloc(&tmp, tb, s));
-    LV_CUDA(cub::DeviceRadixSort::SortPairs(tmp, tb, scls, scls2, rid, rows, np, 0, 2, s));  // 4 classes
+    LV_CUDA(cub::DeviceRadixSort::SortPairs(tmp, tb, scls, scls2, rid, rows, np, 0, 3, s));  // kSegClasses classes
     LV_CUB();
     dfree(tmp, s);
   }
   LV_CUDA(cudaStreamSynchronize(s));
   dfree(hist, s);
-  const int64_t nsmall = (int64_t)hh[0], nwarp = (int64_t)hh[1], nmid = (int64_t)hh[2], nbig = (int64_t)hh[3];
+  const int64_t nsmall = (int64_t)hh[0], nwarp = (int64_t)(hh[1] + hh[2]),
+                nmid = (int64_t)(hh[3] + hh[4] + hh[5] + hh[6]), nbig = (int64_t)hh[7];
   dfree(scls, s);
   dfree(scls2, s);
   dfree(rid, s);
@@ -1069,20 +1078,40 @@ int32_t level_contract_fast(Handle& h, Level& L, Level& out, int32_t* d_map, int
     LV_LAUNCHED();
   }
   tr.mark(s, "merge-small");
-  if (nwarp > 0) {
-    k_merge_warp<<<grid_for(nwarp, 4, 148 * 12), 128, 0, ms>>>(rows + nsmall, nwarp, sstart, send_, gc, gw, oc, ow, cnt);
+  if (hh[1] > 0) {
+    k_merge_warp<256><<<grid_for((int64_t)hh[1], 4, 148 * 16), 128, 0, ms>>>(rows + nsmall, (int64_t)hh[1], sstart,
+                                                                              send_, gc, gw, oc, ow, cnt);
+    LV_LAUNCHED();
+  }
+  if (hh[2] > 0) {
+    k_merge_warp<kWarpSlots><<<grid_for((int64_t)hh[2], 4, 148 * 12), 128, 0, ms>>>(
+        rows + nsmall + (int64_t)hh[1], (int64_t)hh[2], sstart, send_, gc, gw, oc, ow, cnt);
     LV_LAUNCHED();
   }
   tr.mark(s, "merge-warp");
   if (nmid > 0) {
     static bool attr = false;
+    static int resident[4] = {0, 0, 0, 0};
     if (!attr) {
       LV_CUDA(cudaFuncSetAttribute(k_merge_mid, cudaFuncAttributeMaxDynamicSharedMemorySize, 8 * kMidSlots));
       attr = true;
     }
-    k_merge_mid<<<grid_for(nmid, 1, 148 * 3), 512, 8 * kMidSlots, ms>>>(rows + nsmall + nwarp, nmid, sstart, send_, gc, gw,
-                                                                    oc, ow, cnt);
-    LV_LAUNCHED();
+    int64_t off = nsmall + nwarp;
+    for (int t = 0; t < 4; ++t) {  // CTA tiers, tables sized to the tier (more segments in flight per SM)
+      const int64_t cntt = (int64_t)hh[3 + t];
+      if (cntt > 0) {
+        const size_t sm = 8 * (size_t)kMidTierCap[t];
+        if (resident[t] == 0) {
+          int nb = 0;
+          LV_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_merge_mid, kMidTierThr[t], sm));
+          resident[t] = std::max(nb, 1);
+        }
+        k_merge_mid<<<grid_for(cntt, 1, 148 * resident[t]), kMidTierThr[t], sm, ms>>>(
+            rows + off, cntt, sstart, send_, gc, gw, oc, ow, cnt, kMidTierCap[t]);
+        LV_LAUNCHED();
+      }
+      off += cntt;
+    }
   }
   tr.mark(s, "merge-mid");
   // LV_BIG_HASH=1: L2-wave global hash tables for the big segments (measured slower
