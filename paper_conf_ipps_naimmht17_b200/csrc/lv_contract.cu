@@ -446,6 +446,119 @@ __global__ void k_big_place(const unsigned long long* __restrict__ ukeys, const 
 
 
 
+// Combiner for the big segments when their keys are 32-bit (few new vertices: the
+// contracted graph is small and the big segments repeat the same neighbours many
+// times -- C5 level 2: 1.7e9 entries -> 3.6e6 distinct).  Each CTA folds a chunk
+// of kCombChunk (key, weight) pairs in a shared-memory table (one slot {key:32 |
+// sum:32}); a pair whose probe sequence passes kCombProbes slots is passed through
+// unchanged.  The output (distinct pairs of every chunk + pass-throughs) has the
+// same sums per key as the input, so the radix sort + reduce-by-key that follow
+// give the same result on far fewer elements.
+constexpr int kCombSlots = 16384;
+constexpr int kCombChunk = 65536;
+constexpr int kCombProbes = 32;
+__global__ void __launch_bounds__(1024, 1) k_big_combine(const uint32_t* __restrict__ keys,
+                                                         const uint32_t* __restrict__ vals, int64_t m,
+                                                         uint32_t* __restrict__ okeys, uint32_t* __restrict__ ovals,
+                                                         unsigned long long* ocount) {
+  extern __shared__ unsigned long long T[];  // kCombSlots
+  __shared__ unsigned wcnt[32];
+  __shared__ unsigned long long sh_base;
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  for (int t = threadIdx.x; t < kCombSlots; t += blockDim.x) T[t] = kEmpty;
+  __syncthreads();
+  const int64_t nch = (m + kCombChunk - 1) / kCombChunk;
+  for (int64_t ch = blockIdx.x; ch < nch; ch += gridDim.x) {
+    const int64_t e0 = ch * kCombChunk, e1 = min(m, e0 + kCombChunk);
+    for (int64_t eb = e0 + threadIdx.x; eb - threadIdx.x < e1; eb += 4 * (int64_t)blockDim.x) {
+      uint32_t k[4], v[4];
+      bool pass[4];
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        const int64_t e = eb + (int64_t)q * blockDim.x;
+        pass[q] = false;
+        k[q] = 0xFFFFFFFFu;
+        v[q] = 0;
+        if (e < e1) {
+          k[q] = __ldcs(&keys[e]);
+          v[q] = __ldcs(&vals[e]);
+        }
+      }
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {  // equal keys of a warp merged first (hot neighbours)
+        const unsigned mm = __match_any_sync(kFull, k[q]);
+        v[q] = __reduce_add_sync(mm, v[q]);
+        if (lane != __ffs(mm) - 1) k[q] = 0xFFFFFFFFu;
+      }
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        if (k[q] == 0xFFFFFFFFu) continue;
+        const unsigned long long kx = ((unsigned long long)k[q] << 32) | v[q];
+        uint32_t h = (k[q] * 2654435761u) >> (32 - 14);
+        int pr = 0;
+        for (; pr < kCombProbes; ++pr) {
+          const unsigned long long old = atomicCAS(&T[h], kEmpty, kx);
+          if (old == kEmpty) break;
+          if ((uint32_t)(old >> 32) == k[q]) {
+            atomicAdd(&T[h], (unsigned long long)v[q]);
+            break;
+          }
+          h = (h + 1) & (kCombSlots - 1);
+        }
+        pass[q] = pr == kCombProbes;
+      }
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {  // pass-throughs: warp-aggregated global append
+        const unsigned mk = __ballot_sync(kFull, pass[q]);
+        if (!mk) continue;
+        unsigned long long b = 0;
+        if (lane == __ffs(mk) - 1) b = atomicAdd(ocount, (unsigned long long)__popc(mk));
+        b = __shfl_sync(kFull, b, __ffs(mk) - 1);
+        if (pass[q]) {
+          const unsigned long long o = b + __popc(mk & ((1u << lane) - 1u));
+          okeys[o] = k[q];
+          ovals[o] = v[q];
+        }
+      }
+    }
+    __syncthreads();
+    // emit the distinct pairs: per-warp counts -> one global atomic per CTA
+    constexpr int kPer = kCombSlots / 1024;  // slots per thread (contiguous per warp)
+    const int s0 = wid * 32 * kPer;
+    unsigned mine = 0;
+    for (int u = 0; u < kPer; ++u) mine += T[s0 + u * 32 + lane] != kEmpty;
+    unsigned wsum = mine;
+    for (int o = 16; o >= 1; o >>= 1) wsum += __shfl_xor_sync(kFull, wsum, o);
+    if (lane == 0) wcnt[wid] = wsum;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      unsigned tot = 0;
+      for (int w = 0; w < 32; ++w) {
+        const unsigned c = wcnt[w];
+        wcnt[w] = tot;
+        tot += c;
+      }
+      sh_base = tot ? atomicAdd(ocount, (unsigned long long)tot) : 0ull;
+    }
+    __syncthreads();
+    unsigned long long o = sh_base + wcnt[wid];
+    for (int u = 0; u < kPer; ++u) {
+      const int t = s0 + u * 32 + lane;
+      const unsigned long long x = T[t];
+      const bool has = x != kEmpty;
+      const unsigned mk = __ballot_sync(kFull, has);
+      if (has) {
+        const unsigned long long oo = o + __popc(mk & ((1u << lane) - 1u));
+        okeys[oo] = (uint32_t)(x >> 32);
+        ovals[oo] = (uint32_t)x;
+        T[t] = kEmpty;
+      }
+      o += __popc(mk);
+    }
+    __syncthreads();
+  }
+}
+
 // Lengths of the big segments (the scan turns them into key-array offsets).
 __global__ void k_big_len(const int32_t* __restrict__ rows, int64_t nbig, const int64_t* __restrict__ sstart,
                           int64_t* len) {
@@ -1377,6 +1490,31 @@ int32_t level_contract_fast(Handle& h, Level& L, Level& out, int32_t* d_map, int
       }
       tr.mark(s, "big-keys");
       cub::DoubleBuffer<uint32_t> kq(k0, k1), vq(v0, v1);
+      // combiner: worthwhile when the big segments repeat neighbours (few new
+      // vertices per big entry); 0xFFFFFFFF must not be a real key (table marker)
+      static const char* comb_env = getenv("LV_BIG_COMBINE");
+      const bool key_ok = (((uint64_t)(nbig - 1) << nb) | (uint64_t)(np - 1)) < 0xFFFFFFFFull;
+      const bool comb = key_ok && (comb_env ? comb_env[0] == '1' : m >= 64 * np);
+      if (comb) {
+        static bool cattr = false;
+        if (!cattr) {
+          LV_CUDA(cudaFuncSetAttribute(k_big_combine, cudaFuncAttributeMaxDynamicSharedMemorySize, 8 * kCombSlots));
+          cattr = true;
+        }
+        unsigned long long* dcnt = reinterpret_cast<unsigned long long*>(&h.ctl->bad);
+        LV_CUDA(cudaMemsetAsync(dcnt, 0, 8, s));
+        k_big_combine<<<grid_for((m + kCombChunk - 1) / kCombChunk, 1, 148), 1024, 8 * kCombSlots, s>>>(k0, v0, m, k1,
+                                                                                                      v1, dcnt);
+        LV_LAUNCHED();
+        unsigned long long m2 = 0;
+        LV_CUDA(cudaMemcpyAsync(&m2, dcnt, 8, cudaMemcpyDeviceToHost, s));
+        LV_CUDA(cudaStreamSynchronize(s));
+        if (tr.on) fprintf(stderr, "[lv]    contract combine: %lld -> %llu entries\n", (long long)m, m2);
+        m = (int64_t)m2;
+        kq = cub::DoubleBuffer<uint32_t>(k1, k0);
+        vq = cub::DoubleBuffer<uint32_t>(v1, v0);
+        tr.mark(s, "big-combine");
+      }
       size_t tb = 0;
       LV_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, tb, kq, vq, m, 0, nb + kb, s));
       void* tmp = nullptr;

@@ -344,6 +344,9 @@ def _alt_path_worker(env_items, names, q):
     (("LV_LIST_CTA", "1"),),
     # contraction: batched 32-bit sorts of the big segments
     (("LV_BIG_SORT32", "1"),),
+    # contraction: shared-memory combiner before the big-segment sort (forced on / off)
+    (("LV_BIG_COMBINE", "1"),),
+    (("LV_BIG_COMBINE", "0"),),
 ])
 def test_alternative_paths_match_oracle(env):
     import torch.multiprocessing as tmp
