@@ -1288,7 +1288,6 @@ __global__ void __launch_bounds__(1024) sweep_part_stream(const int32_t* __restr
   if (threadIdx.x == 0) claimed = 0;
   __syncthreads();
   const int lane = threadIdx.x & 31;
-  const unsigned limit = (unsigned)(kPartSlots / 8 * 7);
   for (int64_t task = t_begin + blockIdx.x; task < t_end; task += gridDim.x) {
     const int32_t vi = task_vpos[task];
     const uint32_t p = (uint32_t)task_p[task];
@@ -1298,6 +1297,11 @@ __global__ void __launch_bounds__(1024) sweep_part_stream(const int32_t* __restr
     const int64_t sb = __ldg(&soff[pos]), deg = __ldg(&soff[pos + 1]) - sb;
     const uint2* S = stage + sb;
     const uint32_t* Wt = UNIT ? nullptr : A.w + __ldg(&A.rowptr[v]);
+    // table sized to the task: ~2x its expected labels (deg / P) + slack, so the
+    // scan visits ~2 slots per label instead of all kPartSlots (C5 level 0: the
+    // full-table scans were most of this kernel's work)
+    const uint32_t cap = (uint32_t)min((int64_t)kPartSlots, 2 * ((deg + P - 1) / P) + 512);
+    const unsigned limit = cap / 8 * 7;
     // Only ~1/P of the streamed entries belong to this task: each warp compacts
     // the matching entries into a shared queue (ballot + popc) and inserts them
     // 32 at a time, so the insert code runs with full warps.
@@ -1307,7 +1311,7 @@ __global__ void __launch_bounds__(1024) sweep_part_stream(const int32_t* __restr
     auto insert_one = [&](uint2 e, uint32_t x) {
       const int32_t c = (int32_t)e.x;
       const unsigned long long key = ((unsigned long long)(uint32_t)c) << 32;
-      uint32_t h = hash_slot(c, kPartSlots);
+      uint32_t h = hash_slot(c, cap);
       for (;;) {
         const unsigned long long old = atomicCAS(&T[h], kEmpty, key | x);
         if (old == kEmpty) {
@@ -1318,8 +1322,8 @@ __global__ void __launch_bounds__(1024) sweep_part_stream(const int32_t* __restr
           atomicAdd(&T[h], (unsigned long long)x);
           break;
         }
-        h = (h + 1 == (uint32_t)kPartSlots) ? 0 : h + 1;
-        if (claimed >= (unsigned)kPartSlots - 1) {
+        h = (h + 1 == cap) ? 0 : h + 1;
+        if (claimed >= cap - 1) {
           atomicAdd(overflow, 1ull);
           break;
         }
@@ -1383,7 +1387,7 @@ __global__ void __launch_bounds__(1024) sweep_part_stream(const int32_t* __restr
     long long s = (long long)0x8000000000000000ull;
     int cb = 0x7FFFFFFF;
     unsigned eown = 0;
-    scan_table(T, TA, kPartSlots, threadIdx.x, blockDim.x, own, own_single, ki, A, s, cb, eown);
+    scan_table(T, TA, cap, threadIdx.x, blockDim.x, own, own_single, ki, A, s, cb, eown);
     block_reduce(s, cb, eown, sh_s, sh_c, sh_e);
     if (threadIdx.x == 0) {
       part[task] = Partial{s, cb, eown};
