@@ -46,6 +46,11 @@ void dfree(void* p, cudaStream_t s) {
   if (p) cudaFreeAsync(p, s);
 }
 
+int32_t scratch_size(Handle& h, int slot, size_t* bytes) {
+  *bytes = h.scratch.bytes[slot];
+  return LOUVAIN_OK;
+}
+
 int32_t scratch_get(Handle& h, int slot, size_t bytes, void** out) {
   Scratch& S = h.scratch;
   if (S.bytes[slot] < bytes) {

@@ -203,13 +203,15 @@ struct Level {
 // every level and every run): avoids multi-GB stream-ordered allocations
 // churning the memory pool between levels.
 enum ScratchSlot {
-  SC_STAGE = 0, SC_GC, SC_GW, SC_OC, SC_OW, SC_K1, SC_V0, SC_V1, SC_TMP, SC_TILES,
+  SC_STAGE = 0, SC_GC, SC_GW, SC_OC, SC_OW, SC_K1, SC_V0, SC_V1, SC_TMP, SC_TILES, SC_GTAB,
   // arrays of a contracted level inside louvain_run, double-buffered by level parity
   SC_LVL0, SC_LVL_END = SC_LVL0 + 2 * 12, SC_COUNT = SC_LVL_END
 };
 enum LevelArray { LA_ROWPTR = 0, LA_COL, LA_W, LA_K, LA_CA, LA_SIZE, LA_MVV, LA_MVN, LA_MVO, LA_BIN, LA_SOFF, LA_C };
 struct Scratch {
   void* p[SC_COUNT] = {nullptr};
+  void* gtab_init = nullptr;  // SC_GTAB buffer whose slots were initialised to empty (sweep_gtab)
+  size_t gtab_init_bytes = 0;
   size_t bytes[SC_COUNT] = {0};
 };
 
@@ -246,6 +248,7 @@ int32_t dalloc(T** p, size_t count, cudaStream_t s) {
 }
 bool is_device_ptr(const void* p);
 int32_t scratch_get(Handle& h, int slot, size_t bytes, void** out);  // grow-only per-handle buffer
+int32_t scratch_size(Handle& h, int slot, size_t* bytes);  // current size of a scratch buffer
 void scratch_free(Handle& h);
 
 // ------------------------------------------------------------------ level ops (lv_level.cu)

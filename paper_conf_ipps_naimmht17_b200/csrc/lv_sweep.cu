@@ -171,6 +171,7 @@ __global__ void __launch_bounds__(256) sweep_small(const int32_t* __restrict__ v
 // Table scan shared by the warp and CTA kernels: slots [t0, cap) step `stride`.
 // Clears every visited slot for the next vertex.  4 slots per pass so the a_c
 // gathers of labels without a representative in the row overlap.
+template <bool GLOBAL = false>
 __device__ __forceinline__ void scan_table(unsigned long long* T, uint32_t* TA, uint32_t cap, uint32_t t0,
                                            uint32_t stride, int32_t own, bool own_single, uint32_t ki,
                                            const SweepArgs& A, long long& s, int& cb, unsigned& eown) {
@@ -183,11 +184,16 @@ __device__ __forceinline__ void scan_table(unsigned long long* T, uint32_t* TA, 
       x[q] = kEmpty;
       ac[q] = kUnknownA;
       if (t < cap) {
-        x[q] = T[t];
+        x[q] = GLOBAL ? __ldcg(&T[t]) : T[t];  // global tables: L2 (atomics live there), never a stale L1 line
         if (x[q] != kEmpty) {
-          ac[q] = TA[t];
-          T[t] = kEmpty;
-          TA[t] = kUnknownA;
+          ac[q] = GLOBAL ? __ldcg(&TA[t]) : TA[t];
+          if (GLOBAL) {
+            __stcg(&T[t], kEmpty);
+            __stcg(&TA[t], kUnknownA);
+          } else {
+            T[t] = kEmpty;
+            TA[t] = kUnknownA;
+          }
         }
       }
     }
@@ -1420,6 +1426,55 @@ __global__ void __launch_bounds__(1024) sweep_part_stream(const int32_t* __restr
 }
 
 
+// Hub vertices of the label-partitioned path (the streaming ones, deg >= kSub5Min)
+// with a per-CTA table in global memory instead of P label partitions: each CTA
+// takes the next vertex (dynamic, the plan lists them by degree, descending),
+// inserts its staged labels once into a 2*deg-slot region of its own (4-slot
+// buckets, gtable_insert4: one L2 round trip per insert), scans and clears it.
+// The live regions of all CTAs (~148 x 2 x deg x 12 B) stay in L2.  Replaces the
+// P-fold streaming of sweep_part_stream (ncu, C5 level 0: 8.6e9 instructions,
+// issue-bound) -- but measured 4x slower (see gtab_on); off by default.
+template <bool UNIT, bool AGG>
+__global__ void __launch_bounds__(512) sweep_gtab(const int32_t* __restrict__ vert_pos, int64_t v_begin,
+                                                  int64_t v_end, unsigned* next, const int32_t* __restrict__ bv,
+                                                  const int64_t* __restrict__ soff, const uint2* __restrict__ stage,
+                                                  SweepArgs A, unsigned long long* gT, uint32_t* gTA,
+                                                  int64_t region) {
+  __shared__ long long sh_s[32];
+  __shared__ int sh_c[32];
+  __shared__ unsigned sh_e[32];
+  __shared__ int64_t sh_vi;
+  unsigned long long* T = gT + (int64_t)blockIdx.x * region;
+  uint32_t* TA = gTA + (int64_t)blockIdx.x * region;
+  for (;;) {
+    if (threadIdx.x == 0) sh_vi = v_begin + (int64_t)atomicAdd(next, 1u);
+    __syncthreads();
+    const int64_t vi = sh_vi;
+    if (vi >= v_end) break;
+    const int32_t pos = vert_pos[vi];
+    const int32_t v = __ldg(&bv[pos]);
+    const int64_t sb = __ldg(&soff[pos]), deg = __ldg(&soff[pos + 1]) - sb;
+    const uint32_t cap = (uint32_t)(((2 * deg + 3) / 4) * 4);
+    insert_staged<UNIT, AGG, true>(T, TA, cap, stage + sb, UNIT ? nullptr : A.w + __ldg(&A.rowptr[v]), deg,
+                                   threadIdx.x, blockDim.x);
+    __syncthreads();
+    const int32_t own = (int32_t)__ldg(&A.ca[v]).x;
+    const uint32_t ki = __ldg(&A.k[v]);
+    const bool own_single = A.rule == 2 && __ldg(&A.size[own]) == 1;
+    long long s = (long long)0x8000000000000000ull;
+    int cb = 0x7FFFFFFF;
+    unsigned eown = 0;
+    scan_table<true>(T, TA, cap, threadIdx.x, blockDim.x, own, own_single, ki, A, s, cb, eown);
+    block_reduce(s, cb, eown, sh_s, sh_c, sh_e);
+    if (threadIdx.x < 32) {
+      int32_t tgt = own;
+      if (threadIdx.x == 0) tgt = finish(s, cb, eown, own, __ldg(&A.ca[own]).y, ki, A);
+      log_moves(threadIdx.x == 0 && tgt != own, v, tgt, A);
+    }
+    __syncthreads();
+  }
+}
+
 // Cluster variant of the streaming tasks (LV_CLU=1, experiment): a cluster of kCluCS CTAs
 // takes kCluCS consecutive partitions p0 .. p0+kCluCS-1 of one vertex.  Every
 // CTA streams 1/kCluCS of the vertex's staged labels and inserts each label of
@@ -1780,6 +1835,36 @@ int32_t launch_hub(Handle& h, Level& L, const SweepArgs& A, const uint2* stage, 
   return LOUVAIN_OK;
 }
 
+// LV_GTAB=1: per-CTA global tables instead of the single-CTA streaming partition
+// tasks.  Measured 4x slower on C5 (level 0: 28.3 -> 111.7 ms per 2 sweeps, with or
+// without warp label merging): L2 atomic round trips per label cost far more than
+// the P-fold L2 streaming they replace.  Kept as an experiment (parity-tested).
+static bool gtab_on() {
+  static const bool on = getenv("LV_GTAB") && getenv("LV_GTAB")[0] == '1';
+  return on;
+}
+// Per-CTA global hash regions for sweep_gtab (grow-only, kept clean: every scan
+// clears what it visited), plus the dynamic vertex counter.
+static int32_t gtab_get(Handle& h, int64_t slots, unsigned long long** T, uint32_t** TA, unsigned** next) {
+  void* p = nullptr;
+  LV_TRY(scratch_get(h, SC_GTAB, 12 * (size_t)slots + 256, &p));
+  size_t have = 0;
+  LV_TRY(scratch_size(h, SC_GTAB, &have));
+  const int64_t cap_slots = (int64_t)((have - 256) / 12);
+  unsigned long long* t = static_cast<unsigned long long*>(p);
+  if (h.scratch.gtab_init != p || h.scratch.gtab_init_bytes != have) {  // new or grown: every slot empty once
+
+    LV_CUDA(cudaMemsetAsync(t, 0xFF, 8 * (size_t)cap_slots, h.stream));             // kEmpty
+    LV_CUDA(cudaMemsetAsync(t + cap_slots, 0xFF, 4 * (size_t)cap_slots, h.stream));  // kUnknownA
+    h.scratch.gtab_init = p;
+    h.scratch.gtab_init_bytes = have;
+  }
+  *T = t;
+  *TA = reinterpret_cast<uint32_t*>(t + cap_slots);
+  *next = reinterpret_cast<unsigned*>(reinterpret_cast<char*>(p) + 12 * (size_t)cap_slots);
+  return LOUVAIN_OK;
+}
+
 // LV_CLU=1: cluster (DSMEM) streaming groups instead of single-CTA streaming tasks.
 // Measured 2.4x slower on C5 (level 0: 30.7 -> 72.5 ms per 2 sweeps; level 1:
 // 14.9 -> 36.9 ms): one remote CAS round trip per label costs more than the
@@ -1872,7 +1957,42 @@ int32_t launch_part(Handle& h, Level& L, const SweepArgs& A, int bucket, bool un
     mark("pre-tasks");
   }
   const int64_t g0 = Q.bucket_grp[bucket - 1], g1 = Q.bucket_grp[bucket];
-  if (t1 > ts && clu_on() && g1 > g0) {  // streaming tasks, cluster variant (LV_CLU=1)
+  if (t1 > ts && gtab_on()) {  // streaming vertices [vs, v1): per-CTA global tables (LV_GTAB=1)
+    int64_t maxdeg = 0;  // the plan lists vertices by degree, descending: the first is the largest
+    {
+      int32_t pos = 0;
+      int64_t so[2] = {0, 0};
+      LV_CUDA(cudaMemcpyAsync(&pos, Q.vert_pos + vs, 4, cudaMemcpyDeviceToHost, s));
+      LV_CUDA(cudaStreamSynchronize(s));
+      LV_CUDA(cudaMemcpyAsync(so, L.soff + pos, 16, cudaMemcpyDeviceToHost, s));
+      LV_CUDA(cudaStreamSynchronize(s));
+      maxdeg = so[1] - so[0];
+    }
+    const int64_t region = ((2 * maxdeg + 3) / 4) * 4;
+    static int resident = 0;
+    if (resident == 0) {
+      int nb = 0;
+      LV_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, sweep_gtab<true, false>, 512, 0));
+      resident = std::max(nb, 1);
+    }
+    const int64_t nblk = std::min<int64_t>(148 * resident, v1 - vs);
+    unsigned long long* gT = nullptr;
+    uint32_t* gTA = nullptr;
+    unsigned* next = nullptr;
+    LV_TRY(gtab_get(h, nblk * region, &gT, &gTA, &next));
+    LV_CUDA(cudaMemsetAsync(next, 0, 4, s));
+    static const char* ge = getenv("LV_GTAB_AGG");
+    const bool gagg = ge ? ge[0] == '1' : !unit;
+    if (unit) {
+      if (gagg) sweep_gtab<true, true><<<(unsigned)nblk, 512, 0, s>>>(Q.vert_pos, vs, v1, next, L.bin_vertices, L.soff, stage, A, gT, gTA, region);
+      else sweep_gtab<true, false><<<(unsigned)nblk, 512, 0, s>>>(Q.vert_pos, vs, v1, next, L.bin_vertices, L.soff, stage, A, gT, gTA, region);
+    } else {
+      if (gagg) sweep_gtab<false, true><<<(unsigned)nblk, 512, 0, s>>>(Q.vert_pos, vs, v1, next, L.bin_vertices, L.soff, stage, A, gT, gTA, region);
+      else sweep_gtab<false, false><<<(unsigned)nblk, 512, 0, s>>>(Q.vert_pos, vs, v1, next, L.bin_vertices, L.soff, stage, A, gT, gTA, region);
+    }
+    LV_LAUNCHED();
+    mark("stream");
+  } else if (t1 > ts && clu_on() && g1 > g0) {  // streaming tasks, cluster variant (LV_CLU=1)
     static bool cattr = false;
     if (!cattr) {
       LV_TRY(set_smem(sweep_part_clu<true>, 12 * (size_t)kPartSlots));

@@ -334,6 +334,9 @@ def _alt_path_worker(env_items, names, q):
     (("LV_BIG_HASH", "1"),),
     # sweep: batched table kernel for sub-class 0
     (("LV_BATCH", "1"),),
+    # sweep: per-CTA global tables instead of single-CTA streaming partition tasks
+    (("LV_GTAB", "1"),),
+    (("LV_GTAB", "1"), ("LV_GTAB_AGG", "1")),
     # sweep: cluster (DSMEM) streaming groups instead of single-CTA streaming tasks
     (("LV_CLU", "1"),),
     (("LV_CLU", "1"), ("LV_STREAM_MAXP", "100000")),
