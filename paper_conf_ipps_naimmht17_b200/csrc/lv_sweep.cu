@@ -2287,21 +2287,12 @@ int32_t launch_sweep_bucket(Handle& h, Level& L, const louvain_params_t& p, int 
   A.mv_new = L.mv_new;
   A.logn = &h.ctl->logn;
   const int64_t hi = (bucket <= 6) ? p.deg_bounds[bucket - 1] : INT64_MAX;
-  // phase 1: gather the records of every neighbour of the bucket's table-based vertices
-  {
-    const bool sub0_small = std::min<int64_t>(hi, kSub1Min - 1) <= 32;
-    const int64_t pos0 = L.class_off[kSubPerBucket * bucket + (sub0_small ? 1 : 0)];
-    const int64_t pos1 = L.class_off[kSubPerBucket * (bucket + 1)];
-    const int c0 = kSubPerBucket * bucket + (sub0_small ? 1 : 0), c1 = kSubPerBucket * (bucket + 1);
-    if (pos1 > pos0) LV_TRY(launch_stage(h, L, pos0, pos1, L.class_soff[c0], L.class_soff[c1]));
-    if (trace_on()) trace_step(h, L, bucket, -1, pos0, pos1);
-  }
-  for (int sub = 0; sub < kSubPerBucket; ++sub) {
+  static const char* agg_env = getenv("LV_AGG");  // diagnostics: LV_AGG=1 forces warp label merging on
+  const bool agg = agg_env && agg_env[0] == '1';
+  auto dispatch = [&](int sub) -> int32_t {
     const int64_t max_deg = (sub == 0) ? std::min<int64_t>(hi, kSub1Min - 1) : hi;
     // warp-level label merging (__match_any_sync before the table insert) is
     // off: measured slower at every level and sweep of C5 (profiles/README.md)
-    static const char* agg_env = getenv("LV_AGG");  // diagnostics: LV_AGG=1 forces it on
-    const bool agg = agg_env && agg_env[0] == '1';
     if (L.w) {
       if (agg) LV_TRY((dispatch_class<false, true>(h, L, A, bucket, sub, max_deg)));
       else LV_TRY((dispatch_class<false, false>(h, L, A, bucket, sub, max_deg)));
@@ -2312,7 +2303,38 @@ int32_t launch_sweep_bucket(Handle& h, Level& L, const louvain_params_t& p, int 
     if (trace_on())
       trace_step(h, L, bucket, sub, L.class_off[kSubPerBucket * bucket + sub],
                  L.class_off[kSubPerBucket * bucket + sub + 1]);
+    return LOUVAIN_OK;
+  };
+  // phase 1: gather the records of every neighbour of the bucket's table-based vertices
+  const bool sub0_small = std::min<int64_t>(hi, kSub1Min - 1) <= 32;
+  const int c0 = kSubPerBucket * bucket + (sub0_small ? 1 : 0), c1 = kSubPerBucket * (bucket + 1);
+  const int cp = kSubPerBucket * bucket + kSubPart;  // first label-partitioned class
+  const int64_t pos0 = L.class_off[c0], pos1 = L.class_off[c1], posp = L.class_off[cp];
+  // The label-partitioned hub classes (issue-bound) run on the side stream,
+  // concurrently with the staging (memory-bound) and the CTA tiers of the rest of
+  // the bucket: both read only the bucket-start snapshot and append to the move
+  // log; the commit waits for both.  LV_OVERLAP=0 serialises.
+  static const bool overlap_env = !(getenv("LV_OVERLAP") && getenv("LV_OVERLAP")[0] == '0');
+  const bool overlap = overlap_env && !trace_on() && posp < pos1 && posp > pos0 && L.hub.nh == 0;
+  if (overlap) {
+    LV_TRY(launch_stage(h, L, posp, pos1, L.class_soff[cp], L.class_soff[c1]));
+    LV_CUDA(cudaEventRecord(h.ev_fork, h.stream));
+    LV_CUDA(cudaStreamWaitEvent(h.side, h.ev_fork, 0));
+    cudaStream_t main_s = h.stream;
+    h.stream = h.side;
+    int32_t rc = LOUVAIN_OK;
+    for (int sub = kSubPart; sub < kSubPerBucket && rc == LOUVAIN_OK; ++sub) rc = dispatch(sub);
+    h.stream = main_s;
+    LV_TRY(rc);
+    LV_CUDA(cudaEventRecord(h.ev_join, h.side));
+    LV_TRY(launch_stage(h, L, pos0, posp, L.class_soff[c0], L.class_soff[cp]));
+    for (int sub = 0; sub < kSubPart; ++sub) LV_TRY(dispatch(sub));
+    LV_CUDA(cudaStreamWaitEvent(h.stream, h.ev_join, 0));
+    return LOUVAIN_OK;
   }
+  if (pos1 > pos0) LV_TRY(launch_stage(h, L, pos0, pos1, L.class_soff[c0], L.class_soff[c1]));
+  if (trace_on()) trace_step(h, L, bucket, -1, pos0, pos1);
+  for (int sub = 0; sub < kSubPerBucket; ++sub) LV_TRY(dispatch(sub));
   return LOUVAIN_OK;
 }
 

@@ -334,6 +334,8 @@ def _alt_path_worker(env_items, names, q):
     (("LV_BIG_HASH", "1"),),
     # sweep: batched table kernel for sub-class 0
     (("LV_BATCH", "1"),),
+    # sweep: hub classes serialised with the rest of their bucket (no side stream)
+    (("LV_OVERLAP", "0"),),
     # sweep: per-CTA global tables instead of single-CTA streaming partition tasks
     (("LV_GTAB", "1"),),
     (("LV_GTAB", "1"), ("LV_GTAB_AGG", "1")),
