@@ -214,8 +214,15 @@ __global__ void __launch_bounds__(256) k_modularity(const int64_t* rowptr, int64
   for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
     const int64_t e0 = e_begin + tile * kTileEdges, e1 = min(nnz, e0 + kTileEdges);
     for_tile_edges(rowptr, n, e0, e1, tr, tile, sh_rows, &sh_u0, &sh_nr, [&](int64_t u, int64_t e) {
+      // the CSR is symmetric (both directions stored; a precondition of
+      // every louvain_* call), so each pair u < v is counted twice from row u and
+      // row v's copy is skipped: half the random label gathers, same L
       const int32_t v = __ldcs(&col[e]);
-      if (__ldg(&lab[v]) == __ldg(&lab[u])) acc += w ? __ldcs(&w[e]) : 1u;
+      if (v >= (int32_t)u) {
+        const uint32_t we = w ? __ldcs(&w[e]) : 1u;
+        if (v == (int32_t)u) acc += we;  // self-loop (stored once, R2)
+        else if (__ldg(&lab[v]) == __ldg(&lab[u])) acc += 2ull * we;
+      }
     });
   }
   unsigned long long s2 = 0;
