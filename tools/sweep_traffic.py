@@ -11,7 +11,7 @@ import json
 import os
 import sys
 
-SWEEP = ("sweep_", "k_stage", "k_commit", "hub_coop")
+SWEEP = ("sweep_", "k_stage", "k_commit", "hub_coop", "k_part_", "k_tile_starts")
 
 
 def main():
