@@ -32,6 +32,8 @@ CONFIGS = {
     "C2": (lambda: graphgen.lfr(1_000_000, seed=1), "LFR-style n=1e6 (C2)"),
     "C3-s20": (lambda: graphgen.rmat(20, seed=1), "R-MAT scale 20"),
     "C3": (lambda: graphgen.rmat(24, seed=1), "R-MAT scale 24 (C3)"),
+    "C4a": (lambda: graphgen.mesh3d(368, True), "3-D 7-point mesh 368^3, Morton ids (C4a)"),
+    "C4b": (lambda: graphgen.rgg(50_000_000, seed=1), "RGG n=5e7, r = 0.55 sqrt(ln n / n) (C4b)"),
 }
 
 
