@@ -42,7 +42,7 @@ int32_t cuda_fail(cudaError_t e, const char* what, const char* file, int line);
 //   sub 1..4: CTA per vertex, table of <= kCap[sub] slots sized to the tier's
 //             degree range so that small tiers keep more vertices in flight per SM:
 //             [512,1024) 256 thr, [1024,2048) 512, [2048,4096) 512, [4096,12288) 1024
-//   sub 5..7: >= 12288      label-partitioned CTA tasks (P = ceil(deg/6144) smem tables,
+//   sub 5..7: >= 12288      label-partitioned CTA tasks (P = ceil(deg/kPartLabels) smem tables,
 //                           the staged entries pre-partitioned); sub 7 (>= 393216) with
 //                           P > kPartMaxP only: hub, cooperative grid, global table ring
 constexpr int kSubPerBucket = 8;
@@ -50,10 +50,10 @@ constexpr int kNumClasses = 8 * kSubPerBucket;
 constexpr int kSubPart = 5, kSubHub = 7;  // first partitioned sub-class, hub sub-class
 constexpr int64_t kSub1Min = 512, kSub2Min = 1024, kSub3Min = 2048, kSub4Min = 4096, kSub5Min = 12288,
                   kSub6Min = 32768, kHubMin = 393216;
-constexpr int kCapT[5] = {1024, 2048, 4096, 8192, 16384};  // smem table slots (12 B each) of sub 0..4
+constexpr int kCapT[5] = {2048, 4096, 8192, 16384, 18432};  // max smem table slots (12 B each) of sub 0..4
 constexpr int kThrT[5] = {128, 256, 512, 512, 1024};
 constexpr int kPerSmT[5] = {16, 8, 4, 2, 1};
-constexpr int kCapMax = 16384;
+constexpr int kCapMax = 18432;
 __host__ __device__ inline int sub_of_degree(int64_t d) {
   return d < kSub1Min ? 0 : d < kSub2Min ? 1 : d < kSub3Min ? 2 : d < kSub4Min ? 3 : d < kSub5Min ? 4
        : d < kSub6Min ? 5 : d < kHubMin ? 6 : 7;
@@ -111,7 +111,7 @@ struct HubPlan {
 // chunks of kPartChunk entries), so task p reads only its own share and keeps
 // it in one shared-memory table.  Vertices with P_v > kPartMaxP (deg > 50 M)
 // go to the cooperative hub kernel instead.
-constexpr int64_t kPartLabels = 6144;  // expected distinct labels per task (table load <= 3/8)
+constexpr int64_t kPartLabels = 10240;  // expected labels per task (table load ~5/8; C5: 6144 / 8192 / 10240 / 12288 -> 28.3 / 22.2 / 21.4 / 21.0 ms at level 0)
 constexpr int kPartSlots = 16384;      // smem table slots per task (12 B each: 192 KB)
 constexpr int kPartMaxP = 8192;        // partitions per vertex (smem histogram of a chunk)
 constexpr int64_t kPartChunk = 32768;  // staged entries per histogram / scatter item

@@ -347,6 +347,15 @@ int32_t level_alloc_state(Level& L, cudaStream_t s) {
 }
 
 static void part_free(PartPlan& Q, cudaStream_t s);
+// Expected labels per partition task (kPartLabels; LV_PART_LABELS overrides, A/B only).
+static int64_t part_labels() {
+  static const int64_t v = [] {
+    const char* e = getenv("LV_PART_LABELS");
+    const long long x = e ? atoll(e) : 0;
+    return (x >= 1024 && x <= kPartSlots * 3 / 4) ? (int64_t)x : kPartLabels;
+  }();
+  return v;
+}
 // Most partitions a vertex may get on the label-partitioned path (more: hub kernel).
 // LV_PART_MAXP lowers it (tests use it to exercise the cooperative hub kernel).
 static int64_t part_maxp() {
@@ -516,7 +525,7 @@ static int32_t build_hub_plan(Handle& h, Level& L) {
     LV_CUDA(cudaStreamSynchronize(s));
     dfree(dd, s);
     for (int64_t i = 0; i < cnt; ++i) {
-      if ((d[i] + kPartLabels - 1) / kPartLabels <= part_maxp()) continue;  // label-partitioned path
+      if ((d[i] + part_labels() - 1) / part_labels() <= part_maxp()) continue;  // label-partitioned path
       hsoff.push_back(so[i]);
       hv.push_back(v[i]);
       hdeg.push_back(d[i]);
@@ -628,7 +637,7 @@ int32_t build_part_plan(Handle& h, Level& L) {
                      [&](int64_t a, int64_t b) { return so[a + 1] - so[a] > so[b + 1] - so[b]; });
     for (int64_t i : ord) {
       const int64_t deg = so[i + 1] - so[i];
-      const int64_t P = (deg + kPartLabels - 1) / kPartLabels;
+      const int64_t P = (deg + part_labels() - 1) / part_labels();
       if (P > part_maxp()) continue;  // giant: cooperative hub kernel
       const int32_t vi = (int32_t)vpos.size();
       vpos.push_back((int32_t)(off + i));

@@ -561,7 +561,7 @@ __global__ void __launch_bounds__(32 * WARPS) sweep_warp(const int32_t* __restri
 template <bool UNIT, bool AGG>
 __global__ void __launch_bounds__(1024) sweep_cta(const int32_t* __restrict__ verts, const int64_t* __restrict__ soff,
                                                   int64_t nv, const uint2* __restrict__ stage, SweepArgs A,
-                                                  int capmax) {
+                                                  int capmax, int fnum) {
   extern __shared__ unsigned long long smem[];
   unsigned long long* T = smem;
   uint32_t* TA = reinterpret_cast<uint32_t*>(smem + capmax);
@@ -579,7 +579,9 @@ __global__ void __launch_bounds__(1024) sweep_cta(const int32_t* __restrict__ ve
     const int64_t deg = __ldg(&A.rowptr[v + 1]) - rb;
     const int32_t own = (int32_t)__ldg(&A.ca[v]).x;
     const uint32_t ki = __ldg(&A.k[v]);
-    const uint32_t cap = (uint32_t)((2 * deg < (int64_t)capmax) ? 2 * deg : (int64_t)capmax);
+    // table of deg * (1 + fnum/8) slots (fnum = 8: load 1/2), at most capmax
+    const int64_t want = deg + ((deg * fnum) >> 3) + 1;
+    const uint32_t cap = (uint32_t)(want < (int64_t)capmax ? want : (int64_t)capmax);
     insert_staged<UNIT, AGG>(T, TA, cap, stage + __ldg(&soff[vi]), UNIT ? nullptr : A.w + rb, deg, threadIdx.x,
                              blockDim.x);
     __syncthreads();
@@ -2065,6 +2067,10 @@ static bool list_cta() {
   static const bool on = getenv("LV_LIST_CTA") && getenv("LV_LIST_CTA")[0] == '1';
   return on;
 }
+static bool pipe_on() {
+  static const bool on = getenv("LV_CTA_PIPE") && getenv("LV_CTA_PIPE")[0] == '1';
+  return on;
+}
 // largest degree of CTA tier `sub` (lv_internal.cuh)
 static int64_t max_deg_of_tier(int sub) {
   static const int64_t ub[5] = {kSub1Min - 1, kSub2Min - 1, kSub3Min - 1, kSub4Min - 1, kSub5Min - 1};
@@ -2128,12 +2134,13 @@ int32_t dispatch_class(Handle& h, Level& L, const SweepArgs& A, int bucket, int 
     }
     if (list_cta()) {  // claimed-slot list variant (LV_LIST_CTA=1; measured slower on C5, tables are 2*deg here)
       static int resident[5] = {0, 0, 0, 0, 0};
-      const int lcap = (int)std::min<int64_t>(caps[sub], max_deg_of_tier(sub));
-      const size_t lsmem = 12 * (size_t)caps[sub] + 2 * (size_t)((lcap + 7) & ~7);
+      const int capl = std::min(caps[sub], 16384);
+      const int lcap = (int)std::min<int64_t>(capl, max_deg_of_tier(sub));
+      const size_t lsmem = 12 * (size_t)capl + 2 * (size_t)((lcap + 7) & ~7);
       static bool lattr = false;
       if (!lattr) {
-        LV_TRY(set_smem(sweep_cta_l<true>, 12 * (size_t)kCapMax + 2 * 12288));
-        LV_TRY(set_smem(sweep_cta_l<false>, 12 * (size_t)kCapMax + 2 * 12288));
+        LV_TRY(set_smem(sweep_cta_l<true>, 12 * (size_t)16384 + 2 * 12288));
+        LV_TRY(set_smem(sweep_cta_l<false>, 12 * (size_t)16384 + 2 * 12288));
         lattr = true;
       }
       if (resident[sub] == 0) {
@@ -2142,7 +2149,27 @@ int32_t dispatch_class(Handle& h, Level& L, const SweepArgs& A, int bucket, int 
         resident[sub] = std::max(nb, 1);
       }
       const unsigned lgrid = grid_for(nv, 1, 148 * resident[sub]);
-      sweep_cta_l<UNIT><<<lgrid, threads[sub], lsmem, s>>>(verts, soff, nv, stage, A, caps[sub]);
+      sweep_cta_l<UNIT><<<lgrid, threads[sub], lsmem, s>>>(verts, soff, nv, stage, A, capl);
+      LV_LAUNCHED();
+      LV_CUDA(cudaGetLastError());
+      return LOUVAIN_OK;
+    }
+    static const int fnum = [] {  // table size factor 1 + fnum/8 (LV_CAP_F, A/B only)
+      const char* e = getenv("LV_CAP_F");
+      const int x = e ? atoi(e) : 0;
+      return (x >= 2 && x <= 24) ? x : 8;
+    }();
+    if (!pipe_on()) {
+      static int resident[5] = {0, 0, 0, 0, 0};
+      const int64_t md = max_deg_of_tier(sub);
+      const int capt = (int)std::min<int64_t>(caps[sub], ((md + ((md * fnum) >> 3) + 1 + 31) / 32) * 32);
+      if (resident[sub] == 0) {
+        int nb = 0;
+        LV_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, sweep_cta<UNIT, AGG>, threads[sub], 12 * (size_t)capt));
+        resident[sub] = std::max(nb, 1);
+      }
+      sweep_cta<UNIT, AGG><<<grid_for(nv, 1, 148 * resident[sub]), threads[sub], 12 * (size_t)capt, s>>>(
+          verts, soff, nv, stage, A, capt, fnum);
       LV_LAUNCHED();
       LV_CUDA(cudaGetLastError());
       return LOUVAIN_OK;
@@ -2159,8 +2186,6 @@ int32_t dispatch_class(Handle& h, Level& L, const SweepArgs& A, int bucket, int 
         pattr = true;
       }
       sweep_cta_pipe<UNIT, AGG><<<grid, threads[sub], smem, s>>>(verts, soff, nv, stage, A, caps[sub]);
-    } else {
-      sweep_cta<UNIT, AGG><<<grid, threads[sub], smem, s>>>(verts, soff, nv, stage, A, caps[sub]);
     }
     LV_LAUNCHED();
   }
