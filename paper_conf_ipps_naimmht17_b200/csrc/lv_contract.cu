@@ -559,6 +559,40 @@ __global__ void __launch_bounds__(1024, 1) k_big_combine(const uint32_t* __restr
   }
 }
 
+// Segmented variant of the big-segment merge (when segment + neighbour bits pass
+// 32): each big segment's neighbours are sorted on their own (CUB segmented radix
+// sort over the nb neighbour bits: 4-byte keys, ceil(nb/8) passes instead of the
+// flat 64-bit sort's 5 passes of 12 bytes), then runs are cut at segment starts
+// and key changes, numbered by a scan and summed by reduce-by-key.
+__global__ void k_seg_mark(const int64_t* __restrict__ boff, int64_t nbig, uint32_t* heads) {
+  for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < nbig; k += (int64_t)gridDim.x * blockDim.x)
+    heads[boff[k]] = 1u;
+}
+__global__ void k_seg_heads(const uint32_t* __restrict__ keys, int64_t m, uint32_t* heads) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < m; i += (int64_t)gridDim.x * blockDim.x)
+    heads[i] = (i == 0 || heads[i] != 0u || keys[i] != keys[i - 1]) ? 1u : 0u;
+}
+__global__ void k_seg_place(const uint32_t* __restrict__ keys, const uint32_t* __restrict__ runid,
+                            const uint32_t* __restrict__ sums, int64_t m, const int64_t* __restrict__ boff,
+                            int64_t nbig, const int32_t* __restrict__ rows, const int64_t* __restrict__ sstart,
+                            int32_t* oc, uint32_t* ow, int64_t* cnt) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < m; i += (int64_t)gridDim.x * blockDim.x) {
+    const uint32_t r = runid[i];
+    if (i > 0 && runid[i - 1] == r) continue;  // not the head of its run
+    int64_t lo = 0, hi = nbig - 1;  // segment of i: largest k with boff[k] <= i
+    while (lo < hi) {
+      const int64_t mid = (lo + hi + 1) >> 1;
+      if (boff[mid] <= i) lo = mid; else hi = mid - 1;
+    }
+    const uint32_t r0 = runid[boff[lo]];
+    const int64_t local = (int64_t)(r - r0);
+    const int32_t row = rows[lo];
+    oc[sstart[row] + local] = (int32_t)keys[i];
+    ow[sstart[row] + local] = sums[r - 1];
+    if (i + 1 == boff[lo + 1] || runid[boff[lo + 1] - 1] == r) cnt[row] = local + 1;
+  }
+}
+
 // Lengths of the big segments (the scan turns them into key-array offsets).
 __global__ void k_big_len(const int32_t* __restrict__ rows, int64_t nbig, const int64_t* __restrict__ sstart,
                           int64_t* len) {
@@ -609,7 +643,7 @@ __global__ void __launch_bounds__(256) k_big_keys_t(const int32_t* __restrict__ 
         k = lo;
         src = sstart[rows[lo]] + (t - boff[lo]);
       }
-      keys[t] = ((K)k << nb) | (K)(uint32_t)__ldcs(&gc[src]);
+      keys[t] = (nb < 0) ? (K)(uint32_t)__ldcs(&gc[src]) : (((K)k << nb) | (K)(uint32_t)__ldcs(&gc[src]));
       vals[t] = gw ? __ldcs(&gw[src]) : 1u;
     }
   }
@@ -1470,7 +1504,66 @@ int32_t level_contract_fast(Handle& h, Level& L, Level& out, int32_t* d_map, int
               (long long)nsmall, (long long)nwarp, (long long)nmid, (long long)nbig, (long long)m, (long long)nnz);
     int kb = 1;
     while (kb < 40 && (1ll << kb) < nbig) ++kb;
-    if (nb + kb <= 32) {  // 32-bit keys: 8 instead of 12 bytes per element and pass
+    // LV_BIG_SEG=1 (experiment): measured slower on C5 -- level 0 26.3 vs 23.5 ms, level 1 270 vs 43 ms
+    // (CUB's segmented radix sort gives a huge segment a single thread block)
+    static const bool seg_env = getenv("LV_BIG_SEG") && getenv("LV_BIG_SEG")[0] == '1';
+    if (nb + kb > 32 && seg_env && nb <= 31 && m < ((int64_t)1 << 31)) {  // segmented sort of neighbour keys
+      uint32_t *k0 = nullptr, *k1 = nullptr, *v0 = nullptr, *v1 = nullptr, *sums = nullptr;
+      {
+        void* p0 = nullptr;
+        LV_TRY(scratch_get(h, SC_STAGE, 8 * (size_t)m, &p0));  // the level's stage is dead during contraction
+        k0 = static_cast<uint32_t*>(p0);
+        k1 = k0 + m;
+        LV_TRY(scratch_get(h, SC_K1, 8 * (size_t)m, &p0));
+        v0 = static_cast<uint32_t*>(p0);
+        v1 = v0 + m;
+        LV_TRY(scratch_get(h, SC_V0, 4 * (size_t)m, &p0));
+        sums = static_cast<uint32_t*>(p0);
+      }
+      {
+        const int64_t* btr = nullptr;
+        LV_TRY(tile_starts(h, dboff, 0, nbig, 0, m, kBigTile, &btr));
+        k_big_keys_t<uint32_t><<<grid_for((m + kBigTile - 1) / kBigTile, 1, 148 * 8), 256, 0, s>>>(
+            brows, nbig, sstart, dboff, btr, m, gc, gw, -1, k0, v0);
+        LV_LAUNCHED();
+      }
+      tr.mark(s, "big-keys");
+      size_t tb = 0;
+      LV_CUDA(cub::DeviceSegmentedRadixSort::SortPairs(nullptr, tb, k0, k1, v0, v1, (int)m, (int)nbig, dboff,
+                                                      dboff + 1, 0, nb, s));
+      void* tmp = nullptr;
+      LV_TRY(dmalloc(&tmp, tb, s));
+      LV_CUDA(cub::DeviceSegmentedRadixSort::SortPairs(tmp, tb, k0, k1, v0, v1, (int)m, (int)nbig, dboff, dboff + 1,
+                                                      0, nb, s));
+      LV_CUB();
+      dfree(tmp, s);
+      tr.mark(s, "big-segsort");
+      // runs: heads (segment starts | key changes) -> inclusive scan = run id -> sums
+      LV_CUDA(cudaMemsetAsync(k0, 0, 4 * (size_t)m, s));
+      k_seg_mark<<<grid_for(nbig, 256), 256, 0, s>>>(dboff, nbig, k0);
+      LV_LAUNCHED();
+      k_seg_heads<<<grid_for(m, 256, 148 * 16), 256, 0, s>>>(k1, m, k0);
+      LV_LAUNCHED();
+      tb = 0;
+      LV_CUDA(cub::DeviceScan::InclusiveSum(nullptr, tb, k0, v0, m, s));
+      LV_TRY(dmalloc(&tmp, tb, s));
+      LV_CUDA(cub::DeviceScan::InclusiveSum(tmp, tb, k0, v0, m, s));
+      LV_CUB();
+      dfree(tmp, s);
+      int64_t* dnum = reinterpret_cast<int64_t*>(&h.ctl->bad);
+      tb = 0;
+      LV_CUDA(cub::DeviceReduce::ReduceByKey(nullptr, tb, v0, k0, v1, sums, dnum, cub::Sum(), m, s));
+      LV_TRY(dmalloc(&tmp, tb, s));
+      LV_CUDA(cub::DeviceReduce::ReduceByKey(tmp, tb, v0, k0, v1, sums, dnum, cub::Sum(), m, s));
+      LV_CUB();
+      dfree(tmp, s);
+      tr.mark(s, "big-reduce");
+      k_seg_place<<<grid_for(m, 256, 148 * 16), 256, 0, s>>>(k1, v0, sums, m, dboff, nbig, brows, sstart, oc, ow, cnt);
+      LV_LAUNCHED();
+      dfree(dboff, s);
+      LV_CUDA(cudaMemsetAsync(&h.ctl->bad, 0, 8, s));
+      tr.mark(s, "big-place");
+    } else if (nb + kb <= 32) {  // 32-bit keys: 8 instead of 12 bytes per element and pass
       uint32_t *k0 = nullptr, *k1 = nullptr, *v0 = nullptr, *v1 = nullptr;
       {
         void* p0 = nullptr;
