@@ -327,11 +327,11 @@ int32_t run_impl(Handle& h, const louvain_params_t& p, int32_t* labels_out, louv
   int32_t* lab = nullptr;
   LV_TRY(dalloc(&lab, n0, s));
   if (n0) { k_iota<<<grid_for(n0, 256), 256, 0, s>>>(lab, n0); LV_LAUNCHED(); }
-  // level 0 starts from singletons; a full run owns every vertex
-  if (L0.own_hi >= 0) {
-    L0.own_hi = -1;
-    L0.bins_valid = false;
-  }
+  // level 0 starts from singletons; a full run owns every vertex.  The
+  // degree binning (a2) is redone by every run -- nothing of a previous run is
+  // reused, so a timed run includes every step of the path.
+  L0.own_hi = -1;
+  L0.bins_valid = false;
   if (n0) LV_TRY(level_set_labels(h, L0, nullptr));
   uint64_t Lq = 0, Sq = 0;  // exact parts of the current level's kept partition
   Level owned;   // current contracted level (levels >= 1)
