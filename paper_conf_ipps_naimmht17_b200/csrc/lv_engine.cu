@@ -9,7 +9,9 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <mutex>
 #include <string>
+#include <tuple>
 #include <vector>
 
 #include "lv_internal.cuh"
@@ -51,6 +53,46 @@ int32_t scratch_size(Handle& h, int slot, size_t* bytes) {
   return LOUVAIN_OK;
 }
 
+// Process-wide cache of scratch buffers released by destroyed handles (per
+// device), so a new handle on the same device -- e.g. every end-to-end call of
+// louvain_create_csr + louvain_run -- reuses device memory instead of paying
+// tens of GB of cudaMalloc again.  LV_SCRATCH_CACHE=0 disables it; an allocation
+// failure releases the cache and retries.
+namespace {
+std::mutex g_cache_mu;
+std::vector<std::tuple<int, void*, size_t>> g_cache;  // (device, ptr, bytes)
+bool cache_on() {
+  static const bool on = !(getenv("LV_SCRATCH_CACHE") && getenv("LV_SCRATCH_CACHE")[0] == '0');
+  return on;
+}
+void* cache_take(int dev, size_t bytes, size_t* got) {
+  std::lock_guard<std::mutex> lk(g_cache_mu);
+  int best = -1;
+  for (int i = 0; i < (int)g_cache.size(); ++i) {
+    const auto& c = g_cache[i];
+    if (std::get<0>(c) == dev && std::get<2>(c) >= bytes &&
+        (best < 0 || std::get<2>(c) < std::get<2>(g_cache[best])))
+      best = i;
+  }
+  if (best < 0) return nullptr;
+  void* p = std::get<1>(g_cache[best]);
+  *got = std::get<2>(g_cache[best]);
+  g_cache.erase(g_cache.begin() + best);
+  return p;
+}
+void cache_release(int dev) {
+  std::lock_guard<std::mutex> lk(g_cache_mu);
+  for (auto it = g_cache.begin(); it != g_cache.end();) {
+    if (std::get<0>(*it) == dev) {
+      cudaFree(std::get<1>(*it));
+      it = g_cache.erase(it);
+    } else {
+      ++it;
+    }
+  }
+}
+}  // namespace
+
 int32_t scratch_get(Handle& h, int slot, size_t bytes, void** out) {
   Scratch& S = h.scratch;
   if (S.bytes[slot] < bytes) {
@@ -60,14 +102,33 @@ int32_t scratch_get(Handle& h, int slot, size_t bytes, void** out) {
       S.p[slot] = nullptr;
       S.bytes[slot] = 0;
     }
-    const size_t want = bytes + bytes / 8;  // headroom: later levels are usually smaller
-    cudaError_t e = cudaMalloc(&S.p[slot], want);
-    if (e != cudaSuccess) {
-      cudaGetLastError();
-      g_err = "scratch allocation of " + std::to_string(want) + " bytes failed: " + cudaGetErrorString(e);
-      return LOUVAIN_E_NOMEM;
+    size_t got = 0;
+    void* c = cache_on() ? cache_take(h.device, bytes, &got) : nullptr;
+    if (c) {
+      S.p[slot] = c;
+      S.bytes[slot] = got;
+    } else {
+      const size_t want = bytes + bytes / 8;  // headroom: later levels are usually smaller
+      cudaError_t e = cudaMalloc(&S.p[slot], want);
+      if (e != cudaSuccess) {  // give cached buffers and pooled stream-ordered memory back, retry once
+        cudaGetLastError();
+        cache_release(h.device);
+        cudaMemPool_t pool;
+        if (cudaDeviceGetDefaultMemPool(&pool, h.device) == cudaSuccess) {
+          cudaStreamSynchronize(h.stream);
+          cudaMemPoolTrimTo(pool, 0);
+        }
+        e = cudaMalloc(&S.p[slot], want);
+      }
+      if (e != cudaSuccess) {
+        cudaGetLastError();
+        S.p[slot] = nullptr;
+        g_err = "scratch allocation of " + std::to_string(want) + " bytes failed: " + cudaGetErrorString(e);
+        return LOUVAIN_E_NOMEM;
+      }
+      S.bytes[slot] = want;
     }
-    S.bytes[slot] = want;
+    if (slot == SC_GTAB) S.gtab_init = nullptr;  // contents unknown: re-initialise
   }
   *out = S.p[slot];
   return LOUVAIN_OK;
@@ -75,7 +136,14 @@ int32_t scratch_get(Handle& h, int slot, size_t bytes, void** out) {
 
 void scratch_free(Handle& h) {
   for (int i = 0; i < SC_COUNT; ++i) {
-    if (h.scratch.p[i]) cudaFree(h.scratch.p[i]);
+    if (h.scratch.p[i]) {
+      if (cache_on()) {
+        std::lock_guard<std::mutex> lk(g_cache_mu);
+        g_cache.emplace_back(h.device, h.scratch.p[i], h.scratch.bytes[i]);
+      } else {
+        cudaFree(h.scratch.p[i]);
+      }
+    }
     h.scratch.p[i] = nullptr;
     h.scratch.bytes[i] = 0;
   }
