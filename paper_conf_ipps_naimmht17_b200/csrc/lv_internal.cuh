@@ -143,7 +143,7 @@ struct PartPlan {
   int64_t bucket_vsplit[8] = {0};  // bucket b's vertices [bucket_vert[b-1], vsplit) are pre-partitioned,
   int64_t bucket_tsplit[8] = {0};  // tasks [bucket_task[b-1], tsplit); the rest stream (P <= kStreamMaxP)
 };
-constexpr int64_t kStreamMaxP = 64;
+constexpr int64_t kStreamMaxP = 16;
 constexpr int kCluGroup = 8;  // partitions per cluster group (= sweep_part_clu's cluster size)
 
 // Batched plan for the table-based vertices of degree <= kBatchMaxDeg (sub-class 0

@@ -367,14 +367,15 @@ static int64_t part_maxp() {
   return v;
 }
 // Vertices with more partitions than this take the pre-partitioned tasks, the
-// others stream.  Measured on C5: streaming wins at levels 0/1 (31 vs 34 ms,
-// 16 vs 25 ms), pre-partitioning at level 2 (34 vs 47 ms), where the rows are
-// long (mean degree ~300) and labels concentrate; so a level with mean degree
-// >= 256 pre-partitions every hub vertex.  LV_STREAM_MAXP overrides.
+// others stream.  Measured on C5 with kPartLabels = 10240 (per 2 sweeps, levels
+// 0/1/2): everything streaming 21.3 / 11.2 / 68.1 ms; P > 16 pre-partitioned
+// 21.2 / 10.4 / 27.1 ms; the earlier rule (pre-partition all hubs of levels with
+// mean degree >= 256, else P > 64) 21.8 / 10.8 / 31.7 ms.  LV_STREAM_MAXP overrides.
 static int64_t stream_maxp(const Level& L) {
   static const char* e = getenv("LV_STREAM_MAXP");
   if (e) return (int64_t)atoll(e);
-  return (L.n > 0 && L.nnz / L.n >= 256) ? 0 : kStreamMaxP;
+  (void)L;
+  return kStreamMaxP;
 }
 static void hub_free(HubPlan& P, cudaStream_t s) {
   dfree(P.ins, s); dfree(P.scans, s); dfree(P.ins_off, s); dfree(P.scan_off, s); dfree(P.wave_hub, s);
