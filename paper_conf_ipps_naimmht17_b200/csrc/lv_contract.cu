@@ -457,19 +457,32 @@ __global__ void k_big_place(const unsigned long long* __restrict__ ukeys, const 
 constexpr int kCombSlots = 16384;
 constexpr int kCombChunk = 65536;
 constexpr int kCombProbes = 32;
-__global__ void __launch_bounds__(1024, 1) k_big_combine(const uint32_t* __restrict__ keys,
+// keys == nullptr: fused with the key build -- entry e of the concatenated big
+// segments is read straight from the grouped copy (segment by binary search over
+// boff, few segments when keys are 32-bit), key = segment << nb | neighbour.
+struct BigSrc {
+  const int32_t* rows;
+  int64_t nbig;
+  const int64_t* sstart;
+  const int64_t* boff;
+  const int32_t* gc;
+  const uint32_t* gw;
+  int nb;
+};
+template <int SLOTS, int BITS, int CHUNK, int THREADS>
+__global__ void __launch_bounds__(THREADS) k_big_combine(const uint32_t* __restrict__ keys,
                                                          const uint32_t* __restrict__ vals, int64_t m,
                                                          uint32_t* __restrict__ okeys, uint32_t* __restrict__ ovals,
-                                                         unsigned long long* ocount) {
-  extern __shared__ unsigned long long T[];  // kCombSlots
+                                                         unsigned long long* ocount, BigSrc src) {
+  extern __shared__ unsigned long long T[];  // SLOTS
   __shared__ unsigned wcnt[32];
   __shared__ unsigned long long sh_base;
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-  for (int t = threadIdx.x; t < kCombSlots; t += blockDim.x) T[t] = kEmpty;
+  for (int t = threadIdx.x; t < SLOTS; t += blockDim.x) T[t] = kEmpty;
   __syncthreads();
-  const int64_t nch = (m + kCombChunk - 1) / kCombChunk;
+  const int64_t nch = (m + CHUNK - 1) / CHUNK;
   for (int64_t ch = blockIdx.x; ch < nch; ch += gridDim.x) {
-    const int64_t e0 = ch * kCombChunk, e1 = min(m, e0 + kCombChunk);
+    const int64_t e0 = ch * CHUNK, e1 = min(m, e0 + CHUNK);
     for (int64_t eb = e0 + threadIdx.x; eb - threadIdx.x < e1; eb += 4 * (int64_t)blockDim.x) {
       uint32_t k[4], v[4];
       bool pass[4];
@@ -480,8 +493,19 @@ __global__ void __launch_bounds__(1024, 1) k_big_combine(const uint32_t* __restr
         k[q] = 0xFFFFFFFFu;
         v[q] = 0;
         if (e < e1) {
-          k[q] = __ldcs(&keys[e]);
-          v[q] = __ldcs(&vals[e]);
+          if (keys) {
+            k[q] = __ldcs(&keys[e]);
+            v[q] = __ldcs(&vals[e]);
+          } else {
+            int64_t lo = 0, hi = src.nbig - 1;  // largest segment with boff <= e
+            while (lo < hi) {
+              const int64_t mid = (lo + hi + 1) >> 1;
+              if (__ldg(&src.boff[mid]) <= e) lo = mid; else hi = mid - 1;
+            }
+            const int64_t at = __ldg(&src.sstart[__ldg(&src.rows[lo])]) + (e - __ldg(&src.boff[lo]));
+            k[q] = ((uint32_t)lo << src.nb) | (uint32_t)__ldcs(&src.gc[at]);
+            v[q] = src.gw ? __ldcs(&src.gw[at]) : 1u;
+          }
         }
       }
 #pragma unroll
@@ -494,7 +518,7 @@ __global__ void __launch_bounds__(1024, 1) k_big_combine(const uint32_t* __restr
       for (int q = 0; q < 4; ++q) {
         if (k[q] == 0xFFFFFFFFu) continue;
         const unsigned long long kx = ((unsigned long long)k[q] << 32) | v[q];
-        uint32_t h = (k[q] * 2654435761u) >> (32 - 14);
+        uint32_t h = (k[q] * 2654435761u) >> (32 - BITS);
         int pr = 0;
         for (; pr < kCombProbes; ++pr) {
           const unsigned long long old = atomicCAS(&T[h], kEmpty, kx);
@@ -503,7 +527,7 @@ __global__ void __launch_bounds__(1024, 1) k_big_combine(const uint32_t* __restr
             atomicAdd(&T[h], (unsigned long long)v[q]);
             break;
           }
-          h = (h + 1) & (kCombSlots - 1);
+          h = (h + 1) & (SLOTS - 1);
         }
         pass[q] = pr == kCombProbes;
       }
@@ -523,7 +547,7 @@ __global__ void __launch_bounds__(1024, 1) k_big_combine(const uint32_t* __restr
     }
     __syncthreads();
     // emit the distinct pairs: per-warp counts -> one global atomic per CTA
-    constexpr int kPer = kCombSlots / 1024;  // slots per thread (contiguous per warp)
+    constexpr int kPer = SLOTS / THREADS;  // slots per thread (contiguous per warp)
     const int s0 = wid * 32 * kPer;
     unsigned mine = 0;
     for (int u = 0; u < kPer; ++u) mine += T[s0 + u * 32 + lane] != kEmpty;
@@ -533,7 +557,7 @@ __global__ void __launch_bounds__(1024, 1) k_big_combine(const uint32_t* __restr
     __syncthreads();
     if (threadIdx.x == 0) {
       unsigned tot = 0;
-      for (int w = 0; w < 32; ++w) {
+      for (int w = 0; w < THREADS / 32; ++w) {
         const unsigned c = wcnt[w];
         wcnt[w] = tot;
         tot += c;
@@ -1574,7 +1598,15 @@ int32_t level_contract_fast(Handle& h, Level& L, Level& out, int32_t* d_map, int
         v0 = static_cast<uint32_t*>(p0);
         v1 = v0 + m;
       }
-      {
+      // combiner: worthwhile when the big segments repeat neighbours (few new
+      // vertices per big entry); 0xFFFFFFFF must not be a real key (table marker)
+      static const char* comb_env = getenv("LV_BIG_COMBINE");
+      const bool key_ok = (((uint64_t)(nbig - 1) << nb) | (uint64_t)(np - 1)) < 0xFFFFFFFFull;
+      const bool comb = key_ok && (comb_env ? comb_env[0] == '1' : m >= 64 * np);
+      // LV_COMB_FUSED=1: the combiner reads the grouped copy directly (no key array) --
+      // measured slower on C5 level 2 (38.4 ms vs 7.4 + 29.1 ms): per-entry segment search
+      static const bool fused = getenv("LV_COMB_FUSED") && getenv("LV_COMB_FUSED")[0] == '1';
+      if (!(comb && fused)) {
         const int64_t* btr = nullptr;
         LV_TRY(tile_starts(h, dboff, 0, nbig, 0, m, kBigTile, &btr));
         k_big_keys_t<uint32_t><<<grid_for((m + kBigTile - 1) / kBigTile, 1, 148 * 8), 256, 0, s>>>(
@@ -1583,21 +1615,26 @@ int32_t level_contract_fast(Handle& h, Level& L, Level& out, int32_t* d_map, int
       }
       tr.mark(s, "big-keys");
       cub::DoubleBuffer<uint32_t> kq(k0, k1), vq(v0, v1);
-      // combiner: worthwhile when the big segments repeat neighbours (few new
-      // vertices per big entry); 0xFFFFFFFF must not be a real key (table marker)
-      static const char* comb_env = getenv("LV_BIG_COMBINE");
-      const bool key_ok = (((uint64_t)(nbig - 1) << nb) | (uint64_t)(np - 1)) < 0xFFFFFFFFull;
-      const bool comb = key_ok && (comb_env ? comb_env[0] == '1' : m >= 64 * np);
       if (comb) {
+        static const bool small = getenv("LV_COMB_SMALL") && getenv("LV_COMB_SMALL")[0] == '1';
         static bool cattr = false;
         if (!cattr) {
-          LV_CUDA(cudaFuncSetAttribute(k_big_combine, cudaFuncAttributeMaxDynamicSharedMemorySize, 8 * kCombSlots));
+          LV_CUDA(cudaFuncSetAttribute(k_big_combine<kCombSlots, 14, kCombChunk, 1024>,
+                                       cudaFuncAttributeMaxDynamicSharedMemorySize, 8 * kCombSlots));
+          LV_CUDA(cudaFuncSetAttribute(k_big_combine<8192, 13, 32768, 512>,
+                                       cudaFuncAttributeMaxDynamicSharedMemorySize, 8 * 8192));
           cattr = true;
         }
         unsigned long long* dcnt = reinterpret_cast<unsigned long long*>(&h.ctl->bad);
         LV_CUDA(cudaMemsetAsync(dcnt, 0, 8, s));
-        k_big_combine<<<grid_for((m + kCombChunk - 1) / kCombChunk, 1, 148), 1024, 8 * kCombSlots, s>>>(k0, v0, m, k1,
-                                                                                                      v1, dcnt);
+        const BigSrc bsrc{brows, nbig, sstart, dboff, gc, gw, nb};
+        const uint32_t* kin = fused ? nullptr : k0;
+        if (small)
+          k_big_combine<8192, 13, 32768, 512><<<grid_for((m + 32767) / 32768, 1, 148 * 3), 512, 8 * 8192, s>>>(
+              kin, v0, m, k1, v1, dcnt, bsrc);
+        else
+          k_big_combine<kCombSlots, 14, kCombChunk, 1024><<<grid_for((m + kCombChunk - 1) / kCombChunk, 1, 148), 1024,
+                                                            8 * kCombSlots, s>>>(kin, v0, m, k1, v1, dcnt, bsrc);
         LV_LAUNCHED();
         unsigned long long m2 = 0;
         LV_CUDA(cudaMemcpyAsync(&m2, dcnt, 8, cudaMemcpyDeviceToHost, s));

@@ -354,6 +354,7 @@ def _alt_path_worker(env_items, names, q):
     # contraction: shared-memory combiner before the big-segment sort (forced on / off)
     (("LV_BIG_COMBINE", "1"),),
     (("LV_BIG_COMBINE", "0"),),
+    (("LV_BIG_COMBINE", "1"), ("LV_COMB_FUSED", "1")),
 ])
 def test_alternative_paths_match_oracle(env):
     import torch.multiprocessing as tmp
