@@ -43,6 +43,7 @@ def parse_args():
     ap.add_argument("--seed", type=int, default=1)
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--e2e-warmup", type=int, default=1)
+    ap.add_argument("--backend", default="nccl", help="process-group backend for N > 1 (gloo: tests only)")
     ap.add_argument("--cpu-seconds", type=float, default=15.0, help="oracle sample budget")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     return ap.parse_args()
@@ -110,6 +111,10 @@ def measured_peak_hbm():
             return float(json.load(f)["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
     except Exception:
         return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+def cfg_name(scale):
+    return {27: "C5", 24: "C3"}.get(scale, "scaled")
 
 
 def recorded_traffic():
@@ -192,7 +197,7 @@ def run_reference(args, rank, world):
           "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * secs / args.steps,
           "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int64",
           "data": "synthetic",
-          "config": {"workload": f"C5 R-MAT scale {args.scale}, {8 << args.scale} tuples, seed {args.seed}",
+          "config": {"workload": f"{cfg_name(args.scale)} R-MAT scale {args.scale}, {8 << args.scale} tuples, seed {args.seed}",
                      "n": hg.n, "nnz": hg.nnz, "parallelism": "1 host core"},
           "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
           "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
@@ -215,6 +220,9 @@ def run_sharded_bench(args, rank, world):
     n, nnz = dg.n, dg.nnz
     p = lvb.params()
 
+    deg = dg.rowptr[1:] - dg.rowptr[:-1]
+    n_act = int((deg > 0).sum().item())
+
     def one_run():
         g = lvb.Graph.from_csr(dg.rowptr, dg.col, borrow=True)
         lab, st = run_sharded(CudaShard(g), p)
@@ -227,28 +235,65 @@ def run_sharded_bench(args, rank, world):
         torch.cuda.synchronize()
         dist.barrier()
         ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        launches0 = lvb.launch_counts()[0]
         ev0.record()
         for _ in range(args.steps):
             stats.append(one_run())
         ev1.record()
         torch.cuda.synchronize()
+        launches = lvb.launch_counts()[0] - launches0
         dist.barrier()
     ms = ev0.elapsed_time(ev1)
-    t = torch.tensor([ms], device=dev)
+    t = torch.tensor([ms, statistics.mean(s_["t_sweep_ms_first"] for s_ in stats)], device=dev,
+                     dtype=torch.float64)
     dist.all_reduce(t, op=dist.ReduceOp.MAX)
-    ms_per_step = float(t.item()) / args.steps
+    ms_per_step = float(t[0].item()) / args.steps
+    t_sw1 = float(t[1].item())  # slowest rank's level-0 sweep 1 (incl. the per-bucket exchanges)
     st0 = stats[0]
     edges_per_run = sum(nz * sw for nz, sw in zip(st0["nnz"], st0["sweeps_per_level"]))
+    # roofline per GPU: the byte model of the sweep split over edge-balanced ranks
+    B = sweep_bytes(n_act, nnz, D=nnz, moved=st0["moved_first"]) / world
+    achieved = B / (t_sw1 / 1e3) / 1e9
+    peak, peak_src = measured_peak_hbm()
+    traffic, traffic_src = recorded_traffic() if args.scale == 27 else (None, None)  # the capture is of C5
+    roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
+                "traffic": traffic / world if traffic else None,
+                "kernel": "level-0 sweep 1 body per GPU (bucket kernels + commits + move all-gathers)",
+                "algorithmic_bytes": B, "t_ms": t_sw1, "peak_source": peak_src,
+                "traffic_source": (traffic_src + " (1-GPU capture / N)") if traffic else None}
+    # end to end: every rank uploads the CSR from pinned host memory, runs, reads the labels back
+    h_rowptr = torch.empty(n + 1, dtype=torch.int64, pin_memory=True)
+    h_col = torch.empty(nnz, dtype=torch.int32, pin_memory=True)
+    h_rowptr.copy_(dg.rowptr)
+    h_col.copy_(dg.col)
+    e2e_s = []
+    for it in range(max(0, args.e2e_warmup) + max(1, args.e2e_steps)):
+        dist.barrier()
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        with lvb.Graph.from_csr(h_rowptr, h_col) as ge:
+            lab, _ = run_sharded(CudaShard(ge), p)
+            lab_h = lab.cpu() if hasattr(lab, "cpu") else lab
+        torch.cuda.synchronize()
+        if it >= max(0, args.e2e_warmup):
+            e2e_s.append(time.perf_counter() - t0)
+    te = torch.tensor([statistics.median(e2e_s)], device=dev, dtype=torch.float64)
+    dist.all_reduce(te, op=dist.ReduceOp.MAX)
+    t_e2e = float(te.item())
     out = {"metric": METRIC, "value": edges_per_run / (ms_per_step / 1e3), "unit": UNIT, "n_gpus": world,
            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
            "scaling": "strong", "vs_baseline": None, "dtype": "int64", "data": "synthetic",
-           "config": {"workload": f"C5 R-MAT scale {args.scale}, {8 << args.scale} tuples, seed {args.seed}, "
+           "config": {"workload": f"{cfg_name(args.scale)} R-MAT scale {args.scale}, {8 << args.scale} tuples, seed {args.seed}, "
                                   "unit weights, isolated vertices removed",
                       "n": n, "nnz": nnz, "l2": "inputs larger than L2",
                       "parallelism": f"{world} GPUs, sweep vertex-sharded (edge-balanced ranges), "
                                      "per-bucket NCCL all-gather of moves, per-sweep L all-reduce"},
-           "clocks": clk.summary(), "q_final": st0["q"], "levels": st0["levels"],
-           "sweeps_per_level": st0["sweeps_per_level"], "louvain_wall_ms": ms_per_step}
+           "roofline": roofline, "clocks": clk.summary(), "gpu_launches": int(launches),
+           "q_final": st0["q"] if "q" in st0 else None, "levels": st0["levels"],
+           "sweeps_per_level": st0["sweeps_per_level"], "louvain_wall_ms": ms_per_step,
+           "sweep1_ms": t_sw1,
+           "e2e": {"value": edges_per_run / t_e2e, "unit": UNIT, "h2d_bytes_per_step": 8 * (n + 1) + 4 * nnz,
+                   "d2h_bytes_per_step": 4 * n, "ms_per_step": 1e3 * t_e2e}}
     if rank == 0:
         emit(out)
 
@@ -311,7 +356,7 @@ def run_ours(args, rank, world):
     B = sweep_bytes(n_act, nnz, D=nnz, moved=moved1)
     achieved = B / (t_sw1 / 1e3) / 1e9
     peak, peak_src = measured_peak_hbm()
-    traffic, traffic_src = recorded_traffic()
+    traffic, traffic_src = recorded_traffic() if args.scale == 27 else (None, None)  # the capture is of C5
     roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
                 "traffic": traffic, "kernel": "level-0 sweep 1 body (7 bucket kernels + commits)",
                 "algorithmic_bytes": B, "t_ms": t_sw1, "peak_source": peak_src,
@@ -320,7 +365,7 @@ def run_ours(args, rank, world):
     out = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
            "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
            "scaling": "weak", "vs_baseline": None, "dtype": "int64", "data": "synthetic",
-           "config": {"workload": f"C5 R-MAT scale {args.scale}, {8 << args.scale} tuples, seed {args.seed}, "
+           "config": {"workload": f"{cfg_name(args.scale)} R-MAT scale {args.scale}, {8 << args.scale} tuples, seed {args.seed}, "
                                   "unit weights, isolated vertices removed",
                       "n": n, "nnz": nnz, "n_active": n_act,
                       "l2": "inputs larger than L2 (col array alone is 4*nnz bytes >> 126 MB)",
@@ -382,10 +427,15 @@ def main():
         run_reference(args, rank, world)
         return
     import torch
-    torch.cuda.set_device(local)
+    # LV_BENCH_ONE_GPU=1 (tests only): every rank on cuda:0, to exercise the N > 1 path on one GPU
+    dev_index = 0 if os.environ.get("LV_BENCH_ONE_GPU") == "1" else local
+    torch.cuda.set_device(dev_index)
     if world > 1:
         import torch.distributed as dist
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if args.backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", dev_index))
+        else:
+            dist.init_process_group(args.backend)
     try:
         if world > 1:
             run_sharded_bench(args, rank, world)

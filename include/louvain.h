@@ -137,6 +137,11 @@ int32_t louvain_run(louvain_graph_t g, const louvain_params_t* p, int32_t* label
                     louvain_stats_t* stats);
 /* Thread-local message of the last error ("" if none). */
 const char* louvain_last_error(void);
+/* Process-wide counters of the kernels (and CUB device calls) this library has
+ * launched so far, on every handle; either pointer may be NULL.  Diagnostics:
+ * the difference around a call counts its launches (louvain_stats_t reports
+ * the same for louvain_run). */
+void louvain_launch_counts(int64_t* kernel_launches, int64_t* cub_calls);
 
 /* ---- sharded sweep primitives (multi-GPU, one process per GPU) ----
  * Every rank holds the same level graph and a replica of the partition state.

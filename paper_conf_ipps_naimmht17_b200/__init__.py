@@ -91,6 +91,7 @@ FUNCS = {
     "louvain_run": (ctypes.c_int32, [ctypes.c_void_p, ctypes.POINTER(Params), ctypes.c_void_p,
                                      ctypes.POINTER(QNum), ctypes.POINTER(Stats)]),
     "louvain_last_error": (ctypes.c_char_p, []),
+    "louvain_launch_counts": (None, [ctypes.c_void_p, ctypes.c_void_p]),
     "louvain_set_owned_range": (ctypes.c_int32, [ctypes.c_void_p, ctypes.c_int64, ctypes.c_int64]),
     "louvain_begin_sweep": (ctypes.c_int32, [ctypes.c_void_p]),
     "louvain_decide_bucket": (ctypes.c_int32, [ctypes.c_void_p, ctypes.POINTER(Params), ctypes.c_int32,
@@ -334,3 +335,11 @@ def run(rowptr, col, w=None, p: Optional[Params] = None, **kw):
     """One-call convenience: CSR in (host or device), (labels, QNum, stats) out."""
     with Graph.from_csr(rowptr, col, w, **kw) as g:
         return g.run(p)
+
+
+def launch_counts() -> tuple[int, int]:
+    """Process-wide (kernel launches, CUB calls) of the library so far."""
+    k = ctypes.c_int64()
+    c = ctypes.c_int64()
+    lib().louvain_launch_counts(ctypes.byref(k), ctypes.byref(c))
+    return int(k.value), int(c.value)

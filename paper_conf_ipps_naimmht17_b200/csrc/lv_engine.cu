@@ -558,6 +558,10 @@ LV_API void louvain_params_default(louvain_params_t* p) {
 }
 
 LV_API const char* louvain_last_error(void) { return g_err.c_str(); }
+LV_API void louvain_launch_counts(int64_t* kernel_launches, int64_t* cub_calls) {
+  if (kernel_launches) *kernel_launches = g_launches;
+  if (cub_calls) *cub_calls = g_cub_calls;
+}
 
 LV_API int32_t louvain_create_csr(int64_t n, int64_t nnz, const int64_t* rowptr, const int32_t* col, const uint32_t* w,
                                   uint32_t flags, void* cuda_stream, louvain_graph_t* out) {

@@ -174,6 +174,12 @@ def run_sharded(engine, p, group=None, max_levels: int = 256):
         while True:
             if p.max_sweeps > 0 and sweeps >= p.max_sweeps:
                 break
+            # level-0 sweep 1 timed on CUDA engines (bench roofline)
+            timed = level == 0 and sweeps == 0 and getattr(dev, "type", dev) == "cuda"
+            if timed:
+                torch.cuda.synchronize()
+                ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                ev0.record()
             cur.begin_sweep()
             moved = 0
             pending = []
@@ -186,6 +192,12 @@ def run_sharded(engine, p, group=None, max_levels: int = 256):
                 moved += int(allm.shape[0])
             if p.mode != 0 and pending:
                 cur.commit_moves(torch.cat(pending, dim=0))
+            if timed:  # device synchronised: every stream's work of the sweep is inside the events
+                torch.cuda.synchronize()
+                ev1.record()
+                ev1.synchronize()
+                st["t_sweep_ms_first"] = ev0.elapsed_time(ev1)
+                st["moved_first"] = moved
             sweeps += 1
             L_own, S, _ = cur.modularity_owned()
             L = _allreduce_int(L_own, dist, group, world, dev)
