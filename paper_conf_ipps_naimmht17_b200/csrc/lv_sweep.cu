@@ -313,7 +313,7 @@ __global__ void __launch_bounds__(256) k_stage(const int32_t* __restrict__ bv, c
                                                int64_t pos0, int64_t pos1, const int64_t* __restrict__ tr,
                                                const int64_t* __restrict__ rowptr,
                                                const int32_t* __restrict__ col, const uint2* __restrict__ ca,
-                                               uint2* __restrict__ stage, bool cs_store) {
+                                               uint2* __restrict__ stage, bool cs_store, bool full_a) {
   __shared__ int64_t sh_so[kStageRows + 1];
   __shared__ int64_t sh_rb[kStageRows];
   __shared__ int32_t sh_v[kStageRows];
@@ -370,13 +370,19 @@ __global__ void __launch_bounds__(256) k_stage(const int32_t* __restrict__ bv, c
       }
 #pragma unroll
       for (int q = 0; q < 4; ++q) rr[q] = (jj[q] >= 0 && jj[q] != vv[q]) ? __ldg(&ca[jj[q]]) : make_uint2(kSelf, 0);
+      if (full_a) {  // a_c of labels whose neighbour is not their representative: a second gather
+#pragma unroll       // here (edge-parallel, latency hidden) instead of in the table scans
+        for (int q = 0; q < 4; ++q)
+          if (jj[q] >= 0 && jj[q] != vv[q] && rr[q].x != (uint32_t)jj[q]) rr[q].y = __ldg(&ca[rr[q].x]).y;
+      }
 #pragma unroll
       for (int q = 0; q < 4; ++q) {
         const int64_t t = base + (int64_t)q * blockDim.x;
         // evict-first store: the stage streams through L2 once and must not
         // displace the gathered records (LV_STAGE_WB=1: plain write-back store)
         const uint2 val = (jj[q] == vv[q]) ? make_uint2(kSelf, 0u)
-                                           : make_uint2(rr[q].x, rr[q].x == (uint32_t)jj[q] ? rr[q].y : kUnknownA);
+                                           : make_uint2(rr[q].x, (full_a || rr[q].x == (uint32_t)jj[q]) ? rr[q].y
+                                                                                                        : kUnknownA);
         if (t < t1) {
           if (cs_store) __stcs(&stage[t], val);
           else stage[t] = val;
@@ -2277,6 +2283,12 @@ static void trace_step(Handle& h, Level& L, int bucket, int sub, int64_t pos0, i
           (long)(e[1] - e[0]), ms, ms > 0 ? (e[1] - e[0]) / ms / 1e6 : 0.0);
 }
 
+// LV_STAGE_A=1: the stage carries a_c for every label (see k_stage), A/B
+static bool stage_full_a() {
+  static const bool on = getenv("LV_STAGE_A") && getenv("LV_STAGE_A")[0] == '1';
+  return on;
+}
+
 int32_t launch_stage(Handle& h, Level& L, int64_t pos0, int64_t pos1, int64_t s0, int64_t s1) {
   if (s1 <= s0) return LOUVAIN_OK;
   static const bool wb = getenv("LV_STAGE_WB") && getenv("LV_STAGE_WB")[0] == '1';
@@ -2285,7 +2297,7 @@ int32_t launch_stage(Handle& h, Level& L, int64_t pos0, int64_t pos1, int64_t s0
   if (tiled || wb) {  // CTA-tiled variant (default)
     LV_TRY(tile_starts(h, L.soff, pos0, pos1, s0, s1, kStageTile, &tr));
     k_stage<<<grid_for((s1 - s0 + kStageTile - 1) / kStageTile, 1, 148 * 8), 256, 0, h.stream>>>(
-        L.bin_vertices, L.soff, pos0, pos1, tr, L.rowptr, L.col, L.ca, L.stage, !wb);
+        L.bin_vertices, L.soff, pos0, pos1, tr, L.rowptr, L.col, L.ca, L.stage, !wb, stage_full_a());
   } else {
     LV_TRY(tile_starts(h, L.soff, pos0, pos1, s0, s1, kStageChunk, &tr));
     k_stage_w<<<grid_for((s1 - s0 + kStageChunk - 1) / kStageChunk, 8, 148 * 8), 256, 0, h.stream>>>(
