@@ -42,13 +42,28 @@ __global__ void k_set_C(const int32_t* labels, int64_t n, uint2* ca, int32_t* si
   }
 }
 
+// a_c = sum_{i in c} k_i and size_c; the lanes of a warp holding the same
+// label are merged first (__match_any_sync): a final partition has few, large
+// communities, and one atomic per vertex on them serialises.
 __global__ void k_totals_add(const uint2* ca, const uint32_t* k, int64_t n, int32_t* size, unsigned long long* bad) {
   uint32_t* a = const_cast<uint32_t*>(reinterpret_cast<const uint32_t*>(ca)) + 1;  // a word, stride 2
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
-    const int32_t c = (int32_t)ca[i].x;
-    if (c < 0 || c >= n) { atomicAdd(bad, 1ull); continue; }
-    atomicAdd(&a[2 * (int64_t)c], k[i]);  // a_c = sum_{i in c} k_i
-    atomicAdd(&size[c], 1);
+  const int lane = threadIdx.x & 31;
+  const int64_t nw = (int64_t)gridDim.x * (blockDim.x >> 5);
+  for (int64_t base = ((int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5)) * 32; base < n; base += nw * 32) {
+    const int64_t i = base + lane;
+    int32_t c = (i < n) ? (int32_t)ca[i].x : -1;
+    if (i < n && (c < 0 || c >= n)) {
+      atomicAdd(bad, 1ull);
+      c = -1;
+    }
+    const bool valid = c >= 0;
+    const uint32_t ki = valid ? k[i] : 0u;
+    const unsigned m = __match_any_sync(kFull, valid ? c : (int32_t)(0x80000000u | (unsigned)lane));
+    const uint32_t ks = __reduce_add_sync(m, ki);
+    if (valid && lane == __ffs(m) - 1) {
+      atomicAdd(&a[2 * (int64_t)c], ks);
+      atomicAdd(&size[c], __popc(m));
+    }
   }
 }
 
@@ -469,6 +484,12 @@ int32_t level_set_labels(Handle& h, Level& L, const int32_t* d_labels) {
   cudaStream_t s = h.stream;
   L.sweeps_done = d_labels ? 1 : 0;
   if (L.n == 0) return LOUVAIN_OK;
+  if (!d_labels) {  // singletons: a = k, size = 1 directly
+    k_init_singletons<<<grid_for(L.n, 256), 256, 0, s>>>(L.k, L.n, L.ca, L.size, L.C);
+    LV_LAUNCHED();
+    LV_CUDA(cudaGetLastError());
+    return LOUVAIN_OK;
+  }
   k_set_C<<<grid_for(L.n, 256), 256, 0, s>>>(d_labels, L.n, L.ca, L.size, L.C);
   LV_LAUNCHED();
   LV_CUDA(cudaMemsetAsync(&h.ctl->bad, 0, 8, s));

@@ -104,6 +104,7 @@ BUILD = {
     "C3": lambda: graphgen.rmat(24, seed=1, device=True),
     "C4a": lambda: graphgen.mesh3d(368, True, device=True),
     "C4b": lambda: graphgen.rgg(50_000_000, seed=1, device=True),
+    "C5": lambda: graphgen.rmat(27, seed=1, device=True),
 }
 
 

@@ -34,6 +34,7 @@ CONFIGS = {
     "C3": (lambda: graphgen.rmat(24, seed=1), "R-MAT scale 24 (C3)"),
     "C4a": (lambda: graphgen.mesh3d(368, True), "3-D 7-point mesh 368^3, Morton ids (C4a)"),
     "C4b": (lambda: graphgen.rgg(50_000_000, seed=1), "RGG n=5e7, r = 0.55 sqrt(ln n / n) (C4b)"),
+    "C5": (lambda: graphgen.rmat(27, seed=1), "R-MAT scale 27 (C5, the bench workload)"),
 }
 
 
