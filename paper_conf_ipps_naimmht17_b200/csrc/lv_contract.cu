@@ -17,6 +17,7 @@
 // sum or a total-order argmax); louvain_aggregate keeps the canonical sorted
 // variant (level_contract in lv_level.cu).
 #include <cub/cub.cuh>
+#include <thrust/iterator/transform_iterator.h>
 #include <cuda_runtime.h>
 
 #include <algorithm>
@@ -617,6 +618,23 @@ __global__ void k_seg_place(const uint32_t* __restrict__ keys, const uint32_t* _
   }
 }
 
+// Views of packed (segment, neighbour, weight) keys for reduce-by-key.
+struct KeyHi {
+  int s;
+  __host__ __device__ unsigned long long operator()(unsigned long long x) const { return x >> s; }
+};
+struct KeyLo {
+  unsigned long long mask;
+  __host__ __device__ uint32_t operator()(unsigned long long x) const { return (uint32_t)(x & mask); }
+};
+__global__ void k_max_u32(const uint32_t* x, int64_t n, unsigned* out) {
+  unsigned mx = 0;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    mx = max(mx, __ldcs(&x[i]));
+  for (int o = 16; o >= 1; o >>= 1) mx = max(mx, __shfl_xor_sync(kFull, mx, o));
+  if ((threadIdx.x & 31) == 0 && mx) atomicMax(out, mx);
+}
+
 // Lengths of the big segments (the scan turns them into key-array offsets).
 __global__ void k_big_len(const int32_t* __restrict__ rows, int64_t nbig, const int64_t* __restrict__ sstart,
                           int64_t* len) {
@@ -634,7 +652,8 @@ __global__ void __launch_bounds__(256) k_big_keys_t(const int32_t* __restrict__ 
                                                     const int64_t* __restrict__ boff, const int64_t* __restrict__ btr,
                                                     int64_t m, const int32_t* __restrict__ gc,
                                                     const uint32_t* __restrict__ gw, int nb,
-                                                    K* __restrict__ keys, uint32_t* __restrict__ vals) {
+                                                    K* __restrict__ keys, uint32_t* __restrict__ vals,
+                                                    int wbits = 0) {
   __shared__ int64_t sh_b[kBigTileSegs + 1];
   __shared__ int64_t sh_src[kBigTileSegs];
   const int64_t ntiles = (m + kBigTile - 1) / kBigTile;
@@ -667,8 +686,13 @@ __global__ void __launch_bounds__(256) k_big_keys_t(const int32_t* __restrict__ 
         k = lo;
         src = sstart[rows[lo]] + (t - boff[lo]);
       }
-      keys[t] = (nb < 0) ? (K)(uint32_t)__ldcs(&gc[src]) : (((K)k << nb) | (K)(uint32_t)__ldcs(&gc[src]));
-      vals[t] = gw ? __ldcs(&gw[src]) : 1u;
+      const K key = (nb < 0) ? (K)(uint32_t)__ldcs(&gc[src]) : (((K)k << nb) | (K)(uint32_t)__ldcs(&gc[src]));
+      const uint32_t wv = gw ? __ldcs(&gw[src]) : 1u;
+      if (wbits > 0) keys[t] = (key << wbits) | (K)wv;  // weight in the low bits: keys-only sort
+      else {
+        keys[t] = key;
+        vals[t] = wv;
+      }
     }
   }
 }
@@ -1669,6 +1693,77 @@ int32_t level_contract_fast(Handle& h, Level& L, Level& out, int32_t* d_map, int
       dfree(dboff, s);
       LV_CUDA(cudaMemsetAsync(&h.ctl->bad, 0, 8, s));
     } else {
+      // weight bits: the largest single entry weight of the level (sums go to a separate array)
+      int wbits = 1;
+      static const bool pack_req = getenv("LV_BIG_PACK") && getenv("LV_BIG_PACK")[0] == '1';
+      if (gw && pack_req) {
+        unsigned* dmx = reinterpret_cast<unsigned*>(&h.ctl->bad);
+        LV_CUDA(cudaMemsetAsync(dmx, 0, 8, s));
+        k_max_u32<<<grid_for(nnz, 256, 148 * 8), 256, 0, s>>>(gw, nnz, dmx);
+        LV_LAUNCHED();
+        unsigned mx = 0;
+        LV_CUDA(cudaMemcpyAsync(&mx, dmx, 4, cudaMemcpyDeviceToHost, s));
+        LV_CUDA(cudaStreamSynchronize(s));
+        LV_CUDA(cudaMemsetAsync(&h.ctl->bad, 0, 8, s));
+        wbits = 1;
+        while (wbits < 32 && (mx >> wbits) != 0u) ++wbits;
+      }
+      // LV_BIG_PACK=1: keys-only sort with the weight packed into the low key bits --
+      // measured slower on C5 (levels 0/1: 15.8 / 30.4 -> 19.3 / 37.1 ms), off
+      static const bool packed_env = getenv("LV_BIG_PACK") && getenv("LV_BIG_PACK")[0] == '1';
+      if (packed_env && nb + kb + wbits <= 64) {  // keys-only sort: 8 instead of 12 bytes per element and pass
+        unsigned long long *k0 = nullptr, *k1 = nullptr;
+        uint32_t* sums = nullptr;
+        {
+          void* p0 = nullptr;
+          LV_TRY(scratch_get(h, SC_STAGE, 8 * (size_t)m, &p0));
+          k0 = static_cast<unsigned long long*>(p0);
+          LV_TRY(scratch_get(h, SC_K1, 8 * (size_t)m, &p0));
+          k1 = static_cast<unsigned long long*>(p0);
+          LV_TRY(scratch_get(h, SC_V0, 4 * (size_t)m, &p0));
+          sums = static_cast<uint32_t*>(p0);
+        }
+        {
+          const int64_t* btr = nullptr;
+          LV_TRY(tile_starts(h, dboff, 0, nbig, 0, m, kBigTile, &btr));
+          k_big_keys_t<unsigned long long><<<grid_for((m + kBigTile - 1) / kBigTile, 1, 148 * 8), 256, 0, s>>>(
+              brows, nbig, sstart, dboff, btr, m, gc, gw, nb, k0, nullptr, wbits);
+          LV_LAUNCHED();
+        }
+        tr.mark(s, "big-keys");
+        cub::DoubleBuffer<unsigned long long> kbuf(k0, k1);
+        size_t tb = 0;
+        LV_CUDA(cub::DeviceRadixSort::SortKeys(nullptr, tb, kbuf, m, wbits, wbits + nb + kb, s));
+        void* tmp = nullptr;
+        LV_TRY(dmalloc(&tmp, tb, s));
+        LV_CUDA(cub::DeviceRadixSort::SortKeys(tmp, tb, kbuf, m, wbits, wbits + nb + kb, s));
+        LV_CUB();
+        dfree(tmp, s);
+        tr.mark(s, "big-sort");
+        int64_t* dnum = reinterpret_cast<int64_t*>(&h.ctl->bad);
+        auto khi = thrust::make_transform_iterator(kbuf.Current(), KeyHi{wbits});
+        auto klo = thrust::make_transform_iterator(kbuf.Current(), KeyLo{(1ull << wbits) - 1ull});
+        unsigned long long* ukeys = kbuf.Alternate();
+        tb = 0;
+        LV_CUDA(cub::DeviceReduce::ReduceByKey(nullptr, tb, khi, ukeys, klo, sums, dnum, cub::Sum(), m, s));
+        LV_TRY(dmalloc(&tmp, tb, s));
+        LV_CUDA(cub::DeviceReduce::ReduceByKey(tmp, tb, khi, ukeys, klo, sums, dnum, cub::Sum(), m, s));
+        LV_CUB();
+        dfree(tmp, s);
+        int64_t nruns = 0;
+        LV_CUDA(cudaMemcpyAsync(&nruns, dnum, 8, cudaMemcpyDeviceToHost, s));
+        LV_CUDA(cudaStreamSynchronize(s));
+        tr.mark(s, "big-reduce");
+        int64_t* first_run = nullptr;
+        LV_TRY(dalloc(&first_run, nbig, s));
+        k_big_first<<<grid_for(nruns, 256), 256, 0, s>>>(ukeys, nruns, nb, first_run);
+        LV_LAUNCHED();
+        k_big_place<<<grid_for(nruns, 256), 256, 0, s>>>(ukeys, sums, nruns, nb, brows, sstart, first_run, oc, ow, cnt);
+        LV_LAUNCHED();
+        dfree(first_run, s);
+        dfree(dboff, s);
+        LV_CUDA(cudaMemsetAsync(&h.ctl->bad, 0, 8, s));
+      } else {
       unsigned long long *k0 = nullptr, *k1 = nullptr;
       uint32_t *v0 = nullptr, *v1 = nullptr;
       {
@@ -1723,6 +1818,7 @@ int32_t level_contract_fast(Handle& h, Level& L, Level& out, int32_t* d_map, int
       dfree(first_run, s);
       dfree(dboff, s);
       LV_CUDA(cudaMemsetAsync(&h.ctl->bad, 0, 8, s));
+      }
     }
     tr.mark(s, "big-place");
   }

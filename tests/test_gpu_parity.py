@@ -349,6 +349,8 @@ def _alt_path_worker(env_items, names, q):
     (("LV_LIST_CTA", "1"),),
     # contraction: batched 32-bit sorts of the big segments
     (("LV_BIG_SORT32", "1"),),
+    # contraction: keys-only sort with packed weights instead of the 64-bit key/value sort
+    (("LV_BIG_PACK", "1"),),
     # contraction: segmented sort of neighbour keys instead of the flat 64-bit sort
     (("LV_BIG_SEG", "1"),),
     # contraction: shared-memory combiner before the big-segment sort (forced on / off)
