@@ -180,6 +180,21 @@ def test_relaxed_full_run():
     assert np.array_equal(lab, r.labels) and st["sweeps_per_level"] == r.sweeps_per_level
 
 
+@pytest.mark.parametrize("name", ["rmat15", "lfr5k", "mesh12_morton", "hubs"])
+@pytest.mark.parametrize("tb,tf,rev", [(1, 3, 1), (3, 6, 1), (4, 7, 1), (2, 6, 0)])
+def test_full_run_threshold_grid(name, tb, tf, rev):
+    """NEXT-4 (Figs. 1-2, 4): the grid tools/threshold_grid.py replays at full size,
+    bit-exact against oracle (b) at small size; rev = 0 keeps a Q-lowering sweep (R15 off)."""
+    g = GRAPHS[name]()
+    # size_limit below n so both thresholds are exercised on these small graphs
+    kw = dict(th_bin_exp=tb, th_final_exp=tf, revert_on_decrease=rev, size_limit=g.n // 8)
+    r = oracle.louvain(g, oracle.params(**kw))
+    lab, q, st = dev_graph(g).run(lvb.params(**kw))
+    assert st["sweeps_per_level"] == r.sweeps_per_level
+    assert st["num_start"] == r.num_start and st["num_end"] == r.num_end
+    assert np.array_equal(lab, r.labels)
+
+
 def test_size_limit_schedule():
     g = GRAPHS["rmat15"]()
     r = oracle.louvain(g, oracle.params(size_limit=1000))
