@@ -394,6 +394,14 @@ int32_t run_impl(Handle& h, const louvain_params_t& p, int32_t* labels_out, louv
   const long long launches0 = g_launches, cub0 = g_cub_calls;
   int32_t* lab = nullptr;
   LV_TRY(dalloc(&lab, n0, s));
+  // labels at each sweep start, for the delta pass of Eq. (1) (LV_MOD_DELTA=0: full passes only)
+  static const bool mod_delta = !(getenv("LV_MOD_DELTA") && getenv("LV_MOD_DELTA")[0] == '0');
+  struct PcnGuard {  // h.pcn lives for this run only
+    Handle& h;
+    ~PcnGuard() { h.pcn = nullptr; }
+  } pcn_guard{h};
+  uint2* pcn = nullptr;
+  if (mod_delta) LV_TRY(dalloc(&pcn, std::max<int64_t>(n0, 1), s));
   if (n0) { k_iota<<<grid_for(n0, 256), 256, 0, s>>>(lab, n0); LV_LAUNCHED(); }
   // level 0 starts from singletons; a full run owns every vertex.  The
   // degree binning (a2) is redone by every run -- nothing of a previous run is
@@ -429,10 +437,13 @@ int32_t run_impl(Handle& h, const louvain_params_t& p, int32_t* labels_out, louv
       for (;;) {
         if (p.max_sweeps > 0 && sweeps >= p.max_sweeps) break;
         cudaEventRecord(h.ev[0], s);
+        h.pcn = pcn;
+        if (mod_delta) LV_TRY(launch_snapshot(h, L));
         LV_TRY(sweep_body(h, L, p));
         cudaEventRecord(h.ev[1], s);
         tr.mark(s, "sweep", level);
-        LV_TRY(launch_modularity(h, L, nullptr));
+        if (mod_delta) LV_TRY(launch_modularity_delta(h, L));
+        else LV_TRY(launch_modularity(h, L, nullptr));
         cudaEventRecord(h.ev[2], s);
         tr.mark(s, "modularity", level);
         LV_CUDA(cudaMemcpyAsync(h.h_ctl, h.ctl, sizeof(DevCtl), cudaMemcpyDeviceToHost, s));
@@ -451,12 +462,19 @@ int32_t run_impl(Handle& h, const louvain_params_t& p, int32_t* labels_out, louv
           return LOUVAIN_E_CUDA;
         }
         const int64_t moved = (int64_t)h.h_ctl->logn;
-        const int64_t num = qnum_of(h.h_ctl->L, h.h_ctl->S, W);
+        // Eq. (1) numerator of the swept partition: delta pass (L_before + dL, exact
+        // modular arithmetic) or full pass
+        const uint64_t L_after = (mod_delta && delta_chosen(*h.h_ctl, L.nnz)) ? Lq + h.h_ctl->dL : h.h_ctl->L;
+        const int64_t num = qnum_of(L_after, h.h_ctl->S, W);
+        if (tr.on)
+          fprintf(stderr, "[lv] level %d sweep %d: moved %llu, moved entries %.4f of nnz, %s pass\n", level, sweeps,
+                  h.h_ctl->logn, L.nnz ? (double)h.h_ctl->mdeg / (double)L.nnz : 0.0,
+                  (mod_delta && delta_chosen(*h.h_ctl, L.nnz)) ? "delta" : "full");
         if (p.revert_on_decrease && num < num_prev) {  // R15
           LV_TRY(launch_revert(h, L));
           break;
         }
-        Lq = h.h_ctl->L;
+        Lq = L_after;
         Sq = h.h_ctl->S;
         moved_level += moved;
         if (moved == 0 || below_threshold(num, num_prev, W, pexp)) break;  // Alg. 1 l.12, R13
@@ -512,6 +530,8 @@ int32_t run_impl(Handle& h, const louvain_params_t& p, int32_t* labels_out, louv
   LV_TRY(copy_out(labels_out, lab, sizeof(int32_t) * (size_t)n0, s));
   LV_CUDA(cudaStreamSynchronize(s));
   dfree(lab, s);
+  h.pcn = nullptr;
+  if (pcn) dfree(pcn, s);
   fill_q(&local.q, Lq, Sq, W);
   local.t_total_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t_begin).count();
   local.kernel_launches = g_launches - launches0;

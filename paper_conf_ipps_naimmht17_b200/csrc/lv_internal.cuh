@@ -66,9 +66,14 @@ constexpr int64_t kHubWaveSlots = 3 << 19;  // table slots per wave (12 B each; 
 struct DevCtl {
   unsigned long long logn;       // move-log entries appended in this sweep
   unsigned long long bounds[9];  // log offset at the start of bucket b's commit
+  unsigned long long mdeg;       // sum of the degrees of the vertices moved in this sweep
   unsigned long long L, S;       // modularity parts
   unsigned long long bad;        // validation flag
   unsigned long long overflow;   // a partitioned hash table filled up (must stay 0)
+  unsigned long long dL;         // delta pass: L_after - L_before (two's complement)
+  unsigned long long nbig;       // delta pass: moved vertices left to the block kernel
+  unsigned long long nmid;       // delta pass: moved vertices left to the warp kernel
+  unsigned long long ddiv;       // delta pass chosen iff mdeg * ddiv <= nnz
 };
 
 // Hub work plan (one per level).  Hubs are grouped into waves whose tables fit
@@ -228,6 +233,9 @@ struct Handle {
   // side stream for independent kernels inside one phase (fork/join through events)
   cudaStream_t side = nullptr;
   cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
+  // louvain_run only: {label at the sweep start, label after} per vertex; the
+  // commit writes .y of every moved vertex (delta pass of Eq. (1))
+  uint2* pcn = nullptr;
   // distributed (nullptr when single GPU)
   void* dist = nullptr;
 };
@@ -263,6 +271,13 @@ int32_t level_binning(Handle& h, Level& L, const louvain_params_t& p);  // class
 // d_C == nullptr: the level's own partition (maintained a_c); else external labels
 int32_t level_modularity(Handle& h, Level& L, const int32_t* d_C, uint64_t* Lout, uint64_t* Sout);
 int32_t launch_modularity(Handle& h, Level& L, const int32_t* d_C);  // async: ctl->L, ctl->S
+// Eq. (1) after a sweep from the sweep's move log (async).  h.pcn[v] = {label at
+// the sweep start, label now}.  If the moved vertices hold <= nnz/3 entries:
+// ctl->dL = L_after - L_before (delta pass), else ctl->L = L_after (full pass);
+// ctl->S either way.  The host tells which from ctl->mdeg (delta_chosen).
+int32_t launch_snapshot(Handle& h, Level& L);  // h.pcn[v] = {C[v], C[v]}
+int32_t launch_modularity_delta(Handle& h, Level& L);
+__host__ __device__ __forceinline__ bool delta_chosen(const DevCtl& c, int64_t nnz) { return c.mdeg * c.ddiv <= (unsigned long long)nnz; }
 int32_t launch_commit(Handle& h, Level& L, int bucket);
 int32_t set_ctl_u64(Handle& h, unsigned long long* dst, unsigned long long v);
 int32_t pack_moves(Handle& h, Level& L, int64_t c0, int64_t cnt, int32_t* out);          // log -> (v,new) pairs

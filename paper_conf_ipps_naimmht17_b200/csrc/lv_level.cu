@@ -137,11 +137,13 @@ __global__ void k_fill_u32v(uint32_t* p, int64_t n, uint32_t v) {
 // Commit of one bucket (Alg. 1 l.8-11): C[i] = newComm[i] and the exact
 // integer a_c / size_c deltas (identical to recomputing a_c, R12).
 __global__ void k_commit(DevCtl* ctl, int bucket, const int32_t* mv_v, const int32_t* mv_new, int32_t* mv_old,
-                         uint2* ca, int32_t* size, const uint32_t* k, int32_t* C) {
+                         uint2* ca, int32_t* size, const uint32_t* k, int32_t* C, const int64_t* rowptr,
+                         uint2* pcn) {
   const unsigned long long start = ctl->bounds[bucket];
   const unsigned long long end = *(volatile unsigned long long*)&ctl->logn;
   if (blockIdx.x == 0 && threadIdx.x == 0) ctl->bounds[bucket + 1] = end;
   uint32_t* w32 = reinterpret_cast<uint32_t*>(ca);
+  unsigned long long md = 0;
   for (unsigned long long p = start + blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; p < end;
        p += (unsigned long long)gridDim.x * blockDim.x) {
     const int32_t i = mv_v[p], t = mv_new[p];
@@ -149,12 +151,16 @@ __global__ void k_commit(DevCtl* ctl, int bucket, const int32_t* mv_v, const int
     mv_old[p] = old;
     w32[2 * (int64_t)i] = (uint32_t)t;
     C[i] = t;
+    if (pcn) pcn[i].y = (uint32_t)t;
     const uint32_t ki = k[i];
     atomicSub(&w32[2 * (int64_t)old + 1], ki);
     atomicAdd(&w32[2 * (int64_t)t + 1], ki);
     atomicSub(&size[old], 1);
     atomicAdd(&size[t], 1);
+    md += (unsigned long long)(rowptr[i + 1] - rowptr[i]);
   }
+  md = warp_sum_u64(md);
+  if ((threadIdx.x & 31) == 0 && md) atomicAdd(&ctl->mdeg, md);
 }
 
 // Undo every move of the sweep (R15).
@@ -219,7 +225,8 @@ __global__ void __launch_bounds__(256) k_modularity(const int64_t* rowptr, int64
                                                     const uint32_t* w, const uint2* ca, const int32_t* C,
                                                     const uint32_t* a, int64_t e_begin, int64_t nnz,
                                                     const int64_t* __restrict__ tr, unsigned long long* Lout,
-                                                    unsigned long long* Sout) {
+                                                    unsigned long long* Sout, const DevCtl* gate = nullptr) {
+  if (gate && delta_chosen(*gate, nnz)) return;  // the delta pass evaluates this sweep
   __shared__ int64_t sh_rows[kTileRows];
   __shared__ int64_t sh_u0;
   __shared__ int sh_nr;
@@ -250,6 +257,114 @@ __global__ void __launch_bounds__(256) k_modularity(const int64_t* rowptr, int64
   if ((threadIdx.x & 31) == 0) {
     if (acc) atomicAdd(Lout, acc);
     if (s2) atomicAdd(Sout, s2);
+  }
+}
+
+// Delta pass of Eq. (1) after a sweep (used by louvain_run when the moved vertices
+// hold <= nnz/4 entries).  L = sum over directed entries (u->v) of w [C(u) == C(v)]
+// (self-loops once, R2) changes only on entries with a moved endpoint.  For a moved
+// i (old label o, new t) and each entry (i->j), j != i:
+//   d = [C'(j) == t] - [C(j) == o]     (C = labels at the sweep start, C' = after)
+// counts for both directions (x2) when j did not move -- the mirror (j->i) holds
+// the same w and the same d (symmetric CSR) -- and once when j moved too (its own
+// row supplies (j->i)).  Self-loops never change.  Exact integers, any order.
+constexpr int64_t kDeltaBigDeg = 4096;  // rows longer than this: one CTA each
+__device__ __forceinline__ long long delta_entry(const uint2* __restrict__ P, int32_t i, int32_t j, uint32_t we,
+                                                 int32_t t, int32_t o) {
+  if (j == i) return 0;
+  const uint2 pj = __ldg(&P[j]);  // {C(j), C'(j)}: one sector for both labels
+  const int d = (int)((int32_t)pj.y == t) - (int)((int32_t)pj.x == o);
+  return d ? (long long)d * (long long)we * (pj.x != pj.y ? 1 : 2) : 0;
+}
+
+__global__ void k_snapshot(const int32_t* __restrict__ C, int64_t n, uint2* P) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    const uint32_t c = (uint32_t)C[i];
+    P[i] = make_uint2(c, c);
+  }
+}
+
+constexpr int64_t kDeltaThrDeg = 32;    // rows up to this length: one thread each
+__global__ void __launch_bounds__(256) k_mod_delta_thr(DevCtl* ctl, const int32_t* __restrict__ mv_v,
+                                                       const int32_t* __restrict__ mv_new,
+                                                       const int32_t* __restrict__ mv_old,
+                                                       const int64_t* __restrict__ rowptr,
+                                                       const int32_t* __restrict__ col,
+                                                       const uint32_t* __restrict__ w, const uint2* __restrict__ P,
+                                                       int64_t nnz, int32_t* mid,
+                                                       int32_t* big) {
+  if (!delta_chosen(*ctl, nnz)) return;
+  const long long logn = (long long)ctl->logn;
+  long long acc = 0;
+  for (long long p = (long long)blockIdx.x * blockDim.x + threadIdx.x; p < logn; p += (long long)gridDim.x * blockDim.x) {
+    const int32_t i = mv_v[p];
+    const int64_t b = rowptr[i], e = rowptr[i + 1];
+    if (e - b > kDeltaBigDeg) {
+      big[atomicAdd(&ctl->nbig, 1ull)] = (int32_t)p;
+    } else if (e - b > kDeltaThrDeg) {
+      mid[atomicAdd(&ctl->nmid, 1ull)] = (int32_t)p;
+    } else {
+      const int32_t t = mv_new[p], o = mv_old[p];
+      for (int64_t q = b; q < e; ++q) acc += delta_entry(P, i, __ldcs(&col[q]), w ? __ldcs(&w[q]) : 1u, t, o);
+    }
+  }
+  const unsigned long long s = warp_sum_u64((unsigned long long)acc);
+  if ((threadIdx.x & 31) == 0 && s) atomicAdd(&ctl->dL, s);
+}
+
+__global__ void __launch_bounds__(256) k_mod_delta_warp(DevCtl* ctl, const int32_t* __restrict__ mid,
+                                                        const int32_t* __restrict__ mv_v,
+                                                        const int32_t* __restrict__ mv_new,
+                                                        const int32_t* __restrict__ mv_old,
+                                                        const int64_t* __restrict__ rowptr,
+                                                        const int32_t* __restrict__ col,
+                                                        const uint32_t* __restrict__ w, const uint2* __restrict__ P,
+                                                        int64_t nnz) {
+  if (!delta_chosen(*ctl, nnz)) return;
+  const long long nmid = (long long)ctl->nmid;
+  const int lane = threadIdx.x & 31;
+  const long long nw = (long long)gridDim.x * (blockDim.x >> 5);
+  long long acc = 0;
+  for (long long k = (long long)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); k < nmid; k += nw) {
+    const int32_t p = mid[k];
+    const int32_t i = mv_v[p], t = mv_new[p], o = mv_old[p];
+    const int64_t b = rowptr[i], e = rowptr[i + 1];
+    for (int64_t q = b + lane; q < e; q += 32)
+      acc += delta_entry(P, i, __ldcs(&col[q]), w ? __ldcs(&w[q]) : 1u, t, o);
+  }
+  const unsigned long long s = warp_sum_u64((unsigned long long)acc);
+  if (lane == 0 && s) atomicAdd(&ctl->dL, s);
+}
+
+// Long rows of the delta pass (one CTA per moved vertex) and S = sum_c a_c^2.
+__global__ void __launch_bounds__(512) k_mod_delta_cta(DevCtl* ctl, const int32_t* __restrict__ big,
+                                                       const int32_t* __restrict__ mv_v,
+                                                       const int32_t* __restrict__ mv_new,
+                                                       const int32_t* __restrict__ mv_old,
+                                                       const int64_t* __restrict__ rowptr,
+                                                       const int32_t* __restrict__ col,
+                                                       const uint32_t* __restrict__ w, const uint2* __restrict__ P,
+                                                       int64_t nnz, const uint2* ca,
+                                                       int64_t n) {
+  if (!delta_chosen(*ctl, nnz)) return;
+  const unsigned long long nbig = ctl->nbig;
+  long long acc = 0;
+  for (unsigned long long k = blockIdx.x; k < nbig; k += gridDim.x) {
+    const int32_t p = big[k];
+    const int32_t i = mv_v[p], t = mv_new[p], o = mv_old[p];
+    for (int64_t q = rowptr[i] + threadIdx.x; q < rowptr[i + 1]; q += blockDim.x)
+      acc += delta_entry(P, i, __ldcs(&col[q]), w ? __ldcs(&w[q]) : 1u, t, o);
+  }
+  unsigned long long s2 = 0;
+  for (int64_t c = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; c < n; c += (int64_t)gridDim.x * blockDim.x) {
+    const unsigned long long x = ca[c].y;
+    s2 += x * x;
+  }
+  const unsigned long long s = warp_sum_u64((unsigned long long)acc);
+  s2 = warp_sum_u64(s2);
+  if ((threadIdx.x & 31) == 0) {
+    if (s) atomicAdd(&ctl->dL, s);
+    if (s2) atomicAdd(&ctl->S, s2);
   }
 }
 
@@ -823,6 +938,50 @@ int32_t launch_modularity(Handle& h, Level& L, const int32_t* d_C) {
   return LOUVAIN_OK;
 }
 
+int32_t launch_snapshot(Handle& h, Level& L) {
+  if (L.n == 0) return LOUVAIN_OK;
+  k_snapshot<<<grid_for(L.n, 256), 256, 0, h.stream>>>(L.C, L.n, h.pcn);
+  LV_LAUNCHED();
+  LV_CUDA(cudaGetLastError());
+  return LOUVAIN_OK;
+}
+
+int32_t launch_modularity_delta(Handle& h, Level& L) {
+  const uint2* P = h.pcn;
+  cudaStream_t s = h.stream;
+  LV_CUDA(cudaMemsetAsync(&h.ctl->L, 0, 16, s));
+  LV_CUDA(cudaMemsetAsync(&h.ctl->dL, 0, 24, s));
+  // moved entries <= nnz / ddiv: delta pass (LV_DELTA_DIV, default 3: one 8-byte
+  // gather per moved entry against one 4-byte gather per pair and the col stream)
+  static const unsigned long long ddiv = getenv("LV_DELTA_DIV") ? strtoull(getenv("LV_DELTA_DIV"), nullptr, 10) : 3ull;
+  LV_TRY(set_ctl_u64(h, &h.ctl->ddiv, ddiv));
+  if (L.n == 0) return LOUVAIN_OK;
+  int32_t *big = nullptr, *mid = nullptr;
+  LV_TRY(dalloc(&big, (size_t)(L.nnz / kDeltaBigDeg + 1), s));
+  LV_TRY(dalloc(&mid, (size_t)(L.nnz / kDeltaThrDeg + 1), s));
+  k_mod_delta_thr<<<148 * 8, 256, 0, s>>>(h.ctl, L.mv_v, L.mv_new, L.mv_old, L.rowptr, L.col, L.w, P,
+                                          L.nnz, mid, big);
+  LV_LAUNCHED();
+  k_mod_delta_warp<<<148 * 8, 256, 0, s>>>(h.ctl, mid, L.mv_v, L.mv_new, L.mv_old, L.rowptr, L.col, L.w, P,
+                                           L.nnz);
+  LV_LAUNCHED();
+  k_mod_delta_cta<<<148 * 4, 512, 0, s>>>(h.ctl, big, L.mv_v, L.mv_new, L.mv_old, L.rowptr, L.col, L.w, P,
+                                          L.nnz, L.ca, L.n);
+  LV_LAUNCHED();
+  dfree(big, s);
+  dfree(mid, s);
+  // full pass, skipped on the device when the delta pass was chosen
+  const int64_t ntiles = (L.nnz + kTileEdges - 1) / kTileEdges;
+  const unsigned grid = grid_for(std::max<int64_t>(ntiles, (L.n + 255) / 256), 1, 148 * 8);
+  const int64_t* tr = nullptr;
+  LV_TRY(tile_starts(h, L.rowptr, 0, L.n, 0, std::max<int64_t>(L.nnz, 1), kTileEdges, &tr));
+  k_modularity<true><<<grid, 256, 0, s>>>(L.rowptr, L.n, L.col, L.w, L.ca, L.C, nullptr, 0, L.nnz, tr, &h.ctl->L,
+                                          &h.ctl->S, h.ctl);
+  LV_LAUNCHED();
+  LV_CUDA(cudaGetLastError());
+  return LOUVAIN_OK;
+}
+
 int32_t level_modularity(Handle& h, Level& L, const int32_t* d_C, uint64_t* Lout, uint64_t* Sout) {
   LV_CUDA(cudaMemsetAsync(&h.ctl->bad, 0, 8, h.stream));
   LV_TRY(launch_modularity(h, L, d_C));
@@ -838,7 +997,8 @@ int32_t level_modularity(Handle& h, Level& L, const int32_t* d_C, uint64_t* Lout
 }
 
 int32_t launch_commit(Handle& h, Level& L, int bucket) {
-  k_commit<<<148 * 4, 256, 0, h.stream>>>(h.ctl, bucket, L.mv_v, L.mv_new, L.mv_old, L.ca, L.size, L.k, L.C);
+  k_commit<<<148 * 4, 256, 0, h.stream>>>(h.ctl, bucket, L.mv_v, L.mv_new, L.mv_old, L.ca, L.size, L.k, L.C,
+                                         L.rowptr, h.pcn);
   LV_LAUNCHED();
   LV_CUDA(cudaGetLastError());
   return LOUVAIN_OK;
