@@ -272,7 +272,7 @@ int32_t level_binning(Handle& h, Level& L, const louvain_params_t& p);  // class
 int32_t level_modularity(Handle& h, Level& L, const int32_t* d_C, uint64_t* Lout, uint64_t* Sout);
 int32_t launch_modularity(Handle& h, Level& L, const int32_t* d_C);  // async: ctl->L, ctl->S
 // Eq. (1) after a sweep from the sweep's move log (async).  h.pcn[v] = {label at
-// the sweep start, label now}.  If the moved vertices hold <= nnz/3 entries:
+// the sweep start, label now}.  If the moved vertices hold <= nnz/ddiv entries:
 // ctl->dL = L_after - L_before (delta pass), else ctl->L = L_after (full pass);
 // ctl->S either way.  The host tells which from ctl->mdeg (delta_chosen).
 int32_t launch_snapshot(Handle& h, Level& L);  // h.pcn[v] = {C[v], C[v]}
