@@ -113,3 +113,42 @@ def test_overflow_guard():
     g = graphgen.weighted_csr(2, [0], [1], [1_600_000_000])
     with pytest.raises(OverflowError):
         oracle.modularity(g, np.arange(2))
+
+
+def _delta_L(g, C0, C1):
+    """The identity the GPU delta pass of Eq. (1) evaluates (DESIGN a5): only entries with a
+    moved endpoint change L; from each moved row, an entry to an unmoved j counts twice (its
+    mirror has the same weight and the same change), to a moved j once."""
+    w = g.w if g.w is not None else np.ones(len(g.col), dtype=np.int64)
+    moved = C0 != C1
+    d = 0
+    for i in np.flatnonzero(moved):
+        for e in range(g.rowptr[i], g.rowptr[i + 1]):
+            j = g.col[e]
+            if j == i:
+                continue
+            ch = int(C1[j] == C1[i]) - int(C0[j] == C0[i])
+            d += ch * int(w[e]) * (1 if moved[j] else 2)
+    return d
+
+
+@pytest.mark.parametrize("maker", [lambda: graphgen.karate(), lambda: graphgen.rmat(10, seed=3),
+                                   lambda: graphgen.weighted_csr(60, [0, 1, 2, 3, 4, 5, 0, 7], [0, 2, 3, 3, 9, 6, 7, 8],
+                                                                 [5, 1, 2, 7, 1, 3, 2, 4])])
+def test_delta_identity_against_eq1(maker):
+    """Pin of the delta-pass reading: L(after) - L(before) of a real sweep (oracle (b)) and of
+    random relabellings equals the moved-rows sum, with L from Eq. (1) (orc_modularity)."""
+    g = maker()
+    rng = np.random.default_rng(0)
+    st = oracle.State(g)
+    for _ in range(3):
+        C0 = st.C.copy()
+        st.sweep(oracle.params())
+        C1 = st.C.copy()
+        assert oracle.modularity(g, C1)[0] - oracle.modularity(g, C0)[0] == _delta_L(g, C0, C1)
+    for _ in range(3):
+        C0 = rng.integers(0, max(2, g.n // 3), size=g.n).astype(np.int32)
+        C1 = C0.copy()
+        flip = rng.random(g.n) < 0.3
+        C1[flip] = rng.integers(0, max(2, g.n // 3), size=int(flip.sum()))
+        assert oracle.modularity(g, C1)[0] - oracle.modularity(g, C0)[0] == _delta_L(g, C0, C1)
