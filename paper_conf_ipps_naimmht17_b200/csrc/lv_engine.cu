@@ -429,7 +429,7 @@ int32_t run_impl(Handle& h, const louvain_params_t& p, int32_t* labels_out, louv
       // level start: singletons.  Level 0 evaluates Eq. (1); a contracted level
       // starts exactly where the previous one ended (contraction preserves L and
       // S, R18 -- pinned by the oracle tests and the parity suite).
-      if (level == 0) LV_TRY(level_modularity(h, L, nullptr, &Lq, &Sq));
+      if (level == 0) LV_TRY(level_modularity(h, L, nullptr, &Lq, &Sq, /*singletons=*/true));
       const int64_t num_start = qnum_of(Lq, Sq, W);
       int64_t num_prev = num_start;
       int64_t moved_level = 0;

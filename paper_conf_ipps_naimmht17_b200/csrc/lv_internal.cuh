@@ -269,13 +269,16 @@ int32_t level_get_labels(Handle& h, Level& L, int32_t* d_out);          // C -> 
 int32_t level_get_a(Handle& h, Level& L, uint32_t* d_out);              // a -> d_out (device)
 int32_t level_binning(Handle& h, Level& L, const louvain_params_t& p);  // classes + hub plan
 // d_C == nullptr: the level's own partition (maintained a_c); else external labels
-int32_t level_modularity(Handle& h, Level& L, const int32_t* d_C, uint64_t* Lout, uint64_t* Sout);
-int32_t launch_modularity(Handle& h, Level& L, const int32_t* d_C);  // async: ctl->L, ctl->S
+// singletons: the caller guarantees C is the singleton partition (no label gathers)
+int32_t level_modularity(Handle& h, Level& L, const int32_t* d_C, uint64_t* Lout, uint64_t* Sout,
+                         bool singletons = false);
+int32_t launch_modularity(Handle& h, Level& L, const int32_t* d_C, bool singletons = false);  // async: ctl->L, ctl->S
 // Eq. (1) after a sweep from the sweep's move log (async).  h.pcn[v] = {label at
 // the sweep start, label now}.  If the moved vertices hold <= nnz/ddiv entries:
 // ctl->dL = L_after - L_before (delta pass), else ctl->L = L_after (full pass);
 // ctl->S either way.  The host tells which from ctl->mdeg (delta_chosen).
 int32_t launch_snapshot(Handle& h, Level& L);  // h.pcn[v] = {C[v], C[v]}
+unsigned long long delta_div();                 // LV_DELTA_DIV (default 1)
 int32_t launch_modularity_delta(Handle& h, Level& L);
 __host__ __device__ __forceinline__ bool delta_chosen(const DevCtl& c, int64_t nnz) { return c.mdeg * c.ddiv <= (unsigned long long)nnz; }
 int32_t launch_commit(Handle& h, Level& L, int bucket);

@@ -157,7 +157,7 @@ __global__ void k_commit(DevCtl* ctl, int bucket, const int32_t* mv_v, const int
     atomicAdd(&w32[2 * (int64_t)t + 1], ki);
     atomicSub(&size[old], 1);
     atomicAdd(&size[t], 1);
-    md += (unsigned long long)(rowptr[i + 1] - rowptr[i]);
+    if (rowptr) md += (unsigned long long)(rowptr[i + 1] - rowptr[i]);
   }
   md = warp_sum_u64(md);
   if ((threadIdx.x & 31) == 0 && md) atomicAdd(&ctl->mdeg, md);
@@ -220,7 +220,9 @@ __device__ __forceinline__ void for_tile_edges(const int64_t* rowptr, int64_t n,
 // Eq. (1): L = sum of w over entries (u,v) with C[u] = C[v] (self-loops
 // included, R2); S = sum_c a_c^2.  Integer atomics: deterministic.  Labels come
 // from the packed records (C = ca.x, a = ca.y) or from an external labelling.
-template <bool PACKED>
+// SINGLE: the partition is known to be singletons (distinct labels, level start,
+// P:164), so C(u) = C(v) iff u = v: L = sum of self-loop weights, no label gathers.
+template <bool PACKED, bool SINGLE = false>
 __global__ void __launch_bounds__(256) k_modularity(const int64_t* rowptr, int64_t n, const int32_t* col,
                                                     const uint32_t* w, const uint2* ca, const int32_t* C,
                                                     const uint32_t* a, int64_t e_begin, int64_t nnz,
@@ -243,7 +245,7 @@ __global__ void __launch_bounds__(256) k_modularity(const int64_t* rowptr, int64
       if (v >= (int32_t)u) {
         const uint32_t we = w ? __ldcs(&w[e]) : 1u;
         if (v == (int32_t)u) acc += we;  // self-loop (stored once, R2)
-        else if (__ldg(&lab[v]) == __ldg(&lab[u])) acc += 2ull * we;
+        else if (!SINGLE && __ldg(&lab[v]) == __ldg(&lab[u])) acc += 2ull * we;
       }
     });
   }
@@ -906,7 +908,7 @@ int32_t level_binning(Handle& h, Level& L, const louvain_params_t& p) {
 
 // Eq. (1) parts into ctl->L / ctl->S (stream-ordered, no sync).  d_C == nullptr:
 // the level's own partition with its maintained a_c; else an external labelling.
-int32_t launch_modularity(Handle& h, Level& L, const int32_t* d_C) {
+int32_t launch_modularity(Handle& h, Level& L, const int32_t* d_C, bool singletons) {
   cudaStream_t s = h.stream;
   LV_CUDA(cudaMemsetAsync(&h.ctl->L, 0, 16, s));
   if (L.n == 0) return LOUVAIN_OK;
@@ -919,7 +921,11 @@ int32_t launch_modularity(Handle& h, Level& L, const int32_t* d_C) {
   } else {
     LV_TRY(tile_starts(h, L.rowptr, 0, L.n, 0, 1, kTileEdges, &tr));  // unused (no tiles)
   }
-  if (!d_C) {
+  if (!d_C && singletons) {
+    k_modularity<true, true><<<grid, 256, 0, s>>>(L.rowptr, L.n, L.col, L.w, L.ca, L.C, nullptr, e0, e1, tr,
+                                                  &h.ctl->L, &h.ctl->S);
+    LV_LAUNCHED();
+  } else if (!d_C) {
     k_modularity<true><<<grid, 256, 0, s>>>(L.rowptr, L.n, L.col, L.w, L.ca, L.C, nullptr, e0, e1, tr, &h.ctl->L,
                                             &h.ctl->S);
     LV_LAUNCHED();
@@ -938,6 +944,15 @@ int32_t launch_modularity(Handle& h, Level& L, const int32_t* d_C) {
   return LOUVAIN_OK;
 }
 
+// Delta pass iff moved entries <= nnz / LV_DELTA_DIV.  Default 1 (always; the
+// commit then skips the moved-degree sum): measured faster than the full pass on
+// every config even at 84% moved entries (DESIGN 13); LV_DELTA_DIV=1000000 forces
+// the full pass.
+unsigned long long delta_div() {
+  static const unsigned long long d = getenv("LV_DELTA_DIV") ? strtoull(getenv("LV_DELTA_DIV"), nullptr, 10) : 1ull;
+  return d;
+}
+
 int32_t launch_snapshot(Handle& h, Level& L) {
   if (L.n == 0) return LOUVAIN_OK;
   k_snapshot<<<grid_for(L.n, 256), 256, 0, h.stream>>>(L.C, L.n, h.pcn);
@@ -951,11 +966,7 @@ int32_t launch_modularity_delta(Handle& h, Level& L) {
   cudaStream_t s = h.stream;
   LV_CUDA(cudaMemsetAsync(&h.ctl->L, 0, 16, s));
   LV_CUDA(cudaMemsetAsync(&h.ctl->dL, 0, 24, s));
-  // moved entries <= nnz / ddiv: delta pass.  Default 1 (always): measured faster
-  // than the full pass on every config even at 84% moved entries (DESIGN 13);
-  // LV_DELTA_DIV=1000000 forces the full pass
-  static const unsigned long long ddiv = getenv("LV_DELTA_DIV") ? strtoull(getenv("LV_DELTA_DIV"), nullptr, 10) : 1ull;
-  LV_TRY(set_ctl_u64(h, &h.ctl->ddiv, ddiv));
+  LV_TRY(set_ctl_u64(h, &h.ctl->ddiv, delta_div()));
   if (L.n == 0) return LOUVAIN_OK;
   int32_t *big = nullptr, *mid = nullptr;
   LV_TRY(dalloc(&big, (size_t)(L.nnz / kDeltaBigDeg + 1), s));
@@ -983,9 +994,9 @@ int32_t launch_modularity_delta(Handle& h, Level& L) {
   return LOUVAIN_OK;
 }
 
-int32_t level_modularity(Handle& h, Level& L, const int32_t* d_C, uint64_t* Lout, uint64_t* Sout) {
+int32_t level_modularity(Handle& h, Level& L, const int32_t* d_C, uint64_t* Lout, uint64_t* Sout, bool singletons) {
   LV_CUDA(cudaMemsetAsync(&h.ctl->bad, 0, 8, h.stream));
-  LV_TRY(launch_modularity(h, L, d_C));
+  LV_TRY(launch_modularity(h, L, d_C, singletons));
   LV_CUDA(cudaMemcpyAsync(h.h_ctl, h.ctl, sizeof(DevCtl), cudaMemcpyDeviceToHost, h.stream));
   LV_CUDA(cudaStreamSynchronize(h.stream));
   if (h.h_ctl->bad) {
@@ -999,7 +1010,7 @@ int32_t level_modularity(Handle& h, Level& L, const int32_t* d_C, uint64_t* Lout
 
 int32_t launch_commit(Handle& h, Level& L, int bucket) {
   k_commit<<<148 * 4, 256, 0, h.stream>>>(h.ctl, bucket, L.mv_v, L.mv_new, L.mv_old, L.ca, L.size, L.k, L.C,
-                                         L.rowptr, h.pcn);
+                                         (h.pcn && delta_div() > 1) ? L.rowptr : nullptr, h.pcn);
   LV_LAUNCHED();
   LV_CUDA(cudaGetLastError());
   return LOUVAIN_OK;
