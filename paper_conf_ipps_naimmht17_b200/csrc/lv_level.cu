@@ -93,8 +93,12 @@ __global__ void k_classify(const int64_t* rowptr, int64_t n, int64_t b0, int64_t
   __shared__ unsigned long long sh[kNumClasses];
   if (threadIdx.x < kNumClasses) sh[threadIdx.x] = 0;
   __syncthreads();
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t d = rowptr[i + 1] - rowptr[i];  // R11: row length incl. self-loop
+  // uniform trip count per warp so the class counts can be merged with __match_any_sync
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  for (int64_t i0 = blockIdx.x * (int64_t)blockDim.x + (threadIdx.x & ~31); i0 < n; i0 += stride) {
+    const int64_t i = i0 + (threadIdx.x & 31);
+    const bool has = i < n;
+    const int64_t d = has ? rowptr[i + 1] - rowptr[i] : 0;  // R11: row length incl. self-loop
     int b;
     if (d == 0 || i < lo || i >= hi) b = 0;  // not decided here (no edges, or owned by another rank)
     else if (d <= b0) b = 1;
@@ -106,9 +110,12 @@ __global__ void k_classify(const int64_t* rowptr, int64_t n, int64_t b0, int64_t
     else b = 7;
     const int sub = sub_of_degree(d);
     const uint8_t c = (uint8_t)(kSubPerBucket * b + sub);
-    cls[i] = c;
-    iota[i] = (int32_t)i;
-    atomicAdd(&sh[c], 1ull);
+    if (has) {
+      cls[i] = c;
+      iota[i] = (int32_t)i;
+    }
+    const unsigned m = __match_any_sync(0xffffffffu, has ? (int)c : -1);  // one smem atomic per class per warp
+    if (has && (threadIdx.x & 31) == __ffs(m) - 1) atomicAdd(&sh[c], (unsigned long long)__popc(m));
   }
   __syncthreads();
   if (threadIdx.x < kNumClasses && sh[threadIdx.x]) atomicAdd(&hist[threadIdx.x], sh[threadIdx.x]);
