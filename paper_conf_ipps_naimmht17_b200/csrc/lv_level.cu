@@ -314,7 +314,17 @@ __global__ void __launch_bounds__(256) k_mod_delta_thr(DevCtl* ctl, const int32_
       mid[atomicAdd(&ctl->nmid, 1ull)] = (int32_t)p;
     } else {
       const int32_t t = mv_new[p], o = mv_old[p];
-      for (int64_t q = b; q < e; ++q) acc += delta_entry(P, i, __ldcs(&col[q]), w ? __ldcs(&w[q]) : 1u, t, o);
+      for (int64_t q = b; q < e; q += 4) {  // 4 independent gathers in flight
+        int32_t j[4];
+        uint32_t x[4];
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          j[u] = q + u < e ? __ldcs(&col[q + u]) : i;  // j = i contributes 0 without a gather
+          x[u] = (w && q + u < e) ? __ldcs(&w[q + u]) : 1u;
+        }
+#pragma unroll
+        for (int u = 0; u < 4; ++u) acc += delta_entry(P, i, j[u], x[u], t, o);
+      }
     }
   }
   const unsigned long long s = warp_sum_u64((unsigned long long)acc);
@@ -338,8 +348,12 @@ __global__ void __launch_bounds__(256) k_mod_delta_warp(DevCtl* ctl, const int32
     const int32_t p = mid[k];
     const int32_t i = mv_v[p], t = mv_new[p], o = mv_old[p];
     const int64_t b = rowptr[i], e = rowptr[i + 1];
-    for (int64_t q = b + lane; q < e; q += 32)
-      acc += delta_entry(P, i, __ldcs(&col[q]), w ? __ldcs(&w[q]) : 1u, t, o);
+    for (int64_t q = b + lane; q < e; q += 64) {  // 2 independent gathers in flight per lane
+      const bool has1 = q + 32 < e;
+      const int32_t j0 = __ldcs(&col[q]), j1 = has1 ? __ldcs(&col[q + 32]) : i;
+      const uint32_t x0 = w ? __ldcs(&w[q]) : 1u, x1 = (w && has1) ? __ldcs(&w[q + 32]) : 1u;
+      acc += delta_entry(P, i, j0, x0, t, o) + delta_entry(P, i, j1, x1, t, o);
+    }
   }
   const unsigned long long s = warp_sum_u64((unsigned long long)acc);
   if (lane == 0 && s) atomicAdd(&ctl->dL, s);
