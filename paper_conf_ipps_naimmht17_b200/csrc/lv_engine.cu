@@ -523,10 +523,15 @@ int32_t run_impl(Handle& h, const louvain_params_t& p, int32_t* labels_out, louv
       cur = &owned;
     }
   }
-  if (cur != &L0) level_free(owned, s);
   // the handle's partition becomes the final one; (Lq, Sq) are the exact parts of
   // the last level's kept partition, equal to those of `lab` on the input graph
-  LV_TRY(level_set_labels(h, L0, lab));
+  bool final_set = false;
+  if (cur != &L0 && owned.n <= kFinalHistMax) {  // totals from the last level, sizes by an smem histogram
+    LV_TRY(level_set_final(h, L0, lab, owned.ca, owned.n));
+    final_set = true;
+  }
+  if (cur != &L0) level_free(owned, s);
+  if (!final_set) LV_TRY(level_set_labels(h, L0, lab));
   LV_TRY(copy_out(labels_out, lab, sizeof(int32_t) * (size_t)n0, s));
   LV_CUDA(cudaStreamSynchronize(s));
   dfree(lab, s);

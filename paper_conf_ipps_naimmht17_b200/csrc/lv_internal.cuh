@@ -265,6 +265,9 @@ int32_t level_alloc_scratch(Handle& h, Level& L, int parity);  // state arrays f
 void level_free(Level& L, cudaStream_t s);
 int32_t level_setup(Handle& h, Level& L);  // k, W, singleton partition (Alg. 1 l.2)
 int32_t level_set_labels(Handle& h, Level& L, const int32_t* d_labels);  // C given (nullptr = iota), recompute a/size
+// end of louvain_run: labels in [0, n_last) of the last level (state ca_last); n_last <= kFinalHistMax
+constexpr int64_t kFinalHistMax = 49152;  // size histogram in shared memory (4 B per label)
+int32_t level_set_final(Handle& h, Level& L, const int32_t* d_labels, const uint2* ca_last, int64_t n_last);
 int32_t level_get_labels(Handle& h, Level& L, int32_t* d_out);          // C -> d_out (device)
 int32_t level_get_a(Handle& h, Level& L, uint32_t* d_out);              // a -> d_out (device)
 int32_t level_binning(Handle& h, Level& L, const louvain_params_t& p);  // classes + hub plan

@@ -643,6 +643,46 @@ int32_t level_set_labels(Handle& h, Level& L, const int32_t* d_labels) {
   return LOUVAIN_OK;
 }
 
+// Final partition of a run on the input level (labels in the last level's id
+// space [0, n_last)): a_c is the last level's total of c (contraction preserves
+// totals, R18) and size_c counts the input vertices labelled c -- one shared-memory
+// histogram per CTA instead of global atomics on a few giant communities.
+__global__ void k_copy_a(const uint2* __restrict__ ca_last, int64_t n_last, uint2* ca) {
+  for (int64_t c = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; c < n_last; c += (int64_t)gridDim.x * blockDim.x)
+    ca[c].y = ca_last[c].y;
+}
+__global__ void __launch_bounds__(1024) k_size_hist(const int32_t* __restrict__ lab, int64_t n, int nl, int32_t* size) {
+  extern __shared__ int32_t hs[];
+  for (int c = threadIdx.x; c < nl; c += blockDim.x) hs[c] = 0;
+  __syncthreads();
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  for (int64_t i0 = blockIdx.x * (int64_t)blockDim.x + (threadIdx.x & ~31); i0 < n; i0 += stride) {
+    const int64_t i = i0 + (threadIdx.x & 31);
+    const int32_t c = i < n ? lab[i] : -1;
+    const unsigned m = __match_any_sync(0xffffffffu, c);
+    if (c >= 0 && (threadIdx.x & 31) == __ffs(m) - 1) atomicAdd(&hs[c], __popc(m));
+  }
+  __syncthreads();
+  for (int c = threadIdx.x; c < nl; c += blockDim.x)
+    if (hs[c]) atomicAdd(&size[c], hs[c]);
+}
+
+int32_t level_set_final(Handle& h, Level& L, const int32_t* d_labels, const uint2* ca_last, int64_t n_last) {
+  cudaStream_t s = h.stream;
+  L.sweeps_done = 1;
+  if (L.n == 0) return LOUVAIN_OK;
+  k_set_C<<<grid_for(L.n, 256), 256, 0, s>>>(d_labels, L.n, L.ca, L.size, L.C);
+  LV_LAUNCHED();
+  k_copy_a<<<grid_for(n_last, 256), 256, 0, s>>>(ca_last, n_last, L.ca);
+  LV_LAUNCHED();
+  const int smem = (int)(4 * n_last);
+  LV_CUDA(cudaFuncSetAttribute(k_size_hist, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+  k_size_hist<<<148, 1024, smem, s>>>(d_labels, L.n, (int)n_last, L.size);
+  LV_LAUNCHED();
+  LV_CUDA(cudaGetLastError());
+  return LOUVAIN_OK;
+}
+
 int32_t level_get_labels(Handle& h, Level& L, int32_t* d_out) {
   if (L.n == 0) return LOUVAIN_OK;
   k_get_C<<<grid_for(L.n, 256), 256, 0, h.stream>>>(L.ca, L.n, d_out);

@@ -163,6 +163,10 @@ def test_full_run_bit_exact(name):
     assert (int(q.L), q.S, int(q.W)) == (r.L, r.S, r.W)
     assert abs(q.q - r.q) <= 1e-9 * max(1.0, abs(r.q))
     assert np.array_equal(gd.labels(), r.labels)  # handle keeps the final partition
+    a, size = gd.totals()  # ... with its exact a_c and size_c (R12)
+    a_o, size_o = oracle.totals(g, r.labels)
+    assert np.array_equal(a.astype(np.uint64), np.asarray(a_o, dtype=np.uint64))
+    assert np.array_equal(size.astype(np.int64), np.asarray(size_o, dtype=np.int64))
 
 
 def test_karate_quality_bar():
@@ -193,6 +197,22 @@ def test_full_run_threshold_grid(name, tb, tf, rev):
     assert st["sweeps_per_level"] == r.sweeps_per_level
     assert st["num_start"] == r.num_start and st["num_end"] == r.num_end
     assert np.array_equal(lab, r.labels)
+
+
+@pytest.mark.parametrize("name", ["rmat15", "hubs", "lfr5k"])
+@pytest.mark.parametrize("max_levels", [1, 2])
+def test_level_cap_final_totals(name, max_levels):
+    """A run cut by max_levels ends on a freshly contracted level (labels = its vertex ids);
+    the handle's final partition and totals must still be the oracle's."""
+    g = GRAPHS[name]()
+    r = oracle.louvain(g, oracle.params(max_levels=max_levels))
+    gd = dev_graph(g)
+    lab, q, st = gd.run(lvb.params(max_levels=max_levels))
+    assert np.array_equal(lab, r.labels) and st["sweeps_per_level"] == r.sweeps_per_level
+    a, size = gd.totals()
+    a_o, size_o = oracle.totals(g, r.labels)
+    assert np.array_equal(a.astype(np.uint64), np.asarray(a_o, dtype=np.uint64))
+    assert np.array_equal(size.astype(np.int64), np.asarray(size_o, dtype=np.int64))
 
 
 def test_size_limit_schedule():
