@@ -467,8 +467,9 @@ int32_t run_impl(Handle& h, const louvain_params_t& p, int32_t* labels_out, louv
         const uint64_t L_after = (mod_delta && delta_chosen(*h.h_ctl, L.nnz)) ? Lq + h.h_ctl->dL : h.h_ctl->L;
         const int64_t num = qnum_of(L_after, h.h_ctl->S, W);
         if (tr.on)
-          fprintf(stderr, "[lv] level %d sweep %d: moved %llu, moved entries %.4f of nnz, %s pass\n", level, sweeps,
-                  h.h_ctl->logn, L.nnz ? (double)h.h_ctl->mdeg / (double)L.nnz : 0.0,
+          fprintf(stderr, "[lv] level %d sweep %d: moved %llu, moved entries %s%.4f of nnz, %s pass\n", level, sweeps,
+                  h.h_ctl->logn, delta_div() > 1 ? "" : "(not summed, gate off) ",
+                  L.nnz ? (double)h.h_ctl->mdeg / (double)L.nnz : 0.0,
                   (mod_delta && delta_chosen(*h.h_ctl, L.nnz)) ? "delta" : "full");
         if (p.revert_on_decrease && num < num_prev) {  // R15
           LV_TRY(launch_revert(h, L));

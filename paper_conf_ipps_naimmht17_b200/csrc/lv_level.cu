@@ -270,7 +270,7 @@ __global__ void __launch_bounds__(256) k_modularity(const int64_t* rowptr, int64
 }
 
 // Delta pass of Eq. (1) after a sweep (used by louvain_run when the moved vertices
-// hold <= nnz/4 entries).  L = sum over directed entries (u->v) of w [C(u) == C(v)]
+// hold <= nnz/LV_DELTA_DIV entries; default: always).  L = sum over directed entries (u->v) of w [C(u) == C(v)]
 // (self-loops once, R2) changes only on entries with a moved endpoint.  For a moved
 // i (old label o, new t) and each entry (i->j), j != i:
 //   d = [C'(j) == t] - [C(j) == o]     (C = labels at the sweep start, C' = after)
