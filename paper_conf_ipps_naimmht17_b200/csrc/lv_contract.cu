@@ -95,79 +95,7 @@ __global__ void k_seg_bounds(const int64_t* rfirst, const int64_t* gpos, int64_t
   if (threadIdx.x < kSegClasses && sh[threadIdx.x]) atomicAdd(&hist[threadIdx.x], sh[threadIdx.x]);
 }
 
-// Step 3: grouped[t] = (map[col[e]], w[e]) for the t-th grouped entry.
-__global__ void __launch_bounds__(256) k_group_copy(const int32_t* __restrict__ vorder,
-                                                    const int64_t* __restrict__ gpos, int64_t n,
-                                                    const int64_t* __restrict__ rowptr,
-                                                    const int32_t* __restrict__ col, const uint32_t* __restrict__ w,
-                                                    const int32_t* __restrict__ map, const int64_t* __restrict__ tr,
-                                                    int32_t* gc, uint32_t* gw) {
-  __shared__ int64_t sh_g[kCRows + 1];
-  __shared__ int64_t sh_rb[kCRows];
-  __shared__ int64_t sh_i0;
-  __shared__ int sh_nr;
-  const int64_t total = gpos[n];
-  const int64_t ntiles = (total + kCTile - 1) / kCTile;
-  for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
-    const int64_t t0 = tile * kCTile, t1 = min(total, t0 + kCTile);
-    if (threadIdx.x == 0) {  // tile plan (tile_starts)
-      const int64_t i0 = tr[tile], i1 = tr[tile + 1];
-      sh_i0 = i0;
-      sh_nr = (i1 - i0 + 1 <= kCRows) ? (int)(i1 - i0 + 1) : -1;
-    }
-    __syncthreads();
-    const int64_t i0 = sh_i0;
-    const int nr = sh_nr;
-    for (int r = threadIdx.x; r < nr; r += blockDim.x) {
-      sh_g[r] = gpos[i0 + r];
-      sh_rb[r] = rowptr[vorder[i0 + r]];
-    }
-    __syncthreads();
-    for (int64_t base = t0 + threadIdx.x; base < t1; base += 4 * (int64_t)blockDim.x) {
-      int32_t jj[4];
-      int64_t ee[4];
-#pragma unroll
-      for (int q = 0; q < 4; ++q) {
-        const int64_t t = base + (int64_t)q * blockDim.x;
-        jj[q] = -1;
-        ee[q] = 0;
-        if (t < t1) {
-          if (nr > 0) {
-            int lo = 0, hi = nr - 1;
-            while (lo < hi) {
-              const int mid = (lo + hi + 1) >> 1;
-              if (sh_g[mid] <= t) lo = mid; else hi = mid - 1;
-            }
-            ee[q] = sh_rb[lo] + (t - sh_g[lo]);
-          } else {
-            int64_t lo = 0, hi = n - 1;
-            while (lo < hi) {
-              const int64_t mid = (lo + hi + 1) >> 1;
-              if (gpos[mid] <= t) lo = mid; else hi = mid - 1;
-            }
-            ee[q] = rowptr[vorder[lo]] + (t - gpos[lo]);
-          }
-          jj[q] = __ldcs(&col[ee[q]]);
-        }
-      }
-      int32_t mm[4];
-#pragma unroll
-      for (int q = 0; q < 4; ++q) mm[q] = jj[q] >= 0 ? __ldg(&map[jj[q]]) : 0;
-#pragma unroll
-      for (int q = 0; q < 4; ++q) {
-        const int64_t t = base + (int64_t)q * blockDim.x;
-        if (t < t1) {  // evict-first: streamed once, must not displace map[] in L2
-          __stcs(&gc[t], mm[q]);
-          if (gw) __stcs(&gw[t], w ? __ldcs(&w[ee[q]]) : 1u);
-        }
-      }
-    }
-    __syncthreads();
-  }
-}
-
-
-// Step 3 (default): the same copy in source order -- rows read sequentially, each
+// Step 3: every member row copied in source order -- rows read sequentially, each
 // row's entries written to its member's slot of the grouped layout (dbase[u] =
 // gpos[rank of u]); the only random access per entry is the map[col] gather.
 __global__ void k_dest_base(const int32_t* __restrict__ vorder, const int64_t* __restrict__ gpos, int64_t n,
@@ -376,30 +304,6 @@ __global__ void __launch_bounds__(512) k_merge_mid(const int32_t* __restrict__ r
 }
 
 
-// Batched 32-bit variant (default when n' < 2^31): the big segments are cut into
-// batches of at most 2^(32 - nb) segments and kBigBatchEntries entries (a larger
-// segment is a batch of its own); each batch is sorted with 32-bit keys
-// (local segment << nb | neighbour) -- 8 instead of 12 bytes per element and
-// pass, and small batches stay L2-resident -- then reduced and placed.  The run
-// count stays on the device (no host round trip per batch).
-constexpr int64_t kBigBatchEntries = 4 << 20;
-__global__ void k_big_keys32(const int32_t* __restrict__ rows, int64_t nseg, const int64_t* __restrict__ boff,
-                             int64_t base, int64_t m, const int64_t* __restrict__ sstart,
-                             const int32_t* __restrict__ gc, const uint32_t* __restrict__ gw, int nb, uint32_t* keys,
-                             uint32_t* vals) {
-  for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < m; t += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t g = base + t;
-    int64_t lo = 0, hi = nseg - 1;  // largest k with boff[k] <= g
-    while (lo < hi) {
-      const int64_t mid = (lo + hi + 1) >> 1;
-      if (boff[mid] <= g) lo = mid; else hi = mid - 1;
-    }
-    const int64_t src = sstart[rows[lo]] + (g - boff[lo]);
-    keys[t] = ((uint32_t)lo << nb) | (uint32_t)gc[src];
-    vals[t] = gw ? __ldcs(&gw[src]) : 1u;
-  }
-}
-
 __global__ void k_big_place32(const uint32_t* __restrict__ ukeys, const uint32_t* __restrict__ sums,
                               const int64_t* __restrict__ dnum, int nb, const int32_t* __restrict__ rows,
                               const int64_t* __restrict__ sstart, int32_t* oc, uint32_t* ow, int64_t* cnt) {
@@ -458,23 +362,11 @@ __global__ void k_big_place(const unsigned long long* __restrict__ ukeys, const 
 constexpr int kCombSlots = 16384;
 constexpr int kCombChunk = 65536;
 constexpr int kCombProbes = 32;
-// keys == nullptr: fused with the key build -- entry e of the concatenated big
-// segments is read straight from the grouped copy (segment by binary search over
-// boff, few segments when keys are 32-bit), key = segment << nb | neighbour.
-struct BigSrc {
-  const int32_t* rows;
-  int64_t nbig;
-  const int64_t* sstart;
-  const int64_t* boff;
-  const int32_t* gc;
-  const uint32_t* gw;
-  int nb;
-};
 template <int SLOTS, int BITS, int CHUNK, int THREADS>
 __global__ void __launch_bounds__(THREADS) k_big_combine(const uint32_t* __restrict__ keys,
                                                          const uint32_t* __restrict__ vals, int64_t m,
                                                          uint32_t* __restrict__ okeys, uint32_t* __restrict__ ovals,
-                                                         unsigned long long* ocount, BigSrc src) {
+                                                         unsigned long long* ocount) {
   extern __shared__ unsigned long long T[];  // SLOTS
   __shared__ unsigned wcnt[32];
   __shared__ unsigned long long sh_base;
@@ -494,19 +386,8 @@ __global__ void __launch_bounds__(THREADS) k_big_combine(const uint32_t* __restr
         k[q] = 0xFFFFFFFFu;
         v[q] = 0;
         if (e < e1) {
-          if (keys) {
-            k[q] = __ldcs(&keys[e]);
-            v[q] = __ldcs(&vals[e]);
-          } else {
-            int64_t lo = 0, hi = src.nbig - 1;  // largest segment with boff <= e
-            while (lo < hi) {
-              const int64_t mid = (lo + hi + 1) >> 1;
-              if (__ldg(&src.boff[mid]) <= e) lo = mid; else hi = mid - 1;
-            }
-            const int64_t at = __ldg(&src.sstart[__ldg(&src.rows[lo])]) + (e - __ldg(&src.boff[lo]));
-            k[q] = ((uint32_t)lo << src.nb) | (uint32_t)__ldcs(&src.gc[at]);
-            v[q] = src.gw ? __ldcs(&src.gw[at]) : 1u;
-          }
+          k[q] = __ldcs(&keys[e]);
+          v[q] = __ldcs(&vals[e]);
         }
       }
 #pragma unroll
@@ -584,57 +465,6 @@ __global__ void __launch_bounds__(THREADS) k_big_combine(const uint32_t* __restr
   }
 }
 
-// Segmented variant of the big-segment merge (when segment + neighbour bits pass
-// 32): each big segment's neighbours are sorted on their own (CUB segmented radix
-// sort over the nb neighbour bits: 4-byte keys, ceil(nb/8) passes instead of the
-// flat 64-bit sort's 5 passes of 12 bytes), then runs are cut at segment starts
-// and key changes, numbered by a scan and summed by reduce-by-key.
-__global__ void k_seg_mark(const int64_t* __restrict__ boff, int64_t nbig, uint32_t* heads) {
-  for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < nbig; k += (int64_t)gridDim.x * blockDim.x)
-    heads[boff[k]] = 1u;
-}
-__global__ void k_seg_heads(const uint32_t* __restrict__ keys, int64_t m, uint32_t* heads) {
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < m; i += (int64_t)gridDim.x * blockDim.x)
-    heads[i] = (i == 0 || heads[i] != 0u || keys[i] != keys[i - 1]) ? 1u : 0u;
-}
-__global__ void k_seg_place(const uint32_t* __restrict__ keys, const uint32_t* __restrict__ runid,
-                            const uint32_t* __restrict__ sums, int64_t m, const int64_t* __restrict__ boff,
-                            int64_t nbig, const int32_t* __restrict__ rows, const int64_t* __restrict__ sstart,
-                            int32_t* oc, uint32_t* ow, int64_t* cnt) {
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < m; i += (int64_t)gridDim.x * blockDim.x) {
-    const uint32_t r = runid[i];
-    if (i > 0 && runid[i - 1] == r) continue;  // not the head of its run
-    int64_t lo = 0, hi = nbig - 1;  // segment of i: largest k with boff[k] <= i
-    while (lo < hi) {
-      const int64_t mid = (lo + hi + 1) >> 1;
-      if (boff[mid] <= i) lo = mid; else hi = mid - 1;
-    }
-    const uint32_t r0 = runid[boff[lo]];
-    const int64_t local = (int64_t)(r - r0);
-    const int32_t row = rows[lo];
-    oc[sstart[row] + local] = (int32_t)keys[i];
-    ow[sstart[row] + local] = sums[r - 1];
-    if (i + 1 == boff[lo + 1] || runid[boff[lo + 1] - 1] == r) cnt[row] = local + 1;
-  }
-}
-
-// Views of packed (segment, neighbour, weight) keys for reduce-by-key.
-struct KeyHi {
-  int s;
-  __host__ __device__ unsigned long long operator()(unsigned long long x) const { return x >> s; }
-};
-struct KeyLo {
-  unsigned long long mask;
-  __host__ __device__ uint32_t operator()(unsigned long long x) const { return (uint32_t)(x & mask); }
-};
-__global__ void k_max_u32(const uint32_t* x, int64_t n, unsigned* out) {
-  unsigned mx = 0;
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
-    mx = max(mx, __ldcs(&x[i]));
-  for (int o = 16; o >= 1; o >>= 1) mx = max(mx, __shfl_xor_sync(kFull, mx, o));
-  if ((threadIdx.x & 31) == 0 && mx) atomicMax(out, mx);
-}
-
 // Lengths of the big segments (the scan turns them into key-array offsets).
 __global__ void k_big_len(const int32_t* __restrict__ rows, int64_t nbig, const int64_t* __restrict__ sstart,
                           int64_t* len) {
@@ -695,336 +525,6 @@ __global__ void __launch_bounds__(256) k_big_keys_t(const int32_t* __restrict__ 
       }
     }
   }
-}
-
-// Step 4d (LV_BIG_PART=1): big segments merged by label partitioning.  Segment k gets
-// P_k = ceil(min(len, n') / kCPartLabels) partitions (part_of(label, P_k)); its
-// entries are scattered into partition order (histogram -> per-segment scan ->
-// scatter, in chunks), then one CTA per (segment, partition) sums its share in a
-// shared-memory table and appends the distinct (neighbour, weight) pairs to the
-// segment's output (warp-aggregated cursor cnt[row]).  A table passing 7/8 load
-// sets a flag and the host redoes the big segments with the radix sort.
-constexpr int64_t kCPartLabels = 4096;  // expected distinct labels per partition (load <= 1/4)
-constexpr int kCPartSlots = 16384;      // 8-byte slots per partition table (128 KB)
-constexpr int kCPartMaxP = 4096;
-constexpr int64_t kCPartChunk = 32768;
-struct CSeg {
-  int64_t src;    // segment start in gc/gw (== its output start in oc/ow)
-  int64_t pbase;  // first poff index (sum of P + 1 of earlier segments)
-  int32_t row;
-  int32_t P;
-  int32_t first;  // first task / cursor index
-  int32_t pad;
-};
-struct CChunk {
-  int32_t seg;
-  int32_t pad;
-  int64_t begin, end;
-};
-struct CTask {
-  int32_t seg;
-  int32_t p;
-};
-
-__global__ void __launch_bounds__(1024) k_cpart_hist(const CChunk* __restrict__ chunks, int64_t nch,
-                                                     const CSeg* __restrict__ segs, const int32_t* __restrict__ gc,
-                                                     int64_t* poff) {
-  __shared__ uint32_t hist[kCPartMaxP];
-  const int lane = threadIdx.x & 31;
-  for (int64_t ci = blockIdx.x; ci < nch; ci += gridDim.x) {
-    const CChunk ch = chunks[ci];
-    const CSeg sg = segs[ch.seg];
-    const uint32_t P = (uint32_t)sg.P;
-    for (uint32_t q = threadIdx.x; q < P; q += blockDim.x) hist[q] = 0;
-    __syncthreads();
-    for (int64_t t0 = ch.begin + (threadIdx.x - lane); t0 < ch.end; t0 += blockDim.x) {
-      const int64_t t = t0 + lane;
-      const uint32_t q = (t < ch.end) ? part_of(__ldcs(&gc[sg.src + t]), P) : 0xFFFFFFFFu;
-      const unsigned m = __match_any_sync(kFull, q);
-      if (q != 0xFFFFFFFFu && lane == __ffs(m) - 1) atomicAdd(&hist[q], (uint32_t)__popc(m));
-    }
-    __syncthreads();
-    for (uint32_t q = threadIdx.x; q < P; q += blockDim.x)
-      if (hist[q]) atomicAdd(reinterpret_cast<unsigned long long*>(&poff[sg.pbase + 1 + q]), (unsigned long long)hist[q]);
-    __syncthreads();
-  }
-}
-
-// warp per segment: counts -> partition starts (relative to the segment) + scatter cursors
-__global__ void k_cpart_scan(const CSeg* __restrict__ segs, int64_t nseg, int64_t* poff, unsigned long long* cur) {
-  const int lane = threadIdx.x & 31;
-  const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
-  for (int64_t k = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); k < nseg; k += warps) {
-    const CSeg sg = segs[k];
-    long long run = 0;
-    for (int32_t q0 = 0; q0 < sg.P; q0 += 32) {
-      const int32_t q = q0 + lane;
-      const long long c = (q < sg.P) ? poff[sg.pbase + 1 + q] : 0;
-      long long x = c;
-#pragma unroll
-      for (int o = 1; o < 32; o <<= 1) {
-        const long long y = __shfl_up_sync(kFull, x, o);
-        if (lane >= o) x += y;
-      }
-      if (q < sg.P) {
-        poff[sg.pbase + q] = run + x - c;
-        cur[sg.first + q] = (unsigned long long)(run + x - c);
-      }
-      run += __shfl_sync(kFull, x, 31);
-    }
-    if (lane == 0) poff[sg.pbase + sg.P] = run;
-  }
-}
-
-__global__ void __launch_bounds__(1024) k_cpart_scatter(const CChunk* __restrict__ chunks, int64_t nch,
-                                                        const CSeg* __restrict__ segs, const int32_t* __restrict__ gc,
-                                                        const uint32_t* __restrict__ gw, unsigned long long* cur,
-                                                        uint2* P2) {
-  __shared__ uint32_t hist[kCPartMaxP];
-  constexpr uint32_t kSeg = 1024;
-  __shared__ unsigned long long base[kSeg];
-  const int lane = threadIdx.x & 31;
-  for (int64_t ci = blockIdx.x; ci < nch; ci += gridDim.x) {
-    const CChunk ch = chunks[ci];
-    const CSeg sg = segs[ch.seg];
-    const uint32_t P = (uint32_t)sg.P;
-    for (uint32_t q = threadIdx.x; q < P; q += blockDim.x) hist[q] = 0;
-    __syncthreads();
-    for (int64_t t0 = ch.begin + (threadIdx.x - lane); t0 < ch.end; t0 += blockDim.x) {
-      const int64_t t = t0 + lane;
-      const uint32_t q = (t < ch.end) ? part_of(__ldcs(&gc[sg.src + t]), P) : 0xFFFFFFFFu;
-      const unsigned m = __match_any_sync(kFull, q);
-      if (q != 0xFFFFFFFFu && lane == __ffs(m) - 1) atomicAdd(&hist[q], (uint32_t)__popc(m));
-    }
-    __syncthreads();
-    for (uint32_t h0 = 0; h0 < P; h0 += kSeg) {
-      const uint32_t h1 = min(P, h0 + kSeg);
-      for (uint32_t q = h0 + threadIdx.x; q < h1; q += blockDim.x)
-        base[q - h0] = hist[q] ? atomicAdd(&cur[sg.first + q], (unsigned long long)hist[q]) : 0ull;
-      __syncthreads();
-      for (int64_t t0 = ch.begin + (threadIdx.x - lane); t0 < ch.end; t0 += blockDim.x) {
-        const int64_t t = t0 + lane;
-        int32_t c = 0;
-        uint32_t q = 0xFFFFFFFFu;
-        if (t < ch.end) {
-          c = __ldcs(&gc[sg.src + t]);
-          q = part_of(c, P);
-          if (q < h0 || q >= h1) q = 0xFFFFFFFFu;
-        }
-        const unsigned m = __match_any_sync(kFull, q);
-        unsigned long long b = 0;
-        const int leader = __ffs(m) - 1;
-        if (q != 0xFFFFFFFFu && lane == leader) b = atomicAdd(&base[q - h0], (unsigned long long)__popc(m));
-        b = __shfl_sync(m, b, leader);
-        if (q != 0xFFFFFFFFu) {
-          const unsigned long long dst = sg.src + b + __popc(m & ((1u << lane) - 1u));
-          __stcs(&P2[dst], make_uint2((uint32_t)c, gw ? __ldcs(&gw[sg.src + t]) : 1u));
-        }
-      }
-      __syncthreads();
-    }
-  }
-}
-
-// Task (segment, partition): insert the partition's entries into the smem table
-// (2 * n_p slots: no overflow possible; kCPartSlots with a distinct-label count
-// when n_p is larger), append the distinct (neighbour, weight) pairs to the
-// segment's output (warp-aggregated cursor cnt[row]), clearing the table.
-__global__ void __launch_bounds__(1024) k_cpart_merge(const CTask* __restrict__ tasks, int64_t ntasks,
-                                                      const CSeg* __restrict__ segs, const int64_t* __restrict__ poff,
-                                                      const uint2* __restrict__ P2, int32_t* oc, uint32_t* ow,
-                                                      int64_t* cnt, unsigned long long* overflow) {
-  extern __shared__ unsigned long long T[];  // kCPartSlots
-  __shared__ unsigned claimed;
-  for (int t = threadIdx.x; t < kCPartSlots; t += blockDim.x) T[t] = kEmpty;
-  if (threadIdx.x == 0) claimed = 0;
-  __syncthreads();
-  const int lane = threadIdx.x & 31;
-  const unsigned limit = (unsigned)(kCPartSlots / 8 * 7);
-  for (int64_t k = blockIdx.x; k < ntasks; k += gridDim.x) {
-    const CTask tk = tasks[k];
-    const CSeg sg = segs[tk.seg];
-    const int64_t q0 = sg.src + poff[sg.pbase + tk.p], q1 = sg.src + poff[sg.pbase + tk.p + 1];
-    const int64_t n_p = q1 - q0;
-    const bool big = 2 * n_p > kCPartSlots;
-    const uint32_t cap = big ? (uint32_t)kCPartSlots : (uint32_t)(n_p > 0 ? 2 * n_p : 1);
-    unsigned claims = 0;
-    // warp-uniform trips; equal labels of a warp summed first (hot labels: one atomic per warp)
-    for (int64_t base = q0 + (threadIdx.x - lane); base < q1; base += 4 * (int64_t)blockDim.x) {
-      uint2 rr[4];
-#pragma unroll
-      for (int u = 0; u < 4; ++u) {
-        const int64_t t = base + lane + (int64_t)u * blockDim.x;
-        rr[u] = (t < q1) ? __ldcs(&P2[t]) : make_uint2(0xFFFFFFFFu, 0u);
-      }
-#pragma unroll
-      for (int u = 0; u < 4; ++u) {
-        const unsigned m = __match_any_sync(kFull, rr[u].x);
-        const uint32_t sum = __reduce_add_sync(m, rr[u].y);
-        bool cl = false;
-        if (rr[u].x != 0xFFFFFFFFu && lane == __ffs(m) - 1) {
-          const int32_t c = (int32_t)rr[u].x;
-          const unsigned long long key = ((unsigned long long)(uint32_t)c) << 32;
-          uint32_t h = hash_slot(c, cap);
-          for (uint32_t probes = 0; probes < cap; ++probes) {
-            const unsigned long long old = atomicCAS(&T[h], kEmpty, key | sum);
-            if (old == kEmpty) { cl = true; break; }
-            if ((old >> 32) == (unsigned long long)(uint32_t)c) {
-              atomicAdd(&T[h], (unsigned long long)sum);
-              break;
-            }
-            h = (h + 1 == cap) ? 0 : h + 1;
-          }
-        }
-        if (big) claims += __popc(__ballot_sync(kFull, cl));
-      }
-    }
-    if (big && lane == 0 && claims) atomicAdd(&claimed, claims);
-    __syncthreads();
-    if (big && threadIdx.x == 0) {
-      if (claimed > limit) atomicAdd(overflow, 1ull);
-      claimed = 0;
-    }
-    for (uint32_t t0 = 0; t0 < cap; t0 += blockDim.x) {
-      const uint32_t t = t0 + threadIdx.x;
-      const unsigned long long x = (t < cap) ? T[t] : kEmpty;
-      const bool has = x != kEmpty;
-      if (has) T[t] = kEmpty;
-      const unsigned m = __ballot_sync(kFull, has);
-      if (!m) continue;
-      unsigned long long b = 0;
-      const int leader = __ffs(m) - 1;
-      if (lane == leader) b = atomicAdd(reinterpret_cast<unsigned long long*>(&cnt[sg.row]), (unsigned long long)__popc(m));
-      b = __shfl_sync(kFull, b, leader);
-      if (has) {
-        const int64_t pos = sg.src + (int64_t)b + __popc(m & ((1u << lane) - 1u));
-        oc[pos] = (int32_t)(x >> 32);
-        ow[pos] = (uint32_t)x;
-      }
-    }
-    __syncthreads();
-  }
-}
-
-// Step 4d (LV_BIG_HASH=1, experimental): big segments merged in global-memory hash tables kept
-// L2-resident by processing the segments in waves (each wave's tables <= kBigWaveSlots
-// slots).  Table of a segment: cap = 2 * min(len, n') slots (load <= 1/2), split into
-// 4-slot buckets read with two 16-byte loads; a label is claimed at the first
-// empty slot of its probe sequence (one CAS) and summed with atomicAdd afterwards.
-struct BigSeg {
-  int64_t src;   // segment start in gc/gw and in oc/ow
-  int64_t toff;  // table offset in the wave table
-  int64_t cap;   // slots, multiple of 4
-  int32_t row;
-  int32_t pad;
-};
-struct BigItem {
-  int32_t seg;
-  int32_t pad;
-  int64_t begin, end;  // insert: entries [begin, end) of the segment; extract: slots
-};
-constexpr int64_t kBigWaveSlots = 6 << 20;  // 48 MB of 8-byte slots per wave
-constexpr int64_t kBigChunk = 4096;
-
-__device__ __forceinline__ void big_insert4(unsigned long long* T, uint32_t cap, const int32_t c[4],
-                                            const uint32_t x[4], bool todo[4]) {
-  const uint32_t nb = cap >> 2;
-  uint32_t b[4];
-#pragma unroll
-  for (int q = 0; q < 4; ++q) b[q] = todo[q] ? (hash_slot(c[q], nb) << 2) : 0u;
-  while (todo[0] || todo[1] || todo[2] || todo[3]) {
-    unsigned long long k[4][4];
-#pragma unroll
-    for (int q = 0; q < 4; ++q) {
-      if (!todo[q]) continue;
-      const ulonglong2 lo = __ldcg(reinterpret_cast<const ulonglong2*>(&T[b[q]]));
-      const ulonglong2 hi = __ldcg(reinterpret_cast<const ulonglong2*>(&T[b[q] + 2]));
-      k[q][0] = lo.x; k[q][1] = lo.y; k[q][2] = hi.x; k[q][3] = hi.y;
-    }
-#pragma unroll
-    for (int q = 0; q < 4; ++q) {
-      if (!todo[q]) continue;
-      int tgt = -1;
-      bool found = false;
-#pragma unroll
-      for (int u = 3; u >= 0; --u)
-        if (k[q][u] == kEmpty) tgt = u;
-#pragma unroll
-      for (int u = 3; u >= 0; --u)
-        if (k[q][u] != kEmpty && (k[q][u] >> 32) == (unsigned long long)(uint32_t)c[q]) { tgt = u; found = true; }
-      if (tgt < 0) {  // bucket full: next bucket
-        b[q] = (b[q] + 4 >= cap) ? 0u : b[q] + 4;
-        continue;
-      }
-      if (!found) {
-        const unsigned long long old =
-            atomicCAS(&T[b[q] + tgt], kEmpty, (((unsigned long long)(uint32_t)c[q]) << 32) | x[q]);
-        if (old == kEmpty) { todo[q] = false; continue; }
-        if ((old >> 32) != (unsigned long long)(uint32_t)c[q]) continue;  // lost the slot: re-read the bucket
-      }
-      atomicAdd(&T[b[q] + tgt], (unsigned long long)x[q]);
-      todo[q] = false;
-    }
-  }
-}
-
-__global__ void __launch_bounds__(256) k_big_insert(const BigItem* __restrict__ items, int64_t nitems,
-                                                    const BigSeg* __restrict__ segs, const int32_t* __restrict__ gc,
-                                                    const uint32_t* __restrict__ gw, unsigned long long* T) {
-  for (int64_t it = blockIdx.x; it < nitems; it += gridDim.x) {
-    const BigItem item = items[it];
-    const BigSeg sg = segs[item.seg];
-    unsigned long long* Ts = T + sg.toff;
-    for (int64_t base = item.begin + threadIdx.x; base < item.end; base += 4 * (int64_t)blockDim.x) {
-      int32_t c[4];
-      uint32_t x[4];
-      bool todo[4];
-#pragma unroll
-      for (int q = 0; q < 4; ++q) {
-        const int64_t t = base + (int64_t)q * blockDim.x;
-        todo[q] = t < item.end;
-        c[q] = todo[q] ? __ldcs(&gc[sg.src + t]) : 0;
-        x[q] = todo[q] ? (gw ? __ldcs(&gw[sg.src + t]) : 1u) : 0u;
-      }
-      big_insert4(Ts, (uint32_t)sg.cap, c, x, todo);
-    }
-  }
-}
-
-__global__ void __launch_bounds__(256) k_big_extract(const BigItem* __restrict__ items, int64_t nitems,
-                                                     const BigSeg* __restrict__ segs, unsigned long long* T,
-                                                     int32_t* oc, uint32_t* ow, int64_t* cnt) {
-  const int lane = threadIdx.x & 31;
-  for (int64_t it = blockIdx.x; it < nitems; it += gridDim.x) {
-    const BigItem item = items[it];
-    const BigSeg sg = segs[item.seg];
-    unsigned long long* Ts = T + sg.toff;
-    for (int64_t t0 = item.begin + (threadIdx.x - lane); t0 < item.end; t0 += blockDim.x) {  // warp-uniform trips
-      const int64_t t = t0 + lane;
-      unsigned long long x = kEmpty;
-      if (t < item.end) {
-        x = __ldcg(&Ts[t]);
-        if (x != kEmpty) Ts[t] = kEmpty;  // clean for the next wave
-      }
-      const bool has = x != kEmpty;
-      const unsigned m = __ballot_sync(kFull, has);
-      if (!m) continue;
-      unsigned long long base = 0;
-      const int leader = __ffs(m) - 1;
-      if (lane == leader) base = atomicAdd(reinterpret_cast<unsigned long long*>(&cnt[sg.row]), (unsigned long long)__popc(m));
-      base = __shfl_sync(kFull, base, leader);
-      if (has) {
-        const int64_t pos = sg.src + (int64_t)base + __popc(m & ((1u << lane) - 1u));
-        oc[pos] = (int32_t)(x >> 32);
-        ow[pos] = (uint32_t)x;
-      }
-    }
-  }
-}
-
-__global__ void k_fill_empty(unsigned long long* p, int64_t n) {
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
-    p[i] = kEmpty;
 }
 
 // Step 5: compaction into the final CSR, edge-parallel over the output entries
@@ -1189,14 +689,7 @@ int32_t level_contract_fast(Handle& h, Level& L, Level& out, int32_t* d_map, int
       gw = static_cast<uint32_t*>(p0);
     }
   }
-  static const bool grouped_copy = getenv("LV_GROUPED_COPY") && getenv("LV_GROUPED_COPY")[0] == '1';
-  if (grouped_copy) {  // grouped order (reads member rows where they lie)
-    const int64_t* tr = nullptr;
-    LV_TRY(tile_starts(h, gpos, 0, n, 0, nnz, kCTile, &tr));
-    k_group_copy<<<grid_for((nnz + kCTile - 1) / kCTile, 1, 148 * 8), 256, 0, s>>>(vorder, gpos, n, L.rowptr, L.col,
-                                                                                      L.w, d_map, tr, gc, gw);
-    LV_LAUNCHED();
-  } else {  // source order (default)
+  {  // source order
     int64_t* dbase = nullptr;
     LV_TRY(dalloc(&dbase, n, s));
     k_dest_base<<<grid_for(n, 256), 256, 0, s>>>(vorder, gpos, n, dbase);
@@ -1262,8 +755,7 @@ int32_t level_contract_fast(Handle& h, Level& L, Level& out, int32_t* d_map, int
   LV_CUDA(cudaMemsetAsync(cnt, 0, 8 * (np + 1), s));
   // small / warp / mid merges on the side stream, concurrent with the big-segment
   // waves on the main stream (independent segments, disjoint outputs)
-  static const bool serial = getenv("LV_SERIAL") && getenv("LV_SERIAL")[0] == '1';
-  cudaStream_t ms = (serial || tr.on) ? s : h.side;
+  cudaStream_t ms = tr.on ? s : h.side;
   if (ms != s) {
     LV_CUDA(cudaEventRecord(h.ev_fork, s));
     LV_CUDA(cudaStreamWaitEvent(ms, h.ev_fork, 0));
@@ -1309,234 +801,7 @@ int32_t level_contract_fast(Handle& h, Level& L, Level& out, int32_t* d_map, int
     }
   }
   tr.mark(s, "merge-mid");
-  // LV_BIG_HASH=1: L2-wave global hash tables for the big segments (measured slower
-  // than the radix sort on C5: 70/99/240 ms vs 63/69/72 ms at levels 0/1/2 -- atomic
-  // round trips and hot-label contention), kept as an experiment
-  static const bool big_hash = getenv("LV_BIG_HASH") && getenv("LV_BIG_HASH")[0] == '1';
-  // LV_BIG_PART=1: label-partitioned smem merge of the big segments (measured 66/75/114 ms
-  // vs the radix sort's 63/69/72 ms at C5 levels 0/1/2; kept as an option)
-  static const bool big_part = getenv("LV_BIG_PART") && getenv("LV_BIG_PART")[0] == '1';
-  bool big_done = false;
-  if (nbig > 0 && !big_hash && big_part) {
-    const int32_t* brows = rows + nsmall + nwarp + nmid;
-    std::vector<int32_t> hb(nbig);
-    LV_CUDA(cudaMemcpyAsync(hb.data(), brows, 4 * nbig, cudaMemcpyDeviceToHost, s));
-    std::vector<int64_t> hs(np + 1);
-    LV_CUDA(cudaMemcpyAsync(hs.data(), sstart, 8 * (np + 1), cudaMemcpyDeviceToHost, s));
-    LV_CUDA(cudaStreamSynchronize(s));
-    std::vector<CSeg> segs;
-    std::vector<CChunk> chunks;
-    std::vector<CTask> tasks;
-    int64_t pb = 0, big_entries = 0;
-    bool fits = true;
-    std::stable_sort(hb.begin(), hb.end(),  // longest first: one CTA walks a whole segment
-                     [&](int32_t a, int32_t b) { return hs[a + 1] - hs[a] > hs[b + 1] - hs[b]; });
-    for (int64_t k = 0; k < nbig; ++k) {
-      const int32_t r = hb[k];
-      const int64_t len = hs[r + 1] - hs[r];
-      big_entries += len;
-      const int64_t P = (std::min<int64_t>(len, np) + kCPartLabels - 1) / kCPartLabels;
-      if (P > kCPartMaxP) { fits = false; break; }
-      segs.push_back(CSeg{hs[r], pb, r, (int32_t)P, (int32_t)tasks.size(), 0});
-      pb += P + 1;
-      for (int32_t q = 0; q < (int32_t)P; ++q) tasks.push_back(CTask{(int32_t)k, q});
-      for (int64_t e = 0; e < len; e += kCPartChunk) chunks.push_back(CChunk{(int32_t)k, 0, e, std::min(len, e + kCPartChunk)});
-    }
-    if (tr.on)
-      fprintf(stderr, "[lv]    contract segments: small %lld warp %lld mid %lld big %lld (big entries %lld of %lld, "
-              "%zu partition tasks)\n", (long long)nsmall, (long long)nwarp, (long long)nmid, (long long)nbig,
-              (long long)big_entries, (long long)nnz, tasks.size());
-    if (fits) {
-      const int64_t ns = (int64_t)segs.size(), nt = (int64_t)tasks.size(), nc = (int64_t)chunks.size();
-      CSeg* dsegs = nullptr;
-      CChunk* dch = nullptr;
-      CTask* dt = nullptr;
-      int64_t* poff = nullptr;
-      unsigned long long* cur = nullptr;
-      LV_TRY(dalloc(&dsegs, ns, s));
-      LV_TRY(dalloc(&dch, nc, s));
-      LV_TRY(dalloc(&dt, nt, s));
-      LV_TRY(dalloc(&poff, pb, s));
-      LV_TRY(dalloc(&cur, nt, s));
-      LV_CUDA(cudaMemcpyAsync(dsegs, segs.data(), sizeof(CSeg) * ns, cudaMemcpyHostToDevice, s));
-      LV_CUDA(cudaMemcpyAsync(dch, chunks.data(), sizeof(CChunk) * nc, cudaMemcpyHostToDevice, s));
-      LV_CUDA(cudaMemcpyAsync(dt, tasks.data(), sizeof(CTask) * nt, cudaMemcpyHostToDevice, s));
-      LV_CUDA(cudaMemsetAsync(poff, 0, 8 * (size_t)pb, s));
-      LV_CUDA(cudaMemsetAsync(&h.ctl->overflow, 0, 8, s));
-      uint2* P2 = nullptr;
-      {
-        void* p0 = nullptr;
-        LV_TRY(scratch_get(h, SC_STAGE, 8 * (size_t)nnz, &p0));  // the level's stage is dead during contraction
-        P2 = static_cast<uint2*>(p0);
-      }
-      static bool attr = false;
-      if (!attr) {
-        LV_CUDA(cudaFuncSetAttribute(k_cpart_merge, cudaFuncAttributeMaxDynamicSharedMemorySize, 8 * kCPartSlots));
-        attr = true;
-      }
-      k_cpart_hist<<<grid_for(nc, 1, 148 * 2), 1024, 0, s>>>(dch, nc, dsegs, gc, poff);
-      LV_LAUNCHED();
-      k_cpart_scan<<<grid_for(ns, 8, 148 * 4), 256, 0, s>>>(dsegs, ns, poff, cur);
-      LV_LAUNCHED();
-      k_cpart_scatter<<<grid_for(nc, 1, 148 * 2), 1024, 0, s>>>(dch, nc, dsegs, gc, gw, cur, P2);
-      LV_LAUNCHED();
-      k_cpart_merge<<<grid_for(nt, 1, 148), 1024, 8 * kCPartSlots, s>>>(dt, nt, dsegs, poff, P2, oc, ow, cnt,
-                                                                        &h.ctl->overflow);
-      LV_LAUNCHED();
-      LV_CUDA(cudaGetLastError());
-      unsigned long long ovf = 0;
-      LV_CUDA(cudaMemcpyAsync(&ovf, &h.ctl->overflow, 8, cudaMemcpyDeviceToHost, s));
-      LV_CUDA(cudaStreamSynchronize(s));  // host vectors die here
-      dfree(dsegs, s);
-      dfree(dch, s);
-      dfree(dt, s);
-      dfree(poff, s);
-      dfree(cur, s);
-      big_done = ovf == 0;  // else: a partition table overflowed -> radix-sort fallback below
-      if (ovf) LV_CUDA(cudaMemsetAsync(&h.ctl->overflow, 0, 8, s));
-    }
-  }
-  if (nbig > 0 && big_hash && !big_done) {
-    const int32_t* brows = rows + nsmall + nwarp + nmid;
-    std::vector<int32_t> hb(nbig);
-    LV_CUDA(cudaMemcpyAsync(hb.data(), brows, 4 * nbig, cudaMemcpyDeviceToHost, s));
-    std::vector<int64_t> hs(np + 1);
-    LV_CUDA(cudaMemcpyAsync(hs.data(), sstart, 8 * (np + 1), cudaMemcpyDeviceToHost, s));
-    LV_CUDA(cudaStreamSynchronize(s));
-    // waves of segments whose tables fit kBigWaveSlots (a larger segment gets a wave of its own)
-    std::vector<BigSeg> segs(nbig);
-    std::vector<BigItem> ins, ext;
-    std::vector<int64_t> ins_off{0}, ext_off{0};
-    int64_t acc = 0, maxslots = 0, big_entries = 0;
-    for (int64_t k = 0; k < nbig; ++k) {
-      const int32_t r = hb[k];
-      const int64_t len = hs[r + 1] - hs[r];
-      big_entries += len;
-      const int64_t cap = ((2 * std::min<int64_t>(len, np) + 3) / 4) * 4;
-      if (acc > 0 && acc + cap > kBigWaveSlots) {
-        ins_off.push_back((int64_t)ins.size());
-        ext_off.push_back((int64_t)ext.size());
-        acc = 0;
-      }
-      segs[k] = BigSeg{hs[r], acc, cap, r, 0};
-      for (int64_t e = 0; e < len; e += kBigChunk) ins.push_back(BigItem{(int32_t)k, 0, e, std::min(len, e + kBigChunk)});
-      for (int64_t e = 0; e < cap; e += kBigChunk) ext.push_back(BigItem{(int32_t)k, 0, e, std::min(cap, e + kBigChunk)});
-      acc += cap;
-      maxslots = std::max(maxslots, acc);
-    }
-    ins_off.push_back((int64_t)ins.size());
-    ext_off.push_back((int64_t)ext.size());
-    const int64_t nwaves = (int64_t)ins_off.size() - 1;
-    if (tr.on)
-      fprintf(stderr, "[lv]    contract segments: small %lld warp %lld mid %lld big %lld (big entries %lld of %lld, "
-              "%lld waves)\n", (long long)nsmall, (long long)nwarp, (long long)nmid, (long long)nbig,
-              (long long)big_entries, (long long)nnz, (long long)nwaves);
-    BigSeg* dsegs = nullptr;
-    BigItem *dins = nullptr, *dext = nullptr;
-    LV_TRY(dalloc(&dsegs, nbig, s));
-    LV_TRY(dalloc(&dins, ins.size(), s));
-    LV_TRY(dalloc(&dext, ext.size(), s));
-    LV_CUDA(cudaMemcpyAsync(dsegs, segs.data(), sizeof(BigSeg) * nbig, cudaMemcpyHostToDevice, s));
-    LV_CUDA(cudaMemcpyAsync(dins, ins.data(), sizeof(BigItem) * ins.size(), cudaMemcpyHostToDevice, s));
-    LV_CUDA(cudaMemcpyAsync(dext, ext.data(), sizeof(BigItem) * ext.size(), cudaMemcpyHostToDevice, s));
-    unsigned long long* T = nullptr;
-    {
-      void* p0 = nullptr;
-      LV_TRY(scratch_get(h, SC_K1, 8 * (size_t)maxslots, &p0));
-      T = static_cast<unsigned long long*>(p0);
-    }
-    k_fill_empty<<<grid_for(maxslots, 256, 148 * 8), 256, 0, s>>>(T, maxslots);
-    LV_LAUNCHED();
-    for (int64_t wv = 0; wv < nwaves; ++wv) {
-      const int64_t i0 = ins_off[wv], i1 = ins_off[wv + 1], x0 = ext_off[wv], x1 = ext_off[wv + 1];
-      k_big_insert<<<grid_for(i1 - i0, 1, 148 * 8), 256, 0, s>>>(dins + i0, i1 - i0, dsegs, gc, gw, T);
-      LV_LAUNCHED();
-      k_big_extract<<<grid_for(x1 - x0, 1, 148 * 8), 256, 0, s>>>(dext + x0, x1 - x0, dsegs, T, oc, ow, cnt);
-      LV_LAUNCHED();
-    }
-    LV_CUDA(cudaGetLastError());
-    dfree(dsegs, s);
-    dfree(dins, s);
-    dfree(dext, s);
-    LV_CUDA(cudaStreamSynchronize(s));  // host vectors die here
-    big_done = true;
-  }
-  static const bool big_sort32 = getenv("LV_BIG_SORT32") && getenv("LV_BIG_SORT32")[0] == '1';
-  if (nbig > 0 && !big_done && big_sort32 && nb < 32) {  // batched 32-bit sorts
-    const int32_t* brows = rows + nsmall + nwarp + nmid;
-    std::vector<int32_t> hb(nbig);
-    LV_CUDA(cudaMemcpyAsync(hb.data(), brows, 4 * nbig, cudaMemcpyDeviceToHost, s));
-    std::vector<int64_t> hs(np + 1);
-    LV_CUDA(cudaMemcpyAsync(hs.data(), sstart, 8 * (np + 1), cudaMemcpyDeviceToHost, s));
-    LV_CUDA(cudaStreamSynchronize(s));
-    std::vector<int64_t> boff(nbig + 1, 0);
-    for (int64_t k = 0; k < nbig; ++k) boff[k + 1] = boff[k] + (hs[hb[k] + 1] - hs[hb[k]]);
-    const int64_t maxseg = (int64_t)1 << (32 - nb);
-    std::vector<int64_t> cuts{0};  // batch boundaries in segment index
-    int64_t mmax = 0;
-    for (int64_t k = 0; k < nbig; ++k) {
-      const int64_t k0 = cuts.back();
-      if (k > k0 && (k - k0 >= maxseg || boff[k + 1] - boff[k0] > kBigBatchEntries)) {
-        mmax = std::max(mmax, boff[k] - boff[k0]);
-        cuts.push_back(k);
-      }
-    }
-    mmax = std::max(mmax, boff[nbig] - boff[cuts.back()]);
-    cuts.push_back(nbig);
-    if (tr.on)
-      fprintf(stderr, "[lv]    contract segments: small %lld warp %lld mid %lld big %lld (big entries %lld of %lld, "
-              "%zu sort batches)\n", (long long)nsmall, (long long)nwarp, (long long)nmid, (long long)nbig,
-              (long long)boff[nbig], (long long)nnz, cuts.size() - 1);
-    int64_t* dboff = nullptr;
-    LV_TRY(dalloc(&dboff, nbig + 1, s));
-    LV_CUDA(cudaMemcpyAsync(dboff, boff.data(), 8 * (nbig + 1), cudaMemcpyHostToDevice, s));
-    uint32_t *k0b = nullptr, *k1b = nullptr, *v0b = nullptr, *v1b = nullptr;
-    {
-      void* p0 = nullptr;
-      LV_TRY(scratch_get(h, SC_STAGE, 8 * (size_t)mmax, &p0));  // the level's stage is dead during contraction
-      k0b = static_cast<uint32_t*>(p0);
-      k1b = k0b + mmax;
-      LV_TRY(scratch_get(h, SC_K1, 8 * (size_t)mmax, &p0));
-      v0b = static_cast<uint32_t*>(p0);
-      v1b = v0b + mmax;
-    }
-    int64_t* dnum = reinterpret_cast<int64_t*>(&h.ctl->bad);
-    size_t tb_sort = 0, tb_red = 0;
-    {
-      cub::DoubleBuffer<uint32_t> kq(k0b, k1b), vq(v0b, v1b);
-      LV_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, tb_sort, kq, vq, mmax, 0, 32, s));
-      LV_CUDA(cub::DeviceReduce::ReduceByKey(nullptr, tb_red, k0b, k1b, v0b, v1b, dnum, cub::Sum(), mmax, s));
-    }
-    void* tmp = nullptr;
-    LV_TRY(dmalloc(&tmp, std::max(tb_sort, tb_red), s));
-    for (size_t bi = 0; bi + 1 < cuts.size(); ++bi) {
-      const int64_t ka = cuts[bi], kz = cuts[bi + 1], nseg = kz - ka;
-      const int64_t base = boff[ka], mb = boff[kz] - base;
-      if (mb <= 0) continue;
-      int kbits = 0;
-      while (kbits < 32 && ((int64_t)1 << kbits) < nseg) ++kbits;
-      k_big_keys32<<<grid_for(mb, 256, 148 * 16), 256, 0, s>>>(brows + ka, nseg, dboff + ka, base, mb, sstart, gc, gw,
-                                                               nb, k0b, v0b);
-      LV_LAUNCHED();
-      cub::DoubleBuffer<uint32_t> kq(k0b, k1b), vq(v0b, v1b);
-      size_t tbs = tb_sort;
-      LV_CUDA(cub::DeviceRadixSort::SortPairs(tmp, tbs, kq, vq, mb, 0, nb + kbits, s));
-      LV_CUB();
-      size_t tbr = tb_red;
-      LV_CUDA(cub::DeviceReduce::ReduceByKey(tmp, tbr, kq.Current(), kq.Alternate(), vq.Current(), vq.Alternate(), dnum,
-                                             cub::Sum(), mb, s));
-      LV_CUB();
-      k_big_place32<<<grid_for(mb, 256, 148 * 16), 256, 0, s>>>(kq.Alternate(), vq.Alternate(), dnum, nb, brows + ka,
-                                                                sstart, oc, ow, cnt);
-      LV_LAUNCHED();
-    }
-    LV_CUDA(cudaGetLastError());
-    dfree(tmp, s);
-    dfree(dboff, s);
-    LV_CUDA(cudaStreamSynchronize(s));  // host vectors die here
-    big_done = true;
-  }
-  if (nbig > 0 && !big_done) {  // one radix sort of 64-bit (segment rank, neighbour) keys + reduce-by-key
+  if (nbig > 0) {  // one radix sort of 64-bit (segment rank, neighbour) keys + reduce-by-key
     const int32_t* brows = rows + nsmall + nwarp + nmid;
     // offsets of the big segments in the key array: lengths + scan on the device
     int64_t* dboff = nullptr;
@@ -1552,66 +817,7 @@ int32_t level_contract_fast(Handle& h, Level& L, Level& out, int32_t* d_map, int
               (long long)nsmall, (long long)nwarp, (long long)nmid, (long long)nbig, (long long)m, (long long)nnz);
     int kb = 1;
     while (kb < 40 && (1ll << kb) < nbig) ++kb;
-    // LV_BIG_SEG=1 (experiment): measured slower on C5 -- level 0 26.3 vs 23.5 ms, level 1 270 vs 43 ms
-    // (CUB's segmented radix sort gives a huge segment a single thread block)
-    static const bool seg_env = getenv("LV_BIG_SEG") && getenv("LV_BIG_SEG")[0] == '1';
-    if (nb + kb > 32 && seg_env && nb <= 31 && m < ((int64_t)1 << 31)) {  // segmented sort of neighbour keys
-      uint32_t *k0 = nullptr, *k1 = nullptr, *v0 = nullptr, *v1 = nullptr, *sums = nullptr;
-      {
-        void* p0 = nullptr;
-        LV_TRY(scratch_get(h, SC_STAGE, 8 * (size_t)m, &p0));  // the level's stage is dead during contraction
-        k0 = static_cast<uint32_t*>(p0);
-        k1 = k0 + m;
-        LV_TRY(scratch_get(h, SC_K1, 8 * (size_t)m, &p0));
-        v0 = static_cast<uint32_t*>(p0);
-        v1 = v0 + m;
-        LV_TRY(scratch_get(h, SC_V0, 4 * (size_t)m, &p0));
-        sums = static_cast<uint32_t*>(p0);
-      }
-      {
-        const int64_t* btr = nullptr;
-        LV_TRY(tile_starts(h, dboff, 0, nbig, 0, m, kBigTile, &btr));
-        k_big_keys_t<uint32_t><<<grid_for((m + kBigTile - 1) / kBigTile, 1, 148 * 8), 256, 0, s>>>(
-            brows, nbig, sstart, dboff, btr, m, gc, gw, -1, k0, v0);
-        LV_LAUNCHED();
-      }
-      tr.mark(s, "big-keys");
-      size_t tb = 0;
-      LV_CUDA(cub::DeviceSegmentedRadixSort::SortPairs(nullptr, tb, k0, k1, v0, v1, (int)m, (int)nbig, dboff,
-                                                      dboff + 1, 0, nb, s));
-      void* tmp = nullptr;
-      LV_TRY(dmalloc(&tmp, tb, s));
-      LV_CUDA(cub::DeviceSegmentedRadixSort::SortPairs(tmp, tb, k0, k1, v0, v1, (int)m, (int)nbig, dboff, dboff + 1,
-                                                      0, nb, s));
-      LV_CUB();
-      dfree(tmp, s);
-      tr.mark(s, "big-segsort");
-      // runs: heads (segment starts | key changes) -> inclusive scan = run id -> sums
-      LV_CUDA(cudaMemsetAsync(k0, 0, 4 * (size_t)m, s));
-      k_seg_mark<<<grid_for(nbig, 256), 256, 0, s>>>(dboff, nbig, k0);
-      LV_LAUNCHED();
-      k_seg_heads<<<grid_for(m, 256, 148 * 16), 256, 0, s>>>(k1, m, k0);
-      LV_LAUNCHED();
-      tb = 0;
-      LV_CUDA(cub::DeviceScan::InclusiveSum(nullptr, tb, k0, v0, m, s));
-      LV_TRY(dmalloc(&tmp, tb, s));
-      LV_CUDA(cub::DeviceScan::InclusiveSum(tmp, tb, k0, v0, m, s));
-      LV_CUB();
-      dfree(tmp, s);
-      int64_t* dnum = reinterpret_cast<int64_t*>(&h.ctl->bad);
-      tb = 0;
-      LV_CUDA(cub::DeviceReduce::ReduceByKey(nullptr, tb, v0, k0, v1, sums, dnum, cub::Sum(), m, s));
-      LV_TRY(dmalloc(&tmp, tb, s));
-      LV_CUDA(cub::DeviceReduce::ReduceByKey(tmp, tb, v0, k0, v1, sums, dnum, cub::Sum(), m, s));
-      LV_CUB();
-      dfree(tmp, s);
-      tr.mark(s, "big-reduce");
-      k_seg_place<<<grid_for(m, 256, 148 * 16), 256, 0, s>>>(k1, v0, sums, m, dboff, nbig, brows, sstart, oc, ow, cnt);
-      LV_LAUNCHED();
-      dfree(dboff, s);
-      LV_CUDA(cudaMemsetAsync(&h.ctl->bad, 0, 8, s));
-      tr.mark(s, "big-place");
-    } else if (nb + kb <= 32) {  // 32-bit keys: 8 instead of 12 bytes per element and pass
+    if (nb + kb <= 32) {  // 32-bit keys: 8 instead of 12 bytes per element and pass
       uint32_t *k0 = nullptr, *k1 = nullptr, *v0 = nullptr, *v1 = nullptr;
       {
         void* p0 = nullptr;
@@ -1624,13 +830,9 @@ int32_t level_contract_fast(Handle& h, Level& L, Level& out, int32_t* d_map, int
       }
       // combiner: worthwhile when the big segments repeat neighbours (few new
       // vertices per big entry); 0xFFFFFFFF must not be a real key (table marker)
-      static const char* comb_env = getenv("LV_BIG_COMBINE");
       const bool key_ok = (((uint64_t)(nbig - 1) << nb) | (uint64_t)(np - 1)) < 0xFFFFFFFFull;
-      const bool comb = key_ok && (comb_env ? comb_env[0] == '1' : m >= 64 * np);
-      // LV_COMB_FUSED=1: the combiner reads the grouped copy directly (no key array) --
-      // measured slower on C5 level 2 (38.4 ms vs 7.4 + 29.1 ms): per-entry segment search
-      static const bool fused = getenv("LV_COMB_FUSED") && getenv("LV_COMB_FUSED")[0] == '1';
-      if (!(comb && fused)) {
+      const bool comb = key_ok && m >= 64 * np;
+      {
         const int64_t* btr = nullptr;
         LV_TRY(tile_starts(h, dboff, 0, nbig, 0, m, kBigTile, &btr));
         k_big_keys_t<uint32_t><<<grid_for((m + kBigTile - 1) / kBigTile, 1, 148 * 8), 256, 0, s>>>(
@@ -1640,25 +842,16 @@ int32_t level_contract_fast(Handle& h, Level& L, Level& out, int32_t* d_map, int
       tr.mark(s, "big-keys");
       cub::DoubleBuffer<uint32_t> kq(k0, k1), vq(v0, v1);
       if (comb) {
-        static const bool small = getenv("LV_COMB_SMALL") && getenv("LV_COMB_SMALL")[0] == '1';
         static bool cattr = false;
         if (!cattr) {
           LV_CUDA(cudaFuncSetAttribute(k_big_combine<kCombSlots, 14, kCombChunk, 1024>,
                                        cudaFuncAttributeMaxDynamicSharedMemorySize, 8 * kCombSlots));
-          LV_CUDA(cudaFuncSetAttribute(k_big_combine<8192, 13, 32768, 512>,
-                                       cudaFuncAttributeMaxDynamicSharedMemorySize, 8 * 8192));
           cattr = true;
         }
         unsigned long long* dcnt = reinterpret_cast<unsigned long long*>(&h.ctl->bad);
         LV_CUDA(cudaMemsetAsync(dcnt, 0, 8, s));
-        const BigSrc bsrc{brows, nbig, sstart, dboff, gc, gw, nb};
-        const uint32_t* kin = fused ? nullptr : k0;
-        if (small)
-          k_big_combine<8192, 13, 32768, 512><<<grid_for((m + 32767) / 32768, 1, 148 * 3), 512, 8 * 8192, s>>>(
-              kin, v0, m, k1, v1, dcnt, bsrc);
-        else
-          k_big_combine<kCombSlots, 14, kCombChunk, 1024><<<grid_for((m + kCombChunk - 1) / kCombChunk, 1, 148), 1024,
-                                                            8 * kCombSlots, s>>>(kin, v0, m, k1, v1, dcnt, bsrc);
+        k_big_combine<kCombSlots, 14, kCombChunk, 1024><<<grid_for((m + kCombChunk - 1) / kCombChunk, 1, 148), 1024,
+                                                          8 * kCombSlots, s>>>(k0, v0, m, k1, v1, dcnt);
         LV_LAUNCHED();
         unsigned long long m2 = 0;
         LV_CUDA(cudaMemcpyAsync(&m2, dcnt, 8, cudaMemcpyDeviceToHost, s));
@@ -1693,77 +886,6 @@ int32_t level_contract_fast(Handle& h, Level& L, Level& out, int32_t* d_map, int
       dfree(dboff, s);
       LV_CUDA(cudaMemsetAsync(&h.ctl->bad, 0, 8, s));
     } else {
-      // weight bits: the largest single entry weight of the level (sums go to a separate array)
-      int wbits = 1;
-      static const bool pack_req = getenv("LV_BIG_PACK") && getenv("LV_BIG_PACK")[0] == '1';
-      if (gw && pack_req) {
-        unsigned* dmx = reinterpret_cast<unsigned*>(&h.ctl->bad);
-        LV_CUDA(cudaMemsetAsync(dmx, 0, 8, s));
-        k_max_u32<<<grid_for(nnz, 256, 148 * 8), 256, 0, s>>>(gw, nnz, dmx);
-        LV_LAUNCHED();
-        unsigned mx = 0;
-        LV_CUDA(cudaMemcpyAsync(&mx, dmx, 4, cudaMemcpyDeviceToHost, s));
-        LV_CUDA(cudaStreamSynchronize(s));
-        LV_CUDA(cudaMemsetAsync(&h.ctl->bad, 0, 8, s));
-        wbits = 1;
-        while (wbits < 32 && (mx >> wbits) != 0u) ++wbits;
-      }
-      // LV_BIG_PACK=1: keys-only sort with the weight packed into the low key bits --
-      // measured slower on C5 (levels 0/1: 15.8 / 30.4 -> 19.3 / 37.1 ms), off
-      static const bool packed_env = getenv("LV_BIG_PACK") && getenv("LV_BIG_PACK")[0] == '1';
-      if (packed_env && nb + kb + wbits <= 64) {  // keys-only sort: 8 instead of 12 bytes per element and pass
-        unsigned long long *k0 = nullptr, *k1 = nullptr;
-        uint32_t* sums = nullptr;
-        {
-          void* p0 = nullptr;
-          LV_TRY(scratch_get(h, SC_STAGE, 8 * (size_t)m, &p0));
-          k0 = static_cast<unsigned long long*>(p0);
-          LV_TRY(scratch_get(h, SC_K1, 8 * (size_t)m, &p0));
-          k1 = static_cast<unsigned long long*>(p0);
-          LV_TRY(scratch_get(h, SC_V0, 4 * (size_t)m, &p0));
-          sums = static_cast<uint32_t*>(p0);
-        }
-        {
-          const int64_t* btr = nullptr;
-          LV_TRY(tile_starts(h, dboff, 0, nbig, 0, m, kBigTile, &btr));
-          k_big_keys_t<unsigned long long><<<grid_for((m + kBigTile - 1) / kBigTile, 1, 148 * 8), 256, 0, s>>>(
-              brows, nbig, sstart, dboff, btr, m, gc, gw, nb, k0, nullptr, wbits);
-          LV_LAUNCHED();
-        }
-        tr.mark(s, "big-keys");
-        cub::DoubleBuffer<unsigned long long> kbuf(k0, k1);
-        size_t tb = 0;
-        LV_CUDA(cub::DeviceRadixSort::SortKeys(nullptr, tb, kbuf, m, wbits, wbits + nb + kb, s));
-        void* tmp = nullptr;
-        LV_TRY(dmalloc(&tmp, tb, s));
-        LV_CUDA(cub::DeviceRadixSort::SortKeys(tmp, tb, kbuf, m, wbits, wbits + nb + kb, s));
-        LV_CUB();
-        dfree(tmp, s);
-        tr.mark(s, "big-sort");
-        int64_t* dnum = reinterpret_cast<int64_t*>(&h.ctl->bad);
-        auto khi = thrust::make_transform_iterator(kbuf.Current(), KeyHi{wbits});
-        auto klo = thrust::make_transform_iterator(kbuf.Current(), KeyLo{(1ull << wbits) - 1ull});
-        unsigned long long* ukeys = kbuf.Alternate();
-        tb = 0;
-        LV_CUDA(cub::DeviceReduce::ReduceByKey(nullptr, tb, khi, ukeys, klo, sums, dnum, cub::Sum(), m, s));
-        LV_TRY(dmalloc(&tmp, tb, s));
-        LV_CUDA(cub::DeviceReduce::ReduceByKey(tmp, tb, khi, ukeys, klo, sums, dnum, cub::Sum(), m, s));
-        LV_CUB();
-        dfree(tmp, s);
-        int64_t nruns = 0;
-        LV_CUDA(cudaMemcpyAsync(&nruns, dnum, 8, cudaMemcpyDeviceToHost, s));
-        LV_CUDA(cudaStreamSynchronize(s));
-        tr.mark(s, "big-reduce");
-        int64_t* first_run = nullptr;
-        LV_TRY(dalloc(&first_run, nbig, s));
-        k_big_first<<<grid_for(nruns, 256), 256, 0, s>>>(ukeys, nruns, nb, first_run);
-        LV_LAUNCHED();
-        k_big_place<<<grid_for(nruns, 256), 256, 0, s>>>(ukeys, sums, nruns, nb, brows, sstart, first_run, oc, ow, cnt);
-        LV_LAUNCHED();
-        dfree(first_run, s);
-        dfree(dboff, s);
-        LV_CUDA(cudaMemsetAsync(&h.ctl->bad, 0, 8, s));
-      } else {
       unsigned long long *k0 = nullptr, *k1 = nullptr;
       uint32_t *v0 = nullptr, *v1 = nullptr;
       {
@@ -1818,7 +940,6 @@ int32_t level_contract_fast(Handle& h, Level& L, Level& out, int32_t* d_map, int
       dfree(first_run, s);
       dfree(dboff, s);
       LV_CUDA(cudaMemsetAsync(&h.ctl->bad, 0, 8, s));
-      }
     }
     tr.mark(s, "big-place");
   }

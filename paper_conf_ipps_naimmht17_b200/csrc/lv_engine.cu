@@ -285,28 +285,6 @@ bool bucket_nonempty(const Level& L, int b) {
 // commit (BIN_SYNC) -- or a single commit at the end (RELAXED).
 int32_t sweep_body(Handle& h, Level& L, const louvain_params_t& p) {
   static const bool trace = getenv("LV_TRACE") && std::string(getenv("LV_TRACE")) == "2";
-  static const char* l2win = getenv("LV_L2WIN");  // experiment: persisting L2 window over ca[0..bytes)
-  if (l2win) {
-    cudaDeviceProp pr;
-    cudaGetDeviceProperties(&pr, h.device);
-    size_t want = (size_t)atoll(l2win);
-    want = std::min(want, (size_t)L.n * sizeof(uint2));
-    want = std::min(want, (size_t)pr.accessPolicyMaxWindowSize);
-    cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, std::min(want, (size_t)pr.persistingL2CacheMaxSize));
-    cudaStreamAttrValue v = {};
-    v.accessPolicyWindow.base_ptr = L.ca;
-    v.accessPolicyWindow.num_bytes = want;
-    v.accessPolicyWindow.hitRatio = 1.0f;
-    v.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
-    v.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
-    cudaStreamSetAttribute(h.stream, cudaStreamAttributeAccessPolicyWindow, &v);
-    static bool once = false;
-    if (!once) {
-      fprintf(stderr, "[lv] L2 window %zu B (max window %d, max persisting %d, L2 %d)\n", want,
-              pr.accessPolicyMaxWindowSize, pr.persistingL2CacheMaxSize, pr.l2CacheSize);
-      once = true;
-    }
-  }
   LV_CUDA(cudaMemsetAsync(h.ctl, 0, offsetof(DevCtl, L), h.stream));  // logn + bounds
   int commits = 0;
   for (int b = 1; b <= 7; ++b) {

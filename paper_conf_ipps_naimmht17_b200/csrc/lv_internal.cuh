@@ -141,30 +141,10 @@ struct PartPlan {
   int64_t bucket_task[9] = {0};   // tasks of bucket b: [bucket_task[b-1], bucket_task[b])
   int64_t bucket_vert[9] = {0};   // plan vertices of bucket b
   int64_t bucket_chunk[9] = {0};  // chunks of bucket b (pre-partitioned vertices only)
-  int64_t ngroups = 0;            // cluster groups of the streaming vertices (sweep_part_clu)
-  int32_t* grp_vi = nullptr;      // [ngroups] plan vertex of the group
-  int32_t* grp_p0 = nullptr;      // [ngroups] first partition of the group (multiple of kCluCS)
-  int64_t bucket_grp[9] = {0};    // groups of bucket b: [bucket_grp[b-1], bucket_grp[b])
   int64_t bucket_vsplit[8] = {0};  // bucket b's vertices [bucket_vert[b-1], vsplit) are pre-partitioned,
   int64_t bucket_tsplit[8] = {0};  // tasks [bucket_task[b-1], tsplit); the rest stream (P <= kStreamMaxP)
 };
 constexpr int64_t kStreamMaxP = 16;
-constexpr int kCluGroup = 8;  // partitions per cluster group (= sweep_part_clu's cluster size)
-
-// Batched plan for the table-based vertices of degree <= kBatchMaxDeg (sub-class 0
-// of buckets whose bound exceeds 32): consecutive bin positions are cut into
-// batches of bounded total weight (deg + kBatchVertexWeight each), so a CTA
-// inserts a whole batch edge-parallel into per-vertex regions of one
-// shared-memory table (sweep_batch, lv_sweep.cu).
-constexpr int kBatchSlots = 8448;        // table slots per CTA (12 B each)
-constexpr int kBatchMaxVerts = 136;      // vertices per batch (<= kBatchSlots / 2 / kBatchVertexWeight + 1)
-constexpr int kBatchVertexWeight = 32;   // per-vertex weight added to its degree when cutting batches
-constexpr int64_t kBatchMaxDeg = 1023;
-struct BatchPlan {
-  int32_t* bstart = nullptr;      // batch start positions of every bucket, concatenated (+ end sentinels)
-  int64_t off[9] = {0};           // batches of bucket b: bstart[off[b-1] .. off[b]) (each list + 1 sentinel)
-  int64_t cap = 0;
-};
 
 struct Level {
   int64_t n = 0, nnz = 0;
@@ -201,7 +181,6 @@ struct Level {
   uint2* stage = nullptr;
   HubPlan hub;
   PartPlan part;
-  BatchPlan batch;
 };
 
 // Grow-only scratch buffers owned by a handle (cudaMalloc'ed once, reused by
@@ -309,8 +288,6 @@ int32_t launch_sweep_bucket(Handle& h, Level& L, const louvain_params_t& p, int 
 // phase 1 gather for bin positions [pos0,pos1), staged entries [s0,s1)
 int32_t launch_stage(Handle& h, Level& L, int64_t pos0, int64_t pos1, int64_t s0, int64_t s1);
 int32_t build_part_plan(Handle& h, Level& L);
-int32_t build_batch_plan(Handle& h, Level& L, const louvain_params_t& p);
-void batch_free(BatchPlan& B, cudaStream_t s);
 
 // ------------------------------------------------------------------ launch geometry
 inline unsigned grid_for(int64_t items, int per_block, int max_blocks = 148 * 16) {

@@ -500,15 +500,6 @@ int32_t level_alloc_state(Level& L, cudaStream_t s) {
 }
 
 static void part_free(PartPlan& Q, cudaStream_t s);
-// Expected labels per partition task (kPartLabels; LV_PART_LABELS overrides, A/B only).
-static int64_t part_labels() {
-  static const int64_t v = [] {
-    const char* e = getenv("LV_PART_LABELS");
-    const long long x = e ? atoll(e) : 0;
-    return (x >= 1024 && x <= kPartSlots * 3 / 4) ? (int64_t)x : kPartLabels;
-  }();
-  return v;
-}
 // Most partitions a vertex may get on the label-partitioned path (more: hub kernel).
 // LV_PART_MAXP lowers it (tests use it to exercise the cooperative hub kernel).
 static int64_t part_maxp() {
@@ -523,13 +514,7 @@ static int64_t part_maxp() {
 // others stream.  Measured on C5 with kPartLabels = 10240 (per 2 sweeps, levels
 // 0/1/2): everything streaming 21.3 / 11.2 / 68.1 ms; P > 16 pre-partitioned
 // 21.2 / 10.4 / 27.1 ms; the earlier rule (pre-partition all hubs of levels with
-// mean degree >= 256, else P > 64) 21.8 / 10.8 / 31.7 ms.  LV_STREAM_MAXP overrides.
-static int64_t stream_maxp(const Level& L) {
-  static const char* e = getenv("LV_STREAM_MAXP");
-  if (e) return (int64_t)atoll(e);
-  (void)L;
-  return kStreamMaxP;
-}
+// mean degree >= 256, else P > 64) 21.8 / 10.8 / 31.7 ms.
 static void hub_free(HubPlan& P, cudaStream_t s) {
   dfree(P.ins, s); dfree(P.scans, s); dfree(P.ins_off, s); dfree(P.scan_off, s); dfree(P.wave_hub, s);
   dfree(P.info, s); dfree(P.ring, s);
@@ -559,7 +544,6 @@ void level_free(Level& L, cudaStream_t s) {
   if (L.scratch_backed) {  // arrays belong to the handle's scratch; plans are per level
     hub_free(L.hub, s);
     part_free(L.part, s);
-    batch_free(L.batch, s);
     L = Level();
     return;
   }
@@ -573,7 +557,6 @@ void level_free(Level& L, cudaStream_t s) {
   dfree(L.soff, s);  // L.stage lives in the handle's scratch
   hub_free(L.hub, s);
   part_free(L.part, s);
-  batch_free(L.batch, s);
   L = Level();
 }
 
@@ -725,7 +708,7 @@ static int32_t build_hub_plan(Handle& h, Level& L) {
     LV_CUDA(cudaStreamSynchronize(s));
     dfree(dd, s);
     for (int64_t i = 0; i < cnt; ++i) {
-      if ((d[i] + part_labels() - 1) / part_labels() <= part_maxp()) continue;  // label-partitioned path
+      if ((d[i] + kPartLabels - 1) / kPartLabels <= part_maxp()) continue;  // label-partitioned path
       hsoff.push_back(so[i]);
       hv.push_back(v[i]);
       hdeg.push_back(d[i]);
@@ -803,7 +786,7 @@ static int32_t build_hub_plan(Handle& h, Level& L) {
 static void part_free(PartPlan& Q, cudaStream_t s) {
   dfree(Q.task_vpos, s); dfree(Q.task_p, s); dfree(Q.vert_pos, s); dfree(Q.vert_P, s); dfree(Q.vert_first, s);
   dfree(Q.vert_pbase, s); dfree(Q.done, s); dfree(Q.partial, s); dfree(Q.poff, s); dfree(Q.pcur, s);
-  dfree(Q.chunks, s); dfree(Q.grp_vi, s); dfree(Q.grp_p0, s);
+  dfree(Q.chunks, s);
   Q = PartPlan();
 }
 
@@ -813,12 +796,11 @@ int32_t build_part_plan(Handle& h, Level& L) {
   cudaStream_t s = h.stream;
   PartPlan& Q = L.part;
   part_free(Q, s);
-  std::vector<int32_t> vpos, vP, vfirst, tv, tp, gvi, gp0;
+  std::vector<int32_t> vpos, vP, vfirst, tv, tp;
   std::vector<int64_t> vpb;
   std::vector<PartChunk> ch;
   int64_t pb = 0;
   for (int b = 1; b <= 7; ++b) {
-    Q.bucket_grp[b - 1] = (int64_t)gvi.size();
     Q.bucket_task[b - 1] = (int64_t)tv.size();
     Q.bucket_vert[b - 1] = (int64_t)vpos.size();
     Q.bucket_chunk[b - 1] = (int64_t)ch.size();
@@ -837,7 +819,7 @@ int32_t build_part_plan(Handle& h, Level& L) {
                      [&](int64_t a, int64_t b) { return so[a + 1] - so[a] > so[b + 1] - so[b]; });
     for (int64_t i : ord) {
       const int64_t deg = so[i + 1] - so[i];
-      const int64_t P = (deg + part_labels() - 1) / part_labels();
+      const int64_t P = (deg + kPartLabels - 1) / kPartLabels;
       if (P > part_maxp()) continue;  // giant: cooperative hub kernel
       const int32_t vi = (int32_t)vpos.size();
       vpos.push_back((int32_t)(off + i));
@@ -849,20 +831,13 @@ int32_t build_part_plan(Handle& h, Level& L) {
         tv.push_back(vi);
         tp.push_back(q);
       }
-      if (P > stream_maxp(L)) {  // pre-partitioned (a prefix: degrees descending)
+      if (P > kStreamMaxP) {  // pre-partitioned (a prefix: degrees descending)
         for (int64_t e = 0; e < deg; e += kPartChunk) ch.push_back(PartChunk{vi, 0, e, std::min(deg, e + kPartChunk)});
         Q.bucket_vsplit[b - 1] = (int64_t)vpos.size();
         Q.bucket_tsplit[b - 1] = (int64_t)tv.size();
-      } else {  // streaming: cluster groups of kCluGroup partitions
-        for (int32_t q = 0; q < (int32_t)P; q += kCluGroup) {
-          gvi.push_back(vi);
-          gp0.push_back(q);
-        }
       }
     }
   }
-  Q.bucket_grp[7] = (int64_t)gvi.size();
-  Q.ngroups = (int64_t)gvi.size();
   Q.nverts = (int64_t)vpos.size();
   Q.ntasks = (int64_t)tv.size();
   Q.nchunks = (int64_t)ch.size();
@@ -889,12 +864,6 @@ int32_t build_part_plan(Handle& h, Level& L) {
   LV_CUDA(cudaMemcpyAsync(Q.vert_first, vfirst.data(), 4 * vfirst.size(), cudaMemcpyHostToDevice, s));
   LV_CUDA(cudaMemcpyAsync(Q.vert_pbase, vpb.data(), 8 * vpb.size(), cudaMemcpyHostToDevice, s));
   LV_CUDA(cudaMemcpyAsync(Q.chunks, ch.data(), sizeof(PartChunk) * ch.size(), cudaMemcpyHostToDevice, s));
-  if (Q.ngroups > 0) {
-    LV_TRY(dalloc(&Q.grp_vi, Q.ngroups, s));
-    LV_TRY(dalloc(&Q.grp_p0, Q.ngroups, s));
-    LV_CUDA(cudaMemcpyAsync(Q.grp_vi, gvi.data(), 4 * gvi.size(), cudaMemcpyHostToDevice, s));
-    LV_CUDA(cudaMemcpyAsync(Q.grp_p0, gp0.data(), 4 * gp0.size(), cudaMemcpyHostToDevice, s));
-  }
   LV_CUDA(cudaStreamSynchronize(s));  // host vectors die here
   return LOUVAIN_OK;
 }
@@ -961,7 +930,6 @@ int32_t level_binning(Handle& h, Level& L, const louvain_params_t& p) {
   }
   LV_TRY(build_hub_plan(h, L));
   LV_TRY(build_part_plan(h, L));
-  LV_TRY(build_batch_plan(h, L, p));
   std::memcpy(L.bins_bounds, p.deg_bounds, sizeof L.bins_bounds);
   L.bins_valid = true;
   return LOUVAIN_OK;

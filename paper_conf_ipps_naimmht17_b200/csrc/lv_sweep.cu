@@ -313,7 +313,7 @@ __global__ void __launch_bounds__(256) k_stage(const int32_t* __restrict__ bv, c
                                                int64_t pos0, int64_t pos1, const int64_t* __restrict__ tr,
                                                const int64_t* __restrict__ rowptr,
                                                const int32_t* __restrict__ col, const uint2* __restrict__ ca,
-                                               uint2* __restrict__ stage, bool cs_store, bool full_a) {
+                                               uint2* __restrict__ stage) {
   __shared__ int64_t sh_so[kStageRows + 1];
   __shared__ int64_t sh_rb[kStageRows];
   __shared__ int32_t sh_v[kStageRows];
@@ -370,103 +370,17 @@ __global__ void __launch_bounds__(256) k_stage(const int32_t* __restrict__ bv, c
       }
 #pragma unroll
       for (int q = 0; q < 4; ++q) rr[q] = (jj[q] >= 0 && jj[q] != vv[q]) ? __ldg(&ca[jj[q]]) : make_uint2(kSelf, 0);
-      if (full_a) {  // a_c of labels whose neighbour is not their representative: a second gather
-#pragma unroll       // here (edge-parallel, latency hidden) instead of in the table scans
-        for (int q = 0; q < 4; ++q)
-          if (jj[q] >= 0 && jj[q] != vv[q] && rr[q].x != (uint32_t)jj[q]) rr[q].y = __ldg(&ca[rr[q].x]).y;
-      }
 #pragma unroll
       for (int q = 0; q < 4; ++q) {
         const int64_t t = base + (int64_t)q * blockDim.x;
         // evict-first store: the stage streams through L2 once and must not
-        // displace the gathered records (LV_STAGE_WB=1: plain write-back store)
+        // displace the gathered records
         const uint2 val = (jj[q] == vv[q]) ? make_uint2(kSelf, 0u)
-                                           : make_uint2(rr[q].x, (full_a || rr[q].x == (uint32_t)jj[q]) ? rr[q].y
-                                                                                                        : kUnknownA);
-        if (t < t1) {
-          if (cs_store) __stcs(&stage[t], val);
-          else stage[t] = val;
-        }
+                                           : make_uint2(rr[q].x, rr[q].x == (uint32_t)jj[q] ? rr[q].y : kUnknownA);
+        if (t < t1) __stcs(&stage[t], val);
       }
     }
     __syncthreads();
-  }
-}
-
-// Warp-chunked variant of phase 1 (LV_STAGE_W=1): every warp takes chunks of
-// kStageChunk staged entries on its own -- no CTA barriers.  Lane r holds the
-// descriptor (entry offset, row start, vertex) of the r-th row touching the
-// chunk (tile plan at chunk granularity); a lane finds the row of each of its
-// entries by a 5-step shuffle search, and keeps 8 gathers in flight.  A chunk
-// touching more than 32 rows (rows shorter than 32 entries on average) falls
-// back to a binary search over soff.
-constexpr int kStageChunk = 1024;
-__global__ void __launch_bounds__(256) k_stage_w(const int32_t* __restrict__ bv, const int64_t* __restrict__ soff,
-                                                 int64_t pos0, int64_t pos1, int64_t s0, int64_t s1,
-                                                 const int64_t* __restrict__ tr, const int64_t* __restrict__ rowptr,
-                                                 const int32_t* __restrict__ col, const uint2* __restrict__ ca,
-                                                 uint2* __restrict__ stage) {
-  const int lane = threadIdx.x & 31;
-  const int64_t nchunks = (s1 - s0 + kStageChunk - 1) / kStageChunk;
-  const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
-  for (int64_t ch = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); ch < nchunks; ch += warps) {
-    const int64_t t0 = s0 + ch * kStageChunk, t1 = min(s1, t0 + kStageChunk);
-    const int64_t i0 = tr[ch], i1 = tr[ch + 1];
-    const int nr = (int)((i1 - i0 + 1 < 33) ? i1 - i0 + 1 : 33);
-    const bool fits = i1 - i0 + 1 <= 32;
-    // lane r: row i0 + r
-    int64_t my_so = INT64_MAX, my_rb = 0;
-    int32_t my_v = -1;
-    if (fits && lane < nr && i0 + lane < pos1) {
-      my_v = bv[i0 + lane];
-      my_so = soff[i0 + lane];
-      my_rb = rowptr[my_v];
-    }
-    for (int64_t b0 = t0; b0 < t1; b0 += 8 * 32) {  // warp-uniform trips (shuffles below)
-      const int64_t base = b0 + lane;
-      int32_t jj[8], vv[8];
-#pragma unroll
-      for (int q = 0; q < 8; ++q) {
-        const int64_t t = base + 32 * q;
-        int64_t e = 0;
-        vv[q] = -1;
-        jj[q] = -1;
-        if (fits) {
-          int lo = 0;  // largest r with so_r <= t (all lanes take part in the shuffles)
-#pragma unroll
-          for (int step = 16; step >= 1; step >>= 1) {
-            const int64_t so_mid = __shfl_sync(kFull, my_so, lo + step);
-            if (lo + step < nr && so_mid <= t) lo += step;
-          }
-          const int64_t so_r = __shfl_sync(kFull, my_so, lo);
-          const int64_t rb_r = __shfl_sync(kFull, my_rb, lo);
-          const int32_t v_r = __shfl_sync(kFull, my_v, lo);
-          if (t < t1) {
-            vv[q] = v_r;
-            e = rb_r + (t - so_r);
-          }
-        } else if (t < t1) {
-          int64_t lo = pos0, hi = pos1 - 1;
-          while (lo < hi) {
-            const int64_t mid = (lo + hi + 1) >> 1;
-            if (soff[mid] <= t) lo = mid; else hi = mid - 1;
-          }
-          vv[q] = bv[lo];
-          e = rowptr[vv[q]] + (t - soff[lo]);
-        }
-        if (t < t1) jj[q] = __ldcs(&col[e]);
-      }
-      uint2 rr[8];
-#pragma unroll
-      for (int q = 0; q < 8; ++q) rr[q] = (jj[q] >= 0 && jj[q] != vv[q]) ? __ldg(&ca[jj[q]]) : make_uint2(kSelf, 0);
-#pragma unroll
-      for (int q = 0; q < 8; ++q) {
-        const int64_t t = base + 32 * q;
-        if (t < t1)
-          __stcs(&stage[t], (jj[q] == vv[q]) ? make_uint2(kSelf, 0u)
-                                             : make_uint2(rr[q].x, rr[q].x == (uint32_t)jj[q] ? rr[q].y : kUnknownA));
-      }
-    }
   }
 }
 
@@ -757,328 +671,6 @@ __global__ void __launch_bounds__(32 * WARPS) sweep_warp_l(const int32_t* __rest
     }
     log_moves(lane == 0 && tgt != own, v, tgt, A);
     __syncwarp();
-  }
-}
-
-// CTA per vertex with a claimed-slot list; dynamic smem = capmax slots (12 B)
-// + lcap list entries (2 B).
-template <bool UNIT>
-__global__ void __launch_bounds__(1024) sweep_cta_l(const int32_t* __restrict__ verts,
-                                                    const int64_t* __restrict__ soff, int64_t nv,
-                                                    const uint2* __restrict__ stage, SweepArgs A, int capmax) {
-  extern __shared__ unsigned long long smem[];
-  unsigned long long* T = smem;
-  uint32_t* TA = reinterpret_cast<uint32_t*>(smem + capmax);
-  uint16_t* Lst = reinterpret_cast<uint16_t*>(TA + capmax);
-  __shared__ long long sh_s[32];
-  __shared__ int sh_c[32];
-  __shared__ unsigned sh_e[32];
-  __shared__ int sh_n;
-  for (int t = threadIdx.x; t < capmax; t += blockDim.x) {
-    T[t] = kEmpty;
-    TA[t] = kUnknownA;
-  }
-  if (threadIdx.x == 0) sh_n = 0;
-  __syncthreads();
-  for (int64_t vi = blockIdx.x; vi < nv; vi += gridDim.x) {
-    const int32_t v = __ldg(&verts[vi]);
-    const int64_t rb = __ldg(&A.rowptr[v]);
-    const int64_t deg = __ldg(&A.rowptr[v + 1]) - rb;
-    const int32_t own = (int32_t)__ldg(&A.ca[v]).x;
-    const uint32_t ki = __ldg(&A.k[v]);
-    const uint32_t cap = (uint32_t)((2 * deg < (int64_t)capmax) ? 2 * deg : (int64_t)capmax);
-    insert_list<UNIT>(T, TA, cap, stage + __ldg(&soff[vi]), UNIT ? nullptr : A.w + rb, deg, threadIdx.x, blockDim.x,
-                      Lst, &sh_n);
-    __syncthreads();
-    const int nl = sh_n;
-    const bool own_single = A.rule == 2 && __ldg(&A.size[own]) == 1;
-    long long s = (long long)0x8000000000000000ull;
-    int cb = 0x7FFFFFFF;
-    unsigned eown = 0;
-    scan_list(T, TA, Lst, nl, threadIdx.x, blockDim.x, own, own_single, ki, A, s, cb, eown);
-    block_reduce(s, cb, eown, sh_s, sh_c, sh_e);  // its barrier orders every read of sh_n before the reset
-    if (threadIdx.x < 32) {
-      int32_t tgt = own;
-      if (threadIdx.x == 0) {
-        tgt = finish(s, cb, eown, own, __ldg(&A.ca[own]).y, ki, A);
-        sh_n = 0;
-      }
-      log_moves(threadIdx.x == 0 && tgt != own, v, tgt, A);
-    }
-    __syncthreads();
-  }
-}
-
-
-// ------------------------------------------------------------ CTA per vertex, pipelined (LV_CTA_PIPE=1)
-// Persistent CTAs, one vertex at a time, software-pipelined so the per-vertex
-// chain of dependent global loads is off the critical path: while the CTA
-// hashes vertex j, lanes of warp 0 already load the bin entry of vertex j+2 and
-// the row bounds / record / degree of vertex j+1 (results parked in registers and
-// stored to shared memory at the end of the iteration), and a_own / size_own of
-// vertex j for its decision.  Moves go to a shared buffer flushed with one
-// atomic per kLogBuf moves.
-constexpr int kLogBuf = 128;
-
-__device__ __forceinline__ void flush_moves(int32_t* buf_v, int32_t* buf_t, int n, const SweepArgs& A) {
-  // warp 0, all lanes
-  const int lane = threadIdx.x & 31;
-  unsigned long long base = 0;
-  if (lane == 0 && n) base = atomicAdd(A.logn, (unsigned long long)n);
-  base = __shfl_sync(kFull, base, 0);
-  for (int i = lane; i < n; i += 32) {
-    A.mv_v[base + i] = buf_v[i];
-    A.mv_new[base + i] = buf_t[i];
-  }
-}
-
-template <bool UNIT, bool AGG>
-__global__ void __launch_bounds__(1024) sweep_cta_pipe(const int32_t* __restrict__ verts, const int64_t* __restrict__ soff,
-                                                  int64_t nv, const uint2* __restrict__ stage, SweepArgs A,
-                                                  int capmax) {
-  extern __shared__ unsigned long long smem[];
-  unsigned long long* T = smem;
-  uint32_t* TA = reinterpret_cast<uint32_t*>(smem + capmax);
-  __shared__ long long sh_s[32];
-  __shared__ int sh_c[32];
-  __shared__ unsigned sh_e[32];
-  // header of the current vertex (j) and the bin entry of the next one (j+1)
-  __shared__ int64_t h_rb, h_deg, h_so;
-  __shared__ int32_t h_v, h_own, h_vnext;
-  __shared__ uint32_t h_ki;
-  __shared__ int32_t buf_v[kLogBuf], buf_t[kLogBuf];
-  __shared__ int nbuf;
-  const int lane = threadIdx.x & 31;
-  const int64_t G = gridDim.x;
-  for (int t = threadIdx.x; t < capmax; t += blockDim.x) {
-    T[t] = kEmpty;
-    TA[t] = kUnknownA;
-  }
-  if (threadIdx.x == 0) {  // prologue: header of vertex 0, bin entry of vertex 1
-    nbuf = 0;
-    const int64_t vi = blockIdx.x;
-    if (vi < nv) {
-      const int32_t v = verts[vi];
-      h_v = v;
-      h_rb = A.rowptr[v];
-      h_deg = A.rowptr[v + 1] - h_rb;
-      h_so = soff[vi];
-      h_own = (int32_t)A.ca[v].x;
-      h_ki = A.k[v];
-    }
-    h_vnext = (vi + G < nv) ? verts[vi + G] : -1;
-  }
-  __syncthreads();
-  for (int64_t vi = blockIdx.x; vi < nv; vi += G) {
-    const int32_t v = h_v, own = h_own, vn = h_vnext;
-    const int64_t rb = h_rb, deg = h_deg, so = h_so;
-    const uint32_t ki = h_ki;
-    // warp 0 issues the loads of the next vertices now and consumes them at the end
-    int64_t pf = 0;
-    if (threadIdx.x < 32) {
-      if (lane == 0 && vi + 2 * G < nv) pf = verts[vi + 2 * G];
-      if (vn >= 0) {
-        if (lane == 1) pf = A.rowptr[vn];
-        if (lane == 2) pf = A.rowptr[vn + 1];
-        if (lane == 3) pf = soff[vi + G];
-        if (lane == 4) pf = (int64_t)A.ca[vn].x;
-        if (lane == 5) pf = (int64_t)A.k[vn];
-      }
-      if (lane == 6) pf = (int64_t)A.ca[own].y;
-      if (lane == 7) pf = (int64_t)A.size[own];
-    }
-    const uint32_t cap = (uint32_t)((2 * deg < (int64_t)capmax) ? 2 * deg : (int64_t)capmax);
-    insert_staged<UNIT, AGG>(T, TA, cap, stage + so, UNIT ? nullptr : A.w + rb, deg, threadIdx.x, blockDim.x);
-    __syncthreads();
-    const bool own_single = A.rule == 2 && __ldg(&A.size[own]) == 1;
-    long long s = (long long)0x8000000000000000ull;
-    int cb = 0x7FFFFFFF;
-    unsigned eown = 0;
-    scan_table(T, TA, cap, threadIdx.x, blockDim.x, own, own_single, ki, A, s, cb, eown);
-    block_reduce(s, cb, eown, sh_s, sh_c, sh_e);
-    if (threadIdx.x < 32) {
-      const uint32_t a_own = (uint32_t)__shfl_sync(kFull, pf, 6);
-      const int32_t size_own = (int32_t)__shfl_sync(kFull, pf, 7);
-      if (threadIdx.x == 0 && cb != 0x7FFFFFFF) {
-        int32_t tgt = own;
-        const long long sstay = A.W * (long long)eown - (long long)ki * ((long long)a_own - (long long)ki);
-        if (s > sstay) {
-          tgt = cb;
-          if (A.rule == 1 && cb > own && size_own == 1 && __ldg(&A.size[cb]) == 1) tgt = own;  // R8 veto
-        }
-        if (tgt != own) {
-          buf_v[nbuf] = v;
-          buf_t[nbuf] = tgt;
-          ++nbuf;
-        }
-      }
-      __syncwarp();
-      if (nbuf == kLogBuf) {
-        flush_moves(buf_v, buf_t, kLogBuf, A);
-        __syncwarp();
-        if (lane == 0) nbuf = 0;
-      }
-      // park the prefetched header of vertex j+1 and the bin entry of vertex j+2
-      if (lane == 0) h_vnext = (vi + 2 * G < nv) ? (int32_t)pf : -1;
-      if (vn >= 0) {
-        if (lane == 0) h_v = vn;
-        if (lane == 1) h_rb = pf;
-        if (lane == 2) h_deg = pf;  // rowptr[v+1]; minus rb below
-        if (lane == 3) h_so = pf;
-        if (lane == 4) h_own = (int32_t)pf;
-        if (lane == 5) h_ki = (uint32_t)pf;
-      }
-      __syncwarp();
-      if (lane == 0 && vn >= 0) h_deg -= h_rb;
-    }
-    __syncthreads();
-  }
-  if (threadIdx.x < 32) {
-    __syncwarp();
-    const int n = nbuf;
-    flush_moves(buf_v, buf_t, n, A);
-  }
-}
-
-// ------------------------------------------------------------ batched vertices
-// Table-based vertices of degree <= kBatchMaxDeg (33..1023 with the paper's
-// bounds): a CTA takes a batch of consecutive bin positions (total weight
-// bounded by the batch plan) and works on all of them at once, so the per-vertex
-// latency chains (row bounds, records, finish) overlap instead of serialising:
-//   1. batch metadata into smem (vertex, row start, entry offset);
-//   2. edge-parallel over the batch's staged entries: insert into the vertex's
-//      own region of the table (2*deg slots at offset 2*x0);
-//   3. each vertex's region is scanned by a group of G warps (G = 16 / nv
-//      rounded down to a power of two), partials to smem;
-//   4. a warp per vertex reduces its partials and decides (stay test, veto).
-// The records come from the staging array (k_stage gathered them edge-parallel
-// at full occupancy; gathering here, inside the batch's latency chain, measured
-// 3x slower on C5).
-template <bool UNIT>
-__global__ void __launch_bounds__(512, 2) sweep_batch(const int32_t* __restrict__ bv,
-                                                    const int64_t* __restrict__ soff,
-                                                    const int32_t* __restrict__ bstart, int64_t nbatch,
-                                                    const uint2* __restrict__ stage, SweepArgs A) {
-  extern __shared__ unsigned long long smem[];
-  unsigned long long* T = smem;
-  uint32_t* TA = reinterpret_cast<uint32_t*>(smem + kBatchSlots);
-  __shared__ int32_t s_v[kBatchMaxVerts];
-  __shared__ int64_t s_rb[kBatchMaxVerts];
-  __shared__ int32_t s_x[kBatchMaxVerts + 1];
-  __shared__ Partial s_part[16];
-  __shared__ int s_nv;
-  constexpr int NW = 16;
-  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  for (int t = threadIdx.x; t < kBatchSlots; t += blockDim.x) {
-    T[t] = kEmpty;
-    TA[t] = kUnknownA;
-  }
-  for (int64_t b = blockIdx.x; b < nbatch; b += gridDim.x) {
-    // 1. metadata
-    const int32_t p0 = __ldg(&bstart[b]), p1 = __ldg(&bstart[b + 1]);
-    const int nv = p1 - p0;
-    const int64_t base = __ldg(&soff[p0]);
-    for (int r = threadIdx.x; r <= nv; r += blockDim.x) {
-      s_x[r] = (int32_t)(__ldg(&soff[p0 + r]) - base);
-      if (r < nv) {
-        const int32_t v = __ldg(&bv[p0 + r]);
-        s_v[r] = v;
-        s_rb[r] = __ldg(&A.rowptr[v]);
-      }
-    }
-    if (threadIdx.x == 0) s_nv = nv;
-    __syncthreads();
-    const int E = s_x[nv];
-    // 2. inserts from the staged records (coalesced), 4 entries per thread per pass
-    const uint2* S = stage + base;
-    for (int x0 = threadIdx.x; x0 < E; x0 += 4 * blockDim.x) {
-      uint2 rec[4];
-      uint32_t ww[4];
-      int rr[4];
-#pragma unroll
-      for (int q = 0; q < 4; ++q) {
-        const int x = x0 + q * blockDim.x;
-        rec[q] = (x < E) ? __ldcs(&S[x]) : make_uint2(kSelf, 0u);
-        rr[q] = 0;
-        ww[q] = 1u;
-        if (x < E) {
-          int lo = 0, hi = nv - 1;  // largest r with s_x[r] <= x
-          while (lo < hi) {
-            const int mid = (lo + hi + 1) >> 1;
-            if (s_x[mid] <= x) lo = mid; else hi = mid - 1;
-          }
-          rr[q] = lo;
-          if (!UNIT) ww[q] = __ldcs(&A.w[s_rb[lo] + (x - s_x[lo])]);
-        }
-      }
-#pragma unroll
-      for (int q = 0; q < 4; ++q) {
-        if (rec[q].x == kSelf) continue;  // padding or the self-loop (R3)
-        const int r = rr[q];
-        const uint32_t off = 2u * (uint32_t)s_x[r];
-        const uint32_t cap = 2u * (uint32_t)(s_x[r + 1] - s_x[r]);
-        const uint32_t hq = table_insert(T + off, cap, (int32_t)rec[q].x, ww[q]);
-        if (rec[q].y != kUnknownA) TA[off + hq] = rec[q].y;  // the neighbour represents its label: a_c known
-      }
-    }
-    __syncthreads();
-    // 3. scan: vertex r by warps [r*G, r*G + G) (nv <= 16), else warp-strided vertices
-    int G = 1;
-    while (G * 2 * nv <= NW) G *= 2;
-    const int gw = warp % G;  // warp index inside its group
-    for (int r = warp / G; r < nv; r += NW / G) {
-      const int32_t v = s_v[r];
-      const int32_t own = (int32_t)__ldg(&A.ca[v]).x;
-      const uint32_t ki = __ldg(&A.k[v]);
-      const bool own_single = A.rule == 2 && __ldg(&A.size[own]) == 1;
-      const uint32_t off = 2u * (uint32_t)s_x[r];
-      const uint32_t cap = 2u * (uint32_t)(s_x[r + 1] - s_x[r]);
-      long long sc = (long long)0x8000000000000000ull;
-      int cb = 0x7FFFFFFF;
-      unsigned eown = 0;
-      scan_table(T + off, TA + off, cap, (uint32_t)(gw * 32 + lane), (uint32_t)(32 * G), own, own_single, ki, A, sc,
-                 cb, eown);
-      group_reduce<32>(sc, cb, eown);
-      if (G == 1) {
-        int32_t tgt = own;
-        if (lane == 0 && cb != 0x7FFFFFFF) tgt = finish(sc, cb, eown, own, __ldg(&A.ca[own]).y, ki, A);
-        log_moves(lane == 0 && tgt != own, v, tgt, A);
-      } else if (lane == 0) {
-        s_part[warp] = Partial{sc, cb, eown};
-      }
-    }
-    if (G > 1) {
-      __syncthreads();
-      // 4. a warp per vertex reduces its G partials
-      if (warp < nv) {
-        const int r = warp;
-        long long sc = (long long)0x8000000000000000ull;
-        int cb = 0x7FFFFFFF;
-        unsigned eown = 0;
-        if (lane < G) {
-          const Partial pp = s_part[r * G + lane];
-          sc = pp.s;
-          cb = pp.c;
-          eown = pp.eown;
-        }
-        group_reduce<32>(sc, cb, eown);
-        const int32_t v = s_v[r];
-        const int32_t own = (int32_t)__ldg(&A.ca[v]).x;
-        int32_t tgt = own;
-        if (lane == 0 && cb != 0x7FFFFFFF) tgt = finish(sc, cb, eown, own, __ldg(&A.ca[own]).y, __ldg(&A.k[v]), A);
-        log_moves(lane == 0 && tgt != own, v, tgt, A);
-      }
-    }
-    __syncthreads();
-  }
-}
-
-__global__ void k_batch_flags(const int64_t* __restrict__ soff, int64_t p0, int64_t p1, int64_t s0, int64_t bw,
-                              uint8_t* flag) {
-  for (int64_t i = p0 + blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < p1; i += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t wi = (soff[i] - s0 + kBatchVertexWeight * (i - p0)) / bw;
-    const int64_t wp = (i == p0) ? -1 : (soff[i - 1] - s0 + kBatchVertexWeight * (i - 1 - p0)) / bw;
-    flag[i - p0] = (wi != wp) ? 1 : 0;
   }
 }
 
@@ -1434,189 +1026,6 @@ __global__ void __launch_bounds__(1024) sweep_part_stream(const int32_t* __restr
 }
 
 
-// Hub vertices of the label-partitioned path (the streaming ones, deg >= kSub5Min)
-// with a per-CTA table in global memory instead of P label partitions: each CTA
-// takes the next vertex (dynamic, the plan lists them by degree, descending),
-// inserts its staged labels once into a 2*deg-slot region of its own (4-slot
-// buckets, gtable_insert4: one L2 round trip per insert), scans and clears it.
-// The live regions of all CTAs (~148 x 2 x deg x 12 B) stay in L2.  Replaces the
-// P-fold streaming of sweep_part_stream (ncu, C5 level 0: 8.6e9 instructions,
-// issue-bound) -- but measured 4x slower (see gtab_on); off by default.
-template <bool UNIT, bool AGG>
-__global__ void __launch_bounds__(512) sweep_gtab(const int32_t* __restrict__ vert_pos, int64_t v_begin,
-                                                  int64_t v_end, unsigned* next, const int32_t* __restrict__ bv,
-                                                  const int64_t* __restrict__ soff, const uint2* __restrict__ stage,
-                                                  SweepArgs A, unsigned long long* gT, uint32_t* gTA,
-                                                  int64_t region) {
-  __shared__ long long sh_s[32];
-  __shared__ int sh_c[32];
-  __shared__ unsigned sh_e[32];
-  __shared__ int64_t sh_vi;
-  unsigned long long* T = gT + (int64_t)blockIdx.x * region;
-  uint32_t* TA = gTA + (int64_t)blockIdx.x * region;
-  for (;;) {
-    if (threadIdx.x == 0) sh_vi = v_begin + (int64_t)atomicAdd(next, 1u);
-    __syncthreads();
-    const int64_t vi = sh_vi;
-    if (vi >= v_end) break;
-    const int32_t pos = vert_pos[vi];
-    const int32_t v = __ldg(&bv[pos]);
-    const int64_t sb = __ldg(&soff[pos]), deg = __ldg(&soff[pos + 1]) - sb;
-    const uint32_t cap = (uint32_t)(((2 * deg + 3) / 4) * 4);
-    insert_staged<UNIT, AGG, true>(T, TA, cap, stage + sb, UNIT ? nullptr : A.w + __ldg(&A.rowptr[v]), deg,
-                                   threadIdx.x, blockDim.x);
-    __syncthreads();
-    const int32_t own = (int32_t)__ldg(&A.ca[v]).x;
-    const uint32_t ki = __ldg(&A.k[v]);
-    const bool own_single = A.rule == 2 && __ldg(&A.size[own]) == 1;
-    long long s = (long long)0x8000000000000000ull;
-    int cb = 0x7FFFFFFF;
-    unsigned eown = 0;
-    scan_table<true>(T, TA, cap, threadIdx.x, blockDim.x, own, own_single, ki, A, s, cb, eown);
-    block_reduce(s, cb, eown, sh_s, sh_c, sh_e);
-    if (threadIdx.x < 32) {
-      int32_t tgt = own;
-      if (threadIdx.x == 0) tgt = finish(s, cb, eown, own, __ldg(&A.ca[own]).y, ki, A);
-      log_moves(threadIdx.x == 0 && tgt != own, v, tgt, A);
-    }
-    __syncthreads();
-  }
-}
-
-// Cluster variant of the streaming tasks (LV_CLU=1, experiment): a cluster of kCluCS CTAs
-// takes kCluCS consecutive partitions p0 .. p0+kCluCS-1 of one vertex.  Every
-// CTA streams 1/kCluCS of the vertex's staged labels and inserts each label of
-// those partitions into the table of the CTA that owns it, through distributed
-// shared memory (one remote CAS per distinct label), so the vertex's list is read
-// ceil(P / kCluCS) times instead of P times.  After a cluster barrier each CTA
-// scans its own table exactly like sweep_part_stream and the CTA finishing v's
-// last partition reduces the partials.
-constexpr int kCluCS = 8;
-template <bool UNIT>
-__global__ void __launch_bounds__(1024, 1) sweep_part_clu(const int32_t* __restrict__ grp_vi,
-                                                          const int32_t* __restrict__ grp_p0, int64_t g_begin,
-                                                          int64_t g_end, const int32_t* __restrict__ vert_pos,
-                                                          const int32_t* __restrict__ vert_P,
-                                                          const int32_t* __restrict__ vert_first, int32_t* done,
-                                                          Partial* part, unsigned long long* overflow,
-                                                          const int32_t* __restrict__ bv,
-                                                          const int64_t* __restrict__ soff,
-                                                          const uint2* __restrict__ stage, SweepArgs A) {
-  namespace cg = cooperative_groups;
-  cg::cluster_group cl = cg::this_cluster();
-  const unsigned rank = cl.block_rank();
-  extern __shared__ unsigned long long smem[];
-  unsigned long long* T = smem;
-  uint32_t* TA = reinterpret_cast<uint32_t*>(smem + kPartSlots);
-  __shared__ long long sh_s[32];
-  __shared__ int sh_c[32];
-  __shared__ unsigned sh_e[32];
-  __shared__ int is_last;
-  for (int t = threadIdx.x; t < kPartSlots; t += blockDim.x) {
-    T[t] = kEmpty;
-    TA[t] = kUnknownA;
-  }
-  cl.sync();  // every table of the cluster is initialised before remote inserts
-  const int lane = threadIdx.x & 31;
-  const int64_t ncl = gridDim.x / kCluCS, cid = blockIdx.x / kCluCS;
-  for (int64_t g = g_begin + cid; g < g_end; g += ncl) {
-    const int32_t vi = grp_vi[g];
-    const uint32_t p0 = (uint32_t)grp_p0[g];
-    const int32_t pos = vert_pos[vi];
-    const uint32_t P = (uint32_t)vert_P[vi];
-    const int32_t v = __ldg(&bv[pos]);
-    const int64_t sb = __ldg(&soff[pos]), deg = __ldg(&soff[pos + 1]) - sb;
-    // table size of this group: 2x the expected labels per partition + slack
-    const uint32_t cap = (uint32_t)min((int64_t)kPartSlots, 2 * ((deg + P - 1) / P) + 512);
-    const uint2* S = stage + sb;
-    const uint32_t* Wt = UNIT ? nullptr : A.w + __ldg(&A.rowptr[v]);
-    const int64_t lo = deg * rank / kCluCS, hi = deg * (rank + 1) / kCluCS;
-    for (int64_t base = lo; base + (int64_t)(threadIdx.x - lane) < hi; base += 4 * (int64_t)blockDim.x) {
-      uint2 rr[4];
-      uint32_t ww[4];
-#pragma unroll
-      for (int q = 0; q < 4; ++q) {
-        const int64_t t = base + threadIdx.x + (int64_t)q * blockDim.x;
-        rr[q] = (t < hi) ? __ldcg(&S[t]) : make_uint2(kSelf, 0u);
-        ww[q] = UNIT ? 1u : ((t < hi) ? __ldcg(&Wt[t]) : 0u);
-      }
-#pragma unroll
-      for (int q = 0; q < 4; ++q) {
-        const uint32_t d = (rr[q].x != kSelf) ? part_of((int32_t)rr[q].x, P) - p0 : 0xFFFFFFFFu;
-        bool keep = d < (uint32_t)kCluCS;
-        uint32_t x = ww[q], arep = rr[q].y;
-        // equal labels of a warp are merged first when adjacent lanes share one
-        const uint32_t key = keep ? rr[q].x : (0x80000000u | (unsigned)lane);
-        if (__any_sync(kFull, key == __shfl_xor_sync(kFull, key, 1))) {
-          const unsigned m = __match_any_sync(kFull, key);
-          x = __reduce_add_sync(m, x);
-          const unsigned rep = __ballot_sync(kFull, keep && rr[q].y != kUnknownA) & m;
-          arep = __shfl_sync(kFull, rr[q].y, rep ? __ffs(rep) - 1 : lane);
-          if (!rep) arep = kUnknownA;
-          keep = keep && lane == __ffs(m) - 1;
-        }
-        if (!keep) continue;
-        unsigned long long* Tr = cl.map_shared_rank(T, d);
-        const unsigned long long kx = ((unsigned long long)rr[q].x << 32) | x;
-        uint32_t h = hash_slot((int32_t)rr[q].x, cap);
-        uint32_t probes = 0;
-        for (;;) {
-          const unsigned long long old = atomicCAS(&Tr[h], kEmpty, kx);
-          if (old == kEmpty) break;
-          if ((uint32_t)(old >> 32) == rr[q].x) {
-            atomicAdd(&Tr[h], (unsigned long long)x);
-            break;
-          }
-          h = (h + 1 == cap) ? 0u : h + 1;
-          if (++probes >= cap) {  // table full: cannot happen at the planned load; reported as an error
-            atomicAdd(overflow, 1ull);
-            break;
-          }
-        }
-        if (arep != kUnknownA) cl.map_shared_rank(TA, d)[h] = arep;
-      }
-    }
-    cl.sync();  // all inserts into every table of the cluster are done
-    const uint32_t p = p0 + rank;
-    if (p < P) {
-      const int32_t own = (int32_t)__ldg(&A.ca[v]).x;
-      const uint32_t ki = __ldg(&A.k[v]);
-      const bool own_single = A.rule == 2 && __ldg(&A.size[own]) == 1;
-      long long s = (long long)0x8000000000000000ull;
-      int cb = 0x7FFFFFFF;
-      unsigned eown = 0;
-      scan_table(T, TA, cap, threadIdx.x, blockDim.x, own, own_single, ki, A, s, cb, eown);
-      block_reduce(s, cb, eown, sh_s, sh_c, sh_e);
-      const int32_t f = vert_first[vi];
-      if (threadIdx.x == 0) {
-        part[f + p] = Partial{s, cb, eown};
-        __threadfence();
-        is_last = (atomicAdd(&done[vi], 1) == (int)P - 1);
-      }
-      __syncthreads();
-      if (is_last && threadIdx.x < 32) {
-        __threadfence();
-        s = (long long)0x8000000000000000ull;
-        cb = 0x7FFFFFFF;
-        eown = 0;
-        for (uint32_t q = threadIdx.x; q < P; q += 32) {
-          const longlong2 raw = __ldcg(reinterpret_cast<const longlong2*>(&part[f + q]));
-          const long long ps = raw.x;
-          const int pc = (int)(raw.y & 0xFFFFFFFFll);
-          const unsigned pe = (unsigned)((unsigned long long)raw.y >> 32);
-          if (better(ps, pc, s, cb)) { s = ps; cb = pc; }
-          eown += pe;
-        }
-        group_reduce<32>(s, cb, eown);
-        int32_t tgt = own;
-        if (threadIdx.x == 0) tgt = finish(s, cb, eown, own, __ldg(&A.ca[own]).y, ki, A);
-        log_moves(threadIdx.x == 0 && tgt != own, v, tgt, A);
-      }
-    }
-    cl.sync();  // every table is scanned (and cleared) before the next group's inserts
-  }
-}
-
 // Task (v, p) of the plan: inserts the partition's pre-scattered entries
 // (S2[poff[p] .. poff[p+1])) into a smem table of 2 * n_p slots (n_p = entries >=
 // distinct labels: load <= 1/2, no overflow possible) -- or kPartSlots with a
@@ -1843,45 +1252,6 @@ int32_t launch_hub(Handle& h, Level& L, const SweepArgs& A, const uint2* stage, 
   return LOUVAIN_OK;
 }
 
-// LV_GTAB=1: per-CTA global tables instead of the single-CTA streaming partition
-// tasks.  Measured 4x slower on C5 (level 0: 28.3 -> 111.7 ms per 2 sweeps, with or
-// without warp label merging): L2 atomic round trips per label cost far more than
-// the P-fold L2 streaming they replace.  Kept as an experiment (parity-tested).
-static bool gtab_on() {
-  static const bool on = getenv("LV_GTAB") && getenv("LV_GTAB")[0] == '1';
-  return on;
-}
-// Per-CTA global hash regions for sweep_gtab (grow-only, kept clean: every scan
-// clears what it visited), plus the dynamic vertex counter.
-static int32_t gtab_get(Handle& h, int64_t slots, unsigned long long** T, uint32_t** TA, unsigned** next) {
-  void* p = nullptr;
-  LV_TRY(scratch_get(h, SC_GTAB, 12 * (size_t)slots + 256, &p));
-  size_t have = 0;
-  LV_TRY(scratch_size(h, SC_GTAB, &have));
-  const int64_t cap_slots = (int64_t)((have - 256) / 12);
-  unsigned long long* t = static_cast<unsigned long long*>(p);
-  if (h.scratch.gtab_init != p || h.scratch.gtab_init_bytes != have) {  // new or grown: every slot empty once
-
-    LV_CUDA(cudaMemsetAsync(t, 0xFF, 8 * (size_t)cap_slots, h.stream));             // kEmpty
-    LV_CUDA(cudaMemsetAsync(t + cap_slots, 0xFF, 4 * (size_t)cap_slots, h.stream));  // kUnknownA
-    h.scratch.gtab_init = p;
-    h.scratch.gtab_init_bytes = have;
-  }
-  *T = t;
-  *TA = reinterpret_cast<uint32_t*>(t + cap_slots);
-  *next = reinterpret_cast<unsigned*>(reinterpret_cast<char*>(p) + 12 * (size_t)cap_slots);
-  return LOUVAIN_OK;
-}
-
-// LV_CLU=1: cluster (DSMEM) streaming groups instead of single-CTA streaming tasks.
-// Measured 2.4x slower on C5 (level 0: 30.7 -> 72.5 ms per 2 sweeps; level 1:
-// 14.9 -> 36.9 ms): one remote CAS round trip per label costs more than the
-// redundant L2 streaming it saves.  Kept as an experiment (parity-tested).
-static bool clu_on() {
-  static const bool on = getenv("LV_CLU") && getenv("LV_CLU")[0] == '1';
-  return on;
-}
-
 // The label-partitioned path of one bucket.  Plan vertices are ordered by degree
 // (descending); those with P > kStreamMaxP form a prefix and take the
 // pre-partitioned pipeline (histogram -> scan -> scatter -> tasks), the rest
@@ -1943,8 +1313,7 @@ int32_t launch_part(Handle& h, Level& L, const SweepArgs& A, int bucket, bool un
                                                                L.soff, Q.poff, Q.pcur);
     LV_LAUNCHED();
     mark("scan");
-    static const char* agg_env = getenv("LV_PART_AGG");
-    const bool agg = agg_env ? agg_env[0] == '1' : !unit;  // merging pays off once labels concentrate
+    const bool agg = !unit;  // merging pays off once labels concentrate (contracted levels)
     if (unit) {
       k_part_scatter<true><<<grid_for(c1 - c0, 1, 148 * 2), 1024, 0, s>>>(Q.chunks, c0, c1, Q.vert_pos, Q.vert_P,
                                                                           Q.vert_first, L.bin_vertices, L.soff, stage,
@@ -1964,83 +1333,7 @@ int32_t launch_part(Handle& h, Level& L, const SweepArgs& A, int bucket, bool un
     }
     mark("pre-tasks");
   }
-  const int64_t g0 = Q.bucket_grp[bucket - 1], g1 = Q.bucket_grp[bucket];
-  if (t1 > ts && gtab_on()) {  // streaming vertices [vs, v1): per-CTA global tables (LV_GTAB=1)
-    int64_t maxdeg = 0;  // the plan lists vertices by degree, descending: the first is the largest
-    {
-      int32_t pos = 0;
-      int64_t so[2] = {0, 0};
-      LV_CUDA(cudaMemcpyAsync(&pos, Q.vert_pos + vs, 4, cudaMemcpyDeviceToHost, s));
-      LV_CUDA(cudaStreamSynchronize(s));
-      LV_CUDA(cudaMemcpyAsync(so, L.soff + pos, 16, cudaMemcpyDeviceToHost, s));
-      LV_CUDA(cudaStreamSynchronize(s));
-      maxdeg = so[1] - so[0];
-    }
-    const int64_t region = ((2 * maxdeg + 3) / 4) * 4;
-    static int resident = 0;
-    if (resident == 0) {
-      int nb = 0;
-      LV_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, sweep_gtab<true, false>, 512, 0));
-      resident = std::max(nb, 1);
-    }
-    const int64_t nblk = std::min<int64_t>(148 * resident, v1 - vs);
-    unsigned long long* gT = nullptr;
-    uint32_t* gTA = nullptr;
-    unsigned* next = nullptr;
-    LV_TRY(gtab_get(h, nblk * region, &gT, &gTA, &next));
-    LV_CUDA(cudaMemsetAsync(next, 0, 4, s));
-    static const char* ge = getenv("LV_GTAB_AGG");
-    const bool gagg = ge ? ge[0] == '1' : !unit;
-    if (unit) {
-      if (gagg) sweep_gtab<true, true><<<(unsigned)nblk, 512, 0, s>>>(Q.vert_pos, vs, v1, next, L.bin_vertices, L.soff, stage, A, gT, gTA, region);
-      else sweep_gtab<true, false><<<(unsigned)nblk, 512, 0, s>>>(Q.vert_pos, vs, v1, next, L.bin_vertices, L.soff, stage, A, gT, gTA, region);
-    } else {
-      if (gagg) sweep_gtab<false, true><<<(unsigned)nblk, 512, 0, s>>>(Q.vert_pos, vs, v1, next, L.bin_vertices, L.soff, stage, A, gT, gTA, region);
-      else sweep_gtab<false, false><<<(unsigned)nblk, 512, 0, s>>>(Q.vert_pos, vs, v1, next, L.bin_vertices, L.soff, stage, A, gT, gTA, region);
-    }
-    LV_LAUNCHED();
-    mark("stream");
-  } else if (t1 > ts && clu_on() && g1 > g0) {  // streaming tasks, cluster variant (LV_CLU=1)
-    static bool cattr = false;
-    if (!cattr) {
-      LV_TRY(set_smem(sweep_part_clu<true>, 12 * (size_t)kPartSlots));
-      LV_TRY(set_smem(sweep_part_clu<false>, 12 * (size_t)kPartSlots));
-      cattr = true;
-    }
-    static_assert(kCluCS == kCluGroup, "cluster size must match the plan's group size");
-    cudaLaunchConfig_t cfg = {};
-    cfg.blockDim = dim3(1024, 1, 1);
-    cfg.dynamicSmemBytes = 12 * (size_t)kPartSlots;
-    cfg.stream = s;
-    cudaLaunchAttribute at[1];
-    at[0].id = cudaLaunchAttributeClusterDimension;
-    at[0].val.clusterDim.x = kCluCS;
-    at[0].val.clusterDim.y = 1;
-    at[0].val.clusterDim.z = 1;
-    cfg.attrs = at;
-    cfg.numAttrs = 1;
-    static int max_clu = 0;  // co-resident clusters (GPC packing decides, not 148 / kCluCS)
-    if (max_clu == 0) {
-      cfg.gridDim = dim3(148 / kCluCS * kCluCS, 1, 1);
-      int nc = 0;
-      LV_CUDA(cudaOccupancyMaxActiveClusters(&nc, sweep_part_clu<true>, &cfg));
-      max_clu = std::max(nc, 1);
-    }
-    const int64_t nclu = std::min<int64_t>(g1 - g0, max_clu);
-    cfg.gridDim = dim3((unsigned)(nclu * kCluCS), 1, 1);
-    if (unit)
-      LV_CUDA(cudaLaunchKernelEx(&cfg, sweep_part_clu<true>, (const int32_t*)Q.grp_vi, (const int32_t*)Q.grp_p0, g0, g1,
-                                 (const int32_t*)Q.vert_pos, (const int32_t*)Q.vert_P, (const int32_t*)Q.vert_first,
-                                 Q.done, (Partial*)Q.partial, &h.ctl->overflow, (const int32_t*)L.bin_vertices,
-                                 (const int64_t*)L.soff, stage, A));
-    else
-      LV_CUDA(cudaLaunchKernelEx(&cfg, sweep_part_clu<false>, (const int32_t*)Q.grp_vi, (const int32_t*)Q.grp_p0, g0,
-                                 g1, (const int32_t*)Q.vert_pos, (const int32_t*)Q.vert_P,
-                                 (const int32_t*)Q.vert_first, Q.done, (Partial*)Q.partial, &h.ctl->overflow,
-                                 (const int32_t*)L.bin_vertices, (const int64_t*)L.soff, stage, A));
-    LV_LAUNCHED();
-    mark("stream");
-  } else if (t1 > ts) {  // streaming tasks
+  if (t1 > ts) {  // streaming tasks
     if (unit)
       sweep_part_stream<true><<<grid_for(t1 - ts, 1, 148 * 2), 1024, 12 * (size_t)kPartSlots, s>>>(
           Q.task_vpos, Q.task_p, ts, t1, Q.vert_pos, Q.vert_P, Q.vert_first, Q.done, (Partial*)Q.partial,
@@ -2056,27 +1349,10 @@ int32_t launch_part(Handle& h, Level& L, const SweepArgs& A, int bucket, bool un
   return LOUVAIN_OK;
 }
 
-bool batch_on(const Level& L, int bucket) {
-  return L.batch.bstart && L.batch.off[bucket] - L.batch.off[bucket - 1] > 1;
-}
-
 // Claimed-slot lists pay where the table is much larger than the distinct count:
 // the fixed 512-slot warp tables of bucket 6 (C5 level 0: 10.2 -> 6.3 ms per 2
 // sweeps).  The CTA tables are sized 2*deg, where the list measured slower
 // (b7 [1024,2048): 12.5 -> 19.4 ms), and so was the 128-slot warp table of bucket 5.
-// LV_LIST=0 turns it off; LV_LIST_CTA=1 turns it on for the CTA tiers (A/B only).
-static bool use_list() {
-  static const bool on = !(getenv("LV_LIST") && getenv("LV_LIST")[0] == '0');
-  return on;
-}
-static bool list_cta() {
-  static const bool on = getenv("LV_LIST_CTA") && getenv("LV_LIST_CTA")[0] == '1';
-  return on;
-}
-static bool pipe_on() {
-  static const bool on = getenv("LV_CTA_PIPE") && getenv("LV_CTA_PIPE")[0] == '1';
-  return on;
-}
 // largest degree of CTA tier `sub` (lv_internal.cuh)
 static int64_t max_deg_of_tier(int sub) {
   static const int64_t ub[5] = {kSub1Min - 1, kSub2Min - 1, kSub3Min - 1, kSub4Min - 1, kSub5Min - 1};
@@ -2102,18 +1378,7 @@ int32_t dispatch_class(Handle& h, Level& L, const SweepArgs& A, int bucket, int 
       default: sweep_small<32, UNIT><<<grid, 256, 0, s>>>(verts, nv, A); break;
     }
     LV_LAUNCHED();
-  } else if (sub == 0 && batch_on(L, bucket)) {
-    static bool battr = false;
-    if (!battr) {
-      LV_TRY(set_smem(sweep_batch<true>, 12 * (size_t)kBatchSlots));
-      LV_TRY(set_smem(sweep_batch<false>, 12 * (size_t)kBatchSlots));
-      battr = true;
-    }
-    const int64_t b0 = L.batch.off[bucket - 1], nb = L.batch.off[bucket] - b0 - 1;  // minus the sentinel
-    sweep_batch<UNIT><<<grid_for(nb, 1, 148 * 2), 512, 12 * (size_t)kBatchSlots, s>>>(L.bin_vertices, L.soff,
-                                                                                    L.batch.bstart + b0, nb, stage, A);
-    LV_LAUNCHED();
-  } else if (sub == 0 && max_deg > 84 && max_deg <= 340 && use_list()) {
+  } else if (sub == 0 && max_deg > 84 && max_deg <= 340) {
     sweep_warp_l<512, 352, 4, UNIT><<<grid_for(nv, 4, 148 * 8), 128, 0, s>>>(verts, soff, nv, stage, A);
     LV_LAUNCHED();
   } else if (sub == 0 && max_deg <= 84) {
@@ -2128,8 +1393,6 @@ int32_t dispatch_class(Handle& h, Level& L, const SweepArgs& A, int bucket, int 
   } else {
     static const int* caps = kCapT;
     static const int* threads = kThrT;
-    static const int* per_sm = kPerSmT;
-    const size_t smem = 12 * (size_t)caps[sub];
     static bool attr_done = false;
     if (!attr_done) {
       LV_TRY(set_smem(sweep_cta<true, false>, 12 * (size_t)kCapMax));
@@ -2138,62 +1401,20 @@ int32_t dispatch_class(Handle& h, Level& L, const SweepArgs& A, int bucket, int 
       LV_TRY(set_smem(sweep_cta<false, true>, 12 * (size_t)kCapMax));
       attr_done = true;
     }
-    if (list_cta()) {  // claimed-slot list variant (LV_LIST_CTA=1; measured slower on C5, tables are 2*deg here)
-      static int resident[5] = {0, 0, 0, 0, 0};
-      const int capl = std::min(caps[sub], 16384);
-      const int lcap = (int)std::min<int64_t>(capl, max_deg_of_tier(sub));
-      const size_t lsmem = 12 * (size_t)capl + 2 * (size_t)((lcap + 7) & ~7);
-      static bool lattr = false;
-      if (!lattr) {
-        LV_TRY(set_smem(sweep_cta_l<true>, 12 * (size_t)16384 + 2 * 12288));
-        LV_TRY(set_smem(sweep_cta_l<false>, 12 * (size_t)16384 + 2 * 12288));
-        lattr = true;
-      }
-      if (resident[sub] == 0) {
-        int nb = 0;
-        LV_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, sweep_cta_l<UNIT>, threads[sub], lsmem));
-        resident[sub] = std::max(nb, 1);
-      }
-      const unsigned lgrid = grid_for(nv, 1, 148 * resident[sub]);
-      sweep_cta_l<UNIT><<<lgrid, threads[sub], lsmem, s>>>(verts, soff, nv, stage, A, capl);
-      LV_LAUNCHED();
-      LV_CUDA(cudaGetLastError());
-      return LOUVAIN_OK;
+    constexpr int fnum = 8;  // table of 2*deg slots (1.5x / 1.75x / 2.5x / 3x measured slower)
+    static int resident[5] = {0, 0, 0, 0, 0};
+    const int64_t md = max_deg_of_tier(sub);
+    const int capt = (int)std::min<int64_t>(caps[sub], ((md + ((md * fnum) >> 3) + 1 + 31) / 32) * 32);
+    if (resident[sub] == 0) {
+      int nb = 0;
+      LV_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, sweep_cta<UNIT, AGG>, threads[sub], 12 * (size_t)capt));
+      resident[sub] = std::max(nb, 1);
     }
-    static const int fnum = [] {  // table size factor 1 + fnum/8 (LV_CAP_F, A/B only)
-      const char* e = getenv("LV_CAP_F");
-      const int x = e ? atoi(e) : 0;
-      return (x >= 2 && x <= 24) ? x : 8;
-    }();
-    if (!pipe_on()) {
-      static int resident[5] = {0, 0, 0, 0, 0};
-      const int64_t md = max_deg_of_tier(sub);
-      const int capt = (int)std::min<int64_t>(caps[sub], ((md + ((md * fnum) >> 3) + 1 + 31) / 32) * 32);
-      if (resident[sub] == 0) {
-        int nb = 0;
-        LV_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, sweep_cta<UNIT, AGG>, threads[sub], 12 * (size_t)capt));
-        resident[sub] = std::max(nb, 1);
-      }
-      sweep_cta<UNIT, AGG><<<grid_for(nv, 1, 148 * resident[sub]), threads[sub], 12 * (size_t)capt, s>>>(
-          verts, soff, nv, stage, A, capt, fnum);
-      LV_LAUNCHED();
-      LV_CUDA(cudaGetLastError());
-      return LOUVAIN_OK;
-    }
-    const unsigned grid = grid_for(nv, 1, 148 * per_sm[sub]);
-    static const bool pipe = getenv("LV_CTA_PIPE") && getenv("LV_CTA_PIPE")[0] == '1';
-    if (pipe) {
-      static bool pattr = false;
-      if (!pattr) {
-        LV_TRY(set_smem(sweep_cta_pipe<true, false>, 12 * (size_t)kCapMax));
-        LV_TRY(set_smem(sweep_cta_pipe<false, false>, 12 * (size_t)kCapMax));
-        LV_TRY(set_smem(sweep_cta_pipe<true, true>, 12 * (size_t)kCapMax));
-        LV_TRY(set_smem(sweep_cta_pipe<false, true>, 12 * (size_t)kCapMax));
-        pattr = true;
-      }
-      sweep_cta_pipe<UNIT, AGG><<<grid, threads[sub], smem, s>>>(verts, soff, nv, stage, A, caps[sub]);
-    }
+    sweep_cta<UNIT, AGG><<<grid_for(nv, 1, 148 * resident[sub]), threads[sub], 12 * (size_t)capt, s>>>(
+        verts, soff, nv, stage, A, capt, fnum);
     LV_LAUNCHED();
+    LV_CUDA(cudaGetLastError());
+    return LOUVAIN_OK;
   }
   LV_CUDA(cudaGetLastError());
   return LOUVAIN_OK;
@@ -2202,65 +1423,6 @@ int32_t dispatch_class(Handle& h, Level& L, const SweepArgs& A, int bucket, int 
 }  // namespace
 
 size_t hub_partial_bytes() { return sizeof(Partial); }
-
-void batch_free(BatchPlan& B, cudaStream_t s) {
-  dfree(B.bstart, s);
-  B = BatchPlan();
-}
-
-// Batch plan (see kBatchSlots): for every bucket whose sub-class 0 is table-based
-// (bound > 32), positions where floor((soff[i] - soff[p0] + 32 (i - p0)) / bw)
-// changes start a batch; bw keeps every batch's entries <= kBatchSlots / 2.
-// Experimental, off by default (LV_BATCH=1): on C5 it measured 2x slower than the
-// warp / CTA kernels it replaces (per-batch phases serialise the per-vertex loads).
-int32_t build_batch_plan(Handle& h, Level& L, const louvain_params_t& p) {
-  cudaStream_t s = h.stream;
-  batch_free(L.batch, s);
-  static const bool on = getenv("LV_BATCH") && getenv("LV_BATCH")[0] == '1';
-  if (!on || L.n == 0) return LOUVAIN_OK;
-  BatchPlan& B = L.batch;
-  int64_t total = 0;
-  for (int b = 1; b <= 7; ++b) {
-    const int c = kSubPerBucket * b;
-    total += L.class_off[c + 1] - L.class_off[c] + 1;
-  }
-  LV_TRY(dalloc(&B.bstart, total + 1, s));
-  uint8_t* flag = nullptr;
-  LV_TRY(dalloc(&flag, std::max<int64_t>(L.n, 1), s));
-  int64_t* d_num = reinterpret_cast<int64_t*>(&h.ctl->bad);
-  int64_t pos = 0;
-  B.off[0] = 0;
-  for (int b = 1; b <= 7; ++b) {
-    const int c = kSubPerBucket * b;
-    const int64_t p0 = L.class_off[c], p1 = L.class_off[c + 1];
-    const int64_t hi = (b <= 6) ? p.deg_bounds[b - 1] : INT64_MAX;
-    const int64_t max_deg = std::min<int64_t>(hi, kSub1Min - 1);
-    if (p1 > p0 && max_deg > 32 && max_deg <= kBatchMaxDeg) {
-      const int64_t bw = kBatchSlots / 2 - (max_deg + kBatchVertexWeight);
-      k_batch_flags<<<grid_for(p1 - p0, 256), 256, 0, s>>>(L.soff, p0, p1, L.class_soff[c], bw, flag);
-      LV_LAUNCHED();
-      thrust::counting_iterator<int32_t> it((int32_t)p0);
-      size_t tb = 0;
-      LV_CUDA(cub::DeviceSelect::Flagged(nullptr, tb, it, flag, B.bstart + pos, d_num, p1 - p0, s));
-      void* tmp = nullptr;
-      LV_TRY(dmalloc(&tmp, tb, s));
-      LV_CUDA(cub::DeviceSelect::Flagged(tmp, tb, it, flag, B.bstart + pos, d_num, p1 - p0, s));
-      LV_CUB();
-      dfree(tmp, s);
-      int64_t cnt = 0;
-      LV_CUDA(cudaMemcpyAsync(&cnt, d_num, 8, cudaMemcpyDeviceToHost, s));
-      LV_CUDA(cudaStreamSynchronize(s));
-      const int32_t end = (int32_t)p1;
-      LV_CUDA(cudaMemcpyAsync(B.bstart + pos + cnt, &end, 4, cudaMemcpyHostToDevice, s));
-      LV_CUDA(cudaStreamSynchronize(s));  // `end` is a host stack value
-      pos += cnt + 1;
-    }
-    B.off[b] = pos;
-  }
-  dfree(flag, s);
-  LV_CUDA(cudaMemsetAsync(&h.ctl->bad, 0, 8, s));
-  return LOUVAIN_OK;
-}
 
 // LV_TRACE=2: per-class timing (synchronises the stream; diagnostics only)
 static bool trace_on() {
@@ -2283,26 +1445,12 @@ static void trace_step(Handle& h, Level& L, int bucket, int sub, int64_t pos0, i
           (long)(e[1] - e[0]), ms, ms > 0 ? (e[1] - e[0]) / ms / 1e6 : 0.0);
 }
 
-// LV_STAGE_A=1: the stage carries a_c for every label (see k_stage), A/B
-static bool stage_full_a() {
-  static const bool on = getenv("LV_STAGE_A") && getenv("LV_STAGE_A")[0] == '1';
-  return on;
-}
-
 int32_t launch_stage(Handle& h, Level& L, int64_t pos0, int64_t pos1, int64_t s0, int64_t s1) {
   if (s1 <= s0) return LOUVAIN_OK;
-  static const bool wb = getenv("LV_STAGE_WB") && getenv("LV_STAGE_WB")[0] == '1';
-  static const bool tiled = !(getenv("LV_STAGE_W") && getenv("LV_STAGE_W")[0] == '1');
   const int64_t* tr = nullptr;
-  if (tiled || wb) {  // CTA-tiled variant (default)
-    LV_TRY(tile_starts(h, L.soff, pos0, pos1, s0, s1, kStageTile, &tr));
-    k_stage<<<grid_for((s1 - s0 + kStageTile - 1) / kStageTile, 1, 148 * 8), 256, 0, h.stream>>>(
-        L.bin_vertices, L.soff, pos0, pos1, tr, L.rowptr, L.col, L.ca, L.stage, !wb, stage_full_a());
-  } else {
-    LV_TRY(tile_starts(h, L.soff, pos0, pos1, s0, s1, kStageChunk, &tr));
-    k_stage_w<<<grid_for((s1 - s0 + kStageChunk - 1) / kStageChunk, 8, 148 * 8), 256, 0, h.stream>>>(
-        L.bin_vertices, L.soff, pos0, pos1, s0, s1, tr, L.rowptr, L.col, L.ca, L.stage);
-  }
+  LV_TRY(tile_starts(h, L.soff, pos0, pos1, s0, s1, kStageTile, &tr));
+  k_stage<<<grid_for((s1 - s0 + kStageTile - 1) / kStageTile, 1, 148 * 8), 256, 0, h.stream>>>(
+      L.bin_vertices, L.soff, pos0, pos1, tr, L.rowptr, L.col, L.ca, L.stage);
   LV_LAUNCHED();
   LV_CUDA(cudaGetLastError());
   return LOUVAIN_OK;
@@ -2324,19 +1472,12 @@ int32_t launch_sweep_bucket(Handle& h, Level& L, const louvain_params_t& p, int 
   A.mv_new = L.mv_new;
   A.logn = &h.ctl->logn;
   const int64_t hi = (bucket <= 6) ? p.deg_bounds[bucket - 1] : INT64_MAX;
-  static const char* agg_env = getenv("LV_AGG");  // diagnostics: LV_AGG=1 forces warp label merging on
-  const bool agg = agg_env && agg_env[0] == '1';
   auto dispatch = [&](int sub) -> int32_t {
     const int64_t max_deg = (sub == 0) ? std::min<int64_t>(hi, kSub1Min - 1) : hi;
     // warp-level label merging (__match_any_sync before the table insert) is
     // off: measured slower at every level and sweep of C5 (profiles/README.md)
-    if (L.w) {
-      if (agg) LV_TRY((dispatch_class<false, true>(h, L, A, bucket, sub, max_deg)));
-      else LV_TRY((dispatch_class<false, false>(h, L, A, bucket, sub, max_deg)));
-    } else {
-      if (agg) LV_TRY((dispatch_class<true, true>(h, L, A, bucket, sub, max_deg)));
-      else LV_TRY((dispatch_class<true, false>(h, L, A, bucket, sub, max_deg)));
-    }
+    if (L.w) LV_TRY((dispatch_class<false, false>(h, L, A, bucket, sub, max_deg)));
+    else LV_TRY((dispatch_class<true, false>(h, L, A, bucket, sub, max_deg)));
     if (trace_on())
       trace_step(h, L, bucket, sub, L.class_off[kSubPerBucket * bucket + sub],
                  L.class_off[kSubPerBucket * bucket + sub + 1]);
@@ -2350,9 +1491,8 @@ int32_t launch_sweep_bucket(Handle& h, Level& L, const louvain_params_t& p, int 
   // The label-partitioned hub classes (issue-bound) run on the side stream,
   // concurrently with the staging (memory-bound) and the CTA tiers of the rest of
   // the bucket: both read only the bucket-start snapshot and append to the move
-  // log; the commit waits for both.  LV_OVERLAP=0 serialises.
-  static const bool overlap_env = !(getenv("LV_OVERLAP") && getenv("LV_OVERLAP")[0] == '0');
-  const bool overlap = overlap_env && !trace_on() && posp < pos1 && posp > pos0 && L.hub.nh == 0;
+  // log; the commit waits for both (LV_TRACE=2 serialises).
+  const bool overlap = !trace_on() && posp < pos1 && posp > pos0 && L.hub.nh == 0;
   if (overlap) {
     LV_TRY(launch_stage(h, L, posp, pos1, L.class_soff[cp], L.class_soff[c1]));
     LV_CUDA(cudaEventRecord(h.ev_fork, h.stream));

@@ -349,12 +349,13 @@ def _alt_path_worker(env_items, names, q):
         gd = lv.Graph.from_csr(g.rowptr, g.col, g.w)
         lab, qq, st = gd.run(lv.params())
         out[name] = (bool(np.array_equal(lab, r.labels)), st["sweeps_per_level"] == r.sweeps_per_level,
-                     (int(qq.L), qq.S) == (r.L, r.S))
+                     (int(qq.L), qq.S) == (r.L, r.S),
+                     list(st["num_start"]) == list(r.num_start) and list(st["num_end"]) == list(r.num_end))
         # one sweep from singletons, state after it
         gd2 = lv.Graph.from_csr(g.rowptr, g.col, g.w)
         st2 = orc.State(g)
         moved = gd2.sweep(lv.params())[0]
-        out[name + "/sweep"] = (moved == st2.sweep(orc.params()), bool(np.array_equal(gd2.labels(), st2.C)), True)
+        out[name + "/sweep"] = (moved == st2.sweep(orc.params()), bool(np.array_equal(gd2.labels(), st2.C)), True, True)
     q.put(out)
 
 
@@ -363,41 +364,19 @@ def _alt_path_worker(env_items, names, q):
     (("LV_PART_MAXP", "2"),),
     # contraction: canonical sort-based variant inside louvain_run
     (("LV_CONTRACT", "sort"),),
-    # contraction: big segments through label-partitioned smem tables instead of the radix sort
-    (("LV_BIG_PART", "1"),),
-    # contraction: big segments through L2-wave global hash tables
-    (("LV_BIG_HASH", "1"),),
-    # sweep: batched table kernel for sub-class 0
-    (("LV_BATCH", "1"),),
-    # sweep: hub classes serialised with the rest of their bucket (no side stream)
-    (("LV_OVERLAP", "0"),),
-    # sweep: per-CTA global tables instead of single-CTA streaming partition tasks
-    (("LV_GTAB", "1"),),
-    (("LV_GTAB", "1"), ("LV_GTAB_AGG", "1")),
-    # sweep: cluster (DSMEM) streaming groups instead of single-CTA streaming tasks
-    (("LV_CLU", "1"),),
-    (("LV_CLU", "1"), ("LV_STREAM_MAXP", "100000")),
-    # sweep: every hub vertex on the streaming path (no pre-partitioned prefix)
-    (("LV_STREAM_MAXP", "100000"),),
-    # sweep: full-table scans instead of claimed-slot lists; lists on the CTA tiers
-    (("LV_LIST", "0"),),
-    (("LV_LIST_CTA", "1"),),
-    # contraction: batched 32-bit sorts of the big segments
-    (("LV_BIG_SORT32", "1"),),
-    # contraction: keys-only sort with packed weights instead of the 64-bit key/value sort
-    (("LV_BIG_PACK", "1"),),
-    # contraction: segmented sort of neighbour keys instead of the flat 64-bit sort
-    (("LV_BIG_SEG", "1"),),
-    # contraction: shared-memory combiner before the big-segment sort (forced on / off)
-    (("LV_BIG_COMBINE", "1"),),
-    (("LV_BIG_COMBINE", "0"),),
-    (("LV_BIG_COMBINE", "1"), ("LV_COMB_FUSED", "1")),
+    # modularity after every sweep by the full pass of Eq. (1) instead of the delta pass
+    (("LV_MOD_DELTA", "0"),),
+    # delta pass gated on moved entries <= nnz / 4: the device-side choice between
+    # the delta and the full pass, and the moved-degree sum in k_commit
+    (("LV_DELTA_DIV", "4"),),
+    # serialised per-class timing (no side stream for the hub classes)
+    (("LV_TRACE", "2"),),
 ])
 def test_alternative_paths_match_oracle(env):
     import torch.multiprocessing as tmp
     ctx = tmp.get_context("spawn")
     q = ctx.Queue()
-    names = ["hubs", "giant_hub", "weighted_loops"]
+    names = ["karate", "rmat15", "lfr5k", "hubs", "giant_hub", "weighted_loops"]
     pr = ctx.Process(target=_alt_path_worker, args=(env, names, q))
     pr.start()
     out = q.get(timeout=900)
