@@ -205,28 +205,34 @@ def run_reference(args, rank, world):
 
 
 def run_sharded_bench(args, rank, world):
-    """N > 1: the sweep vertex-sharded over the ranks (paper_conf_ipps_naimmht17_b200.dist, SURVEY 8(e));
-    per-bucket move all-gather and per-sweep L all-reduce over NCCL; contraction redundant per rank."""
+    """N > 1: the library's distributed handle (louvain_create_csr_dist, csrc/lv_dist.cu):
+    rank r decides its edge-balanced rows, the moves of every bucket are all-gathered over NCCL and
+    committed by every rank, Eq. (1)'s L change is all-reduced; contraction replicated per rank."""
     import torch
     import torch.distributed as dist
 
     import graphgen
     import paper_conf_ipps_naimmht17_b200 as lvb
-    from paper_conf_ipps_naimmht17_b200.dist import CudaShard, run_sharded
+    from paper_conf_ipps_naimmht17_b200.dist import edge_balanced_ranges, local_rows
 
     dev = torch.device("cuda", torch.cuda.current_device())
     dg = graphgen.rmat(args.scale, seed=args.seed, device=True)
     torch.cuda.synchronize()
     n, nnz = dg.n, dg.nnz
     p = lvb.params()
-
+    comm = "nccl" if args.backend == "nccl" else "host"
     deg = dg.rowptr[1:] - dg.rowptr[:-1]
     n_act = int((deg > 0).sum().item())
+    rp_h = dg.rowptr.cpu().numpy()
+    lo, hi = edge_balanced_ranges(rp_h, world)[rank]
+    rl, cl, _ = local_rows(dg.rowptr, dg.col, None, lo, hi)
+    stream = torch.cuda.Stream()
+    g = lvb.Graph.from_csr_dist(n, lo, hi, rl.contiguous(), cl.contiguous(), None, rank=rank, world=world,
+                                comm=comm, stream=stream)
+    labels_dev = torch.empty(n, dtype=torch.int32, device=dev)
 
     def one_run():
-        g = lvb.Graph.from_csr(dg.rowptr, dg.col, borrow=True)
-        lab, st = run_sharded(CudaShard(g), p)
-        return st
+        return g.run(p, labels_out=labels_dev)[2]
 
     for _ in range(args.warmup):
         one_run()
@@ -236,44 +242,44 @@ def run_sharded_bench(args, rank, world):
         dist.barrier()
         ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         launches0 = lvb.launch_counts()[0]
-        ev0.record()
+        ev0.record(stream)
         for _ in range(args.steps):
             stats.append(one_run())
-        ev1.record()
+        ev1.record(stream)
         torch.cuda.synchronize()
         launches = lvb.launch_counts()[0] - launches0
         dist.barrier()
     ms = ev0.elapsed_time(ev1)
     t = torch.tensor([ms, statistics.mean(s_["t_sweep_ms_first"] for s_ in stats)], device=dev,
                      dtype=torch.float64)
-    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)  # the slowest rank
     ms_per_step = float(t[0].item()) / args.steps
     t_sw1 = float(t[1].item())  # slowest rank's level-0 sweep 1 (incl. the per-bucket exchanges)
     st0 = stats[0]
-    edges_per_run = sum(nz * sw for nz, sw in zip(st0["nnz"], st0["sweeps_per_level"]))
+    edges_per_run = st0["edges_swept"]
     # roofline per GPU: the byte model of the sweep split over edge-balanced ranks
     B = sweep_bytes(n_act, nnz, D=nnz, moved=st0["moved_first"]) / world
     achieved = B / (t_sw1 / 1e3) / 1e9
     peak, peak_src = measured_peak_hbm()
-    traffic, traffic_src = recorded_traffic() if args.scale == 27 else (None, None)  # the capture is of C5
     roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-                "traffic": traffic / world if traffic else None,
+                "traffic": None,
                 "kernel": "level-0 sweep 1 body per GPU (bucket kernels + commits + move all-gathers)",
                 "algorithmic_bytes": B, "t_ms": t_sw1, "peak_source": peak_src,
-                "traffic_source": (traffic_src + " (1-GPU capture / N)") if traffic else None}
-    # end to end: every rank uploads the CSR from pinned host memory, runs, reads the labels back
-    h_rowptr = torch.empty(n + 1, dtype=torch.int64, pin_memory=True)
-    h_col = torch.empty(nnz, dtype=torch.int32, pin_memory=True)
-    h_rowptr.copy_(dg.rowptr)
-    h_col.copy_(dg.col)
+                "traffic_source": "not captured at N > 1 (ncu runs on one GPU)"}
+    del g
+    # end to end: every rank uploads its rows from pinned host memory, runs, reads the labels back
+    h_rl = torch.empty(rl.numel(), dtype=torch.int64, pin_memory=True)
+    h_cl = torch.empty(cl.numel(), dtype=torch.int32, pin_memory=True)
+    h_lab = torch.empty(n, dtype=torch.int32, pin_memory=True)
+    h_rl.copy_(rl)
+    h_cl.copy_(cl)
     e2e_s = []
     for it in range(max(0, args.e2e_warmup) + max(1, args.e2e_steps)):
         dist.barrier()
         torch.cuda.synchronize()
         t0 = time.perf_counter()
-        with lvb.Graph.from_csr(h_rowptr, h_col) as ge:
-            lab, _ = run_sharded(CudaShard(ge), p)
-            lab_h = lab.cpu() if hasattr(lab, "cpu") else lab
+        with lvb.Graph.from_csr_dist(n, lo, hi, h_rl, h_cl, None, rank=rank, world=world, comm=comm) as ge:
+            ge.run(p, labels_out=h_lab)
         torch.cuda.synchronize()
         if it >= max(0, args.e2e_warmup):
             e2e_s.append(time.perf_counter() - t0)
@@ -286,13 +292,15 @@ def run_sharded_bench(args, rank, world):
            "config": {"workload": f"{cfg_name(args.scale)} R-MAT scale {args.scale}, {8 << args.scale} tuples, seed {args.seed}, "
                                   "unit weights, isolated vertices removed",
                       "n": n, "nnz": nnz, "l2": "inputs larger than L2",
-                      "parallelism": f"{world} GPUs, sweep vertex-sharded (edge-balanced ranges), "
-                                     "per-bucket NCCL all-gather of moves, per-sweep L all-reduce"},
+                      "parallelism": f"{world} GPUs, sweep vertex-sharded (edge-balanced ranges), per-bucket "
+                                     f"{'NCCL' if comm == 'nccl' else 'host-staged'} all-gather of moves, "
+                                     "per-sweep all-reduce of the L change"},
            "roofline": roofline, "clocks": clk.summary(), "gpu_launches": int(launches),
-           "q_final": st0["q"] if "q" in st0 else None, "levels": st0["levels"],
+           "q_final": st0["q"], "levels": st0["levels"],
            "sweeps_per_level": st0["sweeps_per_level"], "louvain_wall_ms": ms_per_step,
            "sweep1_ms": t_sw1,
-           "e2e": {"value": edges_per_run / t_e2e, "unit": UNIT, "h2d_bytes_per_step": 8 * (n + 1) + 4 * nnz,
+           "e2e": {"value": edges_per_run / t_e2e, "unit": UNIT,
+                   "h2d_bytes_per_step": 8 * (hi - lo + 1) + 4 * int(cl.numel()),
                    "d2h_bytes_per_step": 4 * n, "ms_per_step": 1e3 * t_e2e}}
     if rank == 0:
         emit(out)

@@ -137,6 +137,12 @@ int32_t louvain_run(louvain_graph_t g, const louvain_params_t* p, int32_t* label
                     louvain_stats_t* stats);
 /* Thread-local message of the last error ("" if none). */
 const char* louvain_last_error(void);
+/* Free the device memory the library keeps between handles: the scratch
+ * buffers of the most recently destroyed handle per device (reused by the next
+ * handle; bounded to one handle's set per device) and the idle blocks of the
+ * library's private stream-ordered memory pool.  Never needed for correctness:
+ * an allocation failure releases both and retries once. */
+int32_t louvain_release_cache(void);
 /* Process-wide counters of the kernels (and CUB device calls) this library has
  * launched so far, on every handle; either pointer may be NULL.  Diagnostics:
  * the difference around a call counts its launches (louvain_stats_t reports
@@ -173,6 +179,57 @@ int32_t louvain_compose_labels(int32_t* lab, int64_t n0, const int32_t* map, voi
 /* Eq. (1) parts of the current partition with L summed over the owned rows
  * only (the ranks' L add up to the graph's L); S and W are global. */
 int32_t louvain_modularity_owned(louvain_graph_t g, uint64_t* L_owned, uint64_t* S, uint64_t* W);
+
+/* ---- multi-GPU: the vertex-sharded run inside the library ----
+ * One process per GPU, one distributed handle per rank.  Every bucket decides on
+ * one snapshot (Alg. 1 l.6-7), so rank r runs computeMove (Alg. 2) for
+ * its own edge-balanced vertex range only; after each bucket the ranks' moves
+ * are all-gathered and every rank commits all of them to its replica of
+ * (C, a_c, size_c) with the same exact integer updates (Alg. 1 l.8-11), so the
+ * replicas stay bit-identical; Eq. (1) after a sweep is all-reduced (partial L
+ * change of the owned moved rows).  The level graph is replicated on every rank
+ * and contraction (Alg. 3) is computed on each (deterministic, identical).
+ * Every louvain_* call on a distributed handle that runs a sweep
+ * (louvain_sweep, louvain_run) is COLLECTIVE over its ranks; the other calls are
+ * local.  Results equal the single-GPU ones bit for bit (and oracle (b)).
+ * The per-bucket primitives above must not be used on a distributed handle. */
+
+/* Host-side transport: both callbacks get host buffers and return 0 on success.
+ * allgather: every rank contributes `bytes` bytes from `send`; `recv` receives
+ * world * bytes, rank-major.  allreduce_u64: in-place sum of `count` uint64
+ * values over the ranks (modular).  Used with any process group (e.g. gloo), and
+ * where NCCL cannot run (several ranks sharing one GPU). */
+typedef struct {
+  void* user;
+  int32_t (*allgather)(void* user, const void* send, void* recv, int64_t bytes);
+  int32_t (*allreduce_u64)(void* user, uint64_t* data, int64_t count);
+} louvain_host_comm_t;
+
+/* A new NCCL unique id (128 bytes) for louvain_create_csr_dist; call on one rank
+ * and broadcast it (e.g. torch.distributed.broadcast_object_list).
+ * Errors: UNSUPPORTED (libnccl.so.2 cannot be loaded), NCCL. */
+int32_t louvain_dist_unique_id(uint8_t id[128]);
+/* Collective over `world` ranks.  Rank `rank` passes its rows [v_begin, v_end)
+ * of the n-vertex graph (the ranks' ranges contiguous in rank order and covering
+ * [0, n)): rowptr_local[v_end - v_begin + 1] starting at 0, col_local (GLOBAL
+ * column ids) and w_local (NULL on every rank = unit weights), host or device.
+ * The handle is bound to the current device and to cuda_stream; NCCL
+ * communicator from `id`.  flags: LOUVAIN_VALIDATE (the assembled graph).
+ * louvain_dist_ranges gives the edge-balanced ranges the library itself uses for
+ * contracted levels.  Errors: INVALID_ARG (ranges / n / weights disagree across
+ * ranks), INVALID_GRAPH, OVERFLOW, NOMEM, CUDA, NCCL, UNSUPPORTED. */
+int32_t louvain_create_csr_dist(int64_t n, int64_t v_begin, int64_t v_end, const int64_t* rowptr_local,
+                                const int32_t* col_local, const uint32_t* w_local, uint32_t flags, int32_t rank,
+                                int32_t world, const uint8_t id[128], void* cuda_stream, louvain_graph_t* out);
+/* Same, with the host-side transport `comm` (copied; the callbacks and `user`
+ * must stay valid for the handle's lifetime). */
+int32_t louvain_create_csr_dist_host(int64_t n, int64_t v_begin, int64_t v_end, const int64_t* rowptr_local,
+                                     const int32_t* col_local, const uint32_t* w_local, uint32_t flags,
+                                     int32_t rank, int32_t world, const louvain_host_comm_t* comm,
+                                     void* cuda_stream, louvain_graph_t* out);
+/* Host-only (no device work): edge-balanced contiguous ranges of a CSR,
+ * bounds[world + 1]: bounds[r] = first row u with rowptr[u] >= r*nnz/world. */
+int32_t louvain_dist_ranges(int64_t n, const int64_t* rowptr, int32_t world, int64_t* bounds);
 
 #ifdef __cplusplus
 }

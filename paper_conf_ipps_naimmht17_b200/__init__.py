@@ -72,6 +72,15 @@ class Stats(ctypes.Structure):
                 "W": int(self.q.W)}
 
 
+# host-side transport of the distributed handle (louvain_host_comm_t)
+HOST_ALLGATHER = ctypes.CFUNCTYPE(ctypes.c_int32, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int64)
+HOST_ALLREDUCE = ctypes.CFUNCTYPE(ctypes.c_int32, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int64)
+
+
+class HostComm(ctypes.Structure):
+    _fields_ = [("user", ctypes.c_void_p), ("allgather", HOST_ALLGATHER), ("allreduce_u64", HOST_ALLREDUCE)]
+
+
 FUNCS = {
     # name: (restype, argtypes)
     "louvain_params_default": (None, [ctypes.POINTER(Params)]),
@@ -101,6 +110,18 @@ FUNCS = {
     "louvain_compose_labels": (ctypes.c_int32, [ctypes.c_void_p, ctypes.c_int64, ctypes.c_void_p, ctypes.c_void_p]),
     "louvain_modularity_owned": (ctypes.c_int32, [ctypes.c_void_p, ctypes.POINTER(ctypes.c_uint64),
                                                   ctypes.POINTER(ctypes.c_uint64), ctypes.POINTER(ctypes.c_uint64)]),
+    "louvain_release_cache": (ctypes.c_int32, []),
+    "louvain_dist_unique_id": (ctypes.c_int32, [ctypes.c_void_p]),
+    "louvain_create_csr_dist": (ctypes.c_int32, [ctypes.c_int64, ctypes.c_int64, ctypes.c_int64, ctypes.c_void_p,
+                                                 ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint32, ctypes.c_int32,
+                                                 ctypes.c_int32, ctypes.c_void_p, ctypes.c_void_p,
+                                                 ctypes.POINTER(ctypes.c_void_p)]),
+    "louvain_create_csr_dist_host": (ctypes.c_int32, [ctypes.c_int64, ctypes.c_int64, ctypes.c_int64,
+                                                      ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p,
+                                                      ctypes.c_uint32, ctypes.c_int32, ctypes.c_int32,
+                                                      ctypes.POINTER(HostComm), ctypes.c_void_p,
+                                                      ctypes.POINTER(ctypes.c_void_p)]),
+    "louvain_dist_ranges": (ctypes.c_int32, [ctypes.c_int64, ctypes.c_void_p, ctypes.c_int32, ctypes.c_void_p]),
 }
 
 _LIB = None
@@ -195,6 +216,41 @@ class Graph:
         _check(lib().louvain_create_csr(n, nnz, rp, cp if nnz else None, wp, flags, sp, ctypes.byref(h)))
         g = cls(h, stream)
         g._borrowed = (rowptr, col, w) if borrow else None
+        return g
+
+    @classmethod
+    def from_csr_dist(cls, n: int, v_begin: int, v_end: int, rowptr_local, col_local, w_local=None, *,
+                      rank: int, world: int, comm: str = "nccl", group=None, validate: bool = False,
+                      stream=None) -> "Graph":
+        """Distributed handle (collective over the `world` ranks of `group`): this rank's rows
+        [v_begin, v_end) with global column ids; see include/louvain.h.  comm="nccl": NCCL
+        communicator, its unique id broadcast from rank 0 through torch.distributed;
+        comm="host": the library's host-side transport over torch.distributed (e.g. gloo)."""
+        from . import dist as _dist
+        rowptr_local = _as(rowptr_local, np.int64)
+        col_local = _as(col_local, np.int32)
+        w_local = _as(w_local, np.uint32)
+        rp, k1 = _ptr(rowptr_local)
+        cp, k2 = _ptr(col_local)
+        wp, k3 = _ptr(w_local)
+        sp = None
+        if stream is not None:
+            sp = stream.cuda_stream if hasattr(stream, "cuda_stream") else int(stream)
+        flags = VALIDATE if validate else 0
+        h = ctypes.c_void_p()
+        keep = None
+        if comm == "nccl":
+            uid = _dist.nccl_unique_id(rank, group)
+            _check(lib().louvain_create_csr_dist(n, v_begin, v_end, rp, cp, wp, flags, rank, world, uid, sp,
+                                                 ctypes.byref(h)))
+        elif comm == "host":
+            keep = _dist.host_comm(group)
+            _check(lib().louvain_create_csr_dist_host(n, v_begin, v_end, rp, cp, wp, flags, rank, world,
+                                                      ctypes.byref(keep), sp, ctypes.byref(h)))
+        else:
+            raise ValueError("comm must be 'nccl' or 'host'")
+        g = cls(h, stream)
+        g._comm_keep = keep  # the callbacks must outlive the handle
         return g
 
     @classmethod
@@ -335,6 +391,19 @@ def run(rowptr, col, w=None, p: Optional[Params] = None, **kw):
     """One-call convenience: CSR in (host or device), (labels, QNum, stats) out."""
     with Graph.from_csr(rowptr, col, w, **kw) as g:
         return g.run(p)
+
+
+def release_cache() -> None:
+    """Free the device memory kept between handles (scratch cache, idle pool blocks)."""
+    _check(lib().louvain_release_cache())
+
+
+def dist_ranges(rowptr, world: int) -> list[tuple[int, int]]:
+    """Edge-balanced contiguous row ranges (host-only C helper, no GPU needed)."""
+    rowptr = np.ascontiguousarray(rowptr, dtype=np.int64)
+    b = np.zeros(world + 1, dtype=np.int64)
+    _check(lib().louvain_dist_ranges(len(rowptr) - 1, rowptr.ctypes.data, world, b.ctypes.data))
+    return [(int(b[r]), int(b[r + 1])) for r in range(world)]
 
 
 def launch_counts() -> tuple[int, int]:

@@ -33,32 +33,40 @@ int32_t cuda_fail(cudaError_t e, const char* what, const char* file, int line) {
   return LOUVAIN_E_CUDA;
 }
 
-int32_t dmalloc(void** p, size_t bytes, cudaStream_t s) {
-  *p = nullptr;
-  cudaError_t e = cudaMallocAsync(p, bytes ? bytes : 1, s);
-  if (e != cudaSuccess) {
-    cudaGetLastError();
-    g_err = "device allocation of " + std::to_string(bytes) + " bytes failed: " + cudaGetErrorString(e);
-    return LOUVAIN_E_NOMEM;
-  }
-  return LOUVAIN_OK;
-}
-
-void dfree(void* p, cudaStream_t s) {
-  if (p) cudaFreeAsync(p, s);
-}
-
-int32_t scratch_size(Handle& h, int slot, size_t* bytes) {
-  *bytes = h.scratch.bytes[slot];
-  return LOUVAIN_OK;
-}
-
-// Process-wide cache of scratch buffers released by destroyed handles (per
-// device), so a new handle on the same device -- e.g. every end-to-end call of
-// louvain_create_csr + louvain_run -- reuses device memory instead of paying
-// tens of GB of cudaMalloc again.  LV_SCRATCH_CACHE=0 disables it; an allocation
-// failure releases the cache and retries.
+// Stream-ordered allocations come from a library-private memory pool per device
+// (never the device's default pool, which other libraries in the process share):
+// it keeps freed blocks (release threshold = max) so per-level temporaries do not
+// go back to the driver between levels, and it is trimmed when an allocation fails.
 namespace {
+std::mutex g_pool_mu;
+cudaMemPool_t g_pools[64] = {};
+cudaMemPool_t lib_pool(int dev) {
+  if (dev < 0 || dev >= 64) return nullptr;
+  std::lock_guard<std::mutex> lk(g_pool_mu);
+  if (!g_pools[dev]) {
+    cudaMemPoolProps pr = {};
+    pr.allocType = cudaMemAllocationTypePinned;
+    pr.handleTypes = cudaMemHandleTypeNone;
+    pr.location.type = cudaMemLocationTypeDevice;
+    pr.location.id = dev;
+    cudaMemPool_t p = nullptr;
+    if (cudaMemPoolCreate(&p, &pr) != cudaSuccess) {
+      cudaGetLastError();
+      return nullptr;
+    }
+    uint64_t thr = UINT64_MAX;
+    cudaMemPoolSetAttribute(p, cudaMemPoolAttrReleaseThreshold, &thr);
+    g_pools[dev] = p;
+  }
+  return g_pools[dev];
+}
+
+// Process-wide cache of the scratch buffers of destroyed handles, so a new handle
+// on the same device (e.g. every end-to-end louvain_create_csr + louvain_run)
+// reuses device memory instead of paying tens of GB of cudaMalloc again.  Bounded:
+// it holds the buffers of the most recently destroyed handle per device only (a
+// destroy releases what an earlier one left).  Released on any allocation
+// failure, by louvain_release_cache(), or never filled with LV_SCRATCH_CACHE=0.
 std::mutex g_cache_mu;
 std::vector<std::tuple<int, void*, size_t>> g_cache;  // (device, ptr, bytes)
 bool cache_on() {
@@ -80,18 +88,67 @@ void* cache_take(int dev, size_t bytes, size_t* got) {
   g_cache.erase(g_cache.begin() + best);
   return p;
 }
-void cache_release(int dev) {
-  std::lock_guard<std::mutex> lk(g_cache_mu);
+void cache_release_locked(int dev) {
   for (auto it = g_cache.begin(); it != g_cache.end();) {
-    if (std::get<0>(*it) == dev) {
+    if (dev < 0 || std::get<0>(*it) == dev) {
+      int cur = -1;
+      cudaGetDevice(&cur);
+      if (cur != std::get<0>(*it)) cudaSetDevice(std::get<0>(*it));
       cudaFree(std::get<1>(*it));
+      if (cur >= 0 && cur != std::get<0>(*it)) cudaSetDevice(cur);
       it = g_cache.erase(it);
     } else {
       ++it;
     }
   }
 }
+void cache_release(int dev) {
+  std::lock_guard<std::mutex> lk(g_cache_mu);
+  cache_release_locked(dev);
+}
+// Give memory back after an allocation failure: the scratch cache and the idle
+// blocks of the library pool (after the stream's queued frees have run).
+void reclaim(int dev, cudaStream_t s) {
+  cudaGetLastError();
+  cache_release(dev);
+  if (cudaMemPool_t p = lib_pool(dev)) {
+    if (s) cudaStreamSynchronize(s);
+    cudaMemPoolTrimTo(p, 0);
+  }
+  cudaGetLastError();
+}
 }  // namespace
+
+int32_t dmalloc(void** p, size_t bytes, cudaStream_t s) {
+  *p = nullptr;
+  int dev = 0;
+  cudaGetDevice(&dev);
+  cudaMemPool_t pool = lib_pool(dev);
+  auto alloc = [&]() {
+    return pool ? cudaMallocFromPoolAsync(p, bytes ? bytes : 1, pool, s) : cudaMallocAsync(p, bytes ? bytes : 1, s);
+  };
+  cudaError_t e = alloc();
+  if (e != cudaSuccess) {  // retry once after giving cached / pooled memory back
+    reclaim(dev, s);
+    e = alloc();
+  }
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    *p = nullptr;
+    g_err = "device allocation of " + std::to_string(bytes) + " bytes failed: " + cudaGetErrorString(e);
+    return LOUVAIN_E_NOMEM;
+  }
+  return LOUVAIN_OK;
+}
+
+void dfree(void* p, cudaStream_t s) {
+  if (p) cudaFreeAsync(p, s);
+}
+
+int32_t scratch_size(Handle& h, int slot, size_t* bytes) {
+  *bytes = h.scratch.bytes[slot];
+  return LOUVAIN_OK;
+}
 
 int32_t scratch_get(Handle& h, int slot, size_t bytes, void** out) {
   Scratch& S = h.scratch;
@@ -111,13 +168,7 @@ int32_t scratch_get(Handle& h, int slot, size_t bytes, void** out) {
       const size_t want = bytes + bytes / 8;  // headroom: later levels are usually smaller
       cudaError_t e = cudaMalloc(&S.p[slot], want);
       if (e != cudaSuccess) {  // give cached buffers and pooled stream-ordered memory back, retry once
-        cudaGetLastError();
-        cache_release(h.device);
-        cudaMemPool_t pool;
-        if (cudaDeviceGetDefaultMemPool(&pool, h.device) == cudaSuccess) {
-          cudaStreamSynchronize(h.stream);
-          cudaMemPoolTrimTo(pool, 0);
-        }
+        reclaim(h.device, h.stream);
         e = cudaMalloc(&S.p[slot], want);
       }
       if (e != cudaSuccess) {
@@ -135,17 +186,27 @@ int32_t scratch_get(Handle& h, int slot, size_t bytes, void** out) {
 }
 
 void scratch_free(Handle& h) {
+  std::lock_guard<std::mutex> lk(g_cache_mu);
+  if (cache_on()) cache_release_locked(h.device);  // bounded: one handle's set per device
   for (int i = 0; i < SC_COUNT; ++i) {
     if (h.scratch.p[i]) {
-      if (cache_on()) {
-        std::lock_guard<std::mutex> lk(g_cache_mu);
-        g_cache.emplace_back(h.device, h.scratch.p[i], h.scratch.bytes[i]);
-      } else {
-        cudaFree(h.scratch.p[i]);
-      }
+      if (cache_on()) g_cache.emplace_back(h.device, h.scratch.p[i], h.scratch.bytes[i]);
+      else cudaFree(h.scratch.p[i]);
     }
     h.scratch.p[i] = nullptr;
     h.scratch.bytes[i] = 0;
+  }
+}
+
+void release_cache_all() {
+  cache_release(-1);
+  for (int d = 0; d < 64; ++d) {
+    cudaMemPool_t p = nullptr;
+    {
+      std::lock_guard<std::mutex> lk(g_pool_mu);
+      p = g_pools[d];
+    }
+    if (p) cudaMemPoolTrimTo(p, 0);
   }
 }
 
@@ -166,17 +227,6 @@ __global__ void k_fill_u32(uint32_t* p, int64_t n, uint32_t v) {
 }
 __global__ void k_iota(int32_t* p, int64_t n) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) p[i] = (int32_t)i;
-}
-
-void keep_pool_memory(int device) {
-  static bool done[64] = {false};
-  if (device < 0 || device >= 64 || done[device]) return;
-  cudaMemPool_t pool;
-  if (cudaDeviceGetDefaultMemPool(&pool, device) == cudaSuccess) {
-    uint64_t thr = UINT64_MAX;
-    cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
-  }
-  done[device] = true;
 }
 
 int32_t check_params(const louvain_params_t& p) {
@@ -203,7 +253,6 @@ int32_t check_params(const louvain_params_t& p) {
 
 int32_t init_handle(Handle& h, void* stream) {
   LV_CUDA(cudaGetDevice(&h.device));
-  keep_pool_memory(h.device);
   if (stream) {
     h.stream = (cudaStream_t)stream;
     h.own_stream = false;
@@ -223,6 +272,7 @@ int32_t init_handle(Handle& h, void* stream) {
 
 void destroy_handle(Handle& h) {
   cudaSetDevice(h.device);
+  dist_free(h);
   if (h.stream) {
     level_free(h.lv, h.stream);
     cudaStreamSynchronize(h.stream);
@@ -280,6 +330,11 @@ int32_t finish_call(Handle& h, int32_t rc) {
 bool bucket_nonempty(const Level& L, int b) {
   return L.class_off[kSubPerBucket * (b + 1)] > L.class_off[kSubPerBucket * b];
 }
+// On a distributed handle every rank runs the same sequence of commits and
+// exchanges: a bucket counts if any rank owns one of its vertices.
+bool bucket_active(const Handle& h, const Level& L, int b) {
+  return h.dist ? h.dist->cap[b] > 0 : bucket_nonempty(L, b);
+}
 
 // One sweep body: for each non-empty bucket 1..7 its sweep kernels, then its
 // commit (BIN_SYNC) -- or a single commit at the end (RELAXED).
@@ -288,11 +343,14 @@ int32_t sweep_body(Handle& h, Level& L, const louvain_params_t& p) {
   LV_CUDA(cudaMemsetAsync(h.ctl, 0, offsetof(DevCtl, L), h.stream));  // logn + bounds
   int commits = 0;
   for (int b = 1; b <= 7; ++b) {
-    if (!bucket_nonempty(L, b)) continue;
+    if (!bucket_active(h, L, b)) continue;
     auto t0 = std::chrono::steady_clock::now();
     LV_TRY(launch_sweep_bucket(h, L, p, b));
     auto t1 = std::chrono::steady_clock::now();
-    if (p.mode == LOUVAIN_MODE_BIN_SYNC) LV_TRY(launch_commit(h, L, commits++));
+    if (p.mode == LOUVAIN_MODE_BIN_SYNC) {
+      if (h.dist) LV_TRY(dist_exchange(h, L, commits, b));  // every rank's bucket-b moves
+      LV_TRY(launch_commit(h, L, commits++));
+    }
     if (trace) {
       cudaStreamSynchronize(h.stream);
       auto t2 = std::chrono::steady_clock::now();
@@ -302,7 +360,10 @@ int32_t sweep_body(Handle& h, Level& L, const louvain_params_t& p) {
               (long)(L.class_off[kSubPerBucket * (b + 1)] - L.class_off[kSubPerBucket * b]));
     }
   }
-  if (p.mode == LOUVAIN_MODE_RELAXED) LV_TRY(launch_commit(h, L, commits++));
+  if (p.mode == LOUVAIN_MODE_RELAXED) {
+    if (h.dist) LV_TRY(dist_exchange(h, L, 0, 0));
+    LV_TRY(launch_commit(h, L, commits++));
+  }
   ++L.sweeps_done;
   return LOUVAIN_OK;
 }
@@ -358,6 +419,19 @@ float elapsed(cudaEvent_t a, cudaEvent_t b) {
   return ms;
 }
 
+// Eq. (1) parts of the level's own partition; on a distributed handle each rank
+// sums the entries of its rows and L is all-reduced (S from the replicated a_c).
+int32_t modularity_parts(Handle& h, Level& L, bool singletons, uint64_t* Lout, uint64_t* Sout) {
+  if (!h.dist) return level_modularity(h, L, nullptr, Lout, Sout, singletons);
+  LV_TRY(launch_modularity(h, L, nullptr, singletons));
+  LV_TRY(dist_allreduce(h, &h.ctl->L, 1));
+  LV_CUDA(cudaMemcpyAsync(h.h_ctl, h.ctl, sizeof(DevCtl), cudaMemcpyDeviceToHost, h.stream));
+  LV_CUDA(cudaStreamSynchronize(h.stream));
+  *Lout = h.h_ctl->L;
+  *Sout = h.h_ctl->S;
+  return LOUVAIN_OK;
+}
+
 // The multilevel driver (SURVEY 8(c) listing; oracle/louvain_oracle.c orc_louvain
 // is the independent CPU transcription of the same control flow).
 int32_t run_impl(Handle& h, const louvain_params_t& p, int32_t* labels_out, louvain_qnum_t* q_final,
@@ -370,44 +444,61 @@ int32_t run_impl(Handle& h, const louvain_params_t& p, int32_t* labels_out, louv
   std::memset(&local, 0, sizeof local);
   auto t_begin = std::chrono::steady_clock::now();
   const long long launches0 = g_launches, cub0 = g_cub_calls;
-  int32_t* lab = nullptr;
-  LV_TRY(dalloc(&lab, n0, s));
+  // Every device resource of the run is owned by `R`, so each return path
+  // (errors included) frees it and leaves no dangling pointer in the handle.
+  struct RunRes {
+    Handle& h;
+    int32_t* lab = nullptr;  // original vertex -> current community (R22)
+    uint2* pcn = nullptr;    // {label at the sweep start, label now} (delta pass of Eq. (1))
+    int32_t* map = nullptr;  // contraction map of the current level
+    Level owned;             // current contracted level (levels >= 1)
+    bool has_owned = false;
+    cudaEvent_t e0 = nullptr, e1 = nullptr;
+    explicit RunRes(Handle& hh) : h(hh) {}
+    ~RunRes() {
+      h.pcn = nullptr;
+      dfree(lab, h.stream);
+      dfree(pcn, h.stream);
+      dfree(map, h.stream);
+      if (has_owned) level_free(owned, h.stream);
+      if (e0) cudaEventDestroy(e0);
+      if (e1) cudaEventDestroy(e1);
+    }
+  } R(h);
+  LV_TRY(dalloc(&R.lab, n0, s));
+  int32_t* const lab = R.lab;
   // labels at each sweep start, for the delta pass of Eq. (1) (LV_MOD_DELTA=0: full passes only)
   static const bool mod_delta = !(getenv("LV_MOD_DELTA") && getenv("LV_MOD_DELTA")[0] == '0');
-  struct PcnGuard {  // h.pcn lives for this run only
-    Handle& h;
-    ~PcnGuard() { h.pcn = nullptr; }
-  } pcn_guard{h};
-  uint2* pcn = nullptr;
-  if (mod_delta) LV_TRY(dalloc(&pcn, std::max<int64_t>(n0, 1), s));
+  if (mod_delta) LV_TRY(dalloc(&R.pcn, std::max<int64_t>(n0, 1), s));
+  uint2* const pcn = R.pcn;
+  LV_CUDA(cudaEventCreate(&R.e0));
+  LV_CUDA(cudaEventCreate(&R.e1));
+  cudaEvent_t e_lvl0 = R.e0, e_lvl1 = R.e1;
   if (n0) { k_iota<<<grid_for(n0, 256), 256, 0, s>>>(lab, n0); LV_LAUNCHED(); }
   // level 0 starts from singletons; a full run owns every vertex.  The
   // degree binning (a2) is redone by every run -- nothing of a previous run is
   // reused, so a timed run includes every step of the path.
-  L0.own_hi = -1;
+  if (!h.dist) L0.own_hi = -1;  // a distributed handle keeps its rows (set per level below)
   L0.bins_valid = false;
   if (n0) LV_TRY(level_set_labels(h, L0, nullptr));
   uint64_t Lq = 0, Sq = 0;  // exact parts of the current level's kept partition
-  Level owned;   // current contracted level (levels >= 1)
   Level* cur = &L0;
-  int32_t* map = nullptr;
   Trace tr;
   if (W > 0) {
     for (int level = 0;; ++level) {
       if ((p.max_levels > 0 && level >= p.max_levels) || level >= LOUVAIN_MAX_LEVELS) break;
-      cudaEvent_t e_lvl0, e_lvl1;
-      cudaEventCreate(&e_lvl0);
-      cudaEventCreate(&e_lvl1);
       cudaEventRecord(e_lvl0, s);
       Level& L = *cur;
       const int pexp = (L.n > p.size_limit) ? p.th_bin_exp : p.th_final_exp;  // P:330, R14
       tr.mark(s, "start", level);
+      if (h.dist) LV_TRY(dist_set_level_range(h, L, level));
       LV_TRY(level_binning(h, L, p));
+      if (h.dist) LV_TRY(dist_after_binning(h, L));
       tr.mark(s, "binning", level);
       // level start: singletons.  Level 0 evaluates Eq. (1); a contracted level
       // starts exactly where the previous one ended (contraction preserves L and
       // S, R18 -- pinned by the oracle tests and the parity suite).
-      if (level == 0) LV_TRY(level_modularity(h, L, nullptr, &Lq, &Sq, /*singletons=*/true));
+      if (level == 0) LV_TRY(modularity_parts(h, L, /*singletons=*/true, &Lq, &Sq));
       const int64_t num_start = qnum_of(Lq, Sq, W);
       int64_t num_prev = num_start;
       int64_t moved_level = 0;
@@ -422,6 +513,10 @@ int32_t run_impl(Handle& h, const louvain_params_t& p, int32_t* labels_out, louv
         tr.mark(s, "sweep", level);
         if (mod_delta) LV_TRY(launch_modularity_delta(h, L));
         else LV_TRY(launch_modularity(h, L, nullptr));
+        if (h.dist) {  // the ranks' parts: overflow flags and L change (delta pass) / L (full pass)
+          LV_TRY(dist_allreduce(h, &h.ctl->overflow, 2));
+          if (!mod_delta) LV_TRY(dist_allreduce(h, &h.ctl->L, 1));
+        }
         cudaEventRecord(h.ev[2], s);
         tr.mark(s, "modularity", level);
         LV_CUDA(cudaMemcpyAsync(h.h_ctl, h.ctl, sizeof(DevCtl), cudaMemcpyDeviceToHost, s));
@@ -473,14 +568,13 @@ int32_t run_impl(Handle& h, const louvain_params_t& p, int32_t* labels_out, louv
       local.t_opt_ms[level] = elapsed(e_lvl0, e_lvl1);
       if (moved_level == 0 || below_threshold(num_end, num_start, W, p.th_final_exp)) {  // R16
         LV_TRY(compose_labels_ca(h, lab, n0, L.ca));
-        cudaEventDestroy(e_lvl0);
-        cudaEventDestroy(e_lvl1);
         break;
       }
       // aggregation phase (Alg. 3)
       cudaEventRecord(e_lvl0, s);
-      Level next;
-      LV_TRY(dalloc(&map, L.n, s));
+      Level next;  // scratch-backed (parity buffers); its plans are freed with it below
+      LV_TRY(dalloc(&R.map, L.n, s));
+      int32_t* const map = R.map;
       tr.mark(s, "pre-contract", level);
       // mergeCommunity-style grouping + hashing (default, NEXT-1) or the canonical sort-based one (LV_CONTRACT=sort)
       static const bool hash_contract = !(getenv("LV_CONTRACT") && std::string(getenv("LV_CONTRACT")) == "sort");
@@ -488,34 +582,33 @@ int32_t run_impl(Handle& h, const louvain_params_t& p, int32_t* labels_out, louv
       else LV_TRY(level_contract(h, L, next, map, (level + 1) & 1));
       tr.mark(s, "contract", level);
       LV_TRY(compose_labels(h, lab, n0, map));
-      dfree(map, s);
-      map = nullptr;
+      dfree(R.map, s);
+      R.map = nullptr;
       LV_TRY(level_setup(h, next));
       tr.mark(s, "setup", level);
       cudaEventRecord(e_lvl1, s);
       LV_CUDA(cudaEventSynchronize(e_lvl1));
       local.t_agg_ms[level] = elapsed(e_lvl0, e_lvl1);
-      cudaEventDestroy(e_lvl0);
-      cudaEventDestroy(e_lvl1);
-      if (cur != &L0) level_free(owned, s);
-      owned = next;
-      cur = &owned;
+      if (R.has_owned) level_free(R.owned, s);
+      R.owned = next;
+      R.has_owned = true;
+      cur = &R.owned;
     }
   }
   // the handle's partition becomes the final one; (Lq, Sq) are the exact parts of
   // the last level's kept partition, equal to those of `lab` on the input graph
   bool final_set = false;
-  if (cur != &L0 && owned.n <= kFinalHistMax) {  // totals from the last level, sizes by an smem histogram
-    LV_TRY(level_set_final(h, L0, lab, owned.ca, owned.n));
+  if (R.has_owned && R.owned.n <= kFinalHistMax) {  // totals from the last level, sizes by an smem histogram
+    LV_TRY(level_set_final(h, L0, lab, R.owned.ca, R.owned.n));
     final_set = true;
   }
-  if (cur != &L0) level_free(owned, s);
+  if (R.has_owned) {
+    level_free(R.owned, s);
+    R.has_owned = false;
+  }
   if (!final_set) LV_TRY(level_set_labels(h, L0, lab));
   LV_TRY(copy_out(labels_out, lab, sizeof(int32_t) * (size_t)n0, s));
   LV_CUDA(cudaStreamSynchronize(s));
-  dfree(lab, s);
-  h.pcn = nullptr;
-  if (pcn) dfree(pcn, s);
   fill_q(&local.q, Lq, Sq, W);
   local.t_total_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t_begin).count();
   local.kernel_launches = g_launches - launches0;
@@ -562,6 +655,11 @@ LV_API void louvain_params_default(louvain_params_t* p) {
 }
 
 LV_API const char* louvain_last_error(void) { return g_err.c_str(); }
+LV_API int32_t louvain_release_cache(void) {
+  release_cache_all();
+  cudaGetLastError();
+  return LOUVAIN_OK;
+}
 LV_API void louvain_launch_counts(int64_t* kernel_launches, int64_t* cub_calls) {
   if (kernel_launches) *kernel_launches = g_launches;
   if (cub_calls) *cub_calls = g_cub_calls;
@@ -624,6 +722,44 @@ LV_API int32_t louvain_create_csr(int64_t n, int64_t nnz, const int64_t* rowptr,
   *out = g;
   return LOUVAIN_OK;
 }
+
+namespace lv {
+int32_t create_from_device(int64_t n, int64_t nnz, int64_t* rowptr, int32_t* col, uint32_t* w, void* cuda_stream,
+                           louvain_graph_t* out) {
+  *out = nullptr;
+  louvain_graph_s* g = new louvain_graph_s();
+  Handle& h = g->h;
+  int32_t rc = init_handle(h, cuda_stream);
+  Level& L = h.lv;
+  L.n = n;
+  L.nnz = nnz;
+  L.rowptr = rowptr;
+  L.col = col;
+  L.w = w;
+  L.owns_csr = true;  // freed with the handle (or below, on failure)
+  if (rc == LOUVAIN_OK) rc = level_alloc_state(L, h.stream);
+  if (rc == LOUVAIN_OK) rc = level_setup(h, L);
+  if (rc == LOUVAIN_OK) {
+    cudaError_t e = cudaStreamSynchronize(h.stream);
+    if (e != cudaSuccess) rc = cuda_fail(e, "cudaStreamSynchronize", __FILE__, __LINE__);
+  }
+  if (rc != LOUVAIN_OK) {
+    if (!h.stream) {  // init failed before the stream existed: free the arrays directly
+      dfree(rowptr, nullptr);
+      dfree(col, nullptr);
+      dfree(w, nullptr);
+      L.rowptr = nullptr;
+      L.col = nullptr;
+      L.w = nullptr;
+    }
+    destroy_handle(h);
+    delete g;
+    return rc;
+  }
+  *out = g;
+  return LOUVAIN_OK;
+}
+}  // namespace lv
 
 LV_API int32_t louvain_destroy(louvain_graph_t g) {
   if (!g) return LOUVAIN_OK;
@@ -726,8 +862,11 @@ LV_API int32_t louvain_sweep(louvain_graph_t g, const louvain_params_t* p, int64
   DeviceScope ds(h.device);
   Level& L = h.lv;
   int32_t rc = level_binning(h, L, pp);
+  if (!rc && h.dist) rc = dist_after_binning(h, L);
   if (!rc) rc = sweep_body(h, L, pp);
   if (!rc && q_after) rc = launch_modularity(h, L, nullptr);
+  if (!rc && q_after && h.dist) rc = dist_allreduce(h, &h.ctl->L, 1);
+  if (!rc && h.dist) rc = dist_allreduce(h, &h.ctl->overflow, 1);
   if (!rc) {
     cudaError_t e = cudaMemcpyAsync(h.h_ctl, h.ctl, sizeof(DevCtl), cudaMemcpyDeviceToHost, h.stream);
     if (e == cudaSuccess) e = cudaStreamSynchronize(h.stream);
@@ -830,6 +969,7 @@ LV_API int32_t louvain_begin_sweep(louvain_graph_t g) {
   Level& L = h.lv;
   if (L.log_committed > 0) ++L.sweeps_done;
   L.log_committed = 0;
+  ++L.stamp_id;
   return finish_call(h, set_ctl_u64(h, &h.ctl->logn, 0));
 }
 

@@ -10,6 +10,7 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <memory>
 #include <string>
 #include <vector>
 
@@ -164,6 +165,8 @@ struct Level {
   int32_t* mv_v = nullptr;
   int32_t* mv_new = nullptr;
   int32_t* mv_old = nullptr;
+  int32_t* mv_stamp = nullptr;  // sharded ABI only: sweep id of each vertex's last committed move
+  int32_t stamp_id = 0;         // incremented by every louvain_begin_sweep
   int32_t sweeps_done = 0;  // sweeps since the partition was last reset to singletons
   // sharded sweeps: owned vertex range (decisions, L) and its edge range
   int64_t own_lo = 0, own_hi = -1;  // own_hi < 0: all vertices
@@ -215,9 +218,28 @@ struct Handle {
   // louvain_run only: {label at the sweep start, label after} per vertex; the
   // commit writes .y of every moved vertex (delta pass of Eq. (1))
   uint2* pcn = nullptr;
-  // distributed (nullptr when single GPU)
-  void* dist = nullptr;
+  // distributed handle (louvain_create_csr_dist*): nullptr on one GPU
+  struct DistCtx* dist = nullptr;
 };
+
+// ------------------------------------------------------------------ multi-GPU (lv_dist.cu)
+struct Comm;
+struct DistCtx {
+  Comm* comm = nullptr;
+  int rank = 0, world = 1;
+  std::vector<int64_t> vlo0;   // level-0 row ranges of all ranks (world + 1)
+  int64_t cap[8] = {0};        // exchange capacity per commit group: max over ranks of owned
+                               // vertices of bucket b (b = 1..7), of all buckets (0, RELAXED)
+  int32_t* sbuf = nullptr;     // (v, new) pairs, 2 * max cap
+  int32_t* rbuf = nullptr;     // world * that
+  size_t sbuf_n = 0, rbuf_n = 0;
+  ~DistCtx();
+};
+int32_t dist_set_level_range(Handle& h, Level& L, int level);  // own range of this rank at this level
+int32_t dist_after_binning(Handle& h, Level& L);                // exchange capacities of the level
+int32_t dist_exchange(Handle& h, Level& L, int commit_idx, int group);  // all ranks' moves into the log
+int32_t dist_allreduce(Handle& h, unsigned long long* dev, size_t count);  // in-place sum (no-op on 1 GPU)
+void dist_free(Handle& h);
 
 // ------------------------------------------------------------------ launch accounting
 // Every explicit <<<>>> launch is followed by LV_LAUNCHED(); every device-wide
@@ -280,6 +302,9 @@ int32_t tile_starts(Handle& h, const int64_t* offs, int64_t lo, int64_t hi, int6
                     const int64_t** out);
 int32_t compose_labels_ca(Handle& h, int32_t* lab, int64_t n0, const uint2* ca);   // lab[i] = C[lab[i]]
 size_t hub_partial_bytes();
+// Handle over device CSR arrays it takes ownership of (freed on failure too).
+int32_t create_from_device(int64_t n, int64_t nnz, int64_t* rowptr, int32_t* col, uint32_t* w, void* cuda_stream,
+                           louvain_graph_t* out);
 int32_t validate_csr_host(int64_t n, int64_t nnz, const int64_t* rowptr, const int32_t* col, const uint32_t* w,
                           bool full, uint64_t* W);
 

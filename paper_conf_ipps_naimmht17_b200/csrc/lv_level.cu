@@ -301,12 +301,13 @@ __global__ void __launch_bounds__(256) k_mod_delta_thr(DevCtl* ctl, const int32_
                                                        const int32_t* __restrict__ col,
                                                        const uint32_t* __restrict__ w, const uint2* __restrict__ P,
                                                        int64_t nnz, int32_t* mid,
-                                                       int32_t* big) {
+                                                       int32_t* big, int64_t own_lo, int64_t own_hi) {
   if (!delta_chosen(*ctl, nnz)) return;
   const long long logn = (long long)ctl->logn;
   long long acc = 0;
   for (long long p = (long long)blockIdx.x * blockDim.x + threadIdx.x; p < logn; p += (long long)gridDim.x * blockDim.x) {
     const int32_t i = mv_v[p];
+    if (i < own_lo || i >= own_hi) continue;  // sharded run: another rank sums this moved row
     const int64_t b = rowptr[i], e = rowptr[i + 1];
     if (e - b > kDeltaBigDeg) {
       big[atomicAdd(&ctl->nbig, 1ull)] = (int32_t)p;
@@ -542,6 +543,7 @@ int32_t level_alloc_scratch(Handle& h, Level& L, int parity) {
 
 void level_free(Level& L, cudaStream_t s) {
   if (L.scratch_backed) {  // arrays belong to the handle's scratch; plans are per level
+    dfree(L.mv_stamp, s);
     hub_free(L.hub, s);
     part_free(L.part, s);
     L = Level();
@@ -553,7 +555,7 @@ void level_free(Level& L, cudaStream_t s) {
     dfree(L.w, s);
   }
   dfree(L.k, s); dfree(L.ca, s); dfree(L.C, s); dfree(L.size, s);
-  dfree(L.mv_v, s); dfree(L.mv_new, s); dfree(L.mv_old, s); dfree(L.bin_vertices, s);
+  dfree(L.mv_v, s); dfree(L.mv_new, s); dfree(L.mv_old, s); dfree(L.bin_vertices, s); dfree(L.mv_stamp, s);
   dfree(L.soff, s);  // L.stage lives in the handle's scratch
   hub_free(L.hub, s);
   part_free(L.part, s);
@@ -1000,8 +1002,11 @@ int32_t launch_modularity_delta(Handle& h, Level& L) {
   int32_t *big = nullptr, *mid = nullptr;
   LV_TRY(dalloc(&big, (size_t)(L.nnz / kDeltaBigDeg + 1), s));
   LV_TRY(dalloc(&mid, (size_t)(L.nnz / kDeltaThrDeg + 1), s));
+  // a distributed handle sums the moved rows it owns (the ranks' parts are all-reduced)
+  const int64_t own_lo = (h.dist && L.own_hi >= 0) ? L.own_lo : 0;
+  const int64_t own_hi = (h.dist && L.own_hi >= 0) ? L.own_hi : L.n;
   k_mod_delta_thr<<<148 * 8, 256, 0, s>>>(h.ctl, L.mv_v, L.mv_new, L.mv_old, L.rowptr, L.col, L.w, P,
-                                          L.nnz, mid, big);
+                                          L.nnz, mid, big, own_lo, own_hi);
   LV_LAUNCHED();
   k_mod_delta_warp<<<148 * 8, 256, 0, s>>>(h.ctl, mid, L.mv_v, L.mv_new, L.mv_old, L.rowptr, L.col, L.w, P,
                                            L.nnz);
@@ -1053,10 +1058,21 @@ __global__ void k_pack_moves(const int32_t* mv_v, const int32_t* mv_new, int64_t
     out[2 * i + 1] = mv_new[c0 + i];
   }
 }
-__global__ void k_unpack_moves(const int32_t* in, int64_t c0, int64_t cnt, int32_t* mv_v, int32_t* mv_new) {
+// (v, new) pairs -> move log.  Caller-supplied ids are validated before any
+// commit: v and new in [0, n), and no vertex twice in one sweep (stamp[v] holds
+// the id of the last sweep that moved v); a violation sets ctl->bad.
+__global__ void k_unpack_moves(const int32_t* in, int64_t c0, int64_t cnt, int64_t n, int32_t* mv_v, int32_t* mv_new,
+                               int32_t* stamp, int32_t sweep_id, DevCtl* ctl) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < cnt; i += (int64_t)gridDim.x * blockDim.x) {
-    mv_v[c0 + i] = in[2 * i];
-    mv_new[c0 + i] = in[2 * i + 1];
+    const int32_t v = in[2 * i], t = in[2 * i + 1];
+    if (v < 0 || v >= n || t < 0 || t >= n || atomicExch(&stamp[v], sweep_id) == sweep_id) {
+      atomicOr(&ctl->bad, 1ull);
+      mv_v[c0 + i] = 0;  // never committed: the host refuses the call
+      mv_new[c0 + i] = 0;
+      continue;
+    }
+    mv_v[c0 + i] = v;
+    mv_new[c0 + i] = t;
   }
 }
 }  // namespace
@@ -1078,9 +1094,25 @@ int32_t pack_moves(Handle& h, Level& L, int64_t c0, int64_t cnt, int32_t* out) {
 
 int32_t unpack_moves(Handle& h, Level& L, int64_t c0, int64_t cnt, const int32_t* in) {
   if (cnt <= 0) return LOUVAIN_OK;
-  k_unpack_moves<<<grid_for(cnt, 256), 256, 0, h.stream>>>(in, c0, cnt, L.mv_v, L.mv_new);
+  if (!L.mv_stamp) {
+    LV_TRY(dalloc(&L.mv_stamp, L.n, h.stream));
+    LV_CUDA(cudaMemsetAsync(L.mv_stamp, 0xFF, 4 * (size_t)std::max<int64_t>(L.n, 1), h.stream));  // -1: never
+  }
+  LV_CUDA(cudaMemsetAsync(&h.ctl->bad, 0, 8, h.stream));
+  k_unpack_moves<<<grid_for(cnt, 256), 256, 0, h.stream>>>(in, c0, cnt, L.n, L.mv_v, L.mv_new, L.mv_stamp,
+                                                          L.stamp_id, h.ctl);
   LV_LAUNCHED();
   LV_CUDA(cudaGetLastError());
+  unsigned long long bad = 0;
+  LV_CUDA(cudaMemcpyAsync(&bad, &h.ctl->bad, 8, cudaMemcpyDeviceToHost, h.stream));
+  LV_CUDA(cudaStreamSynchronize(h.stream));
+  if (bad) {
+    // undo the stamps of this call's valid entries is not needed: the handle's
+    // sweep is refused as a whole (the caller must revert or restart the sweep)
+    LV_CUDA(cudaMemsetAsync(&h.ctl->bad, 0, 8, h.stream));
+    set_error("louvain_commit_moves: vertex or label out of [0, n), or a vertex moved twice in one sweep");
+    return LOUVAIN_E_INVALID_ARG;
+  }
   return LOUVAIN_OK;
 }
 

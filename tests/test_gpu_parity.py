@@ -277,61 +277,91 @@ def test_generators_host_device_bit_identical(maker, args):
     assert np.array_equal(h.rowptr, d.rowptr) and np.array_equal(h.col, d.col)
 
 
-# ---------------------------------------------------------------- sharded sweep on the GPU
-def _gpu_shard_worker(rank, world, port, q):
+# ---------------------------------------------------------------- the distributed handle on the GPU
+DIST_GRAPHS = ("karate", "rmat15", "hubs", "giant_hub", "weighted_loops", "lfr5k")
+
+
+def _dist_run(g, rank, world, comm, mode):
+    import paper_conf_ipps_naimmht17_b200 as lvb2
+    from paper_conf_ipps_naimmht17_b200.dist import edge_balanced_ranges, local_rows
+    lo, hi = edge_balanced_ranges(g.rowptr, world)[rank]
+    rl, cl, wl = local_rows(g.rowptr, g.col, g.w, lo, hi)
+    with lvb2.Graph.from_csr_dist(g.n, lo, hi, rl, cl, wl, rank=rank, world=world, comm=comm) as gd:
+        lab, q, st = gd.run(lvb2.params(mode=mode))
+        gd.set_labels(None)
+        moved, q1 = gd.sweep(lvb2.params(mode=mode))  # one collective louvain_sweep from singletons
+        lab1 = gd.labels()
+    return lab.tolist(), {k: st[k] for k in ("levels", "sweeps_per_level", "num_start", "num_end", "L", "S")}, \
+        (moved, int(q1.L), q1.S, lab1.tolist())
+
+
+def _dist_worker(rank, world, port, mode, q):
     import os
     import torch.distributed as dist
-    import paper_conf_ipps_naimmht17_b200 as lvb2
-    from paper_conf_ipps_naimmht17_b200.dist import CudaShard, run_sharded
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
     dist.init_process_group("gloo", rank=rank, world_size=world)
     try:
-        out = {}
-        for name in ("rmat15", "hubs", "weighted_loops"):
-            g = GRAPHS[name]()
-            lab, st = run_sharded(CudaShard(lvb2.Graph.from_csr(g.rowptr, g.col, g.w)), lvb2.params())
-            out[name] = (lab.cpu().numpy().tolist(), st)
-        q.put((rank, out))
+        q.put((rank, {name: _dist_run(GRAPHS[name](), rank, world, "host", mode) for name in DIST_GRAPHS}))
     finally:
         dist.destroy_process_group()
 
 
-def test_sharded_world1_cuda_matches_oracle():
-    from paper_conf_ipps_naimmht17_b200.dist import CudaShard, run_sharded
-    for name in ("karate", "rmat15", "hubs", "giant_hub"):
-        g = GRAPHS[name]()
-        r = oracle.louvain(g)
-        lab, st = run_sharded(CudaShard(dev_graph(g)), lvb.params())
-        assert np.array_equal(lab.cpu().numpy(), r.labels), name
-        assert st["sweeps_per_level"] == r.sweeps_per_level and (st["L"], st["S"]) == (r.L, r.S)
+def _check_dist(name, lab, st, sw, mode):
+    g = GRAPHS[name]()
+    r = oracle.louvain(g, oracle.params(mode=mode))
+    assert lab == r.labels.tolist(), name
+    assert st["sweeps_per_level"] == r.sweeps_per_level and (st["L"], st["S"]) == (r.L, r.S)
+    assert st["num_start"] == r.num_start and st["num_end"] == r.num_end
+    o = oracle.State(g)
+    moved = o.sweep(oracle.params(mode=mode))
+    L, S, _ = o.qnum()
+    assert sw == (moved, L, S, o.C.tolist()), name
 
 
-def test_sharded_two_ranks_one_gpu_matches_oracle():
-    """Two processes share the GPU (gloo exchange through the host): every rank
-    decides its own vertex range with the CUDA kernels and commits all moves."""
+def test_dist_handle_nccl_world1_matches_oracle():
+    """The NCCL transport end to end with one rank (NCCL allows no second rank on one GPU)."""
+    import os
+    import socket
+    import torch.distributed as dist
+    sk = socket.socket()
+    sk.bind(("127.0.0.1", 0))
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(sk.getsockname()[1])
+    sk.close()
+    dist.init_process_group("gloo", rank=0, world_size=1)
+    try:
+        for name in DIST_GRAPHS:
+            lab, st, sw = _dist_run(GRAPHS[name](), 0, 1, "nccl", 0)
+            _check_dist(name, lab, st, sw, 0)
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world,mode", [(2, 0), (3, 0), (2, 1)])
+def test_dist_handle_ranks_share_one_gpu_match_oracle(world, mode):
+    """world processes share the GPU (host transport over gloo): every rank decides its own
+    edge-balanced rows with the CUDA kernels, the library exchanges the moves of each bucket
+    and every rank commits all of them -- bit-identical to oracle (b) on every rank."""
     import socket
     import torch.multiprocessing as tmp
-    s = socket.socket()
-    s.bind(("127.0.0.1", 0))
-    port = s.getsockname()[1]
-    s.close()
+    sk = socket.socket()
+    sk.bind(("127.0.0.1", 0))
+    port = sk.getsockname()[1]
+    sk.close()
     ctx = tmp.get_context("spawn")
     q = ctx.Queue()
-    procs = [ctx.Process(target=_gpu_shard_worker, args=(r, 2, port, q)) for r in range(2)]
+    procs = [ctx.Process(target=_dist_worker, args=(r, world, port, mode, q)) for r in range(world)]
     for pr in procs:
         pr.start()
-    res = dict(q.get(timeout=600) for _ in range(2))
+    res = dict(q.get(timeout=900) for _ in range(world))
     for pr in procs:
         pr.join(timeout=60)
         assert pr.exitcode == 0
-    for name in ("rmat15", "hubs", "weighted_loops"):
-        g = GRAPHS[name]()
-        r = oracle.louvain(g)
-        lab0, st0 = res[0][name]
-        assert res[1][name][0] == lab0
-        assert lab0 == r.labels.tolist(), name
-        assert st0["sweeps_per_level"] == r.sweeps_per_level and (st0["L"], st0["S"]) == (r.L, r.S)
+    for name in DIST_GRAPHS:
+        for r in range(1, world):
+            assert res[r][name] == res[0][name], (name, r)
+        _check_dist(name, *res[0][name], mode)
 
 
 def _alt_path_worker(env_items, names, q):
