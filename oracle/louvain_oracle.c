@@ -11,9 +11,11 @@
  * community, disjoint cliques, ring of cliques), networkx modularity on random
  * partitions, exact-rational Eq. (2) gains vs re-evaluated Eq. (1), brute force
  * over all partitions (n <= 9), contraction == P^T A P (scipy) with W and Q
- * preserved, karate values, singleton-rule micro cases.  The bucket/commit
- * rules R10-R12 are "parity unpinned" by the paper (no worked example);
- * DESIGN.md records that.
+ * preserved, karate values, singleton-rule micro cases, hand-computed worked
+ * cases of RELAXED (star K_{1,5}: one snapshot vs bucket commits) and of the
+ * (adaptive) sequential variant (path P_4 with the theta_bin schedule).  The
+ * bucket/commit rules R10-R12 are "parity unpinned" by the paper (no worked
+ * example); DESIGN.md records that.
  */
 #include "louvain_oracle.h"
 

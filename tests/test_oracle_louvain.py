@@ -148,3 +148,73 @@ def test_relaxed_is_one_bucket(karate):
     s2 = oracle.State(karate)
     s2.sweep(oracle.params(deg_bounds=[10**9] * 6))
     assert s1.C.tolist() == s2.C.tolist()
+
+
+def _star5():
+    # K_{1,5}: hub 0, leaves 1..5, unit weights; W = 2m = 10, k = (5, 1, 1, 1, 1, 1)
+    return graphgen.from_edges(6, [0, 0, 0, 0, 0], [1, 2, 3, 4, 5], compact=False)
+
+
+def test_relaxed_worked_star():
+    """RELAXED decides every vertex on ONE snapshot, BIN_SYNC commits bucket 1
+    (the leaves, deg 1) before bucket 2 (the hub, deg 5) decides (Alg. 1 l.4-11).
+    Hand computation with the singleton rule off (rule 0), from singletons:
+      leaf i: one candidate, the hub: s = W*1 - k_i*a_0 = 10 - 5 = 5 > s_stay = 0 -> moves to 0;
+      hub, RELAXED (all singletons): every leaf c has s = 10*1 - 5*1 = 5, tie -> lowest label 1,
+        s_stay = 10*0 - 5*(5 - 5) = 0 -> moves to 1;
+      hub, BIN_SYNC (leaves already in 0): its only label is its own -> stays.
+    RELAXED: C = [1,0,0,0,0,0], L = 0, a = {0: 5, 1: 5}, S = 50, Q = (0*10 - 50)/100 = -1/2.
+    BIN_SYNC: C = [0]*6, L = 10, S = 100, Q = 0.  With the veto rule (1) the RELAXED hub's
+    best (label 1 > own 0, both singletons) is vetoed: C = [0]*6."""
+    g = _star5()
+    st = oracle.State(g)
+    assert st.sweep(oracle.params(mode=oracle.RELAXED, singleton_rule=0)) == 6
+    assert st.C.tolist() == [1, 0, 0, 0, 0, 0]
+    assert st.qnum() == (0, 50, 10)
+    st = oracle.State(g)
+    assert st.sweep(oracle.params(mode=oracle.BIN_SYNC, singleton_rule=0)) == 5
+    assert st.C.tolist() == [0] * 6 and st.qnum() == (10, 100, 10)
+    st = oracle.State(g)
+    assert st.sweep(oracle.params(mode=oracle.RELAXED, singleton_rule=1)) == 5
+    assert st.C.tolist() == [0] * 6
+    # whole run, RELAXED rule 0: the sweep lowers Q from -30/100 (singletons: S = 25 + 5)
+    # to -50/100, so it is reverted (R15) and nothing moved: labels stay singletons
+    r = oracle.louvain(g, oracle.params(mode=oracle.RELAXED, singleton_rule=0))
+    assert r.labels.tolist() == [0, 1, 2, 3, 4, 5] and (r.L, r.S, r.W) == (0, 30, 10)
+    assert r.levels == 1 and r.sweeps_per_level == [1]
+
+
+def test_adaptive_sequential_worked_path():
+    """Sequential Louvain (R23) and its adaptive variant (the n-dependent
+    threshold theta_bin while n > size_limit) on the path 0-1-2-3 (W = 6, k = (1, 2, 2, 1)).
+    Hand computation, ascending ids, immediate updates, no singleton rule:
+      sweep 1: v0 -> 1 (s = 6 - 1*2 = 4 > 0); v1 stays (s_stay = 6*1 - 2*(3-2) = 4 > s_2 = 6 - 2*2 = 2);
+               v2 -> 3 (s_3 = 6 - 2*1 = 4 > s_1 = 6 - 2*3 = 0 = s_stay); v3 stays.
+               C = [1,1,3,3], numerator L*W - S = 4*6 - 18 = 6 (start: 0 - 10 = -10).
+      sweep 2: nothing moves -> phase ends after 2 sweeps (theta_final = 1e-6).
+      level 1: two vertices, self-loops 2, edge weight 1, k = 3: s = 6*1 - 3*3 = -3 < 0, no move.
+    Adaptive with size_limit = 2 and theta_bin = 10^0: level 0 (n = 4 > 2) stops after sweep 1
+    because (6 - (-10)) * 10^0 < W^2 = 36; the labels are the same."""
+    g = graphgen.from_edges(4, [0, 1, 2], [1, 2, 3], compact=False)
+    st = oracle.State(g)
+    assert st.sweep(oracle.params(mode=oracle.SEQ)) == 2
+    assert st.C.tolist() == [1, 1, 3, 3] and st.qnum() == (4, 18, 6)
+    r = oracle.louvain(g, oracle.params(mode=oracle.SEQ))
+    assert r.sweeps_per_level == [2, 1] and r.labels.tolist() == [0, 0, 1, 1]
+    assert (r.L * r.W - r.S, r.num_start) == (6, [-10, 6])
+    ra = oracle.louvain(g, oracle.params(mode=oracle.SEQ_ADAPTIVE, size_limit=2, th_bin_exp=0))
+    assert ra.sweeps_per_level == [1, 1] and ra.labels.tolist() == [0, 0, 1, 1]
+    # n <= size_limit at every level: adaptive == sequential exactly
+    for gg in (g, graphgen.karate(), graphgen.rmat(9, seed=4)):
+        a = oracle.louvain(gg, oracle.params(mode=oracle.SEQ))
+        b = oracle.louvain(gg, oracle.params(mode=oracle.SEQ_ADAPTIVE))
+        assert a.labels.tolist() == b.labels.tolist() and a.sweeps_per_level == b.sweeps_per_level
+
+
+def test_adaptive_theta_one_sweep_per_large_level():
+    # theta_bin = 10^0 and size_limit = 0: every level runs exactly one sweep (a Q gain is < 1)
+    g = graphgen.rmat(10, seed=3)
+    r = oracle.louvain(g, oracle.params(mode=oracle.SEQ_ADAPTIVE, size_limit=0, th_bin_exp=0))
+    assert all(s == 1 for s in r.sweeps_per_level)
+    L, S, W = oracle.modularity(g, r.labels)
+    assert (L, S) == (r.L, r.S)
