@@ -49,6 +49,16 @@ def lib():
         L.gg_copy_out.argtypes = [vp, vp, vp]
         L.gg_free.argtypes = [vp]
         L.gg_last_error.restype = ctypes.c_char_p
+        L.gg_load.argtypes = [ctypes.c_char_p, i32, i32, pp]
+        L.gg_save_csrbin.argtypes = [ctypes.c_char_p, i64, i64, vp, vp, vp]
+        for f in ("gg_csr_n", "gg_csr_nnz"):
+            getattr(L, f).argtypes = [vp]
+            getattr(L, f).restype = i64
+        for f in ("gg_csr_rowptr", "gg_csr_col", "gg_csr_w"):
+            getattr(L, f).argtypes = [vp]
+            getattr(L, f).restype = vp
+        L.gg_csr_free.argtypes = [vp]
+        L.gg_io_last_error.restype = ctypes.c_char_p
         _LIB = L
     return _LIB
 
@@ -117,6 +127,56 @@ def _take(h: ctypes.c_void_p, name: str, device: bool, meta: dict):
         return Graph(n, rowptr, col, None, labels, name, meta)
     finally:
         L.gg_free(h)
+
+
+FORMATS = {"auto": 0, "mtx": 1, "edgelist": 2, "csrbin": 3}
+
+
+def load(path: str, fmt: str = "auto", one_based: Optional[bool] = None, compact: bool = False) -> Graph:
+    """Read a graph file (graph_io.cpp): Matrix Market coordinate (.mtx), edge list
+    ("u v [w]" per line) or the binary .csrbin container -> R1 CSR (both directions,
+    self-loop once, rows sorted).  w is None for unweighted inputs.  compact=True
+    drops isolated vertices with an order-preserving relabel (R21)."""
+    L = lib()
+    h = ctypes.c_void_p()
+    ob = -1 if one_based is None else int(bool(one_based))
+    rc = L.gg_load(os.fsencode(path), FORMATS[fmt], ob, ctypes.byref(h))
+    if rc != 0:
+        raise ValueError(f"graphgen.load({path!r}): {L.gg_io_last_error().decode()}")
+    try:
+        n, nnz = L.gg_csr_n(h), L.gg_csr_nnz(h)
+        rowptr = np.ctypeslib.as_array(ctypes.cast(L.gg_csr_rowptr(h), ctypes.POINTER(ctypes.c_int64)),
+                                       shape=(n + 1,)).copy()
+        col = np.zeros(0, dtype=np.int32)
+        if nnz:
+            col = np.ctypeslib.as_array(ctypes.cast(L.gg_csr_col(h), ctypes.POINTER(ctypes.c_int32)),
+                                        shape=(nnz,)).copy()
+        wp = L.gg_csr_w(h)
+        w = None
+        if wp and nnz:
+            w = np.ctypeslib.as_array(ctypes.cast(wp, ctypes.POINTER(ctypes.c_uint32)), shape=(nnz,)).copy()
+    finally:
+        L.gg_csr_free(h)
+    g = Graph(int(n), rowptr, col, w, None, os.path.basename(path), {"file": path})
+    if compact:
+        deg = np.diff(g.rowptr)
+        keep = np.flatnonzero(deg > 0)
+        newid = np.full(g.n, -1, dtype=np.int64)
+        newid[keep] = np.arange(len(keep))
+        g = Graph(len(keep), np.concatenate([[0], np.cumsum(deg[keep])]).astype(np.int64),
+                  newid[g.col].astype(np.int32), g.w, None, g.name, dict(g.meta))
+    return g
+
+
+def save_csrbin(g: Graph, path: str) -> None:
+    """Write g as .csrbin (read back bit for bit by load())."""
+    rowptr = np.ascontiguousarray(g.rowptr, dtype=np.int64)
+    col = np.ascontiguousarray(g.col, dtype=np.int32)
+    w = None if g.w is None else np.ascontiguousarray(g.w, dtype=np.uint32)
+    rc = lib().gg_save_csrbin(os.fsencode(path), g.n, int(rowptr[-1]), rowptr.ctypes.data,
+                              col.ctypes.data if len(col) else None, None if w is None else w.ctypes.data)
+    if rc != 0:
+        raise OSError(lib().gg_io_last_error().decode())
 
 
 def karate() -> Graph:

@@ -56,6 +56,24 @@ int gg_copy_out(gg_graph_t g, int64_t* rowptr_dst, int32_t* col_dst);
 void gg_free(gg_graph_t g);
 const char* gg_last_error(void);
 
+/* ---- graph files (graph_io.cpp): a loader for real inputs next to the generators ----
+ * format: 0 = by extension (.mtx Matrix Market, .csrbin binary CSR, else edge list),
+ * 1 = Matrix Market coordinate, 2 = edge list "u v [w]", 3 = .csrbin.
+ * one_based (edge lists): 1, 0, or -1 = 1-based iff no id is 0.  Text inputs are
+ * undirected and become R1 CSR (both directions, self-loop once, rows sorted);
+ * see graph_io.cpp for weights and repeated edges. */
+typedef struct gg_csr_s* gg_csr_t;
+int gg_load(const char* path, int format, int one_based, gg_csr_t* out);
+int gg_save_csrbin(const char* path, int64_t n, int64_t nnz, const int64_t* rowptr, const int32_t* col,
+                   const uint32_t* w /* NULL = unit */);
+int64_t gg_csr_n(gg_csr_t g);
+int64_t gg_csr_nnz(gg_csr_t g);
+const int64_t* gg_csr_rowptr(gg_csr_t g);
+const int32_t* gg_csr_col(gg_csr_t g);
+const uint32_t* gg_csr_w(gg_csr_t g); /* NULL = unit weights */
+void gg_csr_free(gg_csr_t g);
+const char* gg_io_last_error(void);
+
 #ifdef __cplusplus
 }
 #endif

@@ -414,3 +414,24 @@ def test_alternative_paths_match_oracle(env):
     assert pr.exitcode == 0
     for k, v in out.items():
         assert all(v), (env, k, v)
+
+
+def test_loaded_files_match_oracle(tmp_path):
+    """Graphs read by the loader (graphgen.load: Matrix Market fixture, weighted edge list
+    with self-loops, .csrbin round trip) run through the C-ABI bit-exactly against oracle (b)."""
+    import os
+    gold = os.path.join(os.path.dirname(__file__), "golden", "karate.mtx")
+    wl = weighted_with_loops(2000, 11)
+    p = tmp_path / "w.txt"
+    with open(p, "w") as f:
+        for u in range(wl.n):
+            for e in range(wl.rowptr[u], wl.rowptr[u + 1]):
+                if wl.col[e] >= u:  # each undirected edge once
+                    f.write(f"{u} {wl.col[e]} {wl.w[e]}\n")
+    graphgen.save_csrbin(GRAPHS["hubs"](), str(tmp_path / "h.csrbin"))
+    for path in (gold, str(p), str(tmp_path / "h.csrbin")):
+        g = graphgen.load(path)
+        r = oracle.louvain(g)
+        lab, q, st = dev_graph(g).run(lvb.params())
+        assert np.array_equal(lab, r.labels), path
+        assert (int(q.L), q.S) == (r.L, r.S) and st["sweeps_per_level"] == r.sweeps_per_level
