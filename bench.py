@@ -10,10 +10,14 @@ already resident in HBM.  value = directed edges swept per second over the
 whole run (sum over executed sweeps of the level's nnz / run time).
 
 Also reported: the roofline of the dominant kernel sequence (the level-0
-sweep body), the oracle timed on the host (cpu_baseline), an end-to-end number
-through the C-ABI with host buffers (e2e), SM clocks during the timed region.
+sweep body; D of the byte model from the oracle's count when recorded), the
+oracle timed on one pinned host core (cpu_baseline), an end-to-end number
+through the C-ABI with host buffers (e2e, with its parts), SM clocks during the
+timed region, and the per-config rates of SURVEY 8(d) (median level-0 sweep,
+phase-1 TEPS per |E| and per 2|E|).  --config C1..C4b gives the other
+BASELINE.json workloads the same line (the default, C5, is the headline).
 
-    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference] [--config C5]
 """
 from __future__ import annotations
 
@@ -32,6 +36,17 @@ sys.path.insert(0, ROOT)
 METRIC = "sweep edges/s (multilevel Louvain run)"
 UNIT = "edges/s"
 
+# BASELINE.json configs as synthetic inputs
+CONFIGS = {
+    "C1": "Zachary karate club (34 vertices, 78 unit edges)",
+    "C2": "LFR-style planted partition, n = 1e6 (gamma 2.5 on [8,1000], beta 1.5 on [50,5000], mu 0.3)",
+    "C3": "R-MAT scale 24, 8*2^24 tuples (A,B,C = .57,.19,.19), seed 1, unit weights, isolated vertices removed",
+    "C4a": "3-D 7-point mesh 368^3, Morton ids",
+    "C4b": "random geometric graph, n = 5e7, r = 0.55 sqrt(ln n / n), ids by grid cell",
+    "C5": "R-MAT scale 27, 8*2^27 tuples (A,B,C = .57,.19,.19), seed 1, unit weights, isolated vertices removed",
+}
+DEVICE_GEN = ("C3", "C4a", "C4b", "C5")  # device generators (bit-identical to the host ones)
+
 
 def parse_args():
     ap = argparse.ArgumentParser()
@@ -39,7 +54,8 @@ def parse_args():
     ap.add_argument("--steps", type=int, default=3)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
-    ap.add_argument("--scale", type=int, default=27, help="R-MAT scale (27 = C5)")
+    ap.add_argument("--config", default="C5", choices=list(CONFIGS),
+                    help="BASELINE.json workload (C5 = the headline; C1-C4b: per-config lines)")
     ap.add_argument("--seed", type=int, default=1)
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--e2e-warmup", type=int, default=1)
@@ -113,8 +129,36 @@ def measured_peak_hbm():
         return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
 
 
-def cfg_name(scale):
-    return {27: "C5", 24: "C3"}.get(scale, "scaled")
+def device_graph(cfg, seed):
+    """The config's CSR on the device (torch tensors): rowptr int64, col int32."""
+    import torch
+    import graphgen
+    if cfg in DEVICE_GEN:
+        return graphgen.config(cfg, device=True, seed=seed)
+    hg = graphgen.config(cfg, seed=seed)
+    return graphgen.DeviceGraph(hg.n, torch.from_numpy(hg.rowptr).cuda(), torch.from_numpy(hg.col).cuda(), hg.name)
+
+
+def oracle_D(cfg):
+    """D of level-0 sweep 1 (distinct (vertex, candidate label) pairs of the byte model), computed by
+    the oracle (tools/make_golden.py --sweeps-only, oracle/ only); None if not recorded."""
+    try:
+        with open(os.path.join(ROOT, "tests", "golden", "oracle_runs.json")) as f:
+            return int(json.load(f)[cfg]["level0_sweeps_b"][0]["D"])
+    except Exception:
+        return None
+
+
+def cpu_info():
+    model = None
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                model = line.split(":", 1)[1].strip()
+                break
+    except OSError:
+        pass
+    return {"nproc": os.cpu_count(), "cpu_model": model}
 
 
 def recorded_traffic():
@@ -141,15 +185,14 @@ def oracle_rate(hg, seconds: float, seed: int = 0):
     n = hg.n
     deg = np.diff(hg.rowptr)
     C = np.arange(n, dtype=np.int32)
-    a = deg.astype(np.uint64)
+    a = deg.astype(np.uint64) if hg.w is None else np.add.reduceat(hg.w.astype(np.uint64), hg.rowptr[:-1])
     size = np.ones(n, dtype=np.int64)
-    W = int(deg.sum())
+    W = int(a.sum())
     rng = np.random.default_rng(seed)
 
     def sample(edges):
         frac = min(1.0, edges / max(1, hg.nnz))
-        verts = np.flatnonzero(rng.random(n) < frac).astype(np.int64)
-        return verts
+        return np.flatnonzero(rng.random(n) < frac).astype(np.int64)
 
     # random-vertex chunks until the time budget is spent (a bounded sample of the workload)
     edges, spent, nv, chunk = 0, 0.0, 0, 2_000_000
@@ -167,41 +210,103 @@ def oracle_rate(hg, seconds: float, seed: int = 0):
     return edges / spent, edges, spent, nv
 
 
+class PinnedCore:
+    """The oracle is single-threaded: pin this process to one host core while it runs
+    (sched_setaffinity), so its rate is a one-core number; restored afterwards."""
+
+    def __enter__(self):
+        self.old = os.sched_getaffinity(0)
+        self.core = max(self.old)
+        os.sched_setaffinity(0, {self.core})
+        return self
+
+    def __exit__(self, *a):
+        os.sched_setaffinity(0, self.old)
+
+
+def cpu_baseline_line(hg, seconds, seed=0):
+    with PinnedCore() as pc:
+        r, e, dt, nv = oracle_rate(hg, seconds, seed)
+    info = cpu_info()
+    return {"value": r, "unit": UNIT, "cores": 1, "kind": "oracle", "pinned_core": pc.core,
+            "nproc": info["nproc"], "cpu_model": info["cpu_model"],
+            "sample": f"oracle computeMove (Alg. 2, plain C, 1 thread pinned to core {pc.core} of "
+                      f"{info['nproc']}) for {nv} random vertices ({e} directed edges, {dt:.1f} s) of the level-0 "
+                      "singleton state of the same graph"}
+
+
 def emit(d: dict):
     print(json.dumps(d), flush=True)
 
 
+def workload(args, n, nnz):
+    return {"workload": f"{args.config}: {CONFIGS[args.config]}", "seed": args.seed, "n": n, "nnz": nnz}
+
+
 # ----------------------------------------------------------------------------- arms
 def run_reference(args, rank, world):
-    """--impl reference: the oracle (plain single-threaded C) on the host cores,
+    """--impl reference: the oracle (plain single-threaded C, pinned to one host core),
     each step a bounded sample of the same workload, same metric/unit."""
     if rank != 0:
         return
-    import graphgen
     t0 = time.perf_counter()
-    hg = graphgen.rmat(args.scale, seed=args.seed, device=True).to_host()
+    dg = device_graph(args.config, args.seed) if args.config in DEVICE_GEN else None
+    import graphgen
+    hg = dg.to_host() if dg is not None else graphgen.config(args.config, seed=args.seed)
     gen_s = time.perf_counter() - t0
     per_step = max(2.0, min(args.cpu_seconds, 150.0 / max(1, args.steps + args.warmup)))
-    for _ in range(args.warmup):
-        oracle_rate(hg, per_step / 4)
-    rates, edges, secs = [], 0, 0.0
-    for k in range(args.steps):
-        r, e, dt, nv = oracle_rate(hg, per_step, seed=k + 1)
-        rates.append(r)
-        edges += e
-        secs += dt
+    with PinnedCore() as pc:
+        for _ in range(args.warmup):
+            oracle_rate(hg, per_step / 4)
+        edges, secs = 0, 0.0
+        for k in range(args.steps):
+            r, e, dt, nv = oracle_rate(hg, per_step, seed=k + 1)
+            edges += e
+            secs += dt
     value = edges / secs
+    info = cpu_info()
     sample = (f"oracle computeMove (Alg. 2) on {args.steps} random vertex samples of the level-0 singleton "
-              f"state of R-MAT s{args.scale}, {edges} directed edges total")
+              f"state of {args.config}, {edges} directed edges total, 1 thread pinned to core {pc.core}")
     emit({"metric": METRIC, "value": value, "unit": UNIT, "impl": "reference", "n_gpus": world,
           "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * secs / args.steps,
           "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int64",
-          "data": "synthetic",
-          "config": {"workload": f"{cfg_name(args.scale)} R-MAT scale {args.scale}, {8 << args.scale} tuples, seed {args.seed}",
-                     "n": hg.n, "nnz": hg.nnz, "parallelism": "1 host core"},
-          "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
+          "data": "synthetic", "config": dict(workload(args, hg.n, hg.nnz), parallelism="1 host core"),
+          "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle", "pinned_core": pc.core,
+                           "nproc": info["nproc"], "cpu_model": info["cpu_model"], "sample": sample},
           "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
           "gen_s": gen_s})
+
+
+def level0_fields(st, nnz):
+    """Per-config rates of SURVEY 8(d): level-0 sweep 1 and the median level-0 sweep (sweep
+    bodies, no modularity pass), and phase-1 TEPS (all level-0 sweeps over the level-0
+    optimisation time incl. modularity), quoted per |E| (= nnz/2) and per 2|E| (= nnz)."""
+    l0 = st["t_sweep_ms_level0"]
+    k0 = st["sweeps_per_level"][0] if st["levels"] else 0
+    t_ph1 = st["t_opt_ms"][0] if st["levels"] else 0.0
+    med = statistics.median(l0) if l0 else None
+    return {"level0_sweeps_ms": l0, "level0_sweep_median_ms": med,
+            "level0_sweep_median_edges_per_s": nnz / (med / 1e3) if med else None,
+            "phase1_ms": t_ph1,
+            "phase1_teps_2E": k0 * nnz / (t_ph1 / 1e3) if t_ph1 else None,
+            "phase1_teps_E": k0 * (nnz // 2) / (t_ph1 / 1e3) if t_ph1 else None}
+
+
+def roofline_of(args, n_act, nnz, st, t_sw1, world=1):
+    D = oracle_D(args.config)
+    B = sweep_bytes(n_act, nnz, D=D if D is not None else nnz, moved=st["moved_first"]) / world
+    achieved = B / (t_sw1 / 1e3) / 1e9
+    peak, peak_src = measured_peak_hbm()
+    traffic, traffic_src = recorded_traffic() if (args.config == "C5" and world == 1) else (None, None)
+    return {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
+            "traffic": traffic / world if traffic else None,
+            "kernel": "level-0 sweep 1 body" + (" per GPU (bucket kernels + commits + move all-gathers)"
+                                               if world > 1 else " (7 bucket kernels + commits)"),
+            "algorithmic_bytes": B, "t_ms": t_sw1, "peak_source": peak_src,
+            "D": D if D is not None else nnz,
+            "D_source": ("exact: oracle (b) level-0 sweep 1 (tests/golden/oracle_runs.json, tools/make_golden.py)"
+                         if D is not None else "upper bound D = nnz (no oracle count recorded for this config)"),
+            "traffic_source": traffic_src if traffic else "not captured for this config / N"}
 
 
 def run_sharded_bench(args, rank, world):
@@ -211,20 +316,18 @@ def run_sharded_bench(args, rank, world):
     import torch
     import torch.distributed as dist
 
-    import graphgen
     import paper_conf_ipps_naimmht17_b200 as lvb
     from paper_conf_ipps_naimmht17_b200.dist import edge_balanced_ranges, local_rows
 
     dev = torch.device("cuda", torch.cuda.current_device())
-    dg = graphgen.rmat(args.scale, seed=args.seed, device=True)
+    dg = device_graph(args.config, args.seed)
     torch.cuda.synchronize()
     n, nnz = dg.n, dg.nnz
     p = lvb.params()
     comm = "nccl" if args.backend == "nccl" else "host"
     deg = dg.rowptr[1:] - dg.rowptr[:-1]
     n_act = int((deg > 0).sum().item())
-    rp_h = dg.rowptr.cpu().numpy()
-    lo, hi = edge_balanced_ranges(rp_h, world)[rank]
+    lo, hi = edge_balanced_ranges(dg.rowptr.cpu().numpy(), world)[rank]
     rl, cl, _ = local_rows(dg.rowptr, dg.col, None, lo, hi)
     stream = torch.cuda.Stream()
     g = lvb.Graph.from_csr_dist(n, lo, hi, rl.contiguous(), cl.contiguous(), None, rank=rank, world=world,
@@ -257,15 +360,7 @@ def run_sharded_bench(args, rank, world):
     t_sw1 = float(t[1].item())  # slowest rank's level-0 sweep 1 (incl. the per-bucket exchanges)
     st0 = stats[0]
     edges_per_run = st0["edges_swept"]
-    # roofline per GPU: the byte model of the sweep split over edge-balanced ranks
-    B = sweep_bytes(n_act, nnz, D=nnz, moved=st0["moved_first"]) / world
-    achieved = B / (t_sw1 / 1e3) / 1e9
-    peak, peak_src = measured_peak_hbm()
-    roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-                "traffic": None,
-                "kernel": "level-0 sweep 1 body per GPU (bucket kernels + commits + move all-gathers)",
-                "algorithmic_bytes": B, "t_ms": t_sw1, "peak_source": peak_src,
-                "traffic_source": "not captured at N > 1 (ncu runs on one GPU)"}
+    roofline = roofline_of(args, n_act, nnz, st0, t_sw1, world)
     del g
     # end to end: every rank uploads its rows from pinned host memory, runs, reads the labels back
     h_rl = torch.empty(rl.numel(), dtype=torch.int64, pin_memory=True)
@@ -289,12 +384,10 @@ def run_sharded_bench(args, rank, world):
     out = {"metric": METRIC, "value": edges_per_run / (ms_per_step / 1e3), "unit": UNIT, "n_gpus": world,
            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
            "scaling": "strong", "vs_baseline": None, "dtype": "int64", "data": "synthetic",
-           "config": {"workload": f"{cfg_name(args.scale)} R-MAT scale {args.scale}, {8 << args.scale} tuples, seed {args.seed}, "
-                                  "unit weights, isolated vertices removed",
-                      "n": n, "nnz": nnz, "l2": "inputs larger than L2",
-                      "parallelism": f"{world} GPUs, sweep vertex-sharded (edge-balanced ranges), per-bucket "
-                                     f"{'NCCL' if comm == 'nccl' else 'host-staged'} all-gather of moves, "
-                                     "per-sweep all-reduce of the L change"},
+           "config": dict(workload(args, n, nnz), l2="inputs larger than L2",
+                          parallelism=f"{world} GPUs, sweep vertex-sharded (edge-balanced ranges), per-bucket "
+                                      f"{'NCCL' if comm == 'nccl' else 'host-staged'} all-gather of moves, "
+                                      "per-sweep all-reduce of the L change"),
            "roofline": roofline, "clocks": clk.summary(), "gpu_launches": int(launches),
            "q_final": st0["q"], "levels": st0["levels"],
            "sweeps_per_level": st0["sweeps_per_level"], "louvain_wall_ms": ms_per_step,
@@ -307,7 +400,6 @@ def run_sharded_bench(args, rank, world):
 
 
 def run_ours(args, rank, world):
-    import numpy as np
     import torch
     import torch.distributed as dist
 
@@ -316,7 +408,7 @@ def run_ours(args, rank, world):
 
     dev = torch.device("cuda", torch.cuda.current_device())
     t0 = time.perf_counter()
-    dg = graphgen.rmat(args.scale, seed=args.seed, device=True)
+    dg = device_graph(args.config, args.seed)
     torch.cuda.synchronize()
     gen_s = time.perf_counter() - t0
     n, nnz = dg.n, dg.nnz
@@ -360,35 +452,32 @@ def run_ours(args, rank, world):
 
     # roofline of the dominant kernel sequence: the level-0 sweep body (sweep 1)
     t_sw1 = statistics.mean(s["t_sweep_ms_first"] for s in stats)
-    moved1 = st0["moved_first"]
-    B = sweep_bytes(n_act, nnz, D=nnz, moved=moved1)
-    achieved = B / (t_sw1 / 1e3) / 1e9
-    peak, peak_src = measured_peak_hbm()
-    traffic, traffic_src = recorded_traffic() if args.scale == 27 else (None, None)  # the capture is of C5
-    roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-                "traffic": traffic, "kernel": "level-0 sweep 1 body (7 bucket kernels + commits)",
-                "algorithmic_bytes": B, "t_ms": t_sw1, "peak_source": peak_src,
-                "traffic_source": traffic_src}
-
+    roofline = roofline_of(args, n_act, nnz, st0, t_sw1)
+    med = {k: statistics.median(s[k] for s in stats) for k in ("t_sweep_ms_total", "t_modularity_ms_total")}
     out = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
            "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
            "scaling": "weak", "vs_baseline": None, "dtype": "int64", "data": "synthetic",
-           "config": {"workload": f"{cfg_name(args.scale)} R-MAT scale {args.scale}, {8 << args.scale} tuples, seed {args.seed}, "
-                                  "unit weights, isolated vertices removed",
-                      "n": n, "nnz": nnz, "n_active": n_act,
-                      "l2": "inputs larger than L2 (col array alone is 4*nnz bytes >> 126 MB)",
-                      "parallelism": "1 GPU" if world == 1 else f"{world} independent replicas"},
+           "config": dict(workload(args, n, nnz), n_active=n_act,
+                          l2="inputs larger than L2" if nnz * 4 > 126e6 else
+                          "graph fits L2 (small config; no flush: every run re-reads it after the previous "
+                          "run's writes)",
+                          parallelism="1 GPU" if world == 1 else f"{world} independent replicas"),
            "roofline": roofline, "clocks": clocks,
            "gpu_launches": int(sum(s["kernel_launches"] for s in stats)),
            "cub_calls": int(sum(s["cub_calls"] for s in stats)),
            "louvain_wall_ms": ms_per_step, "q_final": st0["q"], "levels": st0["levels"],
            "sweeps_per_level": st0["sweeps_per_level"], "n_per_level": st0["n"], "nnz_per_level": st0["nnz"],
            "sweep1_ms": t_sw1, "sweep1_edges_per_s": nnz / (t_sw1 / 1e3),
-           "sweep_edges_per_s_all": edges_per_run / (st0["t_sweep_ms_total"] / 1e3),
-           "t_sweep_ms_total": st0["t_sweep_ms_total"], "t_modularity_ms_total": st0["t_modularity_ms_total"],
-           "t_opt_ms": sum(st0["t_opt_ms"]), "t_agg_ms": sum(st0["t_agg_ms"]), "gen_s": gen_s}
+           "sweep_edges_per_s_all": edges_per_run / (med["t_sweep_ms_total"] / 1e3),
+           "t_sweep_ms_total": med["t_sweep_ms_total"], "t_modularity_ms_total": med["t_modularity_ms_total"],
+           "t_opt_ms": sum(st0["t_opt_ms"]), "t_agg_ms": sum(st0["t_agg_ms"]),
+           "agg_share": sum(st0["t_agg_ms"]) / st0["t_total_ms"] if st0["t_total_ms"] else None,
+           "gen_s": gen_s}
+    out.update(level0_fields(st0, nnz))
 
-    # end to end through the C-ABI with host buffers (H2D of the CSR and D2H of labels every step)
+    # end to end through the C-ABI with host buffers: every step copies the CSR from pinned
+    # host memory (louvain_create_csr), runs, and reads the labels back; the parts are timed
+    # on the host (wall clock), one untimed warm-up step, then the median of the steps
     h_rowptr = torch.empty(n + 1, dtype=torch.int64, pin_memory=True)
     h_col = torch.empty(nnz, dtype=torch.int32, pin_memory=True)
     h_lab = torch.empty(n, dtype=torch.int32, pin_memory=True)
@@ -396,32 +485,37 @@ def run_ours(args, rank, world):
     h_col.copy_(dg.col)
     del g
     torch.cuda.synchronize()
-    e2e_s = []
+    parts = []
     for it in range(max(0, args.e2e_warmup) + max(1, args.e2e_steps)):
         if world > 1:
             dist.barrier()
         torch.cuda.synchronize()
-        t = time.perf_counter()
-        with lvb.Graph.from_csr(h_rowptr, h_col) as ge:
-            ge.run(p, labels_out=h_lab)
+        t_a = time.perf_counter()
+        ge = lvb.Graph.from_csr(h_rowptr, h_col)  # H2D + level setup (synchronous)
+        t_b = time.perf_counter()
+        ge.run(p, labels_out=h_lab)                # run + labels D2H (synchronous)
+        t_c = time.perf_counter()
+        ge.close()
         torch.cuda.synchronize()
+        t_d = time.perf_counter()
         if it >= max(0, args.e2e_warmup):  # untimed warm-up steps first, like the device-timed metric
-            e2e_s.append(time.perf_counter() - t)
-    t_e2e = statistics.median(e2e_s)
+            parts.append((t_d - t_a, t_b - t_a, t_c - t_b, t_d - t_c))
+    parts.sort()
+    t_e2e, t_create, t_run, t_close = parts[len(parts) // 2]
     if world > 1:
         t = torch.tensor([t_e2e], device=dev, dtype=torch.float64)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         t_e2e = float(t.item())
     out["e2e"] = {"value": world * edges_per_run / t_e2e, "unit": UNIT,
                   "h2d_bytes_per_step": 8 * (n + 1) + 4 * nnz, "d2h_bytes_per_step": 4 * n,
-                  "ms_per_step": 1e3 * t_e2e}
+                  "ms_per_step": 1e3 * t_e2e,
+                  "parts_ms": {"create_h2d_setup": 1e3 * t_create, "run_and_labels_d2h": 1e3 * t_run,
+                               "destroy": 1e3 * t_close},
+                  "steps": len(parts), "warmup": max(0, args.e2e_warmup)}
 
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         hg = graphgen.Graph(n, h_rowptr.numpy(), h_col.numpy())
-        r, e, dt, nv = oracle_rate(hg, args.cpu_seconds)
-        out["cpu_baseline"] = {"value": r, "unit": UNIT, "cores": 1, "kind": "oracle",
-                               "sample": f"oracle computeMove (Alg. 2) for {nv} random vertices ({e} directed "
-                                         f"edges, {dt:.1f} s) of the level-0 singleton state of the same graph"}
+        out["cpu_baseline"] = cpu_baseline_line(hg, args.cpu_seconds)
     if rank == 0:
         emit(out)
 

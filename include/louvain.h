@@ -83,6 +83,7 @@ typedef struct {
   double t_modularity_ms_total;
   int64_t edges_swept;        /* sum over executed sweeps of nnz of their level */
   int64_t moved_first;        /* moves of level 0, sweep 1 */
+  double t_sweep_ms_level0[32]; /* each of the first 32 level-0 sweep bodies (median / phase-1 rates) */
   int64_t kernel_launches;    /* explicit kernel launches by the library during the call */
   int64_t cub_calls;          /* device-wide CUB primitives (scan/sort/reduce) during the call */
   louvain_qnum_t q;

@@ -53,6 +53,8 @@ def lib():
         L.orc_decide_batch.argtypes = [i64, vp, vp, vp, vp, vp, vp, ctypes.c_uint64, ctypes.c_int32, i64, vp, vp]
         L.orc_sweep.argtypes = [i64, vp, vp, vp, ctypes.POINTER(Params), vp, vp, vp, ctypes.c_uint64]
         L.orc_sweep.restype = i64
+        L.orc_sweep_counted.argtypes = [i64, vp, vp, vp, ctypes.POINTER(Params), vp, vp, vp, ctypes.c_uint64, vp]
+        L.orc_sweep_counted.restype = i64
         L.orc_contract.argtypes = [i64, vp, vp, vp, vp, vp, vp, vp, vp, vp]
         L.orc_contract.restype = i64
         L.orc_louvain.argtypes = [i64, vp, vp, vp, ctypes.POINTER(Params), vp, ctypes.POINTER(Stats)]
@@ -144,6 +146,14 @@ class State:
         n, rowptr, col, w = _g(self.g)
         return int(lib().orc_sweep(n, _ptr(rowptr), _ptr(col), _ptr(w), ctypes.byref(p), _ptr(self.C),
                                    _ptr(self.a), _ptr(self.size), self.W))
+
+    def sweep_counted(self, p: Params) -> tuple[int, int]:
+        """One sweep; returns (moved, D) with D the distinct (vertex, candidate label) pairs evaluated."""
+        n, rowptr, col, w = _g(self.g)
+        D = ctypes.c_int64()
+        moved = int(lib().orc_sweep_counted(n, _ptr(rowptr), _ptr(col), _ptr(w), ctypes.byref(p), _ptr(self.C),
+                                            _ptr(self.a), _ptr(self.size), self.W, ctypes.addressof(D)))
+        return moved, int(D.value)
 
     def qnum(self) -> tuple[int, int, int]:
         return modularity(self.g, self.C)

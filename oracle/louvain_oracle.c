@@ -117,7 +117,7 @@ static void ws_free(orc_ws* ws) { free(ws->acc); free(ws->touched); }
  * strictly positive gain (R6); singleton rule of P:148-152/P:172 (R8, R9). */
 static int32_t decide_ws(orc_ws* ws, const int64_t* rowptr, const int32_t* col, const uint32_t* w,
                          const int32_t* C, const uint64_t* a, const int64_t* size, uint64_t W,
-                         int64_t i, int32_t rule) {
+                         int64_t i, int32_t rule, int64_t* dcount) {
   int32_t own = C[i];
   uint64_t ki = 0;
   int64_t nt = 0;
@@ -136,6 +136,7 @@ static int32_t decide_ws(orc_ws* ws, const int64_t* rowptr, const int32_t* col, 
   for (int64_t t = 0; t < nt; ++t) {
     int32_t c = ws->touched[t];
     if (c == own) continue;
+    if (dcount) ++*dcount; /* measurement only: distinct candidate labels */
     if (rule == 2 && size[own] == 1 && size[c] == 1 && c > own) continue; /* R8 filter */
     int64_t s = (int64_t)W * (int64_t)ws->acc[c] - (int64_t)ki * (int64_t)a[c];
     if (best < 0 || s > s_best || (s == s_best && c < best)) { best = c; s_best = s; }
@@ -151,7 +152,7 @@ int32_t orc_decide(int64_t n, const int64_t* rowptr, const int32_t* col, const u
                    int64_t i, int32_t singleton_rule) {
   orc_ws ws;
   ws_init(&ws, n);
-  int32_t r = decide_ws(&ws, rowptr, col, w, C, a, size, W, i, singleton_rule);
+  int32_t r = decide_ws(&ws, rowptr, col, w, C, a, size, W, i, singleton_rule, NULL);
   ws_free(&ws);
   return r;
 }
@@ -162,7 +163,7 @@ void orc_decide_batch(int64_t n, const int64_t* rowptr, const int32_t* col, cons
   orc_ws ws;
   ws_init(&ws, n);
   for (int64_t t = 0; t < nv; ++t)
-    out[t] = decide_ws(&ws, rowptr, col, w, C, a, size, W, verts[t], singleton_rule);
+    out[t] = decide_ws(&ws, rowptr, col, w, C, a, size, W, verts[t], singleton_rule, NULL);
   ws_free(&ws);
 }
 
@@ -186,6 +187,13 @@ static void move_vertex(int32_t* C, uint64_t* a, int64_t* size, int64_t i, int32
 
 int64_t orc_sweep(int64_t n, const int64_t* rowptr, const int32_t* col, const uint32_t* w,
                   const orc_params* p, int32_t* C, uint64_t* a, int64_t* size, uint64_t W) {
+  return orc_sweep_counted(n, rowptr, col, w, p, C, a, size, W, NULL);
+}
+
+int64_t orc_sweep_counted(int64_t n, const int64_t* rowptr, const int32_t* col, const uint32_t* w,
+                          const orc_params* p, int32_t* C, uint64_t* a, int64_t* size, uint64_t W,
+                          int64_t* D_out) {
+  if (D_out) *D_out = 0;
   orc_ws ws;
   ws_init(&ws, n);
   uint64_t* k = (uint64_t*)malloc(sizeof(uint64_t) * (size_t)(n > 0 ? n : 1));
@@ -195,7 +203,7 @@ int64_t orc_sweep(int64_t n, const int64_t* rowptr, const int32_t* col, const ui
     /* Sequential Louvain: each vertex in turn, ascending id, immediate
      * update, no singleton rule (R23). */
     for (int64_t i = 0; i < n; ++i) {
-      int32_t t = decide_ws(&ws, rowptr, col, w, C, a, size, W, i, 0);
+      int32_t t = decide_ws(&ws, rowptr, col, w, C, a, size, W, i, 0, D_out);
       if (t != C[i]) { move_vertex(C, a, size, i, t, k[i]); ++moved; }
     }
   } else {
@@ -212,7 +220,7 @@ int64_t orc_sweep(int64_t n, const int64_t* rowptr, const int32_t* col, const ui
         if (p->mode == ORC_RELAXED || bi == b) vset[nv++] = i;
       }
       for (int64_t t = 0; t < nv; ++t)
-        newComm[t] = decide_ws(&ws, rowptr, col, w, C, a, size, W, vset[t], p->singleton_rule);
+        newComm[t] = decide_ws(&ws, rowptr, col, w, C, a, size, W, vset[t], p->singleton_rule, D_out);
       for (int64_t t = 0; t < nv; ++t) {
         int64_t i = vset[t];
         if (newComm[t] != C[i]) { move_vertex(C, a, size, i, newComm[t], k[i]); ++moved; }

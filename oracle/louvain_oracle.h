@@ -69,6 +69,12 @@ void orc_decide_batch(int64_t n, const int64_t* rowptr, const int32_t* col, cons
  * (SEQ).  Updates C, a, size in place; returns the number of moves. */
 int64_t orc_sweep(int64_t n, const int64_t* rowptr, const int32_t* col, const uint32_t* w,
                   const orc_params* p, int32_t* C, uint64_t* a, int64_t* size, uint64_t W);
+/* orc_sweep that also returns D (measurement only, SURVEY 8(d) byte model): the
+ * number of distinct (vertex, candidate label != own) pairs the sweep's
+ * decisions evaluated, each against its own bucket-start snapshot. */
+int64_t orc_sweep_counted(int64_t n, const int64_t* rowptr, const int32_t* col, const uint32_t* w,
+                          const orc_params* p, int32_t* C, uint64_t* a, int64_t* size, uint64_t W,
+                          int64_t* D_out);
 
 /* Alg. 3 CONTRACT with R17/R18.  Outputs go to caller buffers of
  * capacity rowptr_out[n+1], col_out[nnz], w_out[nnz], map_out[n].  Returns n'. */

@@ -56,6 +56,7 @@ class Stats(ctypes.Structure):
                 ("t_total_ms", ctypes.c_double), ("t_sweep_ms_total", ctypes.c_double),
                 ("t_sweep_ms_first", ctypes.c_double), ("t_modularity_ms_total", ctypes.c_double),
                 ("edges_swept", ctypes.c_int64), ("moved_first", ctypes.c_int64),
+                ("t_sweep_ms_level0", ctypes.c_double * 32),
                 ("kernel_launches", ctypes.c_int64), ("cub_calls", ctypes.c_int64), ("q", QNum)]
 
     def as_dict(self) -> dict:
@@ -68,6 +69,7 @@ class Stats(ctypes.Structure):
                 "t_total_ms": self.t_total_ms, "t_sweep_ms_total": self.t_sweep_ms_total,
                 "t_sweep_ms_first": self.t_sweep_ms_first, "t_modularity_ms_total": self.t_modularity_ms_total,
                 "edges_swept": self.edges_swept, "moved_first": self.moved_first,
+                "t_sweep_ms_level0": list(self.t_sweep_ms_level0[:min(32, self.sweeps_per_level[0] if lv else 0)]),
                 "kernel_launches": self.kernel_launches, "cub_calls": self.cub_calls, "q": self.q.q, "L": int(self.q.L), "S": self.q.S,
                 "W": int(self.q.W)}
 

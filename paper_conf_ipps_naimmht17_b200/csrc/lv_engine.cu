@@ -179,7 +179,6 @@ int32_t scratch_get(Handle& h, int slot, size_t bytes, void** out) {
       }
       S.bytes[slot] = want;
     }
-    if (slot == SC_GTAB) S.gtab_init = nullptr;  // contents unknown: re-initialise
   }
   *out = S.p[slot];
   return LOUVAIN_OK;
@@ -528,6 +527,7 @@ int32_t run_impl(Handle& h, const louvain_params_t& p, int32_t* labels_out, louv
           local.t_sweep_ms_first = t_sw;
           local.moved_first = (int64_t)h.h_ctl->logn;
         }
+        if (level == 0 && sweeps < 32) local.t_sweep_ms_level0[sweeps] = t_sw;
         local.edges_swept += L.nnz;
         ++sweeps;
         if (h.h_ctl->overflow) {

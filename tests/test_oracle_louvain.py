@@ -218,3 +218,23 @@ def test_adaptive_theta_one_sweep_per_large_level():
     assert all(s == 1 for s in r.sweeps_per_level)
     L, S, W = oracle.modularity(g, r.labels)
     assert (L, S) == (r.L, r.S)
+
+
+def test_sweep_D_count():
+    """D of the byte model: distinct (i, c != C(i)) pairs evaluated by a sweep.
+    Closed form on a simple graph from singletons under RELAXED (one snapshot, every neighbour
+    its own label): D = nnz - (number of self-loop entries) = nnz.  Under BIN_SYNC later buckets
+    see merged labels, so D <= nnz; the counted sweep moves exactly like the plain one."""
+    for g in (graphgen.karate(), graphgen.rmat(10, seed=3), graphgen.lfr(2000, kmin=4, kmax=60, smin=20,
+                                                                              smax=200, seed=4)):
+        st = oracle.State(g)
+        moved, D = st.sweep_counted(oracle.params(mode=oracle.RELAXED))
+        assert D == g.nnz
+        s1, s2 = oracle.State(g), oracle.State(g)
+        m1, D1 = s1.sweep_counted(oracle.params())
+        m2 = s2.sweep(oracle.params())
+        assert m1 == m2 and s1.C.tolist() == s2.C.tolist() and D1 <= g.nnz
+    # a weighted graph with self-loops: the loop is not a candidate (R3)
+    g = graphgen.weighted_csr(3, [0, 0, 1], [0, 1, 2], [5, 1, 2])
+    _, D = oracle.State(g).sweep_counted(oracle.params(mode=oracle.RELAXED))
+    assert D == g.nnz - 1

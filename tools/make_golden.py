@@ -42,7 +42,7 @@ def labels_sha(lab) -> str:
     return hashlib.sha256(np.ascontiguousarray(lab, dtype=np.int32).tobytes()).hexdigest()
 
 
-def run(name):
+def run(name, sweeps_only=False):
     build, desc = CONFIGS[name]
     t0 = time.time()
     g = build()
@@ -55,12 +55,14 @@ def run(name):
     sw = []
     for s in range(2):
         t0 = time.time()
-        moved = st.sweep(p)
+        moved, D = st.sweep_counted(p)  # D: distinct (vertex, candidate label) pairs (byte model)
         L, S, W = st.qnum()
-        sw.append({"moved": moved, "L": L, "S": S, "W": W, "labels_sha256": labels_sha(st.C),
+        sw.append({"moved": moved, "D": D, "L": L, "S": S, "W": W, "labels_sha256": labels_sha(st.C),
                    "oracle_s": time.time() - t0})
     res["level0_sweeps_b"] = sw
     del st
+    if sweeps_only:
+        return res
     for tag, mode in (("b", oracle.BIN_SYNC), ("a", oracle.SEQ), ("a_adaptive", oracle.SEQ_ADAPTIVE)):
         t0 = time.time()
         r = oracle.louvain(g, oracle.params(mode=mode))
@@ -77,7 +79,9 @@ def run(name):
 
 
 def main():
-    names = sys.argv[1:] or list(CONFIGS)
+    args = [a for a in sys.argv[1:] if not a.startswith("--")]
+    sweeps_only = "--sweeps-only" in sys.argv  # level-0 sweeps 1-2 only (merged into the config's record)
+    names = args or list(CONFIGS)
     data = {}
     if os.path.exists(OUT):
         with open(OUT) as f:
@@ -86,6 +90,15 @@ def main():
                        "graphgen/; see DESIGN.md 'Input recipe'")
     for name in names:
         print(f"[{time.strftime('%X')}] {name} ...", flush=True)
+        if sweeps_only:
+            cur = json.load(open(OUT)) if os.path.exists(OUT) else {}
+            rec = cur.get(name, {})
+            rec["level0_sweeps_b"] = run(name, True)["level0_sweeps_b"]
+            cur[name] = rec
+            with open(OUT, "w") as f:
+                json.dump(cur, f, indent=1, sort_keys=True)
+            print(f"   {name}: level-0 sweeps {rec['level0_sweeps_b']}", flush=True)
+            continue
         data[name] = run(name)
         print(f"   b: Q={data[name]['b']['q']:.6f} levels={data[name]['b']['levels']}  "
               f"a: Q={data[name]['a']['q']:.6f}  gap={data[name]['gap_a_minus_b']:+.5f}  "
