@@ -142,8 +142,6 @@ struct PartPlan {
   int64_t bucket_task[9] = {0};   // tasks of bucket b: [bucket_task[b-1], bucket_task[b])
   int64_t bucket_vert[9] = {0};   // plan vertices of bucket b
   int64_t bucket_chunk[9] = {0};  // chunks of bucket b (pre-partitioned vertices only)
-  uint8_t* posP = nullptr;        // [n] per bin position: P of a streaming plan vertex, else 0
-  uint8_t* pb = nullptr;          // [nnz + 64] stage partition bytes (scratch SC_PB): part_of(label, P)
   int64_t bucket_vsplit[8] = {0};  // bucket b's vertices [bucket_vert[b-1], vsplit) are pre-partitioned,
   int64_t bucket_tsplit[8] = {0};  // tasks [bucket_task[b-1], tsplit); the rest stream (P <= kStreamMaxP)
 };
@@ -192,7 +190,7 @@ struct Level {
 // every level and every run): avoids multi-GB stream-ordered allocations
 // churning the memory pool between levels.
 enum ScratchSlot {
-  SC_STAGE = 0, SC_GC, SC_GW, SC_OC, SC_OW, SC_K1, SC_V0, SC_V1, SC_TMP, SC_TILES, SC_PB,
+  SC_STAGE = 0, SC_GC, SC_GW, SC_OC, SC_OW, SC_K1, SC_V0, SC_V1, SC_TMP, SC_TILES,
   // arrays of a contracted level inside louvain_run, double-buffered by level parity
   SC_LVL0, SC_LVL_END = SC_LVL0 + 2 * 12, SC_COUNT = SC_LVL_END
 };
@@ -311,8 +309,7 @@ int32_t validate_csr_host(int64_t n, int64_t nnz, const int64_t* rowptr, const i
 // ------------------------------------------------------------------ sweep (lv_sweep.cu)
 int32_t launch_sweep_bucket(Handle& h, Level& L, const louvain_params_t& p, int bucket);
 // phase 1 gather for bin positions [pos0,pos1), staged entries [s0,s1)
-int32_t launch_stage(Handle& h, Level& L, int64_t pos0, int64_t pos1, int64_t s0, int64_t s1, bool pb);
-bool pb_on();  // partition bytes for the streaming hub tasks (LV_PB=0: re-hash the records)
+int32_t launch_stage(Handle& h, Level& L, int64_t pos0, int64_t pos1, int64_t s0, int64_t s1);
 int32_t build_part_plan(Handle& h, Level& L);
 
 // ------------------------------------------------------------------ launch geometry

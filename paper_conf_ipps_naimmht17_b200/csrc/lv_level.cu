@@ -785,16 +785,10 @@ static int32_t build_hub_plan(Handle& h, Level& L) {
   return LOUVAIN_OK;
 }
 
-__global__ void k_set_posP(const int32_t* __restrict__ vert_pos, const int32_t* __restrict__ vert_P, int64_t nv,
-                           int32_t maxp, uint8_t* posP) {
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < nv; i += (int64_t)gridDim.x * blockDim.x)
-    if (vert_P[i] <= maxp) posP[vert_pos[i]] = (uint8_t)vert_P[i];
-}
-
 static void part_free(PartPlan& Q, cudaStream_t s) {
   dfree(Q.task_vpos, s); dfree(Q.task_p, s); dfree(Q.vert_pos, s); dfree(Q.vert_P, s); dfree(Q.vert_first, s);
   dfree(Q.vert_pbase, s); dfree(Q.done, s); dfree(Q.partial, s); dfree(Q.poff, s); dfree(Q.pcur, s);
-  dfree(Q.chunks, s); dfree(Q.posP, s);
+  dfree(Q.chunks, s);
   Q = PartPlan();
 }
 
@@ -872,19 +866,6 @@ int32_t build_part_plan(Handle& h, Level& L) {
   LV_CUDA(cudaMemcpyAsync(Q.vert_first, vfirst.data(), 4 * vfirst.size(), cudaMemcpyHostToDevice, s));
   LV_CUDA(cudaMemcpyAsync(Q.vert_pbase, vpb.data(), 8 * vpb.size(), cudaMemcpyHostToDevice, s));
   LV_CUDA(cudaMemcpyAsync(Q.chunks, ch.data(), sizeof(PartChunk) * ch.size(), cudaMemcpyHostToDevice, s));
-  if (pb_on()) {  // per bin position: P of every streaming vertex (k_stage writes its partition bytes)
-    int64_t nstream = 0;
-    for (int64_t i = 0; i < Q.nverts; ++i) nstream += vP[i] <= kStreamMaxP;
-    if (nstream > 0) {
-      LV_TRY(dalloc(&Q.posP, L.n, s));
-      LV_CUDA(cudaMemsetAsync(Q.posP, 0, (size_t)L.n, s));
-      k_set_posP<<<grid_for(Q.nverts, 256), 256, 0, s>>>(Q.vert_pos, Q.vert_P, Q.nverts, (int32_t)kStreamMaxP, Q.posP);
-      LV_LAUNCHED();
-      void* p = nullptr;
-      LV_TRY(scratch_get(h, SC_PB, (size_t)L.nnz + 64, &p));
-      Q.pb = static_cast<uint8_t*>(p);
-    }
-  }
   LV_CUDA(cudaStreamSynchronize(s));  // host vectors die here
   return LOUVAIN_OK;
 }

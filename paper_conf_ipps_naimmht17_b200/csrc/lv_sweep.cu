@@ -309,21 +309,14 @@ constexpr uint32_t kSelf = 0xFFFFFFFFu;
 constexpr int kStageTile = 4096;
 constexpr int kStageRows = 256;
 
-// PB (the hub range of a bucket): entries of the streaming hub vertices (posP[i] =
-// P > 0 label partitions) also get pb[t] = part_of(label, P), 0xFF for the
-// self-loop, so each of the P tasks of the vertex scans one byte per entry
-// instead of re-reading and re-hashing the 8-byte records (sweep_part_stream).
-template <bool PB>
 __global__ void __launch_bounds__(256) k_stage(const int32_t* __restrict__ bv, const int64_t* __restrict__ soff,
                                                int64_t pos0, int64_t pos1, const int64_t* __restrict__ tr,
                                                const int64_t* __restrict__ rowptr,
                                                const int32_t* __restrict__ col, const uint2* __restrict__ ca,
-                                               uint2* __restrict__ stage, const uint8_t* __restrict__ posP,
-                                               uint8_t* __restrict__ pb) {
+                                               uint2* __restrict__ stage) {
   __shared__ int64_t sh_so[kStageRows + 1];
   __shared__ int64_t sh_rb[kStageRows];
   __shared__ int32_t sh_v[kStageRows];
-  __shared__ uint8_t sh_P[PB ? kStageRows : 1];
   __shared__ int64_t sh_i0;
   __shared__ int sh_nr;
   const int64_t s0 = soff[pos0], s1 = soff[pos1];
@@ -343,12 +336,10 @@ __global__ void __launch_bounds__(256) k_stage(const int32_t* __restrict__ bv, c
       sh_v[r] = v;
       sh_so[r] = soff[i0 + r];
       sh_rb[r] = rowptr[v];
-      if (PB) sh_P[r] = posP[i0 + r];
     }
     __syncthreads();
     for (int64_t base = t0 + threadIdx.x; base < t1; base += 4 * (int64_t)blockDim.x) {
       int32_t jj[4], vv[4];
-      uint32_t PP[4];
       uint2 rr[4];
 #pragma unroll
       for (int q = 0; q < 4; ++q) {
@@ -365,7 +356,6 @@ __global__ void __launch_bounds__(256) k_stage(const int32_t* __restrict__ bv, c
             }
             vv[q] = sh_v[lo];
             e = sh_rb[lo] + (t - sh_so[lo]);
-            if (PB) PP[q] = sh_P[lo];
           } else {
             int64_t lo = pos0, hi = pos1 - 1;
             while (lo < hi) {
@@ -374,7 +364,6 @@ __global__ void __launch_bounds__(256) k_stage(const int32_t* __restrict__ bv, c
             }
             vv[q] = bv[lo];
             e = rowptr[vv[q]] + (t - soff[lo]);
-            if (PB) PP[q] = posP[lo];
           }
           jj[q] = __ldcs(&col[e]);
         }
@@ -388,10 +377,7 @@ __global__ void __launch_bounds__(256) k_stage(const int32_t* __restrict__ bv, c
         // displace the gathered records
         const uint2 val = (jj[q] == vv[q]) ? make_uint2(kSelf, 0u)
                                            : make_uint2(rr[q].x, rr[q].x == (uint32_t)jj[q] ? rr[q].y : kUnknownA);
-        if (t < t1) {
-          __stcs(&stage[t], val);
-          if (PB && PP[q]) pb[t] = (jj[q] == vv[q]) ? (uint8_t)0xFF : (uint8_t)part_of((int32_t)rr[q].x, PP[q]);
-        }
+        if (t < t1) __stcs(&stage[t], val);
       }
     }
     __syncthreads();
@@ -882,9 +868,7 @@ __device__ __forceinline__ unsigned part_insert(unsigned long long* T, uint32_t*
 // matching entries into a shared queue (ballot + popc) and inserts 32 at a time.
 // Measured faster than pre-partitioning at C5 level 0 (15 vs 24 ms), slower for
 // the giant hubs of the contracted levels, which take the pre-partitioned tasks.
-// PB: the task scans the vertex's partition bytes (k_stage<true>), 16 per lane
-// and load, and reads the 8-byte records of its own entries only.
-template <bool UNIT, bool PB>
+template <bool UNIT>
 __global__ void __launch_bounds__(1024) sweep_part_stream(const int32_t* __restrict__ task_vpos,
                                                   const int32_t* __restrict__ task_p, int64_t t_begin, int64_t t_end,
                                                   const int32_t* __restrict__ vert_pos,
@@ -892,8 +876,7 @@ __global__ void __launch_bounds__(1024) sweep_part_stream(const int32_t* __restr
                                                   const int32_t* __restrict__ vert_first, int32_t* done,
                                                   Partial* part, unsigned long long* overflow,
                                                   const int32_t* __restrict__ bv, const int64_t* __restrict__ soff,
-                                                  const uint2* __restrict__ stage, SweepArgs A,
-                                                  const uint8_t* __restrict__ pb) {
+                                                  const uint2* __restrict__ stage, SweepArgs A) {
   extern __shared__ unsigned long long smem[];
   unsigned long long* T = smem;
   uint32_t* TA = reinterpret_cast<uint32_t*>(smem + kPartSlots);
@@ -967,66 +950,38 @@ __global__ void __launch_bounds__(1024) sweep_part_stream(const int32_t* __restr
         insert_one(e, x);
       }
     };
-    // push one candidate per lane (or none) into the warp queue; a full queue is inserted
-    auto push = [&](bool valid, uint2 e, uint32_t x) {
-      const unsigned m = __ballot_sync(kFull, valid);
-      if (valid) {
-        const int slot = qn + __popc(m & lanemask_lt());
-        Q[slot] = e;
-        QW[slot] = x;
-      }
-      qn += __popc(m);
-      if (qn >= 32) {
-        __syncwarp();
-        insert_warp(Q[lane], QW[lane], true);
-        const uint2 mv = (lane < qn - 32) ? Q[32 + lane] : make_uint2(0, 0);
-        const uint32_t mw = (lane < qn - 32) ? QW[32 + lane] : 0u;
-        __syncwarp();
-        if (lane < qn - 32) {
-          Q[lane] = mv;
-          QW[lane] = mw;
-        }
-        qn -= 32;
-        __syncwarp();
-      }
-    };
-    if (PB) {
-      // bytes [sb, sb + deg) of pb, in 16-byte words from the aligned word below sb
-      const int64_t g1 = sb + deg, a0 = sb & ~(int64_t)15;
-      const uint32_t pp = p * 0x01010101u;
-      for (int64_t wb = a0 + 16 * (int64_t)(threadIdx.x - lane); wb < g1; wb += 16 * (int64_t)blockDim.x) {
-        const int64_t w = wb + 16 * lane;
-        uint32_t m = 0;
-        if (w < g1) {
-          const uint4 b = __ldcg(reinterpret_cast<const uint4*>(pb + w));
-          const uint32_t bw[4] = {b.x, b.y, b.z, b.w};
+    for (int64_t base = 0; base + (int64_t)(threadIdx.x - lane) < deg; base += 4 * (int64_t)blockDim.x) {
+      uint2 rr[4];
+      uint32_t ww[4];
 #pragma unroll
-          for (int k = 0; k < 4; ++k)  // one bit per byte equal to p (no carries between the terms)
-            m |= ((((__vcmpeq4(bw[k], pp) >> 7) & 0x01010101u) * 0x01020408u) >> 24 & 0xFu) << (4 * k);
-          const int64_t lo = sb > w ? sb - w : 0, hi = g1 - w < 16 ? g1 - w : 16;
-          m &= (hi >= 16 ? 0xFFFFu : ((1u << hi) - 1u)) & ~((1u << lo) - 1u);
-        }
-        while (__any_sync(kFull, m != 0)) {
-          const bool has = m != 0;
-          const int bit = has ? __ffs(m) - 1 : 0;
-          m &= m - 1;
-          const int64_t t = w + bit - sb;
-          push(has, has ? __ldcg(&S[t]) : make_uint2(kSelf, 0u), UNIT ? 1u : (has ? __ldcg(&Wt[t]) : 0u));
-        }
+      for (int q = 0; q < 4; ++q) {
+        const int64_t t = base + threadIdx.x + (int64_t)q * blockDim.x;
+        rr[q] = (t < deg) ? __ldcg(&S[t]) : make_uint2(kSelf, 0u);
+        ww[q] = UNIT ? 1u : ((t < deg) ? __ldcg(&Wt[t]) : 0u);
       }
-    } else {
-      for (int64_t base = 0; base + (int64_t)(threadIdx.x - lane) < deg; base += 4 * (int64_t)blockDim.x) {
-        uint2 rr[4];
-        uint32_t ww[4];
 #pragma unroll
-        for (int q = 0; q < 4; ++q) {
-          const int64_t t = base + threadIdx.x + (int64_t)q * blockDim.x;
-          rr[q] = (t < deg) ? __ldcg(&S[t]) : make_uint2(kSelf, 0u);
-          ww[q] = UNIT ? 1u : ((t < deg) ? __ldcg(&Wt[t]) : 0u);
+      for (int q = 0; q < 4; ++q) {
+        const bool valid = rr[q].x != kSelf && part_of((int32_t)rr[q].x, P) == p;
+        const unsigned m = __ballot_sync(kFull, valid);
+        if (valid) {
+          const int slot = qn + __popc(m & lanemask_lt());
+          Q[slot] = rr[q];
+          QW[slot] = ww[q];
         }
-#pragma unroll
-        for (int q = 0; q < 4; ++q)
-          push(rr[q].x != kSelf && part_of((int32_t)rr[q].x, P) == p, rr[q], ww[q]);
+        qn += __popc(m);
+        if (qn >= 32) {
+          __syncwarp();
+          insert_warp(Q[lane], QW[lane], true);
+          const uint2 mv = (lane < qn - 32) ? Q[32 + lane] : make_uint2(0, 0);
+          const uint32_t mw = (lane < qn - 32) ? QW[32 + lane] : 0u;
+          __syncwarp();
+          if (lane < qn - 32) {
+            Q[lane] = mv;
+            QW[lane] = mw;
+          }
+          qn -= 32;
+          __syncwarp();
+        }
       }
     }
     __syncwarp();
@@ -1324,10 +1279,8 @@ int32_t launch_part(Handle& h, Level& L, const SweepArgs& A, int bucket, bool un
     LV_TRY(set_smem(sweep_part<false, false>, 12 * (size_t)kPartSlots));
     LV_TRY(set_smem(sweep_part<true, true>, 12 * (size_t)kPartSlots));
     LV_TRY(set_smem(sweep_part<false, true>, 12 * (size_t)kPartSlots));
-    LV_TRY(set_smem(sweep_part_stream<true, false>, 12 * (size_t)kPartSlots));
-    LV_TRY(set_smem(sweep_part_stream<false, false>, 12 * (size_t)kPartSlots));
-    LV_TRY(set_smem(sweep_part_stream<true, true>, 12 * (size_t)kPartSlots));
-    LV_TRY(set_smem(sweep_part_stream<false, true>, 12 * (size_t)kPartSlots));
+    LV_TRY(set_smem(sweep_part_stream<true>, 12 * (size_t)kPartSlots));
+    LV_TRY(set_smem(sweep_part_stream<false>, 12 * (size_t)kPartSlots));
     attr = true;
   }
   auto mark = [&](const char* what) {
@@ -1381,18 +1334,14 @@ int32_t launch_part(Handle& h, Level& L, const SweepArgs& A, int bucket, bool un
     mark("pre-tasks");
   }
   if (t1 > ts) {  // streaming tasks
-    const bool pb = Q.posP != nullptr;  // the stage wrote their partition bytes
-    const unsigned g = grid_for(t1 - ts, 1, 148 * 2);
-    const size_t sm = 12 * (size_t)kPartSlots;
-#define LV_STREAM(U, B)                                                                                           \
-  sweep_part_stream<U, B><<<g, 1024, sm, s>>>(Q.task_vpos, Q.task_p, ts, t1, Q.vert_pos, Q.vert_P, Q.vert_first, \
-                                             Q.done, (Partial*)Q.partial, &h.ctl->overflow, L.bin_vertices,      \
-                                             L.soff, stage, A, Q.pb)
-    if (unit && pb) LV_STREAM(true, true);
-    else if (unit) LV_STREAM(true, false);
-    else if (pb) LV_STREAM(false, true);
-    else LV_STREAM(false, false);
-#undef LV_STREAM
+    if (unit)
+      sweep_part_stream<true><<<grid_for(t1 - ts, 1, 148 * 2), 1024, 12 * (size_t)kPartSlots, s>>>(
+          Q.task_vpos, Q.task_p, ts, t1, Q.vert_pos, Q.vert_P, Q.vert_first, Q.done, (Partial*)Q.partial,
+          &h.ctl->overflow, L.bin_vertices, L.soff, stage, A);
+    else
+      sweep_part_stream<false><<<grid_for(t1 - ts, 1, 148 * 2), 1024, 12 * (size_t)kPartSlots, s>>>(
+          Q.task_vpos, Q.task_p, ts, t1, Q.vert_pos, Q.vert_P, Q.vert_first, Q.done, (Partial*)Q.partial,
+          &h.ctl->overflow, L.bin_vertices, L.soff, stage, A);
     LV_LAUNCHED();
     mark("stream");
   }
@@ -1443,11 +1392,7 @@ int32_t dispatch_class(Handle& h, Level& L, const SweepArgs& A, int bucket, int 
     if (sub == kSubHub && L.hub.nh > 0) LV_TRY(launch_hub<UNIT>(h, L, A, stage, bucket));  // giants (P > kPartMaxP)
   } else {
     static const int* caps = kCapT;
-    static const int* threads = [] {  // LV_THR=a,b,c,d,e: threads per CTA tier (A/B only)
-      static int t[5] = {kThrT[0], kThrT[1], kThrT[2], kThrT[3], kThrT[4]};
-      if (const char* e = getenv("LV_THR")) sscanf(e, "%d,%d,%d,%d,%d", &t[0], &t[1], &t[2], &t[3], &t[4]);
-      return (const int*)t;
-    }();
+    static const int* threads = kThrT;
     static bool attr_done = false;
     if (!attr_done) {
       LV_TRY(set_smem(sweep_cta<true, false>, 12 * (size_t)kCapMax));
@@ -1479,11 +1424,6 @@ int32_t dispatch_class(Handle& h, Level& L, const SweepArgs& A, int bucket, int 
 
 size_t hub_partial_bytes() { return sizeof(Partial); }
 
-bool pb_on() {
-  static const bool on = !(getenv("LV_PB") && getenv("LV_PB")[0] == '0');
-  return on;
-}
-
 // LV_TRACE=2: per-class timing (synchronises the stream; diagnostics only)
 static bool trace_on() {
   static const bool on = getenv("LV_TRACE") && std::string(getenv("LV_TRACE")) == "2";
@@ -1505,17 +1445,12 @@ static void trace_step(Handle& h, Level& L, int bucket, int sub, int64_t pos0, i
           (long)(e[1] - e[0]), ms, ms > 0 ? (e[1] - e[0]) / ms / 1e6 : 0.0);
 }
 
-int32_t launch_stage(Handle& h, Level& L, int64_t pos0, int64_t pos1, int64_t s0, int64_t s1, bool pb) {
+int32_t launch_stage(Handle& h, Level& L, int64_t pos0, int64_t pos1, int64_t s0, int64_t s1) {
   if (s1 <= s0) return LOUVAIN_OK;
   const int64_t* tr = nullptr;
   LV_TRY(tile_starts(h, L.soff, pos0, pos1, s0, s1, kStageTile, &tr));
-  const unsigned grid = grid_for((s1 - s0 + kStageTile - 1) / kStageTile, 1, 148 * 8);
-  if (pb && L.part.posP && pb_on())
-    k_stage<true><<<grid, 256, 0, h.stream>>>(L.bin_vertices, L.soff, pos0, pos1, tr, L.rowptr, L.col, L.ca,
-                                              L.stage, L.part.posP, L.part.pb);
-  else
-    k_stage<false><<<grid, 256, 0, h.stream>>>(L.bin_vertices, L.soff, pos0, pos1, tr, L.rowptr, L.col, L.ca,
-                                               L.stage, nullptr, nullptr);
+  k_stage<<<grid_for((s1 - s0 + kStageTile - 1) / kStageTile, 1, 148 * 8), 256, 0, h.stream>>>(
+      L.bin_vertices, L.soff, pos0, pos1, tr, L.rowptr, L.col, L.ca, L.stage);
   LV_LAUNCHED();
   LV_CUDA(cudaGetLastError());
   return LOUVAIN_OK;
@@ -1559,7 +1494,7 @@ int32_t launch_sweep_bucket(Handle& h, Level& L, const louvain_params_t& p, int 
   // log; the commit waits for both (LV_TRACE=2 serialises).
   const bool overlap = !trace_on() && posp < pos1 && posp > pos0 && L.hub.nh == 0;
   if (overlap) {
-    LV_TRY(launch_stage(h, L, posp, pos1, L.class_soff[cp], L.class_soff[c1], true));
+    LV_TRY(launch_stage(h, L, posp, pos1, L.class_soff[cp], L.class_soff[c1]));
     LV_CUDA(cudaEventRecord(h.ev_fork, h.stream));
     LV_CUDA(cudaStreamWaitEvent(h.side, h.ev_fork, 0));
     cudaStream_t main_s = h.stream;
@@ -1569,12 +1504,12 @@ int32_t launch_sweep_bucket(Handle& h, Level& L, const louvain_params_t& p, int 
     h.stream = main_s;
     LV_TRY(rc);
     LV_CUDA(cudaEventRecord(h.ev_join, h.side));
-    LV_TRY(launch_stage(h, L, pos0, posp, L.class_soff[c0], L.class_soff[cp], false));
+    LV_TRY(launch_stage(h, L, pos0, posp, L.class_soff[c0], L.class_soff[cp]));
     for (int sub = 0; sub < kSubPart; ++sub) LV_TRY(dispatch(sub));
     LV_CUDA(cudaStreamWaitEvent(h.stream, h.ev_join, 0));
     return LOUVAIN_OK;
   }
-  if (pos1 > pos0) LV_TRY(launch_stage(h, L, pos0, pos1, L.class_soff[c0], L.class_soff[c1], true));
+  if (pos1 > pos0) LV_TRY(launch_stage(h, L, pos0, pos1, L.class_soff[c0], L.class_soff[c1]));
   if (trace_on()) trace_step(h, L, bucket, -1, pos0, pos1);
   for (int sub = 0; sub < kSubPerBucket; ++sub) LV_TRY(dispatch(sub));
   return LOUVAIN_OK;
