@@ -188,8 +188,9 @@ int32_t louvain_modularity_owned(louvain_graph_t g, uint64_t* L_owned, uint64_t*
  * are all-gathered and every rank commits all of them to its replica of
  * (C, a_c, size_c) with the same exact integer updates (Alg. 1 l.8-11), so the
  * replicas stay bit-identical; Eq. (1) after a sweep is all-reduced (partial L
- * change of the owned moved rows).  The level graph is replicated on every rank
- * and contraction (Alg. 3) is computed on each (deterministic, identical).
+ * change of the owned moved rows).  The level graph is replicated on every rank;
+ * contraction (Alg. 3) is sharded by new vertex (each rank merges the member rows
+ * of its share of the communities) and the merged rows are all-gathered.
  * Every louvain_* call on a distributed handle that runs a sweep
  * (louvain_sweep, louvain_run) is COLLECTIVE over its ranks; the other calls are
  * local.  Results equal the single-GPU ones bit for bit (and oracle (b)).

@@ -77,13 +77,14 @@ __global__ void k_group_meta(const int32_t* skey, const int32_t* vorder, int64_t
 }
 
 __global__ void k_seg_bounds(const int64_t* rfirst, const int64_t* gpos, int64_t np, int64_t n, int64_t* sstart,
-                             uint8_t* scls, int32_t* rid, unsigned long long* hist) {
+                             uint8_t* scls, int32_t* rid, unsigned long long* hist, int64_t c_lo, int64_t c_hi) {
   __shared__ unsigned long long sh[kSegClasses];
   if (threadIdx.x < kSegClasses) sh[threadIdx.x] = 0;
   __syncthreads();
   for (int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; r < np; r += (int64_t)gridDim.x * blockDim.x) {
     const int64_t b = gpos[rfirst[r]], e = gpos[(r + 1 < np) ? rfirst[r + 1] : n];
     sstart[r] = b;
+    if (r < c_lo || r >= c_hi) continue;  // merged by another rank (sharded contraction)
     const int64_t len = e - b;
     const int c = len <= 32 ? 0 : len <= 128 ? 1 : len <= kWarpMax ? 2 : len < 1024 ? 3 : len < 2048 ? 4
                 : len < 4096 ? 5 : len <= kMidMax ? 6 : 7;
@@ -93,6 +94,25 @@ __global__ void k_seg_bounds(const int64_t* rfirst, const int64_t* gpos, int64_t
   }
   __syncthreads();
   if (threadIdx.x < kSegClasses && sh[threadIdx.x]) atomicAdd(&hist[threadIdx.x], sh[threadIdx.x]);
+}
+
+// Sharded contraction (distributed handle): new vertices [cut[r], cut[r+1]) are merged by
+// rank r, cut[r] = first new vertex whose grouped segment starts at >= r * nnz / world.
+__global__ void k_seg_split(const int64_t* __restrict__ rfirst, const int64_t* __restrict__ gpos, int64_t np,
+                            int64_t nnz, int world, int64_t* cut) {
+  const int r = threadIdx.x;
+  if (r > world) return;
+  if (r == 0 || r == world) {
+    cut[r] = r == 0 ? 0 : np;
+    return;
+  }
+  const int64_t target = (int64_t)((__int128)r * nnz / world);
+  int64_t lo = 0, hi = np;  // lower_bound over segment starts gpos[rfirst[c]]
+  while (lo < hi) {
+    const int64_t mid = (lo + hi) >> 1;
+    if (gpos[rfirst[mid]] < target) lo = mid + 1; else hi = mid;
+  }
+  cut[r] = lo;
 }
 
 // Step 3: every member row copied in source order -- rows read sequentially, each
@@ -111,9 +131,11 @@ __global__ void __launch_bounds__(256) k_scatter_copy(const int64_t* __restrict_
                                                       const uint32_t* __restrict__ w,
                                                       const int32_t* __restrict__ map,
                                                       const int64_t* __restrict__ dbase, int64_t nnz,
-                                                      const int64_t* __restrict__ tr, int32_t* gc, uint32_t* gw) {
+                                                      const int64_t* __restrict__ tr, int32_t* gc, uint32_t* gw,
+                                                      int32_t c_lo, int32_t c_hi) {
   __shared__ int64_t sh_rp[kSRows + 1];
   __shared__ int64_t sh_db[kSRows];
+  __shared__ int32_t sh_mine[kSRows];  // the row's new vertex is in this rank's range [c_lo, c_hi)
   __shared__ int64_t sh_u0;
   __shared__ int sh_nr;
   const int64_t ntiles = (nnz + kSTile - 1) / kSTile;
@@ -130,6 +152,10 @@ __global__ void __launch_bounds__(256) k_scatter_copy(const int64_t* __restrict_
     for (int r = threadIdx.x; r < nr; r += blockDim.x) {
       sh_rp[r] = rowptr[u0 + r];
       sh_db[r] = dbase[u0 + r];
+      if (u0 + r < n) {
+        const int32_t c = map[u0 + r];
+        sh_mine[r] = c >= c_lo && c < c_hi;
+      }
     }
     __syncthreads();
     for (int64_t base = e0 + threadIdx.x; base < e1; base += 4 * (int64_t)blockDim.x) {
@@ -148,6 +174,7 @@ __global__ void __launch_bounds__(256) k_scatter_copy(const int64_t* __restrict_
               if (sh_rp[mid] <= e) lo = mid; else hi = mid - 1;
             }
             dd[q] = sh_db[lo] + (e - sh_rp[lo]);
+            if (!sh_mine[lo]) continue;  // another rank merges this row's community
           } else {
             int64_t lo = 0, hi = n - 1;
             while (lo < hi) {
@@ -155,6 +182,8 @@ __global__ void __launch_bounds__(256) k_scatter_copy(const int64_t* __restrict_
               if (rowptr[mid] <= e) lo = mid; else hi = mid - 1;
             }
             dd[q] = dbase[lo] + (e - rowptr[lo]);
+            const int32_t c = map[lo];
+            if (c < c_lo || c >= c_hi) continue;
           }
           jj[q] = __ldcs(&col[e]);
         }
@@ -165,7 +194,7 @@ __global__ void __launch_bounds__(256) k_scatter_copy(const int64_t* __restrict_
 #pragma unroll
       for (int q = 0; q < 4; ++q) {
         const int64_t e = base + (int64_t)q * blockDim.x;
-        if (e < e1) {
+        if (e < e1 && jj[q] >= 0) {
           gc[dd[q]] = mm[q];
           if (gw) gw[dd[q]] = w ? __ldcs(&w[e]) : 1u;
         }
@@ -675,6 +704,24 @@ int32_t level_contract_fast(Handle& h, Level& L, Level& out, int32_t* d_map, int
   LV_TRY(cub_scan_excl(s, mdeg, gpos, n + 1));
   dfree(mdeg, s);
   dfree(skey, s);
+  // sharded contraction: this rank merges the new vertices [c_lo, c_hi) only (the
+  // steps before are O(n) and replicated); the rows are all-gathered at the end
+  int64_t c_lo = 0, c_hi = np;
+  std::vector<int64_t> cuts;
+  if (h.dist && h.dist->world > 1) {
+    const int world = h.dist->world;
+    int64_t* dcut = nullptr;
+    LV_TRY(dalloc(&dcut, world + 1, s));
+    k_seg_split<<<1, 1024, 0, s>>>(rfirst, gpos, np, nnz, world, dcut);
+    LV_LAUNCHED();
+    cuts.resize(world + 1);
+    LV_CUDA(cudaMemcpyAsync(cuts.data(), dcut, 8 * (world + 1), cudaMemcpyDeviceToHost, s));
+    LV_CUDA(cudaStreamSynchronize(s));
+    dfree(dcut, s);
+    for (int r = 1; r <= world; ++r) cuts[r] = std::max(cuts[r], cuts[r - 1]);
+    c_lo = cuts[h.dist->rank];
+    c_hi = cuts[h.dist->rank + 1];
+  }
   tr.mark(s, "group");
   // 3. grouped copy
   const bool weighted = L.w != nullptr;
@@ -697,7 +744,8 @@ int32_t level_contract_fast(Handle& h, Level& L, Level& out, int32_t* d_map, int
     const int64_t* tr = nullptr;
     LV_TRY(tile_starts(h, L.rowptr, 0, n, 0, nnz, kSTile, &tr));
     k_scatter_copy<<<grid_for((nnz + kSTile - 1) / kSTile, 1, 148 * 8), 256, 0, s>>>(L.rowptr, n, L.col, L.w, d_map,
-                                                                                       dbase, nnz, tr, gc, gw);
+                                                                                       dbase, nnz, tr, gc, gw,
+                                                                                       (int32_t)c_lo, (int32_t)c_hi);
     LV_LAUNCHED();
     dfree(dbase, s);
   }
@@ -715,7 +763,7 @@ int32_t level_contract_fast(Handle& h, Level& L, Level& out, int32_t* d_map, int
   unsigned long long* hist = nullptr;
   LV_TRY(dalloc(&hist, kSegClasses, s));
   LV_CUDA(cudaMemsetAsync(hist, 0, 8 * kSegClasses, s));
-  k_seg_bounds<<<grid_for(np, 256), 256, 0, s>>>(rfirst, gpos, np, n, sstart, scls, rid, hist);
+  k_seg_bounds<<<grid_for(np, 256), 256, 0, s>>>(rfirst, gpos, np, n, sstart, scls, rid, hist, c_lo, c_hi);
   LV_LAUNCHED();
   unsigned long long hh[kSegClasses];
   LV_CUDA(cudaMemcpyAsync(hh, hist, 8 * kSegClasses, cudaMemcpyDeviceToHost, s));
@@ -725,10 +773,11 @@ int32_t level_contract_fast(Handle& h, Level& L, Level& out, int32_t* d_map, int
   dfree(gpos, s);
   {
     size_t tb = 0;
-    LV_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, tb, scls, scls2, rid, rows, np, 0, 3, s));
+    const int64_t nown = c_hi - c_lo;  // own segments only (all of them on one GPU)
+    LV_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, tb, scls + c_lo, scls2, rid + c_lo, rows, nown, 0, 3, s));
     void* tmp = nullptr;
     LV_TRY(dmalloc(&tmp, tb, s));
-    LV_CUDA(cub::DeviceRadixSort::SortPairs(tmp, tb, scls, scls2, rid, rows, np, 0, 3, s));  // kSegClasses classes
+    LV_CUDA(cub::DeviceRadixSort::SortPairs(tmp, tb, scls + c_lo, scls2, rid + c_lo, rows, nown, 0, 3, s));  // kSegClasses classes
     LV_CUB();
     dfree(tmp, s);
   }
@@ -956,16 +1005,61 @@ int32_t level_contract_fast(Handle& h, Level& L, Level& out, int32_t* d_map, int
   int64_t m2 = 0;
   LV_CUDA(cudaMemcpyAsync(&m2, out.rowptr + np, 8, cudaMemcpyDeviceToHost, s));
   LV_CUDA(cudaStreamSynchronize(s));
-  out.nnz = m2;
-  LV_TRY(lvl(LA_COL, 4 * (size_t)std::max<int64_t>(m2, 1), (void**)&out.col));
-  LV_TRY(lvl(LA_W, 4 * (size_t)std::max<int64_t>(m2, 1), (void**)&out.w));
-  if (m2 > 0) {
-    const int64_t* tr = nullptr;
-    LV_TRY(tile_starts(h, out.rowptr, 0, np, 0, m2, kCTile, &tr));
-    k_compact<<<grid_for((m2 + kCTile - 1) / kCTile, 1, 148 * 8), 256, 0, s>>>(sstart, out.rowptr, np, oc, ow, tr,
-                                                                                out.col, out.w);
+  if (cuts.empty()) {
+    out.nnz = m2;
+    LV_TRY(lvl(LA_COL, 4 * (size_t)std::max<int64_t>(m2, 1), (void**)&out.col));
+    LV_TRY(lvl(LA_W, 4 * (size_t)std::max<int64_t>(m2, 1), (void**)&out.w));
+    if (m2 > 0) {
+      const int64_t* tr = nullptr;
+      LV_TRY(tile_starts(h, out.rowptr, 0, np, 0, m2, kCTile, &tr));
+      k_compact<<<grid_for((m2 + kCTile - 1) / kCTile, 1, 148 * 8), 256, 0, s>>>(sstart, out.rowptr, np, oc, ow, tr,
+                                                                                  out.col, out.w);
+      LV_LAUNCHED();
+    }
+  } else {
+    // sharded: this rank's rows [c_lo, c_hi) hold m2 entries (the others' counts are 0 here);
+    // compact them, then all-gather the row lengths and the rows into the replicated CSR'
+    const int world = h.dist->world;
+    int32_t* col_own = nullptr;
+    uint32_t* w_own = nullptr;
+    LV_TRY(dalloc(&col_own, std::max<int64_t>(m2, 1), s));
+    LV_TRY(dalloc(&w_own, std::max<int64_t>(m2, 1), s));
+    if (m2 > 0) {
+      const int64_t* tr = nullptr;
+      LV_TRY(tile_starts(h, out.rowptr, 0, np, 0, m2, kCTile, &tr));
+      k_compact<<<grid_for((m2 + kCTile - 1) / kCTile, 1, 148 * 8), 256, 0, s>>>(sstart, out.rowptr, np, oc, ow, tr,
+                                                                                  col_own, w_own);
+      LV_LAUNCHED();
+    }
+    std::vector<int64_t> nrow(world), drow(world);
+    for (int r = 0; r < world; ++r) {
+      nrow[r] = cuts[r + 1] - cuts[r];
+      drow[r] = cuts[r];
+    }
+    int64_t* cnt_all = nullptr;
+    LV_TRY(dalloc(&cnt_all, np + 1, s));
+    LV_CUDA(cudaMemsetAsync(cnt_all + np, 0, 8, s));
+    LV_TRY(dist_allgatherv(h, cnt + c_lo, cnt_all, nrow, drow, 8));
+    LV_TRY(cub_scan_excl(s, cnt_all, out.rowptr, np + 1));
+    std::vector<int64_t> rp_cut(world + 1);
+    for (int r = 0; r <= world; ++r)
+      LV_CUDA(cudaMemcpyAsync(&rp_cut[r], out.rowptr + cuts[r], 8, cudaMemcpyDeviceToHost, s));
+    LV_CUDA(cudaStreamSynchronize(s));
+    const int64_t total = rp_cut[world];
+    out.nnz = total;
+    LV_TRY(lvl(LA_COL, 4 * (size_t)std::max<int64_t>(total, 1), (void**)&out.col));
+    LV_TRY(lvl(LA_W, 4 * (size_t)std::max<int64_t>(total, 1), (void**)&out.w));
+    std::vector<int64_t> ne(world), de(world);
+    for (int r = 0; r < world; ++r) {
+      ne[r] = rp_cut[r + 1] - rp_cut[r];
+      de[r] = rp_cut[r];
+    }
+    LV_TRY(dist_allgatherv(h, col_own, out.col, ne, de, 4));
+    LV_TRY(dist_allgatherv(h, w_own, out.w, ne, de, 4));
+    dfree(cnt_all, s);
+    dfree(col_own, s);
+    dfree(w_own, s);
   }
-  LV_LAUNCHED();
   LV_CUDA(cudaGetLastError());
   dfree(cnt, s);
   dfree(sstart, s);

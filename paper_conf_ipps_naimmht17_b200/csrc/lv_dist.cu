@@ -17,9 +17,11 @@
 //   * Eq. (1) after a sweep: the delta pass runs over the moved rows the rank owns
 //     and the partial L change is all-reduced (one uint64); S = sum a_c^2 comes
 //     from the replicated a_c;
-//   * contraction (Alg. 3) runs on every rank on the replicated graph
-//     (deterministic, identical), so no graph data crosses the interconnect after
-//     creation.
+//   * contraction (Alg. 3) is sharded by new vertex: the O(n) steps (renumbering,
+//     member grouping) run on every rank, then rank r copies and merges only the
+//     member rows of the new vertices [c_r, c_{r+1}) (balanced by merged-row
+//     length, lv_contract.cu k_seg_split) and the ranks' rows are all-gathered
+//     into the replicated CSR' of the next level.
 // Transports: NCCL (ncclAllGather / ncclAllReduce / grouped ncclBroadcast on the
 // handle's stream; libnccl is loaded at run time, the unique id is bootstrapped by
 // the caller, e.g. torch.distributed) or host callbacks (tests: gloo, or several
@@ -274,6 +276,11 @@ DistCtx::~DistCtx() { delete comm; }
 int32_t dist_allreduce(Handle& h, unsigned long long* dev, size_t count) {
   if (!h.dist) return LOUVAIN_OK;
   return h.dist->comm->allreduce_u64(dev, count, h.stream);
+}
+
+int32_t dist_allgatherv(Handle& h, const void* send, void* recv, const std::vector<int64_t>& cnt,
+                        const std::vector<int64_t>& displ, size_t elem) {
+  return h.dist->comm->allgatherv(send, recv, cnt, displ, elem, h.stream);
 }
 
 static int32_t set_range(Level& L, int64_t lo, int64_t hi) {

@@ -237,6 +237,9 @@ int32_t dist_set_level_range(Handle& h, Level& L, int level);  // own range of t
 int32_t dist_after_binning(Handle& h, Level& L);                // exchange capacities of the level
 int32_t dist_exchange(Handle& h, Level& L, int commit_idx, int group);  // all ranks' moves into the log
 int32_t dist_allreduce(Handle& h, unsigned long long* dev, size_t count);  // in-place sum (no-op on 1 GPU)
+// recv[displ[r] .. + cnt[r]) <- rank r's send (units of elem bytes; device buffers, handle's stream)
+int32_t dist_allgatherv(Handle& h, const void* send, void* recv, const std::vector<int64_t>& cnt,
+                        const std::vector<int64_t>& displ, size_t elem);
 void dist_free(Handle& h);
 
 // ------------------------------------------------------------------ launch accounting
