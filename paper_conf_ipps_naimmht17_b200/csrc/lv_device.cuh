@@ -53,16 +53,37 @@ __device__ __forceinline__ uint32_t part_of(int32_t c, uint32_t P) {
   return (uint32_t)(((unsigned long long)h * P) >> 32);
 }
 
+// Whole-warp version with the warp reduction unit (REDUX): max of the high word
+// (signed), max of the low word among those lanes (unsigned) -- together the
+// int64 max -- then the lowest label among the lanes holding it, and the
+// sum.  3 + 1 single-instruction reductions instead of a 5-step butterfly of
+// 64-bit shuffles and compares.  Every lane gets the result.
+__device__ __forceinline__ void warp_reduce(long long& s, int& c, unsigned& eown) {
+  const int hi = (int)((unsigned long long)s >> 32);
+  const unsigned lo = (unsigned)(unsigned long long)s;
+  const int mhi = __reduce_max_sync(kFull, hi);
+  const unsigned mlo = __reduce_max_sync(kFull, hi == mhi ? lo : 0u);
+  const long long ms = (long long)(((unsigned long long)(unsigned)mhi << 32) | mlo);
+  const int mc = __reduce_min_sync(kFull, s == ms ? c : 0x7FFFFFFF);
+  eown = __reduce_add_sync(kFull, eown);
+  s = ms;
+  c = mc;
+}
+
 // xor-butterfly reduction over aligned groups of G lanes: best candidate + sum.
 template <int G>
 __device__ __forceinline__ void group_reduce(long long& s, int& c, unsigned& eown) {
+  if constexpr (G == 32) {
+    warp_reduce(s, c, eown);
+  } else {
 #pragma unroll
-  for (int off = G / 2; off >= 1; off >>= 1) {
-    long long s2 = __shfl_xor_sync(kFull, s, off);
-    int c2 = __shfl_xor_sync(kFull, c, off);
-    unsigned e2 = __shfl_xor_sync(kFull, eown, off);
-    if (better(s2, c2, s, c)) { s = s2; c = c2; }
-    eown += e2;
+    for (int off = G / 2; off >= 1; off >>= 1) {
+      long long s2 = __shfl_xor_sync(kFull, s, off);
+      int c2 = __shfl_xor_sync(kFull, c, off);
+      unsigned e2 = __shfl_xor_sync(kFull, eown, off);
+      if (better(s2, c2, s, c)) { s = s2; c = c2; }
+      eown += e2;
+    }
   }
 }
 

@@ -55,6 +55,15 @@ constexpr int kCapT[5] = {2048, 4096, 8192, 16384, 18432};  // max smem table sl
 constexpr int kThrT[5] = {128, 256, 512, 512, 1024};
 constexpr int kPerSmT[5] = {16, 8, 4, 2, 1};
 constexpr int kCapMax = 18432;
+// Buckets whose degree bound is <= kSmallMaxDeg (1-4 with the paper's bounds) run the
+// register kernels; their sub-class is 1 + ceil(log2 deg) (1..6): lane groups of 1,
+// 2, 4, ..., 32 lanes per vertex.
+constexpr int64_t kSmallMaxDeg = 32;
+__host__ __device__ inline int small_sub_of_degree(int64_t d) {
+  int s = 1;
+  while (s < 6 && (int64_t(1) << (s - 1)) < d) ++s;
+  return s;
+}
 __host__ __device__ inline int sub_of_degree(int64_t d) {
   return d < kSub1Min ? 0 : d < kSub2Min ? 1 : d < kSub3Min ? 2 : d < kSub4Min ? 3 : d < kSub5Min ? 4
        : d < kSub6Min ? 5 : d < kHubMin ? 6 : 7;
@@ -175,6 +184,7 @@ struct Level {
   // binning (valid for bins_bounds)
   bool bins_valid = false;
   int64_t bins_bounds[6] = {0, 0, 0, 0, 0, 0};
+  int64_t bins_bounds_pending[6] = {0, 0, 0, 0, 0, 0};  // bounds of the binning being built (plans)
   int32_t* bin_vertices = nullptr;
   int64_t class_off[kNumClasses + 1] = {0};
   int64_t class_soff[kNumClasses + 1] = {0};  // soff[class_off[c]] (host copy)

@@ -108,7 +108,10 @@ __global__ void k_classify(const int64_t* rowptr, int64_t n, int64_t b0, int64_t
     else if (d <= b4) b = 5;
     else if (d <= b5) b = 6;
     else b = 7;
-    const int sub = sub_of_degree(d);
+    // buckets whose bound is <= 32 (the register kernels): sub-class by the power of two
+    // of the degree, so each vertex gets a lane group of its own size (deg 1: one lane)
+    const int64_t bound = b == 1 ? b0 : b == 2 ? b1 : b == 3 ? b2 : b == 4 ? b3 : b == 5 ? b4 : b == 6 ? b5 : INT64_MAX;
+    const int sub = (b >= 1 && bound <= kSmallMaxDeg) ? small_sub_of_degree(d) : sub_of_degree(d);
     const uint8_t c = (uint8_t)(kSubPerBucket * b + sub);
     if (has) {
       cls[i] = c;
@@ -694,6 +697,7 @@ static int32_t build_hub_plan(Handle& h, Level& L) {
   std::vector<int64_t> hdeg, rb, hsoff;
   std::vector<int32_t> hbucket;
   for (int b = 1; b <= 7; ++b) {
+    if (b <= 6 && L.bins_bounds_pending[b - 1] <= kSmallMaxDeg) continue;  // register-kernel bucket: no hubs
     const int c = kSubPerBucket * b + kSubPart;  // partitioned sub-classes (P > part_maxp() only)
     const int64_t off = L.class_off[c], cnt = L.class_off[kSubPerBucket * (b + 1)] - off;
     if (cnt <= 0) continue;
@@ -808,6 +812,7 @@ int32_t build_part_plan(Handle& h, Level& L) {
     Q.bucket_chunk[b - 1] = (int64_t)ch.size();
     Q.bucket_vsplit[b - 1] = (int64_t)vpos.size();
     Q.bucket_tsplit[b - 1] = (int64_t)tv.size();
+    if (b <= 6 && L.bins_bounds_pending[b - 1] <= kSmallMaxDeg) continue;  // register-kernel bucket: no hubs
     const int c0 = kSubPerBucket * b + kSubPart, c1 = kSubPerBucket * (b + 1);
     const int64_t off = L.class_off[c0], cnt = L.class_off[c1] - off;
     if (cnt <= 0) continue;
@@ -876,6 +881,7 @@ int32_t level_binning(Handle& h, Level& L, const louvain_params_t& p) {
   if (same) return LOUVAIN_OK;
   cudaStream_t s = h.stream;
   const int64_t n = L.n;
+  std::memcpy(L.bins_bounds_pending, p.deg_bounds, sizeof L.bins_bounds_pending);
   hub_free(L.hub, s);
   std::fill(L.class_off, L.class_off + kNumClasses + 1, 0);
   if (n > 0) {

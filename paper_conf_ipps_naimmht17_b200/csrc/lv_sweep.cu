@@ -1472,6 +1472,33 @@ int32_t launch_sweep_bucket(Handle& h, Level& L, const louvain_params_t& p, int 
   A.mv_new = L.mv_new;
   A.logn = &h.ctl->logn;
   const int64_t hi = (bucket <= 6) ? p.deg_bounds[bucket - 1] : INT64_MAX;
+  if (hi <= kSmallMaxDeg) {  // register kernels only: lane groups of 1..32 lanes, by degree (k_classify)
+    cudaStream_t s = h.stream;
+    for (int sub = 1; sub <= 6; ++sub) {
+      const int64_t off = L.class_off[kSubPerBucket * bucket + sub];
+      const int64_t nv = L.class_off[kSubPerBucket * bucket + sub + 1] - off;
+      if (nv <= 0) continue;
+      const int32_t* verts = L.bin_vertices + off;
+      const int G = 1 << (sub - 1);
+      const unsigned grid = grid_for(nv, 8 * (32 / G), 148 * 8);
+#define LV_SMALL(GG)                                                              \
+  if (L.w) sweep_small<GG, false><<<grid, 256, 0, s>>>(verts, nv, A);              \
+  else sweep_small<GG, true><<<grid, 256, 0, s>>>(verts, nv, A)
+      switch (G) {
+        case 1: LV_SMALL(1); break;
+        case 2: LV_SMALL(2); break;
+        case 4: LV_SMALL(4); break;
+        case 8: LV_SMALL(8); break;
+        case 16: LV_SMALL(16); break;
+        default: LV_SMALL(32); break;
+      }
+#undef LV_SMALL
+      LV_LAUNCHED();
+      if (trace_on()) trace_step(h, L, bucket, sub, off, off + nv);
+    }
+    LV_CUDA(cudaGetLastError());
+    return LOUVAIN_OK;
+  }
   auto dispatch = [&](int sub) -> int32_t {
     const int64_t max_deg = (sub == 0) ? std::min<int64_t>(hi, kSub1Min - 1) : hi;
     // warp-level label merging (__match_any_sync before the table insert) is
