@@ -440,6 +440,180 @@ __device__ __forceinline__ void insert_staged(unsigned long long* T, uint32_t* T
   }
 }
 
+// ------------------------------------------------------------ register claim lists
+// The thread whose CAS claims an empty slot (the first entry of label c in the
+// row) keeps that slot's index in a register.  After the inserts the claimers --
+// together exactly the distinct labels of the row -- evaluate Eq. (2) for their
+// labels and clear their slots: no scan of the 2*deg-slot table (the scan was half
+// of the CTA tiers' instructions, ncu profiles/r02_sass_lines_cta.txt).
+// Covers rows of up to 4 * PASSES * stride entries.
+constexpr uint32_t kNoClaim = 0xFFFFFFFFu;
+
+__device__ __forceinline__ uint32_t table_insert_c(unsigned long long* T, uint32_t cap, int32_t c, uint32_t x,
+                                                   bool* claimed) {
+  const unsigned long long key = ((unsigned long long)(uint32_t)c) << 32;
+  uint32_t h = hash_slot(c, cap);
+  for (;;) {
+    const unsigned long long old = atomicCAS(&T[h], kEmpty, key | x);
+    if (old == kEmpty) {
+      *claimed = true;
+      return h;
+    }
+    if ((old >> 32) == (unsigned long long)(uint32_t)c) {
+      atomicAdd(&T[h], (unsigned long long)x);
+      *claimed = false;
+      return h;
+    }
+    h = (h + 1 == cap) ? 0 : h + 1;
+  }
+}
+
+template <bool UNIT, int PASSES>
+__device__ __forceinline__ void insert_claim(unsigned long long* T, uint32_t* TA, uint32_t cap,
+                                             const uint2* __restrict__ S, const uint32_t* __restrict__ Wt,
+                                             int64_t deg, int t0, int stride, uint32_t (&cl)[4 * PASSES]) {
+#pragma unroll
+  for (int pass = 0; pass < PASSES; ++pass) {
+    uint2 rr[4];
+    uint32_t ww[4];
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      const int64_t t = (int64_t)t0 + (int64_t)(4 * pass + q) * stride;
+      rr[q] = (t < deg) ? __ldcs(&S[t]) : make_uint2(kSelf, 0u);
+      ww[q] = UNIT ? 1u : ((t < deg) ? __ldcs(&Wt[t]) : 0u);
+    }
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      uint32_t slot = kNoClaim;
+      if (rr[q].x != kSelf) {
+        bool claimed = false;
+        const uint32_t hq = table_insert_c(T, cap, (int32_t)rr[q].x, ww[q], &claimed);
+        if (rr[q].y != kUnknownA) TA[hq] = rr[q].y;
+        if (claimed) slot = hq;
+      }
+      cl[4 * pass + q] = slot;
+    }
+  }
+}
+
+// Eq. (2) for the claimed labels, 4 at a time (a_c gathers of labels without a
+// representative in the row in flight together); clears the claimed slots.
+template <int PASSES>
+__device__ __forceinline__ void eval_claims(unsigned long long* T, uint32_t* TA, const uint32_t (&cl)[4 * PASSES],
+                                            int32_t own, bool own_single, uint32_t ki, const SweepArgs& A,
+                                            long long& s, int& cb, unsigned& eown) {
+#pragma unroll
+  for (int pass = 0; pass < PASSES; ++pass) {
+    unsigned long long x[4];
+    uint32_t ac[4];
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      const uint32_t sl = cl[4 * pass + q];
+      x[q] = kEmpty;
+      ac[q] = kUnknownA;
+      if (sl != kNoClaim) {
+        x[q] = T[sl];
+        ac[q] = TA[sl];
+        T[sl] = kEmpty;
+        TA[sl] = kUnknownA;
+      }
+    }
+#pragma unroll
+    for (int q = 0; q < 4; ++q)
+      if (x[q] != kEmpty && ac[q] == kUnknownA && (int32_t)(x[q] >> 32) != own)
+        ac[q] = __ldg(&A.ca[(int32_t)(x[q] >> 32)]).y;
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      if (x[q] == kEmpty) continue;
+      const int32_t c = (int32_t)(x[q] >> 32);
+      const uint32_t e = (uint32_t)x[q];
+      if (c == own) eown = e;
+      else consider(c, e, ac[q], own, own_single, ki, A, s, cb);
+    }
+  }
+}
+
+// Warp per vertex with register claims (rows of <= 128 * PASSES entries).
+template <int CAP, int WARPS, bool UNIT, int PASSES>
+__global__ void __launch_bounds__(32 * WARPS) sweep_warp_c(const int32_t* __restrict__ verts,
+                                                           const int64_t* __restrict__ soff, int64_t nv,
+                                                           const uint2* __restrict__ stage, SweepArgs A) {
+  __shared__ unsigned long long tab[WARPS][CAP];
+  __shared__ uint32_t taba[WARPS][CAP];
+  const int lane = threadIdx.x & 31, wl = threadIdx.x >> 5;
+  unsigned long long* T = tab[wl];
+  uint32_t* TA = taba[wl];
+  for (int t = lane; t < CAP; t += 32) {
+    T[t] = kEmpty;
+    TA[t] = kUnknownA;
+  }
+  __syncwarp();
+  const int64_t warps = (int64_t)gridDim.x * WARPS;
+  for (int64_t vi = (int64_t)blockIdx.x * WARPS + wl; vi < nv; vi += warps) {
+    const int32_t v = __ldg(&verts[vi]);
+    const int64_t rb = __ldg(&A.rowptr[v]);
+    const int64_t deg = __ldg(&A.rowptr[v + 1]) - rb;
+    const int32_t own = (int32_t)__ldg(&A.ca[v]).x;
+    const uint32_t ki = __ldg(&A.k[v]);
+    uint32_t cl[4 * PASSES];
+    insert_claim<UNIT, PASSES>(T, TA, CAP, stage + __ldg(&soff[vi]), UNIT ? nullptr : A.w + rb, deg, lane, 32, cl);
+    __syncwarp();
+    const bool own_single = A.rule == 2 && __ldg(&A.size[own]) == 1;
+    long long s = (long long)0x8000000000000000ull;
+    int cb = 0x7FFFFFFF;
+    unsigned eown = 0;
+    eval_claims<PASSES>(T, TA, cl, own, own_single, ki, A, s, cb, eown);
+    group_reduce<32>(s, cb, eown);
+    int32_t tgt = own;
+    if (lane == 0) tgt = finish(s, cb, eown, own, __ldg(&A.ca[own]).y, ki, A);
+    log_moves(lane == 0 && tgt != own, v, tgt, A);
+    __syncwarp();
+  }
+}
+
+// CTA per vertex with register claims (rows of <= 4 * PASSES * blockDim entries).
+template <bool UNIT, int PASSES>
+__global__ void __launch_bounds__(1024) sweep_cta_c(const int32_t* __restrict__ verts,
+                                                    const int64_t* __restrict__ soff, int64_t nv,
+                                                    const uint2* __restrict__ stage, SweepArgs A, int capmax) {
+  extern __shared__ unsigned long long smem[];
+  unsigned long long* T = smem;
+  uint32_t* TA = reinterpret_cast<uint32_t*>(smem + capmax);
+  __shared__ long long sh_s[32];
+  __shared__ int sh_c[32];
+  __shared__ unsigned sh_e[32];
+  for (int t = threadIdx.x; t < capmax; t += blockDim.x) {
+    T[t] = kEmpty;
+    TA[t] = kUnknownA;
+  }
+  __syncthreads();
+  for (int64_t vi = blockIdx.x; vi < nv; vi += gridDim.x) {
+    const int32_t v = __ldg(&verts[vi]);
+    const int64_t rb = __ldg(&A.rowptr[v]);
+    const int64_t deg = __ldg(&A.rowptr[v + 1]) - rb;
+    const int32_t own = (int32_t)__ldg(&A.ca[v]).x;
+    const uint32_t ki = __ldg(&A.k[v]);
+    const int64_t want = 2 * deg + 1;  // load <= 1/2
+    const uint32_t cap = (uint32_t)(want < (int64_t)capmax ? want : (int64_t)capmax);
+    uint32_t cl[4 * PASSES];
+    insert_claim<UNIT, PASSES>(T, TA, cap, stage + __ldg(&soff[vi]), UNIT ? nullptr : A.w + rb, deg, threadIdx.x,
+                               blockDim.x, cl);
+    __syncthreads();
+    const bool own_single = A.rule == 2 && __ldg(&A.size[own]) == 1;
+    long long s = (long long)0x8000000000000000ull;
+    int cb = 0x7FFFFFFF;
+    unsigned eown = 0;
+    eval_claims<PASSES>(T, TA, cl, own, own_single, ki, A, s, cb, eown);
+    block_reduce(s, cb, eown, sh_s, sh_c, sh_e);
+    if (threadIdx.x < 32) {
+      int32_t tgt = own;
+      if (threadIdx.x == 0) tgt = finish(s, cb, eown, own, __ldg(&A.ca[own]).y, ki, A);
+      log_moves(threadIdx.x == 0 && tgt != own, v, tgt, A);
+    }
+    __syncthreads();
+  }
+}
+
 // ------------------------------------------------------------ warp per vertex
 template <int CAP, int WARPS, bool UNIT, bool AGG>
 __global__ void __launch_bounds__(32 * WARPS) sweep_warp(const int32_t* __restrict__ verts,
@@ -1353,6 +1527,11 @@ int32_t launch_part(Handle& h, Level& L, const SweepArgs& A, int bucket, bool un
 // the fixed 512-slot warp tables of bucket 6 (C5 level 0: 10.2 -> 6.3 ms per 2
 // sweeps).  The CTA tables are sized 2*deg, where the list measured slower
 // (b7 [1024,2048): 12.5 -> 19.4 ms), and so was the 128-slot warp table of bucket 5.
+// register claim lists instead of table scans in the warp / CTA kernels (LV_CLAIM=0: scans; A/B)
+static bool claim_on() {
+  static const bool on = !(getenv("LV_CLAIM") && getenv("LV_CLAIM")[0] == '0');
+  return on;
+}
 // largest degree of CTA tier `sub` (lv_internal.cuh)
 static int64_t max_deg_of_tier(int sub) {
   static const int64_t ub[5] = {kSub1Min - 1, kSub2Min - 1, kSub3Min - 1, kSub4Min - 1, kSub5Min - 1};
@@ -1377,6 +1556,12 @@ int32_t dispatch_class(Handle& h, Level& L, const SweepArgs& A, int bucket, int 
       case 16: sweep_small<16, UNIT><<<grid, 256, 0, s>>>(verts, nv, A); break;
       default: sweep_small<32, UNIT><<<grid, 256, 0, s>>>(verts, nv, A); break;
     }
+    LV_LAUNCHED();
+  } else if (sub == 0 && max_deg > 84 && max_deg <= 340 && claim_on()) {
+    sweep_warp_c<512, 4, UNIT, 3><<<grid_for(nv, 4, 148 * 8), 128, 0, s>>>(verts, soff, nv, stage, A);
+    LV_LAUNCHED();
+  } else if (sub == 0 && max_deg <= 84 && claim_on()) {
+    sweep_warp_c<128, 8, UNIT, 1><<<grid_for(nv, 8, 148 * 8), 256, 0, s>>>(verts, soff, nv, stage, A);
     LV_LAUNCHED();
   } else if (sub == 0 && max_deg > 84 && max_deg <= 340) {
     sweep_warp_l<512, 352, 4, UNIT><<<grid_for(nv, 4, 148 * 8), 128, 0, s>>>(verts, soff, nv, stage, A);
@@ -1403,7 +1588,39 @@ int32_t dispatch_class(Handle& h, Level& L, const SweepArgs& A, int bucket, int 
     }
     constexpr int fnum = 8;  // table of 2*deg slots (1.5x / 1.75x / 2.5x / 3x measured slower)
     static int resident[5] = {0, 0, 0, 0, 0};
-    const int64_t md = max_deg_of_tier(sub);
+    const int64_t md = std::min<int64_t>(max_deg_of_tier(sub), max_deg);
+    if (claim_on()) {
+      static bool cattr = false;
+      if (!cattr) {
+        LV_TRY(set_smem(sweep_cta_c<true, 1>, 12 * (size_t)kCapMax));
+        LV_TRY(set_smem(sweep_cta_c<false, 1>, 12 * (size_t)kCapMax));
+        LV_TRY(set_smem(sweep_cta_c<true, 2>, 12 * (size_t)kCapMax));
+        LV_TRY(set_smem(sweep_cta_c<false, 2>, 12 * (size_t)kCapMax));
+        LV_TRY(set_smem(sweep_cta_c<true, 3>, 12 * (size_t)kCapMax));
+        LV_TRY(set_smem(sweep_cta_c<false, 3>, 12 * (size_t)kCapMax));
+        cattr = true;
+      }
+      const int passes = (int)((md + 4 * threads[sub] - 1) / (4 * threads[sub]));
+      const int capt = (int)std::min<int64_t>(caps[sub], ((2 * md + 1 + 31) / 32) * 32);
+      static int cres[5][4] = {{0}};
+      auto go = [&](auto kern) -> int32_t {
+        if (cres[sub][passes] == 0) {
+          int nb = 0;
+          LV_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, kern, threads[sub], 12 * (size_t)capt));
+          cres[sub][passes] = std::max(nb, 1);
+        }
+        kern<<<grid_for(nv, 1, 148 * cres[sub][passes]), threads[sub], 12 * (size_t)capt, s>>>(verts, soff, nv,
+                                                                                             stage, A, capt);
+        LV_LAUNCHED();
+        LV_CUDA(cudaGetLastError());
+        return LOUVAIN_OK;
+      };
+      if (passes <= 1) return go(sweep_cta_c<UNIT, 1>);
+      if (passes == 2) return go(sweep_cta_c<UNIT, 2>);
+      if (passes == 3) return go(sweep_cta_c<UNIT, 3>);
+      set_error("sweep: CTA tier degree beyond the claim-list capacity");
+      return LOUVAIN_E_UNSUPPORTED;
+    }
     const int capt = (int)std::min<int64_t>(caps[sub], ((md + ((md * fnum) >> 3) + 1 + 31) / 32) * 32);
     if (resident[sub] == 0) {
       int nb = 0;
