@@ -126,6 +126,7 @@ __global__ void k_dest_base(const int32_t* __restrict__ vorder, const int64_t* _
 
 constexpr int kSTile = 4096;  // CSR entries per scatter-copy tile
 constexpr int kSRows = 1024;  // rows staged per tile (else per-entry search in global memory)
+template <bool RANGE>  // RANGE: sharded contraction, only rows whose new vertex is in [c_lo, c_hi)
 __global__ void __launch_bounds__(256) k_scatter_copy(const int64_t* __restrict__ rowptr, int64_t n,
                                                       const int32_t* __restrict__ col,
                                                       const uint32_t* __restrict__ w,
@@ -135,7 +136,7 @@ __global__ void __launch_bounds__(256) k_scatter_copy(const int64_t* __restrict_
                                                       int32_t c_lo, int32_t c_hi) {
   __shared__ int64_t sh_rp[kSRows + 1];
   __shared__ int64_t sh_db[kSRows];
-  __shared__ int32_t sh_mine[kSRows];  // the row's new vertex is in this rank's range [c_lo, c_hi)
+  __shared__ int32_t sh_mine[RANGE ? kSRows : 1];  // the row's new vertex is in this rank's range
   __shared__ int64_t sh_u0;
   __shared__ int sh_nr;
   const int64_t ntiles = (nnz + kSTile - 1) / kSTile;
@@ -152,7 +153,7 @@ __global__ void __launch_bounds__(256) k_scatter_copy(const int64_t* __restrict_
     for (int r = threadIdx.x; r < nr; r += blockDim.x) {
       sh_rp[r] = rowptr[u0 + r];
       sh_db[r] = dbase[u0 + r];
-      if (u0 + r < n) {
+      if (RANGE && u0 + r < n) {
         const int32_t c = map[u0 + r];
         sh_mine[r] = c >= c_lo && c < c_hi;
       }
@@ -174,7 +175,7 @@ __global__ void __launch_bounds__(256) k_scatter_copy(const int64_t* __restrict_
               if (sh_rp[mid] <= e) lo = mid; else hi = mid - 1;
             }
             dd[q] = sh_db[lo] + (e - sh_rp[lo]);
-            if (!sh_mine[lo]) continue;  // another rank merges this row's community
+            if (RANGE && !sh_mine[lo]) continue;  // another rank merges this row's community
           } else {
             int64_t lo = 0, hi = n - 1;
             while (lo < hi) {
@@ -182,8 +183,10 @@ __global__ void __launch_bounds__(256) k_scatter_copy(const int64_t* __restrict_
               if (rowptr[mid] <= e) lo = mid; else hi = mid - 1;
             }
             dd[q] = dbase[lo] + (e - rowptr[lo]);
-            const int32_t c = map[lo];
-            if (c < c_lo || c >= c_hi) continue;
+            if (RANGE) {
+              const int32_t c = map[lo];
+              if (c < c_lo || c >= c_hi) continue;
+            }
           }
           jj[q] = __ldcs(&col[e]);
         }
@@ -743,9 +746,12 @@ int32_t level_contract_fast(Handle& h, Level& L, Level& out, int32_t* d_map, int
     LV_LAUNCHED();
     const int64_t* tr = nullptr;
     LV_TRY(tile_starts(h, L.rowptr, 0, n, 0, nnz, kSTile, &tr));
-    k_scatter_copy<<<grid_for((nnz + kSTile - 1) / kSTile, 1, 148 * 8), 256, 0, s>>>(L.rowptr, n, L.col, L.w, d_map,
-                                                                                       dbase, nnz, tr, gc, gw,
-                                                                                       (int32_t)c_lo, (int32_t)c_hi);
+    const unsigned g = grid_for((nnz + kSTile - 1) / kSTile, 1, 148 * 8);
+    if (cuts.empty())
+      k_scatter_copy<false><<<g, 256, 0, s>>>(L.rowptr, n, L.col, L.w, d_map, dbase, nnz, tr, gc, gw, 0, 0);
+    else
+      k_scatter_copy<true><<<g, 256, 0, s>>>(L.rowptr, n, L.col, L.w, d_map, dbase, nnz, tr, gc, gw, (int32_t)c_lo,
+                                             (int32_t)c_hi);
     LV_LAUNCHED();
     dfree(dbase, s);
   }

@@ -242,6 +242,53 @@ def test_edge_cases():
     assert lab.tolist() == r.labels.tolist() and (int(q.L), q.S) == (r.L, r.S)
 
 
+def test_degree_zero_vertices_inside_a_graph():
+    """R11: a vertex of degree 0 is in no bucket and never moves, also when W > 0 and the
+    degree-0 vertices sit between and around connected ones (no compaction, R21 off)."""
+    rng = np.random.default_rng(7)
+    n = 3000
+    u = rng.integers(0, n, size=9000)
+    v = (u + rng.integers(1, 30, size=9000)) % n
+    keep = (u % 7 != 3) & (v % 7 != 3)  # every 7th vertex (offset 3) isolated
+    g = graphgen.from_edges(n, u[keep], v[keep], compact=False)
+    iso = np.flatnonzero(np.diff(g.rowptr) == 0)
+    assert len(iso) >= n // 7 and 0 < g.nnz
+    st = oracle.State(g)
+    gd = dev_graph(g)
+    for _ in range(2):
+        assert gd.sweep(lvb.params())[0] == st.sweep(oracle.params())
+        assert_state_equal(gd, st)
+    r = oracle.louvain(g)
+    lab, q, stt = dev_graph(g).run(lvb.params())
+    assert np.array_equal(lab, r.labels) and (int(q.L), q.S) == (r.L, r.S)
+    assert stt["sweeps_per_level"] == r.sweeps_per_level
+    # isolated vertices end as singleton communities of their own (labels distinct)
+    assert len(set(r.labels[iso].tolist())) == len(iso)
+
+
+def test_weights_near_the_W_guard():
+    """R4: scores s = W*e - k*a in int64 need W <= 3,037,000,499; e, k, a in uint32.  A graph
+    with W just below the guard runs bit-exactly; one with W just above is refused
+    (LOUVAIN_E_OVERFLOW) before any device work."""
+    guard = 3037000499
+    # path of 6 vertices + a heavy edge: W = 2 * (heavy + 4) + 2 * loop
+    heavy = (guard - 10) // 2
+    g = graphgen.weighted_csr(6, [0, 1, 2, 3, 4, 5], [1, 2, 3, 4, 5, 5], [heavy, 1, 1, 1, 1, 1])
+    W = int(g.weights().sum())
+    assert W <= guard and W > guard - 20
+    r = oracle.louvain(g)
+    lab, q, st = dev_graph(g).run(lvb.params())
+    assert np.array_equal(lab, r.labels) and (int(q.L), q.S, int(q.W)) == (r.L, r.S, r.W)
+    st_o = oracle.State(g)
+    gd = dev_graph(g)
+    assert gd.sweep(lvb.params())[0] == st_o.sweep(oracle.params())
+    assert_state_equal(gd, st_o)
+    g2 = graphgen.weighted_csr(6, [0, 1, 2, 3, 4, 5], [1, 2, 3, 4, 5, 5], [heavy + 20, 1, 1, 1, 1, 1])
+    with pytest.raises(lvb.LouvainError) as ei:
+        dev_graph(g2)
+    assert ei.value.code == lvb.E_OVERFLOW
+
+
 def test_device_inputs_and_borrow():
     torch = pytest.importorskip("torch")
     g = GRAPHS["rmat15"]()
