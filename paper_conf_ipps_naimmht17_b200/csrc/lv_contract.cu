@@ -318,13 +318,24 @@ __global__ void __launch_bounds__(512) k_merge_mid(const int32_t* __restrict__ r
       }
     }
     __syncthreads();
-    for (uint32_t t = threadIdx.x; t < cap; t += blockDim.x) {
-      const unsigned long long x = T[t];
-      if (x == kEmpty) continue;
-      T[t] = kEmpty;
-      const unsigned pos = atomicAdd(&ncnt, 1u);
-      oc[b + pos] = (int32_t)(x >> 32);
-      ow[b + pos] = (uint32_t)x;
+    // distinct keys appended with one shared atomic per warp and pass (not per key:
+    // a single counter serialised every key of the CTA)
+    const int lane = threadIdx.x & 31;
+    for (uint32_t t0 = threadIdx.x - lane; t0 < cap; t0 += blockDim.x) {
+      const uint32_t t = t0 + lane;
+      const unsigned long long x = t < cap ? T[t] : kEmpty;
+      const bool has = x != kEmpty;
+      const unsigned m = __ballot_sync(kFull, has);
+      if (!m) continue;
+      unsigned base = 0;
+      if (lane == 0) base = atomicAdd(&ncnt, (unsigned)__popc(m));
+      base = __shfl_sync(kFull, base, 0);
+      if (has) {
+        T[t] = kEmpty;
+        const unsigned pos = base + __popc(m & ((1u << lane) - 1u));
+        oc[b + pos] = (int32_t)(x >> 32);
+        ow[b + pos] = (uint32_t)x;
+      }
     }
     __syncthreads();
     if (threadIdx.x == 0) {
