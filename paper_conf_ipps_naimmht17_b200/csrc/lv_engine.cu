@@ -266,9 +266,7 @@ int32_t init_handle(Handle& h, void* stream) {
   LV_CUDA(cudaStreamCreateWithFlags(&h.side, cudaStreamNonBlocking));
   LV_CUDA(cudaEventCreateWithFlags(&h.ev_fork, cudaEventDisableTiming));
   LV_CUDA(cudaEventCreateWithFlags(&h.ev_join, cudaEventDisableTiming));
-  LV_CUDA(cudaStreamCreateWithFlags(&h.tabs, cudaStreamNonBlocking));
-  for (auto& ev : h.ev_chunk) LV_CUDA(cudaEventCreateWithFlags(&ev, cudaEventDisableTiming));
-  LV_CUDA(cudaEventCreateWithFlags(&h.ev_join2, cudaEventDisableTiming));
+
   return LOUVAIN_OK;
 }
 
@@ -290,13 +288,7 @@ void destroy_handle(Handle& h) {
   }
   if (h.ev_fork) cudaEventDestroy(h.ev_fork);
   if (h.ev_join) cudaEventDestroy(h.ev_join);
-  if (h.tabs) {
-    cudaStreamSynchronize(h.tabs);
-    cudaStreamDestroy(h.tabs);
-  }
-  for (auto& ev : h.ev_chunk)
-    if (ev) cudaEventDestroy(ev);
-  if (h.ev_join2) cudaEventDestroy(h.ev_join2);
+
   if (h.own_stream && h.stream) cudaStreamDestroy(h.stream);
 }
 

@@ -188,11 +188,6 @@ struct Level {
   int32_t* bin_vertices = nullptr;
   int64_t class_off[kNumClasses + 1] = {0};
   int64_t class_soff[kNumClasses + 1] = {0};  // soff[class_off[c]] (host copy)
-  // every class cut into kChunks position ranges of ~equal staged entries (stage/table
-  // pipeline): chunk_pos[c][0..kChunks] positions, chunk_soff[c][..] their soff values
-  static constexpr int kChunks = 4;
-  int64_t chunk_pos[kNumClasses][kChunks + 1] = {{0}};
-  int64_t chunk_soff[kNumClasses][kChunks + 1] = {{0}};
   // gather staging (two-phase sweep): soff[i] = sum of degrees of bin_vertices[0..i),
   // stage[soff[i] + t] = {label, a_c or 0xFFFFFFFF} of the t-th neighbour of bin_vertices[i]
   int64_t* soff = nullptr;
@@ -228,13 +223,6 @@ struct Handle {
   // side stream for independent kernels inside one phase (fork/join through events)
   cudaStream_t side = nullptr;
   cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
-  // stage / table pipeline of a bucket: chunk k is staged on the main stream
-  // (memory-bound gathers) while the table kernels of chunk k-1 run on `tabs`
-  // (issue-bound shared-memory hashing); ev_chunk[k] orders table k after stage k
-  cudaStream_t tabs = nullptr;
-  static constexpr int kChunkEvents = 48;
-  cudaEvent_t ev_chunk[kChunkEvents] = {nullptr};
-  cudaEvent_t ev_join2 = nullptr;
   // louvain_run only: {label at the sweep start, label after} per vertex; the
   // commit writes .y of every moved vertex (delta pass of Eq. (1))
   uint2* pcn = nullptr;
@@ -334,7 +322,7 @@ int32_t validate_csr_host(int64_t n, int64_t nnz, const int64_t* rowptr, const i
 // ------------------------------------------------------------------ sweep (lv_sweep.cu)
 int32_t launch_sweep_bucket(Handle& h, Level& L, const louvain_params_t& p, int bucket);
 // phase 1 gather for bin positions [pos0,pos1), staged entries [s0,s1)
-int32_t launch_stage(Handle& h, Level& L, int64_t pos0, int64_t pos1, int64_t s0, int64_t s1, int per_sm);
+int32_t launch_stage(Handle& h, Level& L, int64_t pos0, int64_t pos1, int64_t s0, int64_t s1);
 int32_t build_part_plan(Handle& h, Level& L);
 
 // ------------------------------------------------------------------ launch geometry

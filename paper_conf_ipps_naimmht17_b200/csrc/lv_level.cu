@@ -875,31 +875,6 @@ int32_t build_part_plan(Handle& h, Level& L) {
   return LOUVAIN_OK;
 }
 
-struct ClassBounds {
-  int64_t off[kNumClasses + 1];
-};
-// Chunk k of class c (k = 0..chunks): the first bin position whose staged-entry
-// offset reaches soff[start] + k/chunks of the class's entries, and that offset.
-__global__ void k_chunk_cuts(const int64_t* __restrict__ soff, ClassBounds cb, int chunks, int64_t* out) {
-  const int c = blockIdx.x, k = threadIdx.x;
-  if (k > chunks) return;
-  const int64_t p0 = cb.off[c], p1 = cb.off[c + 1];
-  int64_t pos = p0;
-  if (k == chunks) {
-    pos = p1;
-  } else if (k > 0 && p1 > p0) {
-    const int64_t s0 = soff[p0], target = s0 + (int64_t)((__int128)(soff[p1] - s0) * k / chunks);
-    int64_t lo = p0, hi = p1;
-    while (lo < hi) {
-      const int64_t mid = (lo + hi) >> 1;
-      if (soff[mid] < target) lo = mid + 1; else hi = mid;
-    }
-    pos = lo;
-  }
-  out[((int64_t)c * (chunks + 1) + k) * 2] = pos;
-  out[((int64_t)c * (chunks + 1) + k) * 2 + 1] = soff[pos];
-}
-
 int32_t level_binning(Handle& h, Level& L, const louvain_params_t& p) {
   bool same = L.bins_valid;
   for (int t = 0; t < 6 && same; ++t) same = (L.bins_bounds[t] == p.deg_bounds[t]);
@@ -958,25 +933,6 @@ int32_t level_binning(Handle& h, Level& L, const louvain_params_t& p) {
     for (int c = 0; c <= kNumClasses; ++c)
       LV_CUDA(cudaMemcpyAsync(&L.class_soff[c], L.soff + L.class_off[c], 8, cudaMemcpyDeviceToHost, s));
     LV_CUDA(cudaStreamSynchronize(s));
-    // chunks of ~equal staged entries per class (stage / table pipeline): binary searches
-    // of the chunk targets over soff on the device, one copy back
-    {
-      int64_t* dcut = nullptr;
-      LV_TRY(dalloc(&dcut, (size_t)kNumClasses * (Level::kChunks + 1) * 2, s));
-      ClassBounds cb;
-      std::memcpy(cb.off, L.class_off, sizeof cb.off);
-      k_chunk_cuts<<<kNumClasses, 32, 0, s>>>(L.soff, cb, Level::kChunks, dcut);
-      LV_LAUNCHED();
-      std::vector<int64_t> hc((size_t)kNumClasses * (Level::kChunks + 1) * 2);
-      LV_CUDA(cudaMemcpyAsync(hc.data(), dcut, 8 * hc.size(), cudaMemcpyDeviceToHost, s));
-      LV_CUDA(cudaStreamSynchronize(s));
-      dfree(dcut, s);
-      for (int c = 0; c < kNumClasses; ++c)
-        for (int k = 0; k <= Level::kChunks; ++k) {
-          L.chunk_pos[c][k] = hc[((size_t)c * (Level::kChunks + 1) + k) * 2];
-          L.chunk_soff[c][k] = hc[((size_t)c * (Level::kChunks + 1) + k) * 2 + 1];
-        }
-    }
   } else {
     std::fill(L.class_soff, L.class_soff + kNumClasses + 1, 0);
   }

@@ -1534,16 +1534,6 @@ int32_t launch_part(Handle& h, Level& L, const SweepArgs& A, int bucket, bool un
 // the fixed 512-slot warp tables of bucket 6 (C5 level 0: 10.2 -> 6.3 ms per 2
 // sweeps).  The CTA tables are sized 2*deg, where the list measured slower
 // (b7 [1024,2048): 12.5 -> 19.4 ms), and so was the 128-slot warp table of bucket 5.
-// stage / table pipeline (LV_PIPE=0: stage the whole bucket first; A/B) and the stage grid
-// in CTAs per SM while pipelining (LV_STAGE_SM, A/B)
-static bool pipe_on() {
-  static const bool on = !(getenv("LV_PIPE") && getenv("LV_PIPE")[0] == '0');
-  return on;
-}
-static int stage_per_sm() {
-  static const int v = getenv("LV_STAGE_SM") ? std::max(1, atoi(getenv("LV_STAGE_SM"))) : 4;
-  return v;
-}
 // register claim lists instead of table scans in the warp / CTA kernels (LV_CLAIM=0: scans; A/B)
 static bool claim_on() {
   static const bool on = !(getenv("LV_CLAIM") && getenv("LV_CLAIM")[0] == '0');
@@ -1556,11 +1546,9 @@ static int64_t max_deg_of_tier(int sub) {
 }
 
 template <bool UNIT, bool AGG>
-int32_t dispatch_class(Handle& h, Level& L, const SweepArgs& A, int bucket, int sub, int64_t max_deg,
-                       int64_t p_lo = -1, int64_t p_hi = -1) {
-  // the class's bin positions, or the chunk [p_lo, p_hi) of them (stage / table pipeline)
-  const int64_t off = p_lo >= 0 ? p_lo : L.class_off[kSubPerBucket * bucket + sub];
-  const int64_t nv = (p_lo >= 0 ? p_hi : L.class_off[kSubPerBucket * bucket + sub + 1]) - off;
+int32_t dispatch_class(Handle& h, Level& L, const SweepArgs& A, int bucket, int sub, int64_t max_deg) {
+  const int64_t off = L.class_off[kSubPerBucket * bucket + sub];
+  const int64_t nv = L.class_off[kSubPerBucket * bucket + sub + 1] - off;
   if (nv <= 0) return LOUVAIN_OK;
   const int32_t* verts = L.bin_vertices + off;
   const int64_t* soff = L.soff + off;
@@ -1681,11 +1669,11 @@ static void trace_step(Handle& h, Level& L, int bucket, int sub, int64_t pos0, i
           (long)(e[1] - e[0]), ms, ms > 0 ? (e[1] - e[0]) / ms / 1e6 : 0.0);
 }
 
-int32_t launch_stage(Handle& h, Level& L, int64_t pos0, int64_t pos1, int64_t s0, int64_t s1, int per_sm) {
+int32_t launch_stage(Handle& h, Level& L, int64_t pos0, int64_t pos1, int64_t s0, int64_t s1) {
   if (s1 <= s0) return LOUVAIN_OK;
   const int64_t* tr = nullptr;
   LV_TRY(tile_starts(h, L.soff, pos0, pos1, s0, s1, kStageTile, &tr));
-  k_stage<<<grid_for((s1 - s0 + kStageTile - 1) / kStageTile, 1, 148 * per_sm), 256, 0, h.stream>>>(
+  k_stage<<<grid_for((s1 - s0 + kStageTile - 1) / kStageTile, 1, 148 * 8), 256, 0, h.stream>>>(
       L.bin_vertices, L.soff, pos0, pos1, tr, L.rowptr, L.col, L.ca, L.stage);
   LV_LAUNCHED();
   LV_CUDA(cudaGetLastError());
@@ -1735,12 +1723,12 @@ int32_t launch_sweep_bucket(Handle& h, Level& L, const louvain_params_t& p, int 
     LV_CUDA(cudaGetLastError());
     return LOUVAIN_OK;
   }
-  auto dispatch = [&](int sub, int64_t p_lo = -1, int64_t p_hi = -1) -> int32_t {
+  auto dispatch = [&](int sub) -> int32_t {
     const int64_t max_deg = (sub == 0) ? std::min<int64_t>(hi, kSub1Min - 1) : hi;
     // warp-level label merging (__match_any_sync before the table insert) is
     // off: measured slower at every level and sweep of C5 (profiles/README.md)
-    if (L.w) LV_TRY((dispatch_class<false, false>(h, L, A, bucket, sub, max_deg, p_lo, p_hi)));
-    else LV_TRY((dispatch_class<true, false>(h, L, A, bucket, sub, max_deg, p_lo, p_hi)));
+    if (L.w) LV_TRY((dispatch_class<false, false>(h, L, A, bucket, sub, max_deg)));
+    else LV_TRY((dispatch_class<true, false>(h, L, A, bucket, sub, max_deg)));
     if (trace_on())
       trace_step(h, L, bucket, sub, L.class_off[kSubPerBucket * bucket + sub],
                  L.class_off[kSubPerBucket * bucket + sub + 1]);
@@ -1756,49 +1744,8 @@ int32_t launch_sweep_bucket(Handle& h, Level& L, const louvain_params_t& p, int 
   // the bucket: both read only the bucket-start snapshot and append to the move
   // log; the commit waits for both (LV_TRACE=2 serialises).
   const bool overlap = !trace_on() && posp < pos1 && posp > pos0 && L.hub.nh == 0;
-  if (!trace_on() && L.hub.nh == 0 && pipe_on() && pos1 > pos0) {
-    // hub classes: staged first, their tasks on the side stream (as in `overlap`)
-    if (posp < pos1) {
-      LV_TRY(launch_stage(h, L, posp, pos1, L.class_soff[cp], L.class_soff[c1], 8));
-      LV_CUDA(cudaEventRecord(h.ev_fork, h.stream));
-      LV_CUDA(cudaStreamWaitEvent(h.side, h.ev_fork, 0));
-      cudaStream_t main_s = h.stream;
-      h.stream = h.side;
-      int32_t rc = LOUVAIN_OK;
-      for (int sub = kSubPart; sub < kSubPerBucket && rc == LOUVAIN_OK; ++sub) rc = dispatch(sub);
-      h.stream = main_s;
-      LV_TRY(rc);
-      LV_CUDA(cudaEventRecord(h.ev_join, h.side));
-    }
-    // the other classes in chunks: stage chunk k on the main stream, its table kernel on
-    // h.tabs once stage k is done -- memory-bound gathers of chunk k+1 overlap the
-    // issue-bound hashing of chunk k (both read only the bucket-start snapshot)
-    int ev = 0;
-    for (int c = c0; c < cp; ++c) {
-      for (int k = 0; k < Level::kChunks; ++k) {
-        const int64_t p_lo = L.chunk_pos[c][k], p_hi = L.chunk_pos[c][k + 1];
-        if (p_hi <= p_lo) continue;
-        if (ev >= Handle::kChunkEvents) { set_error("sweep: too many pipeline chunks"); return LOUVAIN_E_STATE; }
-        LV_TRY(launch_stage(h, L, p_lo, p_hi, L.chunk_soff[c][k], L.chunk_soff[c][k + 1], stage_per_sm()));
-        LV_CUDA(cudaEventRecord(h.ev_chunk[ev], h.stream));
-        LV_CUDA(cudaStreamWaitEvent(h.tabs, h.ev_chunk[ev], 0));
-        ++ev;
-        cudaStream_t main_s = h.stream;
-        h.stream = h.tabs;
-        const int32_t rc = dispatch(c - kSubPerBucket * bucket, p_lo, p_hi);
-        h.stream = main_s;
-        LV_TRY(rc);
-      }
-    }
-    if (ev > 0) {
-      LV_CUDA(cudaEventRecord(h.ev_join2, h.tabs));
-      LV_CUDA(cudaStreamWaitEvent(h.stream, h.ev_join2, 0));
-    }
-    if (posp < pos1) LV_CUDA(cudaStreamWaitEvent(h.stream, h.ev_join, 0));
-    return LOUVAIN_OK;
-  }
   if (overlap) {
-    LV_TRY(launch_stage(h, L, posp, pos1, L.class_soff[cp], L.class_soff[c1], 8));
+    LV_TRY(launch_stage(h, L, posp, pos1, L.class_soff[cp], L.class_soff[c1]));
     LV_CUDA(cudaEventRecord(h.ev_fork, h.stream));
     LV_CUDA(cudaStreamWaitEvent(h.side, h.ev_fork, 0));
     cudaStream_t main_s = h.stream;
@@ -1808,12 +1755,12 @@ int32_t launch_sweep_bucket(Handle& h, Level& L, const louvain_params_t& p, int 
     h.stream = main_s;
     LV_TRY(rc);
     LV_CUDA(cudaEventRecord(h.ev_join, h.side));
-    LV_TRY(launch_stage(h, L, pos0, posp, L.class_soff[c0], L.class_soff[cp], 8));
+    LV_TRY(launch_stage(h, L, pos0, posp, L.class_soff[c0], L.class_soff[cp]));
     for (int sub = 0; sub < kSubPart; ++sub) LV_TRY(dispatch(sub));
     LV_CUDA(cudaStreamWaitEvent(h.stream, h.ev_join, 0));
     return LOUVAIN_OK;
   }
-  if (pos1 > pos0) LV_TRY(launch_stage(h, L, pos0, pos1, L.class_soff[c0], L.class_soff[c1], 8));
+  if (pos1 > pos0) LV_TRY(launch_stage(h, L, pos0, pos1, L.class_soff[c0], L.class_soff[c1]));
   if (trace_on()) trace_step(h, L, bucket, -1, pos0, pos1);
   for (int sub = 0; sub < kSubPerBucket; ++sub) LV_TRY(dispatch(sub));
   return LOUVAIN_OK;
