@@ -508,106 +508,6 @@ __global__ void __launch_bounds__(THREADS) k_big_combine(const uint32_t* __restr
   }
 }
 
-// 64-bit-key combiner (segment rank and neighbour need more than 32 bits, e.g. C5
-// level 1: 15 + 23 bits): chunks of kCombChunk entries hashed in shared memory, key
-// slots (CAS) beside 32-bit value slots (atomic adds, order-free), distinct
-// (key, sum) pairs of every chunk appended with one global atomic per CTA; a key
-// whose probe sequence passes kCombProbes slots is passed through unchanged.  The
-// sums per key are those of the input, so the sort + reduce-by-key that follow
-// give the same CSR' on fewer entries.
-constexpr int kComb64Slots = 12288;  // 12 B each: 144 KB
-template <int THREADS>
-__global__ void __launch_bounds__(THREADS) k_big_combine64(const unsigned long long* __restrict__ keys,
-                                                           const uint32_t* __restrict__ vals, int64_t m,
-                                                           unsigned long long* __restrict__ okeys,
-                                                           uint32_t* __restrict__ ovals, unsigned long long* ocount) {
-  extern __shared__ unsigned long long KT[];  // kComb64Slots keys, then kComb64Slots 32-bit values
-  uint32_t* VT = reinterpret_cast<uint32_t*>(KT + kComb64Slots);
-  __shared__ unsigned wcnt[THREADS / 32];
-  __shared__ unsigned long long sh_base;
-  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-  for (int t = threadIdx.x; t < kComb64Slots; t += blockDim.x) {
-    KT[t] = kEmpty;
-    VT[t] = 0;
-  }
-  __syncthreads();
-  const int64_t nch = (m + kCombChunk - 1) / kCombChunk;
-  for (int64_t ch = blockIdx.x; ch < nch; ch += gridDim.x) {
-    const int64_t e0 = ch * kCombChunk, e1 = min(m, e0 + kCombChunk);
-    for (int64_t eb = e0 + threadIdx.x; eb - threadIdx.x < e1; eb += (int64_t)blockDim.x) {
-      const bool has = eb < e1;
-      unsigned long long k = has ? __ldcs(&keys[eb]) : kEmpty;
-      uint32_t v = has ? __ldcs(&vals[eb]) : 0u;
-      // equal keys of the warp merged first (hot neighbours)
-      const unsigned mm = __match_any_sync(kFull, k);
-      v = __reduce_add_sync(mm, v);
-      bool pass = false;
-      if (has && lane == __ffs(mm) - 1) {
-        uint32_t h = (uint32_t)(((k * 0x9E3779B97F4A7C15ull) >> 32) % (unsigned long long)kComb64Slots);
-        int pr = 0;
-        for (; pr < kCombProbes; ++pr) {
-          const unsigned long long old = atomicCAS(&KT[h], kEmpty, k);
-          if (old == kEmpty || old == k) {
-            atomicAdd(&VT[h], v);
-            break;
-          }
-          h = (h + 1 == (uint32_t)kComb64Slots) ? 0u : h + 1;
-        }
-        pass = pr == kCombProbes;
-      }
-      const unsigned mk = __ballot_sync(kFull, pass);  // pass-throughs: warp-aggregated append
-      if (mk) {
-        unsigned long long b = 0;
-        if (lane == __ffs(mk) - 1) b = atomicAdd(ocount, (unsigned long long)__popc(mk));
-        b = __shfl_sync(kFull, b, __ffs(mk) - 1);
-        if (pass) {
-          const unsigned long long o = b + __popc(mk & ((1u << lane) - 1u));
-          okeys[o] = k;
-          ovals[o] = v;
-        }
-      }
-    }
-    __syncthreads();
-    // emit the chunk's distinct pairs: per-warp counts -> one global atomic per CTA
-    constexpr int kPer = (kComb64Slots + THREADS - 1) / THREADS;
-    const int s0 = wid * 32 * kPer;
-    unsigned mine = 0;
-    for (int u = 0; u < kPer; ++u) {
-      const int t = s0 + u * 32 + lane;
-      mine += (t < kComb64Slots && KT[t] != kEmpty) ? 1u : 0u;
-    }
-    const unsigned wsum = __reduce_add_sync(kFull, mine);
-    if (lane == 0) wcnt[wid] = wsum;
-    __syncthreads();
-    if (threadIdx.x == 0) {
-      unsigned tot = 0;
-      for (int w = 0; w < THREADS / 32; ++w) {
-        const unsigned c = wcnt[w];
-        wcnt[w] = tot;
-        tot += c;
-      }
-      sh_base = tot ? atomicAdd(ocount, (unsigned long long)tot) : 0ull;
-    }
-    __syncthreads();
-    unsigned long long o = sh_base + wcnt[wid];
-    for (int u = 0; u < kPer; ++u) {
-      const int t = s0 + u * 32 + lane;
-      const unsigned long long x = t < kComb64Slots ? KT[t] : kEmpty;
-      const bool has = x != kEmpty;
-      const unsigned mk = __ballot_sync(kFull, has);
-      if (has) {
-        const unsigned long long oo = o + __popc(mk & ((1u << lane) - 1u));
-        okeys[oo] = x;
-        ovals[oo] = VT[t];
-        KT[t] = kEmpty;
-        VT[t] = 0;
-      }
-      o += __popc(mk);
-    }
-    __syncthreads();
-  }
-}
-
 // Lengths of the big segments (the scan turns them into key-array offsets).
 __global__ void k_big_len(const int32_t* __restrict__ rows, int64_t nbig, const int64_t* __restrict__ sstart,
                           int64_t* len) {
@@ -750,11 +650,6 @@ int32_t cub_scan_excl(cudaStream_t s, A... a) {
 }  // namespace
 
 namespace {
-// LV_COMB64=0: no 64-bit-key combiner before the big-segment sort (A/B)
-bool comb64_on() {
-  static const bool on = !(getenv("LV_COMB64") && getenv("LV_COMB64")[0] == '0');
-  return on;
-}
 struct CTrace {
   bool on = getenv("LV_TRACE") != nullptr;
   std::chrono::steady_clock::time_point t0 = std::chrono::steady_clock::now();
@@ -1080,28 +975,6 @@ int32_t level_contract_fast(Handle& h, Level& L, Level& out, int32_t* d_map, int
       tr.mark(s, "big-keys");
       cub::DoubleBuffer<unsigned long long> kbuf(k0, k1);
       cub::DoubleBuffer<uint32_t> vbuf(v0, v1);
-      if (m >= 64 * np && comb64_on()) {  // many repeats per new vertex: combine before the sort
-        static bool cattr = false;
-        if (!cattr) {
-          LV_CUDA(cudaFuncSetAttribute(k_big_combine64<1024>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                       12 * kComb64Slots));
-          cattr = true;
-        }
-        unsigned long long* dcnt = reinterpret_cast<unsigned long long*>(&h.ctl->bad);
-        LV_CUDA(cudaMemsetAsync(dcnt, 0, 8, s));
-        k_big_combine64<1024><<<grid_for((m + kCombChunk - 1) / kCombChunk, 1, 148), 1024, 12 * kComb64Slots, s>>>(
-            k0, v0, m, k1, v1, dcnt);
-        LV_LAUNCHED();
-        unsigned long long m2 = 0;
-        LV_CUDA(cudaMemcpyAsync(&m2, dcnt, 8, cudaMemcpyDeviceToHost, s));
-        LV_CUDA(cudaStreamSynchronize(s));
-        if (tr.on) fprintf(stderr, "[lv]    contract combine64: %lld -> %llu entries\n", (long long)m, m2);
-        m = (int64_t)m2;
-        kbuf = cub::DoubleBuffer<unsigned long long>(k1, k0);
-        vbuf = cub::DoubleBuffer<uint32_t>(v1, v0);
-        LV_CUDA(cudaMemsetAsync(&h.ctl->bad, 0, 8, s));
-        tr.mark(s, "big-combine");
-      }
       size_t tb = 0;
       LV_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, tb, kbuf, vbuf, m, 0, nb + kb, s));
       void* tmp = nullptr;
