@@ -533,6 +533,75 @@ __device__ __forceinline__ void eval_claims(unsigned long long* T, uint32_t* TA,
   }
 }
 
+// The same inserts gathering the neighbour records directly (no stage): entry t of
+// row v reads col[rb + t] and ca[col] (all 4 * PASSES gathers of a lane in flight
+// together), the self-loop skipped (R3), a_c known when the neighbour represents
+// its label.
+template <bool UNIT, int PASSES>
+__device__ __forceinline__ void insert_claim_direct(unsigned long long* T, uint32_t* TA, uint32_t cap,
+                                                    const SweepArgs& A, int32_t v, int64_t rb, int64_t deg, int t0,
+                                                    int stride, uint32_t (&cl)[4 * PASSES]) {
+  int32_t jj[4 * PASSES];
+  uint32_t ww[4 * PASSES];
+#pragma unroll
+  for (int u = 0; u < 4 * PASSES; ++u) {
+    const int64_t t = (int64_t)t0 + (int64_t)u * stride;
+    jj[u] = (t < deg) ? __ldcs(&A.col[rb + t]) : -1;
+    ww[u] = UNIT ? 1u : ((t < deg) ? __ldcs(&A.w[rb + t]) : 0u);
+  }
+  uint2 rr[4 * PASSES];
+#pragma unroll
+  for (int u = 0; u < 4 * PASSES; ++u) rr[u] = (jj[u] >= 0 && jj[u] != v) ? __ldg(&A.ca[jj[u]]) : make_uint2(kSelf, 0);
+#pragma unroll
+  for (int u = 0; u < 4 * PASSES; ++u) {
+    uint32_t slot = kNoClaim;
+    if (rr[u].x != kSelf) {
+      bool claimed = false;
+      const uint32_t hq = table_insert_c(T, cap, (int32_t)rr[u].x, ww[u], &claimed);
+      if (rr[u].x == (uint32_t)jj[u]) TA[hq] = rr[u].y;  // the neighbour represents its label
+      if (claimed) slot = hq;
+    }
+    cl[u] = slot;
+  }
+}
+
+// Warp per vertex gathering directly (no stage round trip of 16 B per entry).
+template <int CAP, int WARPS, bool UNIT, int PASSES>
+__global__ void __launch_bounds__(32 * WARPS) sweep_warp_d(const int32_t* __restrict__ verts, int64_t nv,
+                                                           SweepArgs A) {
+  __shared__ unsigned long long tab[WARPS][CAP];
+  __shared__ uint32_t taba[WARPS][CAP];
+  const int lane = threadIdx.x & 31, wl = threadIdx.x >> 5;
+  unsigned long long* T = tab[wl];
+  uint32_t* TA = taba[wl];
+  for (int t = lane; t < CAP; t += 32) {
+    T[t] = kEmpty;
+    TA[t] = kUnknownA;
+  }
+  __syncwarp();
+  const int64_t warps = (int64_t)gridDim.x * WARPS;
+  for (int64_t vi = (int64_t)blockIdx.x * WARPS + wl; vi < nv; vi += warps) {
+    const int32_t v = __ldg(&verts[vi]);
+    const int64_t rb = __ldg(&A.rowptr[v]);
+    const int64_t deg = __ldg(&A.rowptr[v + 1]) - rb;
+    const int32_t own = (int32_t)__ldg(&A.ca[v]).x;
+    const uint32_t ki = __ldg(&A.k[v]);
+    uint32_t cl[4 * PASSES];
+    insert_claim_direct<UNIT, PASSES>(T, TA, CAP, A, v, rb, deg, lane, 32, cl);
+    __syncwarp();
+    const bool own_single = A.rule == 2 && __ldg(&A.size[own]) == 1;
+    long long s = (long long)0x8000000000000000ull;
+    int cb = 0x7FFFFFFF;
+    unsigned eown = 0;
+    eval_claims<PASSES>(T, TA, cl, own, own_single, ki, A, s, cb, eown);
+    group_reduce<32>(s, cb, eown);
+    int32_t tgt = own;
+    if (lane == 0) tgt = finish(s, cb, eown, own, __ldg(&A.ca[own]).y, ki, A);
+    log_moves(lane == 0 && tgt != own, v, tgt, A);
+    __syncwarp();
+  }
+}
+
 // Warp per vertex with register claims (rows of <= 128 * PASSES entries).
 template <int CAP, int WARPS, bool UNIT, int PASSES>
 __global__ void __launch_bounds__(32 * WARPS) sweep_warp_c(const int32_t* __restrict__ verts,
@@ -1534,6 +1603,11 @@ int32_t launch_part(Handle& h, Level& L, const SweepArgs& A, int bucket, bool un
 // the fixed 512-slot warp tables of bucket 6 (C5 level 0: 10.2 -> 6.3 ms per 2
 // sweeps).  The CTA tables are sized 2*deg, where the list measured slower
 // (b7 [1024,2048): 12.5 -> 19.4 ms), and so was the 128-slot warp table of bucket 5.
+// warp kernels of the mid buckets gathering directly instead of reading the stage (LV_DIRECT=1; A/B)
+bool direct_on() {
+  static const bool on = getenv("LV_DIRECT") && getenv("LV_DIRECT")[0] == '1';
+  return on;
+}
 // register claim lists instead of table scans in the warp / CTA kernels (LV_CLAIM=0: scans; A/B)
 static bool claim_on() {
   static const bool on = !(getenv("LV_CLAIM") && getenv("LV_CLAIM")[0] == '0');
@@ -1563,6 +1637,12 @@ int32_t dispatch_class(Handle& h, Level& L, const SweepArgs& A, int bucket, int 
       case 16: sweep_small<16, UNIT><<<grid, 256, 0, s>>>(verts, nv, A); break;
       default: sweep_small<32, UNIT><<<grid, 256, 0, s>>>(verts, nv, A); break;
     }
+    LV_LAUNCHED();
+  } else if (sub == 0 && max_deg > 84 && max_deg <= 340 && direct_on()) {
+    sweep_warp_d<512, 4, UNIT, 3><<<grid_for(nv, 4, 148 * 8), 128, 0, s>>>(verts, nv, A);
+    LV_LAUNCHED();
+  } else if (sub == 0 && max_deg <= 84 && direct_on()) {
+    sweep_warp_d<128, 8, UNIT, 1><<<grid_for(nv, 8, 148 * 8), 256, 0, s>>>(verts, nv, A);
     LV_LAUNCHED();
   } else if (sub == 0 && max_deg > 84 && max_deg <= 340 && claim_on()) {
     sweep_warp_c<512, 4, UNIT, 3><<<grid_for(nv, 4, 148 * 8), 128, 0, s>>>(verts, soff, nv, stage, A);
@@ -1735,7 +1815,8 @@ int32_t launch_sweep_bucket(Handle& h, Level& L, const louvain_params_t& p, int 
     return LOUVAIN_OK;
   };
   // phase 1: gather the records of every neighbour of the bucket's table-based vertices
-  const bool sub0_small = std::min<int64_t>(hi, kSub1Min - 1) <= 32;
+  const int64_t sub0_max = std::min<int64_t>(hi, kSub1Min - 1);
+  const bool sub0_small = sub0_max <= 32 || (direct_on() && sub0_max <= 340);  // not staged
   const int c0 = kSubPerBucket * bucket + (sub0_small ? 1 : 0), c1 = kSubPerBucket * (bucket + 1);
   const int cp = kSubPerBucket * bucket + kSubPart;  // first label-partitioned class
   const int64_t pos0 = L.class_off[c0], pos1 = L.class_off[c1], posp = L.class_off[cp];
