@@ -683,240 +683,6 @@ __global__ void __launch_bounds__(1024) sweep_cta_c(const int32_t* __restrict__ 
   }
 }
 
-// ------------------------------------------------------------ warp per vertex
-template <int CAP, int WARPS, bool UNIT, bool AGG>
-__global__ void __launch_bounds__(32 * WARPS) sweep_warp(const int32_t* __restrict__ verts,
-                                                         const int64_t* __restrict__ soff, int64_t nv,
-                                                         const uint2* __restrict__ stage, SweepArgs A) {
-  __shared__ unsigned long long tab[WARPS][CAP];
-  __shared__ uint32_t taba[WARPS][CAP];
-  const int lane = threadIdx.x & 31, wl = threadIdx.x >> 5;
-  unsigned long long* T = tab[wl];
-  uint32_t* TA = taba[wl];
-  for (int t = lane; t < CAP; t += 32) {
-    T[t] = kEmpty;
-    TA[t] = kUnknownA;
-  }
-  __syncwarp();
-  const int64_t warps = (int64_t)gridDim.x * WARPS;
-  for (int64_t vi = (int64_t)blockIdx.x * WARPS + wl; vi < nv; vi += warps) {
-    const int32_t v = __ldg(&verts[vi]);
-    const int64_t rb = __ldg(&A.rowptr[v]);
-    const int64_t deg = __ldg(&A.rowptr[v + 1]) - rb;
-    const int32_t own = (int32_t)__ldg(&A.ca[v]).x;
-    const uint32_t ki = __ldg(&A.k[v]);
-    insert_staged<UNIT, AGG>(T, TA, CAP, stage + __ldg(&soff[vi]), UNIT ? nullptr : A.w + rb, deg, lane, 32);
-    __syncwarp();
-    const bool own_single = A.rule == 2 && __ldg(&A.size[own]) == 1;
-    long long s = (long long)0x8000000000000000ull;
-    int cb = 0x7FFFFFFF;
-    unsigned eown = 0;
-    scan_table(T, TA, CAP, lane, 32, own, own_single, ki, A, s, cb, eown);
-    group_reduce<32>(s, cb, eown);
-    int32_t tgt = own;
-    if (lane == 0) tgt = finish(s, cb, eown, own, __ldg(&A.ca[own]).y, ki, A);
-    log_moves(lane == 0 && tgt != own, v, tgt, A);
-    __syncwarp();
-  }
-}
-
-// ------------------------------------------------------------ CTA per vertex (default)
-template <bool UNIT, bool AGG>
-__global__ void __launch_bounds__(1024) sweep_cta(const int32_t* __restrict__ verts, const int64_t* __restrict__ soff,
-                                                  int64_t nv, const uint2* __restrict__ stage, SweepArgs A,
-                                                  int capmax, int fnum) {
-  extern __shared__ unsigned long long smem[];
-  unsigned long long* T = smem;
-  uint32_t* TA = reinterpret_cast<uint32_t*>(smem + capmax);
-  __shared__ long long sh_s[32];
-  __shared__ int sh_c[32];
-  __shared__ unsigned sh_e[32];
-  for (int t = threadIdx.x; t < capmax; t += blockDim.x) {
-    T[t] = kEmpty;
-    TA[t] = kUnknownA;
-  }
-  __syncthreads();
-  for (int64_t vi = blockIdx.x; vi < nv; vi += gridDim.x) {
-    const int32_t v = __ldg(&verts[vi]);
-    const int64_t rb = __ldg(&A.rowptr[v]);
-    const int64_t deg = __ldg(&A.rowptr[v + 1]) - rb;
-    const int32_t own = (int32_t)__ldg(&A.ca[v]).x;
-    const uint32_t ki = __ldg(&A.k[v]);
-    // table of deg * (1 + fnum/8) slots (fnum = 8: load 1/2), at most capmax
-    const int64_t want = deg + ((deg * fnum) >> 3) + 1;
-    const uint32_t cap = (uint32_t)(want < (int64_t)capmax ? want : (int64_t)capmax);
-    insert_staged<UNIT, AGG>(T, TA, cap, stage + __ldg(&soff[vi]), UNIT ? nullptr : A.w + rb, deg, threadIdx.x,
-                             blockDim.x);
-    __syncthreads();
-    const bool own_single = A.rule == 2 && __ldg(&A.size[own]) == 1;
-    long long s = (long long)0x8000000000000000ull;
-    int cb = 0x7FFFFFFF;
-    unsigned eown = 0;
-    scan_table(T, TA, cap, threadIdx.x, blockDim.x, own, own_single, ki, A, s, cb, eown);
-    block_reduce(s, cb, eown, sh_s, sh_c, sh_e);
-    if (threadIdx.x < 32) {
-      int32_t tgt = own;
-      if (threadIdx.x == 0) tgt = finish(s, cb, eown, own, __ldg(&A.ca[own]).y, ki, A);
-      log_moves(threadIdx.x == 0 && tgt != own, v, tgt, A);
-    }
-    __syncthreads();
-  }
-}
-
-
-// ------------------------------------------------------------ claimed-slot lists (default)
-// The thread whose CAS claims an empty slot appends the slot index to the
-// table's list (warp-aggregated, one shared atomic per warp and pass), so the
-// scan visits exactly the distinct labels with full warps instead of every
-// slot of the table (ncu, C5 sweep 1: the slot scan of the warp / CTA kernels
-// ran at 10-20 active lanes per instruction and was ~45% of their instructions).
-// The four inserts of a pass share one retry loop (independent CASes in flight
-// instead of four divergent probe loops).
-template <bool UNIT>
-__device__ __forceinline__ void insert_list(unsigned long long* T, uint32_t* TA, uint32_t cap,
-                                            const uint2* __restrict__ S, const uint32_t* __restrict__ Wt,
-                                            int64_t deg, int64_t t0, int64_t stride, uint16_t* Lst, int* nL) {
-  const int lane = threadIdx.x & 31;
-  const int64_t t_warp0 = t0 - lane;
-  for (int64_t base = 0; base + t_warp0 < deg; base += 4 * stride) {  // trip count uniform across the warp
-    uint2 rr[4];
-    uint32_t ww[4];
-#pragma unroll
-    for (int q = 0; q < 4; ++q) {
-      const int64_t t = base + t0 + q * stride;
-      rr[q] = (t < deg) ? __ldcs(&S[t]) : make_uint2(kSelf, 0u);
-      ww[q] = UNIT ? 1u : ((t < deg) ? __ldcs(&Wt[t]) : 0u);
-    }
-    uint32_t h[4];
-    bool todo[4], claimed[4];
-#pragma unroll
-    for (int q = 0; q < 4; ++q) {
-      todo[q] = rr[q].x != kSelf;
-      claimed[q] = false;
-      h[q] = todo[q] ? hash_slot((int32_t)rr[q].x, cap) : 0u;
-    }
-    while (todo[0] || todo[1] || todo[2] || todo[3]) {
-#pragma unroll
-      for (int q = 0; q < 4; ++q) {
-        if (!todo[q]) continue;
-        const unsigned long long kx = ((unsigned long long)rr[q].x << 32) | ww[q];
-        const unsigned long long old = atomicCAS(&T[h[q]], kEmpty, kx);
-        if (old == kEmpty) {
-          claimed[q] = true;
-          todo[q] = false;
-        } else if ((uint32_t)(old >> 32) == rr[q].x) {
-          atomicAdd(&T[h[q]], (unsigned long long)ww[q]);
-          todo[q] = false;
-        } else {
-          h[q] = (h[q] + 1 == cap) ? 0u : h[q] + 1;
-        }
-      }
-    }
-#pragma unroll
-    for (int q = 0; q < 4; ++q)
-      if (rr[q].x != kSelf && rr[q].y != kUnknownA) TA[h[q]] = rr[q].y;
-    unsigned m[4];
-    int tot = 0;
-#pragma unroll
-    for (int q = 0; q < 4; ++q) {
-      m[q] = __ballot_sync(kFull, claimed[q]);
-      tot += __popc(m[q]);
-    }
-    if (tot) {
-      int b0 = 0;
-      if (lane == 0) b0 = atomicAdd(nL, tot);
-      b0 = __shfl_sync(kFull, b0, 0);
-      const unsigned lt = lanemask_lt();
-#pragma unroll
-      for (int q = 0; q < 4; ++q) {
-        if (claimed[q]) Lst[b0 + __popc(m[q] & lt)] = (uint16_t)h[q];
-        b0 += __popc(m[q]);
-      }
-    }
-  }
-}
-
-// Scan of the claimed slots (entries [t0, nl) step `stride` of the list); clears
-// each visited slot for the next vertex.
-__device__ __forceinline__ void scan_list(unsigned long long* T, uint32_t* TA, const uint16_t* Lst, int nl, int t0,
-                                          int stride, int32_t own, bool own_single, uint32_t ki, const SweepArgs& A,
-                                          long long& s, int& cb, unsigned& eown) {
-  for (int base = t0; base < nl; base += 4 * stride) {
-    unsigned long long x[4];
-    uint32_t ac[4];
-#pragma unroll
-    for (int q = 0; q < 4; ++q) {
-      const int t = base + q * stride;
-      x[q] = kEmpty;
-      ac[q] = kUnknownA;
-      if (t < nl) {
-        const uint32_t sl = Lst[t];
-        x[q] = T[sl];
-        ac[q] = TA[sl];
-        T[sl] = kEmpty;
-        TA[sl] = kUnknownA;
-      }
-    }
-#pragma unroll
-    for (int q = 0; q < 4; ++q) {
-      if (x[q] != kEmpty && ac[q] == kUnknownA && (int32_t)(x[q] >> 32) != own)
-        ac[q] = __ldg(&A.ca[(int32_t)(x[q] >> 32)]).y;
-    }
-#pragma unroll
-    for (int q = 0; q < 4; ++q) {
-      if (x[q] == kEmpty) continue;
-      const int32_t c = (int32_t)(x[q] >> 32);
-      const uint32_t e = (uint32_t)x[q];
-      if (c == own) eown = e;
-      else consider(c, e, ac[q], own, own_single, ki, A, s, cb);
-    }
-  }
-}
-
-template <int CAP, int LCAP, int WARPS, bool UNIT>
-__global__ void __launch_bounds__(32 * WARPS) sweep_warp_l(const int32_t* __restrict__ verts,
-                                                           const int64_t* __restrict__ soff, int64_t nv,
-                                                           const uint2* __restrict__ stage, SweepArgs A) {
-  __shared__ unsigned long long tab[WARPS][CAP];
-  __shared__ uint32_t taba[WARPS][CAP];
-  __shared__ uint16_t lst[WARPS][LCAP];
-  __shared__ int nls[WARPS];
-  const int lane = threadIdx.x & 31, wl = threadIdx.x >> 5;
-  unsigned long long* T = tab[wl];
-  uint32_t* TA = taba[wl];
-  for (int t = lane; t < CAP; t += 32) {
-    T[t] = kEmpty;
-    TA[t] = kUnknownA;
-  }
-  if (lane == 0) nls[wl] = 0;
-  __syncwarp();
-  const int64_t warps = (int64_t)gridDim.x * WARPS;
-  for (int64_t vi = (int64_t)blockIdx.x * WARPS + wl; vi < nv; vi += warps) {
-    const int32_t v = __ldg(&verts[vi]);
-    const int64_t rb = __ldg(&A.rowptr[v]);
-    const int64_t deg = __ldg(&A.rowptr[v + 1]) - rb;
-    const int32_t own = (int32_t)__ldg(&A.ca[v]).x;
-    const uint32_t ki = __ldg(&A.k[v]);
-    insert_list<UNIT>(T, TA, CAP, stage + __ldg(&soff[vi]), UNIT ? nullptr : A.w + rb, deg, lane, 32, lst[wl],
-                      &nls[wl]);
-    __syncwarp();
-    const int nl = nls[wl];
-    const bool own_single = A.rule == 2 && __ldg(&A.size[own]) == 1;
-    long long s = (long long)0x8000000000000000ull;
-    int cb = 0x7FFFFFFF;
-    unsigned eown = 0;
-    scan_list(T, TA, lst[wl], nl, lane, 32, own, own_single, ki, A, s, cb, eown);
-    group_reduce<32>(s, cb, eown);
-    int32_t tgt = own;
-    if (lane == 0) {
-      tgt = finish(s, cb, eown, own, __ldg(&A.ca[own]).y, ki, A);
-      nls[wl] = 0;
-    }
-    log_moves(lane == 0 && tgt != own, v, tgt, A);
-    __syncwarp();
-  }
-}
-
 // ------------------------------------------------------------ label-partitioned CTAs
 // deg >= 12288: vertex v gets P = ceil(deg / kPartLabels) independent CTA tasks;
 // task p owns the labels c with part_of(c, P) == p, so a partition sees
@@ -1603,16 +1369,10 @@ int32_t launch_part(Handle& h, Level& L, const SweepArgs& A, int bucket, bool un
 // the fixed 512-slot warp tables of bucket 6 (C5 level 0: 10.2 -> 6.3 ms per 2
 // sweeps).  The CTA tables are sized 2*deg, where the list measured slower
 // (b7 [1024,2048): 12.5 -> 19.4 ms), and so was the 128-slot warp table of bucket 5.
-// warp kernels of the mid buckets gathering directly instead of reading the stage (LV_DIRECT=1; A/B)
-bool direct_on() {
-  static const bool on = getenv("LV_DIRECT") && getenv("LV_DIRECT")[0] == '1';
-  return on;
-}
-// register claim lists instead of table scans in the warp / CTA kernels (LV_CLAIM=0: scans; A/B)
-static bool claim_on() {
-  static const bool on = !(getenv("LV_CLAIM") && getenv("LV_CLAIM")[0] == '0');
-  return on;
-}
+// Rows of <= kDirectMaxDeg entries (bucket 5 with the paper's bounds) are hashed by a warp
+// that gathers the records itself (sweep_warp_d): C5 level 0 bucket 5 stage 2.8 + warp 2.2 ->
+// 4.0 ms; bucket 6 (85-319) measured slower that way (6.5 -> 7.6 ms) and keeps the stage.
+constexpr int64_t kDirectMaxDeg = 84;
 // largest degree of CTA tier `sub` (lv_internal.cuh)
 static int64_t max_deg_of_tier(int sub) {
   static const int64_t ub[5] = {kSub1Min - 1, kSub2Min - 1, kSub3Min - 1, kSub4Min - 1, kSub5Min - 1};
@@ -1638,26 +1398,11 @@ int32_t dispatch_class(Handle& h, Level& L, const SweepArgs& A, int bucket, int 
       default: sweep_small<32, UNIT><<<grid, 256, 0, s>>>(verts, nv, A); break;
     }
     LV_LAUNCHED();
-  } else if (sub == 0 && max_deg > 84 && max_deg <= 340 && direct_on()) {
-    sweep_warp_d<512, 4, UNIT, 3><<<grid_for(nv, 4, 148 * 8), 128, 0, s>>>(verts, nv, A);
-    LV_LAUNCHED();
-  } else if (sub == 0 && max_deg <= 84 && direct_on()) {
+  } else if (sub == 0 && max_deg <= kDirectMaxDeg) {
     sweep_warp_d<128, 8, UNIT, 1><<<grid_for(nv, 8, 148 * 8), 256, 0, s>>>(verts, nv, A);
     LV_LAUNCHED();
-  } else if (sub == 0 && max_deg > 84 && max_deg <= 340 && claim_on()) {
+  } else if (sub == 0 && max_deg <= 340) {  // warp per vertex, 3 claim passes of 4 entries per lane
     sweep_warp_c<512, 4, UNIT, 3><<<grid_for(nv, 4, 148 * 8), 128, 0, s>>>(verts, soff, nv, stage, A);
-    LV_LAUNCHED();
-  } else if (sub == 0 && max_deg <= 84 && claim_on()) {
-    sweep_warp_c<128, 8, UNIT, 1><<<grid_for(nv, 8, 148 * 8), 256, 0, s>>>(verts, soff, nv, stage, A);
-    LV_LAUNCHED();
-  } else if (sub == 0 && max_deg > 84 && max_deg <= 340) {
-    sweep_warp_l<512, 352, 4, UNIT><<<grid_for(nv, 4, 148 * 8), 128, 0, s>>>(verts, soff, nv, stage, A);
-    LV_LAUNCHED();
-  } else if (sub == 0 && max_deg <= 84) {
-    sweep_warp<128, 8, UNIT, AGG><<<grid_for(nv, 8, 148 * 8), 256, 0, s>>>(verts, soff, nv, stage, A);
-    LV_LAUNCHED();
-  } else if (sub == 0 && max_deg <= 340) {
-    sweep_warp<512, 4, UNIT, AGG><<<grid_for(nv, 4, 148 * 12), 128, 0, s>>>(verts, soff, nv, stage, A);
     LV_LAUNCHED();
   } else if (sub >= kSubPart) {
     if (sub == kSubPart) LV_TRY(launch_part(h, L, A, bucket, UNIT));  // one pipeline covers sub-classes kSubPart..
@@ -1665,18 +1410,8 @@ int32_t dispatch_class(Handle& h, Level& L, const SweepArgs& A, int bucket, int 
   } else {
     static const int* caps = kCapT;
     static const int* threads = kThrT;
-    static bool attr_done = false;
-    if (!attr_done) {
-      LV_TRY(set_smem(sweep_cta<true, false>, 12 * (size_t)kCapMax));
-      LV_TRY(set_smem(sweep_cta<false, false>, 12 * (size_t)kCapMax));
-      LV_TRY(set_smem(sweep_cta<true, true>, 12 * (size_t)kCapMax));
-      LV_TRY(set_smem(sweep_cta<false, true>, 12 * (size_t)kCapMax));
-      attr_done = true;
-    }
-    constexpr int fnum = 8;  // table of 2*deg slots (1.5x / 1.75x / 2.5x / 3x measured slower)
-    static int resident[5] = {0, 0, 0, 0, 0};
     const int64_t md = std::min<int64_t>(max_deg_of_tier(sub), max_deg);
-    if (claim_on()) {
+    {
       static bool cattr = false;
       if (!cattr) {
         LV_TRY(set_smem(sweep_cta_c<true, 1>, 12 * (size_t)kCapMax));
@@ -1708,17 +1443,6 @@ int32_t dispatch_class(Handle& h, Level& L, const SweepArgs& A, int bucket, int 
       set_error("sweep: CTA tier degree beyond the claim-list capacity");
       return LOUVAIN_E_UNSUPPORTED;
     }
-    const int capt = (int)std::min<int64_t>(caps[sub], ((md + ((md * fnum) >> 3) + 1 + 31) / 32) * 32);
-    if (resident[sub] == 0) {
-      int nb = 0;
-      LV_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, sweep_cta<UNIT, AGG>, threads[sub], 12 * (size_t)capt));
-      resident[sub] = std::max(nb, 1);
-    }
-    sweep_cta<UNIT, AGG><<<grid_for(nv, 1, 148 * resident[sub]), threads[sub], 12 * (size_t)capt, s>>>(
-        verts, soff, nv, stage, A, capt, fnum);
-    LV_LAUNCHED();
-    LV_CUDA(cudaGetLastError());
-    return LOUVAIN_OK;
   }
   LV_CUDA(cudaGetLastError());
   return LOUVAIN_OK;
@@ -1816,7 +1540,7 @@ int32_t launch_sweep_bucket(Handle& h, Level& L, const louvain_params_t& p, int 
   };
   // phase 1: gather the records of every neighbour of the bucket's table-based vertices
   const int64_t sub0_max = std::min<int64_t>(hi, kSub1Min - 1);
-  const bool sub0_small = sub0_max <= 32 || (direct_on() && sub0_max <= 340);  // not staged
+  const bool sub0_small = sub0_max <= kDirectMaxDeg;  // register kernels / direct warp kernels: not staged
   const int c0 = kSubPerBucket * bucket + (sub0_small ? 1 : 0), c1 = kSubPerBucket * (bucket + 1);
   const int cp = kSubPerBucket * bucket + kSubPart;  // first label-partitioned class
   const int64_t pos0 = L.class_off[c0], pos1 = L.class_off[c1], posp = L.class_off[cp];
