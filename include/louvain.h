@@ -45,6 +45,8 @@ extern "C" {
 /* louvain_create_csr flags */
 #define LOUVAIN_VALIDATE 1u /* full O(n + nnz) validation incl. symmetry; else O(1) checks only */
 #define LOUVAIN_BORROW 2u   /* device inputs are used in place (caller keeps them alive, unmodified) */
+#define LOUVAIN_DIST_P2P 4u /* distributed handles: commits write every rank's replica through peer
+                               memory (CUDA IPC / NVLink P2P) + one barrier per bucket, no all-gather */
 
 /* modes */
 #define LOUVAIN_MODE_BIN_SYNC 0 /* Alg. 1: commit after each degree bucket (default) */

@@ -20,7 +20,7 @@ LIB_PATH = os.path.join(_HERE, "liblouvain.so")
 
 OK, E_INVALID_ARG, E_INVALID_GRAPH, E_OVERFLOW, E_NOMEM, E_CUDA, E_NCCL, E_STATE, E_UNSUPPORTED = \
     0, -1, -2, -3, -4, -5, -6, -7, -8
-VALIDATE, BORROW = 1, 2
+VALIDATE, BORROW, DIST_P2P = 1, 2, 4
 MODE_BIN_SYNC, MODE_RELAXED = 0, 1
 MAX_LEVELS = 256
 
@@ -223,11 +223,13 @@ class Graph:
     @classmethod
     def from_csr_dist(cls, n: int, v_begin: int, v_end: int, rowptr_local, col_local, w_local=None, *,
                       rank: int, world: int, comm: str = "nccl", group=None, validate: bool = False,
-                      stream=None) -> "Graph":
+                      p2p: bool = False, stream=None) -> "Graph":
         """Distributed handle (collective over the `world` ranks of `group`): this rank's rows
         [v_begin, v_end) with global column ids; see include/louvain.h.  comm="nccl": NCCL
         communicator, its unique id broadcast from rank 0 through torch.distributed;
-        comm="host": the library's host-side transport over torch.distributed (e.g. gloo)."""
+        comm="host": the library's host-side transport over torch.distributed (e.g. gloo).
+        p2p=True: commits write every rank's replica through peer memory (CUDA IPC), one
+        barrier per bucket instead of the all-gather of moves (LOUVAIN_DIST_P2P)."""
         from . import dist as _dist
         rowptr_local = _as(rowptr_local, np.int64)
         col_local = _as(col_local, np.int32)
@@ -238,7 +240,7 @@ class Graph:
         sp = None
         if stream is not None:
             sp = stream.cuda_stream if hasattr(stream, "cuda_stream") else int(stream)
-        flags = VALIDATE if validate else 0
+        flags = (VALIDATE if validate else 0) | (DIST_P2P if p2p else 0)
         h = ctypes.c_void_p()
         keep = None
         if comm == "nccl":

@@ -268,10 +268,185 @@ __global__ void k_dist_shift_rowptr(int64_t* rowptr, int64_t v0, int64_t v1, int
   for (int64_t i = v0 + blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < v1; i += (int64_t)gridDim.x * blockDim.x)
     rowptr[i] += add;
 }
+// Peer-memory commit of this rank's moves of one commit group (log [bounds[idx],
+// logn)): the commit of Alg. 1 l.8-11 (C[i] = newComm[i], exact integer a_c /
+// size_c deltas) applied to EVERY rank's replica -- the exchange is part of the
+// commit (remote stores and atomics over NVLink, or the same memory for ranks
+// sharing a GPU), so no move list crosses the interconnect and no all-gather runs.
+__global__ void k_commit_p2p(DevCtl* ctl, int idx, const int32_t* __restrict__ mv_v,
+                             const int32_t* __restrict__ mv_new, int32_t* __restrict__ mv_old,
+                             const PeerPtrs* __restrict__ pp, int world, int rank, const uint32_t* __restrict__ k,
+                             bool with_pcn) {
+  const unsigned long long start = ctl->bounds[idx];
+  const unsigned long long end = *(volatile unsigned long long*)&ctl->logn;
+  if (blockIdx.x == 0 && threadIdx.x == 0) ctl->bounds[idx + 1] = end;
+  const int32_t* Cl = pp->C[rank];
+  for (unsigned long long p = start + blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; p < end;
+       p += (unsigned long long)gridDim.x * blockDim.x) {
+    const int32_t i = mv_v[p], t = mv_new[p];
+    const int32_t old = Cl[i];  // i is this rank's vertex: no other rank writes C[i]
+    mv_old[p] = old;
+    const uint32_t ki = k[i];
+    for (int q = 0; q < world; ++q) {
+      uint32_t* w32 = reinterpret_cast<uint32_t*>(pp->ca[q]);
+      w32[2 * (int64_t)i] = (uint32_t)t;
+      pp->C[q][i] = t;
+      if (with_pcn) pp->pcn[q][i].y = (uint32_t)t;
+      atomicSub(&w32[2 * (int64_t)old + 1], ki);
+      atomicAdd(&w32[2 * (int64_t)t + 1], ki);
+      atomicSub(&pp->size[q][old], 1);
+      atomicAdd(&pp->size[q][t], 1);
+    }
+  }
+  __threadfence_system();  // the stores reach every replica before the barrier
+}
+// R15 for peer-memory commits: every rank undoes its own moves in every replica.
+__global__ void k_revert_p2p(const DevCtl* ctl, const int32_t* __restrict__ mv_v, const int32_t* __restrict__ mv_new,
+                             const int32_t* __restrict__ mv_old, const PeerPtrs* __restrict__ pp, int world,
+                             const uint32_t* __restrict__ k) {
+  const unsigned long long end = ctl->logn;
+  for (unsigned long long p = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; p < end;
+       p += (unsigned long long)gridDim.x * blockDim.x) {
+    const int32_t i = mv_v[p], t = mv_new[p], old = mv_old[p];
+    const uint32_t ki = k[i];
+    for (int q = 0; q < world; ++q) {
+      uint32_t* w32 = reinterpret_cast<uint32_t*>(pp->ca[q]);
+      w32[2 * (int64_t)i] = (uint32_t)old;
+      pp->C[q][i] = old;
+      atomicSub(&w32[2 * (int64_t)t + 1], ki);
+      atomicAdd(&w32[2 * (int64_t)old + 1], ki);
+      atomicSub(&pp->size[q][t], 1);
+      atomicAdd(&pp->size[q][old], 1);
+    }
+  }
+  __threadfence_system();
+}
+__global__ void k_copy_u64(const unsigned long long* src, unsigned long long* dst) { *dst = *src; }
 }  // namespace
 
 // ------------------------------------------------------------------ context
-DistCtx::~DistCtx() { delete comm; }
+DistCtx::~DistCtx() {
+  for (void* p : opened) cudaIpcCloseMemHandle(p);
+  for (void* p : rep_block)
+    if (p) cudaFree(p);
+  if (pcn_block) cudaFree(pcn_block);
+  for (PeerPtrs* p : d_peers)
+    if (p) cudaFree(p);
+  if (d_bar) cudaFree(d_bar);
+  delete comm;
+}
+
+int32_t dist_barrier(Handle& h) {
+  // a one-word all-reduce: it completes on a rank only after every rank's preceding
+  // stream work (the commit kernels and their system-scope fences) has completed
+  return h.dist->comm->allreduce_u64(h.dist->d_bar, 1, h.stream);
+}
+
+int32_t dist_total_moved(Handle& h) {
+  k_copy_u64<<<1, 1, 0, h.stream>>>(&h.ctl->logn, &h.ctl->gmoved);
+  LV_LAUNCHED();
+  if (!dist_p2p(h)) return LOUVAIN_OK;  // the all-gathered log already holds every rank's moves
+  return h.dist->comm->allreduce_u64(&h.ctl->gmoved, 1, h.stream);
+}
+
+int32_t dist_bind_state(Handle& h, Level& L, int set) {
+  DistCtx& D = *h.dist;
+  if (L.n > D.rep_n) {
+    set_error("distributed handle: level larger than the replica capacity");
+    return LOUVAIN_E_STATE;
+  }
+  char* b = static_cast<char*>(D.rep_block[set]);
+  L.ca = reinterpret_cast<uint2*>(b);
+  L.size = reinterpret_cast<int32_t*>(b + 8 * (size_t)D.rep_n);
+  L.C = reinterpret_cast<int32_t*>(b + 12 * (size_t)D.rep_n);
+  L.rep_set = set;
+  L.state_external = true;
+  return LOUVAIN_OK;
+}
+
+int32_t dist_commit_p2p(Handle& h, Level& L, int bucket) {
+  DistCtx& D = *h.dist;
+  k_commit_p2p<<<148 * 4, 256, 0, h.stream>>>(h.ctl, bucket, L.mv_v, L.mv_new, L.mv_old, D.d_peers[L.rep_set],
+                                             D.world, D.rank, L.k, h.pcn != nullptr);
+  LV_LAUNCHED();
+  LV_CUDA(cudaGetLastError());
+  return dist_barrier(h);
+}
+
+int32_t dist_revert_p2p(Handle& h, Level& L) {
+  DistCtx& D = *h.dist;
+  k_revert_p2p<<<148 * 4, 256, 0, h.stream>>>(h.ctl, L.mv_v, L.mv_new, L.mv_old, D.d_peers[L.rep_set], D.world, L.k);
+  LV_LAUNCHED();
+  LV_CUDA(cudaGetLastError());
+  return dist_barrier(h);
+}
+
+// Allocate the IPC-exportable replica sets and the delta-pass snapshot, exchange the
+// IPC handles through the transport and map every peer's blocks.
+static int32_t setup_p2p(Handle& h, int64_t n) {
+  DistCtx& D = *h.dist;
+  if (D.world > kMaxWorld) {
+    set_error("LOUVAIN_DIST_P2P: at most 64 ranks");
+    return LOUVAIN_E_UNSUPPORTED;
+  }
+  D.p2p = true;
+  D.rep_n = std::max<int64_t>(n, 1);
+  const size_t sb = 16 * (size_t)D.rep_n;
+  for (auto& b : D.rep_block) LV_CUDA(cudaMalloc(&b, sb));
+  LV_CUDA(cudaMalloc(&D.pcn_block, 8 * (size_t)D.rep_n));
+  LV_CUDA(cudaMalloc(&D.d_bar, 8));
+  LV_CUDA(cudaMemset(D.d_bar, 0, 8));
+  constexpr int kBlocks = 4;
+  cudaIpcMemHandle_t mine[kBlocks];
+  void* blocks[kBlocks] = {D.rep_block[0], D.rep_block[1], D.rep_block[2], D.pcn_block};
+  for (int b = 0; b < kBlocks; ++b) LV_CUDA(cudaIpcGetMemHandle(&mine[b], blocks[b]));
+  char *dsend = nullptr, *drecv = nullptr;
+  LV_TRY(dmalloc((void**)&dsend, sizeof mine, h.stream));
+  LV_TRY(dmalloc((void**)&drecv, sizeof mine * D.world, h.stream));
+  LV_CUDA(cudaMemcpyAsync(dsend, mine, sizeof mine, cudaMemcpyHostToDevice, h.stream));
+  LV_TRY(D.comm->allgather(dsend, drecv, sizeof mine, h.stream));
+  std::vector<cudaIpcMemHandle_t> all((size_t)kBlocks * D.world);
+  LV_CUDA(cudaMemcpyAsync(all.data(), drecv, sizeof mine * D.world, cudaMemcpyDeviceToHost, h.stream));
+  LV_CUDA(cudaStreamSynchronize(h.stream));
+  dfree(dsend, h.stream);
+  dfree(drecv, h.stream);
+  PeerPtrs hp[3];
+  std::memset(hp, 0, sizeof hp);
+  for (int q = 0; q < D.world; ++q) {
+    void* base[kBlocks];
+    for (int b = 0; b < kBlocks; ++b) {
+      if (q == D.rank) {
+        base[b] = blocks[b];
+      } else {
+        void* p = nullptr;
+        LV_CUDA(cudaIpcOpenMemHandle(&p, all[(size_t)q * kBlocks + b], cudaIpcMemLazyEnablePeerAccess));
+        D.opened.push_back(p);
+        base[b] = p;
+      }
+    }
+    for (int s = 0; s < 3; ++s) {
+      char* c = static_cast<char*>(base[s]);
+      hp[s].ca[q] = reinterpret_cast<uint2*>(c);
+      hp[s].size[q] = reinterpret_cast<int32_t*>(c + 8 * (size_t)D.rep_n);
+      hp[s].C[q] = reinterpret_cast<int32_t*>(c + 12 * (size_t)D.rep_n);
+      hp[s].pcn[q] = static_cast<uint2*>(base[3]);
+    }
+  }
+  for (int s = 0; s < 3; ++s) {
+    LV_CUDA(cudaMalloc(&D.d_peers[s], sizeof(PeerPtrs)));
+    LV_CUDA(cudaMemcpy(D.d_peers[s], &hp[s], sizeof(PeerPtrs), cudaMemcpyHostToDevice));
+  }
+  // level 0 of the handle lives in replica set 0 (its state is re-initialised there)
+  Level& L = h.lv;
+  dfree(L.ca, h.stream);
+  dfree(L.size, h.stream);
+  dfree(L.C, h.stream);
+  LV_TRY(dist_bind_state(h, L, 0));
+  L.k_ready = false;
+  LV_TRY(level_setup(h, L));
+  LV_CUDA(cudaStreamSynchronize(h.stream));
+  return dist_barrier(h);
+}
 
 int32_t dist_allreduce(Handle& h, unsigned long long* dev, size_t count) {
   if (!h.dist) return LOUVAIN_OK;
@@ -487,6 +662,7 @@ int32_t create_dist(Comm* comm, int64_t n, int64_t v_begin, int64_t v_end, const
   h.dist->world = world;
   h.dist->vlo0 = vlo;
   rc = set_range(h.lv, vlo[rank], vlo[rank + 1]);
+  if (!rc && (flags & LOUVAIN_DIST_P2P)) rc = setup_p2p(h, n);
   if (rc) {
     louvain_destroy(g);
     return rc;

@@ -349,7 +349,9 @@ int32_t sweep_body(Handle& h, Level& L, const louvain_params_t& p) {
     LV_TRY(launch_sweep_bucket(h, L, p, b));
     auto t1 = std::chrono::steady_clock::now();
     if (p.mode == LOUVAIN_MODE_BIN_SYNC) {
-      if (h.dist) LV_TRY(dist_exchange(h, L, commits, b));  // every rank's bucket-b moves
+      // every rank's bucket-b moves: all-gathered, or written into every replica by the
+      // peer-memory commit itself (LOUVAIN_DIST_P2P)
+      if (h.dist && !dist_p2p(h)) LV_TRY(dist_exchange(h, L, commits, b));
       LV_TRY(launch_commit(h, L, commits++));
     }
     if (trace) {
@@ -362,7 +364,7 @@ int32_t sweep_body(Handle& h, Level& L, const louvain_params_t& p) {
     }
   }
   if (p.mode == LOUVAIN_MODE_RELAXED) {
-    if (h.dist) LV_TRY(dist_exchange(h, L, 0, 0));
+    if (h.dist && !dist_p2p(h)) LV_TRY(dist_exchange(h, L, 0, 0));
     LV_TRY(launch_commit(h, L, commits++));
   }
   ++L.sweeps_done;
@@ -470,8 +472,9 @@ int32_t run_impl(Handle& h, const louvain_params_t& p, int32_t* labels_out, louv
   int32_t* const lab = R.lab;
   // labels at each sweep start, for the delta pass of Eq. (1) (LV_MOD_DELTA=0: full passes only)
   static const bool mod_delta = !(getenv("LV_MOD_DELTA") && getenv("LV_MOD_DELTA")[0] == '0');
-  if (mod_delta) LV_TRY(dalloc(&R.pcn, std::max<int64_t>(n0, 1), s));
-  uint2* const pcn = R.pcn;
+  if (mod_delta && !dist_p2p(h)) LV_TRY(dalloc(&R.pcn, std::max<int64_t>(n0, 1), s));
+  // peer-memory commits write the snapshot's "label now" of every rank: the shared block
+  uint2* const pcn = (mod_delta && dist_p2p(h)) ? static_cast<uint2*>(h.dist->pcn_block) : R.pcn;
   LV_CUDA(cudaEventCreate(&R.e0));
   LV_CUDA(cudaEventCreate(&R.e1));
   cudaEvent_t e_lvl0 = R.e0, e_lvl1 = R.e1;
@@ -509,6 +512,9 @@ int32_t run_impl(Handle& h, const louvain_params_t& p, int32_t* labels_out, louv
         cudaEventRecord(h.ev[0], s);
         h.pcn = pcn;
         if (mod_delta) LV_TRY(launch_snapshot(h, L));
+        // peer-memory commits: no rank may write into a replica before its owner has taken
+        // the sweep's snapshot (and finished the previous level's setup)
+        if (dist_p2p(h)) LV_TRY(dist_barrier(h));
         LV_TRY(sweep_body(h, L, p));
         cudaEventRecord(h.ev[1], s);
         tr.mark(s, "sweep", level);
@@ -517,6 +523,7 @@ int32_t run_impl(Handle& h, const louvain_params_t& p, int32_t* labels_out, louv
         if (h.dist) {  // the ranks' parts: overflow flags and L change (delta pass) / L (full pass)
           LV_TRY(dist_allreduce(h, &h.ctl->overflow, 2));
           if (!mod_delta) LV_TRY(dist_allreduce(h, &h.ctl->L, 1));
+          LV_TRY(dist_total_moved(h));
         }
         cudaEventRecord(h.ev[2], s);
         tr.mark(s, "modularity", level);
@@ -525,9 +532,11 @@ int32_t run_impl(Handle& h, const louvain_params_t& p, int32_t* labels_out, louv
         const float t_sw = elapsed(h.ev[0], h.ev[1]);
         local.t_sweep_ms_total += t_sw;
         local.t_modularity_ms_total += elapsed(h.ev[1], h.ev[2]);
+        // moves of the sweep (every rank's: peer-memory commits log only this rank's own)
+        const int64_t moved = h.dist ? (int64_t)h.h_ctl->gmoved : (int64_t)h.h_ctl->logn;
         if (level == 0 && sweeps == 0) {
           local.t_sweep_ms_first = t_sw;
-          local.moved_first = (int64_t)h.h_ctl->logn;
+          local.moved_first = moved;
         }
         if (level == 0 && sweeps < 32) local.t_sweep_ms_level0[sweeps] = t_sw;
         local.edges_swept += L.nnz;
@@ -536,7 +545,6 @@ int32_t run_impl(Handle& h, const louvain_params_t& p, int32_t* labels_out, louv
           set_error("partitioned hash table overflow (sweep_part); please report");
           return LOUVAIN_E_CUDA;
         }
-        const int64_t moved = (int64_t)h.h_ctl->logn;
         // Eq. (1) numerator of the swept partition: delta pass (L_before + dL, exact
         // modular arithmetic) or full pass
         const uint64_t L_after = (mod_delta && delta_chosen(*h.h_ctl, L.nnz)) ? Lq + h.h_ctl->dL : h.h_ctl->L;
@@ -869,6 +877,7 @@ LV_API int32_t louvain_sweep(louvain_graph_t g, const louvain_params_t* p, int64
   if (!rc && q_after) rc = launch_modularity(h, L, nullptr);
   if (!rc && q_after && h.dist) rc = dist_allreduce(h, &h.ctl->L, 1);
   if (!rc && h.dist) rc = dist_allreduce(h, &h.ctl->overflow, 1);
+  if (!rc && h.dist) rc = dist_total_moved(h);
   if (!rc) {
     cudaError_t e = cudaMemcpyAsync(h.h_ctl, h.ctl, sizeof(DevCtl), cudaMemcpyDeviceToHost, h.stream);
     if (e == cudaSuccess) e = cudaStreamSynchronize(h.stream);
@@ -879,7 +888,7 @@ LV_API int32_t louvain_sweep(louvain_graph_t g, const louvain_params_t* p, int64
     rc = LOUVAIN_E_CUDA;
   }
   if (!rc) {
-    if (moved) *moved = (int64_t)h.h_ctl->logn;
+    if (moved) *moved = (int64_t)(h.dist ? h.h_ctl->gmoved : h.h_ctl->logn);
     if (q_after) fill_q(q_after, h.h_ctl->L, h.h_ctl->S, L.W);
   }
   return finish_call(h, rc);

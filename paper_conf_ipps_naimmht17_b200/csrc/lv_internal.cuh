@@ -84,6 +84,7 @@ struct DevCtl {
   unsigned long long nbig;       // delta pass: moved vertices left to the block kernel
   unsigned long long nmid;       // delta pass: moved vertices left to the warp kernel
   unsigned long long ddiv;       // delta pass chosen iff mdeg * ddiv <= nnz
+  unsigned long long gmoved;     // distributed peer-memory commits: moves of all ranks in this sweep
 };
 
 // Hub work plan (one per level).  Hubs are grouped into waves whose tables fit
@@ -176,6 +177,10 @@ struct Level {
   int32_t* mv_old = nullptr;
   int32_t* mv_stamp = nullptr;  // sharded ABI only: sweep id of each vertex's last committed move
   int32_t stamp_id = 0;         // incremented by every louvain_begin_sweep
+  // distributed handle with peer-memory commits: ca / size / C live in the replica set
+  // `rep_set` of DistCtx (IPC-exported memory every rank writes into); not freed here
+  int rep_set = -1;
+  bool state_external = false;
   int32_t sweeps_done = 0;  // sweeps since the partition was last reset to singletons
   // sharded sweeps: owned vertex range (decisions, L) and its edge range
   int64_t own_lo = 0, own_hi = -1;  // own_hi < 0: all vertices
@@ -232,6 +237,14 @@ struct Handle {
 
 // ------------------------------------------------------------------ multi-GPU (lv_dist.cu)
 struct Comm;
+constexpr int kMaxWorld = 64;
+// Every rank's replica of one set of partition-state arrays (device-resident table).
+struct PeerPtrs {
+  uint2* ca[kMaxWorld];
+  int32_t* size[kMaxWorld];
+  int32_t* C[kMaxWorld];
+  uint2* pcn[kMaxWorld];
+};
 struct DistCtx {
   Comm* comm = nullptr;
   int rank = 0, world = 1;
@@ -241,6 +254,17 @@ struct DistCtx {
   int32_t* sbuf = nullptr;     // (v, new) pairs, 2 * max cap
   int32_t* rbuf = nullptr;     // world * that
   size_t sbuf_n = 0, rbuf_n = 0;
+  // LOUVAIN_DIST_P2P: the commit kernel writes every move into every rank's replica
+  // through peer memory (CUDA IPC mappings: NVLink P2P across GPUs, the same memory for
+  // ranks sharing one GPU) and a barrier ends each bucket -- no all-gather of moves.
+  // Replica sets: 0 = the handle's level 0, 1 / 2 = contracted levels of even / odd depth.
+  bool p2p = false;
+  int64_t rep_n = 0;                 // capacity (vertices) of every replica array
+  void* rep_block[3] = {nullptr, nullptr, nullptr};  // ca | size | C, cudaMalloc'ed (IPC)
+  void* pcn_block = nullptr;         // uint2[rep_n], cudaMalloc'ed (IPC)
+  std::vector<void*> opened;         // peers' blocks mapped into this process
+  PeerPtrs* d_peers[3] = {nullptr, nullptr, nullptr};  // device tables, one per set
+  unsigned long long* d_bar = nullptr;  // barrier operand
   ~DistCtx();
 };
 int32_t dist_set_level_range(Handle& h, Level& L, int level);  // own range of this rank at this level
@@ -251,6 +275,12 @@ int32_t dist_allreduce(Handle& h, unsigned long long* dev, size_t count);  // in
 int32_t dist_allgatherv(Handle& h, const void* send, void* recv, const std::vector<int64_t>& cnt,
                         const std::vector<int64_t>& displ, size_t elem);
 void dist_free(Handle& h);
+inline bool dist_p2p(const Handle& h) { return h.dist && h.dist->p2p; }
+int32_t dist_barrier(Handle& h);                                // all ranks' preceding work done
+int32_t dist_bind_state(Handle& h, Level& L, int set);          // L.ca / size / C -> replica set
+int32_t dist_commit_p2p(Handle& h, Level& L, int bucket);       // commit own moves into every replica
+int32_t dist_revert_p2p(Handle& h, Level& L);                   // undo own moves in every replica
+int32_t dist_total_moved(Handle& h);                            // ctl->gmoved = sum over ranks of logn
 
 // ------------------------------------------------------------------ launch accounting
 // Every explicit <<<>>> launch is followed by LV_LAUNCHED(); every device-wide

@@ -541,6 +541,9 @@ int32_t level_alloc_scratch(Handle& h, Level& L, int parity) {
   L.scratch_backed = true;
   L.parity = parity;
   L.owns_csr = false;
+  // peer-memory commits: the level's partition state lives in a replica set every rank
+  // writes into (odd depth -> set 2, even depth -> set 1; the handle's level 0 -> set 0)
+  if (dist_p2p(h)) LV_TRY(dist_bind_state(h, L, parity == 1 ? 2 : 1));
   return LOUVAIN_OK;
 }
 
@@ -557,7 +560,12 @@ void level_free(Level& L, cudaStream_t s) {
     dfree(L.col, s);
     dfree(L.w, s);
   }
-  dfree(L.k, s); dfree(L.ca, s); dfree(L.C, s); dfree(L.size, s);
+  dfree(L.k, s);
+  if (!L.state_external) {  // else: a replica set of the distributed handle (lv_dist.cu)
+    dfree(L.ca, s);
+    dfree(L.C, s);
+    dfree(L.size, s);
+  }
   dfree(L.mv_v, s); dfree(L.mv_new, s); dfree(L.mv_old, s); dfree(L.bin_vertices, s); dfree(L.mv_stamp, s);
   dfree(L.soff, s);  // L.stage lives in the handle's scratch
   hub_free(L.hub, s);
@@ -1049,6 +1057,7 @@ int32_t level_modularity(Handle& h, Level& L, const int32_t* d_C, uint64_t* Lout
 }
 
 int32_t launch_commit(Handle& h, Level& L, int bucket) {
+  if (dist_p2p(h)) return dist_commit_p2p(h, L, bucket);
   k_commit<<<148 * 4, 256, 0, h.stream>>>(h.ctl, bucket, L.mv_v, L.mv_new, L.mv_old, L.ca, L.size, L.k, L.C,
                                          (h.pcn && delta_div() > 1) ? L.rowptr : nullptr, h.pcn);
   LV_LAUNCHED();
@@ -1123,6 +1132,7 @@ int32_t unpack_moves(Handle& h, Level& L, int64_t c0, int64_t cnt, const int32_t
 }
 
 int32_t launch_revert(Handle& h, Level& L) {
+  if (dist_p2p(h)) return dist_revert_p2p(h, L);
   k_revert<<<148 * 4, 256, 0, h.stream>>>(h.ctl, L.mv_v, L.mv_new, L.mv_old, L.ca, L.size, L.k, L.C);
   LV_LAUNCHED();
   LV_CUDA(cudaGetLastError());

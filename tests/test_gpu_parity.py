@@ -328,12 +328,12 @@ def test_generators_host_device_bit_identical(maker, args):
 DIST_GRAPHS = ("karate", "rmat15", "hubs", "giant_hub", "weighted_loops", "lfr5k")
 
 
-def _dist_run(g, rank, world, comm, mode):
+def _dist_run(g, rank, world, comm, mode, p2p=False):
     import paper_conf_ipps_naimmht17_b200 as lvb2
     from paper_conf_ipps_naimmht17_b200.dist import edge_balanced_ranges, local_rows
     lo, hi = edge_balanced_ranges(g.rowptr, world)[rank]
     rl, cl, wl = local_rows(g.rowptr, g.col, g.w, lo, hi)
-    with lvb2.Graph.from_csr_dist(g.n, lo, hi, rl, cl, wl, rank=rank, world=world, comm=comm) as gd:
+    with lvb2.Graph.from_csr_dist(g.n, lo, hi, rl, cl, wl, rank=rank, world=world, comm=comm, p2p=p2p) as gd:
         lab, q, st = gd.run(lvb2.params(mode=mode))
         gd.set_labels(None)
         moved, q1 = gd.sweep(lvb2.params(mode=mode))  # one collective louvain_sweep from singletons
@@ -342,14 +342,14 @@ def _dist_run(g, rank, world, comm, mode):
         (moved, int(q1.L), q1.S, lab1.tolist())
 
 
-def _dist_worker(rank, world, port, mode, q):
+def _dist_worker(rank, world, port, mode, p2p, q):
     import os
     import torch.distributed as dist
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
     dist.init_process_group("gloo", rank=rank, world_size=world)
     try:
-        q.put((rank, {name: _dist_run(GRAPHS[name](), rank, world, "host", mode) for name in DIST_GRAPHS}))
+        q.put((rank, {name: _dist_run(GRAPHS[name](), rank, world, "host", mode, p2p) for name in DIST_GRAPHS}))
     finally:
         dist.destroy_process_group()
 
@@ -385,11 +385,13 @@ def test_dist_handle_nccl_world1_matches_oracle():
         dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("world,mode", [(2, 0), (3, 0), (2, 1)])
-def test_dist_handle_ranks_share_one_gpu_match_oracle(world, mode):
+@pytest.mark.parametrize("world,mode,p2p", [(2, 0, False), (3, 0, False), (2, 1, False), (2, 0, True), (3, 0, True),
+                                            (2, 1, True)])
+def test_dist_handle_ranks_share_one_gpu_match_oracle(world, mode, p2p):
     """world processes share the GPU (host transport over gloo): every rank decides its own
-    edge-balanced rows with the CUDA kernels, the library exchanges the moves of each bucket
-    and every rank commits all of them -- bit-identical to oracle (b) on every rank."""
+    edge-balanced rows with the CUDA kernels; the library all-gathers the moves of each bucket
+    and every rank commits all of them, or (p2p) every rank's commit kernel writes its moves
+    into all ranks' replicas through CUDA IPC mappings -- bit-identical to oracle (b)."""
     import socket
     import torch.multiprocessing as tmp
     sk = socket.socket()
@@ -398,7 +400,7 @@ def test_dist_handle_ranks_share_one_gpu_match_oracle(world, mode):
     sk.close()
     ctx = tmp.get_context("spawn")
     q = ctx.Queue()
-    procs = [ctx.Process(target=_dist_worker, args=(r, world, port, mode, q)) for r in range(world)]
+    procs = [ctx.Process(target=_dist_worker, args=(r, world, port, mode, p2p, q)) for r in range(world)]
     for pr in procs:
         pr.start()
     res = dict(q.get(timeout=900) for _ in range(world))
