@@ -366,6 +366,9 @@ int32_t dist_bind_state(Handle& h, Level& L, int set) {
 
 int32_t dist_commit_p2p(Handle& h, Level& L, int bucket) {
   DistCtx& D = *h.dist;
+  // every rank has decided the bucket against the same snapshot before any rank
+  // writes into another's replica (Alg. 1 l.6-9: the commit follows all decisions)
+  LV_TRY(dist_barrier(h));
   k_commit_p2p<<<148 * 4, 256, 0, h.stream>>>(h.ctl, bucket, L.mv_v, L.mv_new, L.mv_old, D.d_peers[L.rep_set],
                                              D.world, D.rank, L.k, h.pcn != nullptr);
   LV_LAUNCHED();
@@ -375,6 +378,7 @@ int32_t dist_commit_p2p(Handle& h, Level& L, int bucket) {
 
 int32_t dist_revert_p2p(Handle& h, Level& L) {
   DistCtx& D = *h.dist;
+  LV_TRY(dist_barrier(h));
   k_revert_p2p<<<148 * 4, 256, 0, h.stream>>>(h.ctl, L.mv_v, L.mv_new, L.mv_old, D.d_peers[L.rep_set], D.world, L.k);
   LV_LAUNCHED();
   LV_CUDA(cudaGetLastError());
