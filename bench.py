@@ -60,6 +60,8 @@ def parse_args():
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--e2e-warmup", type=int, default=1)
     ap.add_argument("--backend", default="nccl", help="process-group backend for N > 1 (gloo: tests only)")
+    ap.add_argument("--exchange", choices=["allgather", "p2p"], default="allgather",
+                    help="N > 1: per-bucket all-gather of moves, or peer-memory commits (LOUVAIN_DIST_P2P)")
     ap.add_argument("--cpu-seconds", type=float, default=15.0, help="oracle sample budget")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     return ap.parse_args()
@@ -330,8 +332,9 @@ def run_sharded_bench(args, rank, world):
     lo, hi = edge_balanced_ranges(dg.rowptr.cpu().numpy(), world)[rank]
     rl, cl, _ = local_rows(dg.rowptr, dg.col, None, lo, hi)
     stream = torch.cuda.Stream()
+    p2p = args.exchange == "p2p"
     g = lvb.Graph.from_csr_dist(n, lo, hi, rl.contiguous(), cl.contiguous(), None, rank=rank, world=world,
-                                comm=comm, stream=stream)
+                                comm=comm, p2p=p2p, stream=stream)
     labels_dev = torch.empty(n, dtype=torch.int32, device=dev)
 
     def one_run():
@@ -373,7 +376,8 @@ def run_sharded_bench(args, rank, world):
         dist.barrier()
         torch.cuda.synchronize()
         t0 = time.perf_counter()
-        with lvb.Graph.from_csr_dist(n, lo, hi, h_rl, h_cl, None, rank=rank, world=world, comm=comm) as ge:
+        with lvb.Graph.from_csr_dist(n, lo, hi, h_rl, h_cl, None, rank=rank, world=world, comm=comm,
+                                     p2p=p2p) as ge:
             ge.run(p, labels_out=h_lab)
         torch.cuda.synchronize()
         if it >= max(0, args.e2e_warmup):
@@ -385,9 +389,10 @@ def run_sharded_bench(args, rank, world):
            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
            "scaling": "strong", "vs_baseline": None, "dtype": "int64", "data": "synthetic",
            "config": dict(workload(args, n, nnz), l2="inputs larger than L2",
-                          parallelism=f"{world} GPUs, sweep vertex-sharded (edge-balanced ranges), per-bucket "
-                                      f"{'NCCL' if comm == 'nccl' else 'host-staged'} all-gather of moves, "
-                                      "per-sweep all-reduce of the L change"),
+                          parallelism=f"{world} GPUs, sweep vertex-sharded (edge-balanced ranges), per bucket "
+                                      + ("peer-memory commits into every replica + barrier" if p2p else
+                                         f"{'NCCL' if comm == 'nccl' else 'host-staged'} all-gather of moves")
+                                      + ", per-sweep all-reduce of the L change, contraction sharded by new vertex"),
            "roofline": roofline, "clocks": clk.summary(), "gpu_launches": int(launches),
            "q_final": st0["q"], "levels": st0["levels"],
            "sweeps_per_level": st0["sweeps_per_level"], "louvain_wall_ms": ms_per_step,
