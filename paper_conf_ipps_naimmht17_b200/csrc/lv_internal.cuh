@@ -231,6 +231,11 @@ struct Handle {
   // louvain_run only: {label at the sweep start, label after} per vertex; the
   // commit writes .y of every moved vertex (delta pass of Eq. (1))
   uint2* pcn = nullptr;
+  // delta pass of Eq. (1): lists of long moved rows (grow-only, reused by every sweep so a
+  // captured sweep graph allocates nothing)
+  int32_t* dl_big = nullptr;
+  int32_t* dl_mid = nullptr;
+  size_t dl_big_n = 0, dl_mid_n = 0;
   // distributed handle (louvain_create_csr_dist*): nullptr on one GPU
   struct DistCtx* dist = nullptr;
 };

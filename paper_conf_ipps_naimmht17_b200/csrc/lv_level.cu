@@ -1013,9 +1013,22 @@ int32_t launch_modularity_delta(Handle& h, Level& L) {
   LV_CUDA(cudaMemsetAsync(&h.ctl->dL, 0, 24, s));
   LV_TRY(set_ctl_u64(h, &h.ctl->ddiv, delta_div()));
   if (L.n == 0) return LOUVAIN_OK;
-  int32_t *big = nullptr, *mid = nullptr;
-  LV_TRY(dalloc(&big, (size_t)(L.nnz / kDeltaBigDeg + 1), s));
-  LV_TRY(dalloc(&mid, (size_t)(L.nnz / kDeltaThrDeg + 1), s));
+  const size_t nbig = (size_t)(L.nnz / kDeltaBigDeg + 1), nmid = (size_t)(L.nnz / kDeltaThrDeg + 1);
+  if (h.dl_big_n < nbig) {
+    dfree(h.dl_big, s);
+    h.dl_big = nullptr;
+    h.dl_big_n = 0;
+    LV_TRY(dalloc(&h.dl_big, nbig, s));
+    h.dl_big_n = nbig;
+  }
+  if (h.dl_mid_n < nmid) {
+    dfree(h.dl_mid, s);
+    h.dl_mid = nullptr;
+    h.dl_mid_n = 0;
+    LV_TRY(dalloc(&h.dl_mid, nmid, s));
+    h.dl_mid_n = nmid;
+  }
+  int32_t *big = h.dl_big, *mid = h.dl_mid;
   // a distributed handle sums the moved rows it owns (the ranks' parts are all-reduced)
   const int64_t own_lo = (h.dist && L.own_hi >= 0) ? L.own_lo : 0;
   const int64_t own_hi = (h.dist && L.own_hi >= 0) ? L.own_hi : L.n;
@@ -1028,8 +1041,6 @@ int32_t launch_modularity_delta(Handle& h, Level& L) {
   k_mod_delta_cta<<<148 * 4, 512, 0, s>>>(h.ctl, big, L.mv_v, L.mv_new, L.mv_old, L.rowptr, L.col, L.w, P,
                                           L.nnz, L.ca, L.n);
   LV_LAUNCHED();
-  dfree(big, s);
-  dfree(mid, s);
   // full pass, skipped on the device when the delta pass was chosen
   const int64_t ntiles = (L.nnz + kTileEdges - 1) / kTileEdges;
   const unsigned grid = grid_for(std::max<int64_t>(ntiles, (L.n + 255) / 256), 1, 148 * 8);
