@@ -66,7 +66,6 @@ struct SweepArgs {
   const int32_t* size;
   long long W;
   int rule;
-  bool b4;  // bucketised claim tables (table_insert_b4)
   int32_t* mv_v;
   int32_t* mv_new;
   unsigned long long* logn;
@@ -469,66 +468,10 @@ __device__ __forceinline__ uint32_t table_insert_c(unsigned long long* T, uint32
   }
 }
 
-// Bucketised variant (cap a multiple of 4): a label probes 4-slot buckets (32 B, two
-// 16-byte shared loads per round) instead of single slots -- it adds to the slot holding
-// its label, or CASes the first empty slot of the first bucket with room (a failed CAS
-// re-reads the same bucket).  Slots only go EMPTY -> key once and a key is only claimed at
-// the first empty slot of its probe sequence, so no label is ever stored twice.  At load
-// 1/2 nearly every insert resolves in its first bucket: fewer divergent probe rounds than
-// single-slot linear probing (ncu: the probe loop ran at 4-9 active lanes).
-// 16-byte shared-memory load that is re-issued on every call (the bucket is re-read after
-// a lost CAS)
-__device__ __forceinline__ ulonglong2 lds128_volatile(const unsigned long long* p) {
-  ulonglong2 r;
-  const unsigned a = (unsigned)__cvta_generic_to_shared(p);
-  asm volatile("ld.volatile.shared.v2.u64 {%0, %1}, [%2];" : "=l"(r.x), "=l"(r.y) : "r"(a) : "memory");
-  return r;
-}
-__device__ __forceinline__ uint32_t table_insert_b4(unsigned long long* T, uint32_t cap, int32_t c, uint32_t x,
-                                                    bool* claimed) {
-  const unsigned long long key = ((unsigned long long)(uint32_t)c) << 32;
-  uint32_t b = hash_slot(c, cap >> 2) << 2;
-  for (;;) {
-    const ulonglong2 lo = lds128_volatile(&T[b]);
-    const ulonglong2 hi = lds128_volatile(&T[b + 2]);
-    const unsigned long long k[4] = {lo.x, lo.y, hi.x, hi.y};
-    int tgt = -1;
-    bool found = false;
-#pragma unroll
-    for (int u = 3; u >= 0; --u)
-      if (k[u] == kEmpty) tgt = u;
-#pragma unroll
-    for (int u = 3; u >= 0; --u)
-      if (k[u] != kEmpty && (k[u] >> 32) == (unsigned long long)(uint32_t)c) {
-        tgt = u;
-        found = true;
-      }
-    if (found) {
-      atomicAdd(&T[b + tgt], (unsigned long long)x);
-      *claimed = false;
-      return b + tgt;
-    }
-    if (tgt >= 0) {
-      const unsigned long long old = atomicCAS(&T[b + tgt], kEmpty, key | x);
-      if (old == kEmpty) {
-        *claimed = true;
-        return b + tgt;
-      }
-      if ((old >> 32) == (unsigned long long)(uint32_t)c) {
-        atomicAdd(&T[b + tgt], (unsigned long long)x);
-        *claimed = false;
-        return b + tgt;
-      }
-      continue;  // another label took the slot: re-read the bucket
-    }
-    b = (b + 4 >= cap) ? 0u : b + 4;  // bucket full
-  }
-}
 template <bool UNIT, int PASSES>
 __device__ __forceinline__ void insert_claim(unsigned long long* T, uint32_t* TA, uint32_t cap,
                                              const uint2* __restrict__ S, const uint32_t* __restrict__ Wt,
-                                             int64_t deg, int t0, int stride, uint32_t (&cl)[4 * PASSES],
-                                             bool A_b4) {
+                                             int64_t deg, int t0, int stride, uint32_t (&cl)[4 * PASSES]) {
 #pragma unroll
   for (int pass = 0; pass < PASSES; ++pass) {
     uint2 rr[4];
@@ -544,8 +487,7 @@ __device__ __forceinline__ void insert_claim(unsigned long long* T, uint32_t* TA
       uint32_t slot = kNoClaim;
       if (rr[q].x != kSelf) {
         bool claimed = false;
-        const uint32_t hq = A_b4 ? table_insert_b4(T, cap, (int32_t)rr[q].x, ww[q], &claimed)
-                                 : table_insert_c(T, cap, (int32_t)rr[q].x, ww[q], &claimed);
+        const uint32_t hq = table_insert_c(T, cap, (int32_t)rr[q].x, ww[q], &claimed);
         if (rr[q].y != kUnknownA) TA[hq] = rr[q].y;
         if (claimed) slot = hq;
       }
@@ -615,8 +557,7 @@ __device__ __forceinline__ void insert_claim_direct(unsigned long long* T, uint3
     uint32_t slot = kNoClaim;
     if (rr[u].x != kSelf) {
       bool claimed = false;
-      const uint32_t hq = A.b4 ? table_insert_b4(T, cap, (int32_t)rr[u].x, ww[u], &claimed)
-                               : table_insert_c(T, cap, (int32_t)rr[u].x, ww[u], &claimed);
+      const uint32_t hq = table_insert_c(T, cap, (int32_t)rr[u].x, ww[u], &claimed);
       if (rr[u].x == (uint32_t)jj[u]) TA[hq] = rr[u].y;  // the neighbour represents its label
       if (claimed) slot = hq;
     }
@@ -684,8 +625,7 @@ __global__ void __launch_bounds__(32 * WARPS) sweep_warp_c(const int32_t* __rest
     const int32_t own = (int32_t)__ldg(&A.ca[v]).x;
     const uint32_t ki = __ldg(&A.k[v]);
     uint32_t cl[4 * PASSES];
-    insert_claim<UNIT, PASSES>(T, TA, CAP, stage + __ldg(&soff[vi]), UNIT ? nullptr : A.w + rb, deg, lane, 32, cl,
-                               A.b4);
+    insert_claim<UNIT, PASSES>(T, TA, CAP, stage + __ldg(&soff[vi]), UNIT ? nullptr : A.w + rb, deg, lane, 32, cl);
     __syncwarp();
     const bool own_single = A.rule == 2 && __ldg(&A.size[own]) == 1;
     long long s = (long long)0x8000000000000000ull;
@@ -722,11 +662,11 @@ __global__ void __launch_bounds__(1024) sweep_cta_c(const int32_t* __restrict__ 
     const int64_t deg = __ldg(&A.rowptr[v + 1]) - rb;
     const int32_t own = (int32_t)__ldg(&A.ca[v]).x;
     const uint32_t ki = __ldg(&A.k[v]);
-    const int64_t want = ((2 * deg + 1) + 3) & ~(int64_t)3;  // load <= 1/2, whole 4-slot buckets
+    const int64_t want = 2 * deg + 1;  // load <= 1/2
     const uint32_t cap = (uint32_t)(want < (int64_t)capmax ? want : (int64_t)capmax);
     uint32_t cl[4 * PASSES];
     insert_claim<UNIT, PASSES>(T, TA, cap, stage + __ldg(&soff[vi]), UNIT ? nullptr : A.w + rb, deg, threadIdx.x,
-                               blockDim.x, cl, A.b4);
+                               blockDim.x, cl);
     __syncthreads();
     const bool own_single = A.rule == 2 && __ldg(&A.size[own]) == 1;
     long long s = (long long)0x8000000000000000ull;
@@ -1429,11 +1369,6 @@ int32_t launch_part(Handle& h, Level& L, const SweepArgs& A, int bucket, bool un
 // the fixed 512-slot warp tables of bucket 6 (C5 level 0: 10.2 -> 6.3 ms per 2
 // sweeps).  The CTA tables are sized 2*deg, where the list measured slower
 // (b7 [1024,2048): 12.5 -> 19.4 ms), and so was the 128-slot warp table of bucket 5.
-// bucketised claim tables (LV_B4=0: single-slot linear probing; A/B)
-static bool b4_on() {
-  static const bool on = !(getenv("LV_B4") && getenv("LV_B4")[0] == '0');
-  return on;
-}
 // Rows of <= kDirectMaxDeg entries (bucket 5 with the paper's bounds) are hashed by a warp
 // that gathers the records itself (sweep_warp_d): C5 level 0 bucket 5 stage 2.8 + warp 2.2 ->
 // 4.0 ms; bucket 6 (85-319) measured slower that way (6.5 -> 7.6 ms) and keeps the stage.
@@ -1561,7 +1496,6 @@ int32_t launch_sweep_bucket(Handle& h, Level& L, const louvain_params_t& p, int 
   A.size = L.size;
   A.W = (long long)L.W;
   A.rule = p.singleton_rule;
-  A.b4 = b4_on();
   A.mv_v = L.mv_v;
   A.mv_new = L.mv_new;
   A.logn = &h.ctl->logn;
