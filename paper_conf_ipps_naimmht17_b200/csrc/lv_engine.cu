@@ -426,12 +426,6 @@ float elapsed(cudaEvent_t a, cudaEvent_t b) {
   return ms;
 }
 
-// Sweeps replayed as captured CUDA graphs from a level's second sweep on (LV_GRAPHS=0: off)
-bool graphs_on() {
-  static const bool on = !(getenv("LV_GRAPHS") && getenv("LV_GRAPHS")[0] == '0');
-  return on;
-}
-
 // Eq. (1) parts of the level's own partition; on a distributed handle each rank
 // sums the entries of its rows and L is all-reduced (S from the replicated a_c).
 int32_t modularity_parts(Handle& h, Level& L, bool singletons, uint64_t* Lout, uint64_t* Sout) {
@@ -467,15 +461,8 @@ int32_t run_impl(Handle& h, const louvain_params_t& p, int32_t* labels_out, louv
     Level owned;             // current contracted level (levels >= 1)
     bool has_owned = false;
     cudaEvent_t e0 = nullptr, e1 = nullptr;
-    cudaGraphExec_t gx = nullptr;  // the current level's captured sweep
-    long long gx_launches = 0;
     explicit RunRes(Handle& hh) : h(hh) {}
-    void drop_graph() {
-      if (gx) cudaGraphExecDestroy(gx);
-      gx = nullptr;
-    }
     ~RunRes() {
-      drop_graph();
       h.pcn = nullptr;
       dfree(lab, h.stream);
       dfree(pcn, h.stream);
@@ -524,12 +511,6 @@ int32_t run_impl(Handle& h, const louvain_params_t& p, int32_t* labels_out, louv
       int64_t num_prev = num_start;
       int64_t moved_level = 0;
       int32_t sweeps = 0;
-      // From the level's second sweep on, a sweep (snapshot, bucket kernels and commits,
-      // Eq. (1) pass) is replayed as one captured CUDA graph: the same launches without the
-      // per-launch host overhead (small levels are launch-bound).  Not for levels with hub
-      // plans (host round trips) nor distributed handles (host-side collectives).
-      const bool graphable = graphs_on() && !h.dist && !tr.on && L.part.nverts == 0 && L.hub.nh == 0;
-      bool graph_failed = false;
       auto sweep_once = [&]() -> int32_t {
         LV_CUDA(cudaEventRecord(h.ev[0], s));
         if (mod_delta) LV_TRY(launch_snapshot(h, L));
@@ -553,34 +534,7 @@ int32_t run_impl(Handle& h, const louvain_params_t& p, int32_t* labels_out, louv
       for (;;) {
         if (p.max_sweeps > 0 && sweeps >= p.max_sweeps) break;
         h.pcn = pcn;
-        bool done = false;
-        if (graphable && sweeps >= 1 && !graph_failed) {
-          if (!R.gx) {
-            const long long l0 = g_launches;
-            LV_CUDA(cudaStreamBeginCapture(s, cudaStreamCaptureModeThreadLocal));
-            const int32_t rc = sweep_once();
-            const long long nk = g_launches - l0;  // kernels one replay launches
-            cudaGraph_t gr = nullptr;
-            const cudaError_t ce = cudaStreamEndCapture(s, &gr);
-            cudaError_t ie = cudaErrorUnknown;
-            if (rc == LOUVAIN_OK && ce == cudaSuccess) ie = cudaGraphInstantiate(&R.gx, gr, 0);
-            if (gr) cudaGraphDestroy(gr);
-            g_launches = l0;
-            if (ie != cudaSuccess) {  // not capturable here: run this level's sweeps as plain launches
-              cudaGetLastError();
-              R.gx = nullptr;
-              graph_failed = true;
-            } else {
-              R.gx_launches = nk;
-            }
-          }
-          if (R.gx) {
-            LV_CUDA(cudaGraphLaunch(R.gx, s));
-            g_launches += R.gx_launches;
-            done = true;
-          }
-        }
-        if (!done) LV_TRY(sweep_once());
+        LV_TRY(sweep_once());
         LV_CUDA(cudaMemcpyAsync(h.h_ctl, h.ctl, sizeof(DevCtl), cudaMemcpyDeviceToHost, s));
         LV_CUDA(cudaStreamSynchronize(s));
         const float t_sw = elapsed(h.ev[0], h.ev[1]);
@@ -618,7 +572,6 @@ int32_t run_impl(Handle& h, const louvain_params_t& p, int32_t* labels_out, louv
         if (moved == 0 || below_threshold(num, num_prev, W, pexp)) break;  // Alg. 1 l.12, R13
         num_prev = num;
       }
-      R.drop_graph();  // the next level has other arrays
       const int64_t num_end = qnum_of(Lq, Sq, W);  // the partition kept at the end of the phase
       cudaEventRecord(e_lvl1, s);
       local.n[level] = L.n;

@@ -448,10 +448,8 @@ def _alt_path_worker(env_items, names, q):
     # delta pass gated on moved entries <= nnz / 4: the device-side choice between
     # the delta and the full pass, and the moved-degree sum in k_commit
     (("LV_DELTA_DIV", "4"),),
-    # serialised per-class timing (no side stream for the hub classes, no sweep graphs)
+    # serialised per-class timing (no side stream for the hub classes)
     (("LV_TRACE", "2"),),
-    # every sweep as plain launches (no captured CUDA graphs from a level's second sweep on)
-    (("LV_GRAPHS", "0"),),
 ])
 def test_alternative_paths_match_oracle(env):
     import torch.multiprocessing as tmp
