@@ -508,13 +508,6 @@ __global__ void __launch_bounds__(THREADS) k_big_combine(const uint32_t* __restr
   }
 }
 
-// Lengths of the big segments (the scan turns them into key-array offsets).
-__global__ void k_big_len(const int32_t* __restrict__ rows, int64_t nbig, const int64_t* __restrict__ sstart,
-                          int64_t* len) {
-  for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k <= nbig; k += (int64_t)gridDim.x * blockDim.x)
-    len[k] = (k < nbig) ? sstart[rows[k] + 1] - sstart[rows[k]] : 0;
-}
-
 // Tiled key build: tile plan btr gives the first big segment of every
 // kBigTile-entry tile; the tile's segment offsets are staged in smem.
 constexpr int kBigTile = 8192;
@@ -567,6 +560,200 @@ __global__ void __launch_bounds__(256) k_big_keys_t(const int32_t* __restrict__ 
         vals[t] = wv;
       }
     }
+  }
+}
+
+// Step 4d (default for big segments whose keys do not fit the 32-bit combiner):
+// mergeCommunity by label partitions instead of a sort.  Big segment k of
+// length L_k is split into P_k = ceil(L_k / kBigPE) partitions by part_of(neighbour,
+// P_k): every copy of a neighbour lands in the same partition, so merging each
+// partition on its own gives exactly the merged row.  Histogram and scatter run
+// edge-parallel over the big entries (the tile plan of k_big_keys_t); the 32 entries
+// of a warp fall into few partitions (P_k is small for most big segments), so one
+// global atomic per warp and partition run.  Then one CTA per partition folds its
+// entries in a shared-memory table and appends the distinct (neighbour, sum) pairs to
+// the segment's output range from a claim list (no table scan).  Expected distinct
+// neighbours per partition <= kBigPE in a table of 2 * kBigPE slots; a table that
+// fills up raises *overflow and the level redoes its big segments with the sort path
+// (deterministic either way).
+constexpr int kBigPE = 8192;
+constexpr int kBigPSlots = 16384;
+
+__global__ void k_bigp_sizes(const int32_t* __restrict__ rows, int64_t nbig, const int64_t* __restrict__ sstart,
+                             int64_t* len, int64_t* nparts) {
+  for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k <= nbig; k += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t l = (k < nbig) ? sstart[rows[k] + 1] - sstart[rows[k]] : 0;
+    len[k] = l;
+    nparts[k] = (l + kBigPE - 1) / kBigPE;
+  }
+}
+
+template <bool SCATTER>
+__global__ void __launch_bounds__(256) k_bigp_pass(const int32_t* __restrict__ rows, int64_t nbig,
+                                                   const int64_t* __restrict__ sstart,
+                                                   const int64_t* __restrict__ boff, const int64_t* __restrict__ btr,
+                                                   int64_t m, const int32_t* __restrict__ gc,
+                                                   const uint32_t* __restrict__ gw, const int64_t* __restrict__ pbase,
+                                                   unsigned long long* __restrict__ pcnt, int32_t* __restrict__ pc,
+                                                   uint32_t* __restrict__ pw) {
+  __shared__ int64_t sh_b[kBigTileSegs + 1];
+  __shared__ int64_t sh_src[kBigTileSegs];
+  __shared__ int64_t sh_pb[kBigTileSegs + 1];
+  const int lane = threadIdx.x & 31;
+  const int64_t ntiles = (m + kBigTile - 1) / kBigTile;
+  for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
+    const int64_t t0 = tile * kBigTile, t1 = min(m, t0 + kBigTile);
+    const int64_t k0 = btr[tile], k1 = btr[tile + 1];
+    const int ns = (k1 - k0 + 1 <= kBigTileSegs) ? (int)(k1 - k0 + 1) : -1;
+    __syncthreads();
+    for (int r = threadIdx.x; r < ns; r += blockDim.x) {
+      sh_b[r] = boff[k0 + r];
+      sh_src[r] = sstart[rows[k0 + r]];
+      sh_pb[r] = pbase[k0 + r];
+    }
+    if (ns > 0 && threadIdx.x == 0) sh_pb[ns] = pbase[min(k0 + ns, nbig)];
+    __syncthreads();
+    for (int64_t tb = t0 + threadIdx.x - lane; tb < t1; tb += blockDim.x) {  // warp-uniform trips
+      const int64_t t = tb + lane;
+      const bool active = t < t1;
+      uint32_t gb = 0xFFFFFFFFu;
+      int32_t c = 0;
+      uint32_t x = 1u;
+      if (active) {
+        int64_t src, p0, p1;
+        if (ns > 0) {
+          int lo = 0, hi = ns - 1;
+          while (lo < hi) {
+            const int mid = (lo + hi + 1) >> 1;
+            if (sh_b[mid] <= t) lo = mid; else hi = mid - 1;
+          }
+          src = sh_src[lo] + (t - sh_b[lo]);
+          p0 = sh_pb[lo];
+          p1 = sh_pb[lo + 1];
+        } else {
+          int64_t lo = k0, hi = min(k1, nbig - 1);
+          while (lo < hi) {
+            const int64_t mid = (lo + hi + 1) >> 1;
+            if (boff[mid] <= t) lo = mid; else hi = mid - 1;
+          }
+          src = sstart[rows[lo]] + (t - boff[lo]);
+          p0 = pbase[lo];
+          p1 = pbase[lo + 1];
+        }
+        c = __ldcs(&gc[src]);
+        if (SCATTER && gw) x = __ldcs(&gw[src]);
+        gb = (uint32_t)p0 + part_of(c, (uint32_t)(p1 - p0));
+      }
+      const unsigned mm = __match_any_sync(kFull, gb);
+      const int leader = __ffs(mm) - 1;
+      if (!SCATTER) {
+        if (active && lane == leader) atomicAdd(&pcnt[gb], (unsigned long long)__popc(mm));
+      } else {
+        unsigned long long b = 0;
+        if (active && lane == leader) b = atomicAdd(&pcnt[gb], (unsigned long long)__popc(mm));
+        b = __shfl_sync(kFull, b, leader);
+        if (active) {
+          const unsigned long long dst = b + __popc(mm & ((1u << lane) - 1u));
+          __stcs(&pc[dst], c);
+          if (gw) __stcs(&pw[dst], x);
+        }
+      }
+    }
+  }
+}
+
+// One CTA per partition (persistent): fold, then append the distinct pairs.
+__global__ void __launch_bounds__(1024) k_bigp_merge(const int64_t* __restrict__ poff, int64_t nparts,
+                                                     const int64_t* __restrict__ pbase, int64_t nbig,
+                                                     const int32_t* __restrict__ rows,
+                                                     const int64_t* __restrict__ sstart,
+                                                     const int32_t* __restrict__ pc, const uint32_t* __restrict__ pw,
+                                                     int32_t* oc, uint32_t* ow, int64_t* cnt,
+                                                     unsigned long long* overflow, uint32_t capmax) {
+  extern __shared__ unsigned long long T[];                            // kBigPSlots slots
+  uint16_t* claim = reinterpret_cast<uint16_t*>(T + kBigPSlots);      // claimed slots, in claim order
+  __shared__ unsigned ncl;
+  __shared__ long long sh_base;
+  __shared__ int32_t sh_r;
+  const int lane = threadIdx.x & 31;
+  for (int t = threadIdx.x; t < kBigPSlots; t += blockDim.x) T[t] = kEmpty;
+  for (int64_t g = blockIdx.x; g < nparts; g += gridDim.x) {
+    const int64_t q0 = poff[g], q1 = poff[g + 1];
+    const int64_t len = q1 - q0;
+    if (len == 0) continue;  // uniform across the CTA
+    uint32_t cap = 64;
+    while (cap < capmax && (int64_t)cap < 2 * len) cap <<= 1;
+    if (threadIdx.x == 0) {
+      int64_t lo = 0, hi = nbig - 1;  // segment of partition g: last k with pbase[k] <= g
+      while (lo < hi) {
+        const int64_t mid = (lo + hi + 1) >> 1;
+        if (pbase[mid] <= g) lo = mid; else hi = mid - 1;
+      }
+      sh_r = rows[lo];
+      ncl = 0;
+    }
+    __syncthreads();
+    for (int64_t tb = q0 + threadIdx.x - lane; tb < q1; tb += 4 * (int64_t)blockDim.x) {  // warp-uniform trips
+      int32_t cc[4];
+      uint32_t xx[4];
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        const int64_t t = tb + lane + (int64_t)u * blockDim.x;
+        const bool has = t < q1;
+        cc[u] = has ? __ldcs(&pc[t]) : (int32_t)(0x80000000u | (unsigned)lane);
+        xx[u] = has ? (pw ? __ldcs(&pw[t]) : 1u) : 0u;
+      }
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        const bool has = cc[u] >= 0;
+        unsigned mm = 1u << lane;
+        uint32_t x = xx[u];
+        if (__any_sync(kFull, cc[u] == __shfl_xor_sync(kFull, cc[u], 1))) {  // adaptive merge of repeats
+          mm = __match_any_sync(kFull, cc[u]);
+          x = __reduce_add_sync(mm, xx[u]);
+        }
+        uint32_t h = 0xFFFFFFFFu;
+        if (has && lane == __ffs(mm) - 1) {
+          const unsigned long long key = ((unsigned long long)(uint32_t)cc[u]) << 32;
+          h = hash_slot(cc[u], cap);
+          for (uint32_t probes = 0;; ++probes) {
+            if (probes >= cap) {
+              atomicExch(overflow, 1ull);
+              h = 0xFFFFFFFFu;
+              break;
+            }
+            const unsigned long long old = atomicCAS(&T[h], kEmpty, key | x);
+            if (old == kEmpty) break;  // claimed: h goes on the claim list
+            if ((old >> 32) == (unsigned long long)(uint32_t)cc[u]) {
+              atomicAdd(&T[h], (unsigned long long)x);
+              h = 0xFFFFFFFFu;
+              break;
+            }
+            h = (h + 1 == cap) ? 0 : h + 1;
+          }
+        }
+        const unsigned cm = __ballot_sync(kFull, h != 0xFFFFFFFFu);
+        if (cm) {
+          unsigned b = 0;
+          if (lane == __ffs(cm) - 1) b = atomicAdd(&ncl, (unsigned)__popc(cm));
+          b = __shfl_sync(kFull, b, __ffs(cm) - 1);
+          if (h != 0xFFFFFFFFu) claim[b + __popc(cm & ((1u << lane) - 1u))] = (uint16_t)h;
+        }
+      }
+    }
+    __syncthreads();
+    const unsigned nd = ncl;
+    if (threadIdx.x == 0) sh_base = (long long)atomicAdd((unsigned long long*)&cnt[sh_r], (unsigned long long)nd);
+    __syncthreads();
+    const int64_t b = sstart[sh_r] + sh_base;
+    for (unsigned i = threadIdx.x; i < nd; i += blockDim.x) {
+      const uint32_t s = claim[i];
+      const unsigned long long x = T[s];
+      T[s] = kEmpty;
+      oc[b + i] = (int32_t)(x >> 32);
+      ow[b + i] = (uint32_t)x;
+    }
+    __syncthreads();
   }
 }
 
@@ -633,6 +820,27 @@ __global__ void __launch_bounds__(256) k_compact(const int64_t* __restrict__ sst
     }
     __syncthreads();
   }
+}
+
+// LV_BIG_SORT=1: big segments always by the radix-sort path (the partition path's
+// fallback; parity-tested as an alternative path)
+bool big_sort_forced() {
+  static const bool f = [] {
+    const char* e = getenv("LV_BIG_SORT");
+    return e && e[0] == '1';
+  }();
+  return f;
+}
+
+// LV_BIGP_SLOTS=s (power of 2 < kBigPSlots): smaller partition tables, so that tests
+// can drive the overflow -> sort fallback
+uint32_t bigp_capmax() {
+  static const uint32_t c = [] {
+    const char* e = getenv("LV_BIGP_SLOTS");
+    const long v = e ? atol(e) : 0;
+    return (v >= 64 && v < kBigPSlots && (v & (v - 1)) == 0) ? (uint32_t)v : (uint32_t)kBigPSlots;
+  }();
+  return c;
 }
 
 template <class... A>
@@ -870,20 +1078,78 @@ int32_t level_contract_fast(Handle& h, Level& L, Level& out, int32_t* d_map, int
   if (nbig > 0) {  // one radix sort of 64-bit (segment rank, neighbour) keys + reduce-by-key
     const int32_t* brows = rows + nsmall + nwarp + nmid;
     // offsets of the big segments in the key array: lengths + scan on the device
-    int64_t* dboff = nullptr;
+    int64_t *dboff = nullptr, *dpb = nullptr;
     LV_TRY(dalloc(&dboff, nbig + 1, s));
-    k_big_len<<<grid_for(nbig + 1, 256), 256, 0, s>>>(brows, nbig, sstart, dboff);
+    LV_TRY(dalloc(&dpb, nbig + 1, s));
+    k_bigp_sizes<<<grid_for(nbig + 1, 256), 256, 0, s>>>(brows, nbig, sstart, dboff, dpb);
     LV_LAUNCHED();
     LV_TRY(cub_scan_excl(s, dboff, dboff, nbig + 1));
-    int64_t m = 0;
-    LV_CUDA(cudaMemcpyAsync(&m, dboff + nbig, 8, cudaMemcpyDeviceToHost, s));
+    LV_TRY(cub_scan_excl(s, dpb, dpb, nbig + 1));
+    int64_t mp[2] = {0, 0};
+    LV_CUDA(cudaMemcpyAsync(&mp[0], dboff + nbig, 8, cudaMemcpyDeviceToHost, s));
+    LV_CUDA(cudaMemcpyAsync(&mp[1], dpb + nbig, 8, cudaMemcpyDeviceToHost, s));
     LV_CUDA(cudaStreamSynchronize(s));
+    int64_t m = mp[0];
+    const int64_t nparts = mp[1];
     if (tr.on)
       fprintf(stderr, "[lv]    contract segments: small %lld warp %lld mid %lld big %lld (big entries %lld of %lld)\n",
               (long long)nsmall, (long long)nwarp, (long long)nmid, (long long)nbig, (long long)m, (long long)nnz);
     int kb = 1;
     while (kb < 40 && (1ll << kb) < nbig) ++kb;
-    if (nb + kb <= 32) {  // 32-bit keys: 8 instead of 12 bytes per element and pass
+    const bool key_ok = nb + kb <= 32 && (((uint64_t)(nbig - 1) << nb) | (uint64_t)(np - 1)) < 0xFFFFFFFFull;
+    const bool comb = key_ok && m >= 64 * np;
+    bool sorted_path = comb || big_sort_forced();
+    if (!sorted_path) {  // label partitions (k_bigp_*)
+      int32_t* pc = nullptr;
+      uint32_t* pw = nullptr;
+      {
+        void* p0 = nullptr;
+        LV_TRY(scratch_get(h, SC_K1, 8 * (size_t)m, &p0));  // the level's stage / key buffers are dead here
+        pc = static_cast<int32_t*>(p0);
+        pw = weighted ? reinterpret_cast<uint32_t*>(pc + m) : nullptr;
+      }
+      unsigned long long* pcnt = nullptr;
+      LV_TRY(dalloc(&pcnt, nparts + 1, s));
+      LV_CUDA(cudaMemsetAsync(pcnt, 0, 8 * (nparts + 1), s));
+      const int64_t* btr = nullptr;
+      LV_TRY(tile_starts(h, dboff, 0, nbig, 0, m, kBigTile, &btr));
+      const unsigned g = grid_for((m + kBigTile - 1) / kBigTile, 1, 148 * 8);
+      k_bigp_pass<false><<<g, 256, 0, s>>>(brows, nbig, sstart, dboff, btr, m, gc, gw, dpb, pcnt, nullptr, nullptr);
+      LV_LAUNCHED();
+      int64_t* poff = reinterpret_cast<int64_t*>(pcnt);
+      LV_TRY(cub_scan_excl(s, poff, poff, nparts + 1));
+      unsigned long long* pcur = nullptr;
+      LV_TRY(dalloc(&pcur, nparts + 1, s));
+      LV_CUDA(cudaMemcpyAsync(pcur, poff, 8 * (nparts + 1), cudaMemcpyDeviceToDevice, s));
+      k_bigp_pass<true><<<g, 256, 0, s>>>(brows, nbig, sstart, dboff, btr, m, gc, gw, dpb, pcur, pc, pw);
+      LV_LAUNCHED();
+      dfree(pcur, s);
+      tr.mark(s, "big-part");
+      static int resident = 0;
+      if (resident == 0) {
+        LV_CUDA(cudaFuncSetAttribute(k_bigp_merge, cudaFuncAttributeMaxDynamicSharedMemorySize, 10 * kBigPSlots));
+        int nbk = 0;
+        LV_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nbk, k_bigp_merge, 1024, 10 * kBigPSlots));
+        resident = std::max(nbk, 1);
+      }
+      unsigned long long* ovf = &h.ctl->overflow;
+      k_bigp_merge<<<grid_for(nparts, 1, 148 * resident), 1024, 10 * kBigPSlots, s>>>(
+          poff, nparts, dpb, nbig, brows, sstart, pc, pw, oc, ow, cnt, ovf, bigp_capmax());
+      LV_LAUNCHED();
+      unsigned long long o = 0;
+      LV_CUDA(cudaMemcpyAsync(&o, ovf, 8, cudaMemcpyDeviceToHost, s));
+      LV_CUDA(cudaStreamSynchronize(s));
+      dfree(pcnt, s);
+      tr.mark(s, "big-merge");
+      if (o) {  // a partition table filled up: redo the big segments with the sort path
+        LV_CUDA(cudaMemsetAsync(ovf, 0, 8, s));
+        if (tr.on) fprintf(stderr, "[lv]    contract big partitions overflowed: sort path\n");
+        sorted_path = true;
+      }
+    }
+    if (!sorted_path) {
+      dfree(dboff, s);
+    } else if (nb + kb <= 32) {  // 32-bit keys: 8 instead of 12 bytes per element and pass
       uint32_t *k0 = nullptr, *k1 = nullptr, *v0 = nullptr, *v1 = nullptr;
       {
         void* p0 = nullptr;
@@ -895,9 +1161,7 @@ int32_t level_contract_fast(Handle& h, Level& L, Level& out, int32_t* d_map, int
         v1 = v0 + m;
       }
       // combiner: worthwhile when the big segments repeat neighbours (few new
-      // vertices per big entry); 0xFFFFFFFF must not be a real key (table marker)
-      const bool key_ok = (((uint64_t)(nbig - 1) << nb) | (uint64_t)(np - 1)) < 0xFFFFFFFFull;
-      const bool comb = key_ok && m >= 64 * np;
+      // vertices per big entry); 0xFFFFFFFF must not be a real key (table marker, key_ok)
       {
         const int64_t* btr = nullptr;
         LV_TRY(tile_starts(h, dboff, 0, nbig, 0, m, kBigTile, &btr));
@@ -1008,6 +1272,7 @@ int32_t level_contract_fast(Handle& h, Level& L, Level& out, int32_t* d_map, int
       LV_CUDA(cudaMemsetAsync(&h.ctl->bad, 0, 8, s));
     }
     tr.mark(s, "big-place");
+    dfree(dpb, s);
   }
   if (ms != s) {
     LV_CUDA(cudaEventRecord(h.ev_join, ms));

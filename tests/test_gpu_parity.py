@@ -450,6 +450,10 @@ def _alt_path_worker(env_items, names, q):
     (("LV_DELTA_DIV", "4"),),
     # serialised per-class timing (no side stream for the hub classes)
     (("LV_TRACE", "2"),),
+    # contraction: big segments by the radix-sort path instead of label partitions
+    (("LV_BIG_SORT", "1"),),
+    # contraction: 64-slot partition tables, so partitions overflow and fall back to the sort path
+    (("LV_BIGP_SLOTS", "64"),),
 ])
 def test_alternative_paths_match_oracle(env):
     import torch.multiprocessing as tmp
