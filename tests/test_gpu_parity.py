@@ -57,6 +57,19 @@ def weighted_with_loops(n, seed):
     return graphgen.weighted_csr(n, uu, vv, w)
 
 
+def rows_reversed(g):
+    """The same graph with every row's entries in descending column order (contracted levels
+    are unsorted too): nothing in the library may depend on sorted rows."""
+    col = g.col.copy()
+    w = None if g.w is None else g.w.copy()
+    for u in range(g.n):
+        a, b = int(g.rowptr[u]), int(g.rowptr[u + 1])
+        col[a:b] = col[a:b][::-1]
+        if w is not None:
+            w[a:b] = w[a:b][::-1]
+    return graphgen.Graph(g.n, g.rowptr.copy(), col, w, name=g.name + "_reversed")
+
+
 GRAPHS = {
     "karate": lambda: graphgen.karate(),
     "rmat10": lambda: graphgen.rmat(10, seed=2),
@@ -68,6 +81,7 @@ GRAPHS = {
     "hubs": lambda: hubs_graph(),
     # a 150000-degree hub: 25 label partitions (the hub kernel with LV_PART_MAXP < 25)
     "giant_hub": lambda: hubs_graph(seed=1, hub_degrees=(150000, 20000, 3000), n=200000, bg_tuples=300000),
+    "hubs_reversed": lambda: rows_reversed(hubs_graph(seed=2)),
 }
 
 
@@ -459,7 +473,7 @@ def test_alternative_paths_match_oracle(env):
     import torch.multiprocessing as tmp
     ctx = tmp.get_context("spawn")
     q = ctx.Queue()
-    names = ["karate", "rmat15", "lfr5k", "hubs", "giant_hub", "weighted_loops"]
+    names = ["karate", "rmat15", "lfr5k", "hubs", "giant_hub", "weighted_loops", "hubs_reversed"]
     pr = ctx.Process(target=_alt_path_worker, args=(env, names, q))
     pr.start()
     out = q.get(timeout=900)
