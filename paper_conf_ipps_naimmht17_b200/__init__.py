@@ -16,7 +16,8 @@ from typing import Optional
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "liblouvain.so")
+# LOUVAIN_LIB: an alternative build of the same C-ABI (tools/ab_build.py, A/B measurements)
+LIB_PATH = os.environ.get("LOUVAIN_LIB") or os.path.join(_HERE, "liblouvain.so")
 
 OK, E_INVALID_ARG, E_INVALID_GRAPH, E_OVERFLOW, E_NOMEM, E_CUDA, E_NCCL, E_STATE, E_UNSUPPORTED = \
     0, -1, -2, -3, -4, -5, -6, -7, -8

@@ -197,6 +197,9 @@ struct Level {
   // stage[soff[i] + t] = {label, a_c or 0xFFFFFFFF} of the t-th neighbour of bin_vertices[i]
   int64_t* soff = nullptr;
   uint2* stage = nullptr;
+  // bin_rb[i] = rowptr[bin_vertices[i]] (with soff: a vertex's row from two sequential
+  // loads by bin position, not the dependent bin_vertices -> rowptr round trips)
+  int64_t* bin_rb = nullptr;
   HubPlan hub;
   PartPlan part;
 };
@@ -207,9 +210,9 @@ struct Level {
 enum ScratchSlot {
   SC_STAGE = 0, SC_GC, SC_GW, SC_OC, SC_OW, SC_K1, SC_V0, SC_V1, SC_TMP, SC_TILES,
   // arrays of a contracted level inside louvain_run, double-buffered by level parity
-  SC_LVL0, SC_LVL_END = SC_LVL0 + 2 * 12, SC_COUNT = SC_LVL_END
+  SC_LVL0, SC_LVL_END = SC_LVL0 + 2 * 13, SC_COUNT = SC_LVL_END
 };
-enum LevelArray { LA_ROWPTR = 0, LA_COL, LA_W, LA_K, LA_CA, LA_SIZE, LA_MVV, LA_MVN, LA_MVO, LA_BIN, LA_SOFF, LA_C };
+enum LevelArray { LA_ROWPTR = 0, LA_COL, LA_W, LA_K, LA_CA, LA_SIZE, LA_MVV, LA_MVN, LA_MVO, LA_BIN, LA_SOFF, LA_C, LA_BINRB };
 struct Scratch {
   void* p[SC_COUNT] = {nullptr};
   size_t bytes[SC_COUNT] = {0};

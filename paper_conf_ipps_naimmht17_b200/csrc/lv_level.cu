@@ -132,9 +132,16 @@ __global__ void k_hub_degrees(const int32_t* hv, int64_t nh, const int64_t* rowp
   }
 }
 
-__global__ void k_bin_degrees(const int32_t* bv, int64_t n, const int64_t* rowptr, int64_t* dg) {
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i <= n; i += (int64_t)gridDim.x * blockDim.x)
-    dg[i] = (i < n) ? rowptr[bv[i] + 1] - rowptr[bv[i]] : 0;
+__global__ void k_bin_degrees(const int32_t* bv, int64_t n, const int64_t* rowptr, int64_t* dg, int64_t* brb) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i <= n; i += (int64_t)gridDim.x * blockDim.x) {
+    if (i < n) {
+      const int64_t rb = rowptr[bv[i]];
+      dg[i] = rowptr[bv[i] + 1] - rb;
+      brb[i] = rb;
+    } else {
+      dg[i] = 0;
+    }
+  }
 }
 
 __global__ void k_fill_u64(unsigned long long* p, int64_t n, unsigned long long v) {
@@ -538,6 +545,7 @@ int32_t level_alloc_scratch(Handle& h, Level& L, int parity) {
   LV_TRY(get(LA_MVO, 4 * n, (void**)&L.mv_old));
   LV_TRY(get(LA_BIN, 4 * n, (void**)&L.bin_vertices));
   LV_TRY(get(LA_SOFF, 8 * (n + 1), (void**)&L.soff));
+  LV_TRY(get(LA_BINRB, 8 * n, (void**)&L.bin_rb));
   L.scratch_backed = true;
   L.parity = parity;
   L.owns_csr = false;
@@ -568,6 +576,7 @@ void level_free(Level& L, cudaStream_t s) {
   }
   dfree(L.mv_v, s); dfree(L.mv_new, s); dfree(L.mv_old, s); dfree(L.bin_vertices, s); dfree(L.mv_stamp, s);
   dfree(L.soff, s);  // L.stage lives in the handle's scratch
+  dfree(L.bin_rb, s);
   hub_free(L.hub, s);
   part_free(L.part, s);
   L = Level();
@@ -920,7 +929,8 @@ int32_t level_binning(Handle& h, Level& L, const louvain_params_t& p) {
     dfree(cls, s); dfree(cls2, s); dfree(iota, s); dfree(hist, s);
     for (int c = 0; c < kNumClasses; ++c) L.class_off[c + 1] = L.class_off[c] + (int64_t)hh[c];
     // staging offsets: exclusive scan of the degrees in bin order
-    if (!L.soff) LV_TRY(dalloc(&L.soff, n + 1, s));  // scratch-backed levels have it already
+    if (!L.soff) LV_TRY(dalloc(&L.soff, n + 1, s));  // scratch-backed levels have them already
+    if (!L.bin_rb) LV_TRY(dalloc(&L.bin_rb, n, s));
     {
       void* st = nullptr;
       LV_TRY(scratch_get(h, SC_STAGE, sizeof(uint2) * (size_t)std::max<int64_t>(L.nnz, 1), &st));
@@ -928,7 +938,7 @@ int32_t level_binning(Handle& h, Level& L, const louvain_params_t& p) {
     }
     int64_t* dg = nullptr;
     LV_TRY(dalloc(&dg, n + 1, s));
-    k_bin_degrees<<<grid_for(n, 256), 256, 0, s>>>(L.bin_vertices, n, L.rowptr, dg);
+    k_bin_degrees<<<grid_for(n, 256), 256, 0, s>>>(L.bin_vertices, n, L.rowptr, dg, L.bin_rb);
     LV_LAUNCHED();
     size_t tb2 = 0;
     LV_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, tb2, dg, L.soff, n + 1, s));

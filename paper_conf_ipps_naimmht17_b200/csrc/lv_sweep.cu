@@ -119,7 +119,8 @@ __device__ __forceinline__ int32_t finish(long long s, int cb, uint32_t eown, in
 
 // ------------------------------------------------------------ deg <= 32
 template <int G, bool UNIT>
-__global__ void __launch_bounds__(256) sweep_small(const int32_t* __restrict__ verts, int64_t nv, SweepArgs A) {
+__global__ void __launch_bounds__(256) sweep_small(const int32_t* __restrict__ verts, const int64_t* __restrict__ brb,
+                                                   const int64_t* __restrict__ soff, int64_t nv, SweepArgs A) {
   const int lane = threadIdx.x & 31;
   const int sub = lane & (G - 1);
   const unsigned gmask = (G == 32) ? kFull : (((1u << G) - 1u) << (lane & ~(G - 1)));
@@ -131,10 +132,10 @@ __global__ void __launch_bounds__(256) sweep_small(const int32_t* __restrict__ v
     int32_t v = 0, own = -1, deg = 0;
     int64_t rb = 0;
     uint32_t ki = 0;
-    if (active) {
+    if (active) {  // row by bin position (sequential loads), then the vertex's own record
       v = __ldg(&verts[vi]);
-      rb = __ldg(&A.rowptr[v]);
-      deg = (int32_t)(__ldg(&A.rowptr[v + 1]) - rb);
+      rb = __ldg(&brb[vi]);
+      deg = (int32_t)(__ldg(&soff[vi + 1]) - __ldg(&soff[vi]));
       own = (int32_t)__ldg(&A.ca[v]).x;
       ki = __ldg(&A.k[v]);
     }
@@ -311,7 +312,7 @@ constexpr int kStageRows = 256;
 
 __global__ void __launch_bounds__(256) k_stage(const int32_t* __restrict__ bv, const int64_t* __restrict__ soff,
                                                int64_t pos0, int64_t pos1, const int64_t* __restrict__ tr,
-                                               const int64_t* __restrict__ rowptr,
+                                               const int64_t* __restrict__ brb,
                                                const int32_t* __restrict__ col, const uint2* __restrict__ ca,
                                                uint2* __restrict__ stage) {
   __shared__ int64_t sh_so[kStageRows + 1];
@@ -332,10 +333,9 @@ __global__ void __launch_bounds__(256) k_stage(const int32_t* __restrict__ bv, c
     const int64_t i0 = sh_i0;
     const int nr = sh_nr;
     for (int r = threadIdx.x; r < nr; r += blockDim.x) {
-      const int32_t v = bv[i0 + r];
-      sh_v[r] = v;
+      sh_v[r] = bv[i0 + r];
       sh_so[r] = soff[i0 + r];
-      sh_rb[r] = rowptr[v];
+      sh_rb[r] = brb[i0 + r];
     }
     __syncthreads();
     for (int64_t base = t0 + threadIdx.x; base < t1; base += 4 * (int64_t)blockDim.x) {
@@ -363,7 +363,7 @@ __global__ void __launch_bounds__(256) k_stage(const int32_t* __restrict__ bv, c
               if (soff[mid] <= t) lo = mid; else hi = mid - 1;
             }
             vv[q] = bv[lo];
-            e = rowptr[vv[q]] + (t - soff[lo]);
+            e = brb[lo] + (t - soff[lo]);
           }
           jj[q] = __ldcs(&col[e]);
         }
@@ -567,7 +567,9 @@ __device__ __forceinline__ void insert_claim_direct(unsigned long long* T, uint3
 
 // Warp per vertex gathering directly (no stage round trip of 16 B per entry).
 template <int CAP, int WARPS, bool UNIT, int PASSES>
-__global__ void __launch_bounds__(32 * WARPS) sweep_warp_d(const int32_t* __restrict__ verts, int64_t nv,
+__global__ void __launch_bounds__(32 * WARPS) sweep_warp_d(const int32_t* __restrict__ verts,
+                                                           const int64_t* __restrict__ brb,
+                                                           const int64_t* __restrict__ soff, int64_t nv,
                                                            SweepArgs A) {
   __shared__ unsigned long long tab[WARPS][CAP];
   __shared__ uint32_t taba[WARPS][CAP];
@@ -582,8 +584,8 @@ __global__ void __launch_bounds__(32 * WARPS) sweep_warp_d(const int32_t* __rest
   const int64_t warps = (int64_t)gridDim.x * WARPS;
   for (int64_t vi = (int64_t)blockIdx.x * WARPS + wl; vi < nv; vi += warps) {
     const int32_t v = __ldg(&verts[vi]);
-    const int64_t rb = __ldg(&A.rowptr[v]);
-    const int64_t deg = __ldg(&A.rowptr[v + 1]) - rb;
+    const int64_t rb = __ldg(&brb[vi]);
+    const int64_t deg = __ldg(&soff[vi + 1]) - __ldg(&soff[vi]);
     const int32_t own = (int32_t)__ldg(&A.ca[v]).x;
     const uint32_t ki = __ldg(&A.k[v]);
     uint32_t cl[4 * PASSES];
@@ -605,6 +607,7 @@ __global__ void __launch_bounds__(32 * WARPS) sweep_warp_d(const int32_t* __rest
 // Warp per vertex with register claims (rows of <= 128 * PASSES entries).
 template <int CAP, int WARPS, bool UNIT, int PASSES>
 __global__ void __launch_bounds__(32 * WARPS) sweep_warp_c(const int32_t* __restrict__ verts,
+                                                           const int64_t* __restrict__ brb,
                                                            const int64_t* __restrict__ soff, int64_t nv,
                                                            const uint2* __restrict__ stage, SweepArgs A) {
   __shared__ unsigned long long tab[WARPS][CAP];
@@ -620,8 +623,8 @@ __global__ void __launch_bounds__(32 * WARPS) sweep_warp_c(const int32_t* __rest
   const int64_t warps = (int64_t)gridDim.x * WARPS;
   for (int64_t vi = (int64_t)blockIdx.x * WARPS + wl; vi < nv; vi += warps) {
     const int32_t v = __ldg(&verts[vi]);
-    const int64_t rb = __ldg(&A.rowptr[v]);
-    const int64_t deg = __ldg(&A.rowptr[v + 1]) - rb;
+    const int64_t rb = __ldg(&brb[vi]);
+    const int64_t deg = __ldg(&soff[vi + 1]) - __ldg(&soff[vi]);
     const int32_t own = (int32_t)__ldg(&A.ca[v]).x;
     const uint32_t ki = __ldg(&A.k[v]);
     uint32_t cl[4 * PASSES];
@@ -643,6 +646,7 @@ __global__ void __launch_bounds__(32 * WARPS) sweep_warp_c(const int32_t* __rest
 // CTA per vertex with register claims (rows of <= 4 * PASSES * blockDim entries).
 template <bool UNIT, int PASSES>
 __global__ void __launch_bounds__(1024) sweep_cta_c(const int32_t* __restrict__ verts,
+                                                    const int64_t* __restrict__ brb,
                                                     const int64_t* __restrict__ soff, int64_t nv,
                                                     const uint2* __restrict__ stage, SweepArgs A, int capmax) {
   extern __shared__ unsigned long long smem[];
@@ -658,8 +662,8 @@ __global__ void __launch_bounds__(1024) sweep_cta_c(const int32_t* __restrict__ 
   __syncthreads();
   for (int64_t vi = blockIdx.x; vi < nv; vi += gridDim.x) {
     const int32_t v = __ldg(&verts[vi]);
-    const int64_t rb = __ldg(&A.rowptr[v]);
-    const int64_t deg = __ldg(&A.rowptr[v + 1]) - rb;
+    const int64_t rb = __ldg(&brb[vi]);
+    const int64_t deg = __ldg(&soff[vi + 1]) - __ldg(&soff[vi]);
     const int32_t own = (int32_t)__ldg(&A.ca[v]).x;
     const uint32_t ki = __ldg(&A.k[v]);
     const int64_t want = 2 * deg + 1;  // load <= 1/2
@@ -1386,23 +1390,24 @@ int32_t dispatch_class(Handle& h, Level& L, const SweepArgs& A, int bucket, int 
   if (nv <= 0) return LOUVAIN_OK;
   const int32_t* verts = L.bin_vertices + off;
   const int64_t* soff = L.soff + off;
+  const int64_t* brb = L.bin_rb + off;
   const uint2* stage = L.stage;
   cudaStream_t s = h.stream;
   if (sub == 0 && max_deg <= 32) {
     const int G = max_deg <= 4 ? 4 : max_deg <= 8 ? 8 : max_deg <= 16 ? 16 : 32;
     const unsigned grid = grid_for(nv, 8 * (32 / G), 148 * 8);
     switch (G) {
-      case 4: sweep_small<4, UNIT><<<grid, 256, 0, s>>>(verts, nv, A); break;
-      case 8: sweep_small<8, UNIT><<<grid, 256, 0, s>>>(verts, nv, A); break;
-      case 16: sweep_small<16, UNIT><<<grid, 256, 0, s>>>(verts, nv, A); break;
-      default: sweep_small<32, UNIT><<<grid, 256, 0, s>>>(verts, nv, A); break;
+      case 4: sweep_small<4, UNIT><<<grid, 256, 0, s>>>(verts, brb, soff, nv, A); break;
+      case 8: sweep_small<8, UNIT><<<grid, 256, 0, s>>>(verts, brb, soff, nv, A); break;
+      case 16: sweep_small<16, UNIT><<<grid, 256, 0, s>>>(verts, brb, soff, nv, A); break;
+      default: sweep_small<32, UNIT><<<grid, 256, 0, s>>>(verts, brb, soff, nv, A); break;
     }
     LV_LAUNCHED();
   } else if (sub == 0 && max_deg <= kDirectMaxDeg) {
-    sweep_warp_d<128, 8, UNIT, 1><<<grid_for(nv, 8, 148 * 8), 256, 0, s>>>(verts, nv, A);
+    sweep_warp_d<128, 8, UNIT, 1><<<grid_for(nv, 8, 148 * 8), 256, 0, s>>>(verts, brb, soff, nv, A);
     LV_LAUNCHED();
   } else if (sub == 0 && max_deg <= 340) {  // warp per vertex, 3 claim passes of 4 entries per lane
-    sweep_warp_c<512, 4, UNIT, 3><<<grid_for(nv, 4, 148 * 8), 128, 0, s>>>(verts, soff, nv, stage, A);
+    sweep_warp_c<512, 4, UNIT, 3><<<grid_for(nv, 4, 148 * 8), 128, 0, s>>>(verts, brb, soff, nv, stage, A);
     LV_LAUNCHED();
   } else if (sub >= kSubPart) {
     if (sub == kSubPart) LV_TRY(launch_part(h, L, A, bucket, UNIT));  // one pipeline covers sub-classes kSubPart..
@@ -1431,8 +1436,8 @@ int32_t dispatch_class(Handle& h, Level& L, const SweepArgs& A, int bucket, int 
           LV_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, kern, threads[sub], 12 * (size_t)capt));
           cres[sub][passes] = std::max(nb, 1);
         }
-        kern<<<grid_for(nv, 1, 148 * cres[sub][passes]), threads[sub], 12 * (size_t)capt, s>>>(verts, soff, nv,
-                                                                                             stage, A, capt);
+        kern<<<grid_for(nv, 1, 148 * cres[sub][passes]), threads[sub], 12 * (size_t)capt, s>>>(verts, brb, soff,
+                                                                                             nv, stage, A, capt);
         LV_LAUNCHED();
         LV_CUDA(cudaGetLastError());
         return LOUVAIN_OK;
@@ -1478,7 +1483,7 @@ int32_t launch_stage(Handle& h, Level& L, int64_t pos0, int64_t pos1, int64_t s0
   const int64_t* tr = nullptr;
   LV_TRY(tile_starts(h, L.soff, pos0, pos1, s0, s1, kStageTile, &tr));
   k_stage<<<grid_for((s1 - s0 + kStageTile - 1) / kStageTile, 1, 148 * 8), 256, 0, h.stream>>>(
-      L.bin_vertices, L.soff, pos0, pos1, tr, L.rowptr, L.col, L.ca, L.stage);
+      L.bin_vertices, L.soff, pos0, pos1, tr, L.bin_rb, L.col, L.ca, L.stage);
   LV_LAUNCHED();
   LV_CUDA(cudaGetLastError());
   return LOUVAIN_OK;
@@ -1507,11 +1512,13 @@ int32_t launch_sweep_bucket(Handle& h, Level& L, const louvain_params_t& p, int 
       const int64_t nv = L.class_off[kSubPerBucket * bucket + sub + 1] - off;
       if (nv <= 0) continue;
       const int32_t* verts = L.bin_vertices + off;
+      const int64_t* brb = L.bin_rb + off;
+      const int64_t* soff = L.soff + off;
       const int G = 1 << (sub - 1);
       const unsigned grid = grid_for(nv, 8 * (32 / G), 148 * 8);
 #define LV_SMALL(GG)                                                              \
-  if (L.w) sweep_small<GG, false><<<grid, 256, 0, s>>>(verts, nv, A);              \
-  else sweep_small<GG, true><<<grid, 256, 0, s>>>(verts, nv, A)
+  if (L.w) sweep_small<GG, false><<<grid, 256, 0, s>>>(verts, brb, soff, nv, A); \
+  else sweep_small<GG, true><<<grid, 256, 0, s>>>(verts, brb, soff, nv, A)
       switch (G) {
         case 1: LV_SMALL(1); break;
         case 2: LV_SMALL(2); break;

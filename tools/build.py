@@ -60,13 +60,14 @@ def build_graphgen(force: bool = False) -> str:
     return out
 
 
-def build_louvain(force: bool = False) -> str:
+def build_louvain(force: bool = False, d: str = "", out: str = "", objdir: str = "") -> str:
+    """The product library; d/out/objdir name another source tree and target (tools/ab_build.py)."""
     pkg = os.path.join(ROOT, "paper_conf_ipps_naimmht17_b200")
-    d = os.path.join(pkg, "csrc")
+    d = d or os.path.join(pkg, "csrc")
     srcs = sorted(glob.glob(os.path.join(d, "*.cu")) + glob.glob(os.path.join(d, "*.cpp")))
     hdrs = glob.glob(os.path.join(d, "*.h")) + glob.glob(os.path.join(d, "*.cuh")) + \
         glob.glob(os.path.join(ROOT, "include", "*.h"))
-    out = os.path.join(pkg, "liblouvain.so")
+    out = out or os.path.join(pkg, "liblouvain.so")
     if not srcs:
         return out
     nccl = _site_nccl()
@@ -74,7 +75,7 @@ def build_louvain(force: bool = False) -> str:
     if nccl:
         nccl_flags = ["-I", os.path.join(nccl, "include"), "-DLOUVAIN_HAVE_NCCL_HEADERS=1"]
     # one object per translation unit (compiled in parallel, only when stale), then one link
-    objdir = os.path.join(ROOT, "build", "louvain")
+    objdir = objdir or os.path.join(ROOT, "build", "louvain")
     os.makedirs(objdir, exist_ok=True)
     flags = [NVCC, "-O3", "-std=c++17", *ARCH, "-lineinfo", "-Xptxas", "-v",
              "-Xcompiler", "-fPIC,-ffp-contract=off,-fvisibility=hidden",
@@ -95,10 +96,20 @@ def build_louvain(force: bool = False) -> str:
     return out
 
 
+def build_micro(force: bool = False) -> str:
+    """tools/micro/libgather_sol.so: the gather speed-of-light kernel bench.py times beside the sweep."""
+    src = os.path.join(ROOT, "tools", "micro", "gather_sol.cu")
+    out = os.path.join(ROOT, "tools", "micro", "libgather_sol.so")
+    if force or _stale(out, [src, __file__]):
+        _run([NVCC, "-O3", "-std=c++17", *ARCH, "-lineinfo", "-shared", "-Xcompiler", "-fPIC", "-o", out, src])
+    return out
+
+
 def build_all(force: bool = False) -> None:
     build_oracle(force)
     build_graphgen(force)
     build_louvain(force)
+    build_micro(force)
 
 
 if __name__ == "__main__":
