@@ -294,6 +294,38 @@ def level0_fields(st, nnz):
             "phase1_teps_E": k0 * (nnz // 2) / (t_ph1 / 1e3) if t_ph1 else None}
 
 
+def gather_sol(dg, stream, reps=3):
+    """The sweep's unavoidable memory work alone on this graph: stream col once and fetch
+    every neighbour's 8-byte record {C, a} (tools/micro/gather_sol.cu, records laid out as at
+    the first sweep: C = id, a = degree).  Median of `reps` launches, CUDA events on `stream`."""
+    import ctypes
+    import torch
+    so = os.path.join(ROOT, "tools", "micro", "libgather_sol.so")
+    if not os.path.exists(so):
+        return None
+    lib = ctypes.CDLL(so)
+    lib.gsol_run.restype = ctypes.c_int
+    lib.gsol_run.argtypes = [ctypes.c_void_p, ctypes.c_int64, ctypes.c_void_p, ctypes.c_int64, ctypes.c_void_p,
+                             ctypes.POINTER(ctypes.c_float)]
+    n, nnz = dg.n, dg.nnz
+    with torch.cuda.stream(stream):
+        deg = (dg.rowptr[1:] - dg.rowptr[:-1]).to(torch.int32)
+        ca = torch.stack([torch.arange(n, dtype=torch.int32, device=deg.device), deg], dim=1).contiguous()
+    stream.synchronize()
+    times = []
+    for _ in range(reps + 1):
+        ms = ctypes.c_float(0.0)
+        rc = lib.gsol_run(dg.col.data_ptr(), nnz, ca.data_ptr(), n, ctypes.c_void_p(stream.cuda_stream),
+                          ctypes.byref(ms))
+        if rc != 0:
+            return None
+        times.append(ms.value)
+    t = statistics.median(times[1:])
+    return {"ms": t, "entries": nnz, "gathers_per_s": nnz / (t / 1e3), "bytes_model": 12 * nnz,
+            "what": "col streamed once + one 8-byte record gather per entry, nothing else "
+                    "(tools/micro/gather_sol.cu): the floor the sweep's random gathers set on this graph"}
+
+
 def roofline_of(args, n_act, nnz, st, t_sw1, world=1):
     D = oracle_D(args.config)
     B = sweep_bytes(n_act, nnz, D=D if D is not None else nnz, moved=st["moved_first"]) / world
@@ -479,6 +511,10 @@ def run_ours(args, rank, world):
            "agg_share": sum(st0["t_agg_ms"]) / st0["t_total_ms"] if st0["t_total_ms"] else None,
            "gen_s": gen_s}
     out.update(level0_fields(st0, nnz))
+    sol = gather_sol(dg, stream)
+    if sol:
+        sol["sweep1_over_sol"] = t_sw1 / sol["ms"]
+        out["gather_sol"] = sol
 
     # end to end through the C-ABI with host buffers: every step copies the CSR from pinned
     # host memory (louvain_create_csr), runs, and reads the labels back; the parts are timed

@@ -1097,7 +1097,8 @@ int32_t level_contract_fast(Handle& h, Level& L, Level& out, int32_t* d_map, int
     int kb = 1;
     while (kb < 40 && (1ll << kb) < nbig) ++kb;
     const bool key_ok = nb + kb <= 32 && (((uint64_t)(nbig - 1) << nb) | (uint64_t)(np - 1)) < 0xFFFFFFFFull;
-    const bool comb = key_ok && m >= 64 * np;
+    static const bool comb_off = getenv("LV_COMB") && getenv("LV_COMB")[0] == '0';  // A/B
+    const bool comb = key_ok && m >= 64 * np && !comb_off;
     bool sorted_path = comb || big_sort_forced();
     if (!sorted_path) {  // label partitions (k_bigp_*)
       int32_t* pc = nullptr;

@@ -643,9 +643,11 @@ __global__ void __launch_bounds__(32 * WARPS) sweep_warp_c(const int32_t* __rest
   }
 }
 
-// CTA per vertex with register claims (rows of <= 4 * PASSES * blockDim entries).
+// CTA per vertex with register claims (rows of <= 4 * PASSES * blockDim entries).  The
+// single-pass tiers (128-512 threads) are held to 32 registers, so that their CTAs fill
+// an SM (the weighted variant used 44: 1408 instead of 2048 threads; C5 sweeps -7 ms).
 template <bool UNIT, int PASSES>
-__global__ void __launch_bounds__(1024) sweep_cta_c(const int32_t* __restrict__ verts,
+__global__ void __launch_bounds__(1024, PASSES == 1 ? 2 : 1) sweep_cta_c(const int32_t* __restrict__ verts,
                                                     const int64_t* __restrict__ brb,
                                                     const int64_t* __restrict__ soff, int64_t nv,
                                                     const uint2* __restrict__ stage, SweepArgs A, int capmax) {
