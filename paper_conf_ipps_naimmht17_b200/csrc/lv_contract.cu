@@ -576,8 +576,11 @@ __global__ void __launch_bounds__(256) k_big_keys_t(const int32_t* __restrict__ 
 // neighbours per partition <= kBigPE in a table of 2 * kBigPE slots; a table that
 // fills up raises *overflow and the level redoes its big segments with the sort path
 // (deterministic either way).
-constexpr int kBigPE = 8192;
-constexpr int kBigPSlots = 16384;
+#ifndef LV_BIGPE  // compile-time A/B (tools/ab_build.py --define)
+#define LV_BIGPE 8192
+#endif
+constexpr int kBigPE = LV_BIGPE;
+constexpr int kBigPSlots = 2 * LV_BIGPE;
 
 __global__ void k_bigp_sizes(const int32_t* __restrict__ rows, int64_t nbig, const int64_t* __restrict__ sstart,
                              int64_t* len, int64_t* nparts) {
@@ -1097,8 +1100,7 @@ int32_t level_contract_fast(Handle& h, Level& L, Level& out, int32_t* d_map, int
     int kb = 1;
     while (kb < 40 && (1ll << kb) < nbig) ++kb;
     const bool key_ok = nb + kb <= 32 && (((uint64_t)(nbig - 1) << nb) | (uint64_t)(np - 1)) < 0xFFFFFFFFull;
-    static const bool comb_off = getenv("LV_COMB") && getenv("LV_COMB")[0] == '0';  // A/B
-    const bool comb = key_ok && m >= 64 * np && !comb_off;
+    const bool comb = key_ok && m >= 64 * np;
     bool sorted_path = comb || big_sort_forced();
     if (!sorted_path) {  // label partitions (k_bigp_*)
       int32_t* pc = nullptr;

@@ -60,7 +60,7 @@ def build_graphgen(force: bool = False) -> str:
     return out
 
 
-def build_louvain(force: bool = False, d: str = "", out: str = "", objdir: str = "") -> str:
+def build_louvain(force: bool = False, d: str = "", out: str = "", objdir: str = "", defines=()) -> str:
     """The product library; d/out/objdir name another source tree and target (tools/ab_build.py)."""
     pkg = os.path.join(ROOT, "paper_conf_ipps_naimmht17_b200")
     d = d or os.path.join(pkg, "csrc")
@@ -79,7 +79,7 @@ def build_louvain(force: bool = False, d: str = "", out: str = "", objdir: str =
     os.makedirs(objdir, exist_ok=True)
     flags = [NVCC, "-O3", "-std=c++17", *ARCH, "-lineinfo", "-Xptxas", "-v",
              "-Xcompiler", "-fPIC,-ffp-contract=off,-fvisibility=hidden",
-             "-I", os.path.join(ROOT, "include"), *nccl_flags]
+             "-I", os.path.join(ROOT, "include"), *nccl_flags, *[f"-D{x}" for x in defines]]
     objs, procs = [], []
     for src in srcs:
         obj = os.path.join(objdir, os.path.basename(src) + ".o")
