@@ -159,32 +159,40 @@ __global__ void __launch_bounds__(256) k_scatter_copy(const int64_t* __restrict_
       }
     }
     __syncthreads();
-    for (int64_t base = e0 + threadIdx.x; base < e1; base += 4 * (int64_t)blockDim.x) {
+    // warp spans of 128 entries (lane + 32 q): one binary search per lane, then a
+    // forward walk (the next entry of a lane is 32 further, mostly in the same row)
+    const int lane = threadIdx.x & 31, wl = threadIdx.x >> 5, nw = blockDim.x >> 5;
+    for (int64_t span = e0 + (int64_t)wl * 128; span < e1; span += (int64_t)nw * 128) {
       int32_t jj[4];
       int64_t dd[4];
+      int lo = 0;
+      if (nr > 0 && span + lane < e1) {
+        int hi = nr - 1;  // largest r with sh_rp[r] <= e
+        const int64_t e = span + lane;
+        while (lo < hi) {
+          const int mid = (lo + hi + 1) >> 1;
+          if (sh_rp[mid] <= e) lo = mid; else hi = mid - 1;
+        }
+      }
 #pragma unroll
       for (int q = 0; q < 4; ++q) {
-        const int64_t e = base + (int64_t)q * blockDim.x;
+        const int64_t e = span + lane + 32 * q;
         jj[q] = -1;
         dd[q] = 0;
         if (e < e1) {
           if (nr > 0) {
-            int lo = 0, hi = nr - 1;  // largest r with sh_rp[r] <= e
-            while (lo < hi) {
-              const int mid = (lo + hi + 1) >> 1;
-              if (sh_rp[mid] <= e) lo = mid; else hi = mid - 1;
-            }
+            while (lo + 1 < nr && sh_rp[lo + 1] <= e) ++lo;
             dd[q] = sh_db[lo] + (e - sh_rp[lo]);
             if (RANGE && !sh_mine[lo]) continue;  // another rank merges this row's community
           } else {
-            int64_t lo = 0, hi = n - 1;
-            while (lo < hi) {
-              const int64_t mid = (lo + hi + 1) >> 1;
-              if (rowptr[mid] <= e) lo = mid; else hi = mid - 1;
+            int64_t a = 0, b = n - 1;
+            while (a < b) {
+              const int64_t mid = (a + b + 1) >> 1;
+              if (rowptr[mid] <= e) a = mid; else b = mid - 1;
             }
-            dd[q] = dbase[lo] + (e - rowptr[lo]);
+            dd[q] = dbase[a] + (e - rowptr[a]);
             if (RANGE) {
-              const int32_t c = map[lo];
+              const int32_t c = map[a];
               if (c < c_lo || c >= c_hi) continue;
             }
           }
@@ -196,7 +204,7 @@ __global__ void __launch_bounds__(256) k_scatter_copy(const int64_t* __restrict_
       for (int q = 0; q < 4; ++q) mm[q] = jj[q] >= 0 ? __ldg(&map[jj[q]]) : 0;
 #pragma unroll
       for (int q = 0; q < 4; ++q) {
-        const int64_t e = base + (int64_t)q * blockDim.x;
+        const int64_t e = span + lane + 32 * q;
         if (e < e1 && jj[q] >= 0) {
           gc[dd[q]] = mm[q];
           if (gw) gw[dd[q]] = w ? __ldcs(&w[e]) : 1u;
@@ -577,7 +585,7 @@ __global__ void __launch_bounds__(256) k_big_keys_t(const int32_t* __restrict__ 
 // fills up raises *overflow and the level redoes its big segments with the sort path
 // (deterministic either way).
 #ifndef LV_BIGPE  // compile-time A/B (tools/ab_build.py --define)
-#define LV_BIGPE 8192
+#define LV_BIGPE 4096
 #endif
 constexpr int kBigPE = LV_BIGPE;
 constexpr int kBigPSlots = 2 * LV_BIGPE;
@@ -787,35 +795,43 @@ __global__ void __launch_bounds__(256) k_compact(const int64_t* __restrict__ sst
       sh_s[r] = sstart[r0 + r];
     }
     __syncthreads();
-    for (int64_t qb = q0 + threadIdx.x; qb < q1; qb += 4 * (int64_t)blockDim.x) {  // 4 entries in flight
+    // warp spans of 128 entries (lane + 32 u), 4 in flight per lane: one binary search
+    // per lane, then a forward walk over the tile's rows
+    const int lane = threadIdx.x & 31, wl = threadIdx.x >> 5, nw = blockDim.x >> 5;
+    for (int64_t span = q0 + (int64_t)wl * 128; span < q1; span += (int64_t)nw * 128) {
       int32_t cc[4];
       uint32_t ww[4];
+      int lo = 0;
+      if (nr > 0 && span + lane < q1) {
+        int hi = nr - 1;
+        const int64_t q = span + lane;
+        while (lo < hi) {
+          const int mid = (lo + hi + 1) >> 1;
+          if (sh_r[mid] <= q) lo = mid; else hi = mid - 1;
+        }
+      }
 #pragma unroll
       for (int u = 0; u < 4; ++u) {
-        const int64_t q = qb + (int64_t)u * blockDim.x;
+        const int64_t q = span + lane + 32 * u;
         if (q >= q1) continue;
         int64_t src;
         if (nr > 0) {
-          int lo = 0, hi = nr - 1;
-          while (lo < hi) {
-            const int mid = (lo + hi + 1) >> 1;
-            if (sh_r[mid] <= q) lo = mid; else hi = mid - 1;
-          }
+          while (lo + 1 < nr && sh_r[lo + 1] <= q) ++lo;
           src = sh_s[lo] + (q - sh_r[lo]);
         } else {
-          int64_t lo = 0, hi = np - 1;
-          while (lo < hi) {
-            const int64_t mid = (lo + hi + 1) >> 1;
-            if (rowptr_out[mid] <= q) lo = mid; else hi = mid - 1;
+          int64_t a = 0, b = np - 1;
+          while (a < b) {
+            const int64_t mid = (a + b + 1) >> 1;
+            if (rowptr_out[mid] <= q) a = mid; else b = mid - 1;
           }
-          src = sstart[lo] + (q - rowptr_out[lo]);
+          src = sstart[a] + (q - rowptr_out[a]);
         }
         cc[u] = __ldcs(&oc[src]);
         ww[u] = __ldcs(&ow[src]);
       }
 #pragma unroll
       for (int u = 0; u < 4; ++u) {
-        const int64_t q = qb + (int64_t)u * blockDim.x;
+        const int64_t q = span + lane + 32 * u;
         if (q >= q1) continue;
         col[q] = cc[u];
         w[q] = ww[u];

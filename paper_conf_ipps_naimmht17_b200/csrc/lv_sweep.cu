@@ -338,32 +338,41 @@ __global__ void __launch_bounds__(256) k_stage(const int32_t* __restrict__ bv, c
       sh_rb[r] = brb[i0 + r];
     }
     __syncthreads();
-    for (int64_t base = t0 + threadIdx.x; base < t1; base += 4 * (int64_t)blockDim.x) {
+    // warp spans of 128 entries (lane + 32 q): one binary search per lane for its first
+    // entry, then a forward walk -- the next entry of a lane is 32 further, mostly in
+    // the same row (the per-entry searches were most of this kernel's instructions)
+    const int lane = threadIdx.x & 31, wl = threadIdx.x >> 5, nw = blockDim.x >> 5;
+    for (int64_t span = t0 + (int64_t)wl * 128; span < t1; span += (int64_t)nw * 128) {
       int32_t jj[4], vv[4];
       uint2 rr[4];
+      int lo = 0;
+      if (nr > 0 && span + lane < t1) {
+        int hi = nr - 1;
+        const int64_t t = span + lane;
+        while (lo < hi) {
+          const int mid = (lo + hi + 1) >> 1;
+          if (sh_so[mid] <= t) lo = mid; else hi = mid - 1;
+        }
+      }
 #pragma unroll
       for (int q = 0; q < 4; ++q) {
-        const int64_t t = base + (int64_t)q * blockDim.x;
+        const int64_t t = span + lane + 32 * q;
         jj[q] = -1;
         vv[q] = -1;
         if (t < t1) {
           int64_t e;
           if (nr > 0) {
-            int lo = 0, hi = nr - 1;
-            while (lo < hi) {
-              const int mid = (lo + hi + 1) >> 1;
-              if (sh_so[mid] <= t) lo = mid; else hi = mid - 1;
-            }
+            while (lo + 1 < nr && sh_so[lo + 1] <= t) ++lo;
             vv[q] = sh_v[lo];
             e = sh_rb[lo] + (t - sh_so[lo]);
           } else {
-            int64_t lo = pos0, hi = pos1 - 1;
-            while (lo < hi) {
-              const int64_t mid = (lo + hi + 1) >> 1;
-              if (soff[mid] <= t) lo = mid; else hi = mid - 1;
+            int64_t a = pos0, b = pos1 - 1;
+            while (a < b) {
+              const int64_t mid = (a + b + 1) >> 1;
+              if (soff[mid] <= t) a = mid; else b = mid - 1;
             }
-            vv[q] = bv[lo];
-            e = brb[lo] + (t - soff[lo]);
+            vv[q] = bv[a];
+            e = brb[a] + (t - soff[a]);
           }
           jj[q] = __ldcs(&col[e]);
         }
@@ -372,7 +381,7 @@ __global__ void __launch_bounds__(256) k_stage(const int32_t* __restrict__ bv, c
       for (int q = 0; q < 4; ++q) rr[q] = (jj[q] >= 0 && jj[q] != vv[q]) ? __ldg(&ca[jj[q]]) : make_uint2(kSelf, 0);
 #pragma unroll
       for (int q = 0; q < 4; ++q) {
-        const int64_t t = base + (int64_t)q * blockDim.x;
+        const int64_t t = span + lane + 32 * q;
         // evict-first store: the stage streams through L2 once and must not
         // displace the gathered records
         const uint2 val = (jj[q] == vv[q]) ? make_uint2(kSelf, 0u)
@@ -688,6 +697,121 @@ __global__ void __launch_bounds__(1024, PASSES == 1 ? 2 : 1) sweep_cta_c(const i
     __syncthreads();
   }
 }
+
+#ifdef LV_TMA
+// Compile-time experiment (tools/ab_build.py -DLV_TMA=1): the unit-weight single-pass CTA
+// tiers with the staged row of the NEXT vertex brought into shared memory by a 1-D bulk
+// copy (cp.async.bulk, TMA) while the current vertex is hashed, double-buffered with two
+// mbarriers; the inserts then read shared memory.  Rows are 8-byte aligned, bulk copies
+// need 16: the copy starts at the 16-byte boundary below the row (one record of slack).
+__device__ __forceinline__ uint32_t smem_addr(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void bulk_row(uint2* buf, unsigned long long* bar, const uint2* stage, int64_t so,
+                                         int64_t deg) {
+  const int64_t a0 = so & ~1ll, a1 = (so + deg + 1) & ~1ll;  // records [a0, a1): 16-byte aligned
+  const uint32_t bytes = (uint32_t)((a1 - a0) * 8);
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_addr(bar)), "r"(bytes) : "memory");
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                   smem_addr(buf)),
+               "l"(stage + a0), "r"(bytes), "r"(smem_addr(bar))
+               : "memory");
+}
+__device__ __forceinline__ void bar_wait(unsigned long long* bar, uint32_t phase) {
+  uint32_t done = 0;
+  while (!done)
+    asm volatile(
+        "{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2; selp.u32 %0, 1, 0, p; }"
+        : "=r"(done)
+        : "r"(smem_addr(bar)), "r"(phase)
+        : "memory");
+}
+
+__global__ void __launch_bounds__(1024, 2) sweep_cta_tma(const int32_t* __restrict__ verts,
+                                                         const int64_t* __restrict__ brb,
+                                                         const int64_t* __restrict__ soff, int64_t nv,
+                                                         const uint2* __restrict__ stage, SweepArgs A, int capmax,
+                                                         int bufrec) {
+  extern __shared__ unsigned long long smem[];
+  unsigned long long* T = smem;
+  uint32_t* TA = reinterpret_cast<uint32_t*>(smem + capmax);
+  uint2* buf0 = reinterpret_cast<uint2*>(TA + capmax + (capmax & 3 ? 4 - (capmax & 3) : 0));
+  uint2* bufs[2] = {buf0, buf0 + bufrec};
+  __shared__ __align__(8) unsigned long long bars[2];
+  __shared__ long long sh_s[32];
+  __shared__ int sh_c[32];
+  __shared__ unsigned sh_e[32];
+  for (int t = threadIdx.x; t < capmax; t += blockDim.x) {
+    T[t] = kEmpty;
+    TA[t] = kUnknownA;
+  }
+  if (threadIdx.x == 0) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_addr(&bars[0])) : "memory");
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_addr(&bars[1])) : "memory");
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+  const int64_t G = gridDim.x;
+  if (threadIdx.x == 0 && blockIdx.x < nv) {
+    const int64_t so = __ldg(&soff[blockIdx.x]);
+    bulk_row(bufs[0], &bars[0], stage, so, __ldg(&soff[blockIdx.x + 1]) - so);
+  }
+  int it = 0;
+  for (int64_t vi = blockIdx.x; vi < nv; vi += G, ++it) {
+    const int b = it & 1;
+    const int32_t v = __ldg(&verts[vi]);
+    const int64_t rb = __ldg(&brb[vi]);
+    const int64_t so = __ldg(&soff[vi]);
+    const int64_t deg = __ldg(&soff[vi + 1]) - so;
+    const int32_t own = (int32_t)__ldg(&A.ca[v]).x;
+    const uint32_t ki = __ldg(&A.k[v]);
+    int64_t so_n = 0, deg_n = 0;
+    const bool has_next = vi + G < nv;
+    if (threadIdx.x == 0 && has_next) {  // next row's place, loaded early (used after the inserts)
+      so_n = __ldg(&soff[vi + G]);
+      deg_n = __ldg(&soff[vi + G + 1]) - so_n;
+    }
+    const int64_t want = 2 * deg + 1;
+    const uint32_t cap = (uint32_t)(want < (int64_t)capmax ? want : (int64_t)capmax);
+    bar_wait(&bars[b], (uint32_t)((it >> 1) & 1));
+    const uint2* S = bufs[b] + (so & 1);
+    uint32_t cl[4];
+    {
+      uint2 rr[4];
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        const int64_t t = (int64_t)threadIdx.x + (int64_t)q * blockDim.x;
+        rr[q] = (t < deg) ? S[t] : make_uint2(kSelf, 0u);
+      }
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        uint32_t slot = kNoClaim;
+        if (rr[q].x != kSelf) {
+          bool claimed = false;
+          const uint32_t hq = table_insert_c(T, cap, (int32_t)rr[q].x, 1u, &claimed);
+          if (rr[q].y != kUnknownA) TA[hq] = rr[q].y;
+          if (claimed) slot = hq;
+        }
+        cl[q] = slot;
+      }
+    }
+    __syncthreads();  // every read of bufs[b] done; bufs[b ^ 1] was read in the last iteration
+    if (threadIdx.x == 0 && has_next) bulk_row(bufs[b ^ 1], &bars[b ^ 1], stage, so_n, deg_n);
+    const bool own_single = A.rule == 2 && __ldg(&A.size[own]) == 1;
+    long long s = (long long)0x8000000000000000ull;
+    int cb = 0x7FFFFFFF;
+    unsigned eown = 0;
+    eval_claims<1>(T, TA, cl, own, own_single, ki, A, s, cb, eown);
+    block_reduce(s, cb, eown, sh_s, sh_c, sh_e);
+    if (threadIdx.x < 32) {
+      int32_t tgt = own;
+      if (threadIdx.x == 0) tgt = finish(s, cb, eown, own, __ldg(&A.ca[own]).y, ki, A);
+      log_moves(threadIdx.x == 0 && tgt != own, v, tgt, A);
+    }
+    __syncthreads();
+    (void)rb;
+  }
+}
+#endif
 
 // ------------------------------------------------------------ label-partitioned CTAs
 // deg >= 12288: vertex v gets P = ceil(deg / kPartLabels) independent CTA tasks;
@@ -1444,6 +1568,28 @@ int32_t dispatch_class(Handle& h, Level& L, const SweepArgs& A, int bucket, int 
         LV_CUDA(cudaGetLastError());
         return LOUVAIN_OK;
       };
+#ifdef LV_TMA
+      if (UNIT && passes <= 1) {
+        const int bufrec = (int)(((md + 2 + 1) / 2) * 2);  // records per buffer (even: 16-byte buffers)
+        const size_t sm = 12 * (size_t)capt + 16 + 2 * 8 * (size_t)bufrec;
+        static bool tattr = false;
+        if (!tattr) {
+          LV_TRY(set_smem(sweep_cta_tma, 12 * (size_t)8192 + 16 + 2 * 8 * (size_t)(kSub3Min + 2)));
+          tattr = true;
+        }
+        static int tres[5] = {0};
+        if (tres[sub] == 0) {
+          int nb = 0;
+          LV_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, sweep_cta_tma, threads[sub], sm));
+          tres[sub] = std::max(nb, 1);
+        }
+        sweep_cta_tma<<<grid_for(nv, 1, 148 * tres[sub]), threads[sub], sm, s>>>(verts, brb, soff, nv, stage, A, capt,
+                                                                                bufrec);
+        LV_LAUNCHED();
+        LV_CUDA(cudaGetLastError());
+        return LOUVAIN_OK;
+      }
+#endif
       if (passes <= 1) return go(sweep_cta_c<UNIT, 1>);
       if (passes == 2) return go(sweep_cta_c<UNIT, 2>);
       if (passes == 3) return go(sweep_cta_c<UNIT, 3>);
