@@ -142,7 +142,8 @@ int32_t louvain_run(louvain_graph_t g, const louvain_params_t* p, int32_t* label
 const char* louvain_last_error(void);
 /* Free the device memory the library keeps between handles: the scratch
  * buffers of the most recently destroyed handle per device (reused by the next
- * handle; bounded to one handle's set per device) and the idle blocks of the
+ * handle, buffer by buffer in the role each served; bounded to one handle's set
+ * per device) and the idle blocks of the
  * library's private stream-ordered memory pool.  Never needed for correctness:
  * an allocation failure releases both and retries once. */
 int32_t louvain_release_cache(void);

@@ -64,23 +64,27 @@ cudaMemPool_t lib_pool(int dev) {
 // Process-wide cache of the scratch buffers of destroyed handles, so a new handle
 // on the same device (e.g. every end-to-end louvain_create_csr + louvain_run)
 // reuses device memory instead of paying tens of GB of cudaMalloc again.  Bounded:
-// it holds the buffers of the most recently destroyed handle per device only (a
-// destroy releases what an earlier one left).  Released on any allocation
-// failure, by louvain_release_cache(), or never filled with LV_SCRATCH_CACHE=0.
+// one handle's set per device (scratch_free).  Released on any allocation failure, by
+// louvain_release_cache(), or never filled with LV_SCRATCH_CACHE=0.
 std::mutex g_cache_mu;
-std::vector<std::tuple<int, void*, size_t>> g_cache;  // (device, ptr, bytes)
+std::vector<std::tuple<int, void*, size_t, int>> g_cache;  // (device, ptr, bytes, scratch slot)
 bool cache_on() {
   static const bool on = !(getenv("LV_SCRATCH_CACHE") && getenv("LV_SCRATCH_CACHE")[0] == '0');
   return on;
 }
-void* cache_take(int dev, size_t bytes, size_t* got) {
+// A buffer that served the same scratch slot before is preferred (handles of one graph
+// ask every slot for the same size, so each buffer goes back to its own role), else the
+// smallest cached buffer that is large enough.
+void* cache_take(int dev, int slot, size_t bytes, size_t* got) {
   std::lock_guard<std::mutex> lk(g_cache_mu);
   int best = -1;
-  for (int i = 0; i < (int)g_cache.size(); ++i) {
-    const auto& c = g_cache[i];
-    if (std::get<0>(c) == dev && std::get<2>(c) >= bytes &&
-        (best < 0 || std::get<2>(c) < std::get<2>(g_cache[best])))
-      best = i;
+  for (int pass = 0; pass < 2 && best < 0; ++pass) {
+    for (int i = 0; i < (int)g_cache.size(); ++i) {
+      const auto& c = g_cache[i];
+      if (std::get<0>(c) == dev && std::get<2>(c) >= bytes && (pass == 1 || std::get<3>(c) == slot) &&
+          (best < 0 || std::get<2>(c) < std::get<2>(g_cache[best])))
+        best = i;
+    }
   }
   if (best < 0) return nullptr;
   void* p = std::get<1>(g_cache[best]);
@@ -160,7 +164,7 @@ int32_t scratch_get(Handle& h, int slot, size_t bytes, void** out) {
       S.bytes[slot] = 0;
     }
     size_t got = 0;
-    void* c = cache_on() ? cache_take(h.device, bytes, &got) : nullptr;
+    void* c = cache_on() ? cache_take(h.device, slot, bytes, &got) : nullptr;
     if (c) {
       S.p[slot] = c;
       S.bytes[slot] = got;
@@ -184,12 +188,16 @@ int32_t scratch_get(Handle& h, int slot, size_t bytes, void** out) {
   return LOUVAIN_OK;
 }
 
+// Bounded: the cache holds one handle's set per device -- a destroy first frees what an
+// earlier handle left unused, then caches its own buffers.  With slot-keyed reuse the next
+// handle of the same graph takes every buffer back, so in the end-to-end loop of create /
+// run / destroy nothing is left over and a destroy frees nothing.
 void scratch_free(Handle& h) {
   std::lock_guard<std::mutex> lk(g_cache_mu);
-  if (cache_on()) cache_release_locked(h.device);  // bounded: one handle's set per device
+  if (cache_on()) cache_release_locked(h.device);
   for (int i = 0; i < SC_COUNT; ++i) {
     if (h.scratch.p[i]) {
-      if (cache_on()) g_cache.emplace_back(h.device, h.scratch.p[i], h.scratch.bytes[i]);
+      if (cache_on()) g_cache.emplace_back(h.device, h.scratch.p[i], h.scratch.bytes[i], i);
       else cudaFree(h.scratch.p[i]);
     }
     h.scratch.p[i] = nullptr;

@@ -161,20 +161,45 @@ __global__ void k_commit(DevCtl* ctl, int bucket, const int32_t* mv_v, const int
   if (blockIdx.x == 0 && threadIdx.x == 0) ctl->bounds[bucket + 1] = end;
   uint32_t* w32 = reinterpret_cast<uint32_t*>(ca);
   unsigned long long md = 0;
-  for (unsigned long long p = start + blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; p < end;
-       p += (unsigned long long)gridDim.x * blockDim.x) {
-    const int32_t i = mv_v[p], t = mv_new[p];
-    const int32_t old = (int32_t)w32[2 * (int64_t)i];
-    mv_old[p] = old;
-    w32[2 * (int64_t)i] = (uint32_t)t;
-    C[i] = t;
-    if (pcn) pcn[i].y = (uint32_t)t;
-    const uint32_t ki = k[i];
-    atomicSub(&w32[2 * (int64_t)old + 1], ki);
-    atomicAdd(&w32[2 * (int64_t)t + 1], ki);
-    atomicSub(&size[old], 1);
-    atomicAdd(&size[t], 1);
-    if (rowptr) md += (unsigned long long)(rowptr[i + 1] - rowptr[i]);
+  const int lane = threadIdx.x & 31;
+  // warp-uniform trips: moves into one community (a hub absorbing its degree-1
+  // neighbours) are summed per warp first, one atomic pair per distinct label
+  for (unsigned long long b = start + blockIdx.x * (unsigned long long)blockDim.x + (threadIdx.x - lane); b < end;
+       b += (unsigned long long)gridDim.x * blockDim.x) {
+    const unsigned long long p = b + lane;
+    const bool act = p < end;
+    int32_t i = 0, t = -1 - lane, old = -1 - lane;  // idle lanes: distinct negative labels
+    uint32_t ki = 0;
+    if (act) {
+      i = mv_v[p];
+      t = mv_new[p];
+      old = (int32_t)w32[2 * (int64_t)i];
+      mv_old[p] = old;
+      w32[2 * (int64_t)i] = (uint32_t)t;
+      C[i] = t;
+      if (pcn) pcn[i].y = (uint32_t)t;
+      ki = k[i];
+      if (rowptr) md += (unsigned long long)(rowptr[i + 1] - rowptr[i]);
+    }
+#pragma unroll
+    for (int side = 0; side < 2; ++side) {
+      const int32_t c = side ? old : t;
+      unsigned m = 1u << lane;
+      uint32_t x = ki;
+      if (__any_sync(kFull, c == __shfl_xor_sync(kFull, c, 1))) {
+        m = __match_any_sync(kFull, c);
+        x = __reduce_add_sync(m, ki);
+      }
+      if (c >= 0 && lane == __ffs(m) - 1) {
+        if (side) {
+          atomicSub(&w32[2 * (int64_t)c + 1], x);
+          atomicSub(&size[c], __popc(m));
+        } else {
+          atomicAdd(&w32[2 * (int64_t)c + 1], x);
+          atomicAdd(&size[c], __popc(m));
+        }
+      }
+    }
   }
   md = warp_sum_u64(md);
   if ((threadIdx.x & 31) == 0 && md) atomicAdd(&ctl->mdeg, md);

@@ -6,7 +6,7 @@ cd "$GRAFT_REPO_ROOT"; mkdir -p gpurun_out; O=gpurun_out/$1; shift; mkdir -p $O
 lib() { [ "$1" = tree ] && echo "" || echo "build/ab/$1/liblouvain.so"; }
 B="python bench.py --steps 5 --warmup 3 --no-cpu-baseline --e2e-steps 1 --e2e-warmup 0"
 for v in "$@"; do
-  if [ "$v" != tree ]; then
+  if [ "$v" != tree ] && [ -z "$ABN_NOTEST" ]; then
     LOUVAIN_LIB=$(lib $v) timeout 1200 python -m pytest tests/test_gpu_parity.py tests/test_gpu_fullsize.py -q -x \
       > $O/pytest_$v.log 2>&1; echo "rc=$?" >> $O/pytest_$v.log
   fi
