@@ -155,7 +155,14 @@ struct PartPlan {
   int64_t bucket_vsplit[8] = {0};  // bucket b's vertices [bucket_vert[b-1], vsplit) are pre-partitioned,
   int64_t bucket_tsplit[8] = {0};  // tasks [bucket_task[b-1], tsplit); the rest stream (P <= kStreamMaxP)
 };
-constexpr int64_t kStreamMaxP = 16;
+#ifndef LV_STREAM_MAXP  // compile-time A/B (tools/ab_build.py -D)
+#define LV_STREAM_MAXP 16
+#endif
+#ifndef LV_STREAM_MAXP_W
+#define LV_STREAM_MAXP_W 16
+#endif
+constexpr int64_t kStreamMaxP = LV_STREAM_MAXP;     // unit-weight level (level 0)
+constexpr int64_t kStreamMaxPW = LV_STREAM_MAXP_W;  // weighted (contracted) levels
 
 struct Level {
   int64_t n = 0, nnz = 0;

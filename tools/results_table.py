@@ -35,7 +35,7 @@ def main():
         rows.append("| {} | 1 | {} | {} | {} | {} | {:.4f} s ({:.1f} ms opt / {:.1f} ms agg, agg {:.0%}) | {:.6f} | {} | {} | yes (labels sha256 per sweep / run) | {} | {} |".format(
             NAMES[c], r(sw1), r(med) if med else "—",
             "n/a" if c == "C1" else f"{100 * frac:.1f}%",
-            f"{r(b['phase1_teps_2E'])} (2|E|) / {r(b['phase1_teps_E'])} (|E|)" if b.get("phase1_teps_2E") else "—",
+            f"{r(b['phase1_teps_2E'])} (2\\|E\\|) / {r(b['phase1_teps_E'])} (\\|E\\|)" if b.get("phase1_teps_2E") else "—",
             b["ms_per_step"] / 1e3, b["t_opt_ms"], b["t_agg_ms"], b["agg_share"] or 0, b["q_final"],
             f"{qa:.6f}" if qa is not None else "—", f"{abs(qa - b['q_final']):.4f}" if qa is not None else "—",
             f"{ots['sweep1_s']:.2f}" if "sweep1_s" in ots else (f"{g['level0_sweeps_b'][0]['oracle_s']:.2f} (build box)" if g.get('level0_sweeps_b') else "—"),
