@@ -162,9 +162,9 @@ __global__ void __launch_bounds__(256) k_scatter_copy(const int64_t* __restrict_
     // warp spans of 128 entries (lane + 32 q): one binary search per lane, then a
     // forward walk (the next entry of a lane is 32 further, mostly in the same row)
     const int lane = threadIdx.x & 31, wl = threadIdx.x >> 5, nw = blockDim.x >> 5;
-    for (int64_t span = e0 + (int64_t)wl * 128; span < e1; span += (int64_t)nw * 128) {
-      int32_t jj[4];
-      int64_t dd[4];
+    for (int64_t span = e0 + (int64_t)wl * 32 * kSpanQ; span < e1; span += (int64_t)nw * 32 * kSpanQ) {
+      int32_t jj[kSpanQ];
+      int64_t dd[kSpanQ];
       int lo = 0;
       if (nr > 0 && span + lane < e1) {
         int hi = nr - 1;  // largest r with sh_rp[r] <= e
@@ -175,7 +175,7 @@ __global__ void __launch_bounds__(256) k_scatter_copy(const int64_t* __restrict_
         }
       }
 #pragma unroll
-      for (int q = 0; q < 4; ++q) {
+      for (int q = 0; q < kSpanQ; ++q) {
         const int64_t e = span + lane + 32 * q;
         jj[q] = -1;
         dd[q] = 0;
@@ -199,11 +199,11 @@ __global__ void __launch_bounds__(256) k_scatter_copy(const int64_t* __restrict_
           jj[q] = __ldcs(&col[e]);
         }
       }
-      int32_t mm[4];
+      int32_t mm[kSpanQ];
 #pragma unroll
-      for (int q = 0; q < 4; ++q) mm[q] = jj[q] >= 0 ? __ldg(&map[jj[q]]) : 0;
+      for (int q = 0; q < kSpanQ; ++q) mm[q] = jj[q] >= 0 ? __ldg(&map[jj[q]]) : 0;
 #pragma unroll
-      for (int q = 0; q < 4; ++q) {
+      for (int q = 0; q < kSpanQ; ++q) {
         const int64_t e = span + lane + 32 * q;
         if (e < e1 && jj[q] >= 0) {
           gc[dd[q]] = mm[q];

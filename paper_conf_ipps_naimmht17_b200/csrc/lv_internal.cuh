@@ -155,14 +155,11 @@ struct PartPlan {
   int64_t bucket_vsplit[8] = {0};  // bucket b's vertices [bucket_vert[b-1], vsplit) are pre-partitioned,
   int64_t bucket_tsplit[8] = {0};  // tasks [bucket_task[b-1], tsplit); the rest stream (P <= kStreamMaxP)
 };
-#ifndef LV_STREAM_MAXP  // compile-time A/B (tools/ab_build.py -D)
-#define LV_STREAM_MAXP 16
+#ifndef LV_SPAN_Q  // compile-time A/B (tools/ab_build.py -D)
+#define LV_SPAN_Q 4
 #endif
-#ifndef LV_STREAM_MAXP_W
-#define LV_STREAM_MAXP_W 16
-#endif
-constexpr int64_t kStreamMaxP = LV_STREAM_MAXP;     // unit-weight level (level 0)
-constexpr int64_t kStreamMaxPW = LV_STREAM_MAXP_W;  // weighted (contracted) levels
+constexpr int kSpanQ = LV_SPAN_Q;  // entries per lane in flight in the warp-span tile kernels
+constexpr int64_t kStreamMaxP = 16;  // (4 at level 0, 1 at the weighted levels: measured no better, DESIGN 13)
 
 struct Level {
   int64_t n = 0, nnz = 0;

@@ -880,7 +880,7 @@ int32_t build_part_plan(Handle& h, Level& L) {
         tv.push_back(vi);
         tp.push_back(q);
       }
-      if (P > (L.w ? kStreamMaxPW : kStreamMaxP)) {  // pre-partitioned (a prefix: degrees descending)
+      if (P > kStreamMaxP) {  // pre-partitioned (a prefix: degrees descending)
         for (int64_t e = 0; e < deg; e += kPartChunk) ch.push_back(PartChunk{vi, 0, e, std::min(deg, e + kPartChunk)});
         Q.bucket_vsplit[b - 1] = (int64_t)vpos.size();
         Q.bucket_tsplit[b - 1] = (int64_t)tv.size();

@@ -342,9 +342,9 @@ __global__ void __launch_bounds__(256) k_stage(const int32_t* __restrict__ bv, c
     // entry, then a forward walk -- the next entry of a lane is 32 further, mostly in
     // the same row (the per-entry searches were most of this kernel's instructions)
     const int lane = threadIdx.x & 31, wl = threadIdx.x >> 5, nw = blockDim.x >> 5;
-    for (int64_t span = t0 + (int64_t)wl * 128; span < t1; span += (int64_t)nw * 128) {
-      int32_t jj[4], vv[4];
-      uint2 rr[4];
+    for (int64_t span = t0 + (int64_t)wl * 32 * kSpanQ; span < t1; span += (int64_t)nw * 32 * kSpanQ) {
+      int32_t jj[kSpanQ], vv[kSpanQ];
+      uint2 rr[kSpanQ];
       int lo = 0;
       if (nr > 0 && span + lane < t1) {
         int hi = nr - 1;
@@ -355,7 +355,7 @@ __global__ void __launch_bounds__(256) k_stage(const int32_t* __restrict__ bv, c
         }
       }
 #pragma unroll
-      for (int q = 0; q < 4; ++q) {
+      for (int q = 0; q < kSpanQ; ++q) {
         const int64_t t = span + lane + 32 * q;
         jj[q] = -1;
         vv[q] = -1;
@@ -378,9 +378,9 @@ __global__ void __launch_bounds__(256) k_stage(const int32_t* __restrict__ bv, c
         }
       }
 #pragma unroll
-      for (int q = 0; q < 4; ++q) rr[q] = (jj[q] >= 0 && jj[q] != vv[q]) ? __ldg(&ca[jj[q]]) : make_uint2(kSelf, 0);
+      for (int q = 0; q < kSpanQ; ++q) rr[q] = (jj[q] >= 0 && jj[q] != vv[q]) ? __ldg(&ca[jj[q]]) : make_uint2(kSelf, 0);
 #pragma unroll
-      for (int q = 0; q < 4; ++q) {
+      for (int q = 0; q < kSpanQ; ++q) {
         const int64_t t = span + lane + 32 * q;
         // evict-first store: the stage streams through L2 once and must not
         // displace the gathered records
