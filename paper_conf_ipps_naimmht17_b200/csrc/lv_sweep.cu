@@ -99,6 +99,43 @@ __device__ __forceinline__ void log_moves(bool mv, int32_t v, int32_t t, const S
   }
 }
 
+// Per-warp move buffer in shared memory: moves are collected warp-locally and appended to
+// the global log up to CAP at a time (one atomic per flush), instead of one atomic on the
+// single log counter per warp iteration -- in the register kernel of degree-1 vertices that
+// atomic was 43% of the stall samples (ncu, profiles/r02/final/ncu_small.sass.csv).  All
+// 32 lanes call add() and flush(); `n` is warp-uniform.
+template <int CAP>
+struct MoveBuf {
+  int32_t* v;
+  int32_t* t;
+  int n;
+  __device__ __forceinline__ void flush(const SweepArgs& A) {
+    if (n == 0) return;
+    const int lane = threadIdx.x & 31;
+    unsigned long long base = 0;
+    if (lane == 0) base = atomicAdd(A.logn, (unsigned long long)n);
+    base = __shfl_sync(kFull, base, 0);
+    __syncwarp();
+    for (int k = lane; k < n; k += 32) {
+      A.mv_v[base + k] = v[k];
+      A.mv_new[base + k] = t[k];
+    }
+    __syncwarp();
+    n = 0;
+  }
+  __device__ __forceinline__ void add(bool mv, int32_t vv, int32_t tt, const SweepArgs& A) {
+    const unsigned m = __ballot_sync(kFull, mv);
+    if (m == 0) return;
+    if (mv) {
+      const int pos = n + __popc(m & lanemask_lt());
+      v[pos] = vv;
+      t[pos] = tt;
+    }
+    n += __popc(m);
+    if (n > CAP - 32) flush(A);
+  }
+};
+
 // Candidate c (!= own) with accumulated weight e and total a_c: fold into (s, cb).
 __device__ __forceinline__ void consider(int32_t c, uint32_t e, uint32_t ac, int32_t own, bool own_single,
                                          uint32_t ki, const SweepArgs& A, long long& s, int& cb) {
@@ -119,13 +156,15 @@ __device__ __forceinline__ int32_t finish(long long s, int cb, uint32_t eown, in
 
 // ------------------------------------------------------------ deg <= 32
 template <int G, bool UNIT>
-__global__ void __launch_bounds__(256) sweep_small(const int32_t* __restrict__ verts, const int64_t* __restrict__ brb,
+__global__ void __launch_bounds__(256, 8) sweep_small(const int32_t* __restrict__ verts, const int64_t* __restrict__ brb,
                                                    const int64_t* __restrict__ soff, int64_t nv, SweepArgs A) {
   const int lane = threadIdx.x & 31;
   const int sub = lane & (G - 1);
   const unsigned gmask = (G == 32) ? kFull : (((1u << G) - 1u) << (lane & ~(G - 1)));
   const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
   const int64_t wid = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+  __shared__ int32_t mb_v[8][256], mb_t[8][256];  // 256 threads = 8 warps
+  MoveBuf<256> mb{mb_v[threadIdx.x >> 5], mb_t[threadIdx.x >> 5], 0};
   for (int64_t base = wid * (32 / G); base < nv; base += warps * (32 / G)) {
     const int64_t vi = base + lane / G;
     const bool active = vi < nv;
@@ -165,8 +204,9 @@ __global__ void __launch_bounds__(256) sweep_small(const int32_t* __restrict__ v
     group_reduce<G>(s, cb, eown);
     int32_t t = own;
     if (active && sub == 0 && cb != 0x7FFFFFFF) t = finish(s, cb, eown, own, __ldg(&A.ca[own]).y, ki, A);
-    log_moves(active && sub == 0 && t != own, v, t, A);
+    mb.add(active && sub == 0 && t != own, v, t, A);
   }
+  mb.flush(A);
 }
 
 // Table scan shared by the warp and CTA kernels: slots [t0, cap) step `stride`.
@@ -582,9 +622,11 @@ __global__ void __launch_bounds__(32 * WARPS) sweep_warp_d(const int32_t* __rest
                                                            SweepArgs A) {
   __shared__ unsigned long long tab[WARPS][CAP];
   __shared__ uint32_t taba[WARPS][CAP];
+  __shared__ int32_t mb_v[WARPS][64], mb_t[WARPS][64];
   const int lane = threadIdx.x & 31, wl = threadIdx.x >> 5;
   unsigned long long* T = tab[wl];
   uint32_t* TA = taba[wl];
+  MoveBuf<64> mb{mb_v[wl], mb_t[wl], 0};
   for (int t = lane; t < CAP; t += 32) {
     T[t] = kEmpty;
     TA[t] = kUnknownA;
@@ -608,9 +650,10 @@ __global__ void __launch_bounds__(32 * WARPS) sweep_warp_d(const int32_t* __rest
     group_reduce<32>(s, cb, eown);
     int32_t tgt = own;
     if (lane == 0) tgt = finish(s, cb, eown, own, __ldg(&A.ca[own]).y, ki, A);
-    log_moves(lane == 0 && tgt != own, v, tgt, A);
+    mb.add(lane == 0 && tgt != own, v, tgt, A);
     __syncwarp();
   }
+  mb.flush(A);
 }
 
 // Warp per vertex with register claims (rows of <= 128 * PASSES entries).
@@ -621,9 +664,11 @@ __global__ void __launch_bounds__(32 * WARPS) sweep_warp_c(const int32_t* __rest
                                                            const uint2* __restrict__ stage, SweepArgs A) {
   __shared__ unsigned long long tab[WARPS][CAP];
   __shared__ uint32_t taba[WARPS][CAP];
+  __shared__ int32_t mb_v[WARPS][64], mb_t[WARPS][64];
   const int lane = threadIdx.x & 31, wl = threadIdx.x >> 5;
   unsigned long long* T = tab[wl];
   uint32_t* TA = taba[wl];
+  MoveBuf<64> mb{mb_v[wl], mb_t[wl], 0};
   for (int t = lane; t < CAP; t += 32) {
     T[t] = kEmpty;
     TA[t] = kUnknownA;
@@ -647,9 +692,10 @@ __global__ void __launch_bounds__(32 * WARPS) sweep_warp_c(const int32_t* __rest
     group_reduce<32>(s, cb, eown);
     int32_t tgt = own;
     if (lane == 0) tgt = finish(s, cb, eown, own, __ldg(&A.ca[own]).y, ki, A);
-    log_moves(lane == 0 && tgt != own, v, tgt, A);
+    mb.add(lane == 0 && tgt != own, v, tgt, A);
     __syncwarp();
   }
+  mb.flush(A);
 }
 
 // CTA per vertex with register claims (rows of <= 4 * PASSES * blockDim entries).  The
@@ -666,6 +712,8 @@ __global__ void __launch_bounds__(1024, PASSES == 1 ? 2 : 1) sweep_cta_c(const i
   __shared__ long long sh_s[32];
   __shared__ int sh_c[32];
   __shared__ unsigned sh_e[32];
+  __shared__ int32_t mb_v[64], mb_t[64];  // warp 0's move buffer
+  MoveBuf<64> mb{mb_v, mb_t, 0};
   for (int t = threadIdx.x; t < capmax; t += blockDim.x) {
     T[t] = kEmpty;
     TA[t] = kUnknownA;
@@ -692,126 +740,12 @@ __global__ void __launch_bounds__(1024, PASSES == 1 ? 2 : 1) sweep_cta_c(const i
     if (threadIdx.x < 32) {
       int32_t tgt = own;
       if (threadIdx.x == 0) tgt = finish(s, cb, eown, own, __ldg(&A.ca[own]).y, ki, A);
-      log_moves(threadIdx.x == 0 && tgt != own, v, tgt, A);
+      mb.add(threadIdx.x == 0 && tgt != own, v, tgt, A);
     }
     __syncthreads();
   }
+  if (threadIdx.x < 32) mb.flush(A);
 }
-
-#ifdef LV_TMA
-// Compile-time experiment (tools/ab_build.py -DLV_TMA=1): the unit-weight single-pass CTA
-// tiers with the staged row of the NEXT vertex brought into shared memory by a 1-D bulk
-// copy (cp.async.bulk, TMA) while the current vertex is hashed, double-buffered with two
-// mbarriers; the inserts then read shared memory.  Rows are 8-byte aligned, bulk copies
-// need 16: the copy starts at the 16-byte boundary below the row (one record of slack).
-__device__ __forceinline__ uint32_t smem_addr(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
-__device__ __forceinline__ void bulk_row(uint2* buf, unsigned long long* bar, const uint2* stage, int64_t so,
-                                         int64_t deg) {
-  const int64_t a0 = so & ~1ll, a1 = (so + deg + 1) & ~1ll;  // records [a0, a1): 16-byte aligned
-  const uint32_t bytes = (uint32_t)((a1 - a0) * 8);
-  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_addr(bar)), "r"(bytes) : "memory");
-  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
-                   smem_addr(buf)),
-               "l"(stage + a0), "r"(bytes), "r"(smem_addr(bar))
-               : "memory");
-}
-__device__ __forceinline__ void bar_wait(unsigned long long* bar, uint32_t phase) {
-  uint32_t done = 0;
-  while (!done)
-    asm volatile(
-        "{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2; selp.u32 %0, 1, 0, p; }"
-        : "=r"(done)
-        : "r"(smem_addr(bar)), "r"(phase)
-        : "memory");
-}
-
-__global__ void __launch_bounds__(1024, 2) sweep_cta_tma(const int32_t* __restrict__ verts,
-                                                         const int64_t* __restrict__ brb,
-                                                         const int64_t* __restrict__ soff, int64_t nv,
-                                                         const uint2* __restrict__ stage, SweepArgs A, int capmax,
-                                                         int bufrec) {
-  extern __shared__ unsigned long long smem[];
-  unsigned long long* T = smem;
-  uint32_t* TA = reinterpret_cast<uint32_t*>(smem + capmax);
-  uint2* buf0 = reinterpret_cast<uint2*>(TA + capmax + (capmax & 3 ? 4 - (capmax & 3) : 0));
-  uint2* bufs[2] = {buf0, buf0 + bufrec};
-  __shared__ __align__(8) unsigned long long bars[2];
-  __shared__ long long sh_s[32];
-  __shared__ int sh_c[32];
-  __shared__ unsigned sh_e[32];
-  for (int t = threadIdx.x; t < capmax; t += blockDim.x) {
-    T[t] = kEmpty;
-    TA[t] = kUnknownA;
-  }
-  if (threadIdx.x == 0) {
-    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_addr(&bars[0])) : "memory");
-    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_addr(&bars[1])) : "memory");
-    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-  }
-  __syncthreads();
-  const int64_t G = gridDim.x;
-  if (threadIdx.x == 0 && blockIdx.x < nv) {
-    const int64_t so = __ldg(&soff[blockIdx.x]);
-    bulk_row(bufs[0], &bars[0], stage, so, __ldg(&soff[blockIdx.x + 1]) - so);
-  }
-  int it = 0;
-  for (int64_t vi = blockIdx.x; vi < nv; vi += G, ++it) {
-    const int b = it & 1;
-    const int32_t v = __ldg(&verts[vi]);
-    const int64_t rb = __ldg(&brb[vi]);
-    const int64_t so = __ldg(&soff[vi]);
-    const int64_t deg = __ldg(&soff[vi + 1]) - so;
-    const int32_t own = (int32_t)__ldg(&A.ca[v]).x;
-    const uint32_t ki = __ldg(&A.k[v]);
-    int64_t so_n = 0, deg_n = 0;
-    const bool has_next = vi + G < nv;
-    if (threadIdx.x == 0 && has_next) {  // next row's place, loaded early (used after the inserts)
-      so_n = __ldg(&soff[vi + G]);
-      deg_n = __ldg(&soff[vi + G + 1]) - so_n;
-    }
-    const int64_t want = 2 * deg + 1;
-    const uint32_t cap = (uint32_t)(want < (int64_t)capmax ? want : (int64_t)capmax);
-    bar_wait(&bars[b], (uint32_t)((it >> 1) & 1));
-    const uint2* S = bufs[b] + (so & 1);
-    uint32_t cl[4];
-    {
-      uint2 rr[4];
-#pragma unroll
-      for (int q = 0; q < 4; ++q) {
-        const int64_t t = (int64_t)threadIdx.x + (int64_t)q * blockDim.x;
-        rr[q] = (t < deg) ? S[t] : make_uint2(kSelf, 0u);
-      }
-#pragma unroll
-      for (int q = 0; q < 4; ++q) {
-        uint32_t slot = kNoClaim;
-        if (rr[q].x != kSelf) {
-          bool claimed = false;
-          const uint32_t hq = table_insert_c(T, cap, (int32_t)rr[q].x, 1u, &claimed);
-          if (rr[q].y != kUnknownA) TA[hq] = rr[q].y;
-          if (claimed) slot = hq;
-        }
-        cl[q] = slot;
-      }
-    }
-    __syncthreads();  // every read of bufs[b] done; bufs[b ^ 1] was read in the last iteration
-    if (threadIdx.x == 0 && has_next) bulk_row(bufs[b ^ 1], &bars[b ^ 1], stage, so_n, deg_n);
-    const bool own_single = A.rule == 2 && __ldg(&A.size[own]) == 1;
-    long long s = (long long)0x8000000000000000ull;
-    int cb = 0x7FFFFFFF;
-    unsigned eown = 0;
-    eval_claims<1>(T, TA, cl, own, own_single, ki, A, s, cb, eown);
-    block_reduce(s, cb, eown, sh_s, sh_c, sh_e);
-    if (threadIdx.x < 32) {
-      int32_t tgt = own;
-      if (threadIdx.x == 0) tgt = finish(s, cb, eown, own, __ldg(&A.ca[own]).y, ki, A);
-      log_moves(threadIdx.x == 0 && tgt != own, v, tgt, A);
-    }
-    __syncthreads();
-    (void)rb;
-  }
-}
-#endif
 
 // ------------------------------------------------------------ label-partitioned CTAs
 // deg >= 12288: vertex v gets P = ceil(deg / kPartLabels) independent CTA tasks;
@@ -1568,28 +1502,6 @@ int32_t dispatch_class(Handle& h, Level& L, const SweepArgs& A, int bucket, int 
         LV_CUDA(cudaGetLastError());
         return LOUVAIN_OK;
       };
-#ifdef LV_TMA
-      if (UNIT && passes <= 1) {
-        const int bufrec = (int)(((md + 2 + 1) / 2) * 2);  // records per buffer (even: 16-byte buffers)
-        const size_t sm = 12 * (size_t)capt + 16 + 2 * 8 * (size_t)bufrec;
-        static bool tattr = false;
-        if (!tattr) {
-          LV_TRY(set_smem(sweep_cta_tma, 12 * (size_t)8192 + 16 + 2 * 8 * (size_t)(kSub3Min + 2)));
-          tattr = true;
-        }
-        static int tres[5] = {0};
-        if (tres[sub] == 0) {
-          int nb = 0;
-          LV_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, sweep_cta_tma, threads[sub], sm));
-          tres[sub] = std::max(nb, 1);
-        }
-        sweep_cta_tma<<<grid_for(nv, 1, 148 * tres[sub]), threads[sub], sm, s>>>(verts, brb, soff, nv, stage, A, capt,
-                                                                                bufrec);
-        LV_LAUNCHED();
-        LV_CUDA(cudaGetLastError());
-        return LOUVAIN_OK;
-      }
-#endif
       if (passes <= 1) return go(sweep_cta_c<UNIT, 1>);
       if (passes == 2) return go(sweep_cta_c<UNIT, 2>);
       if (passes == 3) return go(sweep_cta_c<UNIT, 3>);

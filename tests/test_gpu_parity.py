@@ -316,6 +316,27 @@ def test_device_inputs_and_borrow():
         assert np.array_equal(out.cpu().numpy(), r.labels)
 
 
+def test_handle_churn_reuses_cached_scratch():
+    """create / run / destroy in a loop (the e2e bench step): results stay bit-exact, and
+    the scratch cache is bounded -- after the first handle, device memory in use does not
+    grow from one iteration to the next (each buffer goes back to the slot it served);
+    louvain_release_cache() gives it back."""
+    torch = pytest.importorskip("torch")
+    g = GRAPHS["giant_hub"]()
+    r = oracle.louvain(g)
+    free = []
+    for it in range(4):
+        gd = lvb.Graph.from_csr(g.rowptr, g.col, g.w)
+        lab, q, st = gd.run(lvb.params())
+        assert np.array_equal(lab, r.labels)
+        gd.close()
+        torch.cuda.synchronize()
+        free.append(torch.cuda.mem_get_info()[0])
+    assert max(free[1:]) - min(free[1:]) <= 64 << 20, free  # steady state: no growth, no churn
+    lvb.release_cache()
+    assert torch.cuda.mem_get_info()[0] >= free[-1]
+
+
 def test_validate_on_device_inputs():
     torch = pytest.importorskip("torch")
     rp = torch.tensor([0, 1, 1], dtype=torch.int64, device="cuda")
