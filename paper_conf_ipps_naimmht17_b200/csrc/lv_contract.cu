@@ -244,6 +244,32 @@ __global__ void __launch_bounds__(256) k_merge_small(const int32_t* __restrict__
 }
 
 // Step 4b: segments of 33..512 entries, one warp each with a 1024-slot smem table.
+// One entry t of the segment at gc/gw + b into a smem table (all 32 lanes of the warp
+// call it; t >= len idles): when adjacent entries repeat a neighbour, the warp's copies of
+// each neighbour are summed first (group_sum: one table atomic per neighbour and warp --
+// the members of a community mostly point at a few communities; same-slot atomics serialise).
+__device__ __forceinline__ void merge_insert(unsigned long long* T, uint32_t cap, const int32_t* __restrict__ gc,
+                                             const uint32_t* __restrict__ gw, int64_t b, int64_t t, int64_t len) {
+  const int lane = threadIdx.x & 31;
+  const bool has = t < len;
+  const int32_t c = has ? gc[b + t] : (int32_t)(0x80000000u | (unsigned)lane);
+  uint32_t x = has ? (gw ? gw[b + t] : 1u) : 0u;
+  unsigned m = 1u << lane;
+  if (__any_sync(kFull, c == __shfl_xor_sync(kFull, c, 1))) group_sum((uint32_t)c, x, m);  // adaptive
+  if (!has || lane != __ffs(m) - 1) return;
+  const unsigned long long key = ((unsigned long long)(uint32_t)c) << 32;
+  uint32_t h = hash_slot(c, cap);
+  for (;;) {
+    const unsigned long long old = atomicCAS(&T[h], kEmpty, key | x);
+    if (old == kEmpty) break;
+    if ((old >> 32) == (unsigned long long)(uint32_t)c) {
+      atomicAdd(&T[h], (unsigned long long)x);
+      break;
+    }
+    h = (h + 1 == cap) ? 0 : h + 1;
+  }
+}
+
 template <int SLOTS>
 __global__ void __launch_bounds__(128) k_merge_warp(const int32_t* __restrict__ rows, int64_t nr,
                                                     const int64_t* __restrict__ sstart,
@@ -260,21 +286,7 @@ __global__ void __launch_bounds__(128) k_merge_warp(const int32_t* __restrict__ 
     const int32_t r = rows[k];
     const int64_t b = sstart[r], len = send_[r] - b;
     const uint32_t cap = (uint32_t)(2 * len);
-    for (int64_t t = lane; t < len; t += 32) {
-      const int32_t c = gc[b + t];
-      const uint32_t x = gw ? gw[b + t] : 1u;
-      const unsigned long long key = ((unsigned long long)(uint32_t)c) << 32;
-      uint32_t h = hash_slot(c, cap);
-      for (;;) {
-        const unsigned long long old = atomicCAS(&T[h], kEmpty, key | x);
-        if (old == kEmpty) break;
-        if ((old >> 32) == (unsigned long long)(uint32_t)c) {
-          atomicAdd(&T[h], (unsigned long long)x);
-          break;
-        }
-        h = (h + 1 == cap) ? 0 : h + 1;
-      }
-    }
+    for (int64_t t0 = 0; t0 < len; t0 += 32) merge_insert(T, cap, gc, gw, b, t0 + lane, len);
     __syncwarp();
     int base = 0;
     for (uint32_t t0 = 0; t0 < cap; t0 += 32) {
@@ -310,21 +322,8 @@ __global__ void __launch_bounds__(512) k_merge_mid(const int32_t* __restrict__ r
     const int32_t r = rows[k];
     const int64_t b = sstart[r], len = send_[r] - b;
     const uint32_t cap = (uint32_t)((2 * len < (int64_t)capmax) ? 2 * len : (int64_t)capmax);
-    for (int64_t t = threadIdx.x; t < len; t += blockDim.x) {
-      const int32_t c = gc[b + t];
-      const uint32_t x = gw ? gw[b + t] : 1u;
-      const unsigned long long key = ((unsigned long long)(uint32_t)c) << 32;
-      uint32_t h = hash_slot(c, cap);
-      for (;;) {
-        const unsigned long long old = atomicCAS(&T[h], kEmpty, key | x);
-        if (old == kEmpty) break;
-        if ((old >> 32) == (unsigned long long)(uint32_t)c) {
-          atomicAdd(&T[h], (unsigned long long)x);
-          break;
-        }
-        h = (h + 1 == cap) ? 0 : h + 1;
-      }
-    }
+    for (int64_t tb = threadIdx.x & ~31; tb < len; tb += blockDim.x)  // warp-uniform trips
+      merge_insert(T, cap, gc, gw, b, tb + (threadIdx.x & 31), len);
     __syncthreads();
     // distinct keys appended with one shared atomic per warp and pass (not per key:
     // a single counter serialised every key of the CTA)

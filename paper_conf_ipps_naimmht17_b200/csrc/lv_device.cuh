@@ -41,6 +41,15 @@ __device__ __forceinline__ void table_add(unsigned long long* T, uint32_t cap, i
   }
 }
 
+// Sums x over the lanes holding the same key (all 32 lanes call it; idle lanes need keys of
+// their own): m = the lane's group, the group's lowest lane gets the sum in x.  (The
+// hardware serialises REDUX over the distinct group masks; a bounded loop of full-warp
+// reductions measured slower: DESIGN 13.)
+__device__ __forceinline__ void group_sum(uint32_t key, uint32_t& x, unsigned& m) {
+  m = __match_any_sync(kFull, key);
+  x = __reduce_add_sync(m, x);
+}
+
 // Partition of label c among P label-partitioned tasks: fmix32 (independent of
 // hash_slot's multiplier) scaled to [0, P).
 __device__ __forceinline__ uint32_t part_of(int32_t c, uint32_t P) {

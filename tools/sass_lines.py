@@ -48,7 +48,10 @@ def main():
     for r in rows[2:]:
         if len(r) < len(hdr):
             continue
-        a = int(r[ix["Address"]], 16)
+        try:
+            a = int(r[ix["Address"]], 16)
+        except ValueError:  # the next kernel's section (several launches in one file): first only
+            break
         base = a if base is None else base
         off = a - base
         ln = lm.get(off, "?")
