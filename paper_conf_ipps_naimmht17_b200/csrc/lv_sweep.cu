@@ -1439,6 +1439,9 @@ int32_t launch_part(Handle& h, Level& L, const SweepArgs& A, int bucket, bool un
 // that gathers the records itself (sweep_warp_d): C5 level 0 bucket 5 stage 2.8 + warp 2.2 ->
 // 4.0 ms; bucket 6 (85-319) measured slower that way (6.5 -> 7.6 ms) and keeps the stage.
 constexpr int64_t kDirectMaxDeg = 84;
+#ifndef LV_WARPD_CAP  // table slots per warp of the direct bucket-5 kernel (256: load <= 1/3; 128 measured slower)
+#define LV_WARPD_CAP 256
+#endif
 // largest degree of CTA tier `sub` (lv_internal.cuh)
 static int64_t max_deg_of_tier(int sub) {
   static const int64_t ub[5] = {kSub1Min - 1, kSub2Min - 1, kSub3Min - 1, kSub4Min - 1, kSub5Min - 1};
@@ -1466,7 +1469,7 @@ int32_t dispatch_class(Handle& h, Level& L, const SweepArgs& A, int bucket, int 
     }
     LV_LAUNCHED();
   } else if (sub == 0 && max_deg <= kDirectMaxDeg) {
-    sweep_warp_d<128, 8, UNIT, 1><<<grid_for(nv, 8, 148 * 8), 256, 0, s>>>(verts, brb, soff, nv, A);
+    sweep_warp_d<LV_WARPD_CAP, 8, UNIT, 1><<<grid_for(nv, 8, 148 * 8), 256, 0, s>>>(verts, brb, soff, nv, A);
     LV_LAUNCHED();
   } else if (sub == 0 && max_deg <= 340) {  // warp per vertex, 3 claim passes of 4 entries per lane
     sweep_warp_c<512, 4, UNIT, 3><<<grid_for(nv, 4, 148 * 8), 128, 0, s>>>(verts, brb, soff, nv, stage, A);
