@@ -498,10 +498,19 @@ __device__ __forceinline__ void insert_staged(unsigned long long* T, uint32_t* T
 // Covers rows of up to 4 * PASSES * stride entries.
 constexpr uint32_t kNoClaim = 0xFFFFFFFFu;
 
+#ifndef LV_DOUBLE_HASH  // compile-time A/B
+#define LV_DOUBLE_HASH 1
+#endif
 __device__ __forceinline__ uint32_t table_insert_c(unsigned long long* T, uint32_t cap, int32_t c, uint32_t x,
                                                    bool* claimed) {
   const unsigned long long key = ((unsigned long long)(uint32_t)c) << 32;
   uint32_t h = hash_slot(c, cap);
+#if LV_DOUBLE_HASH
+  // double hashing on power-of-two tables (odd step: a full cycle): no primary clusters,
+  // so the longest probe chain of a warp -- what its divergent loop waits for -- shortens
+  const bool pow2 = (cap & (cap - 1)) == 0;
+  const uint32_t step = (((uint32_t)c * 0x85EBCA6Bu) >> 17) | 1u;  // independent of hash_slot's bits
+#endif
   for (;;) {
     const unsigned long long old = atomicCAS(&T[h], kEmpty, key | x);
     if (old == kEmpty) {
@@ -513,7 +522,11 @@ __device__ __forceinline__ uint32_t table_insert_c(unsigned long long* T, uint32
       *claimed = false;
       return h;
     }
+#if LV_DOUBLE_HASH
+    h = pow2 ? ((h + step) & (cap - 1)) : ((h + 1 == cap) ? 0 : h + 1);
+#else
     h = (h + 1 == cap) ? 0 : h + 1;
+#endif
   }
 }
 
