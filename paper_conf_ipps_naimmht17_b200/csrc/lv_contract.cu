@@ -124,6 +124,12 @@ __global__ void k_dest_base(const int32_t* __restrict__ vorder, const int64_t* _
     dbase[vorder[i]] = gpos[i];
 }
 
+#ifndef LV_DH_CONTRACT  // compile-time A/B: double hashing in the power-of-two contraction tables
+#define LV_DH_CONTRACT 1
+#endif
+#ifndef LV_DH_POW2  // compile-time A/B: merge / hub-task tables rounded up to powers of two + double hashing
+#define LV_DH_POW2 1
+#endif
 constexpr int kSTile = 4096;  // CSR entries per scatter-copy tile
 constexpr int kSRows = 1024;  // rows staged per tile (else per-entry search in global memory)
 template <bool RANGE>  // RANGE: sharded contraction, only rows whose new vertex is in [c_lo, c_hi)
@@ -266,7 +272,11 @@ __device__ __forceinline__ void merge_insert(unsigned long long* T, uint32_t cap
       atomicAdd(&T[h], (unsigned long long)x);
       break;
     }
+#if LV_DH_POW2
+    h = probe_next(h, cap, probe_step(c));
+#else
     h = (h + 1 == cap) ? 0 : h + 1;
+#endif
   }
 }
 
@@ -285,7 +295,11 @@ __global__ void __launch_bounds__(128) k_merge_warp(const int32_t* __restrict__ 
   for (int64_t k = (int64_t)blockIdx.x * 4 + wl; k < nr; k += warps) {
     const int32_t r = rows[k];
     const int64_t b = sstart[r], len = send_[r] - b;
+#if LV_DH_POW2
+    const uint32_t cap = pow2_at_least((uint32_t)(2 * len), SLOTS);
+#else
     const uint32_t cap = (uint32_t)(2 * len);
+#endif
     for (int64_t t0 = 0; t0 < len; t0 += 32) merge_insert(T, cap, gc, gw, b, t0 + lane, len);
     __syncwarp();
     int base = 0;
@@ -321,7 +335,12 @@ __global__ void __launch_bounds__(512) k_merge_mid(const int32_t* __restrict__ r
   for (int64_t k = blockIdx.x; k < nr; k += gridDim.x) {
     const int32_t r = rows[k];
     const int64_t b = sstart[r], len = send_[r] - b;
+#if LV_DH_POW2
+    const uint32_t cap = (2 * len < (int64_t)capmax) ? pow2_at_least((uint32_t)(2 * len), (uint32_t)capmax)
+                                                     : (uint32_t)capmax;
+#else
     const uint32_t cap = (uint32_t)((2 * len < (int64_t)capmax) ? 2 * len : (int64_t)capmax);
+#endif
     for (int64_t tb = threadIdx.x & ~31; tb < len; tb += blockDim.x)  // warp-uniform trips
       merge_insert(T, cap, gc, gw, b, tb + (threadIdx.x & 31), len);
     __syncthreads();
@@ -459,7 +478,11 @@ __global__ void __launch_bounds__(THREADS) k_big_combine(const uint32_t* __restr
             atomicAdd(&T[h], (unsigned long long)v[q]);
             break;
           }
+#if LV_DH_CONTRACT
+          h = (h + probe_step((int32_t)k[q])) & (SLOTS - 1);
+#else
           h = (h + 1) & (SLOTS - 1);
+#endif
         }
         pass[q] = pr == kCombProbes;
       }
@@ -739,7 +762,11 @@ __global__ void __launch_bounds__(1024) k_bigp_merge(const int64_t* __restrict__
               h = 0xFFFFFFFFu;
               break;
             }
+#if LV_DH_CONTRACT
+            h = probe_next(h, cap, probe_step(cc[u]));
+#else
             h = (h + 1 == cap) ? 0 : h + 1;
+#endif
           }
         }
         const unsigned cm = __ballot_sync(kFull, h != 0xFFFFFFFFu);

@@ -50,6 +50,20 @@ __device__ __forceinline__ void group_sum(uint32_t key, uint32_t& x, unsigned& m
   x = __reduce_add_sync(m, x);
 }
 
+// Probe sequence of the open-addressing tables: double hashing (an odd step from a multiplier
+// independent of hash_slot's) on power-of-two tables -- no primary clusters, so the longest
+// chain in a warp's divergent probe loop shortens -- linear otherwise.
+__device__ __forceinline__ uint32_t probe_step(int32_t c) { return (((uint32_t)c * 0x85EBCA6Bu) >> 17) | 1u; }
+__device__ __forceinline__ uint32_t probe_next(uint32_t h, uint32_t cap, uint32_t step) {
+  return ((cap & (cap - 1)) == 0) ? ((h + step) & (cap - 1)) : ((h + 1 == cap) ? 0 : h + 1);
+}
+// Smallest power of two >= x (x >= 1), capped at lim (a power of two).
+__device__ __forceinline__ uint32_t pow2_at_least(uint32_t x, uint32_t lim) {
+  uint32_t p = 1;
+  while (p < x && p < lim) p <<= 1;
+  return p;
+}
+
 // Partition of label c among P label-partitioned tasks: fmix32 (independent of
 // hash_slot's multiplier) scaled to [0, P).
 __device__ __forceinline__ uint32_t part_of(int32_t c, uint32_t P) {

@@ -501,6 +501,9 @@ constexpr uint32_t kNoClaim = 0xFFFFFFFFu;
 #ifndef LV_DOUBLE_HASH  // compile-time A/B
 #define LV_DOUBLE_HASH 1
 #endif
+#ifndef LV_DH_POW2  // compile-time A/B: hub-task tables rounded up to powers of two + double hashing
+#define LV_DH_POW2 1
+#endif
 __device__ __forceinline__ uint32_t table_insert_c(unsigned long long* T, uint32_t cap, int32_t c, uint32_t x,
                                                    bool* claimed) {
   const unsigned long long key = ((unsigned long long)(uint32_t)c) << 32;
@@ -994,7 +997,11 @@ __global__ void __launch_bounds__(1024) sweep_part_stream(const int32_t* __restr
     // table sized to the task: ~2x its expected labels (deg / P) + slack, so the
     // scan visits ~2 slots per label instead of all kPartSlots (C5 level 0: the
     // full-table scans were most of this kernel's work)
+#if LV_DH_POW2
+    const uint32_t cap = pow2_at_least((uint32_t)min((int64_t)kPartSlots, 2 * ((deg + P - 1) / P) + 512), kPartSlots);
+#else
     const uint32_t cap = (uint32_t)min((int64_t)kPartSlots, 2 * ((deg + P - 1) / P) + 512);
+#endif
     const unsigned limit = cap / 8 * 7;
     // Only ~1/P of the streamed entries belong to this task: each warp compacts
     // the matching entries into a shared queue (ballot + popc) and inserts them
@@ -1022,7 +1029,11 @@ __global__ void __launch_bounds__(1024) sweep_part_stream(const int32_t* __restr
           atomicAdd(&T[h], (unsigned long long)x);
           break;
         }
+#if LV_DH_POW2
+        h = probe_next(h, cap, probe_step(c));
+#else
         h = (h + 1 == cap) ? 0 : h + 1;
+#endif
       }
       if (e.y != kUnknownA) TA[h] = e.y;
     };
