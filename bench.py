@@ -397,6 +397,7 @@ def run_sharded_bench(args, rank, world):
     edges_per_run = st0["edges_swept"]
     roofline = roofline_of(args, n_act, nnz, st0, t_sw1, world)
     del g
+    lvb.release_cache()  # the e2e loop starts from an empty library cache (see run_ours)
     # end to end: every rank uploads its rows from pinned host memory, runs, reads the labels back
     h_rl = torch.empty(rl.numel(), dtype=torch.int64, pin_memory=True)
     h_cl = torch.empty(cl.numel(), dtype=torch.int32, pin_memory=True)
@@ -526,6 +527,11 @@ def run_ours(args, rank, world):
     h_col.copy_(dg.col)
     del g
     torch.cuda.synchronize()
+    # start the e2e loop from an empty library cache: the steady state (each step's handle
+    # takes back the previous step's buffers, slot by slot) then does not depend on what the
+    # device-resident bench handle above left behind
+    lvb.release_cache()
+    torch.cuda.empty_cache()
     parts = []
     for it in range(max(0, args.e2e_warmup) + max(1, args.e2e_steps)):
         if world > 1:

@@ -51,7 +51,10 @@ constexpr int kNumClasses = 8 * kSubPerBucket;
 constexpr int kSubPart = 5, kSubHub = 7;  // first partitioned sub-class, hub sub-class
 constexpr int64_t kSub1Min = 512, kSub2Min = 1024, kSub3Min = 2048, kSub4Min = 4096, kSub5Min = 12288,
                   kSub6Min = 32768, kHubMin = 393216;
-constexpr int kCapT[5] = {2048, 4096, 8192, 16384, 18432};  // max smem table slots (12 B each) of sub 0..4
+#ifndef LV_TIER4_SLOTS  // compile-time A/B (16384: a power of two, double hashing)
+#define LV_TIER4_SLOTS 16384
+#endif
+constexpr int kCapT[5] = {2048, 4096, 8192, 16384, LV_TIER4_SLOTS};  // max smem table slots (12 B each) of sub 0..4
 constexpr int kThrT[5] = {128, 256, 512, 512, 1024};
 constexpr int kPerSmT[5] = {16, 8, 4, 2, 1};
 constexpr int kCapMax = 18432;

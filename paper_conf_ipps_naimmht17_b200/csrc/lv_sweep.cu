@@ -504,6 +504,9 @@ constexpr uint32_t kNoClaim = 0xFFFFFFFFu;
 #ifndef LV_DH_POW2  // compile-time A/B: hub-task tables rounded up to powers of two + double hashing
 #define LV_DH_POW2 1
 #endif
+#ifndef LV_DH_PART  // compile-time A/B: the same for the pre-partitioned hub tasks
+#define LV_DH_PART 1
+#endif
 __device__ __forceinline__ uint32_t table_insert_c(unsigned long long* T, uint32_t cap, int32_t c, uint32_t x,
                                                    bool* claimed) {
   const unsigned long long key = ((unsigned long long)(uint32_t)c) << 32;
@@ -942,7 +945,11 @@ __device__ __forceinline__ unsigned part_insert(unsigned long long* T, uint32_t*
             atomicAdd(&T[hq], (unsigned long long)x);
             break;
           }
+#if LV_DH_PART
+          hq = probe_next(hq, cap, probe_step(c));
+#else
           hq = (hq + 1 == cap) ? 0 : hq + 1;
+#endif
           if (probes >= cap) { hq = 0xFFFFFFFFu; break; }  // full table (only possible when counting)
         }
         if (rep && hq != 0xFFFFFFFFu) TA[hq] = a_rep;
@@ -1175,7 +1182,11 @@ __global__ void __launch_bounds__(1024) sweep_part(const int32_t* __restrict__ t
     const int64_t q0 = poff[pb + p], q1 = poff[pb + p + 1];
     const int64_t n_p = q1 - q0;
     const bool big = 2 * n_p > kPartSlots;
+#if LV_DH_PART
+    const uint32_t cap = big ? (uint32_t)kPartSlots : pow2_at_least((uint32_t)(n_p > 0 ? 2 * n_p : 1), kPartSlots);
+#else
     const uint32_t cap = big ? (uint32_t)kPartSlots : (uint32_t)(n_p > 0 ? 2 * n_p : 1);
+#endif
     const unsigned cl = part_insert<UNIT, AGG>(T, TA, cap, S2, UNIT ? nullptr : W2, q0, q1, big);
     if (big && (threadIdx.x & 31) == 0 && cl) atomicAdd(&claimed, cl);
     __syncthreads();
