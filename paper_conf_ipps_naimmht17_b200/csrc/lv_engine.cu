@@ -279,6 +279,15 @@ int32_t init_handle(Handle& h, void* stream) {
 }
 
 void destroy_handle(Handle& h) {
+  // LV_TRACE: where a destroy's time goes (diagnostics only)
+  static const bool tr = getenv("LV_TRACE") != nullptr;
+  auto t0 = std::chrono::steady_clock::now();
+  auto mark = [&](const char* what) {
+    if (!tr) return;
+    const auto t1 = std::chrono::steady_clock::now();
+    fprintf(stderr, "[lv] destroy %-12s %8.3f ms\n", what, std::chrono::duration<double, std::milli>(t1 - t0).count());
+    t0 = t1;
+  };
   cudaSetDevice(h.device);
   dist_free(h);
   if (h.stream) {
@@ -289,9 +298,21 @@ void destroy_handle(Handle& h) {
     level_free(h.lv, h.stream);
     cudaStreamSynchronize(h.stream);
   }
+  mark("level");
+  if (tr) {
+    size_t mine = 0, cached = 0;
+    for (int i = 0; i < SC_COUNT; ++i) mine += h.scratch.bytes[i];
+    {
+      std::lock_guard<std::mutex> lk(g_cache_mu);
+      for (const auto& c : g_cache) cached += std::get<2>(c);
+    }
+    fprintf(stderr, "[lv] destroy scratch %.2f GB, cache before %.2f GB\n", mine / 1e9, cached / 1e9);
+  }
   scratch_free(h);
+  mark("scratch");
   if (h.ctl) cudaFree(h.ctl);
   if (h.h_ctl) cudaFreeHost(h.h_ctl);
+  mark("ctl");
   for (auto& e : h.ev)
     if (e) cudaEventDestroy(e);
   if (h.side) {
