@@ -55,10 +55,7 @@ constexpr int64_t kSub1Min = 512, kSub2Min = 1024, kSub3Min = 2048, kSub4Min = 4
 #define LV_TIER4_SLOTS 16384
 #endif
 constexpr int kCapT[5] = {2048, 4096, 8192, 16384, LV_TIER4_SLOTS};  // max smem table slots (12 B each) of sub 0..4
-#ifndef LV_TIER3_THREADS  // compile-time A/B
-#define LV_TIER3_THREADS 512
-#endif
-constexpr int kThrT[5] = {128, 256, 512, LV_TIER3_THREADS, 1024};
+constexpr int kThrT[5] = {128, 256, 512, 512, 1024};  // (tier 3 with 1024: slower at level 2, DESIGN 13)
 constexpr int kPerSmT[5] = {16, 8, 4, 2, 1};
 constexpr int kCapMax = 18432;
 // Buckets whose degree bound is <= kSmallMaxDeg (1-4 with the paper's bounds) run the

@@ -677,10 +677,7 @@ __global__ void __launch_bounds__(32 * WARPS) sweep_warp_d(const int32_t* __rest
 
 // Warp per vertex with register claims (rows of <= 128 * PASSES entries).
 template <int CAP, int WARPS, bool UNIT, int PASSES>
-#ifndef LV_WARPC_MINB  // compile-time A/B: minimum resident blocks of the bucket-6 warp kernel
-#define LV_WARPC_MINB 1
-#endif
-__global__ void __launch_bounds__(32 * WARPS, LV_WARPC_MINB) sweep_warp_c(const int32_t* __restrict__ verts,
+__global__ void __launch_bounds__(32 * WARPS) sweep_warp_c(const int32_t* __restrict__ verts,
                                                            const int64_t* __restrict__ brb,
                                                            const int64_t* __restrict__ soff, int64_t nv,
                                                            const uint2* __restrict__ stage, SweepArgs A) {
