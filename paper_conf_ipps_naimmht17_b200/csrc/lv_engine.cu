@@ -205,7 +205,41 @@ void scratch_free(Handle& h) {
   }
 }
 
+// Control blocks (device DevCtl + its pinned host mirror) of destroyed handles, reused by the
+// next handles: a cudaFree / cudaFreeHost per destroy synchronised the device and cost up
+// to 0.66 s inside the end-to-end step (LV_TRACE destroy timing).
+std::mutex g_ctl_mu;
+std::vector<std::tuple<int, DevCtl*, DevCtl*>> g_ctl_free;
+bool ctl_take(int dev, DevCtl** d, DevCtl** hh) {
+  std::lock_guard<std::mutex> lk(g_ctl_mu);
+  for (auto it = g_ctl_free.begin(); it != g_ctl_free.end(); ++it)
+    if (std::get<0>(*it) == dev) {
+      *d = std::get<1>(*it);
+      *hh = std::get<2>(*it);
+      g_ctl_free.erase(it);
+      return true;
+    }
+  return false;
+}
+void ctl_give(int dev, DevCtl* d, DevCtl* hh) {
+  std::lock_guard<std::mutex> lk(g_ctl_mu);
+  g_ctl_free.emplace_back(dev, d, hh);
+}
+void ctl_release_all() {
+  std::lock_guard<std::mutex> lk(g_ctl_mu);
+  for (auto& c : g_ctl_free) {
+    int cur = -1;
+    cudaGetDevice(&cur);
+    cudaSetDevice(std::get<0>(c));
+    cudaFree(std::get<1>(c));
+    cudaFreeHost(std::get<2>(c));
+    if (cur >= 0) cudaSetDevice(cur);
+  }
+  g_ctl_free.clear();
+}
+
 void release_cache_all() {
+  ctl_release_all();
   cache_release(-1);
   for (int d = 0; d < 64; ++d) {
     cudaMemPool_t p = nullptr;
@@ -267,9 +301,11 @@ int32_t init_handle(Handle& h, void* stream) {
     LV_CUDA(cudaStreamCreateWithFlags(&h.stream, cudaStreamNonBlocking));
     h.own_stream = true;
   }
-  LV_CUDA(cudaMalloc(&h.ctl, sizeof(DevCtl)));
+  if (!ctl_take(h.device, &h.ctl, &h.h_ctl)) {
+    LV_CUDA(cudaMalloc(&h.ctl, sizeof(DevCtl)));
+    LV_CUDA(cudaMallocHost(&h.h_ctl, sizeof(DevCtl)));
+  }
   LV_CUDA(cudaMemset(h.ctl, 0, sizeof(DevCtl)));
-  LV_CUDA(cudaMallocHost(&h.h_ctl, sizeof(DevCtl)));
   for (auto& e : h.ev) LV_CUDA(cudaEventCreate(&e));
   LV_CUDA(cudaStreamCreateWithFlags(&h.side, cudaStreamNonBlocking));
   LV_CUDA(cudaEventCreateWithFlags(&h.ev_fork, cudaEventDisableTiming));
@@ -310,8 +346,9 @@ void destroy_handle(Handle& h) {
   }
   scratch_free(h);
   mark("scratch");
-  if (h.ctl) cudaFree(h.ctl);
-  if (h.h_ctl) cudaFreeHost(h.h_ctl);
+  if (h.ctl) ctl_give(h.device, h.ctl, h.h_ctl);  // kept for the next handle (no cudaFree:
+  h.ctl = nullptr;                                  // it synchronised the device for up to
+  h.h_ctl = nullptr;                                // 0.66 s per destroy, LV_TRACE)
   mark("ctl");
   for (auto& e : h.ev)
     if (e) cudaEventDestroy(e);
