@@ -130,7 +130,10 @@ struct HubPlan {
 // chunks of kPartChunk entries), so task p reads only its own share and keeps
 // it in one shared-memory table.  Vertices with P_v > kPartMaxP (deg > 50 M)
 // go to the cooperative hub kernel instead.
-constexpr int64_t kPartLabels = 10240;  // expected labels per task (table load ~5/8; C5: 6144 / 8192 / 10240 / 12288 -> 28.3 / 22.2 / 21.4 / 21.0 ms at level 0)
+#ifndef LV_PART_LABELS  // compile-time A/B
+#define LV_PART_LABELS 12288
+#endif
+constexpr int64_t kPartLabels = LV_PART_LABELS;  // expected labels per task (table load ~3/4 with double hashing, overflow check at 7/8; r1: 6144 / 8192 / 10240 / 12288 -> 28.3 / 22.2 / 21.4 / 21.0 ms at level 0; r2 12288 vs 10240: run -1.7 ms)
 constexpr int kPartSlots = 16384;      // smem table slots per task (12 B each: 192 KB)
 constexpr int kPartMaxP = 8192;        // partitions per vertex (smem histogram of a chunk)
 constexpr int64_t kPartChunk = 32768;  // staged entries per histogram / scatter item
