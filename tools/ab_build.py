@@ -8,6 +8,7 @@ Run the other arm with LOUVAIN_LIB=build/ab/NAME/liblouvain.so (paper_conf_ipps_
 loads that file instead of the in-tree build).  The C-ABI header is taken from the working tree.
 """
 import os
+import shutil
 import subprocess
 import sys
 
@@ -38,6 +39,9 @@ def main():
     out = os.path.join(ROOT, "build", "ab", name, "liblouvain.so")
     build.build_louvain(force=True, d=src, out=out, objdir=os.path.join(ROOT, "build", "ab", name, "obj"),
                         defines=defines)
+    # only the library travels to the GPU box (gpurun snapshots are capped at 512 MiB)
+    shutil.rmtree(os.path.join(ROOT, "build", "ab", name, "obj"), ignore_errors=True)
+    shutil.rmtree(src, ignore_errors=True)
     print(out)
 
 
