@@ -633,43 +633,52 @@ __device__ __forceinline__ void insert_claim_direct(unsigned long long* T, uint3
   }
 }
 
-// Warp per vertex gathering directly (no stage round trip of 16 B per entry).
-template <int CAP, int WARPS, bool UNIT, int PASSES>
+// LPV lanes per vertex (a warp, or half a warp: two vertices per warp, twice the vertices in
+// flight per SM) gathering directly (no stage round trip of 16 B per entry).
+template <int CAP, int WARPS, bool UNIT, int PASSES, int LPV = 32>
 __global__ void __launch_bounds__(32 * WARPS) sweep_warp_d(const int32_t* __restrict__ verts,
                                                            const int64_t* __restrict__ brb,
                                                            const int64_t* __restrict__ soff, int64_t nv,
                                                            SweepArgs A) {
-  __shared__ unsigned long long tab[WARPS][CAP];
-  __shared__ uint32_t taba[WARPS][CAP];
+  constexpr int VPW = 32 / LPV;  // vertices per warp
+  __shared__ unsigned long long tab[WARPS * VPW][CAP];
+  __shared__ uint32_t taba[WARPS * VPW][CAP];
   __shared__ int32_t mb_v[WARPS][64], mb_t[WARPS][64];
-  const int lane = threadIdx.x & 31, wl = threadIdx.x >> 5;
-  unsigned long long* T = tab[wl];
-  uint32_t* TA = taba[wl];
+  const int lane = threadIdx.x & 31, wl = threadIdx.x >> 5, sub = lane / LPV, sl = lane % LPV;
+  unsigned long long* T = tab[wl * VPW + sub];
+  uint32_t* TA = taba[wl * VPW + sub];
   MoveBuf<64> mb{mb_v[wl], mb_t[wl], 0};
-  for (int t = lane; t < CAP; t += 32) {
+  for (int t = sl; t < CAP; t += LPV) {
     T[t] = kEmpty;
     TA[t] = kUnknownA;
   }
   __syncwarp();
-  const int64_t warps = (int64_t)gridDim.x * WARPS;
-  for (int64_t vi = (int64_t)blockIdx.x * WARPS + wl; vi < nv; vi += warps) {
-    const int32_t v = __ldg(&verts[vi]);
-    const int64_t rb = __ldg(&brb[vi]);
-    const int64_t deg = __ldg(&soff[vi + 1]) - __ldg(&soff[vi]);
-    const int32_t own = (int32_t)__ldg(&A.ca[v]).x;
-    const uint32_t ki = __ldg(&A.k[v]);
+  const int64_t step = (int64_t)gridDim.x * WARPS * VPW;
+  for (int64_t base = ((int64_t)blockIdx.x * WARPS + wl) * VPW; base < nv; base += step) {  // warp-uniform
+    const int64_t vi = base + sub;
+    const bool act = vi < nv;
+    int32_t v = 0, own = -1;
+    int64_t rb = 0, deg = 0;
+    uint32_t ki = 0;
+    if (act) {
+      v = __ldg(&verts[vi]);
+      rb = __ldg(&brb[vi]);
+      deg = __ldg(&soff[vi + 1]) - __ldg(&soff[vi]);
+      own = (int32_t)__ldg(&A.ca[v]).x;
+      ki = __ldg(&A.k[v]);
+    }
     uint32_t cl[4 * PASSES];
-    insert_claim_direct<UNIT, PASSES>(T, TA, CAP, A, v, rb, deg, lane, 32, cl);
+    insert_claim_direct<UNIT, PASSES>(T, TA, CAP, A, v, rb, deg, sl, LPV, cl);
     __syncwarp();
-    const bool own_single = A.rule == 2 && __ldg(&A.size[own]) == 1;
+    const bool own_single = act && A.rule == 2 && __ldg(&A.size[own]) == 1;
     long long s = (long long)0x8000000000000000ull;
     int cb = 0x7FFFFFFF;
     unsigned eown = 0;
     eval_claims<PASSES>(T, TA, cl, own, own_single, ki, A, s, cb, eown);
-    group_reduce<32>(s, cb, eown);
+    group_reduce<LPV>(s, cb, eown);
     int32_t tgt = own;
-    if (lane == 0) tgt = finish(s, cb, eown, own, __ldg(&A.ca[own]).y, ki, A);
-    mb.add(lane == 0 && tgt != own, v, tgt, A);
+    if (act && sl == 0) tgt = finish(s, cb, eown, own, __ldg(&A.ca[own]).y, ki, A);
+    mb.add(act && sl == 0 && tgt != own, v, tgt, A);
     __syncwarp();
   }
   mb.flush(A);
@@ -1477,6 +1486,9 @@ constexpr int64_t kDirectMaxDeg = 84;
 #ifndef LV_WARPD_CAP  // table slots per warp of the direct bucket-5 kernel (256: load <= 1/3; 128 measured slower)
 #define LV_WARPD_CAP 256
 #endif
+#ifndef LV_WARPD_LPV  // lanes per vertex of the direct bucket-5 kernel (16: two vertices per warp, r2)
+#define LV_WARPD_LPV 16
+#endif
 // largest degree of CTA tier `sub` (lv_internal.cuh)
 static int64_t max_deg_of_tier(int sub) {
   static const int64_t ub[5] = {kSub1Min - 1, kSub2Min - 1, kSub3Min - 1, kSub4Min - 1, kSub5Min - 1};
@@ -1504,7 +1516,12 @@ int32_t dispatch_class(Handle& h, Level& L, const SweepArgs& A, int bucket, int 
     }
     LV_LAUNCHED();
   } else if (sub == 0 && max_deg <= kDirectMaxDeg) {
+#if LV_WARPD_LPV == 16
+    // half-warp tables of 128 slots (16 per block: 24 KB; 256 would pass the 48 KB static limit)
+    sweep_warp_d<128, 8, UNIT, 2, 16><<<grid_for(nv, 16, 148 * 8), 256, 0, s>>>(verts, brb, soff, nv, A);
+#else
     sweep_warp_d<LV_WARPD_CAP, 8, UNIT, 1><<<grid_for(nv, 8, 148 * 8), 256, 0, s>>>(verts, brb, soff, nv, A);
+#endif
     LV_LAUNCHED();
   } else if (sub == 0 && max_deg <= 340) {  // warp per vertex, 3 claim passes of 4 entries per lane
     sweep_warp_c<512, 4, UNIT, 3><<<grid_for(nv, 4, 148 * 8), 128, 0, s>>>(verts, brb, soff, nv, stage, A);
